@@ -1,0 +1,314 @@
+"""Seeded synthetic programs C1, C2 (+ mini sizes) and fuzz programs.
+
+Shapes follow SURVEY.md §8(d) / App. A.5 and BASELINE.json `configs`:
+  C1  vector add c = a + b, n = 1024 FP32, 4 CTAs x 256 threads, one instance.
+  C2  SGEMM C = A.B (A stored K-major, B row-major), 128x128 CTA tile,
+      8x8 micro-tile per thread; 4096^3 at full size, 256^3 as "mini-C2".
+Fuzz programs are random straight-line/branchy kernels used to cross-check the
+two interpreters opcode by opcode.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+from . import isa
+from .isa import Asm, RZ, PT, NEG
+from .program import ProgramBuilder, Program, ptr_words, f32_data, f64_data, u32_data
+
+DATA_SEED = {1: 0xD0000001, 2: 0xD0000002, 3: 0xD0000003}
+CAMPAIGN_SEED = {1: 0xC0000001, 2: 0xC0000002, 3: 0xC0000003}
+
+
+# ---------------------------------------------------------------------------
+# C1: vector add (App. A.5 listing, 18 static instructions)
+# ---------------------------------------------------------------------------
+def c1_code() -> np.ndarray:
+    s = Asm()
+    s.s2r(0, isa.SR_TID)                      # 0
+    s.s2r(1, isa.SR_CTAID)                    # 1
+    s.s2r(2, isa.SR_NTID)                     # 2
+    s.imad(0, 1, 2, 0)                        # 3  gid = ctaid*ntid + tid
+    s.ldc(3, 24)                              # 4  n
+    s.isetp(0, 0, 3, cmp=isa.GE)              # 5  P0 = gid >= n
+    s.exit(guard=0)                           # 6  @P0 EXIT
+    s.ldc(4, 0, wide=True)                    # 7  a
+    s.imad_wide(4, 0, imm=4, c=4)             # 8
+    s.ldc(6, 8, wide=True)                    # 9  b
+    s.imad_wide(6, 0, imm=4, c=6)             # 10
+    s.ldg(8, 4)                               # 11
+    s.ldg(9, 6)                               # 12
+    s.ldc(10, 16, wide=True)                  # 13 c
+    s.imad_wide(10, 0, imm=4, c=10)           # 14
+    s.fadd(8, 8, 9)                           # 15
+    s.stg(10, 8)                              # 16
+    s.exit()                                  # 17
+    return s.assemble()
+
+
+def vector_add(n: int = 1024, grid: int = 4, block: int = 256, seed: int = DATA_SEED[1]) -> Program:
+    pb = ProgramBuilder(f"vecadd_n{n}")
+    k = pb.add_kernel("vecadd", c1_code(), nregs=12)
+    a = pb.add_buffer("a", 4 * n, f32_data(seed, n), dtype=isa.DT_F32)
+    b = pb.add_buffer("b", 4 * n, f32_data(seed + 1, n), dtype=isa.DT_F32)
+    c = pb.add_buffer("c", 4 * n, writer=0, output=True, dtype=isa.DT_F32)
+    pb.add_instance(k, grid, block, ptr_words(a) + ptr_words(b) + ptr_words(c) + [n])
+    return pb.build(config="C1", n=n, grid=grid, block=block)
+
+
+def c1() -> Program:
+    return vector_add()
+
+
+# ---------------------------------------------------------------------------
+# C2: SGEMM, 128x128 CTA tile, 8x8 per thread (App. A.5)
+# ---------------------------------------------------------------------------
+ACC0, AFR, BFR = 8, 72, 80
+PA, PB, KCNT, SA, SB, TMP = 88, 90, 92, 93, 94, 95
+
+
+def sgemm_code(n_ctas_x: int) -> np.ndarray:
+    assert n_ctas_x & (n_ctas_x - 1) == 0
+    lg = n_ctas_x.bit_length() - 1
+    AND = 0xC0                                 # LOP3 lut for a & b
+    s = Asm()
+    s.s2r(0, isa.SR_TID)                       # 0
+    s.s2r(1, isa.SR_CTAID)                     # 1
+    s.lop3(2, 0, RZ, RZ, AND, imm=15)          # 2  tx
+    s.shf(3, 0, imm=4, mode=isa.SHF_R_U32)     # 3  ty
+    s.lop3(4, 1, RZ, RZ, AND, imm=n_ctas_x - 1)  # 4  bx
+    s.shf(5, 1, imm=lg, mode=isa.SHF_R_U32)    # 5  by
+    s.imad(6, 5, imm=128, c=RZ)                # 6
+    s.imad(6, 3, imm=8, c=6)                   # 7  m0
+    s.imad(7, 4, imm=128, c=RZ)                # 8
+    s.imad(7, 2, imm=8, c=7)                   # 9  n0
+    s.ldc(PA, 0, wide=True)                    # 10 A
+    s.imad_wide(PA, 6, imm=4, c=PA, unsigned=True)   # 11
+    s.ldc(PB, 8, wide=True)                    # 12 B
+    s.imad_wide(PB, 7, imm=4, c=PB, unsigned=True)   # 13
+    s.ldc(KCNT, 24)                            # 14 K
+    s.ldc(SA, 28)                              # 15 M*4
+    s.ldc(SB, 32)                              # 16 N*4
+    s.label("loop")                            # 17
+    s.ldg(AFR, PA, 0, isa.W128)
+    s.ldg(AFR + 4, PA, 16, isa.W128)
+    s.ldg(BFR, PB, 0, isa.W128)
+    s.ldg(BFR + 4, PB, 16, isa.W128)
+    for i in range(8):
+        for j in range(8):
+            r = ACC0 + 8 * i + j
+            s.ffma(r, AFR + i, BFR + j, r)
+    s.imad_wide(PA, SA, imm=1, c=PA, unsigned=True)
+    s.imad_wide(PB, SB, imm=1, c=PB, unsigned=True)
+    s.iadd3(KCNT, KCNT, imm=0xFFFFFFFF)
+    s.isetp(0, KCNT, imm=0, cmp=isa.GT)
+    s.bra("loop", guard=0)
+    s.ldc(PA, 16, wide=True)                   # C
+    s.ldc(TMP, 36)                             # N
+    s.imad(TMP, 6, TMP, 7)                     # m0*N + n0
+    s.imad_wide(PA, TMP, imm=4, c=PA, unsigned=True)
+    for i in range(8):
+        s.stg(PA, ACC0 + 8 * i, 0, isa.W128)
+        s.stg(PA, ACC0 + 8 * i + 4, 16, isa.W128)
+        s.imad_wide(PA, SB, imm=1, c=PA, unsigned=True)
+    s.exit()
+    return s.assemble()
+
+
+def sgemm(M: int, N: int, K: int, seed: int = DATA_SEED[2]) -> Program:
+    assert M % 128 == 0 and N % 128 == 0 and K >= 1
+    nx = N // 128
+    pb = ProgramBuilder(f"sgemm_{M}x{N}x{K}")
+    k = pb.add_kernel("sgemm_128x128", sgemm_code(nx), nregs=96)
+    a = pb.add_buffer("A", 4 * K * M, f32_data(seed, K * M), dtype=isa.DT_F32)      # A^T: [K][M]
+    b = pb.add_buffer("B", 4 * K * N, f32_data(seed + 1, K * N), dtype=isa.DT_F32)  # [K][N]
+    c = pb.add_buffer("C", 4 * M * N, writer=0, output=True, dtype=isa.DT_F32)      # [M][N]
+    pb.add_instance(k, (M // 128) * nx, 256,
+                    ptr_words(a) + ptr_words(b) + ptr_words(c) + [K, 4 * M, 4 * N, N])
+    return pb.build(config="C2", M=M, N=N, K=K)
+
+
+def c2(full: bool = True) -> Program:
+    return sgemm(4096, 4096, 4096) if full else sgemm(256, 256, 256)
+
+
+# ---------------------------------------------------------------------------
+# Fuzz programs (random opcode mixes, divergence, SHFL, special FP values)
+# ---------------------------------------------------------------------------
+SPECIAL_F32 = [0x00000000, 0x80000000, 0x7F800000, 0xFF800000, 0x7FC00000, 0xFFC00001,
+               0x00000001, 0x807FFFFF, 0x3F800000, 0xBF800000, 0x4B000000, 0xCF000000,
+               0x4F000000, 0x7F7FFFFF, 0x34000000, 0x3EFFFFFF]
+SPECIAL_F64_HI = [0x00000000, 0x80000000, 0x7FF00000, 0xFFF00000, 0x7FF80000, 0x3FF00000,
+                  0xBFF00000, 0x00000001, 0x41E00000, 0xC1E00000, 0x47EFFFFF, 0x36A00000]
+
+NWORK = 16      # working registers R0..R15 (pairs inside)
+R_GID, R_PIN, R_POUT, R_TMP, R_CNT = 20, 22, 24, 26, 27
+
+
+def _fuzz_body(rng: np.random.Generator, s: Asm, n_ops: int, allow_branch=True):
+    """Random ops on R0..R15 / P0..P5; forward branches only."""
+    def r():
+        return int(rng.integers(0, NWORK))
+
+    def pr():
+        return int(rng.integers(0, NWORK // 2)) * 2
+
+    def g():
+        x = rng.random()
+        if x < 0.75:
+            return PT
+        return int(rng.integers(0, 6)) | (NEG if rng.random() < 0.5 else 0)
+
+    def imm_or_none():
+        return int(rng.integers(0, 2**32)) if rng.random() < 0.3 else None
+
+    pending = []
+    for n in range(n_ops):
+        for lbl in [p for p in pending if p[1] == n]:
+            s.label(lbl[0])
+        k = int(rng.integers(0, 27))
+        if k == 0:
+            s.mov(r(), b=r(), imm=imm_or_none(), guard=g())
+        elif k == 1:
+            s.iadd3(r(), r(), r(), r(), imm=imm_or_none(), nega=rng.random() < 0.3,
+                    negb=rng.random() < 0.3, carry=int(rng.integers(0, 6)) if rng.random() < 0.3 else PT, guard=g())
+        elif k == 2:
+            s.imad(r(), r(), r(), r(), imm=imm_or_none(), guard=g())
+        elif k == 3:
+            s.imad_wide(pr(), r(), r(), c=pr() if rng.random() < 0.7 else RZ, imm=imm_or_none(),
+                        unsigned=rng.random() < 0.5, guard=g())
+        elif k == 4:
+            im = int(rng.integers(0, 40)) if rng.random() < 0.5 else None
+            s.shf(r(), r(), r(), imm=im, mode=int(rng.integers(0, 3)), guard=g())
+        elif k == 5:
+            s.lop3(r(), r(), r(), r(), int(rng.integers(0, 256)), guard=g())
+        elif k == 6:
+            s.sel(r(), r(), r(), int(rng.integers(0, 8)) | (NEG if rng.random() < 0.3 else 0), guard=g())
+        elif k == 7:
+            s.isetp(int(rng.integers(0, 6)), r(), r(), cmp=int(rng.integers(0, 6)), imm=imm_or_none(),
+                    unsigned=rng.random() < 0.5, guard=g())
+        elif k == 8:
+            s.fsetp(int(rng.integers(0, 6)), r(), r(), cmp=int(rng.integers(0, 6)), guard=g())
+        elif k == 9:
+            s.dsetp(int(rng.integers(0, 6)), pr(), pr(), cmp=int(rng.integers(0, 6)), guard=g())
+        elif k in (10, 11, 12):
+            op = [s.fadd, s.fmul, s.ffma][k - 10]
+            args = (r(), r(), r()) if k < 12 else (r(), r(), r(), r())
+            op(*args, nega=rng.random() < 0.3, negb=rng.random() < 0.3, negc=rng.random() < 0.3, guard=g())
+        elif k == 13:
+            s.fmnmx(r(), r(), r(), is_max=rng.random() < 0.5, guard=g())
+        elif k in (14, 15, 16):
+            op = [s.dadd, s.dmul, s.dfma][k - 14]
+            args = (pr(), pr(), pr()) if k < 16 else (pr(), pr(), pr(), pr())
+            op(*args, nega=rng.random() < 0.3, negb=rng.random() < 0.3, negc=rng.random() < 0.3, guard=g())
+        elif k == 17:
+            s.i2f(r(), r(), unsigned=rng.random() < 0.5, guard=g())
+        elif k == 18:
+            s.f2i(r(), r(), guard=g())
+        elif k == 19:
+            s.f2f_f64_f32(pr(), r(), guard=g())
+        elif k == 20:
+            s.f2f_f32_f64(r(), pr(), guard=g())
+        elif k in (21, 22):
+            im = int(rng.integers(0, 40)) if rng.random() < 0.6 else None
+            s.shfl(r(), r(), r(), imm=im, mode=int(rng.integers(0, 4)), guard=g())
+        elif k == 23:
+            s.imnmx(r(), r(), r(), is_max=rng.random() < 0.5, unsigned=rng.random() < 0.5, guard=g())
+        elif k == 24 and allow_branch and n + 2 < n_ops:
+            # forward branch on a (usually lane-divergent) predicate
+            lbl = f"L{n}"
+            tgt = n + 1 + int(rng.integers(1, min(6, n_ops - n)))
+            pending.append((lbl, tgt))
+            s.bra(lbl, guard=int(rng.integers(0, 6)) | (NEG if rng.random() < 0.5 else 0))
+        elif k == 25:
+            s.s2r(r(), int(rng.integers(0, 6)), guard=g())
+        else:
+            s.nop(guard=g())
+    for lbl in [p for p in pending if p[1] >= n_ops]:
+        s.label(lbl[0])
+
+
+def fuzz_program(seed: int, n_ops: int = 120, grid: int = 2, block: int = 80, loop_iters: int = 3) -> Program:
+    """Random kernel: load 16 words per thread (special FP values mixed in), run
+    a random op mix (optionally inside a counted loop), store the 16 registers
+    and the 6 predicates.  block=80 gives a partial third warp per CTA."""
+    rng = np.random.Generator(np.random.PCG64(seed))
+    nthr = grid * block
+    words = u32_data(seed ^ 0x5EED, nthr * NWORK)
+    sp = rng.random(words.size) < 0.25
+    words[sp] = rng.choice(np.array(SPECIAL_F32, dtype=np.uint32), size=int(sp.sum()))
+    hi = (np.arange(words.size) % 2 == 1) & (rng.random(words.size) < 0.2)
+    words[hi] = rng.choice(np.array(SPECIAL_F64_HI, dtype=np.uint32), size=int(hi.sum()))
+
+    s = Asm()
+    s.s2r(R_GID, isa.SR_TID)
+    s.s2r(R_TMP, isa.SR_CTAID)
+    s.s2r(R_TMP + 1, isa.SR_NTID)
+    s.imad(R_GID, R_TMP, R_TMP + 1, R_GID)
+    s.ldc(R_PIN, 0, wide=True)
+    s.imad_wide(R_PIN, R_GID, imm=4 * NWORK, c=R_PIN, unsigned=True)
+    for i in range(0, NWORK, 4):
+        s.ldg(i, R_PIN, 4 * i, isa.W128)
+    if loop_iters > 1:
+        s.mov(R_CNT, imm=loop_iters)
+        s.label("top")
+    _fuzz_body(rng, s, n_ops)
+    if loop_iters > 1:
+        s.iadd3(R_CNT, R_CNT, imm=0xFFFFFFFF)
+        s.isetp(6, R_CNT, imm=0, cmp=isa.GT)
+        s.bra("top", guard=6)
+    s.ldc(R_POUT, 8, wide=True)
+    s.imad_wide(R_POUT, R_GID, imm=4 * (NWORK + 4), c=R_POUT, unsigned=True)
+    for i in range(0, NWORK, 4):
+        s.stg(R_POUT, i, 4 * i, isa.W128)
+    # predicates -> one word (SEL per predicate, accumulate with IMAD)
+    s.mov(R_TMP, imm=0)
+    for p in range(6):
+        s.sel(R_TMP + 1, RZ, RZ, p, imm=1 << p)   # P ? RZ : (1<<p)
+        s.iadd3(R_TMP, R_TMP, R_TMP + 1)
+    s.stg(R_POUT, R_TMP, 4 * NWORK)
+    s.stg(R_POUT, R_GID, 4 * NWORK + 4)
+    s.exit()
+
+    pb = ProgramBuilder(f"fuzz_{seed}")
+    k = pb.add_kernel("fuzz", s.assemble(), nregs=32)
+    xin = pb.add_buffer("X", 4 * nthr * NWORK, words)
+    yout = pb.add_buffer("Y", 4 * nthr * (NWORK + 4), writer=0, output=True)
+    pb.add_instance(k, grid, block, ptr_words(xin) + ptr_words(yout))
+    return pb.build(config="fuzz", seed=seed)
+
+
+def multi_instance_chain(n_inst: int = 3, n: int = 256, block: int = 64, seed: int = 77) -> Program:
+    """y_{i+1} = y_i * s + x (FP32) over n_inst launches of one static kernel, each
+    writing a new SSA buffer version.  Exercises multi-instance profiling,
+    kernel_count, and (oracle full mode) downstream propagation."""
+    s = Asm()
+    s.s2r(0, isa.SR_TID)
+    s.s2r(1, isa.SR_CTAID)
+    s.s2r(2, isa.SR_NTID)
+    s.imad(0, 1, 2, 0)
+    s.ldc(3, 24)
+    s.isetp(0, 0, 3, cmp=isa.GE)
+    s.exit(guard=0)
+    s.ldc(4, 0, wide=True)
+    s.imad_wide(4, 0, imm=4, c=4, unsigned=True)
+    s.ldc(6, 8, wide=True)
+    s.imad_wide(6, 0, imm=4, c=6, unsigned=True)
+    s.ldc(10, 16, wide=True)
+    s.imad_wide(10, 0, imm=4, c=10, unsigned=True)
+    s.ldg(8, 4)
+    s.ldg(9, 6)
+    s.ldc(12, 28)
+    s.ffma(8, 9, 12, 8)
+    s.stg(10, 8)
+    s.exit()
+    code = s.assemble()
+    pb = ProgramBuilder(f"chain_{n_inst}")
+    k = pb.add_kernel("axpy_chain", code, nregs=12)
+    x = pb.add_buffer("x", 4 * n, f32_data(seed, n), dtype=isa.DT_F32)
+    y = pb.add_buffer("y0", 4 * n, f32_data(seed + 1, n), dtype=isa.DT_F32)
+    grid = (n + block - 1) // block
+    for i in range(n_inst):
+        ynew = pb.add_buffer(f"y{i + 1}", 4 * n, writer=i, output=(i == n_inst - 1), dtype=isa.DT_F32)
+        pb.add_instance(k, grid, block, ptr_words(x) + ptr_words(y) + ptr_words(ynew) + [n, isa.f32_bits(0.5)])
+        y = ynew
+    return pb.build(config="chain", n_inst=n_inst, n=n)

@@ -1,0 +1,262 @@
+"""CPU ORACLE — test infrastructure only.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s cpu_baseline /
+``--impl reference`` legs may import this package.  The product path
+(``paper_conf_dsn_0002hsvk21_b200``) never imports it and shares no code with it.
+
+This module is a thin ctypes wrapper around ``oracle/liboracle.so`` (built from
+oracle.cpp with ``-O2 -ffp-contract=off``), plus the confidence-interval formula
+of PAPER.md:214 (§IV-B), which is plain arithmetic kept here in Python.
+
+Parity status: every function is pinned by tests/test_oracle_*.py
+except the outcome *fractions* of whole campaigns, which the paper does not fix
+for synthetic programs ("parity unpinned": the paper's 32.5/4.2/63.3 % needs
+SpecACCEL).
+"""
+from __future__ import annotations
+
+import ctypes as C
+import math
+import os
+import subprocess
+import threading
+
+import numpy as np
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(HERE, "liboracle.so")
+SRC = [os.path.join(HERE, "oracle.cpp"), os.path.join(HERE, "oracle.h")]
+
+G_FP64, G_FP32, G_LD, G_PR, G_NODEST, G_OTHERS, G_GPPR, G_GP = range(8)
+GROUP_NAMES = ["G_FP64", "G_FP32", "G_LD", "G_PR", "G_NODEST", "G_OTHERS", "G_GPPR", "G_GP"]
+MASKED, SDC, DUE = 0, 1, 2
+MODE_FULL, MODE_WARP_LOCAL = 0, 1
+
+RECORD_DTYPE = np.dtype([("instance", "<u4"), ("insn", "<u4"), ("active", "<u4"), ("pred", "<u4")])
+SITE_DTYPE = np.dtype([
+    ("s", "<u8"), ("instruction_count", "<u8"),
+    ("instance", "<u4"), ("kernel_id", "<u4"), ("kernel_count", "<u4"), ("warp", "<u4"),
+    ("step", "<u4"), ("thread", "<u4"), ("pc", "<u4"), ("u_dst", "<u4"), ("u_bit", "<u4"), ("mask", "<u4"),
+    ("lane", "u1"), ("group", "u1"), ("bfm", "u1"), ("slot", "u1"), ("dst_kind", "u1"), ("dst_reg", "u1"),
+    ("n_elig", "u1"), ("pad", "u1"),
+])
+INJ_DTYPE = np.dtype([("before", "<u4"), ("after", "<u4"), ("mask", "<u4"), ("fault_pc", "<u4"),
+                      ("fault_kind", "u1"), ("outcome", "u1"), ("pad", "u1", 2), ("n_faulty_stores", "<u4")])
+assert SITE_DTYPE.itemsize == 64 and INJ_DTYPE.itemsize == 24
+
+
+class _Program(C.Structure):
+    _fields_ = [("code", C.c_void_p), ("n_code", C.c_uint32),
+                ("kern", C.c_void_p), ("n_kern", C.c_uint32),
+                ("inst", C.c_void_p), ("n_inst", C.c_uint32),
+                ("cbank", C.c_void_p), ("n_cbank", C.c_uint32),
+                ("buf", C.c_void_p), ("n_buf", C.c_uint32),
+                ("init_image", C.c_void_p), ("image_bytes", C.c_uint64)]
+
+
+_lock = threading.Lock()
+_lib = None
+
+
+def build(force: bool = False) -> str:
+    """Compile liboracle.so (plain g++, no GPU).  Building the checker is not using it."""
+    stale = not os.path.exists(LIB_PATH) or any(os.path.getmtime(s) > os.path.getmtime(LIB_PATH) for s in SRC)
+    if force or stale:
+        subprocess.run(["g++", "-O2", "-std=c++17", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "-shared",
+                        "-pthread", "-Wall", "-o", LIB_PATH, SRC[0]], check=True)
+    return LIB_PATH
+
+
+def lib():
+    global _lib
+    with _lock:
+        if _lib is None:
+            build()
+            L = C.CDLL(LIB_PATH)
+            vp, u32, u64, i32 = C.c_void_p, C.c_uint32, C.c_uint64, C.c_int
+            L.orc_golden_run.restype = vp
+            L.orc_golden_run.argtypes = [C.POINTER(_Program), i32, i32]
+            L.orc_last_error.restype = C.c_char_p
+            L.orc_error.restype = C.c_char_p
+            L.orc_error.argtypes = [vp]
+            L.orc_free.argtypes = [vp]
+            L.orc_n_warps.restype = u32
+            L.orc_n_warps.argtypes = [vp]
+            L.orc_n_records.restype = u64
+            L.orc_n_records.argtypes = [vp]
+            L.orc_n_golden_stores.restype = u64
+            L.orc_n_golden_stores.argtypes = [vp]
+            for f in ("orc_counts", "orc_warp_counts", "orc_warp_len", "orc_final_image"):
+                getattr(L, f).argtypes = [vp, vp]
+            L.orc_trace.argtypes = [vp, vp]
+            L.orc_count_warps.restype = u64
+            L.orc_count_warps.argtypes = [C.POINTER(_Program), u32, u32, i32, vp]
+            L.orc_select.argtypes = [vp, u64, vp, u32, vp, u32, u64, u32, vp]
+            L.orc_locate.argtypes = [vp, i32, vp, u32, vp]
+            L.orc_inject.argtypes = [vp, vp, u32, i32, i32, vp]
+            L.orc_philox4x32_10.argtypes = [vp, vp, vp]
+            L.orc_draw.argtypes = [u64, u64, u64, C.POINTER(u64), C.POINTER(u32), C.POINTER(u32), C.POINTER(u32)]
+            L.orc_mask.restype = u32
+            L.orc_mask.argtypes = [i32, u32]
+            L.orc_group_mask.restype = u32
+            L.orc_group_mask.argtypes = [vp]
+            L.orc_dest_slots.restype = u32
+            L.orc_dest_slots.argtypes = [vp, i32, vp, vp]
+            _lib = L
+    return _lib
+
+
+def _ptr(a: np.ndarray) -> int:
+    return a.ctypes.data if a.size else 0
+
+
+def _cprog(prog) -> tuple[_Program, list]:
+    keep = [np.ascontiguousarray(x) for x in (prog.code, prog.kernels, prog.instances, prog.cbank,
+                                                prog.buffers, prog.init_image)]
+    code, kern, inst, cb, buf, img = keep
+    p = _Program(_ptr(code), len(code), _ptr(kern), len(kern), _ptr(inst), len(inst),
+                 _ptr(cb), len(cb), _ptr(buf), len(buf), _ptr(img), img.size)
+    return p, keep
+
+
+def n_threads_default() -> int:
+    return os.cpu_count() or 1
+
+
+class Golden:
+    """Golden run of a program by the oracle interpreter (PAPER.md:72 step (1)
+    profile and the golden output state of step (4))."""
+
+    def __init__(self, prog, keep_trace: bool = True, n_threads: int | None = None):
+        self.prog = prog
+        self._p, self._keep = _cprog(prog)
+        L = lib()
+        self.h = L.orc_golden_run(C.byref(self._p), n_threads or n_threads_default(), int(keep_trace))
+        if not self.h:
+            raise RuntimeError("oracle golden run failed: " + L.orc_last_error().decode())
+        self.n_warps = L.orc_n_warps(self.h)
+        self.n_records = L.orc_n_records(self.h)
+        self.keep_trace = keep_trace
+
+    def __del__(self):
+        if getattr(self, "h", None):
+            lib().orc_free(self.h)
+            self.h = None
+
+    def counts(self) -> np.ndarray:
+        out = np.zeros((len(self.prog.instances), 8), dtype=np.uint64)
+        lib().orc_counts(self.h, _ptr(out))
+        return out
+
+    def warp_counts(self) -> np.ndarray:
+        out = np.zeros((self.n_warps, 8), dtype=np.uint64)
+        lib().orc_warp_counts(self.h, _ptr(out))
+        return out
+
+    def warp_len(self) -> np.ndarray:
+        out = np.zeros(self.n_warps, dtype=np.uint64)
+        lib().orc_warp_len(self.h, _ptr(out))
+        return out
+
+    def final_image(self) -> np.ndarray:
+        out = np.zeros(self.prog.image_bytes, dtype=np.uint8)
+        lib().orc_final_image(self.h, _ptr(out))
+        return out
+
+    def n_golden_stores(self) -> int:
+        return int(lib().orc_n_golden_stores(self.h))
+
+    def trace(self) -> np.ndarray:
+        out = np.zeros(self.n_records, dtype=RECORD_DTYPE)
+        if lib().orc_trace(self.h, _ptr(out)):
+            raise RuntimeError("trace not kept")
+        return out
+
+    def select(self, seed: int, groups, bfms, j0: int, n: int) -> np.ndarray:
+        g = np.asarray(groups, dtype=np.uint8)
+        b = np.asarray(bfms, dtype=np.uint8)
+        out = np.zeros(n, dtype=SITE_DTYPE)
+        rc = lib().orc_select(self.h, seed, _ptr(g), len(g), _ptr(b), len(b), j0, n, _ptr(out))
+        if rc:
+            raise OracleError(rc, lib().orc_error(self.h).decode())
+        return out
+
+    def locate(self, group: int, s) -> np.ndarray:
+        s = np.ascontiguousarray(s, dtype=np.uint64)
+        out = np.zeros(len(s), dtype=SITE_DTYPE)
+        rc = lib().orc_locate(self.h, group, _ptr(s), len(s), _ptr(out))
+        if rc:
+            raise OracleError(rc, lib().orc_error(self.h).decode())
+        return out
+
+    def inject(self, sites: np.ndarray, mode: int = MODE_FULL, n_threads: int | None = None) -> np.ndarray:
+        sites = np.ascontiguousarray(sites, dtype=SITE_DTYPE)
+        out = np.zeros(len(sites), dtype=INJ_DTYPE)
+        rc = lib().orc_inject(self.h, _ptr(sites), len(sites), mode, n_threads or n_threads_default(), _ptr(out))
+        if rc:
+            raise OracleError(rc, lib().orc_error(self.h).decode())
+        return out
+
+
+class OracleError(RuntimeError):
+    def __init__(self, code, msg):
+        super().__init__(f"[{code}] {msg}")
+        self.code = code
+
+
+def count_warps(prog, w0: int, w1: int, n_threads: int | None = None) -> tuple[int, np.ndarray]:
+    """Interpret warps [w0, w1) of a single-instance program (bounded CPU baseline)."""
+    p, keep = _cprog(prog)
+    out = np.zeros(8, dtype=np.uint64)
+    n = lib().orc_count_warps(C.byref(p), w0, w1, n_threads or n_threads_default(), _ptr(out))
+    return int(n), out
+
+
+def philox4x32_10(ctr, key) -> list[int]:
+    c = np.asarray(ctr, dtype=np.uint32)
+    k = np.asarray(key, dtype=np.uint32)
+    o = np.zeros(4, dtype=np.uint32)
+    lib().orc_philox4x32_10(_ptr(c), _ptr(k), _ptr(o))
+    return [int(x) for x in o]
+
+
+def draw(seed: int, j: int, n_g: int) -> tuple[int, int, int, int]:
+    s, ud, ub, at = C.c_uint64(), C.c_uint32(), C.c_uint32(), C.c_uint32()
+    lib().orc_draw(seed, j, n_g, C.byref(s), C.byref(ud), C.byref(ub), C.byref(at))
+    return s.value, ud.value, ub.value, at.value
+
+
+def mask(bfm: int, u_bit: int) -> int:
+    return int(lib().orc_mask(bfm, u_bit))
+
+
+def group_mask(insn_row) -> int:
+    a = np.ascontiguousarray(np.asarray(insn_row).reshape(1))
+    return int(lib().orc_group_mask(_ptr(a)))
+
+
+def dest_slots(insn_row, group: int) -> list[tuple[int, int]]:
+    a = np.ascontiguousarray(np.asarray(insn_row).reshape(1))
+    k = np.zeros(8, np.uint8)
+    r = np.zeros(8, np.uint8)
+    n = lib().orc_dest_slots(_ptr(a), group, _ptr(k), _ptr(r))
+    return [(int(k[i]), int(r[i])) for i in range(n)]
+
+
+# ---- PAPER.md:214 §IV-B confidence margins ----------------------------------
+_Z = {0.90: 1.6448536269514722, 0.95: 1.959963984540054, 0.99: 2.5758293035489004}
+
+
+def ci_margin(n: int, confidence: float, p_hat: float | None = None) -> float:
+    """Normal-approximation margin z*sqrt(p(1-p)/n); worst case p = 0.5 when
+    p_hat is None ("100 injections ... 90% ... +-8%; 1000 ... 95% ... +-3%")."""
+    p = 0.5 if p_hat is None else p_hat
+    return _Z[confidence] * math.sqrt(p * (1 - p) / n)
+
+
+def histogram(sites: np.ndarray, inj: np.ndarray) -> np.ndarray:
+    """Outcome histogram [group][bfm][M,S,D] (u64), by plain counting."""
+    h = np.zeros((8, 4, 3), dtype=np.uint64)
+    for s, r in zip(sites, inj):
+        h[int(s["group"]), int(s["bfm"]), int(r["outcome"])] += 1
+    return h
