@@ -1,0 +1,192 @@
+/* fi.h — C ABI of libfi.so, the B200 (sm_100a) NVBitFI hot path.
+ *
+ * PAPER.md = /root/reference/PAPER.md (Tsai et al., "NVBitFI: Dynamic Fault
+ * Injection for GPUs", DSN 2021).  DESIGN.md §3 defines the program model,
+ * §4 the readings C-1..C-20 of the paper that these calls implement.
+ *
+ * Conventions (all entry points):
+ *   - Pointers are DEVICE pointers owned by the caller unless marked host.
+ *     libfi allocates nothing persistent; scratch is the caller's.
+ *   - Calls are asynchronous and ordered on `stream` (a cudaStream_t passed as
+ *     void*; NULL = legacy default stream).  Only calls documented as
+ *     "synchronizes" block the host.
+ *   - Every call returns fi_status; nothing throws or exits across the ABI.
+ *     Launch/CUDA errors return FI_E_CUDA (fi_last_cuda_error() has the text).
+ *     Errors found by device code (a golden-run fault, a site that does not
+ *     match the trace) are OR-ed into the caller's device word `dev_status`
+ *     as (1u << fi_status) bits; read it after the stream completes.
+ *   - Reentrant given distinct output / scratch buffers.
+ */
+#ifndef FI_H
+#define FI_H
+#include <stddef.h>
+#include <stdint.h>
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    FI_OK = 0,
+    FI_E_ARG = 1,              /* bad argument / size */
+    FI_E_EMPTY_GROUP = 2,      /* N_g == 0 for a scheduled group */
+    FI_E_NOT_INJECTABLE = 3,   /* G_NODEST scheduled (C-16) */
+    FI_E_PROGRAM = 4,          /* golden run faulted / program violates DESIGN.md §3.5 */
+    FI_E_CUDA = 5,
+    FI_E_SITE = 6,             /* a site does not match the re-executed warp */
+    FI_E_CAPACITY = 8          /* faulty store log overflow (replica must be re-run with a larger log) */
+} fi_status;
+
+/* Table II arch state ids [PAPER.md:94-104], 0-based (C-1) */
+typedef enum { FI_G_FP64 = 0, FI_G_FP32 = 1, FI_G_LD = 2, FI_G_PR = 3, FI_G_NODEST = 4,
+               FI_G_OTHERS = 5, FI_G_GPPR = 6, FI_G_GP = 7, FI_NGROUPS = 8 } fi_group;
+/* Table II bit-flip models [PAPER.md:105-109], 0-based (C-1) */
+typedef enum { FI_FLIP_SINGLE_BIT = 0, FI_FLIP_TWO_BITS = 1, FI_RANDOM_VALUE = 2, FI_ZERO_VALUE = 3 } fi_bfm;
+/* Table V outcomes [PAPER.md:184-196] */
+typedef enum { FI_MASKED = 0, FI_SDC = 1, FI_DUE = 2 } fi_outcome;
+
+/* ---- program ------------------------------------------- */
+typedef struct { uint8_t op, guard, d0, d1, a, b, c, mod; uint32_t imm, ext; } fi_insn;          /* 16 B */
+typedef struct { uint32_t code_off, code_len, nregs, pad; } fi_kernel;                             /* 16 B */
+typedef struct { uint32_t kernel, kernel_count, grid, block, cbank_off, cbank_len,
+                 warp_begin, warp_end; } fi_instance;                                                /* 32 B */
+typedef struct { uint64_t off, size; int32_t writer; uint32_t flags; } fi_buffer;                  /* 24 B; flags bit0 = output */
+
+typedef struct {
+    const fi_insn* code;      uint32_t n_code;       /* device */
+    const fi_kernel* kern;    uint32_t n_kern;       /* device */
+    const fi_instance* inst;  uint32_t n_inst;       /* device */
+    const uint32_t* cbank;    uint32_t n_cbank;      /* device */
+    const fi_buffer* buf;     uint32_t n_buf;        /* device, sorted by off */
+    const uint32_t* gran;                            /* device [ceil(image_bytes/256)]: buffer id per 256-B granule, from fi_build_granule_map */
+    uint64_t image_bytes;
+    uint32_t n_warps;
+    uint32_t n_regs;                                 /* register rows the emulator keeps: from fi_program_regs() */
+    const fi_insn* code_host;                        /* host mirrors (launch geometry, validation) */
+    const fi_instance* inst_host;
+} fi_program;
+
+/* ---- trace (App. A.3) ---------------------------------- */
+typedef struct { uint32_t instance, insn, active, pred; } fi_record;   /* insn = pc | op<<16 | groupmask<<24 */
+typedef struct { uint64_t va; uint32_t value, step; } fi_store;        /* one stored 32-bit word, 16 B */
+
+typedef struct {
+    const fi_record* rec;     uint64_t n_rec;        /* device */
+    const uint64_t* warp_off;                        /* device [n_warps+1]: first record of each warp */
+    const fi_store* gstore;                          /* device: golden store log, per warp contiguous */
+    const uint64_t* gstore_off;                      /* device [n_warps+1] */
+    uint32_t n_warps;
+} fi_trace;
+
+/* ---- sites, schedule, injection results -------------------------------- */
+typedef struct {
+    uint64_t s, instruction_count;                   /* s in [0, N_g) (C-4); instruction_count = s - P_k[instance] */
+    uint32_t instance, kernel_id, kernel_count, warp, step, thread;   /* kernel_count: ordinal of the instance among its static kernel's */
+    uint32_t pc, u_dst, u_bit, mask;                 /* mask = Table II pattern (0 for ZERO_VALUE: resolved at injection) */
+    uint8_t lane, group, bfm, slot, dst_kind /*0 GP, 1 PR*/, dst_reg, n_elig, pad;
+} fi_site;                                           /* 64 B */
+
+typedef struct {
+    uint64_t seed;                                   /* campaign seed (Philox key) */
+    uint32_t n_groups, n_bfms;
+    uint8_t groups[8];                               /* group(j) = groups[j % n_groups] */
+    uint8_t bfms[4];                                 /* bfm(j) = bfms[(j / n_groups) % n_bfms] */
+} fi_schedule;
+
+typedef struct {
+    uint32_t before, after, mask, fault_pc;          /* mask actually applied (ZERO_VALUE: = before) */
+    uint8_t fault_kind /*0 none, 1 misaligned, 2 unmapped, 3 watchdog, 4 illegal pc*/, outcome, overflow, pad;
+    uint32_t n_faulty_stores;                        /* faulty stores after the site (words) */
+} fi_inj;                                            /* 24 B */
+
+/* ======================================================================== */
+const char* fi_status_str(fi_status s);
+const char* fi_last_cuda_error(void);
+const char* fi_version(void);
+
+/* Register rows the emulator must keep for this program: 1 + the largest
+ * register index the code can touch (host scan of code_host).  Host only. */
+uint32_t fi_program_regs(const fi_insn* code_host, uint32_t n_code);
+
+/* Granule map: gran[i] = id of the buffer containing byte 256*i of the image,
+ * 0xFFFFFFFF if none (C-15).  `gran` has ceil(image_bytes/256) entries. */
+fi_status fi_build_granule_map(const fi_program* p, uint32_t* gran, void* stream);
+
+/* Golden run, pass 1 — PAPER.md:72 step (1)/(4) golden state.  Executes the
+ * instances in launch order on `image` (in: initial image, out: golden final
+ * image), writing per-warp step counts warp_len[n_warps] and
+ * stored-word counts warp_nstore[n_warps].  One launch per instance. */
+fi_status fi_golden_lengths(const fi_program* p, uint8_t* image, uint64_t* warp_len, uint64_t* warp_nstore,
+                            uint32_t* dev_status, void* stream);
+
+/* Exclusive scan of n u64 values into out[n+1] (out[n] = total).  Scratch:
+ * fi_scan_u64_workspace(n) bytes. */
+size_t fi_scan_u64_workspace(uint64_t n);
+fi_status fi_scan_u64(const uint64_t* in, uint64_t* out, uint64_t n, void* ws, size_t ws_bytes, void* stream);
+
+/* Golden run, pass 2: re-executes every warp of every instance in ONE launch
+ * over the golden final image and writes the trace records (App. A.3) and the
+ * golden store log, at warp_off / gstore_off (exclusive scans of pass 1). */
+fi_status fi_golden_trace(const fi_program* p, const uint8_t* image, const uint64_t* warp_off,
+                          const uint64_t* gstore_off, fi_record* rec, fi_store* gstore,
+                          uint32_t* dev_status, void* stream);
+
+/* K1 — profile, "dynamic instruction counts for every opcode in
+ * every thread ... Instructions that are not executed based on a predicate
+ * register are not included", grouped by Table II (C-2):
+ *   inst_counts[k][g] = sum over records r of instance k in [rec_begin, rec_end)
+ *                       of popc(active & pred) * [g in groupmask(r)]      (u64)
+ *   chunk_counts[c][g] = same sum over chunk c = records [1024c, 1024c+1024)
+ *                       (u32), written for every chunk overlapping the range.
+ * rec_begin must be a multiple of 1024 (shards own whole chunks).
+ * inst_counts is zeroed and accumulated by the call (n_inst x 8 u64). */
+fi_status fi_profile(const fi_trace* t, uint64_t rec_begin, uint64_t rec_end, uint32_t n_inst,
+                     uint64_t* inst_counts, uint32_t* chunk_counts, void* stream);
+#define FI_CHUNK 1024
+
+/* K2 — site index: exclusive prefix sums P_k[n_inst+1][8] of inst_counts and
+ * P_c[n_chunks+1][8] of chunk_counts (u64), decoupled-lookback scan.
+ * `index` must hold fi_site_index_bytes(n_inst, n_chunks) bytes. */
+size_t fi_site_index_bytes(uint32_t n_inst, uint64_t n_chunks);
+fi_status fi_build_site_index(const uint64_t* inst_counts, uint32_t n_inst, const uint32_t* chunk_counts,
+                              uint64_t n_chunks, void* index, void* stream);
+/* Totals N_g (host, synchronizes): copies P_k[n_inst][*] */
+fi_status fi_site_totals(const void* index, uint32_t n_inst, uint64_t totals_host[8], void* stream);
+
+/* K3 — draw + search ("random number n from the set 1..N ...
+ * translated into a tuple of <kernel_name, kernel_count, instruction_count>";
+ * Table II destination register / bit-pattern value [PAPER.md:114-121]).
+ * Replica j = j0 + i for i < n: s by Philox4x32-10 + Lemire,
+ * then instance, chunk, record, lane, warp, step, slot and mask.
+ * `sched` is a host pointer.  totals_host from fi_site_totals. */
+fi_status fi_select_sites(const fi_program* p, const fi_trace* t, const void* index, uint32_t n_inst,
+                          uint64_t n_chunks, const uint64_t totals_host[8], const fi_schedule* sched,
+                          uint64_t j0, uint32_t n, fi_site* sites, uint32_t* dev_status, void* stream);
+
+/* K4 — inject: one CUDA warp re-executes the site's
+ * synthetic warp from its first instruction over the golden final image; after
+ * the site's instruction writes its destinations, lane `lane`'s destination
+ * `dst_reg` is XOR-ed with the mask (ZERO_VALUE: mask = before; predicates C-7).
+ * Stores after the site are logged to log[i*log_cap ...] (fi_store words).
+ * Memory faults and the watchdog (C-9, C-10) end the replica. */
+fi_status fi_inject(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
+                    uint32_t n, fi_inj* out, fi_store* log, uint32_t log_cap, uint32_t* dev_status, void* stream);
+
+/* K5 — classify (Table V [PAPER.md:184-196], [PAPER.md:206]; C-9, C-12, C-14):
+ * DUE if a fault/watchdog ended the replica; else SDC if the final value of any
+ * output-buffer word differs bitwise from the golden run; else Masked.
+ * Writes out[i].outcome and adds 1 to hist[group][bfm][outcome] (u64 [8][4][3]).
+ * Replicas with overflow set get outcome 0xFF and FI_E_CAPACITY in dev_status. */
+fi_status fi_classify(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
+                      uint32_t n, fi_inj* out, const fi_store* log, uint32_t log_cap, uint64_t* hist,
+                      uint32_t* dev_status, void* stream);
+
+/* Table II parameter file, one parameter per line in Table II order
+ * [PAPER.md:88]: arch state id, bit-flip model, kernel name, kernel count,
+ * instruction count, destination register value, bit-pattern value (the two
+ * [0,1) values printed as u/2^32 with 10 digits).  Host only. */
+fi_status fi_write_params_txt(const fi_site* site_host, const char* kernel_name, char* buf, size_t buf_bytes);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -53,7 +53,9 @@ void dest_regs(const orc_insn& I, std::vector<int>& gp, std::vector<int>& pr) {
         case F2F_F32_F64: case SHFL: case IMNMX: case FADD: case FMUL: case FFMA: case FMNMX:
             gpn(1); break;
         case IADD3:
-            gpn(1); if (I.d1 != PT) pr.push_back(I.d1 & 7); break;
+            gpn(1);
+            if ((I.d1 & 7) != PT) pr.push_back(I.d1 & 7);   // predicate fields are 3 bits (§3.1)
+            break;
         case IMAD_WIDE: case DADD: case DMUL: case DFMA: case F2F_F64_F32:
             gpn(2); break;
         case LDG: gpn(1 << std::min(I.mod & 3, 2)); break;

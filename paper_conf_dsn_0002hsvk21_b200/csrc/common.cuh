@@ -1,0 +1,91 @@
+// common.cuh — libfi internals shared by the CUDA translation units.
+// Independent of oracle/ (no shared code); semantics from DESIGN.md §3-§4.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "../../include/fi.h"
+
+namespace fi {
+
+enum Op : uint32_t {
+    NOP = 0, EXIT, BRA, MOV, S2R, IADD3, IMAD, IMAD_WIDE, SHF, LOP3, SEL,
+    ISETP, FSETP, DSETP, FADD, FMUL, FFMA, FMNMX, DADD, DMUL, DFMA,
+    LDG, LDC, STG, I2F, F2I, F2F_F64_F32, F2F_F32_F64, SHFL, IMNMX
+};
+constexpr uint32_t kRZ = 127, kPT = 7;
+constexpr uint64_t kVaBase = 0x00007F0000000000ull;          // C-15
+constexpr uint32_t kNoBuf = 0xFFFFFFFFu;
+constexpr uint32_t kQNaN32 = 0x7FFFFFFFu;                      // C-13
+constexpr uint64_t kQNaN64 = 0x7FFFFFFFFFFFFFFFull;
+
+// Architectural destinations of an instruction (DESIGN.md §3.2 "dest"):
+// n_gp consecutive GP registers from d0 (0 if d0 == RZ) and at most one predicate.
+struct Dests { uint32_t gp_base, n_gp, pr; bool has_pr; };
+
+__host__ __device__ inline Dests dests_of(uint32_t op, uint32_t d0, uint32_t d1, uint32_t mod) {
+    Dests d{d0, 0, 0, false};
+    uint32_t n = 0;
+    switch (op) {
+        case MOV: case S2R: case IMAD: case SHF: case LOP3: case SEL: case I2F: case F2I:
+        case F2F_F32_F64: case SHFL: case IMNMX: case FADD: case FMUL: case FFMA: case FMNMX: case IADD3:
+            n = 1; break;
+        case IMAD_WIDE: case DADD: case DMUL: case DFMA: case F2F_F64_F32: n = 2; break;
+        case LDG: n = 1u << ((mod & 3) > 2 ? 2 : (mod & 3)); break;
+        case LDC: n = (mod & 1) ? 2 : 1; break;
+        default: n = 0;
+    }
+    d.n_gp = (d0 == kRZ) ? 0 : n;
+    if (op == IADD3 && (d1 & 7) != kPT) { d.has_pr = true; d.pr = d1 & 7; }
+    if ((op == ISETP || op == FSETP || op == DSETP) && (d0 & 7) != kPT) { d.has_pr = true; d.pr = d0 & 7; }
+    return d;
+}
+
+// Table II membership (reading C-2): bit g set iff the instruction is in group g.
+__host__ __device__ inline uint32_t groupmask_of(uint32_t op, uint32_t d0, uint32_t d1, uint32_t mod) {
+    Dests d = dests_of(op, d0, d1, mod);
+    if (d.n_gp == 0 && !d.has_pr) return 1u << FI_G_NODEST;
+    if (d.n_gp == 0) return (1u << FI_G_PR) | (1u << FI_G_GPPR);
+    uint32_t base = (op == DADD || op == DMUL || op == DFMA) ? FI_G_FP64
+                  : (op == FADD || op == FMUL || op == FFMA || op == FMNMX) ? FI_G_FP32
+                  : (op == LDG || op == LDC) ? FI_G_LD : FI_G_OTHERS;
+    return (1u << base) | (1u << FI_G_GPPR) | (1u << FI_G_GP);
+}
+
+// Eligible destination slots for group g (C-6): GP registers ascending for the
+// GP-type groups, the predicate for G_PR, GP then predicate for G_GPPR.
+__host__ __device__ inline uint32_t n_slots(const Dests& d, uint32_t g) {
+    if (g == FI_G_NODEST) return 0;
+    if (g == FI_G_PR) return d.has_pr ? 1 : 0;
+    if (g == FI_G_GPPR) return d.n_gp + (d.has_pr ? 1 : 0);
+    return d.n_gp;
+}
+__host__ __device__ inline void slot_reg(const Dests& d, uint32_t g, uint32_t slot, uint32_t& kind, uint32_t& reg) {
+    if (g == FI_G_PR || slot >= d.n_gp) { kind = 1; reg = d.pr; }
+    else { kind = 0; reg = d.gp_base + slot; }
+}
+
+// Table II masks with value = u / 2^32 (C-5, C-8); ZERO_VALUE resolved at injection.
+__host__ __device__ inline uint32_t bfm_mask(uint32_t bfm, uint32_t u) {
+    switch (bfm) {
+        case FI_FLIP_SINGLE_BIT: return 1u << (uint32_t)((32ull * u) >> 32);
+        case FI_FLIP_TWO_BITS: return 3u << (uint32_t)((31ull * u) >> 32);
+        case FI_RANDOM_VALUE: return (uint32_t)((0xFFFFFFFFull * u) >> 32);
+        default: return 0;
+    }
+}
+
+}  // namespace fi
+
+// error plumbing for the host side of the ABI
+namespace fi {
+void set_cuda_error(cudaError_t e);
+inline fi_status cuda_status(cudaError_t e) {
+    if (e == cudaSuccess) return FI_OK;
+    set_cuda_error(e);
+    return FI_E_CUDA;
+}
+inline fi_status launch_status() { return cuda_status(cudaGetLastError()); }
+}  // namespace fi
+
+#define FI_DEV_ERR(ptr, code) atomicOr((ptr), 1u << (code))

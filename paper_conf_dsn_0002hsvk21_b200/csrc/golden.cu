@@ -1,0 +1,130 @@
+// golden.cu — the golden run that makes the trace resident in HBM (§8 row a1).
+//
+// PAPER.md:72 step (1) profiles a fault-free run and step (4) compares with the
+// golden output state.  Here the golden run is the emulator in two passes:
+//   pass 1 (fi_golden_lengths): instances in launch order, one launch each;
+//          stores go straight into the image, which ends as the golden final
+//          image; per-warp step and stored-word counts come out.
+//   pass 2 (fi_golden_trace): every warp of every instance in ONE launch over the
+//          final image (DESIGN.md §3.5 writer rule), writing the App. A.3 records
+//          and the golden store log at the offsets scanned from pass 1.
+#include <algorithm>
+#include <vector>
+
+#include "emu.cuh"
+
+namespace fi {
+namespace {
+
+constexpr int kWPB = 4;   // emulated warps per CTA
+
+size_t emu_smem(uint32_t n_regs) { return (size_t)kWPB * (n_regs + 1) * 32 * sizeof(uint32_t); }
+
+__global__ void __launch_bounds__(kWPB * 32)
+k_golden_len(EmuProg P, uint8_t* img, uint32_t k, uint64_t* warp_len, uint64_t* warp_nst, uint32_t* status) {
+    extern __shared__ uint32_t smem[];
+    const uint32_t wib = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const fi_instance in = P.inst[k];
+    const uint32_t lw = blockIdx.x * kWPB + wib;
+    if (lw >= in.warp_end - in.warp_begin) return;
+    const uint32_t wpc = (in.block + 31) / 32;
+    uint32_t* R = smem + wib * (P.n_regs + 1) * 32;
+    EmuOut o = emulate<EMU_LEN>(P, img, img, k, lw / wpc, lw % wpc, R, 0xFFFFFFFFu, nullptr, nullptr, 0, HookIn{});
+    if (lane == 0) {
+        warp_len[in.warp_begin + lw] = o.steps;
+        warp_nst[in.warp_begin + lw] = o.nstore;
+        if (o.fault) FI_DEV_ERR(status, FI_E_PROGRAM);
+    }
+}
+
+__global__ void __launch_bounds__(kWPB * 32)
+k_golden_trace(EmuProg P, const uint8_t* img, uint32_t n_warps, const uint64_t* warp_off, const uint64_t* gst_off,
+               fi_record* rec, fi_store* gst, uint32_t* status) {
+    extern __shared__ uint32_t smem[];
+    const uint32_t wib = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t w = blockIdx.x * kWPB + wib;
+    if (w >= n_warps) return;
+    const uint32_t k = instance_of_warp(P.inst, P.n_inst, w);
+    const fi_instance in = P.inst[k];
+    const uint32_t wpc = (in.block + 31) / 32, lw = w - in.warp_begin;
+    uint32_t* R = smem + wib * (P.n_regs + 1) * 32;
+    const uint64_t r0 = warp_off[w], g0 = gst_off[w];
+    EmuOut o = emulate<EMU_TRACE>(P, nullptr, img, k, lw / wpc, lw % wpc, R, 0xFFFFFFFFu, rec + r0, gst + g0,
+                                  0xFFFFFFFFu, HookIn{});
+    if (lane == 0 && (o.fault || o.steps != warp_off[w + 1] - r0 || o.nstore != gst_off[w + 1] - g0))
+        FI_DEV_ERR(status, FI_E_PROGRAM);
+}
+
+__global__ void k_gran(const fi_buffer* buf, uint32_t n_buf, uint32_t* gran, uint64_t n_gran) {
+    for (uint32_t b = blockIdx.y; b < n_buf; b += gridDim.y) {
+        const uint64_t g0 = buf[b].off >> 8, g1 = (buf[b].off + buf[b].size + 255) >> 8;
+        for (uint64_t g = g0 + blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; g < g1 && g < n_gran;
+             g += (uint64_t)gridDim.x * blockDim.x)
+            gran[g] = b;
+    }
+}
+
+}  // namespace
+
+size_t golden_smem(uint32_t n_regs) { return emu_smem(n_regs); }
+
+}  // namespace fi
+
+using namespace fi;
+
+extern "C" uint32_t fi_program_regs(const fi_insn* code, uint32_t n) {
+    uint32_t mx = 0;
+    for (uint32_t i = 0; i < n; ++i) {
+        const fi_insn& I = code[i];
+        for (uint32_t f : {(uint32_t)I.d0, (uint32_t)I.a, (uint32_t)I.b, (uint32_t)I.c})
+            if (f < kRZ) mx = std::max(mx, f);
+    }
+    return std::min<uint32_t>(kRZ, mx + 4);        // +3: widest multi-register operand (LDG/STG.128)
+}
+
+extern "C" fi_status fi_build_granule_map(const fi_program* p, uint32_t* gran, void* stream) {
+    if (!p || !gran) return FI_E_ARG;
+    cudaStream_t s = (cudaStream_t)stream;
+    const uint64_t n_gran = (p->image_bytes + 255) >> 8;
+    fi_status e = cuda_status(cudaMemsetAsync(gran, 0xFF, n_gran * sizeof(uint32_t), s));
+    if (e || !p->n_buf) return e;
+    dim3 grid(64, std::min<uint32_t>(p->n_buf, 4096));
+    k_gran<<<grid, 256, 0, s>>>(p->buf, p->n_buf, gran, n_gran);
+    return launch_status();
+}
+
+static fi_status set_smem(const void* f, size_t bytes) {
+    return cuda_status(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes));
+}
+
+extern "C" fi_status fi_golden_lengths(const fi_program* p, uint8_t* image, uint64_t* warp_len, uint64_t* warp_nstore,
+                                       uint32_t* dev_status, void* stream) {
+    if (!p || !image || !warp_len || !warp_nstore || !dev_status || !p->inst_host || !p->gran) return FI_E_ARG;
+    if (p->n_regs == 0 || p->n_regs > kRZ) return FI_E_ARG;
+    cudaStream_t s = (cudaStream_t)stream;
+    const size_t smem = emu_smem(p->n_regs);
+    fi_status e = set_smem((const void*)k_golden_len, smem);
+    if (e) return e;
+    const EmuProg P = make_emu_prog(p);
+    for (uint32_t k = 0; k < p->n_inst; ++k) {
+        const uint32_t nw = p->inst_host[k].warp_end - p->inst_host[k].warp_begin;
+        if (!nw) continue;
+        k_golden_len<<<(nw + kWPB - 1) / kWPB, kWPB * 32, smem, s>>>(P, image, k, warp_len, warp_nstore, dev_status);
+        if ((e = launch_status())) return e;
+    }
+    return FI_OK;
+}
+
+extern "C" fi_status fi_golden_trace(const fi_program* p, const uint8_t* image, const uint64_t* warp_off,
+                                     const uint64_t* gstore_off, fi_record* rec, fi_store* gstore,
+                                     uint32_t* dev_status, void* stream) {
+    if (!p || !image || !warp_off || !gstore_off || !rec || !dev_status || !p->gran) return FI_E_ARG;
+    if (!p->n_warps) return FI_OK;
+    cudaStream_t s = (cudaStream_t)stream;
+    const size_t smem = emu_smem(p->n_regs);
+    fi_status e = set_smem((const void*)k_golden_trace, smem);
+    if (e) return e;
+    k_golden_trace<<<(p->n_warps + kWPB - 1) / kWPB, kWPB * 32, smem, s>>>(
+        make_emu_prog(p), image, p->n_warps, warp_off, gstore_off, rec, gstore, dev_status);
+    return launch_status();
+}

@@ -1,0 +1,184 @@
+// inject.cu — K4 injection replicas and K5 outcome classification.
+//
+// K4 ("When that instruction is reached, the injection code will
+// corrupt the destination register of the instruction based on the bit-pattern
+// selection value"; :138 "corrupting a single destination register of a single
+// dynamic instruction"): one CUDA warp per replica re-executes the site's
+// synthetic warp from its first instruction over the golden final image (the
+// NVBitFI analog of instrumenting only the target dynamic kernel);
+// stores after the site go to the replica's log slot.
+//
+// K5 (Table V [PAPER.md:184-196], [PAPER.md:206]): DUE if the replica crashed
+// (memory fault) or hung (watchdog) — C-9, C-10; otherwise the warp's final
+// contribution to memory is compared with the golden run (C-12, C-14):
+//   D = { a in F : last faulty value(a) != golden(a) }
+//     U { a in G_suffix \ F : value before the instance(a) != golden(a) }
+// where F is the faulty store log after the site and G_suffix the golden
+// warp's stores after the site (stores up to the site are identical in both).
+// SDC iff D hits an output buffer, else Masked.
+#include <algorithm>
+
+#include "emu.cuh"
+
+namespace fi {
+size_t golden_smem(uint32_t n_regs);
+namespace {
+
+constexpr int kWPB = 4;
+
+__global__ void __launch_bounds__(kWPB * 32)
+k_inject(EmuProg P, const uint8_t* img, const uint64_t* __restrict__ warp_off, const fi_site* __restrict__ sites,
+         uint32_t n, fi_inj* __restrict__ out, fi_store* __restrict__ log, uint32_t cap, uint32_t* status) {
+    extern __shared__ uint32_t smem[];
+    const uint32_t wib = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t i = blockIdx.x * kWPB + wib;
+    if (i >= n) return;
+    const fi_site S = sites[i];
+    const fi_instance in = P.inst[S.instance];
+    const uint32_t wpc = (in.block + 31) / 32, lw = S.warp - in.warp_begin;
+    const uint64_t L = warp_off[S.warp + 1] - warp_off[S.warp];
+    const uint64_t wd = 10 * L + 1024;                                                   // C-10
+    const uint32_t watchdog = wd > 0xFFFFFFFFull ? 0xFFFFFFFFu : (uint32_t)wd;
+    uint32_t* R = smem + wib * (P.n_regs + 1) * 32;
+    const HookIn h{S.step, S.lane, S.dst_kind, S.dst_reg, S.bfm, S.mask, S.pc};
+    const EmuOut o = emulate<EMU_INJ>(P, nullptr, img, S.instance, lw / wpc, lw % wpc, R, watchdog, nullptr,
+                                      log + (uint64_t)i * cap, cap, h);
+    if (lane == 0) {
+        fi_inj r;
+        r.before = o.before; r.after = o.after; r.mask = o.mask; r.fault_pc = o.fault_pc;
+        r.fault_kind = (uint8_t)o.fault; r.outcome = 0; r.overflow = o.nstore > cap; r.pad = 0;
+        r.n_faulty_stores = o.nstore;
+        out[i] = r;
+        if (!o.fired || o.bad) FI_DEV_ERR(status, FI_E_SITE);
+    }
+}
+
+struct ClsArgs {
+    const fi_buffer* buf; const uint32_t* gran; const uint8_t* img;
+    const fi_store* gstore; const uint64_t* gstore_off;
+    const fi_site* sites; fi_inj* inj; uint32_t n;
+    const fi_store* log; uint32_t cap;
+    uint64_t* hist; uint32_t* status;
+};
+
+__device__ __forceinline__ uint32_t buf_of(const ClsArgs& A, uint64_t va) {
+    return __ldg(&A.gran[(va - kVaBase) >> 8]);
+}
+__device__ __forceinline__ bool is_output(const ClsArgs& A, uint64_t va) {
+    const uint32_t b = buf_of(A, va);
+    return b != kNoBuf && (__ldg(&A.buf[b].flags) & 1u);
+}
+__device__ __forceinline__ uint32_t golden_word(const ClsArgs& A, uint64_t va) {
+    return __ldg(reinterpret_cast<const uint32_t*>(A.img + (va - kVaBase)));
+}
+// value of word va before instance k (DESIGN.md §3.5 writer rule)
+__device__ __forceinline__ uint32_t pre_word(const ClsArgs& A, uint64_t va, uint32_t k) {
+    const uint32_t b = buf_of(A, va);
+    const int32_t wr = __ldg(&A.buf[b].writer);
+    return (wr >= 0 && (uint32_t)wr >= k) ? 0u : golden_word(A, va);
+}
+
+constexpr int kClsWarps = 4;
+
+__global__ void __launch_bounds__(kClsWarps * 32) k_classify(const ClsArgs A) {
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t i = blockIdx.x * kClsWarps + (threadIdx.x >> 5);
+    if (i >= A.n) return;
+    const fi_site S = A.sites[i];
+    const fi_inj R = A.inj[i];
+    uint32_t outcome;
+    if (R.fault_kind) {
+        outcome = FI_DUE;
+    } else if (R.overflow) {
+        outcome = 0xFF;
+    } else {
+        const fi_store* G = A.gstore + A.gstore_off[S.warp];
+        const uint64_t nGall = A.gstore_off[S.warp + 1] - A.gstore_off[S.warp];
+        // first golden entry after the site (entries are in step order)
+        uint64_t gs = 0;
+        for (uint64_t b = 0; b < nGall; b += 32) {
+            const bool after = b + lane < nGall && G[b + lane].step > S.step;
+            const uint32_t m = __ballot_sync(kFull, after);
+            if (m) { gs = b + __ffs(m) - 1; break; }
+            gs = min(b + 32, nGall);
+        }
+        const fi_store* Gs = G + gs;
+        const uint64_t nG = nGall - gs, nF = R.n_faulty_stores;
+        const fi_store* F = A.log + (uint64_t)i * A.cap;
+        bool same_addr = nF == nG;
+        for (uint64_t b = 0; same_addr && b < nF; b += 32) {
+            const bool d = b + lane < nF && F[b + lane].va != Gs[b + lane].va;
+            same_addr = !__any_sync(kFull, d);
+        }
+        bool sdc = false;
+        if (same_addr) {
+            // fast path: same store addresses in the same order; golden words are
+            // stored once per warp so the golden value is Gs[j]
+            for (uint64_t b = 0; b < nF && !sdc; b += 32) {
+                bool d = false;
+                if (b + lane < nF) {
+                    const fi_store f = F[b + lane];
+                    d = f.value != Gs[b + lane].value && is_output(A, f.va);
+                }
+                sdc = __any_sync(kFull, d);
+            }
+        } else {
+            for (uint64_t b = 0; b < nF && !sdc; b += 32) {            // faulty stores: last write wins
+                bool d = false;
+                const uint64_t j = b + lane;
+                if (j < nF) {
+                    const fi_store f = F[j];
+                    bool last = true;
+                    for (uint64_t q = j + 1; q < nF && last; ++q) last = F[q].va != f.va;
+                    d = last && is_output(A, f.va) && f.value != golden_word(A, f.va);
+                }
+                sdc = __any_sync(kFull, d);
+            }
+            for (uint64_t b = 0; b < nG && !sdc; b += 32) {            // golden stores the faulty run skipped
+                bool d = false;
+                const uint64_t j = b + lane;
+                if (j < nG) {
+                    const uint64_t va = Gs[j].va;
+                    bool inF = false;
+                    for (uint64_t q = 0; q < nF && !inF; ++q) inF = F[q].va == va;
+                    d = !inF && is_output(A, va) && pre_word(A, va, S.instance) != golden_word(A, va);
+                }
+                sdc = __any_sync(kFull, d);
+            }
+        }
+        outcome = sdc ? FI_SDC : FI_MASKED;
+    }
+    if (lane == 0) {
+        A.inj[i].outcome = (uint8_t)outcome;
+        if (outcome == 0xFF) FI_DEV_ERR(A.status, FI_E_CAPACITY);
+        else atomicAdd((unsigned long long*)&A.hist[((uint32_t)S.group * 4 + S.bfm) * 3 + outcome], 1ull);
+    }
+}
+
+}  // namespace
+}  // namespace fi
+
+using namespace fi;
+
+extern "C" fi_status fi_inject(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
+                               uint32_t n, fi_inj* out, fi_store* log, uint32_t log_cap, uint32_t* dev_status,
+                               void* stream) {
+    if (!p || !image || !t || !sites || !out || !dev_status || (log_cap && !log) || !p->gran) return FI_E_ARG;
+    if (n == 0) return FI_OK;
+    const size_t smem = golden_smem(p->n_regs);
+    fi_status e = cuda_status(cudaFuncSetAttribute((const void*)k_inject, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    if (e) return e;
+    k_inject<<<(n + kWPB - 1) / kWPB, kWPB * 32, smem, (cudaStream_t)stream>>>(
+        make_emu_prog(p), image, t->warp_off, sites, n, out, log, log_cap, dev_status);
+    return launch_status();
+}
+
+extern "C" fi_status fi_classify(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
+                                 uint32_t n, fi_inj* out, const fi_store* log, uint32_t log_cap, uint64_t* hist,
+                                 uint32_t* dev_status, void* stream) {
+    if (!p || !image || !t || !sites || !out || !hist || !dev_status || !p->gran) return FI_E_ARG;
+    if (n == 0) return FI_OK;
+    ClsArgs A{p->buf, p->gran, image, t->gstore, t->gstore_off, sites, out, n, log, log_cap, hist, dev_status};
+    k_classify<<<(n + kClsWarps - 1) / kClsWarps, kClsWarps * 32, 0, (cudaStream_t)stream>>>(A);
+    return launch_status();
+}

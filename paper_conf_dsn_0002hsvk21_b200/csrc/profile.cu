@@ -1,0 +1,124 @@
+// profile.cu — K1, the exact profiler (§III-A) as an HBM scan.
+//
+// "a profile containing one line for every dynamic kernel and the total dynamic
+// instruction counts ... in every thread ... Instructions that are not executed
+// based on a predicate register are not included" [PAPER.md:78], grouped by the
+// Table II arch state ids [PAPER.md:94-104]:
+//   inst_counts[k][g]  += popc(active & pred) for every record of instance k in group g
+//   chunk_counts[c][g]  = the same sum over the 1,024-record chunk c
+// One 16-B record per warp-instruction (App. A.3) is the only input, read once
+// with 128-bit streaming loads (L1::no_allocate), 8 loads in flight per lane.
+// Each warp owns a contiguous run of chunks; per-lane u32 counters are reduced
+// with REDUX (__reduce_add_sync) once per chunk, chunk counts are plain stores,
+// and instance counts stay in lanes 0-7 until the instance changes (one u64
+// atomic per group per instance per warp).  Chunks that straddle instances
+// (rare: instance boundaries) attribute per record.
+#include <algorithm>
+
+#include "common.cuh"
+
+namespace fi {
+namespace {
+
+constexpr int kThreads = 256;
+constexpr int kUnroll = 8;
+constexpr uint32_t kNone = 0xFFFFFFFFu;
+
+__device__ __forceinline__ uint4 ld_stream(const uint4* p) {
+    uint4 r;
+    asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+    return r;
+}
+
+__global__ void __launch_bounds__(kThreads)
+k_profile(const uint4* __restrict__ rec, uint64_t r_begin, uint64_t r_end, uint64_t c_begin, uint64_t c_end,
+          uint64_t* __restrict__ inst_counts, uint32_t* __restrict__ chunk_counts) {
+    const uint32_t lane = threadIdx.x & 31;
+    const uint64_t gw = ((uint64_t)blockIdx.x * kThreads + threadIdx.x) >> 5;
+    const uint64_t nwarps = ((uint64_t)gridDim.x * kThreads) >> 5;
+    const uint64_t nch = c_end - c_begin;
+    const uint64_t per = (nch + nwarps - 1) / nwarps;
+    const uint64_t c0 = c_begin + gw * per;
+    const uint64_t c1 = min(c0 + per, c_end);
+
+    uint32_t cur_k = kNone;
+    uint64_t acc = 0;                         // lane g < 8: running count of group g for cur_k
+    for (uint64_t c = c0; c < c1; ++c) {
+        const uint64_t a = max(c * FI_CHUNK, r_begin);
+        const uint64_t b = min(c * FI_CHUNK + FI_CHUNK, r_end);
+        const uint32_t n = (uint32_t)(b - a);
+        const uint4* base = rec + a;
+        const uint32_t kf = __ldg(&base[0].x), kl = __ldg(&base[n - 1].x);
+        uint32_t cnt[8];
+#pragma unroll
+        for (int g = 0; g < 8; ++g) cnt[g] = 0;
+        for (uint32_t i = lane; i < n; i += 32 * kUnroll) {
+            uint4 r[kUnroll];
+#pragma unroll
+            for (int u = 0; u < kUnroll; ++u)
+                r[u] = (i + u * 32 < n) ? ld_stream(base + i + u * 32) : make_uint4(0, 0, 0, 0);
+#pragma unroll
+            for (int u = 0; u < kUnroll; ++u) {
+                const uint32_t cc = __popc(r[u].z & r[u].w);
+                const uint32_t gm = r[u].y >> 24;
+#pragma unroll
+                for (int g = 0; g < 8; ++g) cnt[g] += ((gm >> g) & 1u) ? cc : 0u;
+            }
+        }
+        uint32_t mine = 0;
+#pragma unroll
+        for (int g = 0; g < 8; ++g) {
+            const uint32_t s = __reduce_add_sync(0xFFFFFFFFu, cnt[g]);
+            if (lane == (uint32_t)g) mine = s;
+        }
+        if (lane < 8) chunk_counts[c * 8 + lane] = mine;
+        if (kf == kl) {
+            if (kf != cur_k) {
+                if (cur_k != kNone && lane < 8 && acc) atomicAdd((unsigned long long*)&inst_counts[(uint64_t)cur_k * 8 + lane], acc);
+                cur_k = kf;
+                acc = 0;
+            }
+            acc += mine;
+        } else {
+            for (uint32_t i = lane; i < n; i += 32) {
+                const uint4 r = __ldg(base + i);
+                const uint32_t cc = __popc(r.z & r.w);
+                const uint32_t gm = r.y >> 24;
+                if (cc)
+                    for (int g = 0; g < 8; ++g)
+                        if ((gm >> g) & 1u) atomicAdd((unsigned long long*)&inst_counts[(uint64_t)r.x * 8 + g], (unsigned long long)cc);
+            }
+        }
+    }
+    if (cur_k != kNone && lane < 8 && acc) atomicAdd((unsigned long long*)&inst_counts[(uint64_t)cur_k * 8 + lane], acc);
+}
+
+int g_grid = 0;
+
+}  // namespace
+}  // namespace fi
+
+using namespace fi;
+
+extern "C" fi_status fi_profile(const fi_trace* t, uint64_t rec_begin, uint64_t rec_end, uint32_t n_inst,
+                                uint64_t* inst_counts, uint32_t* chunk_counts, void* stream) {
+    if (!t || !inst_counts || !chunk_counts || rec_end > t->n_rec || rec_begin > rec_end) return FI_E_ARG;
+    if (rec_begin % FI_CHUNK) return FI_E_ARG;
+    cudaStream_t s = (cudaStream_t)stream;
+    fi_status e = cuda_status(cudaMemsetAsync(inst_counts, 0, (size_t)n_inst * 8 * sizeof(uint64_t), s));
+    if (e || rec_begin == rec_end) return e;
+    if (!g_grid) {
+        int dev = 0, sms = 0, per = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_profile, kThreads, 0);
+        g_grid = std::max(1, sms * std::max(1, per));
+    }
+    const uint64_t c_begin = rec_begin / FI_CHUNK, c_end = (rec_end + FI_CHUNK - 1) / FI_CHUNK;
+    const uint64_t warps_needed = c_end - c_begin;
+    const int grid = (int)std::min<uint64_t>((uint64_t)g_grid, (warps_needed * 32 + kThreads - 1) / kThreads);
+    k_profile<<<grid, kThreads, 0, s>>>(reinterpret_cast<const uint4*>(t->rec), rec_begin, rec_end, c_begin, c_end,
+                                         inst_counts, chunk_counts);
+    return launch_status();
+}

@@ -1,0 +1,247 @@
+// select.cu — K2 site index (prefix sums) and K3 site selection.
+//
+// "A dynamic instruction will be selected from the set of executed
+// instructions by choosing a random number n from the set 1..N ... This n-th
+// instruction is then translated into a tuple of <kernel_name, kernel_count,
+// instruction_count>"; Table II [PAPER.md:110-121] adds the destination register
+// and bit-pattern values.  The random index is drawn with Philox4x32-10 + Lemire
+// (C-5) and located with two prefix arrays instead of a walk over
+// the trace: P_k over instances gives the instance and instruction_count, P_c
+// over 1,024-record chunks gives the chunk; one warp then scans that chunk's
+// records (warp inclusive scan + ballot) and picks the lane with __fns.
+#include <algorithm>
+
+#include "scan.cuh"
+
+namespace fi {
+namespace {
+
+// ---- Philox4x32-10 (Salmon et al. 2011) ------------------------------------
+__device__ __forceinline__ uint4 philox4x32_10(uint4 c, uint2 k) {
+#pragma unroll
+    for (int r = 0; r < 10; ++r) {
+        if (r) { k.x += 0x9E3779B9u; k.y += 0xBB67AE85u; }
+        const uint32_t hi0 = __umulhi(0xD2511F53u, c.x), lo0 = 0xD2511F53u * c.x;
+        const uint32_t hi1 = __umulhi(0xCD9E8D57u, c.z), lo1 = 0xCD9E8D57u * c.z;
+        c = make_uint4(hi1 ^ c.y ^ k.x, lo1, hi0 ^ c.w ^ k.y, lo0);
+    }
+    return c;
+}
+
+// Lemire's nearly-divisionless unbiased draw of s in [0, n) for replica j (C-5).
+__device__ void draw(uint64_t seed, uint64_t j, uint64_t n, uint64_t& s, uint32_t& u_dst, uint32_t& u_bit) {
+    const uint2 key = make_uint2((uint32_t)seed, (uint32_t)(seed >> 32));
+    uint4 b = philox4x32_10(make_uint4((uint32_t)j, (uint32_t)(j >> 32), 0u, 0x46490001u), key);
+    u_dst = b.z;
+    u_bit = b.w;
+    uint64_t x = (uint64_t)b.x | ((uint64_t)b.y << 32);
+    uint64_t lo = x * n;
+    if (lo < n) {
+        const uint64_t t = (0ull - n) % n;
+        for (uint32_t a = 1; lo < t; ++a) {
+            b = philox4x32_10(make_uint4((uint32_t)j, (uint32_t)(j >> 32), a, 0x46490001u), key);
+            x = (uint64_t)b.x | ((uint64_t)b.y << 32);
+            lo = x * n;
+        }
+    }
+    s = __umul64hi(x, n);
+}
+
+// Largest i in [0, m) with arr[i*stride + g] <= s, given arr[0] <= s < arr[m*stride+g]
+// (monotone).  32-ary warp search: 31 probes per round, ballot narrows the range.
+__device__ uint64_t warp_upper_search(const uint64_t* __restrict__ arr, uint64_t m, uint32_t stride, uint32_t g,
+                                      uint64_t s) {
+    const uint32_t lane = threadIdx.x & 31;
+    uint64_t lo = 0, hi = m;
+    while (hi - lo > 1) {
+        const uint64_t d = hi - lo;
+        const uint64_t p = lo + ((uint64_t)(lane + 1) * d) / 32;
+        const bool le = lane < 31 && p > lo && p < hi && __ldg(&arr[p * stride + g]) <= s;
+        const bool gt = lane < 31 && p > lo && p < hi && !le;
+        const uint32_t bl = __ballot_sync(0xFFFFFFFFu, le), bg = __ballot_sync(0xFFFFFFFFu, gt);
+        uint64_t nlo = lo, nhi = hi;
+        if (bl) nlo = __shfl_sync(0xFFFFFFFFu, p, 31 - __clz(bl));
+        if (bg) nhi = __shfl_sync(0xFFFFFFFFu, p, __ffs(bg) - 1);
+        lo = nlo;
+        hi = nhi;
+    }
+    return lo;
+}
+
+struct SelArgs {
+    const fi_insn* code; const fi_kernel* kern; const fi_instance* inst;
+    const uint4* rec; uint64_t n_rec; const uint64_t* warp_off; uint32_t n_warps;
+    const uint64_t* Pk; uint32_t n_inst; const uint64_t* Pc; uint64_t n_chunks;
+    uint64_t totals[8];
+    fi_schedule sched;
+    uint64_t j0; uint32_t n;
+    fi_site* sites; uint32_t* status;
+};
+
+constexpr int kWarps = 4;
+
+__global__ void __launch_bounds__(kWarps * 32) k_select(const SelArgs A) {
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t i = blockIdx.x * kWarps + (threadIdx.x >> 5);
+    if (i >= A.n) return;
+    const uint64_t j = A.j0 + i;
+    const uint32_t g = A.sched.groups[j % A.sched.n_groups];
+    const uint32_t bfm = A.sched.bfms[(j / A.sched.n_groups) % A.sched.n_bfms];
+    const uint64_t N = A.totals[g];
+
+    uint64_t s = 0;
+    uint32_t u_dst = 0, u_bit = 0;
+    if (lane == 0) draw(A.sched.seed, j, N, s, u_dst, u_bit);
+    s = __shfl_sync(0xFFFFFFFFu, s, 0);
+    u_dst = __shfl_sync(0xFFFFFFFFu, u_dst, 0);
+    u_bit = __shfl_sync(0xFFFFFFFFu, u_bit, 0);
+
+    // instance: last k with P_k[k][g] <= s ; chunk: last c with P_c[c][g] <= s
+    const uint32_t k = (uint32_t)warp_upper_search(A.Pk, A.n_inst, 8, g, s);
+    const uint64_t c = warp_upper_search(A.Pc, A.n_chunks, 8, g, s);
+    uint64_t r = s - __ldg(&A.Pc[c * 8 + g]);
+
+    // scan the chunk's records for the r-th counted lane-instruction of group g
+    const uint64_t base = c * FI_CHUNK;
+    const uint32_t nrec = (uint32_t)min((uint64_t)FI_CHUNK, A.n_rec - base);
+    bool found = false;
+    uint64_t rec_idx = 0;
+    uint32_t rinst = 0, rinsn = 0, lane_sel = 0;
+    for (uint32_t off = 0; off < nrec; off += 32) {
+        const uint32_t idx = off + lane;
+        const uint4 x = idx < nrec ? __ldg(&A.rec[base + idx]) : make_uint4(0, 0, 0, 0);
+        const uint32_t ex = x.z & x.w;
+        const uint32_t cnt = ((x.y >> (24 + g)) & 1u) ? __popc(ex) : 0u;
+        uint32_t incl = cnt;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, incl, d);
+            if (lane >= (uint32_t)d) incl += y;
+        }
+        const uint32_t total = __shfl_sync(0xFFFFFFFFu, incl, 31);
+        if (r < total) {
+            const uint32_t hit = __ballot_sync(0xFFFFFFFFu, incl > r);
+            const uint32_t L = __ffs(hit) - 1;
+            const uint32_t before = __shfl_sync(0xFFFFFFFFu, incl - cnt, L);
+            const uint32_t exL = __shfl_sync(0xFFFFFFFFu, ex, L);
+            rinst = __shfl_sync(0xFFFFFFFFu, x.x, L);
+            rinsn = __shfl_sync(0xFFFFFFFFu, x.y, L);
+            lane_sel = __fns(exL, 0, (int)(r - before) + 1);      // (r-before)-th set bit, ascending (C-3)
+            rec_idx = base + off + L;
+            found = true;
+            break;
+        }
+        r -= total;
+    }
+    if (!found || rinst != k) {
+        if (lane == 0) FI_DEV_ERR(A.status, FI_E_SITE);
+        return;
+    }
+    const uint32_t w = (uint32_t)warp_upper_search(A.warp_off, A.n_warps, 1, 0, rec_idx);
+    if (lane != 0) return;
+    const fi_instance in = A.inst[k];
+    const uint32_t wpc = (in.block + 31) / 32, lw = w - in.warp_begin;
+    const uint32_t pc = rinsn & 0xFFFFu;
+    const fi_insn I = A.code[A.kern[in.kernel].code_off + pc];
+    const Dests d = dests_of(I.op, I.d0, I.d1, I.mod);
+    const uint32_t ne = n_slots(d, g);
+    if (ne == 0) { FI_DEV_ERR(A.status, FI_E_SITE); return; }
+    const uint32_t slot = (uint32_t)(((uint64_t)ne * u_dst) >> 32);        // floor(n x value), C-5/C-6
+    uint32_t kind, reg;
+    slot_reg(d, g, slot, kind, reg);
+
+    fi_site S;
+    S.s = s;
+    S.instruction_count = s - __ldg(&A.Pk[(uint64_t)k * 8 + g]);
+    S.instance = k;
+    S.kernel_id = in.kernel;
+    S.kernel_count = in.kernel_count;
+    S.warp = w;
+    S.step = (uint32_t)(rec_idx - __ldg(&A.warp_off[w]));
+    S.thread = (lw / wpc) * in.block + (lw % wpc) * 32 + lane_sel;
+    S.pc = pc;
+    S.u_dst = u_dst;
+    S.u_bit = u_bit;
+    S.mask = bfm_mask(bfm, u_bit);
+    S.lane = (uint8_t)lane_sel;
+    S.group = (uint8_t)g;
+    S.bfm = (uint8_t)bfm;
+    S.slot = (uint8_t)slot;
+    S.dst_kind = (uint8_t)kind;
+    S.dst_reg = (uint8_t)reg;
+    S.n_elig = (uint8_t)ne;
+    S.pad = 0;
+    A.sites[i] = S;
+}
+
+size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
+
+struct IndexLayout {
+    size_t pk, pc, ws_k, ws_c, total;
+};
+IndexLayout layout(uint32_t n_inst, uint64_t n_chunks) {
+    IndexLayout L;
+    L.pk = 0;
+    L.pc = align256(((size_t)n_inst + 1) * 8 * sizeof(uint64_t));
+    L.ws_k = L.pc + align256(((size_t)n_chunks + 1) * 8 * sizeof(uint64_t));
+    L.ws_c = L.ws_k + align256(scan_rows_ws(n_inst, 8));
+    L.total = L.ws_c + align256(scan_rows_ws(n_chunks, 8));
+    return L;
+}
+
+}  // namespace
+}  // namespace fi
+
+using namespace fi;
+
+extern "C" size_t fi_site_index_bytes(uint32_t n_inst, uint64_t n_chunks) { return layout(n_inst, n_chunks).total; }
+
+extern "C" fi_status fi_build_site_index(const uint64_t* inst_counts, uint32_t n_inst, const uint32_t* chunk_counts,
+                                         uint64_t n_chunks, void* index, void* stream) {
+    if (!inst_counts || !chunk_counts || !index) return FI_E_ARG;
+    const IndexLayout L = layout(n_inst, n_chunks);
+    char* b = reinterpret_cast<char*>(index);
+    cudaStream_t s = (cudaStream_t)stream;
+    fi_status e = scan_rows_u64x8(inst_counts, reinterpret_cast<uint64_t*>(b + L.pk), n_inst, b + L.ws_k,
+                                  L.ws_c - L.ws_k, s);
+    if (e) return e;
+    return scan_rows_u32x8(chunk_counts, reinterpret_cast<uint64_t*>(b + L.pc), n_chunks, b + L.ws_c,
+                           L.total - L.ws_c, s);
+}
+
+extern "C" fi_status fi_site_totals(const void* index, uint32_t n_inst, uint64_t totals_host[8], void* stream) {
+    if (!index || !totals_host) return FI_E_ARG;
+    cudaStream_t s = (cudaStream_t)stream;
+    const uint64_t* pk = reinterpret_cast<const uint64_t*>(index);
+    fi_status e = cuda_status(cudaMemcpyAsync(totals_host, pk + (size_t)n_inst * 8, 8 * sizeof(uint64_t),
+                                              cudaMemcpyDeviceToHost, s));
+    if (e) return e;
+    return cuda_status(cudaStreamSynchronize(s));
+}
+
+extern "C" fi_status fi_select_sites(const fi_program* p, const fi_trace* t, const void* index, uint32_t n_inst,
+                                     uint64_t n_chunks, const uint64_t totals_host[8], const fi_schedule* sched,
+                                     uint64_t j0, uint32_t n, fi_site* sites, uint32_t* dev_status, void* stream) {
+    if (!p || !t || !index || !totals_host || !sched || !sites || !dev_status) return FI_E_ARG;
+    if (sched->n_groups == 0 || sched->n_groups > 8 || sched->n_bfms == 0 || sched->n_bfms > 4) return FI_E_ARG;
+    for (uint32_t i = 0; i < sched->n_groups; ++i) {
+        if (sched->groups[i] >= FI_NGROUPS) return FI_E_ARG;
+        if (sched->groups[i] == FI_G_NODEST) return FI_E_NOT_INJECTABLE;     // C-16
+        if (totals_host[sched->groups[i]] == 0) return FI_E_EMPTY_GROUP;
+    }
+    for (uint32_t i = 0; i < sched->n_bfms; ++i)
+        if (sched->bfms[i] > FI_ZERO_VALUE) return FI_E_ARG;
+    if (n == 0) return FI_OK;
+    const IndexLayout L = layout(n_inst, n_chunks);
+    const char* b = reinterpret_cast<const char*>(index);
+    SelArgs A;
+    A.code = p->code; A.kern = p->kern; A.inst = p->inst;
+    A.rec = reinterpret_cast<const uint4*>(t->rec); A.n_rec = t->n_rec; A.warp_off = t->warp_off; A.n_warps = t->n_warps;
+    A.Pk = reinterpret_cast<const uint64_t*>(b + L.pk); A.n_inst = n_inst;
+    A.Pc = reinterpret_cast<const uint64_t*>(b + L.pc); A.n_chunks = n_chunks;
+    for (int g = 0; g < 8; ++g) A.totals[g] = totals_host[g];
+    A.sched = *sched;
+    A.j0 = j0; A.n = n; A.sites = sites; A.status = dev_status;
+    k_select<<<(n + kWarps - 1) / kWarps, kWarps * 32, 0, (cudaStream_t)stream>>>(A);
+    return launch_status();
+}

@@ -1,0 +1,341 @@
+"""ctypes binding of libfi.so (include/fi.h) — argument marshalling only.
+
+Every step of the path runs in the CUDA kernels behind the C ABI; PyTorch only
+allocates device memory and supplies the current stream.  There is no CPU
+fallback: if libfi.so is missing or no CUDA device is present, calls raise.
+The function names mirror fi.h (fi_golden_lengths, fi_profile, fi_select_sites,
+fi_inject, fi_classify, ...).
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+from dataclasses import dataclass
+
+import numpy as np
+import torch
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(HERE, "libfi.so")
+
+FI_OK, FI_E_ARG, FI_E_EMPTY_GROUP, FI_E_NOT_INJECTABLE, FI_E_PROGRAM, FI_E_CUDA, FI_E_SITE = 0, 1, 2, 3, 4, 5, 6
+FI_E_CAPACITY = 8
+FI_CHUNK = 1024
+G_FP64, G_FP32, G_LD, G_PR, G_NODEST, G_OTHERS, G_GPPR, G_GP = range(8)
+GROUP_NAMES = ["G_FP64", "G_FP32", "G_LD", "G_PR", "G_NODEST", "G_OTHERS", "G_GPPR", "G_GP"]
+BFM_NAMES = ["FLIP_SINGLE_BIT", "FLIP_TWO_BITS", "RANDOM_VALUE", "ZERO_VALUE"]
+MASKED, SDC, DUE = 0, 1, 2
+
+SITE_DTYPE = np.dtype([
+    ("s", "<u8"), ("instruction_count", "<u8"),
+    ("instance", "<u4"), ("kernel_id", "<u4"), ("kernel_count", "<u4"), ("warp", "<u4"),
+    ("step", "<u4"), ("thread", "<u4"), ("pc", "<u4"), ("u_dst", "<u4"), ("u_bit", "<u4"), ("mask", "<u4"),
+    ("lane", "u1"), ("group", "u1"), ("bfm", "u1"), ("slot", "u1"), ("dst_kind", "u1"), ("dst_reg", "u1"),
+    ("n_elig", "u1"), ("pad", "u1"),
+])
+INJ_DTYPE = np.dtype([("before", "<u4"), ("after", "<u4"), ("mask", "<u4"), ("fault_pc", "<u4"),
+                      ("fault_kind", "u1"), ("outcome", "u1"), ("overflow", "u1"), ("pad", "u1"),
+                      ("n_faulty_stores", "<u4")])
+RECORD_DTYPE = np.dtype([("instance", "<u4"), ("insn", "<u4"), ("active", "<u4"), ("pred", "<u4")])
+STORE_DTYPE = np.dtype([("va", "<u8"), ("value", "<u4"), ("step", "<u4")])
+assert SITE_DTYPE.itemsize == 64 and INJ_DTYPE.itemsize == 24
+
+
+class FIError(RuntimeError):
+    def __init__(self, code: int, where: str, detail: str = ""):
+        self.code = code
+        super().__init__(f"{where}: {status_str(code)} ({code}){' — ' + detail if detail else ''}")
+
+
+class fi_program(C.Structure):
+    _fields_ = [("code", C.c_void_p), ("n_code", C.c_uint32),
+                ("kern", C.c_void_p), ("n_kern", C.c_uint32),
+                ("inst", C.c_void_p), ("n_inst", C.c_uint32),
+                ("cbank", C.c_void_p), ("n_cbank", C.c_uint32),
+                ("buf", C.c_void_p), ("n_buf", C.c_uint32),
+                ("gran", C.c_void_p),
+                ("image_bytes", C.c_uint64),
+                ("n_warps", C.c_uint32), ("n_regs", C.c_uint32),
+                ("code_host", C.c_void_p), ("inst_host", C.c_void_p)]
+
+
+class fi_trace(C.Structure):
+    _fields_ = [("rec", C.c_void_p), ("n_rec", C.c_uint64), ("warp_off", C.c_void_p),
+                ("gstore", C.c_void_p), ("gstore_off", C.c_void_p), ("n_warps", C.c_uint32)]
+
+
+class fi_schedule(C.Structure):
+    _fields_ = [("seed", C.c_uint64), ("n_groups", C.c_uint32), ("n_bfms", C.c_uint32),
+                ("groups", C.c_uint8 * 8), ("bfms", C.c_uint8 * 4)]
+
+
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise FIError(FI_E_CUDA, "load", f"{LIB_PATH} not built (run __graft_entry__.build())")
+        L = C.CDLL(LIB_PATH)
+        vp, u32, u64, sz = C.c_void_p, C.c_uint32, C.c_uint64, C.c_size_t
+        st = C.c_int
+        sig = {
+            "fi_status_str": (C.c_char_p, [st]),
+            "fi_last_cuda_error": (C.c_char_p, []),
+            "fi_version": (C.c_char_p, []),
+            "fi_program_regs": (u32, [vp, u32]),
+            "fi_build_granule_map": (st, [vp, vp, vp]),
+            "fi_golden_lengths": (st, [vp, vp, vp, vp, vp, vp]),
+            "fi_scan_u64_workspace": (sz, [u64]),
+            "fi_scan_u64": (st, [vp, vp, u64, vp, sz, vp]),
+            "fi_golden_trace": (st, [vp, vp, vp, vp, vp, vp, vp, vp]),
+            "fi_profile": (st, [vp, u64, u64, u32, vp, vp, vp]),
+            "fi_site_index_bytes": (sz, [u32, u64]),
+            "fi_build_site_index": (st, [vp, u32, vp, u64, vp, vp]),
+            "fi_site_totals": (st, [vp, u32, vp, vp]),
+            "fi_select_sites": (st, [vp, vp, vp, u32, u64, vp, vp, u64, u32, vp, vp, vp]),
+            "fi_inject": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, vp]),
+            "fi_classify": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, vp, vp]),
+            "fi_write_params_txt": (st, [vp, C.c_char_p, C.c_char_p, sz]),
+        }
+        for name, (res, args) in sig.items():
+            f = getattr(L, name)
+            f.restype, f.argtypes = res, args
+        _lib = L
+    return _lib
+
+
+def status_str(code: int) -> str:
+    try:
+        return lib().fi_status_str(code).decode()
+    except Exception:
+        return "unknown"
+
+
+def _check(rc: int, where: str):
+    if rc != FI_OK:
+        detail = lib().fi_last_cuda_error().decode() if rc == FI_E_CUDA else ""
+        raise FIError(rc, where, detail)
+
+
+def _stream() -> int:
+    return torch.cuda.current_stream().cuda_stream
+
+
+def _p(t: torch.Tensor | None) -> int | None:
+    return None if t is None else t.data_ptr()
+
+
+def _to_dev(a: np.ndarray, device) -> torch.Tensor:
+    b = np.ascontiguousarray(a).view(np.uint8).reshape(-1)
+    if b.size == 0:
+        return torch.empty(16, dtype=torch.uint8, device=device)
+    return torch.from_numpy(b.copy()).to(device, non_blocking=False)
+
+
+class DeviceStatus:
+    """The caller-owned device word that kernels OR error bits into."""
+
+    def __init__(self, device):
+        self.t = torch.zeros(1, dtype=torch.int32, device=device)
+
+    @property
+    def ptr(self):
+        return self.t.data_ptr()
+
+    def check(self, where: str):
+        v = int(self.t.item()) & 0xFFFFFFFF
+        if v:
+            code = (v & -v).bit_length() - 1
+            raise FIError(code, where, f"device status bits {v:#x}")
+
+
+class DeviceProgram:
+    """A program (fi_inputs.Program) resident on the GPU, plus its fi_program struct."""
+
+    def __init__(self, prog, device="cuda"):
+        self.prog = prog
+        self.device = torch.device(device)
+        self.code = _to_dev(prog.code, self.device)
+        self.kern = _to_dev(prog.kernels, self.device)
+        self.inst = _to_dev(prog.instances, self.device)
+        self.cbank = _to_dev(prog.cbank, self.device)
+        self.buf = _to_dev(prog.buffers, self.device)
+        self.init_image = _to_dev(prog.init_image, self.device)
+        self.n_gran = (prog.image_bytes + 255) // 256
+        self.gran = torch.empty(max(self.n_gran, 1), dtype=torch.int32, device=self.device)
+        self._code_host = np.ascontiguousarray(prog.code)
+        self._inst_host = np.ascontiguousarray(prog.instances)
+        self.n_regs = int(lib().fi_program_regs(self._code_host.ctypes.data, len(self._code_host)))
+        self.c = fi_program(
+            _p(self.code), len(prog.code), _p(self.kern), len(prog.kernels), _p(self.inst), len(prog.instances),
+            _p(self.cbank), len(prog.cbank), _p(self.buf), len(prog.buffers), _p(self.gran),
+            prog.image_bytes, prog.n_warps, self.n_regs, self._code_host.ctypes.data, self._inst_host.ctypes.data)
+        _check(lib().fi_build_granule_map(C.byref(self.c), _p(self.gran), _stream()), "fi_build_granule_map")
+
+    @property
+    def n_inst(self):
+        return len(self.prog.instances)
+
+    @property
+    def n_warps(self):
+        return self.prog.n_warps
+
+
+@dataclass
+class GoldenTrace:
+    dp: DeviceProgram
+    image: torch.Tensor          # golden final image (u8)
+    warp_len: torch.Tensor
+    warp_off: torch.Tensor       # [W+1] u64 (int64 tensor)
+    gstore_off: torch.Tensor
+    rec: torch.Tensor            # [R*16] u8
+    gstore: torch.Tensor
+    n_rec: int
+    n_gstore: int
+    c: fi_trace
+
+    @property
+    def n_chunks(self):
+        return (self.n_rec + FI_CHUNK - 1) // FI_CHUNK
+
+
+def scan_u64(x: torch.Tensor) -> torch.Tensor:
+    n = x.numel()
+    out = torch.empty(n + 1, dtype=torch.int64, device=x.device)
+    ws_n = lib().fi_scan_u64_workspace(n)
+    ws = torch.empty(max(ws_n, 1), dtype=torch.uint8, device=x.device)
+    _check(lib().fi_scan_u64(_p(x), _p(out), n, _p(ws), ws_n, _stream()), "fi_scan_u64")
+    return out
+
+
+def golden_run(dp: DeviceProgram, keep_records: bool = True) -> GoldenTrace:
+    """fi_golden_lengths (pass 1) -> scans -> fi_golden_trace (pass 2)."""
+    st = DeviceStatus(dp.device)
+    image = dp.init_image.clone()
+    W = dp.n_warps
+    wl = torch.zeros(max(W, 1), dtype=torch.int64, device=dp.device)
+    wn = torch.zeros(max(W, 1), dtype=torch.int64, device=dp.device)
+    _check(lib().fi_golden_lengths(C.byref(dp.c), _p(image), _p(wl), _p(wn), st.ptr, _stream()), "fi_golden_lengths")
+    woff = scan_u64(wl[:W])
+    goff = scan_u64(wn[:W])
+    st.check("fi_golden_lengths")
+    n_rec = int(woff[W].item())
+    n_gst = int(goff[W].item())
+    rec = torch.empty(max(n_rec, 1) * 16, dtype=torch.uint8, device=dp.device)
+    gst = torch.empty(max(n_gst, 1) * 16, dtype=torch.uint8, device=dp.device)
+    _check(lib().fi_golden_trace(C.byref(dp.c), _p(image), _p(woff), _p(goff), _p(rec), _p(gst), st.ptr, _stream()),
+           "fi_golden_trace")
+    st.check("fi_golden_trace")
+    tc = fi_trace(_p(rec), n_rec, _p(woff), _p(gst), _p(goff), W)
+    return GoldenTrace(dp, image, wl[:W], woff, goff, rec, gst, n_rec, n_gst, tc)
+
+
+def profile(gt: GoldenTrace, rec_begin: int = 0, rec_end: int | None = None,
+            inst_counts: torch.Tensor | None = None, chunk_counts: torch.Tensor | None = None):
+    """fi_profile (K1) over records [rec_begin, rec_end)."""
+    rec_end = gt.n_rec if rec_end is None else rec_end
+    K = gt.dp.n_inst
+    if inst_counts is None:
+        inst_counts = torch.empty((K, 8), dtype=torch.int64, device=gt.dp.device)
+    if chunk_counts is None:
+        chunk_counts = torch.zeros((max(gt.n_chunks, 1), 8), dtype=torch.int32, device=gt.dp.device)
+    _check(lib().fi_profile(C.byref(gt.c), rec_begin, rec_end, K, _p(inst_counts), _p(chunk_counts), _stream()),
+           "fi_profile")
+    return inst_counts, chunk_counts
+
+
+class SiteIndex:
+    """fi_build_site_index (K2): P_k and P_c prefix sums; totals N_g."""
+
+    def __init__(self, gt: GoldenTrace, inst_counts: torch.Tensor, chunk_counts: torch.Tensor):
+        self.gt = gt
+        self.n_inst = gt.dp.n_inst
+        self.n_chunks = gt.n_chunks
+        nb = lib().fi_site_index_bytes(self.n_inst, self.n_chunks)
+        self.buf = torch.empty(nb, dtype=torch.uint8, device=gt.dp.device)
+        _check(lib().fi_build_site_index(_p(inst_counts), self.n_inst, _p(chunk_counts), self.n_chunks,
+                                         _p(self.buf), _stream()), "fi_build_site_index")
+        tot = (C.c_uint64 * 8)()
+        _check(lib().fi_site_totals(_p(self.buf), self.n_inst, tot, _stream()), "fi_site_totals")
+        self.totals = [int(x) for x in tot]
+        self._tot = tot
+
+    def prefix_inst(self) -> torch.Tensor:
+        return self.buf[: (self.n_inst + 1) * 64].view(torch.int64).view(self.n_inst + 1, 8)
+
+
+def schedule(seed: int, groups, bfms) -> fi_schedule:
+    s = fi_schedule()
+    s.seed = seed
+    s.n_groups, s.n_bfms = len(groups), len(bfms)
+    for i, g in enumerate(groups):
+        s.groups[i] = g
+    for i, b in enumerate(bfms):
+        s.bfms[i] = b
+    return s
+
+
+def select_sites(idx: SiteIndex, sched: fi_schedule, j0: int, n: int, sites: torch.Tensor | None = None,
+                 status: DeviceStatus | None = None) -> torch.Tensor:
+    """fi_select_sites (K3): returns a [n*64] u8 tensor of fi_site."""
+    gt = idx.gt
+    if sites is None:
+        sites = torch.empty(max(n, 1) * 64, dtype=torch.uint8, device=gt.dp.device)
+    st = status or DeviceStatus(gt.dp.device)
+    _check(lib().fi_select_sites(C.byref(gt.dp.c), C.byref(gt.c), _p(idx.buf), idx.n_inst, idx.n_chunks,
+                                 idx._tot, C.byref(sched), j0, n, _p(sites), st.ptr, _stream()), "fi_select_sites")
+    if status is None:
+        st.check("fi_select_sites")
+    return sites
+
+
+def inject(gt: GoldenTrace, sites: torch.Tensor, n: int, log_cap: int, out: torch.Tensor | None = None,
+           log: torch.Tensor | None = None, status: DeviceStatus | None = None):
+    """fi_inject (K4)."""
+    dev = gt.dp.device
+    if out is None:
+        out = torch.empty(max(n, 1) * 24, dtype=torch.uint8, device=dev)
+    if log is None:
+        log = torch.empty(max(n * log_cap, 1) * 16, dtype=torch.uint8, device=dev)
+    st = status or DeviceStatus(dev)
+    _check(lib().fi_inject(C.byref(gt.dp.c), _p(gt.image), C.byref(gt.c), _p(sites), n, _p(out), _p(log), log_cap,
+                           st.ptr, _stream()), "fi_inject")
+    if status is None:
+        st.check("fi_inject")
+    return out, log
+
+
+def classify(gt: GoldenTrace, sites: torch.Tensor, n: int, out: torch.Tensor, log: torch.Tensor, log_cap: int,
+             hist: torch.Tensor | None = None, status: DeviceStatus | None = None) -> torch.Tensor:
+    """fi_classify (K5): fills out[].outcome, accumulates hist[8][4][3]."""
+    dev = gt.dp.device
+    if hist is None:
+        hist = torch.zeros((8, 4, 3), dtype=torch.int64, device=dev)
+    st = status or DeviceStatus(dev)
+    _check(lib().fi_classify(C.byref(gt.dp.c), _p(gt.image), C.byref(gt.c), _p(sites), n, _p(out), _p(log), log_cap,
+                             _p(hist), st.ptr, _stream()), "fi_classify")
+    if status is None:
+        st.check("fi_classify")
+    return hist
+
+
+def write_params_txt(site_row: np.ndarray, kernel_name: str) -> str:
+    a = np.ascontiguousarray(np.asarray(site_row, dtype=SITE_DTYPE).reshape(1))
+    buf = C.create_string_buffer(1024)
+    _check(lib().fi_write_params_txt(a.ctypes.data, kernel_name.encode(), buf, 1024), "fi_write_params_txt")
+    return buf.value.decode()
+
+
+def as_numpy(t: torch.Tensor, dtype: np.dtype, n: int | None = None) -> np.ndarray:
+    a = t.detach().cpu().numpy().view(np.uint8).reshape(-1).view(dtype)
+    return a if n is None else a[:n]
+
+
+def log_capacity(gt: GoldenTrace) -> int:
+    """Per-replica faulty-store log slots: 2x the largest golden per-warp store
+    count + 4096 (replicas that exceed it are flagged, never mis-classified)."""
+    gs = gt.gstore_off
+    mx = int((gs[1:] - gs[:-1]).max().item()) if gt.dp.n_warps else 0
+    return 2 * mx + 4096

@@ -1,0 +1,163 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Bit-exact for everything (counts, trace bytes, golden images, sites, injected
+values, fault kinds, outcomes) — the whole path is integer or IEEE-exact (C-13),
+so the tolerance is 0 everywhere.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle as O
+import opcases
+from fi_inputs import programs as P
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def F():
+    from paper_conf_dsn_0002hsvk21_b200 import fi
+    return fi
+
+
+def _gpu_golden(F, prog):
+    dp = F.DeviceProgram(prog)
+    gt = F.golden_run(dp)
+    return dp, gt
+
+
+def _trace_np(F, gt):
+    return F.as_numpy(gt.rec, F.RECORD_DTYPE, gt.n_rec)
+
+
+def _site_fields(a):
+    names = [n for n in a.dtype.names if n != "pad"]
+    return np.stack([a[n].astype(np.uint64) for n in names], axis=1), names
+
+
+def _assert_sites_equal(g, o):
+    ga, names = _site_fields(g)
+    oa, _ = _site_fields(o)
+    bad = np.argwhere(ga != oa)
+    assert bad.size == 0, f"site {bad[0][0]} field {names[bad[0][1]]}: gpu {ga[bad[0][0]]} oracle {oa[bad[0][0]]}"
+
+
+def test_ops_conformance(F):
+    for name, rows, words, exp in opcases.cases(seed=77):
+        prog = opcases.build(rows, words, name)
+        dp, gt = _gpu_golden(F, prog)
+        img = gt.image.cpu().numpy()
+        y = prog.view(img, "Y", "<u4").reshape(-1, 8)
+        assert np.array_equal(y, exp), name
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_fuzz_trace_and_image(F, seed):
+    prog = P.fuzz_program(seed, n_ops=int(60 + seed * 7 % 140), block=[80, 64, 96, 33][seed % 4])
+    g = O.Golden(prog)
+    dp, gt = _gpu_golden(F, prog)
+    assert gt.n_rec == g.n_records
+    assert np.array_equal(gt.image.cpu().numpy(), g.final_image())
+    assert np.array_equal(_trace_np(F, gt), g.trace())
+    ic, cc = F.profile(gt)
+    assert np.array_equal(ic.cpu().numpy().astype(np.uint64), g.counts())
+
+
+def _campaign_parity(F, prog, seed, groups, bfms, n, mode):
+    g = O.Golden(prog)
+    dp, gt = _gpu_golden(F, prog)
+    assert np.array_equal(_trace_np(F, gt), g.trace())
+    assert np.array_equal(gt.image.cpu().numpy(), g.final_image())
+    ic, cc = F.profile(gt)
+    assert np.array_equal(ic.cpu().numpy().astype(np.uint64), g.counts())
+    idx = F.SiteIndex(gt, ic, cc)
+    sites = F.select_sites(idx, F.schedule(seed, groups, bfms), 0, n)
+    gs = F.as_numpy(sites, F.SITE_DTYPE, n)
+    os_ = g.select(seed, groups, bfms, 0, n)
+    _assert_sites_equal(gs, os_)
+    cap = F.log_capacity(gt)
+    out, log = F.inject(gt, sites, n, cap)
+    hist = F.classify(gt, sites, n, out, log, cap)
+    gi = F.as_numpy(out, F.INJ_DTYPE, n)
+    oi = g.inject(os_, mode)
+    for f in ("before", "after", "mask", "fault_kind", "outcome"):
+        bad = np.flatnonzero(gi[f] != oi[f])
+        assert bad.size == 0, f"{f}: replica {bad[0]} gpu {gi[bad[0]]} oracle {oi[bad[0]]} site {os_[bad[0]]}"
+    assert (gi["fault_pc"][gi["fault_kind"] > 0] == oi["fault_pc"][oi["fault_kind"] > 0]).all()
+    assert np.array_equal(hist.cpu().numpy().astype(np.uint64), O.histogram(os_, oi))
+    return gi, oi
+
+
+def test_c1_full_parity(F):
+    # C1: 100 replicas, G_GP, FLIP_SINGLE_BIT, oracle in full-program mode (the definition)
+    _campaign_parity(F, P.c1(), P.CAMPAIGN_SEED[1], [F.G_GP], [0], 100, O.MODE_FULL)
+
+
+def test_c1_all_models_groups(F):
+    _campaign_parity(F, P.vector_add(n=1000), 0x1234, [F.G_GP, F.G_PR, F.G_LD, F.G_FP32, F.G_OTHERS, F.G_GPPR],
+                     [0, 1, 2, 3], 600, O.MODE_FULL)
+
+
+def test_mini_c2_parity(F):
+    gi, oi = _campaign_parity(F, P.c2(full=False), P.CAMPAIGN_SEED[2], [F.G_GP], [0, 1, 2, 3], 400, O.MODE_WARP_LOCAL)
+    assert len(np.unique(oi["outcome"])) >= 2
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_fuzz_campaign_parity(F, seed):
+    prog = P.fuzz_program(100 + seed, n_ops=100)
+    _campaign_parity(F, prog, 0xABC0 + seed, [F.G_GPPR, F.G_GP, F.G_PR, F.G_FP32, F.G_FP64, F.G_OTHERS][: 1 + seed % 6],
+                     [0, 1, 2, 3], 300, O.MODE_FULL)
+
+
+def test_multi_instance_profile_and_select(F):
+    prog = P.multi_instance_chain(n_inst=4)
+    g = O.Golden(prog)
+    dp, gt = _gpu_golden(F, prog)
+    assert np.array_equal(_trace_np(F, gt), g.trace())
+    ic, cc = F.profile(gt)
+    assert np.array_equal(ic.cpu().numpy().astype(np.uint64), g.counts())
+    idx = F.SiteIndex(gt, ic, cc)
+    sites = F.select_sites(idx, F.schedule(99, [F.G_GP, F.G_LD], [0, 3]), 0, 200)
+    _assert_sites_equal(F.as_numpy(sites, F.SITE_DTYPE, 200), g.select(99, [F.G_GP, F.G_LD], [0, 3], 0, 200))
+
+
+def test_profile_shards_sum(F):
+    prog = P.c2(full=False)
+    dp, gt = _gpu_golden(F, prog)
+    full, cfull = F.profile(gt)
+    cut = (gt.n_rec // 3) // F.FI_CHUNK * F.FI_CHUNK
+    a, ca = F.profile(gt, 0, cut)
+    b, cb = F.profile(gt, cut, gt.n_rec)
+    assert torch.equal(a + b, full)
+    nc = cut // F.FI_CHUNK
+    assert torch.equal(ca[:nc], cfull[:nc]) and torch.equal(cb[nc:], cfull[nc:])
+
+
+def test_errors(F):
+    prog = P.c1()
+    dp, gt = _gpu_golden(F, prog)
+    ic, cc = F.profile(gt)
+    idx = F.SiteIndex(gt, ic, cc)
+    with pytest.raises(F.FIError) as e:
+        F.select_sites(idx, F.schedule(1, [F.G_NODEST], [0]), 0, 4)
+    assert e.value.code == F.FI_E_NOT_INJECTABLE
+    with pytest.raises(F.FIError) as e:
+        F.select_sites(idx, F.schedule(1, [F.G_FP64], [0]), 0, 4)
+    assert e.value.code == F.FI_E_EMPTY_GROUP
+    s = F.select_sites(idx, F.schedule(1, [F.G_GP], [0]), 0, 1)
+    txt = F.write_params_txt(F.as_numpy(s, F.SITE_DTYPE, 1)[0], "vecadd")
+    lines = txt.strip().split("\n")
+    assert len(lines) == 7 and lines[0] == str(F.G_GP) and lines[2] == "vecadd"
+
+
+def test_empty_and_ragged(F):
+    # ragged: n not a multiple of the block, partial warps (block = 48)
+    prog = P.vector_add(n=777, grid=17, block=48)
+    _campaign_parity(F, prog, 5, [F.G_GP], [0, 3], 150, O.MODE_FULL)
+    # zero replicas is a no-op
+    dp, gt = _gpu_golden(F, prog)
+    ic, cc = F.profile(gt)
+    idx = F.SiteIndex(gt, ic, cc)
+    F.select_sites(idx, F.schedule(1, [F.G_GP], [0]), 0, 0)
