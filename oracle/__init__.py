@@ -94,6 +94,8 @@ def lib():
             L.orc_select.argtypes = [vp, u64, vp, u32, vp, u32, u64, u32, vp]
             L.orc_locate.argtypes = [vp, i32, vp, u32, vp]
             L.orc_inject.argtypes = [vp, vp, u32, i32, i32, vp]
+            L.orc_warp_site_rank.argtypes = [C.POINTER(_Program), u32, i32, u32, u32, C.POINTER(u64), C.POINTER(u64)]
+            L.orc_inject_local.argtypes = [C.POINTER(_Program), vp, u32, i32, vp, vp]
             L.orc_philox4x32_10.argtypes = [vp, vp, vp]
             L.orc_draw.argtypes = [u64, u64, u64, C.POINTER(u64), C.POINTER(u32), C.POINTER(u32), C.POINTER(u32)]
             L.orc_mask.restype = u32
@@ -210,6 +212,31 @@ def count_warps(prog, w0: int, w1: int, n_threads: int | None = None) -> tuple[i
     out = np.zeros(8, dtype=np.uint64)
     n = lib().orc_count_warps(C.byref(p), w0, w1, n_threads or n_threads_default(), _ptr(out))
     return int(n), out
+
+
+def warp_site_rank(prog, warp: int, group: int, step: int, lane: int) -> tuple[int, int] | None:
+    """(rank of (step, lane) among warp `warp`'s group sites, warp total) for a
+    single-instance program, or None if (step, lane) is not a site."""
+    p, keep = _cprog(prog)
+    r, t = C.c_uint64(), C.c_uint64()
+    rc = lib().orc_warp_site_rank(C.byref(p), warp, group, step, lane, C.byref(r), C.byref(t))
+    if rc == 2:
+        raise OracleError(rc, "orc_warp_site_rank: not a single-instance program")
+    return None if rc else (r.value, t.value)
+
+
+def inject_local(prog, sites: np.ndarray, n_threads: int | None = None) -> tuple[np.ndarray, np.ndarray]:
+    """Warp-local injection of a single-instance program without a golden handle.
+    Returns (inj, decided)."""
+    p, keep = _cprog(prog)
+    sites = np.ascontiguousarray(sites, dtype=SITE_DTYPE)
+    out = np.zeros(len(sites), dtype=INJ_DTYPE)
+    dec = np.zeros(len(sites), dtype=np.uint8)
+    rc = lib().orc_inject_local(C.byref(p), _ptr(sites), len(sites), n_threads or n_threads_default(),
+                                _ptr(out), _ptr(dec))
+    if rc:
+        raise OracleError(rc, "orc_inject_local failed")
+    return out, dec.astype(bool)
 
 
 def philox4x32_10(ctr, key) -> list[int]:

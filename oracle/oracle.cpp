@@ -808,3 +808,88 @@ extern "C" int orc_inject(void* h, const orc_site* sites, uint32_t n, int mode, 
     });
     return status;
 }
+
+// ---------------------------------------------------------------------------
+// Single-instance helpers that need no whole-program golden run (full-size
+// sampled parity and bounded CPU baselines).  Same definitions as above,
+// restricted to one warp: the golden warp w and the faulty warp w are
+// interpreted from the initial image (= the memory before the only instance).
+// ---------------------------------------------------------------------------
+
+// Rank of (step, lane) among the group-g sites of warp w in canonical order (C-3),
+// and warp w's total group-g count.  Returns 0, or 1 if (step, lane) is not a site.
+extern "C" int orc_warp_site_rank(const orc_program* p, uint32_t w, int g, uint32_t step, uint32_t lane,
+                                  uint64_t* rank, uint64_t* total) {
+    Prog P;
+    std::string err;
+    if (!prepare(P, p, err) || P.p.n_inst != 1 || w >= P.n_warps) return 2;
+    std::vector<uint8_t> mem(p->init_image, p->init_image + p->image_bytes);
+    std::vector<orc_record> tr;
+    TraceSink ts;
+    ts.rec = &tr;
+    std::vector<StoreW> st;
+    uint32_t cta, wic;
+    warp_coords(P.p.inst[0], w, cta, wic);
+    run_warp(P, mem, 0, cta, wic, nullptr, UINT64_MAX, &st, &ts, nullptr);
+    uint64_t before = 0, tot = 0;
+    bool hit = false;
+    for (size_t r = 0; r < tr.size(); ++r) {
+        if (!((tr[r].insn >> (24 + g)) & 1)) continue;
+        uint32_t ex = tr[r].active & tr[r].pred;
+        for (uint32_t l = 0; l < 32; ++l) {
+            if (!((ex >> l) & 1)) continue;
+            if (r == step && l == lane) { hit = true; before = tot; }
+            ++tot;
+        }
+    }
+    *rank = before;
+    *total = tot;
+    return hit ? 0 : 1;
+}
+
+// Warp-local injection without a whole-program golden run.  decided[i] = 0 when
+// the outcome needs the golden value of a word written by ANOTHER warp (a wild
+// faulty store into an output word outside warp w's golden stores) and no
+// decided SDC word exists; otherwise the outcome is exact.
+extern "C" int orc_inject_local(const orc_program* p, const orc_site* sites, uint32_t n, int n_threads,
+                                orc_inj* out, uint8_t* decided) {
+    Prog P;
+    std::string err;
+    if (!prepare(P, p, err) || P.p.n_inst != 1) return 2;
+    const std::vector<uint8_t> pre(p->init_image, p->init_image + p->image_bytes);
+    std::atomic<int> status{0};
+    parallel_for(n, n_threads, [&](uint32_t i) {
+        const orc_site& S = sites[i];
+        orc_inj& R = out[i];
+        memset(&R, 0, sizeof(R));
+        uint32_t cta, wic;
+        warp_coords(P.p.inst[0], S.warp, cta, wic);
+        std::vector<StoreW> gst, fst;
+        WarpResult gr = run_warp(P, pre, 0, cta, wic, nullptr, UINT64_MAX, &gst, nullptr, nullptr);
+        Hook hk;
+        hk.on = true; hk.step = S.step; hk.lane = S.lane; hk.kind = S.dst_kind; hk.reg = S.dst_reg;
+        hk.bfm = S.bfm; hk.mask = S.mask; hk.pc = S.pc;
+        WarpResult fr = run_warp(P, pre, 0, cta, wic, &hk, 10 * gr.steps + 1024, &fst, nullptr, nullptr);
+        if (!hk.fired || hk.bad) status = 4;
+        R.before = hk.before; R.after = hk.after; R.mask = hk.applied_mask;
+        R.fault_kind = (uint8_t)fr.fault; R.fault_pc = fr.fault_pc;
+        R.n_faulty_stores = (uint32_t)fst.size();
+        decided[i] = 1;
+        if (fr.fault) { R.outcome = ORC_DUE; return; }
+        std::map<uint64_t, uint32_t> gold, fin;
+        for (const StoreW& s : gst) gold[s.va] = s.value;
+        for (const StoreW& s : fst) fin[s.va] = s.value;
+        for (const StoreW& s : gst)
+            if (!fin.count(s.va)) { uint32_t x; memcpy(&x, &pre[s.va - VA_BASE], 4); fin[s.va] = x; }
+        bool sdc = false, unknown = false;
+        for (auto& kv : fin) {
+            if (!is_output_addr(P, kv.first)) continue;
+            auto it = gold.find(kv.first);
+            if (it == gold.end()) { unknown = true; continue; }
+            if (it->second != kv.second) { sdc = true; break; }
+        }
+        R.outcome = sdc ? ORC_SDC : ORC_MASKED;
+        if (!sdc && unknown) decided[i] = 0;
+    });
+    return status;
+}

@@ -92,6 +92,12 @@ int orc_locate(void* h, int group, const uint64_t* s, uint32_t n, orc_site* out)
 /* injection + classification; mode ORC_MODE_FULL re-runs the whole program */
 int orc_inject(void* h, const orc_site* sites, uint32_t n, int mode, int n_threads, orc_inj* out);
 
+/* single-instance, no golden handle (full-size sampled parity, CPU baselines) */
+int orc_warp_site_rank(const orc_program* p, uint32_t w, int g, uint32_t step, uint32_t lane,
+                       uint64_t* rank, uint64_t* total);
+int orc_inject_local(const orc_program* p, const orc_site* sites, uint32_t n, int n_threads,
+                     orc_inj* out, uint8_t* decided);
+
 /* RNG / mask primitives */
 void orc_philox4x32_10(const uint32_t ctr[4], const uint32_t key[2], uint32_t out[4]);
 void orc_draw(uint64_t seed, uint64_t j, uint64_t n_g, uint64_t* s, uint32_t* u_dst, uint32_t* u_bit, uint32_t* attempts);

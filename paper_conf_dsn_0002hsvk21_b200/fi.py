@@ -154,15 +154,22 @@ class DeviceStatus:
 class DeviceProgram:
     """A program (fi_inputs.Program) resident on the GPU, plus its fi_program struct."""
 
-    def __init__(self, prog, device="cuda"):
+    def __init__(self, prog, device="cuda", host: dict | None = None):
+        """host: optional pinned uint8 CPU tensors keyed code/kernels/instances/
+        cbank/buffers/init_image (asynchronous H2D copies from pinned memory)."""
         self.prog = prog
         self.device = torch.device(device)
-        self.code = _to_dev(prog.code, self.device)
-        self.kern = _to_dev(prog.kernels, self.device)
-        self.inst = _to_dev(prog.instances, self.device)
-        self.cbank = _to_dev(prog.cbank, self.device)
-        self.buf = _to_dev(prog.buffers, self.device)
-        self.init_image = _to_dev(prog.init_image, self.device)
+
+        def up(key, arr):
+            if host is not None and host[key].numel():
+                return host[key].to(self.device, non_blocking=True)
+            return _to_dev(arr, self.device)
+        self.code = up("code", prog.code)
+        self.kern = up("kernels", prog.kernels)
+        self.inst = up("instances", prog.instances)
+        self.cbank = up("cbank", prog.cbank)
+        self.buf = up("buffers", prog.buffers)
+        self.init_image = up("init_image", prog.init_image)
         self.n_gran = (prog.image_bytes + 255) // 256
         self.gran = torch.empty(max(self.n_gran, 1), dtype=torch.int32, device=self.device)
         self._code_host = np.ascontiguousarray(prog.code)
