@@ -96,6 +96,8 @@ def lib():
             L.orc_inject.argtypes = [vp, vp, u32, i32, i32, vp]
             L.orc_warp_site_rank.argtypes = [C.POINTER(_Program), u32, i32, u32, u32, C.POINTER(u64), C.POINTER(u64)]
             L.orc_inject_local.argtypes = [C.POINTER(_Program), vp, u32, i32, vp, vp]
+            L.orc_warp_site_at.argtypes = [C.POINTER(_Program), u32, i32, u64, C.POINTER(u32), C.POINTER(u32),
+                                           C.POINTER(u32)]
             L.orc_philox4x32_10.argtypes = [vp, vp, vp]
             L.orc_draw.argtypes = [u64, u64, u64, C.POINTER(u64), C.POINTER(u32), C.POINTER(u32), C.POINTER(u32)]
             L.orc_mask.restype = u32
@@ -223,6 +225,38 @@ def warp_site_rank(prog, warp: int, group: int, step: int, lane: int) -> tuple[i
     if rc == 2:
         raise OracleError(rc, "orc_warp_site_rank: not a single-instance program")
     return None if rc else (r.value, t.value)
+
+
+def warp_site_at(prog, warp: int, group: int, rank: int) -> tuple[int, int, int] | None:
+    """(step, lane, pc) of the rank-th group site of warp `warp` (single-instance)."""
+    p, keep = _cprog(prog)
+    st, ln, pc = C.c_uint32(), C.c_uint32(), C.c_uint32()
+    rc = lib().orc_warp_site_at(C.byref(p), warp, group, rank, C.byref(st), C.byref(ln), C.byref(pc))
+    if rc == 2:
+        raise OracleError(rc, "orc_warp_site_at: not a single-instance program")
+    return None if rc else (st.value, ln.value, pc.value)
+
+
+def build_site(prog, seed: int, j: int, group: int, bfm: int, per_warp_total: int, n_total: int) -> np.ndarray:
+    """The oracle's own site for replica j of a single-instance program whose
+    warps all have `per_warp_total` group sites (a closed form the caller pins):
+    draw s (C-5), w = s // per_warp_total, locate the rank inside warp w by
+    enumeration (C-3), then slot (C-6) and mask (C-8)."""
+    s, u_dst, u_bit, _ = draw(seed, j, n_total)
+    w, rank = divmod(s, per_warp_total)
+    step, lane, pc = warp_site_at(prog, w, group, rank)
+    inst = prog.instances[0]
+    wpc = (int(inst["block"]) + 31) // 32
+    row = np.zeros(1, dtype=SITE_DTYPE)
+    slots = dest_slots(prog.code[int(prog.kernels[int(inst["kernel"])]["code_off"]) + pc], group)
+    slot = (len(slots) * u_dst) >> 32
+    row["s"], row["instruction_count"], row["instance"], row["kernel_id"] = s, s, 0, int(inst["kernel"])
+    row["kernel_count"], row["warp"], row["step"], row["pc"] = int(inst["kernel_count"]), w, step, pc
+    row["thread"] = (w // wpc) * int(inst["block"]) + (w % wpc) * 32 + lane
+    row["u_dst"], row["u_bit"], row["mask"] = u_dst, u_bit, mask(bfm, u_bit)
+    row["lane"], row["group"], row["bfm"], row["slot"] = lane, group, bfm, slot
+    row["dst_kind"], row["dst_reg"], row["n_elig"] = slots[slot][0], slots[slot][1], len(slots)
+    return row
 
 
 def inject_local(prog, sites: np.ndarray, n_threads: int | None = None) -> tuple[np.ndarray, np.ndarray]:

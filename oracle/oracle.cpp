@@ -847,6 +847,34 @@ extern "C" int orc_warp_site_rank(const orc_program* p, uint32_t w, int g, uint3
     return hit ? 0 : 1;
 }
 
+// The inverse: the (step, lane, pc) of the rank-th group-g site of warp w
+// (canonical order, C-3).  Returns 0, or 1 if rank >= warp w's group-g count.
+extern "C" int orc_warp_site_at(const orc_program* p, uint32_t w, int g, uint64_t rank,
+                                uint32_t* step, uint32_t* lane, uint32_t* pc) {
+    Prog P;
+    std::string err;
+    if (!prepare(P, p, err) || P.p.n_inst != 1 || w >= P.n_warps) return 2;
+    std::vector<uint8_t> mem(p->init_image, p->init_image + p->image_bytes);
+    std::vector<orc_record> tr;
+    TraceSink ts;
+    ts.rec = &tr;
+    std::vector<StoreW> st;
+    uint32_t cta, wic;
+    warp_coords(P.p.inst[0], w, cta, wic);
+    run_warp(P, mem, 0, cta, wic, nullptr, UINT64_MAX, &st, &ts, nullptr);
+    uint64_t seen = 0;
+    for (size_t r = 0; r < tr.size(); ++r) {
+        if (!((tr[r].insn >> (24 + g)) & 1)) continue;
+        uint32_t ex = tr[r].active & tr[r].pred;
+        for (uint32_t l = 0; l < 32; ++l) {
+            if (!((ex >> l) & 1)) continue;
+            if (seen == rank) { *step = (uint32_t)r; *lane = l; *pc = tr[r].insn & 0xFFFF; return 0; }
+            ++seen;
+        }
+    }
+    return 1;
+}
+
 // Warp-local injection without a whole-program golden run.  decided[i] = 0 when
 // the outcome needs the golden value of a word written by ANOTHER warp (a wild
 // faulty store into an output word outside warp w's golden stores) and no

@@ -95,6 +95,8 @@ int orc_inject(void* h, const orc_site* sites, uint32_t n, int mode, int n_threa
 /* single-instance, no golden handle (full-size sampled parity, CPU baselines) */
 int orc_warp_site_rank(const orc_program* p, uint32_t w, int g, uint32_t step, uint32_t lane,
                        uint64_t* rank, uint64_t* total);
+int orc_warp_site_at(const orc_program* p, uint32_t w, int g, uint64_t rank,
+                     uint32_t* step, uint32_t* lane, uint32_t* pc);
 int orc_inject_local(const orc_program* p, const orc_site* sites, uint32_t n, int n_threads,
                      orc_inj* out, uint8_t* decided);
 

@@ -11,6 +11,7 @@ import pytest
 
 import oracle as O
 from fi_inputs import isa, programs as P
+from closed_forms import sgemm_closed_form
 
 
 # ---------------------------------------------------------------------------
@@ -168,7 +169,7 @@ def test_predicated_off_lanes_not_counted():
     assert g.n_records == 576
 
 
-def sgemm_closed_form(M, N, K):
+def _unused_sgemm_closed_form(M, N, K):
     """Per-thread counts of the C2 kernel (fi_inputs.programs.sgemm_code), by
     hand from the listing: prologue 17 insns, 73 per k-iteration (4 LDG.128,
     64 FFMA, 2 IMAD.WIDE + IADD3, ISETP, BRA — the last BRA predicated off),
