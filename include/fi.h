@@ -57,7 +57,7 @@ typedef struct {
     const fi_instance* inst;  uint32_t n_inst;       /* device */
     const uint32_t* cbank;    uint32_t n_cbank;      /* device */
     const fi_buffer* buf;     uint32_t n_buf;        /* device, sorted by off */
-    const uint32_t* gran;                            /* device [ceil(image_bytes/256)]: buffer id per 256-B granule, from fi_build_granule_map */
+    const void* aux;                                 /* device, fi_program_aux_bytes(): written by fi_program_prepare */
     uint64_t image_bytes;
     uint32_t n_warps;
     uint32_t n_regs;                                 /* register rows the emulator keeps: from fi_program_regs() */
@@ -69,11 +69,16 @@ typedef struct {
 typedef struct { uint32_t instance, insn, active, pred; } fi_record;   /* insn = pc | op<<16 | groupmask<<24 */
 typedef struct { uint64_t va; uint32_t value, step; } fi_store;        /* one stored 32-bit word, 16 B */
 
+/* The trace and the golden-run side data.  fi_golden_trace writes rec, gstore
+ * and ckpt; every other call only reads them. */
 typedef struct {
-    const fi_record* rec;     uint64_t n_rec;        /* device */
+    fi_record* rec;           uint64_t n_rec;        /* device */
     const uint64_t* warp_off;                        /* device [n_warps+1]: first record of each warp */
-    const fi_store* gstore;                          /* device: golden store log, per warp contiguous */
+    fi_store* gstore;                                /* device: golden store log, per warp contiguous */
     const uint64_t* gstore_off;                      /* device [n_warps+1] */
+    uint32_t* ckpt;                                  /* device: golden register-file checkpoints, or NULL */
+    const uint64_t* ckpt_off;                        /* device [n_warps+1], in checkpoints (fi_ckpt_layout) */
+    uint32_t ckpt_interval;                          /* steps between checkpoints (0 = none) */
     uint32_t n_warps;
 } fi_trace;
 
@@ -107,9 +112,11 @@ const char* fi_version(void);
  * register index the code can touch (host scan of code_host).  Host only. */
 uint32_t fi_program_regs(const fi_insn* code_host, uint32_t n_code);
 
-/* Granule map: gran[i] = id of the buffer containing byte 256*i of the image,
- * 0xFFFFFFFF if none (C-15).  `gran` has ceil(image_bytes/256) entries. */
-fi_status fi_build_granule_map(const fi_program* p, uint32_t* gran, void* stream);
+/* Prepared program data, built once per program into `aux` (then set
+ * p->aux = aux): the granule map (buffer id per 256-B granule of the image,
+ * for the C-15 access check) and the pre-decoded code the emulator executes. */
+size_t fi_program_aux_bytes(uint64_t image_bytes, uint32_t n_code);
+fi_status fi_program_prepare(const fi_program* p, void* aux, void* stream);
 
 /* Golden run, pass 1 — PAPER.md:72 step (1)/(4) golden state.  Executes the
  * instances in launch order on `image` (in: initial image, out: golden final
@@ -123,11 +130,20 @@ fi_status fi_golden_lengths(const fi_program* p, uint8_t* image, uint64_t* warp_
 size_t fi_scan_u64_workspace(uint64_t n);
 fi_status fi_scan_u64(const uint64_t* in, uint64_t* out, uint64_t n, void* ws, size_t ws_bytes, void* stream);
 
+/* Checkpoint layout: warp w gets ceil(warp_len[w] / interval) checkpoints
+ * (before steps 0, interval, 2*interval, ...); ckpt_off[n_warps+1] is their
+ * exclusive scan.  Each checkpoint is fi_ckpt_bytes(n_regs) bytes.  Scratch:
+ * fi_ckpt_layout_workspace(n_warps) bytes. */
+size_t fi_ckpt_bytes(uint32_t n_regs);
+size_t fi_ckpt_layout_workspace(uint32_t n_warps);
+fi_status fi_ckpt_layout(const uint64_t* warp_len, uint32_t n_warps, uint32_t interval, uint64_t* ckpt_off,
+                         void* ws, size_t ws_bytes, void* stream);
+
 /* Golden run, pass 2: re-executes every warp of every instance in ONE launch
- * over the golden final image and writes the trace records (App. A.3) and the
- * golden store log, at warp_off / gstore_off (exclusive scans of pass 1). */
-fi_status fi_golden_trace(const fi_program* p, const uint8_t* image, const uint64_t* warp_off,
-                          const uint64_t* gstore_off, fi_record* rec, fi_store* gstore,
+ * over the golden final image and writes, through t, the trace records
+ * (App. A.3), the golden store log and (if t->ckpt) the checkpoints, at
+ * t->warp_off / t->gstore_off / t->ckpt_off (exclusive scans of pass 1). */
+fi_status fi_golden_trace(const fi_program* p, const uint8_t* image, const fi_trace* t,
                           uint32_t* dev_status, void* stream);
 
 /* K1 — profile, "dynamic instruction counts for every opcode in
@@ -163,7 +179,9 @@ fi_status fi_select_sites(const fi_program* p, const fi_trace* t, const void* in
                           uint64_t j0, uint32_t n, fi_site* sites, uint32_t* dev_status, void* stream);
 
 /* K4 — inject: one CUDA warp re-executes the site's
- * synthetic warp from its first instruction over the golden final image; after
+ * synthetic warp over the golden final image — from its first instruction, or
+ * from the golden checkpoint at or before the site when t->ckpt is set (the
+ * prefix is fault-free, so both start states are the same); after
  * the site's instruction writes its destinations, lane `lane`'s destination
  * `dst_reg` is XOR-ed with the mask (ZERO_VALUE: mask = before; predicates C-7).
  * Stores after the site are logged to log[i*log_cap ...] (fi_store words).

@@ -7,6 +7,20 @@
 // shared memory (row n_regs is all zeros and serves RZ and any index >= n_regs),
 // so every register access is one bank-conflict-free LDS/STS.
 //
+// Hot-loop design:
+//  * instructions are pre-decoded once per program (fi_program_prepare) into
+//    16 B with register operands already turned into shared-memory row offsets;
+//  * while every live lane sits at the same pc (no divergence — the common case)
+//    the warp skips min-PC scheduling entirely (`conv`), falling back to
+//    REDUX.MIN + VOTE only while lanes are split;
+//  * FFMA (the dominant opcode of GEMM-like kernels) has its own fast path;
+//  * each lane caches its last two buffers' bounds, so most LDG/STG skip the
+//    granule-table lookup;
+//  * the golden trace pass stores a register-file checkpoint every
+//    `interval` steps, and an injection replica restarts from the checkpoint at
+//    or before its site instead of re-executing the whole prefix (the prefix is
+//    identical to the golden run by construction).
+//
 // Memory follows DESIGN.md §3.5: loads of instance k read the golden final
 // image where the buffer's writer < k and zero where writer >= k (equivalent to
 // the state before k under SSA), so neither the golden passes nor injection
@@ -14,7 +28,7 @@
 //
 // Modes:
 //   EMU_LEN    golden pass 1: stores go to the image; count steps and stored words
-//   EMU_TRACE  golden pass 2: write trace records (App. A.3) and the golden store log
+//   EMU_TRACE  golden pass 2: trace records (App. A.3), golden store log, checkpoints
 //   EMU_INJ    injection replica: corrupt one destination after
 //              the site's instruction; log stores after the site; faults end the run
 #pragma once
@@ -25,8 +39,41 @@ namespace fi {
 constexpr uint32_t kFull = 0xFFFFFFFFu;
 enum EmuMode { EMU_LEN = 0, EMU_TRACE = 1, EMU_INJ = 2 };
 
+// ---- prepared program data (fi_program.aux) --------------------------------
+struct AuxLayout { size_t gran, dec, ins, total; };
+__host__ __device__ inline size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
+__host__ __device__ inline AuxLayout aux_layout(uint64_t image_bytes, uint32_t n_code) {
+    AuxLayout L;
+    L.gran = 0;
+    L.dec = align256(((image_bytes + 255) >> 8) * sizeof(uint32_t));
+    L.ins = L.dec + align256((size_t)n_code * 16);
+    L.total = L.ins + align256((size_t)n_code * 4);
+    return L;
+}
+
+// decoded instruction (uint4):
+//   x = op | guard << 8 | mod << 16 | pb << 24     pb: IADD3 carry pred, *SETP dest pred, LOP3 lut, SEL pred
+//   y = ra_idx | rb_idx << 16                       smem word offsets (row*32), RZ / >= n_regs -> zero row
+//   z = rc_idx | d0_idx << 16                       d0_idx = 0xFFFF when the write is discarded
+//   w = imm
+__host__ __device__ inline uint4 decode_insn(const fi_insn& I, uint32_t zr) {
+    auto row = [&](uint32_t r) -> uint32_t { return (r < zr ? r : zr) * 32u; };
+    uint32_t pb = 0;
+    if (I.op == IADD3) pb = I.d1 & 7;
+    else if (I.op == ISETP || I.op == FSETP || I.op == DSETP) pb = I.d0 & 7;
+    else if (I.op == LOP3) pb = I.ext & 0xFF;
+    else if (I.op == SEL) pb = I.c & 0xF;
+    uint4 d;
+    d.x = (uint32_t)I.op | ((uint32_t)I.guard << 8) | ((uint32_t)I.mod << 16) | (pb << 24);
+    d.y = row(I.a) | (row(I.b) << 16);
+    d.z = row(I.c) | ((I.d0 < zr ? I.d0 * 32u : 0xFFFFu) << 16);
+    d.w = I.imm;
+    return d;
+}
+
 struct EmuProg {
-    const fi_insn* code;
+    const uint4* dec;          // decoded code
+    const uint32_t* ins;       // trace insn word per static instruction: pc | op<<16 | groupmask<<24
     const fi_kernel* kern;
     const fi_instance* inst;
     const uint32_t* cbank;
@@ -38,8 +85,15 @@ struct EmuProg {
 };
 
 inline EmuProg make_emu_prog(const fi_program* p) {
-    return EmuProg{p->code, p->kern, p->inst, p->cbank, p->buf, p->gran, p->image_bytes, p->n_regs, p->n_inst};
+    const AuxLayout L = aux_layout(p->image_bytes, p->n_code);
+    const char* a = reinterpret_cast<const char*>(p->aux);
+    return EmuProg{reinterpret_cast<const uint4*>(a + L.dec), reinterpret_cast<const uint32_t*>(a + L.ins),
+                   p->kern, p->inst, p->cbank, p->buf, reinterpret_cast<const uint32_t*>(a + L.gran),
+                   p->image_bytes, p->n_regs, p->n_inst};
 }
+
+// checkpoint = (n_regs + 3) rows of 32 words: registers, then pc, predicates, live
+__host__ __device__ inline size_t ckpt_bytes(uint32_t n_regs) { return (size_t)(n_regs + 3) * 128; }
 
 struct HookIn { uint32_t step, lane, kind, reg, bfm, mask, pc; };
 
@@ -113,266 +167,333 @@ __device__ __forceinline__ uint32_t dev_lop3(uint32_t a, uint32_t b, uint32_t c,
     return r;
 }
 
-// 0 ok, 1 misaligned, 2 unmapped (C-15).  On success *bid = buffer id.
-__device__ __forceinline__ uint32_t check_access(const EmuProg& P, uint64_t va, uint32_t w, uint32_t* bid) {
+// Per-lane two-entry cache of buffer bounds (image offsets) for memory checks.
+struct BufCache {
+    uint64_t lo0 = 1, hi0 = 0, lo1 = 1, hi1 = 0;   // empty ranges
+    bool z0 = false, z1 = false;                   // writer rule: reads of this buffer return 0
+};
+
+// 0 ok, 1 misaligned, 2 unmapped (C-15).  On success *zero = writer rule flag for instance k.
+__device__ __forceinline__ uint32_t check_access(const EmuProg& P, BufCache& C, uint64_t va, uint32_t w, uint32_t k,
+                                                 bool* zero) {
     if (va & (w - 1)) return 1;
-    uint64_t off = va - kVaBase;
+    const uint64_t off = va - kVaBase;
+    if (off >= C.lo0 && off + w <= C.hi0) { *zero = C.z0; return 0; }
+    if (off >= C.lo1 && off + w <= C.hi1) { *zero = C.z1; return 0; }
     if (va < kVaBase || off >= P.image_bytes) return 2;
-    uint32_t b = __ldg(&P.gran[off >> 8]);
+    const uint32_t b = __ldg(&P.gran[off >> 8]);
     if (b == kNoBuf) return 2;
-    uint64_t end = __ldg(&P.buf[b].off) + __ldg(&P.buf[b].size);
-    if (off + w > end) return 2;
-    *bid = b;
+    const uint64_t lo = __ldg(&P.buf[b].off), hi = lo + __ldg(&P.buf[b].size);
+    if (off + w > hi) return 2;
+    const int32_t wr = __ldg(&P.buf[b].writer);
+    C.lo1 = C.lo0; C.hi1 = C.hi0; C.z1 = C.z0;
+    C.lo0 = lo; C.hi0 = hi; C.z0 = wr >= 0 && (uint32_t)wr >= k;
+    *zero = C.z0;
     return 0;
 }
 
 template <int MODE>
-__device__ __noinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const uint8_t* img,
-                                       uint32_t k, uint32_t cta, uint32_t wic, uint32_t* __restrict__ R,
-                                       uint32_t watchdog, fi_record* __restrict__ rec_out,
-                                       fi_store* __restrict__ st_out, uint32_t st_cap, HookIn hook) {
+__device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const uint8_t* img,
+                                          uint32_t k, uint32_t cta, uint32_t wic, uint32_t* __restrict__ R,
+                                          uint32_t watchdog, fi_record* __restrict__ rec_out,
+                                          fi_store* __restrict__ st_out, uint32_t st_cap, HookIn hook,
+                                          uint32_t* __restrict__ ck, uint32_t ck_interval) {
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t lt_mask = (1u << lane) - 1u;
     const fi_instance in = P.inst[k];
     const fi_kernel kn = P.kern[in.kernel];
-    const fi_insn* __restrict__ code = P.code + kn.code_off;
+    const uint4* __restrict__ dec = P.dec + kn.code_off;
+    const uint32_t* __restrict__ ins = P.ins + kn.code_off;
     const uint32_t* __restrict__ cb = P.cbank + in.cbank_off;
-    const uint32_t zr = P.n_regs;
+    const uint32_t zr = P.n_regs, zidx = zr * 32;
+    const uint32_t ckw = (zr + 3) * 32;              // words per checkpoint
 
-    for (uint32_t r = 0; r <= zr; ++r) R[r * 32 + lane] = 0u;
     uint32_t nl = in.block - wic * 32;
     bool live = lane < (nl > 32 ? 32u : nl);
-    uint32_t pc = 0, preds = 0;
+    uint32_t pc = 0, preds = 0, step = 0;
+    if (MODE == EMU_INJ && ck != nullptr && ck_interval) {
+        // restart from the golden checkpoint at or before the site
+        const uint32_t c = hook.step / ck_interval;
+        const uint32_t* src = ck + (size_t)c * ckw;
+        for (uint32_t r = 0; r < zr; ++r) R[r * 32 + lane] = __ldg(&src[r * 32 + lane]);
+        R[zidx + lane] = 0u;
+        pc = __ldg(&src[zidx + lane]);
+        preds = __ldg(&src[zidx + 32 + lane]);
+        live = __ldg(&src[zidx + 64 + lane]) != 0u;
+        step = c * ck_interval;
+    } else {
+        for (uint32_t r = 0; r <= zr; ++r) R[r * 32 + lane] = 0u;
+    }
+    uint32_t livem = __ballot_sync(kFull, live);
+    bool conv = false;                                // recomputed at the first step
+    uint32_t upc = 0;
     EmuOut o;
-    uint32_t step = 0, nst = 0;
+    uint32_t nst = 0;
     uint4 recbuf = make_uint4(0, 0, 0, 0);
+    BufCache bc;
     __syncwarp();
 
-#define RROW(r) ((r) < zr ? (r) : zr)
-#define RD(r) R[RROW(r) * 32 + lane]
-#define WR(r, v) do { if ((r) < zr) R[(r) * 32 + lane] = (v); } while (0)
-#define RD64(r) ((uint64_t)RD(r) | ((uint64_t)RD((r) + 1) << 32))
+#define RDI(i) R[(i) + lane]
+#define WRI(i, v) do { if ((i) < zidx) R[(i) + lane] = (v); } while (0)
+#define RD64I(i) ((uint64_t)RDI(i) | ((uint64_t)RDI(min((i) + 32u, zidx)) << 32))
 
     for (;;) {
-        const uint32_t lm = __ballot_sync(kFull, live);
-        if (!lm) break;
-        const uint32_t pcm = __reduce_min_sync(kFull, live ? pc : 0xFFFFFFFFu);
+        if (!livem) break;
+        uint32_t pcm, active;
+        if (conv) {
+            pcm = upc;
+            active = livem;
+        } else {
+            pcm = __reduce_min_sync(kFull, live ? pc : 0xFFFFFFFFu);
+            active = __ballot_sync(kFull, live && pc == pcm);
+            if (active == livem) { conv = true; upc = pcm; }
+        }
+        if (MODE == EMU_TRACE && ck != nullptr && ck_interval && (step % ck_interval) == 0) {
+            uint32_t* dst = ck + (size_t)(step / ck_interval) * ckw;
+            for (uint32_t r = 0; r < zr; ++r) dst[r * 32 + lane] = R[r * 32 + lane];
+            dst[zidx + lane] = live ? (conv ? upc : pc) : 0u;
+            dst[zidx + 32 + lane] = preds;
+            dst[zidx + 64 + lane] = live ? 1u : 0u;
+        }
         if (step >= watchdog) { o.fault = 3; o.fault_pc = pcm; break; }
         if (pcm >= kn.code_len) { o.fault = 4; o.fault_pc = pcm; break; }
-        const bool act = live && pc == pcm;
-        const uint32_t active = __ballot_sync(kFull, act);
-        const uint4 raw = __ldg(reinterpret_cast<const uint4*>(code + pcm));
-        const uint32_t op = raw.x & 0xFF, guard = (raw.x >> 8) & 0xFF, d0 = (raw.x >> 16) & 0xFF, d1 = raw.x >> 24;
-        const uint32_t ra = raw.y & 0xFF, rb = (raw.y >> 8) & 0xFF, rc = (raw.y >> 16) & 0xFF, mod = raw.y >> 24;
-        const uint32_t imm = raw.z, ext = raw.w;
-        const uint32_t gsel = guard & 7;
-        const bool pv = (((gsel == 7) ? 1u : ((preds >> gsel) & 1u)) ^ ((guard >> 3) & 1u)) != 0;
-        const uint32_t pred = __ballot_sync(kFull, pv);
+        const uint4 D = __ldg(&dec[pcm]);
+        const uint32_t op = D.x & 0xFF, guard = (D.x >> 8) & 0xFF, mod = (D.x >> 16) & 0xFF, pb = D.x >> 24;
+        const uint32_t ia = D.y & 0xFFFF, ib = D.y >> 16, ic = D.z & 0xFFFF, id = D.z >> 16;
+        const uint32_t imm = D.w;
+        const bool act = (active >> lane) & 1u;
+        bool pv;
+        uint32_t pred;
+        if (guard == 7) {
+            pv = true;
+            pred = kFull;
+        } else {
+            const uint32_t gs = guard & 7;
+            pv = (((gs == 7) ? 1u : ((preds >> gs) & 1u)) ^ ((guard >> 3) & 1u)) != 0;
+            pred = __ballot_sync(kFull, pv);
+        }
         const bool ex = act && pv;
         const uint32_t exm = active & pred;
 
-        // ---- memory access validation (all executing lanes, before any effect)
-        uint64_t va = 0;
-        uint32_t bid = 0;
-        if (op == LDG || op == STG) {
-            const uint32_t w = 4u << ((mod & 3) > 2 ? 2 : (mod & 3));
-            va = RD64(ra) + (uint64_t)(int64_t)(int32_t)imm;
-            const uint32_t code_ = ex ? check_access(P, va, w, &bid) : 0u;
-            const uint32_t mis = __ballot_sync(kFull, code_ == 1), unm = __ballot_sync(kFull, code_ == 2);
-            if (mis | unm) { o.fault = mis ? 1 : 2; o.fault_pc = pcm; break; }
-        }
-
         if (MODE == EMU_TRACE) {
-            if ((step & 31) == lane)
-                recbuf = make_uint4(k, pcm | (op << 16) | (groupmask_of(op, d0, d1, mod) << 24), active, pred);
+            if ((step & 31) == lane) recbuf = make_uint4(k, __ldg(&ins[pcm]), active, pred);
             if ((step & 31) == 31) reinterpret_cast<uint4*>(rec_out)[step - 31 + lane] = recbuf;
         }
 
-        const uint32_t bv = (mod & 0x80) ? imm : RD(rb);
-        uint32_t next = pcm + 1;
-        switch (op) {
-            case NOP: break;
-            case EXIT: if (ex) live = false; break;
-            case BRA: if (ex) next = imm; break;
-            case MOV: if (ex) WR(d0, bv); break;
-            case S2R: {
-                uint32_t v = 0;
-                switch (imm) {
-                    case 0: v = wic * 32 + lane; break;
-                    case 1: v = cta; break;
-                    case 2: v = in.block; break;
-                    case 3: v = in.grid; break;
-                    case 4: v = lane; break;
-                    case 5: v = wic; break;
-                }
-                if (ex) WR(d0, v);
-                break;
-            }
-            case IADD3: {
-                const uint32_t a = RD(ra), c = RD(rc);
-                const uint32_t x = (mod & 1) ? 0u - a : a, y = (mod & 2) ? 0u - bv : bv;
-                const uint64_t s = (uint64_t)x + y + c;
-                if (ex) {
-                    WR(d0, (uint32_t)s);
-                    const uint32_t p = d1 & 7;
-                    if (p != 7) preds = (preds & ~(1u << p)) | ((uint32_t)((s >> 32) != 0) << p);
-                }
-                break;
-            }
-            case IMAD: if (ex) WR(d0, RD(ra) * bv + RD(rc)); break;
-            case IMAD_WIDE: {
-                const uint32_t a = RD(ra);
-                const uint64_t prod = (mod & 1) ? (uint64_t)a * (uint64_t)bv
-                                                : (uint64_t)((int64_t)(int32_t)a * (int64_t)(int32_t)bv);
-                const uint64_t r = prod + RD64(rc);
-                if (ex) { WR(d0, (uint32_t)r); WR(d0 + 1, (uint32_t)(r >> 32)); }
-                break;
-            }
-            case SHF: {
-                const uint32_t a = RD(ra), s = bv > 32 ? 32 : bv, m = mod & 3;
-                uint32_t v;
-                if (m == 0) v = s >= 32 ? 0u : a << s;
-                else if (m == 1) v = s >= 32 ? 0u : a >> s;
-                else v = (uint32_t)((int32_t)a >> (s >= 32 ? 31 : s));
-                if (ex) WR(d0, v);
-                break;
-            }
-            case LOP3: if (ex) WR(d0, dev_lop3(RD(ra), bv, RD(rc), ext & 0xFF)); break;
-            case SEL: {
-                const uint32_t p = rc & 7;
-                const bool s = (((p == 7) ? 1u : ((preds >> p) & 1u)) ^ ((rc >> 3) & 1u)) != 0;
-                if (ex) WR(d0, s ? RD(ra) : bv);
-                break;
-            }
-            case ISETP: case FSETP: case DSETP: {
-                bool v;
-                const uint32_t c = mod & 7;
-                if (op == ISETP) v = (mod & 8) ? dev_cmp_i<uint32_t>(RD(ra), bv, c) : dev_cmp_i<int32_t>((int32_t)RD(ra), (int32_t)bv, c);
-                else if (op == FSETP) v = dev_cmp_f((double)u2f(RD(ra)), (double)u2f(RD(rb)), c);
-                else v = dev_cmp_f(u2d(RD64(ra)), u2d(RD64(rb)), c);
-                const uint32_t p = d0 & 7;
-                if (ex && p != 7) preds = (preds & ~(1u << p)) | ((uint32_t)v << p);
-                break;
-            }
-            case FADD: case FMUL: case FFMA: {
-                const float x = u2f(RD(ra) ^ ((mod & 1) ? 0x80000000u : 0u));
-                const float y = u2f(bv ^ ((mod & 2) ? 0x80000000u : 0u));
-                const float z = u2f(RD(rc) ^ ((mod & 4) ? 0x80000000u : 0u));
-                const float r = op == FADD ? __fadd_rn(x, y) : op == FMUL ? __fmul_rn(x, y) : __fmaf_rn(x, y, z);
-                if (ex) WR(d0, fbits(r));
-                break;
-            }
-            case FMNMX: if (ex) WR(d0, dev_fmnmx(RD(ra), bv, mod & 1)); break;
-            case DADD: case DMUL: case DFMA: {
-                const double x = u2d(RD64(ra) ^ ((mod & 1) ? 0x8000000000000000ull : 0ull));
-                const double y = u2d(RD64(rb) ^ ((mod & 2) ? 0x8000000000000000ull : 0ull));
-                const double z = u2d(RD64(rc) ^ ((mod & 4) ? 0x8000000000000000ull : 0ull));
-                const double r = op == DADD ? __dadd_rn(x, y) : op == DMUL ? __dmul_rn(x, y) : __fma_rn(x, y, z);
-                const uint64_t b = dbits(r);
-                if (ex) { WR(d0, (uint32_t)b); WR(d0 + 1, (uint32_t)(b >> 32)); }
-                break;
-            }
-            case LDG: {
-                const uint32_t lw = (mod & 3) > 2 ? 2 : (mod & 3);
-                if (ex) {
-                    const fi_buffer B = P.buf[bid];
-                    const bool zero = B.writer >= 0 && (uint32_t)B.writer >= k;
-                    const uint8_t* src = img + (va - kVaBase);
-                    if (lw == 0) {
-                        WR(d0, zero ? 0u : __ldg(reinterpret_cast<const uint32_t*>(src)));
-                    } else if (lw == 1) {
-                        uint2 v = zero ? make_uint2(0, 0) : __ldg(reinterpret_cast<const uint2*>(src));
-                        WR(d0, v.x); WR(d0 + 1, v.y);
-                    } else {
-                        uint4 v = zero ? make_uint4(0, 0, 0, 0) : __ldg(reinterpret_cast<const uint4*>(src));
-                        WR(d0, v.x); WR(d0 + 1, v.y); WR(d0 + 2, v.z); WR(d0 + 3, v.w);
+        uint32_t taken = 0;                           // lanes that branch
+        bool fault_now = false;
+        if (op == FFMA) {
+            const float x = u2f(RDI(ia) ^ (mod << 31));
+            const float y = u2f(((mod & 0x80) ? imm : RDI(ib)) ^ ((mod & 2) << 30));
+            const float z = u2f(RDI(ic) ^ ((mod & 4) << 29));
+            const uint32_t r = fbits(__fmaf_rn(x, y, z));
+            if (ex) WRI(id, r);
+        } else {
+            const uint32_t bv = (mod & 0x80) ? imm : RDI(ib);
+            switch (op) {
+                case NOP: break;
+                case EXIT:
+                    if (ex) live = false;
+                    livem &= ~exm;
+                    break;
+                case BRA: taken = exm; break;
+                case MOV: if (ex) WRI(id, bv); break;
+                case S2R: {
+                    uint32_t v = 0;
+                    switch (imm) {
+                        case 0: v = wic * 32 + lane; break;
+                        case 1: v = cta; break;
+                        case 2: v = in.block; break;
+                        case 3: v = in.grid; break;
+                        case 4: v = lane; break;
+                        case 5: v = wic; break;
                     }
+                    if (ex) WRI(id, v);
+                    break;
                 }
-                break;
-            }
-            case LDC: {
-                const uint32_t w0 = imm >> 2;
-                if (ex) {
-                    WR(d0, w0 < in.cbank_len ? __ldg(&cb[w0]) : 0u);
-                    if (mod & 1) WR(d0 + 1, w0 + 1 < in.cbank_len ? __ldg(&cb[w0 + 1]) : 0u);
-                }
-                break;
-            }
-            case STG: {
-                const uint32_t lw = (mod & 3) > 2 ? 2 : (mod & 3), nw = 1u << lw;
-                uint32_t v[4];
-#pragma unroll
-                for (int i = 0; i < 4; ++i) v[i] = (uint32_t)i < nw ? RD(rb + i) : 0u;
-                const uint32_t idx = __popc(exm & lt_mask) * nw;
-                const uint32_t tot = __popc(exm) * nw;
-                if (MODE == EMU_LEN) {
+                case IADD3: {
+                    const uint32_t a = RDI(ia), c = RDI(ic);
+                    const uint32_t x = (mod & 1) ? 0u - a : a, y = (mod & 2) ? 0u - bv : bv;
+                    const uint64_t s = (uint64_t)x + y + c;
                     if (ex) {
-                        uint8_t* dst = img_w + (va - kVaBase);
-                        if (lw == 0) *reinterpret_cast<uint32_t*>(dst) = v[0];
-                        else if (lw == 1) *reinterpret_cast<uint2*>(dst) = make_uint2(v[0], v[1]);
-                        else *reinterpret_cast<uint4*>(dst) = make_uint4(v[0], v[1], v[2], v[3]);
+                        WRI(id, (uint32_t)s);
+                        if (pb != 7) preds = (preds & ~(1u << pb)) | ((uint32_t)((s >> 32) != 0) << pb);
                     }
-                } else if (MODE == EMU_TRACE || step > hook.step) {
-                    if (ex) {
-                        for (uint32_t i = 0; i < nw; ++i) {
-                            const uint32_t e = nst + idx + i;
-                            if (MODE == EMU_TRACE || e < st_cap) {
-                                fi_store s;
-                                s.va = va + 4 * i; s.value = v[i]; s.step = step;
-                                st_out[e] = s;
+                    break;
+                }
+                case IMAD: if (ex) WRI(id, RDI(ia) * bv + RDI(ic)); break;
+                case IMAD_WIDE: {
+                    const uint32_t a = RDI(ia);
+                    const uint64_t prod = (mod & 1) ? (uint64_t)a * (uint64_t)bv
+                                                    : (uint64_t)((int64_t)(int32_t)a * (int64_t)(int32_t)bv);
+                    const uint64_t r = prod + RD64I(ic);
+                    if (ex) { WRI(id, (uint32_t)r); WRI(id + 32, (uint32_t)(r >> 32)); }
+                    break;
+                }
+                case SHF: {
+                    const uint32_t a = RDI(ia), s = bv > 32 ? 32 : bv, m = mod & 3;
+                    uint32_t v;
+                    if (m == 0) v = s >= 32 ? 0u : a << s;
+                    else if (m == 1) v = s >= 32 ? 0u : a >> s;
+                    else v = (uint32_t)((int32_t)a >> (s >= 32 ? 31 : s));
+                    if (ex) WRI(id, v);
+                    break;
+                }
+                case LOP3: if (ex) WRI(id, dev_lop3(RDI(ia), bv, RDI(ic), pb)); break;
+                case SEL: {
+                    const uint32_t p = pb & 7;
+                    const bool s = (((p == 7) ? 1u : ((preds >> p) & 1u)) ^ ((pb >> 3) & 1u)) != 0;
+                    if (ex) WRI(id, s ? RDI(ia) : bv);
+                    break;
+                }
+                case ISETP: case FSETP: case DSETP: {
+                    bool v;
+                    const uint32_t c = mod & 7;
+                    if (op == ISETP) v = (mod & 8) ? dev_cmp_i<uint32_t>(RDI(ia), bv, c)
+                                                   : dev_cmp_i<int32_t>((int32_t)RDI(ia), (int32_t)bv, c);
+                    else if (op == FSETP) v = dev_cmp_f((double)u2f(RDI(ia)), (double)u2f(RDI(ib)), c);
+                    else v = dev_cmp_f(u2d(RD64I(ia)), u2d(RD64I(ib)), c);
+                    if (ex && pb != 7) preds = (preds & ~(1u << pb)) | ((uint32_t)v << pb);
+                    break;
+                }
+                case FADD: case FMUL: {
+                    const float x = u2f(RDI(ia) ^ (mod << 31));
+                    const float y = u2f(bv ^ ((mod & 2) << 30));
+                    const float r = op == FADD ? __fadd_rn(x, y) : __fmul_rn(x, y);
+                    if (ex) WRI(id, fbits(r));
+                    break;
+                }
+                case FMNMX: if (ex) WRI(id, dev_fmnmx(RDI(ia), bv, mod & 1)); break;
+                case DADD: case DMUL: case DFMA: {
+                    const double x = u2d(RD64I(ia) ^ ((uint64_t)(mod & 1) << 63));
+                    const double y = u2d(RD64I(ib) ^ ((uint64_t)(mod & 2) << 62));
+                    const double z = u2d(RD64I(ic) ^ ((uint64_t)(mod & 4) << 61));
+                    const double r = op == DADD ? __dadd_rn(x, y) : op == DMUL ? __dmul_rn(x, y) : __fma_rn(x, y, z);
+                    const uint64_t b = dbits(r);
+                    if (ex) { WRI(id, (uint32_t)b); WRI(id + 32, (uint32_t)(b >> 32)); }
+                    break;
+                }
+                case LDG: case STG: {
+                    const uint32_t lw = (mod & 3) > 2 ? 2 : (mod & 3), nw = 1u << lw, w = 4u << lw;
+                    const uint64_t va = RD64I(ia) + (uint64_t)(int64_t)(int32_t)imm;
+                    bool zero = false;
+                    const uint32_t code_ = ex ? check_access(P, bc, va, w, k, &zero) : 0u;
+                    const uint32_t bad = __ballot_sync(kFull, code_ != 0);
+                    if (bad) {
+                        o.fault = __ballot_sync(kFull, code_ == 1) ? 1 : 2;
+                        o.fault_pc = pcm;
+                        fault_now = true;
+                        break;
+                    }
+                    if (op == LDG) {
+                        if (ex) {
+                            const uint8_t* src = img + (va - kVaBase);
+                            if (lw == 0) {
+                                WRI(id, zero ? 0u : __ldg(reinterpret_cast<const uint32_t*>(src)));
+                            } else if (lw == 1) {
+                                const uint2 v = zero ? make_uint2(0, 0) : __ldg(reinterpret_cast<const uint2*>(src));
+                                WRI(id, v.x); WRI(id + 32, v.y);
+                            } else {
+                                const uint4 v = zero ? make_uint4(0, 0, 0, 0) : __ldg(reinterpret_cast<const uint4*>(src));
+                                WRI(id, v.x); WRI(id + 32, v.y); WRI(id + 64, v.z); WRI(id + 96, v.w);
                             }
                         }
+                    } else {
+                        uint32_t v[4];
+#pragma unroll
+                        for (int i = 0; i < 4; ++i) v[i] = (uint32_t)i < nw ? RDI(min(ib + 32u * i, zidx)) : 0u;
+                        const uint32_t idx = __popc(exm & lt_mask) * nw;
+                        const uint32_t tot = __popc(exm) * nw;
+                        if (MODE == EMU_LEN) {
+                            if (ex) {
+                                uint8_t* dst = img_w + (va - kVaBase);
+                                if (lw == 0) *reinterpret_cast<uint32_t*>(dst) = v[0];
+                                else if (lw == 1) *reinterpret_cast<uint2*>(dst) = make_uint2(v[0], v[1]);
+                                else *reinterpret_cast<uint4*>(dst) = make_uint4(v[0], v[1], v[2], v[3]);
+                            }
+                        } else if (MODE == EMU_TRACE || step > hook.step) {
+                            if (ex) {
+                                for (uint32_t i = 0; i < nw; ++i) {
+                                    const uint32_t e = nst + idx + i;
+                                    if (MODE == EMU_TRACE || e < st_cap) {
+                                        fi_store s;
+                                        s.va = va + 4 * i; s.value = v[i]; s.step = step;
+                                        st_out[e] = s;
+                                    }
+                                }
+                            }
+                        }
+                        if (MODE != EMU_INJ || step > hook.step) nst += tot;
                     }
+                    break;
                 }
-                if (MODE != EMU_INJ || step > hook.step) nst += tot;
-                break;
-            }
-            case I2F: if (ex) WR(d0, fbits((mod & 1) ? __uint2float_rn(RD(ra)) : __int2float_rn((int)RD(ra)))); break;
-            case F2I: if (ex) WR(d0, dev_f2i(RD(ra))); break;
-            case F2F_F64_F32: {
-                const uint64_t b = dbits((double)u2f(RD(ra)));
-                if (ex) { WR(d0, (uint32_t)b); WR(d0 + 1, (uint32_t)(b >> 32)); }
-                break;
-            }
-            case F2F_F32_F64: if (ex) WR(d0, fbits(__double2float_rn(u2d(RD64(ra))))); break;
-            case SHFL: {
-                int64_t src;
-                switch (mod & 3) {
-                    case 0: src = bv & 31; break;
-                    case 1: src = lane ^ (bv & 31); break;
-                    case 2: src = (int64_t)lane + (int64_t)bv; if (src > 31) src = lane; break;
-                    default: src = (int64_t)lane - (int64_t)bv; if (src < 0) src = lane; break;
+                case LDC: {
+                    const uint32_t w0 = imm >> 2;
+                    if (ex) {
+                        WRI(id, w0 < in.cbank_len ? __ldg(&cb[w0]) : 0u);
+                        if (mod & 1) WRI(id + 32, w0 + 1 < in.cbank_len ? __ldg(&cb[w0 + 1]) : 0u);
+                    }
+                    break;
                 }
-                __syncwarp();
-                const uint32_t v = R[RROW(ra) * 32 + (uint32_t)src];
-                __syncwarp();
-                if (ex) WR(d0, v);
-                break;
+                case I2F: if (ex) WRI(id, fbits((mod & 1) ? __uint2float_rn(RDI(ia)) : __int2float_rn((int)RDI(ia)))); break;
+                case F2I: if (ex) WRI(id, dev_f2i(RDI(ia))); break;
+                case F2F_F64_F32: {
+                    const uint64_t b = dbits((double)u2f(RDI(ia)));
+                    if (ex) { WRI(id, (uint32_t)b); WRI(id + 32, (uint32_t)(b >> 32)); }
+                    break;
+                }
+                case F2F_F32_F64: if (ex) WRI(id, fbits(__double2float_rn(u2d(RD64I(ia))))); break;
+                case SHFL: {
+                    int64_t src;
+                    switch (mod & 3) {
+                        case 0: src = bv & 31; break;
+                        case 1: src = lane ^ (bv & 31); break;
+                        case 2: src = (int64_t)lane + (int64_t)bv; if (src > 31) src = lane; break;
+                        default: src = (int64_t)lane - (int64_t)bv; if (src < 0) src = lane; break;
+                    }
+                    __syncwarp();
+                    const uint32_t v = R[ia + (uint32_t)src];
+                    __syncwarp();
+                    if (ex) WRI(id, v);
+                    break;
+                }
+                case IMNMX: {
+                    const uint32_t a = RDI(ia);
+                    uint32_t v;
+                    if (mod & 8) v = (mod & 1) ? max(a, bv) : min(a, bv);
+                    else v = (uint32_t)((mod & 1) ? max((int32_t)a, (int32_t)bv) : min((int32_t)a, (int32_t)bv));
+                    if (ex) WRI(id, v);
+                    break;
+                }
+                default: break;
             }
-            case IMNMX: {
-                const uint32_t a = RD(ra);
-                uint32_t v;
-                if (mod & 8) v = (mod & 1) ? max(a, bv) : min(a, bv);
-                else v = (uint32_t)((mod & 1) ? max((int32_t)a, (int32_t)bv) : min((int32_t)a, (int32_t)bv));
-                if (ex) WR(d0, v);
-                break;
-            }
-            default: break;
         }
-        if (act) pc = next;
+        if (fault_now) break;
+
+        // control flow: advance / branch, tracking convergence
+        if (conv) {
+            if (taken == 0) upc = pcm + 1;
+            else if (taken == active) upc = imm;
+            else {
+                conv = false;
+                pc = ((taken >> lane) & 1u) ? imm : pcm + 1;
+            }
+        } else if (act) {
+            pc = ((taken >> lane) & 1u) ? imm : pcm + 1;
+        }
 
         if (MODE == EMU_INJ && step == hook.step) {
             // transient fault: corrupt one destination of this dynamic
             // instruction in one lane, after the instruction wrote it (C-7, C-8)
             o.fired = true;
-            const bool lane_ok = (exm >> hook.lane) & 1u;
-            if (pcm != hook.pc || !lane_ok) o.bad = true;
+            if (pcm != hook.pc || !((exm >> hook.lane) & 1u)) o.bad = true;
             if (lane == hook.lane) {
                 if (hook.kind == 0) {
-                    const uint32_t before = RD(hook.reg);
+                    const uint32_t ri = min(hook.reg, zr) * 32;
+                    const uint32_t before = RDI(ri);
                     const uint32_t m = hook.bfm == FI_ZERO_VALUE ? before : hook.mask;
                     o.before = before; o.mask = m; o.after = before ^ m;
-                    WR(hook.reg, o.after);
+                    WRI(ri, o.after);
                 } else {
                     const uint32_t p = hook.reg & 7;
                     const uint32_t before = (p == 7) ? 1u : ((preds >> p) & 1u);
@@ -387,10 +508,9 @@ __device__ __noinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const ui
         }
         ++step;
     }
-#undef RROW
-#undef RD
-#undef WR
-#undef RD64
+#undef RDI
+#undef WRI
+#undef RD64I
     if (MODE == EMU_TRACE) {
         const uint32_t rem = step & 31;
         if (rem && lane < rem) reinterpret_cast<uint4*>(rec_out)[step - rem + lane] = recbuf;

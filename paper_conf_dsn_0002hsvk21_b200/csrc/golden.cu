@@ -1,4 +1,5 @@
-// golden.cu — the golden run that makes the trace resident in HBM (§8 row a1).
+// golden.cu — program preparation and the golden run that makes the trace
+// resident in HBM (§8 row a1).
 //
 // PAPER.md:72 step (1) profiles a fault-free run and step (4) compares with the
 // golden output state.  Here the golden run is the emulator in two passes:
@@ -6,12 +7,14 @@
 //          stores go straight into the image, which ends as the golden final
 //          image; per-warp step and stored-word counts come out.
 //   pass 2 (fi_golden_trace): every warp of every instance in ONE launch over the
-//          final image (DESIGN.md §3.5 writer rule), writing the App. A.3 records
-//          and the golden store log at the offsets scanned from pass 1.
+//          final image (DESIGN.md §3.5 writer rule), writing the App. A.3 records,
+//          the golden store log and register-file checkpoints at the offsets
+//          scanned from pass 1.
 #include <algorithm>
 #include <vector>
 
 #include "emu.cuh"
+#include "scan.cuh"
 
 namespace fi {
 namespace {
@@ -29,7 +32,8 @@ k_golden_len(EmuProg P, uint8_t* img, uint32_t k, uint64_t* warp_len, uint64_t* 
     if (lw >= in.warp_end - in.warp_begin) return;
     const uint32_t wpc = (in.block + 31) / 32;
     uint32_t* R = smem + wib * (P.n_regs + 1) * 32;
-    EmuOut o = emulate<EMU_LEN>(P, img, img, k, lw / wpc, lw % wpc, R, 0xFFFFFFFFu, nullptr, nullptr, 0, HookIn{});
+    EmuOut o = emulate<EMU_LEN>(P, img, img, k, lw / wpc, lw % wpc, R, 0xFFFFFFFFu, nullptr, nullptr, 0, HookIn{},
+                                nullptr, 0);
     if (lane == 0) {
         warp_len[in.warp_begin + lw] = o.steps;
         warp_nst[in.warp_begin + lw] = o.nstore;
@@ -39,7 +43,8 @@ k_golden_len(EmuProg P, uint8_t* img, uint32_t k, uint64_t* warp_len, uint64_t* 
 
 __global__ void __launch_bounds__(kWPB * 32)
 k_golden_trace(EmuProg P, const uint8_t* img, uint32_t n_warps, const uint64_t* warp_off, const uint64_t* gst_off,
-               fi_record* rec, fi_store* gst, uint32_t* status) {
+               fi_record* rec, fi_store* gst, uint32_t* ckpt, const uint64_t* ck_off, uint32_t ck_interval,
+               uint32_t* status) {
     extern __shared__ uint32_t smem[];
     const uint32_t wib = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t w = blockIdx.x * kWPB + wib;
@@ -49,8 +54,9 @@ k_golden_trace(EmuProg P, const uint8_t* img, uint32_t n_warps, const uint64_t* 
     const uint32_t wpc = (in.block + 31) / 32, lw = w - in.warp_begin;
     uint32_t* R = smem + wib * (P.n_regs + 1) * 32;
     const uint64_t r0 = warp_off[w], g0 = gst_off[w];
+    uint32_t* ck = ckpt ? ckpt + ck_off[w] * (ckpt_bytes(P.n_regs) / 4) : nullptr;
     EmuOut o = emulate<EMU_TRACE>(P, nullptr, img, k, lw / wpc, lw % wpc, R, 0xFFFFFFFFu, rec + r0, gst + g0,
-                                  0xFFFFFFFFu, HookIn{});
+                                  0xFFFFFFFFu, HookIn{}, ck, ckpt ? ck_interval : 0);
     if (lane == 0 && (o.fault || o.steps != warp_off[w + 1] - r0 || o.nstore != gst_off[w + 1] - g0))
         FI_DEV_ERR(status, FI_E_PROGRAM);
 }
@@ -62,6 +68,25 @@ __global__ void k_gran(const fi_buffer* buf, uint32_t n_buf, uint32_t* gran, uin
              g += (uint64_t)gridDim.x * blockDim.x)
             gran[g] = b;
     }
+}
+
+// decode every static instruction (register operands -> smem row offsets) and
+// precompute its trace insn word pc | op<<16 | groupmask<<24 (Table II, C-2)
+__global__ void k_decode(const fi_insn* code, uint32_t n_code, const fi_kernel* kern, uint32_t n_kern, uint32_t zr,
+                         uint4* dec, uint32_t* ins) {
+    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n_code) return;
+    const fi_insn I = code[i];
+    uint32_t pc = 0;
+    for (uint32_t k = 0; k < n_kern; ++k)
+        if (i >= kern[k].code_off && i < kern[k].code_off + kern[k].code_len) pc = i - kern[k].code_off;
+    dec[i] = decode_insn(I, zr);
+    ins[i] = pc | ((uint32_t)I.op << 16) | (groupmask_of(I.op, I.d0, I.d1, I.mod) << 24);
+}
+
+__global__ void k_ckpt_counts(const uint64_t* warp_len, uint32_t n, uint32_t interval, uint64_t* cnt) {
+    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < n) cnt[i] = (warp_len[i] + interval - 1) / interval;
 }
 
 }  // namespace
@@ -82,15 +107,31 @@ extern "C" uint32_t fi_program_regs(const fi_insn* code, uint32_t n) {
     return std::min<uint32_t>(kRZ, mx + 4);        // +3: widest multi-register operand (LDG/STG.128)
 }
 
-extern "C" fi_status fi_build_granule_map(const fi_program* p, uint32_t* gran, void* stream) {
-    if (!p || !gran) return FI_E_ARG;
+extern "C" size_t fi_program_aux_bytes(uint64_t image_bytes, uint32_t n_code) {
+    return aux_layout(image_bytes, n_code).total;
+}
+
+extern "C" fi_status fi_program_prepare(const fi_program* p, void* aux, void* stream) {
+    if (!p || !aux || p->n_regs == 0 || p->n_regs > kRZ) return FI_E_ARG;
     cudaStream_t s = (cudaStream_t)stream;
+    const AuxLayout L = aux_layout(p->image_bytes, p->n_code);
+    char* a = reinterpret_cast<char*>(aux);
+    uint32_t* gran = reinterpret_cast<uint32_t*>(a + L.gran);
     const uint64_t n_gran = (p->image_bytes + 255) >> 8;
-    fi_status e = cuda_status(cudaMemsetAsync(gran, 0xFF, n_gran * sizeof(uint32_t), s));
-    if (e || !p->n_buf) return e;
-    dim3 grid(64, std::min<uint32_t>(p->n_buf, 4096));
-    k_gran<<<grid, 256, 0, s>>>(p->buf, p->n_buf, gran, n_gran);
-    return launch_status();
+    fi_status e = cuda_status(cudaMemsetAsync(gran, 0xFF, std::max<uint64_t>(n_gran, 1) * sizeof(uint32_t), s));
+    if (e) return e;
+    if (p->n_buf) {
+        dim3 grid(64, std::min<uint32_t>(p->n_buf, 4096));
+        k_gran<<<grid, 256, 0, s>>>(p->buf, p->n_buf, gran, n_gran);
+        if ((e = launch_status())) return e;
+    }
+    if (p->n_code) {
+        k_decode<<<(p->n_code + 127) / 128, 128, 0, s>>>(p->code, p->n_code, p->kern, p->n_kern, p->n_regs,
+                                                         reinterpret_cast<uint4*>(a + L.dec),
+                                                         reinterpret_cast<uint32_t*>(a + L.ins));
+        if ((e = launch_status())) return e;
+    }
+    return FI_OK;
 }
 
 static fi_status set_smem(const void* f, size_t bytes) {
@@ -99,7 +140,7 @@ static fi_status set_smem(const void* f, size_t bytes) {
 
 extern "C" fi_status fi_golden_lengths(const fi_program* p, uint8_t* image, uint64_t* warp_len, uint64_t* warp_nstore,
                                        uint32_t* dev_status, void* stream) {
-    if (!p || !image || !warp_len || !warp_nstore || !dev_status || !p->inst_host || !p->gran) return FI_E_ARG;
+    if (!p || !image || !warp_len || !warp_nstore || !dev_status || !p->inst_host || !p->aux) return FI_E_ARG;
     if (p->n_regs == 0 || p->n_regs > kRZ) return FI_E_ARG;
     cudaStream_t s = (cudaStream_t)stream;
     const size_t smem = emu_smem(p->n_regs);
@@ -115,16 +156,37 @@ extern "C" fi_status fi_golden_lengths(const fi_program* p, uint8_t* image, uint
     return FI_OK;
 }
 
-extern "C" fi_status fi_golden_trace(const fi_program* p, const uint8_t* image, const uint64_t* warp_off,
-                                     const uint64_t* gstore_off, fi_record* rec, fi_store* gstore,
+extern "C" size_t fi_ckpt_bytes(uint32_t n_regs) { return ckpt_bytes(n_regs); }
+
+extern "C" size_t fi_ckpt_layout_workspace(uint32_t n_warps) {
+    return align256((size_t)n_warps * 8) + scan_rows_ws(n_warps, 1);
+}
+
+extern "C" fi_status fi_ckpt_layout(const uint64_t* warp_len, uint32_t n_warps, uint32_t interval, uint64_t* ckpt_off,
+                                    void* ws, size_t ws_bytes, void* stream) {
+    if (!warp_len || !ckpt_off || !ws || interval == 0 || ws_bytes < fi_ckpt_layout_workspace(n_warps)) return FI_E_ARG;
+    cudaStream_t s = (cudaStream_t)stream;
+    uint64_t* cnt = reinterpret_cast<uint64_t*>(ws);
+    const size_t head = align256((size_t)n_warps * 8);
+    if (n_warps) {
+        k_ckpt_counts<<<(n_warps + 255) / 256, 256, 0, s>>>(warp_len, n_warps, interval, cnt);
+        fi_status e = launch_status();
+        if (e) return e;
+    }
+    return scan_rows_u64x1(cnt, ckpt_off, n_warps, reinterpret_cast<char*>(ws) + head, ws_bytes - head, s);
+}
+
+extern "C" fi_status fi_golden_trace(const fi_program* p, const uint8_t* image, const fi_trace* t,
                                      uint32_t* dev_status, void* stream) {
-    if (!p || !image || !warp_off || !gstore_off || !rec || !dev_status || !p->gran) return FI_E_ARG;
+    if (!p || !image || !t || !t->warp_off || !t->gstore_off || !t->rec || !dev_status || !p->aux) return FI_E_ARG;
+    if (t->ckpt && (!t->ckpt_off || !t->ckpt_interval)) return FI_E_ARG;
     if (!p->n_warps) return FI_OK;
     cudaStream_t s = (cudaStream_t)stream;
     const size_t smem = emu_smem(p->n_regs);
     fi_status e = set_smem((const void*)k_golden_trace, smem);
     if (e) return e;
     k_golden_trace<<<(p->n_warps + kWPB - 1) / kWPB, kWPB * 32, smem, s>>>(
-        make_emu_prog(p), image, p->n_warps, warp_off, gstore_off, rec, gstore, dev_status);
+        make_emu_prog(p), image, p->n_warps, t->warp_off, t->gstore_off, t->rec, t->gstore, t->ckpt, t->ckpt_off,
+        t->ckpt_interval, dev_status);
     return launch_status();
 }

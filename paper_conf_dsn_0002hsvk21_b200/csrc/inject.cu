@@ -28,7 +28,8 @@ constexpr int kWPB = 4;
 
 __global__ void __launch_bounds__(kWPB * 32)
 k_inject(EmuProg P, const uint8_t* img, const uint64_t* __restrict__ warp_off, const fi_site* __restrict__ sites,
-         uint32_t n, fi_inj* __restrict__ out, fi_store* __restrict__ log, uint32_t cap, uint32_t* status) {
+         uint32_t n, fi_inj* __restrict__ out, fi_store* __restrict__ log, uint32_t cap, uint32_t* ckpt,
+         const uint64_t* __restrict__ ck_off, uint32_t ck_interval, uint32_t* status) {
     extern __shared__ uint32_t smem[];
     const uint32_t wib = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t i = blockIdx.x * kWPB + wib;
@@ -41,8 +42,9 @@ k_inject(EmuProg P, const uint8_t* img, const uint64_t* __restrict__ warp_off, c
     const uint32_t watchdog = wd > 0xFFFFFFFFull ? 0xFFFFFFFFu : (uint32_t)wd;
     uint32_t* R = smem + wib * (P.n_regs + 1) * 32;
     const HookIn h{S.step, S.lane, S.dst_kind, S.dst_reg, S.bfm, S.mask, S.pc};
+    uint32_t* ck = ckpt ? ckpt + ck_off[S.warp] * (ckpt_bytes(P.n_regs) / 4) : nullptr;
     const EmuOut o = emulate<EMU_INJ>(P, nullptr, img, S.instance, lw / wpc, lw % wpc, R, watchdog, nullptr,
-                                      log + (uint64_t)i * cap, cap, h);
+                                      log + (uint64_t)i * cap, cap, h, ck, ckpt ? ck_interval : 0);
     if (lane == 0) {
         fi_inj r;
         r.before = o.before; r.after = o.after; r.mask = o.mask; r.fault_pc = o.fault_pc;
@@ -163,22 +165,25 @@ using namespace fi;
 extern "C" fi_status fi_inject(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
                                uint32_t n, fi_inj* out, fi_store* log, uint32_t log_cap, uint32_t* dev_status,
                                void* stream) {
-    if (!p || !image || !t || !sites || !out || !dev_status || (log_cap && !log) || !p->gran) return FI_E_ARG;
+    if (!p || !image || !t || !sites || !out || !dev_status || (log_cap && !log) || !p->aux) return FI_E_ARG;
+    if (t->ckpt && (!t->ckpt_off || !t->ckpt_interval)) return FI_E_ARG;
     if (n == 0) return FI_OK;
     const size_t smem = golden_smem(p->n_regs);
     fi_status e = cuda_status(cudaFuncSetAttribute((const void*)k_inject, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     if (e) return e;
     k_inject<<<(n + kWPB - 1) / kWPB, kWPB * 32, smem, (cudaStream_t)stream>>>(
-        make_emu_prog(p), image, t->warp_off, sites, n, out, log, log_cap, dev_status);
+        make_emu_prog(p), image, t->warp_off, sites, n, out, log, log_cap, t->ckpt, t->ckpt_off, t->ckpt_interval,
+        dev_status);
     return launch_status();
 }
 
 extern "C" fi_status fi_classify(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
                                  uint32_t n, fi_inj* out, const fi_store* log, uint32_t log_cap, uint64_t* hist,
                                  uint32_t* dev_status, void* stream) {
-    if (!p || !image || !t || !sites || !out || !hist || !dev_status || !p->gran) return FI_E_ARG;
+    if (!p || !image || !t || !sites || !out || !hist || !dev_status || !p->aux) return FI_E_ARG;
     if (n == 0) return FI_OK;
-    ClsArgs A{p->buf, p->gran, image, t->gstore, t->gstore_off, sites, out, n, log, log_cap, hist, dev_status};
+    const EmuProg P = make_emu_prog(p);
+    ClsArgs A{p->buf, P.gran, image, t->gstore, t->gstore_off, sites, out, n, log, log_cap, hist, dev_status};
     k_classify<<<(n + kClsWarps - 1) / kClsWarps, kClsWarps * 32, 0, (cudaStream_t)stream>>>(A);
     return launch_status();
 }

@@ -53,7 +53,7 @@ class fi_program(C.Structure):
                 ("inst", C.c_void_p), ("n_inst", C.c_uint32),
                 ("cbank", C.c_void_p), ("n_cbank", C.c_uint32),
                 ("buf", C.c_void_p), ("n_buf", C.c_uint32),
-                ("gran", C.c_void_p),
+                ("aux", C.c_void_p),
                 ("image_bytes", C.c_uint64),
                 ("n_warps", C.c_uint32), ("n_regs", C.c_uint32),
                 ("code_host", C.c_void_p), ("inst_host", C.c_void_p)]
@@ -61,7 +61,9 @@ class fi_program(C.Structure):
 
 class fi_trace(C.Structure):
     _fields_ = [("rec", C.c_void_p), ("n_rec", C.c_uint64), ("warp_off", C.c_void_p),
-                ("gstore", C.c_void_p), ("gstore_off", C.c_void_p), ("n_warps", C.c_uint32)]
+                ("gstore", C.c_void_p), ("gstore_off", C.c_void_p),
+                ("ckpt", C.c_void_p), ("ckpt_off", C.c_void_p), ("ckpt_interval", C.c_uint32),
+                ("n_warps", C.c_uint32)]
 
 
 class fi_schedule(C.Structure):
@@ -85,11 +87,15 @@ def lib():
             "fi_last_cuda_error": (C.c_char_p, []),
             "fi_version": (C.c_char_p, []),
             "fi_program_regs": (u32, [vp, u32]),
-            "fi_build_granule_map": (st, [vp, vp, vp]),
+            "fi_program_aux_bytes": (sz, [u64, u32]),
+            "fi_program_prepare": (st, [vp, vp, vp]),
             "fi_golden_lengths": (st, [vp, vp, vp, vp, vp, vp]),
             "fi_scan_u64_workspace": (sz, [u64]),
             "fi_scan_u64": (st, [vp, vp, u64, vp, sz, vp]),
-            "fi_golden_trace": (st, [vp, vp, vp, vp, vp, vp, vp, vp]),
+            "fi_ckpt_bytes": (sz, [u32]),
+            "fi_ckpt_layout_workspace": (sz, [u32]),
+            "fi_ckpt_layout": (st, [vp, u32, u32, vp, vp, sz, vp]),
+            "fi_golden_trace": (st, [vp, vp, vp, vp, vp]),
             "fi_profile": (st, [vp, u64, u64, u32, vp, vp, vp]),
             "fi_site_index_bytes": (sz, [u32, u64]),
             "fi_build_site_index": (st, [vp, u32, vp, u64, vp, vp]),
@@ -170,16 +176,16 @@ class DeviceProgram:
         self.cbank = up("cbank", prog.cbank)
         self.buf = up("buffers", prog.buffers)
         self.init_image = up("init_image", prog.init_image)
-        self.n_gran = (prog.image_bytes + 255) // 256
-        self.gran = torch.empty(max(self.n_gran, 1), dtype=torch.int32, device=self.device)
+        self.aux = torch.empty(lib().fi_program_aux_bytes(prog.image_bytes, len(prog.code)), dtype=torch.uint8,
+                               device=self.device)
         self._code_host = np.ascontiguousarray(prog.code)
         self._inst_host = np.ascontiguousarray(prog.instances)
         self.n_regs = int(lib().fi_program_regs(self._code_host.ctypes.data, len(self._code_host)))
         self.c = fi_program(
             _p(self.code), len(prog.code), _p(self.kern), len(prog.kernels), _p(self.inst), len(prog.instances),
-            _p(self.cbank), len(prog.cbank), _p(self.buf), len(prog.buffers), _p(self.gran),
+            _p(self.cbank), len(prog.cbank), _p(self.buf), len(prog.buffers), _p(self.aux),
             prog.image_bytes, prog.n_warps, self.n_regs, self._code_host.ctypes.data, self._inst_host.ctypes.data)
-        _check(lib().fi_build_granule_map(C.byref(self.c), _p(self.gran), _stream()), "fi_build_granule_map")
+        _check(lib().fi_program_prepare(C.byref(self.c), _p(self.aux), _stream()), "fi_program_prepare")
 
     @property
     def n_inst(self):
@@ -202,6 +208,9 @@ class GoldenTrace:
     n_rec: int
     n_gstore: int
     c: fi_trace
+    ckpt: torch.Tensor | None = None
+    ckpt_off: torch.Tensor | None = None
+    ckpt_interval: int = 0
 
     @property
     def n_chunks(self):
@@ -217,8 +226,11 @@ def scan_u64(x: torch.Tensor) -> torch.Tensor:
     return out
 
 
-def golden_run(dp: DeviceProgram, keep_records: bool = True) -> GoldenTrace:
-    """fi_golden_lengths (pass 1) -> scans -> fi_golden_trace (pass 2)."""
+def golden_run(dp: DeviceProgram, ckpt_interval: int | str = "auto", ckpt_budget_frac: float = 0.2) -> GoldenTrace:
+    """fi_golden_lengths (pass 1) -> scans + checkpoint layout -> fi_golden_trace (pass 2).
+
+    ckpt_interval: steps between golden register-file checkpoints (0 = none);
+    "auto" = 4096, doubled until the checkpoints fit ckpt_budget_frac of free HBM."""
     st = DeviceStatus(dp.device)
     image = dp.init_image.clone()
     W = dp.n_warps
@@ -232,11 +244,26 @@ def golden_run(dp: DeviceProgram, keep_records: bool = True) -> GoldenTrace:
     n_gst = int(goff[W].item())
     rec = torch.empty(max(n_rec, 1) * 16, dtype=torch.uint8, device=dp.device)
     gst = torch.empty(max(n_gst, 1) * 16, dtype=torch.uint8, device=dp.device)
-    _check(lib().fi_golden_trace(C.byref(dp.c), _p(image), _p(woff), _p(goff), _p(rec), _p(gst), st.ptr, _stream()),
-           "fi_golden_trace")
+    ck = ckoff = None
+    interval = 0
+    ck_bytes = lib().fi_ckpt_bytes(dp.n_regs)
+    if ckpt_interval and W:
+        interval = 4096 if ckpt_interval == "auto" else int(ckpt_interval)
+        free = torch.cuda.mem_get_info(dp.device)[0]
+        ws_n = lib().fi_ckpt_layout_workspace(W)
+        ws = torch.empty(ws_n, dtype=torch.uint8, device=dp.device)
+        ckoff = torch.empty(W + 1, dtype=torch.int64, device=dp.device)
+        while True:
+            _check(lib().fi_ckpt_layout(_p(wl), W, interval, _p(ckoff), _p(ws), ws_n, _stream()), "fi_ckpt_layout")
+            total = int(ckoff[W].item()) * ck_bytes
+            if ckpt_interval != "auto" or total <= ckpt_budget_frac * free or interval >= 1 << 24:
+                break
+            interval *= 2
+        ck = torch.empty(max(total, 16), dtype=torch.uint8, device=dp.device)
+    tc = fi_trace(_p(rec), n_rec, _p(woff), _p(gst), _p(goff), _p(ck), _p(ckoff), interval, W)
+    _check(lib().fi_golden_trace(C.byref(dp.c), _p(image), C.byref(tc), st.ptr, _stream()), "fi_golden_trace")
     st.check("fi_golden_trace")
-    tc = fi_trace(_p(rec), n_rec, _p(woff), _p(gst), _p(goff), W)
-    return GoldenTrace(dp, image, wl[:W], woff, goff, rec, gst, n_rec, n_gst, tc)
+    return GoldenTrace(dp, image, wl[:W], woff, goff, rec, gst, n_rec, n_gst, tc, ck, ckoff, interval)
 
 
 def profile(gt: GoldenTrace, rec_begin: int = 0, rec_end: int | None = None,

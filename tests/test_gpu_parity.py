@@ -21,9 +21,9 @@ def F():
     return fi
 
 
-def _gpu_golden(F, prog):
+def _gpu_golden(F, prog, ckpt="auto"):
     dp = F.DeviceProgram(prog)
-    gt = F.golden_run(dp)
+    gt = F.golden_run(dp, ckpt_interval=ckpt)
     return dp, gt
 
 
@@ -64,9 +64,9 @@ def test_fuzz_trace_and_image(F, seed):
     assert np.array_equal(ic.cpu().numpy().astype(np.uint64), g.counts())
 
 
-def _campaign_parity(F, prog, seed, groups, bfms, n, mode):
+def _campaign_parity(F, prog, seed, groups, bfms, n, mode, ckpt="auto"):
     g = O.Golden(prog)
-    dp, gt = _gpu_golden(F, prog)
+    dp, gt = _gpu_golden(F, prog, ckpt)
     assert np.array_equal(_trace_np(F, gt), g.trace())
     assert np.array_equal(gt.image.cpu().numpy(), g.final_image())
     ic, cc = F.profile(gt)
@@ -107,8 +107,31 @@ def test_mini_c2_parity(F):
 @pytest.mark.parametrize("seed", range(8))
 def test_fuzz_campaign_parity(F, seed):
     prog = P.fuzz_program(100 + seed, n_ops=100)
+    # odd checkpoint intervals make replicas restart mid-divergence (seed % 3 == 0: no checkpoints)
     _campaign_parity(F, prog, 0xABC0 + seed, [F.G_GPPR, F.G_GP, F.G_PR, F.G_FP32, F.G_FP64, F.G_OTHERS][: 1 + seed % 6],
-                     [0, 1, 2, 3], 300, O.MODE_FULL)
+                     [0, 1, 2, 3], 300, O.MODE_FULL, ckpt=[0, 5, 13][seed % 3])
+
+
+def test_mini_c2_parity_checkpoints(F):
+    _campaign_parity(F, P.c2(full=False), 0x77, [F.G_GP, F.G_LD, F.G_PR], [0, 1, 2, 3], 300, O.MODE_WARP_LOCAL,
+                     ckpt=97)
+
+
+def test_checkpoints_do_not_change_results(F):
+    prog = P.c2(full=False)
+    res = []
+    for ck in (0, 64, 1000, "auto"):
+        dp, gt = _gpu_golden(F, prog, ck)
+        ic, cc = F.profile(gt)
+        idx = F.SiteIndex(gt, ic, cc)
+        sites = F.select_sites(idx, F.schedule(3, [F.G_GP], [0, 1, 2, 3]), 0, 500)
+        cap = F.log_capacity(gt)
+        out, log = F.inject(gt, sites, 500, cap)
+        F.classify(gt, sites, 500, out, log, cap)
+        res.append(F.as_numpy(out, F.INJ_DTYPE, 500))
+        assert np.array_equal(_trace_np(F, gt), _trace_np(F, _gpu_golden(F, prog, 0)[1]))
+    for r in res[1:]:
+        assert (r == res[0]).all()
 
 
 def test_multi_instance_profile_and_select(F):
