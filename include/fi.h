@@ -185,9 +185,14 @@ fi_status fi_select_sites(const fi_program* p, const fi_trace* t, const void* in
  * the site's instruction writes its destinations, lane `lane`'s destination
  * `dst_reg` is XOR-ed with the mask (ZERO_VALUE: mask = before; predicates C-7).
  * Stores after the site are logged to log[i*log_cap ...] (fi_store words).
- * Memory faults and the watchdog (C-9, C-10) end the replica. */
+ * Memory faults and the watchdog (C-9, C-10) end the replica.
+ * Scheduling only (results do not depend on it): persistent warps take
+ * replicas from a queue ordered longest-expected-first (counting sort of the
+ * steps left after the restart point); scratch: fi_inject_workspace(n) bytes. */
+size_t fi_inject_workspace(uint32_t n);
 fi_status fi_inject(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
-                    uint32_t n, fi_inj* out, fi_store* log, uint32_t log_cap, uint32_t* dev_status, void* stream);
+                    uint32_t n, fi_inj* out, fi_store* log, uint32_t log_cap, void* ws, size_t ws_bytes,
+                    uint32_t* dev_status, void* stream);
 
 /* K5 — classify (Table V [PAPER.md:184-196], [PAPER.md:206]; C-9, C-12, C-14):
  * DUE if a fault/watchdog ended the replica; else SDC if the final value of any

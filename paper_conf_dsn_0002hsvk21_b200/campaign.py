@@ -87,6 +87,7 @@ class Campaign:
         self.log = torch.empty(nloc * self.cap * 16, dtype=torch.uint8, device=self.device)
         self.hist = torch.zeros((8, 4, 3), dtype=torch.int64, device=self.device)
         self.status = fi.DeviceStatus(self.device)
+        self.inj_ws = torch.empty(fi.lib().fi_inject_workspace(nloc), dtype=torch.uint8, device=self.device)
 
     @property
     def n_local(self):
@@ -114,7 +115,7 @@ class Campaign:
         n = self.n_local
         fi.select_sites(idx, self.sched, self.j0, n, self.sites, self.status)
         mark("select")
-        fi.inject(self.gt, self.sites, n, self.cap, self.out, self.log, self.status)
+        fi.inject(self.gt, self.sites, n, self.cap, self.out, self.log, self.status, self.inj_ws)
         mark("inject")
         self.hist.zero_()
         fi.classify(self.gt, self.sites, n, self.out, self.log, self.cap, self.hist, self.status)

@@ -9,10 +9,13 @@
 //
 // Hot-loop design:
 //  * instructions are pre-decoded once per program (fi_program_prepare) into
-//    16 B with register operands already turned into shared-memory row offsets;
+//    16 B with register operands already turned into shared-memory byte offsets,
+//    plus a per-instruction "run length": how many straight-line instructions
+//    (no branch, exit or global memory access) start there;
 //  * while every live lane sits at the same pc (no divergence — the common case)
-//    the warp skips min-PC scheduling entirely (`conv`), falling back to
-//    REDUX.MIN + VOTE only while lanes are split;
+//    the warp executes whole straight-line runs without per-step scheduling,
+//    watchdog or control-flow bookkeeping, prefetching the next decoded
+//    instruction; only while lanes are split does it use REDUX.MIN + VOTE per step;
 //  * FFMA (the dominant opcode of GEMM-like kernels) has its own fast path;
 //  * each lane caches its last two buffers' bounds, so most LDG/STG skip the
 //    granule-table lookup;
@@ -37,27 +40,32 @@
 namespace fi {
 
 constexpr uint32_t kFull = 0xFFFFFFFFu;
+constexpr int kLdgBatch = 4;          // independent LDGs issued together
 enum EmuMode { EMU_LEN = 0, EMU_TRACE = 1, EMU_INJ = 2 };
 
 // ---- prepared program data (fi_program.aux) --------------------------------
-struct AuxLayout { size_t gran, dec, ins, total; };
+struct AuxLayout { size_t gran, dec, ins, run, total; };
 __host__ __device__ inline size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
 __host__ __device__ inline AuxLayout aux_layout(uint64_t image_bytes, uint32_t n_code) {
     AuxLayout L;
     L.gran = 0;
     L.dec = align256(((image_bytes + 255) >> 8) * sizeof(uint32_t));
     L.ins = L.dec + align256((size_t)n_code * 16);
-    L.total = L.ins + align256((size_t)n_code * 4);
+    L.run = L.ins + align256((size_t)n_code * 4);
+    L.total = L.run + align256((size_t)n_code * 4);
     return L;
 }
 
+// "plain" = may run inside a straight-line run: no control flow, no global memory
+__host__ __device__ inline bool is_plain(uint32_t op) { return op != BRA && op != EXIT && op != LDG && op != STG; }
+
 // decoded instruction (uint4):
 //   x = op | guard << 8 | mod << 16 | pb << 24     pb: IADD3 carry pred, *SETP dest pred, LOP3 lut, SEL pred
-//   y = ra_idx | rb_idx << 16                       smem word offsets (row*32), RZ / >= n_regs -> zero row
-//   z = rc_idx | d0_idx << 16                       d0_idx = 0xFFFF when the write is discarded
+//   y = ra | rb << 16                               smem byte offsets (row*128), RZ / >= n_regs -> zero row
+//   z = rc | rd << 16                               rd = 0xFFFF when the write is discarded
 //   w = imm
 __host__ __device__ inline uint4 decode_insn(const fi_insn& I, uint32_t zr) {
-    auto row = [&](uint32_t r) -> uint32_t { return (r < zr ? r : zr) * 32u; };
+    auto row = [&](uint32_t r) -> uint32_t { return (r < zr ? r : zr) * 128u; };
     uint32_t pb = 0;
     if (I.op == IADD3) pb = I.d1 & 7;
     else if (I.op == ISETP || I.op == FSETP || I.op == DSETP) pb = I.d0 & 7;
@@ -66,7 +74,7 @@ __host__ __device__ inline uint4 decode_insn(const fi_insn& I, uint32_t zr) {
     uint4 d;
     d.x = (uint32_t)I.op | ((uint32_t)I.guard << 8) | ((uint32_t)I.mod << 16) | (pb << 24);
     d.y = row(I.a) | (row(I.b) << 16);
-    d.z = row(I.c) | ((I.d0 < zr ? I.d0 * 32u : 0xFFFFu) << 16);
+    d.z = row(I.c) | ((I.d0 < zr ? I.d0 * 128u : 0xFFFFu) << 16);
     d.w = I.imm;
     return d;
 }
@@ -74,6 +82,7 @@ __host__ __device__ inline uint4 decode_insn(const fi_insn& I, uint32_t zr) {
 struct EmuProg {
     const uint4* dec;          // decoded code
     const uint32_t* ins;       // trace insn word per static instruction: pc | op<<16 | groupmask<<24
+    const uint32_t* run;       // straight-line run length starting at each static instruction
     const fi_kernel* kern;
     const fi_instance* inst;
     const uint32_t* cbank;
@@ -88,8 +97,8 @@ inline EmuProg make_emu_prog(const fi_program* p) {
     const AuxLayout L = aux_layout(p->image_bytes, p->n_code);
     const char* a = reinterpret_cast<const char*>(p->aux);
     return EmuProg{reinterpret_cast<const uint4*>(a + L.dec), reinterpret_cast<const uint32_t*>(a + L.ins),
-                   p->kern, p->inst, p->cbank, p->buf, reinterpret_cast<const uint32_t*>(a + L.gran),
-                   p->image_bytes, p->n_regs, p->n_inst};
+                   reinterpret_cast<const uint32_t*>(a + L.run), p->kern, p->inst, p->cbank, p->buf,
+                   reinterpret_cast<const uint32_t*>(a + L.gran), p->image_bytes, p->n_regs, p->n_inst};
 }
 
 // checkpoint = (n_regs + 3) rows of 32 words: registers, then pc, predicates, live
@@ -192,6 +201,165 @@ __device__ __forceinline__ uint32_t check_access(const EmuProg& P, BufCache& C, 
     return 0;
 }
 
+// Register-file access: Rb = this lane's column as a byte pointer, offsets are row*128.
+struct RegFile {
+    char* Rb;              // (char*)(R + lane)
+    uint32_t* R;           // row 0, lane 0
+    uint32_t zb;           // byte offset of the zero row
+    __device__ __forceinline__ uint32_t rd(uint32_t o) const { return *reinterpret_cast<const uint32_t*>(Rb + o); }
+    __device__ __forceinline__ uint64_t rd64(uint32_t o) const {
+        return (uint64_t)rd(o) | ((uint64_t)rd(min(o + 128u, zb)) << 32);
+    }
+    __device__ __forceinline__ void wr(uint32_t o, uint32_t v) const {
+        if (o < zb) *reinterpret_cast<uint32_t*>(Rb + o) = v;
+    }
+};
+
+struct LaneCtx {
+    uint32_t lane, cta, wic, block, grid, cbank_len;
+    const uint32_t* cb;
+};
+
+// One "plain" instruction (everything but BRA / EXIT / LDG / STG) in this lane.
+// All lanes call it together (SHFL needs the whole warp); `ex` = executes here.
+__device__ __forceinline__ void exec_plain(const RegFile& F, const LaneCtx& L, const uint4 D, const bool ex,
+                                           uint32_t& preds) {
+    const uint32_t op = D.x & 0xFF, mod = (D.x >> 16) & 0xFF, pb = D.x >> 24;
+    const uint32_t ia = D.y & 0xFFFF, ib = D.y >> 16, ic = D.z & 0xFFFF, id = D.z >> 16;
+    const uint32_t imm = D.w;
+    if (op == FFMA) {
+        const float x = u2f(F.rd(ia) ^ (mod << 31));
+        const float y = u2f(((mod & 0x80) ? imm : F.rd(ib)) ^ ((mod & 2) << 30));
+        const float z = u2f(F.rd(ic) ^ ((mod & 4) << 29));
+        const uint32_t r = fbits(__fmaf_rn(x, y, z));
+        if (ex) F.wr(id, r);
+        return;
+    }
+    const uint32_t bv = (mod & 0x80) ? imm : F.rd(ib);
+    switch (op) {
+        case MOV: if (ex) F.wr(id, bv); break;
+        case S2R: {
+            uint32_t v = 0;
+            switch (imm) {
+                case 0: v = L.wic * 32 + L.lane; break;
+                case 1: v = L.cta; break;
+                case 2: v = L.block; break;
+                case 3: v = L.grid; break;
+                case 4: v = L.lane; break;
+                case 5: v = L.wic; break;
+            }
+            if (ex) F.wr(id, v);
+            break;
+        }
+        case IADD3: {
+            const uint32_t a = F.rd(ia), c = F.rd(ic);
+            const uint32_t x = (mod & 1) ? 0u - a : a, y = (mod & 2) ? 0u - bv : bv;
+            const uint64_t s = (uint64_t)x + y + c;
+            if (ex) {
+                F.wr(id, (uint32_t)s);
+                if (pb != 7) preds = (preds & ~(1u << pb)) | ((uint32_t)((s >> 32) != 0) << pb);
+            }
+            break;
+        }
+        case IMAD: if (ex) F.wr(id, F.rd(ia) * bv + F.rd(ic)); break;
+        case IMAD_WIDE: {
+            const uint32_t a = F.rd(ia);
+            const uint64_t prod = (mod & 1) ? (uint64_t)a * (uint64_t)bv
+                                            : (uint64_t)((int64_t)(int32_t)a * (int64_t)(int32_t)bv);
+            const uint64_t r = prod + F.rd64(ic);
+            if (ex) { F.wr(id, (uint32_t)r); F.wr(id + 128, (uint32_t)(r >> 32)); }
+            break;
+        }
+        case SHF: {
+            const uint32_t a = F.rd(ia), s = bv > 32 ? 32 : bv, m = mod & 3;
+            uint32_t v;
+            if (m == 0) v = s >= 32 ? 0u : a << s;
+            else if (m == 1) v = s >= 32 ? 0u : a >> s;
+            else v = (uint32_t)((int32_t)a >> (s >= 32 ? 31 : s));
+            if (ex) F.wr(id, v);
+            break;
+        }
+        case LOP3: if (ex) F.wr(id, dev_lop3(F.rd(ia), bv, F.rd(ic), pb)); break;
+        case SEL: {
+            const uint32_t p = pb & 7;
+            const bool s = (((p == 7) ? 1u : ((preds >> p) & 1u)) ^ ((pb >> 3) & 1u)) != 0;
+            if (ex) F.wr(id, s ? F.rd(ia) : bv);
+            break;
+        }
+        case ISETP: case FSETP: case DSETP: {
+            bool v;
+            const uint32_t c = mod & 7;
+            if (op == ISETP) v = (mod & 8) ? dev_cmp_i<uint32_t>(F.rd(ia), bv, c)
+                                           : dev_cmp_i<int32_t>((int32_t)F.rd(ia), (int32_t)bv, c);
+            else if (op == FSETP) v = dev_cmp_f((double)u2f(F.rd(ia)), (double)u2f(F.rd(ib)), c);
+            else v = dev_cmp_f(u2d(F.rd64(ia)), u2d(F.rd64(ib)), c);
+            if (ex && pb != 7) preds = (preds & ~(1u << pb)) | ((uint32_t)v << pb);
+            break;
+        }
+        case FADD: case FMUL: {
+            const float x = u2f(F.rd(ia) ^ (mod << 31));
+            const float y = u2f(bv ^ ((mod & 2) << 30));
+            const float r = op == FADD ? __fadd_rn(x, y) : __fmul_rn(x, y);
+            if (ex) F.wr(id, fbits(r));
+            break;
+        }
+        case FMNMX: if (ex) F.wr(id, dev_fmnmx(F.rd(ia), bv, mod & 1)); break;
+        case DADD: case DMUL: case DFMA: {
+            const double x = u2d(F.rd64(ia) ^ ((uint64_t)(mod & 1) << 63));
+            const double y = u2d(F.rd64(ib) ^ ((uint64_t)(mod & 2) << 62));
+            const double z = u2d(F.rd64(ic) ^ ((uint64_t)(mod & 4) << 61));
+            const double r = op == DADD ? __dadd_rn(x, y) : op == DMUL ? __dmul_rn(x, y) : __fma_rn(x, y, z);
+            const uint64_t b = dbits(r);
+            if (ex) { F.wr(id, (uint32_t)b); F.wr(id + 128, (uint32_t)(b >> 32)); }
+            break;
+        }
+        case LDC: {
+            const uint32_t w0 = imm >> 2;
+            if (ex) {
+                F.wr(id, w0 < L.cbank_len ? __ldg(&L.cb[w0]) : 0u);
+                if (mod & 1) F.wr(id + 128, w0 + 1 < L.cbank_len ? __ldg(&L.cb[w0 + 1]) : 0u);
+            }
+            break;
+        }
+        case I2F: if (ex) F.wr(id, fbits((mod & 1) ? __uint2float_rn(F.rd(ia)) : __int2float_rn((int)F.rd(ia)))); break;
+        case F2I: if (ex) F.wr(id, dev_f2i(F.rd(ia))); break;
+        case F2F_F64_F32: {
+            const uint64_t b = dbits((double)u2f(F.rd(ia)));
+            if (ex) { F.wr(id, (uint32_t)b); F.wr(id + 128, (uint32_t)(b >> 32)); }
+            break;
+        }
+        case F2F_F32_F64: if (ex) F.wr(id, fbits(__double2float_rn(u2d(F.rd64(ia))))); break;
+        case SHFL: {
+            int64_t src;
+            switch (mod & 3) {
+                case 0: src = bv & 31; break;
+                case 1: src = L.lane ^ (bv & 31); break;
+                case 2: src = (int64_t)L.lane + (int64_t)bv; if (src > 31) src = L.lane; break;
+                default: src = (int64_t)L.lane - (int64_t)bv; if (src < 0) src = L.lane; break;
+            }
+            __syncwarp();
+            const uint32_t v = *reinterpret_cast<const uint32_t*>(reinterpret_cast<const char*>(F.R + src) + ia);
+            __syncwarp();
+            if (ex) F.wr(id, v);
+            break;
+        }
+        case IMNMX: {
+            const uint32_t a = F.rd(ia);
+            uint32_t v;
+            if (mod & 8) v = (mod & 1) ? max(a, bv) : min(a, bv);
+            else v = (uint32_t)((mod & 1) ? max((int32_t)a, (int32_t)bv) : min((int32_t)a, (int32_t)bv));
+            if (ex) F.wr(id, v);
+            break;
+        }
+        default: break;                               // NOP
+    }
+}
+
+__device__ __forceinline__ bool guard_of(uint32_t guard, uint32_t preds) {
+    const uint32_t gs = guard & 7;
+    return (((gs == 7) ? 1u : ((preds >> gs) & 1u)) ^ ((guard >> 3) & 1u)) != 0;
+}
+
 template <int MODE>
 __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const uint8_t* img,
                                           uint32_t k, uint32_t cta, uint32_t wic, uint32_t* __restrict__ R,
@@ -204,22 +372,25 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
     const fi_kernel kn = P.kern[in.kernel];
     const uint4* __restrict__ dec = P.dec + kn.code_off;
     const uint32_t* __restrict__ ins = P.ins + kn.code_off;
-    const uint32_t* __restrict__ cb = P.cbank + in.cbank_off;
-    const uint32_t zr = P.n_regs, zidx = zr * 32;
+    const uint32_t* __restrict__ runl = P.run + kn.code_off;
+    const uint32_t zr = P.n_regs;
     const uint32_t ckw = (zr + 3) * 32;              // words per checkpoint
+    const RegFile F{reinterpret_cast<char*>(R + lane), R, zr * 128};
+    const LaneCtx LC{lane, cta, wic, in.block, in.grid, in.cbank_len, P.cbank + in.cbank_off};
+    const bool use_ck = ck != nullptr && ck_interval != 0;
 
     uint32_t nl = in.block - wic * 32;
     bool live = lane < (nl > 32 ? 32u : nl);
     uint32_t pc = 0, preds = 0, step = 0;
-    if (MODE == EMU_INJ && ck != nullptr && ck_interval) {
+    if (MODE == EMU_INJ && use_ck) {
         // restart from the golden checkpoint at or before the site
         const uint32_t c = hook.step / ck_interval;
         const uint32_t* src = ck + (size_t)c * ckw;
         for (uint32_t r = 0; r < zr; ++r) R[r * 32 + lane] = __ldg(&src[r * 32 + lane]);
-        R[zidx + lane] = 0u;
-        pc = __ldg(&src[zidx + lane]);
-        preds = __ldg(&src[zidx + 32 + lane]);
-        live = __ldg(&src[zidx + 64 + lane]) != 0u;
+        R[zr * 32 + lane] = 0u;
+        pc = __ldg(&src[zr * 32 + lane]);
+        preds = __ldg(&src[zr * 32 + 32 + lane]);
+        live = __ldg(&src[zr * 32 + 64 + lane]) != 0u;
         step = c * ck_interval;
     } else {
         for (uint32_t r = 0; r <= zr; ++r) R[r * 32 + lane] = 0u;
@@ -233,10 +404,6 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
     BufCache bc;
     __syncwarp();
 
-#define RDI(i) R[(i) + lane]
-#define WRI(i, v) do { if ((i) < zidx) R[(i) + lane] = (v); } while (0)
-#define RD64I(i) ((uint64_t)RDI(i) | ((uint64_t)RDI(min((i) + 32u, zidx)) << 32))
-
     for (;;) {
         if (!livem) break;
         uint32_t pcm, active;
@@ -248,30 +415,120 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
             active = __ballot_sync(kFull, live && pc == pcm);
             if (active == livem) { conv = true; upc = pcm; }
         }
-        if (MODE == EMU_TRACE && ck != nullptr && ck_interval && (step % ck_interval) == 0) {
+        if (MODE == EMU_TRACE && use_ck && (step % ck_interval) == 0) {
             uint32_t* dst = ck + (size_t)(step / ck_interval) * ckw;
             for (uint32_t r = 0; r < zr; ++r) dst[r * 32 + lane] = R[r * 32 + lane];
-            dst[zidx + lane] = live ? (conv ? upc : pc) : 0u;
-            dst[zidx + 32 + lane] = preds;
-            dst[zidx + 64 + lane] = live ? 1u : 0u;
+            dst[zr * 32 + lane] = live ? (conv ? upc : pc) : 0u;
+            dst[zr * 32 + 32 + lane] = preds;
+            dst[zr * 32 + 64 + lane] = live ? 1u : 0u;
         }
         if (step >= watchdog) { o.fault = 3; o.fault_pc = pcm; break; }
         if (pcm >= kn.code_len) { o.fault = 4; o.fault_pc = pcm; break; }
+
+        if (conv) {
+            // ---- straight-line run: no scheduling / control bookkeeping per step
+            const uint32_t rw = __ldg(&runl[pcm]);
+            uint32_t run = rw & 0xFFFF, lr = rw >> 16;
+            uint32_t lim = watchdog - step;
+            if (MODE == EMU_TRACE && use_ck) lim = min(lim, ck_interval - step % ck_interval);
+            if (MODE == EMU_INJ && hook.step >= step) lim = min(lim, hook.step - step);
+            run = min(run, lim);
+            lr = min(min(lr, lim), (uint32_t)kLdgBatch);
+            if (lr >= 2) {
+                // ---- LDG batch: independent loads in flight together
+                uint4 vals[kLdgBatch];
+                uint32_t dsts[kLdgBatch], lws[kLdgBatch], preds_b[kLdgBatch];
+                bool exs[kLdgBatch];
+                int first_bad = -1;
+                uint32_t bad_kind = 0;
+#pragma unroll
+                for (int b = 0; b < kLdgBatch; ++b) {
+                    exs[b] = false;
+                    vals[b] = make_uint4(0, 0, 0, 0);
+                    if ((uint32_t)b < lr) {
+                        const uint4 D = __ldg(&dec[pcm + b]);
+                        const uint32_t guard = (D.x >> 8) & 0xFF, mod = (D.x >> 16) & 0xFF;
+                        const bool pv = guard == 7 ? true : guard_of(guard, preds);
+                        preds_b[b] = guard == 7 ? kFull : __ballot_sync(kFull, pv);
+                        const bool ex = live && pv;
+                        const uint32_t lw = (mod & 3) > 2 ? 2 : (mod & 3);
+                        const uint64_t va = F.rd64(D.y & 0xFFFF) + (uint64_t)(int64_t)(int32_t)D.w;
+                        bool zero = false;
+                        const uint32_t c = ex ? check_access(P, bc, va, 4u << lw, k, &zero) : 0u;
+                        const uint32_t bm = __ballot_sync(kFull, c != 0);
+                        if (bm && first_bad < 0) {
+                            first_bad = b;
+                            bad_kind = __ballot_sync(kFull, c == 1) ? 1 : 2;
+                        }
+                        const uint8_t* src = img + (va - kVaBase);
+                        if (ex && !c && !zero) {
+                            if (lw == 0) vals[b].x = __ldg(reinterpret_cast<const uint32_t*>(src));
+                            else if (lw == 1) { const uint2 t = __ldg(reinterpret_cast<const uint2*>(src)); vals[b].x = t.x; vals[b].y = t.y; }
+                            else vals[b] = __ldg(reinterpret_cast<const uint4*>(src));
+                        }
+                        exs[b] = ex;
+                        dsts[b] = D.z >> 16;
+                        lws[b] = lw;
+                    }
+                }
+                if (first_bad >= 0) {                 // the first faulting load in program order (C-9)
+                    o.fault = bad_kind;
+                    o.fault_pc = pcm + first_bad;
+                    step += first_bad;
+                    break;
+                }
+#pragma unroll
+                for (int b = 0; b < kLdgBatch; ++b) {
+                    if ((uint32_t)b < lr) {
+                        if (exs[b]) {
+                            F.wr(dsts[b], vals[b].x);
+                            if (lws[b] >= 1) F.wr(dsts[b] + 128, vals[b].y);
+                            if (lws[b] >= 2) { F.wr(dsts[b] + 256, vals[b].z); F.wr(dsts[b] + 384, vals[b].w); }
+                        }
+                        if (MODE == EMU_TRACE) {
+                            const uint32_t s = step + b;
+                            if ((s & 31) == lane) recbuf = make_uint4(k, __ldg(&ins[pcm + b]), livem, preds_b[b]);
+                            if ((s & 31) == 31) reinterpret_cast<uint4*>(rec_out)[s - 31 + lane] = recbuf;
+                        }
+                    }
+                }
+                step += lr;
+                upc = pcm + lr;
+                continue;
+            }
+            if (run) {
+                uint4 Dn = __ldg(&dec[pcm]);
+                for (uint32_t j = 0; j < run; ++j) {
+                    const uint4 D = Dn;
+                    if (j + 1 < run) Dn = __ldg(&dec[pcm + j + 1]);
+                    const uint32_t guard = (D.x >> 8) & 0xFF;
+                    bool pv = true;
+                    uint32_t pred = kFull;
+                    if (guard != 7) {
+                        pv = guard_of(guard, preds);
+                        pred = __ballot_sync(kFull, pv);
+                    }
+                    if (MODE == EMU_TRACE) {
+                        const uint32_t s = step + j;
+                        if ((s & 31) == lane) recbuf = make_uint4(k, __ldg(&ins[pcm + j]), livem, pred);
+                        if ((s & 31) == 31) reinterpret_cast<uint4*>(rec_out)[s - 31 + lane] = recbuf;
+                    }
+                    exec_plain(F, LC, D, live && pv, preds);
+                }
+                step += run;
+                upc = pcm + run;
+                continue;
+            }
+        }
+
+        // ---- one general step (branch, exit, memory, divergent lanes, the site)
         const uint4 D = __ldg(&dec[pcm]);
-        const uint32_t op = D.x & 0xFF, guard = (D.x >> 8) & 0xFF, mod = (D.x >> 16) & 0xFF, pb = D.x >> 24;
-        const uint32_t ia = D.y & 0xFFFF, ib = D.y >> 16, ic = D.z & 0xFFFF, id = D.z >> 16;
+        const uint32_t op = D.x & 0xFF, guard = (D.x >> 8) & 0xFF, mod = (D.x >> 16) & 0xFF;
+        const uint32_t ia = D.y & 0xFFFF, ib = D.y >> 16, id = D.z >> 16;
         const uint32_t imm = D.w;
         const bool act = (active >> lane) & 1u;
-        bool pv;
-        uint32_t pred;
-        if (guard == 7) {
-            pv = true;
-            pred = kFull;
-        } else {
-            const uint32_t gs = guard & 7;
-            pv = (((gs == 7) ? 1u : ((preds >> gs) & 1u)) ^ ((guard >> 3) & 1u)) != 0;
-            pred = __ballot_sync(kFull, pv);
-        }
+        const bool pv = guard == 7 ? true : guard_of(guard, preds);
+        const uint32_t pred = guard == 7 ? kFull : __ballot_sync(kFull, pv);
         const bool ex = act && pv;
         const uint32_t exm = active & pred;
 
@@ -281,194 +538,65 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
         }
 
         uint32_t taken = 0;                           // lanes that branch
-        bool fault_now = false;
-        if (op == FFMA) {
-            const float x = u2f(RDI(ia) ^ (mod << 31));
-            const float y = u2f(((mod & 0x80) ? imm : RDI(ib)) ^ ((mod & 2) << 30));
-            const float z = u2f(RDI(ic) ^ ((mod & 4) << 29));
-            const uint32_t r = fbits(__fmaf_rn(x, y, z));
-            if (ex) WRI(id, r);
-        } else {
-            const uint32_t bv = (mod & 0x80) ? imm : RDI(ib);
-            switch (op) {
-                case NOP: break;
-                case EXIT:
-                    if (ex) live = false;
-                    livem &= ~exm;
-                    break;
-                case BRA: taken = exm; break;
-                case MOV: if (ex) WRI(id, bv); break;
-                case S2R: {
-                    uint32_t v = 0;
-                    switch (imm) {
-                        case 0: v = wic * 32 + lane; break;
-                        case 1: v = cta; break;
-                        case 2: v = in.block; break;
-                        case 3: v = in.grid; break;
-                        case 4: v = lane; break;
-                        case 5: v = wic; break;
-                    }
-                    if (ex) WRI(id, v);
-                    break;
-                }
-                case IADD3: {
-                    const uint32_t a = RDI(ia), c = RDI(ic);
-                    const uint32_t x = (mod & 1) ? 0u - a : a, y = (mod & 2) ? 0u - bv : bv;
-                    const uint64_t s = (uint64_t)x + y + c;
-                    if (ex) {
-                        WRI(id, (uint32_t)s);
-                        if (pb != 7) preds = (preds & ~(1u << pb)) | ((uint32_t)((s >> 32) != 0) << pb);
-                    }
-                    break;
-                }
-                case IMAD: if (ex) WRI(id, RDI(ia) * bv + RDI(ic)); break;
-                case IMAD_WIDE: {
-                    const uint32_t a = RDI(ia);
-                    const uint64_t prod = (mod & 1) ? (uint64_t)a * (uint64_t)bv
-                                                    : (uint64_t)((int64_t)(int32_t)a * (int64_t)(int32_t)bv);
-                    const uint64_t r = prod + RD64I(ic);
-                    if (ex) { WRI(id, (uint32_t)r); WRI(id + 32, (uint32_t)(r >> 32)); }
-                    break;
-                }
-                case SHF: {
-                    const uint32_t a = RDI(ia), s = bv > 32 ? 32 : bv, m = mod & 3;
-                    uint32_t v;
-                    if (m == 0) v = s >= 32 ? 0u : a << s;
-                    else if (m == 1) v = s >= 32 ? 0u : a >> s;
-                    else v = (uint32_t)((int32_t)a >> (s >= 32 ? 31 : s));
-                    if (ex) WRI(id, v);
-                    break;
-                }
-                case LOP3: if (ex) WRI(id, dev_lop3(RDI(ia), bv, RDI(ic), pb)); break;
-                case SEL: {
-                    const uint32_t p = pb & 7;
-                    const bool s = (((p == 7) ? 1u : ((preds >> p) & 1u)) ^ ((pb >> 3) & 1u)) != 0;
-                    if (ex) WRI(id, s ? RDI(ia) : bv);
-                    break;
-                }
-                case ISETP: case FSETP: case DSETP: {
-                    bool v;
-                    const uint32_t c = mod & 7;
-                    if (op == ISETP) v = (mod & 8) ? dev_cmp_i<uint32_t>(RDI(ia), bv, c)
-                                                   : dev_cmp_i<int32_t>((int32_t)RDI(ia), (int32_t)bv, c);
-                    else if (op == FSETP) v = dev_cmp_f((double)u2f(RDI(ia)), (double)u2f(RDI(ib)), c);
-                    else v = dev_cmp_f(u2d(RD64I(ia)), u2d(RD64I(ib)), c);
-                    if (ex && pb != 7) preds = (preds & ~(1u << pb)) | ((uint32_t)v << pb);
-                    break;
-                }
-                case FADD: case FMUL: {
-                    const float x = u2f(RDI(ia) ^ (mod << 31));
-                    const float y = u2f(bv ^ ((mod & 2) << 30));
-                    const float r = op == FADD ? __fadd_rn(x, y) : __fmul_rn(x, y);
-                    if (ex) WRI(id, fbits(r));
-                    break;
-                }
-                case FMNMX: if (ex) WRI(id, dev_fmnmx(RDI(ia), bv, mod & 1)); break;
-                case DADD: case DMUL: case DFMA: {
-                    const double x = u2d(RD64I(ia) ^ ((uint64_t)(mod & 1) << 63));
-                    const double y = u2d(RD64I(ib) ^ ((uint64_t)(mod & 2) << 62));
-                    const double z = u2d(RD64I(ic) ^ ((uint64_t)(mod & 4) << 61));
-                    const double r = op == DADD ? __dadd_rn(x, y) : op == DMUL ? __dmul_rn(x, y) : __fma_rn(x, y, z);
-                    const uint64_t b = dbits(r);
-                    if (ex) { WRI(id, (uint32_t)b); WRI(id + 32, (uint32_t)(b >> 32)); }
-                    break;
-                }
-                case LDG: case STG: {
-                    const uint32_t lw = (mod & 3) > 2 ? 2 : (mod & 3), nw = 1u << lw, w = 4u << lw;
-                    const uint64_t va = RD64I(ia) + (uint64_t)(int64_t)(int32_t)imm;
-                    bool zero = false;
-                    const uint32_t code_ = ex ? check_access(P, bc, va, w, k, &zero) : 0u;
-                    const uint32_t bad = __ballot_sync(kFull, code_ != 0);
-                    if (bad) {
-                        o.fault = __ballot_sync(kFull, code_ == 1) ? 1 : 2;
-                        o.fault_pc = pcm;
-                        fault_now = true;
-                        break;
-                    }
-                    if (op == LDG) {
-                        if (ex) {
-                            const uint8_t* src = img + (va - kVaBase);
-                            if (lw == 0) {
-                                WRI(id, zero ? 0u : __ldg(reinterpret_cast<const uint32_t*>(src)));
-                            } else if (lw == 1) {
-                                const uint2 v = zero ? make_uint2(0, 0) : __ldg(reinterpret_cast<const uint2*>(src));
-                                WRI(id, v.x); WRI(id + 32, v.y);
-                            } else {
-                                const uint4 v = zero ? make_uint4(0, 0, 0, 0) : __ldg(reinterpret_cast<const uint4*>(src));
-                                WRI(id, v.x); WRI(id + 32, v.y); WRI(id + 64, v.z); WRI(id + 96, v.w);
-                            }
-                        }
-                    } else {
-                        uint32_t v[4];
-#pragma unroll
-                        for (int i = 0; i < 4; ++i) v[i] = (uint32_t)i < nw ? RDI(min(ib + 32u * i, zidx)) : 0u;
-                        const uint32_t idx = __popc(exm & lt_mask) * nw;
-                        const uint32_t tot = __popc(exm) * nw;
-                        if (MODE == EMU_LEN) {
-                            if (ex) {
-                                uint8_t* dst = img_w + (va - kVaBase);
-                                if (lw == 0) *reinterpret_cast<uint32_t*>(dst) = v[0];
-                                else if (lw == 1) *reinterpret_cast<uint2*>(dst) = make_uint2(v[0], v[1]);
-                                else *reinterpret_cast<uint4*>(dst) = make_uint4(v[0], v[1], v[2], v[3]);
-                            }
-                        } else if (MODE == EMU_TRACE || step > hook.step) {
-                            if (ex) {
-                                for (uint32_t i = 0; i < nw; ++i) {
-                                    const uint32_t e = nst + idx + i;
-                                    if (MODE == EMU_TRACE || e < st_cap) {
-                                        fi_store s;
-                                        s.va = va + 4 * i; s.value = v[i]; s.step = step;
-                                        st_out[e] = s;
-                                    }
-                                }
-                            }
-                        }
-                        if (MODE != EMU_INJ || step > hook.step) nst += tot;
-                    }
-                    break;
-                }
-                case LDC: {
-                    const uint32_t w0 = imm >> 2;
-                    if (ex) {
-                        WRI(id, w0 < in.cbank_len ? __ldg(&cb[w0]) : 0u);
-                        if (mod & 1) WRI(id + 32, w0 + 1 < in.cbank_len ? __ldg(&cb[w0 + 1]) : 0u);
-                    }
-                    break;
-                }
-                case I2F: if (ex) WRI(id, fbits((mod & 1) ? __uint2float_rn(RDI(ia)) : __int2float_rn((int)RDI(ia)))); break;
-                case F2I: if (ex) WRI(id, dev_f2i(RDI(ia))); break;
-                case F2F_F64_F32: {
-                    const uint64_t b = dbits((double)u2f(RDI(ia)));
-                    if (ex) { WRI(id, (uint32_t)b); WRI(id + 32, (uint32_t)(b >> 32)); }
-                    break;
-                }
-                case F2F_F32_F64: if (ex) WRI(id, fbits(__double2float_rn(u2d(RD64I(ia))))); break;
-                case SHFL: {
-                    int64_t src;
-                    switch (mod & 3) {
-                        case 0: src = bv & 31; break;
-                        case 1: src = lane ^ (bv & 31); break;
-                        case 2: src = (int64_t)lane + (int64_t)bv; if (src > 31) src = lane; break;
-                        default: src = (int64_t)lane - (int64_t)bv; if (src < 0) src = lane; break;
-                    }
-                    __syncwarp();
-                    const uint32_t v = R[ia + (uint32_t)src];
-                    __syncwarp();
-                    if (ex) WRI(id, v);
-                    break;
-                }
-                case IMNMX: {
-                    const uint32_t a = RDI(ia);
-                    uint32_t v;
-                    if (mod & 8) v = (mod & 1) ? max(a, bv) : min(a, bv);
-                    else v = (uint32_t)((mod & 1) ? max((int32_t)a, (int32_t)bv) : min((int32_t)a, (int32_t)bv));
-                    if (ex) WRI(id, v);
-                    break;
-                }
-                default: break;
+        if (op == EXIT) {
+            if (ex) live = false;
+            livem &= ~exm;
+        } else if (op == BRA) {
+            taken = exm;
+        } else if (op == LDG || op == STG) {
+            const uint32_t lw = (mod & 3) > 2 ? 2 : (mod & 3), nw = 1u << lw, w = 4u << lw;
+            const uint64_t va = F.rd64(ia) + (uint64_t)(int64_t)(int32_t)imm;
+            bool zero = false;
+            const uint32_t code_ = ex ? check_access(P, bc, va, w, k, &zero) : 0u;
+            const uint32_t bad = __ballot_sync(kFull, code_ != 0);
+            if (bad) {                                // memory fault: DUE (C-9); the step has no effect
+                o.fault = __ballot_sync(kFull, code_ == 1) ? 1 : 2;
+                o.fault_pc = pcm;
+                break;
             }
+            if (op == LDG) {
+                if (ex) {
+                    const uint8_t* src = img + (va - kVaBase);
+                    if (lw == 0) {
+                        F.wr(id, zero ? 0u : __ldg(reinterpret_cast<const uint32_t*>(src)));
+                    } else if (lw == 1) {
+                        const uint2 v = zero ? make_uint2(0, 0) : __ldg(reinterpret_cast<const uint2*>(src));
+                        F.wr(id, v.x); F.wr(id + 128, v.y);
+                    } else {
+                        const uint4 v = zero ? make_uint4(0, 0, 0, 0) : __ldg(reinterpret_cast<const uint4*>(src));
+                        F.wr(id, v.x); F.wr(id + 128, v.y); F.wr(id + 256, v.z); F.wr(id + 384, v.w);
+                    }
+                }
+            } else {
+                uint32_t v[4];
+#pragma unroll
+                for (int i = 0; i < 4; ++i) v[i] = (uint32_t)i < nw ? F.rd(min(ib + 128u * i, F.zb)) : 0u;
+                const uint32_t idx = __popc(exm & lt_mask) * nw;
+                const uint32_t tot = __popc(exm) * nw;
+                if (MODE == EMU_LEN) {
+                    if (ex) {
+                        uint8_t* dst = img_w + (va - kVaBase);
+                        if (lw == 0) *reinterpret_cast<uint32_t*>(dst) = v[0];
+                        else if (lw == 1) *reinterpret_cast<uint2*>(dst) = make_uint2(v[0], v[1]);
+                        else *reinterpret_cast<uint4*>(dst) = make_uint4(v[0], v[1], v[2], v[3]);
+                    }
+                } else if (MODE == EMU_TRACE || step > hook.step) {
+                    if (ex) {
+                        for (uint32_t i = 0; i < nw; ++i) {
+                            const uint32_t e = nst + idx + i;
+                            if (MODE == EMU_TRACE || e < st_cap) {
+                                fi_store s;
+                                s.va = va + 4 * i; s.value = v[i]; s.step = step;
+                                st_out[e] = s;
+                            }
+                        }
+                    }
+                }
+                if (MODE != EMU_INJ || step > hook.step) nst += tot;
+            }
+        } else {
+            exec_plain(F, LC, D, ex, preds);
         }
-        if (fault_now) break;
 
         // control flow: advance / branch, tracking convergence
         if (conv) {
@@ -489,11 +617,11 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
             if (pcm != hook.pc || !((exm >> hook.lane) & 1u)) o.bad = true;
             if (lane == hook.lane) {
                 if (hook.kind == 0) {
-                    const uint32_t ri = min(hook.reg, zr) * 32;
-                    const uint32_t before = RDI(ri);
+                    const uint32_t ri = min(hook.reg, zr) * 128;
+                    const uint32_t before = F.rd(ri);
                     const uint32_t m = hook.bfm == FI_ZERO_VALUE ? before : hook.mask;
                     o.before = before; o.mask = m; o.after = before ^ m;
-                    WRI(ri, o.after);
+                    F.wr(ri, o.after);
                 } else {
                     const uint32_t p = hook.reg & 7;
                     const uint32_t before = (p == 7) ? 1u : ((preds >> p) & 1u);
@@ -508,9 +636,6 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
         }
         ++step;
     }
-#undef RDI
-#undef WRI
-#undef RD64I
     if (MODE == EMU_TRACE) {
         const uint32_t rem = step & 31;
         if (rem && lane < rem) reinterpret_cast<uint4*>(rec_out)[step - rem + lane] = recbuf;

@@ -73,15 +73,36 @@ __global__ void k_gran(const fi_buffer* buf, uint32_t n_buf, uint32_t* gran, uin
 // decode every static instruction (register operands -> smem row offsets) and
 // precompute its trace insn word pc | op<<16 | groupmask<<24 (Table II, C-2)
 __global__ void k_decode(const fi_insn* code, uint32_t n_code, const fi_kernel* kern, uint32_t n_kern, uint32_t zr,
-                         uint4* dec, uint32_t* ins) {
+                         uint4* dec, uint32_t* ins, uint32_t* run) {
     const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= n_code) return;
     const fi_insn I = code[i];
-    uint32_t pc = 0;
+    uint32_t pc = 0, end = i + 1;
     for (uint32_t k = 0; k < n_kern; ++k)
-        if (i >= kern[k].code_off && i < kern[k].code_off + kern[k].code_len) pc = i - kern[k].code_off;
+        if (i >= kern[k].code_off && i < kern[k].code_off + kern[k].code_len) {
+            pc = i - kern[k].code_off;
+            end = kern[k].code_off + kern[k].code_len;
+        }
     dec[i] = decode_insn(I, zr);
     ins[i] = pc | ((uint32_t)I.op << 16) | (groupmask_of(I.op, I.d0, I.d1, I.mod) << 24);
+    uint32_t r = 0;                                   // straight-line run starting here
+    for (uint32_t j = i; j < end && is_plain(code[j].op); ++j) ++r;
+    // LDG batch: consecutive LDGs none of whose address pair is written by an
+    // earlier LDG of the batch (their loads can be in flight together)
+    uint32_t lr = 0;
+    for (uint32_t j = i; j < end && code[j].op == LDG && lr < 0xFFFF; ++j) {
+        bool hazard = false;
+        for (uint32_t q = i; q < j && !hazard; ++q) {
+            const Dests d = dests_of(code[q].op, code[q].d0, code[q].d1, code[q].mod);
+            for (uint32_t x = 0; x < 2; ++x) {
+                const uint32_t a = code[j].a + x;
+                if (code[j].a != kRZ && a >= d.gp_base && a < d.gp_base + d.n_gp) hazard = true;
+            }
+        }
+        if (hazard) break;
+        ++lr;
+    }
+    run[i] = (r > 0xFFFF ? 0xFFFFu : r) | (lr << 16);
 }
 
 __global__ void k_ckpt_counts(const uint64_t* warp_len, uint32_t n, uint32_t interval, uint64_t* cnt) {
@@ -128,7 +149,8 @@ extern "C" fi_status fi_program_prepare(const fi_program* p, void* aux, void* st
     if (p->n_code) {
         k_decode<<<(p->n_code + 127) / 128, 128, 0, s>>>(p->code, p->n_code, p->kern, p->n_kern, p->n_regs,
                                                          reinterpret_cast<uint4*>(a + L.dec),
-                                                         reinterpret_cast<uint32_t*>(a + L.ins));
+                                                         reinterpret_cast<uint32_t*>(a + L.ins),
+                                                         reinterpret_cast<uint32_t*>(a + L.run));
         if ((e = launch_status())) return e;
     }
     return FI_OK;

@@ -26,14 +26,58 @@ namespace {
 
 constexpr int kWPB = 4;
 
+constexpr int kBuckets = 1024;
+
+// Longest-expected-first replica order (LPT scheduling): counting sort, one CTA,
+// of the steps each replica must emulate after its restart point.
+__global__ void __launch_bounds__(1024)
+k_lpt_order(const fi_site* __restrict__ sites, const uint64_t* __restrict__ warp_off, uint32_t ck_interval,
+            uint32_t n, uint32_t* __restrict__ order, uint32_t* __restrict__ counter) {
+    __shared__ uint32_t hist[kBuckets];
+    __shared__ uint32_t s_max;
+    auto cost = [&](uint32_t i) -> uint64_t {
+        const fi_site S = sites[i];
+        const uint64_t L = warp_off[S.warp + 1] - warp_off[S.warp];
+        const uint64_t start = ck_interval ? (uint64_t)(S.step / ck_interval) * ck_interval : 0;
+        return L > start ? L - start : 0;
+    };
+    for (uint32_t b = threadIdx.x; b < kBuckets; b += blockDim.x) hist[b] = 0;
+    if (threadIdx.x == 0) { s_max = 0; *counter = 0; }
+    __syncthreads();
+    uint32_t mx = 0;
+    for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) mx = max(mx, (uint32_t)min(cost(i), (uint64_t)0xFFFFFFFFu));
+    atomicMax(&s_max, mx);
+    __syncthreads();
+    const uint32_t shift = max(0, 32 - __clz(s_max) - 10);
+    for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) {
+        const uint32_t b = kBuckets - 1 - min((uint32_t)(min(cost(i), (uint64_t)0xFFFFFFFFu) >> shift), (uint32_t)kBuckets - 1);
+        atomicAdd(&hist[b], 1u);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        uint32_t run = 0;
+        for (int b = 0; b < kBuckets; ++b) { const uint32_t c = hist[b]; hist[b] = run; run += c; }
+    }
+    __syncthreads();
+    for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) {
+        const uint32_t b = kBuckets - 1 - min((uint32_t)(min(cost(i), (uint64_t)0xFFFFFFFFu) >> shift), (uint32_t)kBuckets - 1);
+        order[atomicAdd(&hist[b], 1u)] = i;
+    }
+}
+
 __global__ void __launch_bounds__(kWPB * 32)
 k_inject(EmuProg P, const uint8_t* img, const uint64_t* __restrict__ warp_off, const fi_site* __restrict__ sites,
          uint32_t n, fi_inj* __restrict__ out, fi_store* __restrict__ log, uint32_t cap, uint32_t* ckpt,
-         const uint64_t* __restrict__ ck_off, uint32_t ck_interval, uint32_t* status) {
+         const uint64_t* __restrict__ ck_off, uint32_t ck_interval, const uint32_t* __restrict__ order,
+         uint32_t* counter, uint32_t* status) {
     extern __shared__ uint32_t smem[];
     const uint32_t wib = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const uint32_t i = blockIdx.x * kWPB + wib;
-    if (i >= n) return;
+    for (;;) {                                        // persistent warp: take the next replica
+    uint32_t p = 0;
+    if (lane == 0) p = atomicAdd(counter, 1u);
+    p = __shfl_sync(kFull, p, 0);
+    if (p >= n) return;
+    const uint32_t i = order[p];
     const fi_site S = sites[i];
     const fi_instance in = P.inst[S.instance];
     const uint32_t wpc = (in.block + 31) / 32, lw = S.warp - in.warp_begin;
@@ -52,6 +96,8 @@ k_inject(EmuProg P, const uint8_t* img, const uint64_t* __restrict__ warp_off, c
         r.n_faulty_stores = o.nstore;
         out[i] = r;
         if (!o.fired || o.bad) FI_DEV_ERR(status, FI_E_SITE);
+    }
+    __syncwarp();
     }
 }
 
@@ -162,18 +208,32 @@ __global__ void __launch_bounds__(kClsWarps * 32) k_classify(const ClsArgs A) {
 
 using namespace fi;
 
+extern "C" size_t fi_inject_workspace(uint32_t n) { return 256 + (size_t)n * 4; }
+
 extern "C" fi_status fi_inject(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
-                               uint32_t n, fi_inj* out, fi_store* log, uint32_t log_cap, uint32_t* dev_status,
-                               void* stream) {
+                               uint32_t n, fi_inj* out, fi_store* log, uint32_t log_cap, void* ws, size_t ws_bytes,
+                               uint32_t* dev_status, void* stream) {
     if (!p || !image || !t || !sites || !out || !dev_status || (log_cap && !log) || !p->aux) return FI_E_ARG;
     if (t->ckpt && (!t->ckpt_off || !t->ckpt_interval)) return FI_E_ARG;
     if (n == 0) return FI_OK;
-    const size_t smem = golden_smem(p->n_regs);
-    fi_status e = cuda_status(cudaFuncSetAttribute((const void*)k_inject, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    if (!ws || ws_bytes < fi_inject_workspace(n)) return FI_E_ARG;
+    cudaStream_t s = (cudaStream_t)stream;
+    uint32_t* counter = reinterpret_cast<uint32_t*>(ws);
+    uint32_t* order = reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(ws) + 256);
+    const uint32_t ck_iv = t->ckpt ? t->ckpt_interval : 0;
+    k_lpt_order<<<1, 1024, 0, s>>>(sites, t->warp_off, ck_iv, n, order, counter);
+    fi_status e = launch_status();
     if (e) return e;
-    k_inject<<<(n + kWPB - 1) / kWPB, kWPB * 32, smem, (cudaStream_t)stream>>>(
-        make_emu_prog(p), image, t->warp_off, sites, n, out, log, log_cap, t->ckpt, t->ckpt_off, t->ckpt_interval,
-        dev_status);
+    const size_t smem = golden_smem(p->n_regs);
+    e = cuda_status(cudaFuncSetAttribute((const void*)k_inject, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    if (e) return e;
+    int dev = 0, sms = 0, per = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_inject, kWPB * 32, smem);
+    const uint32_t grid = (uint32_t)std::min<uint64_t>((n + kWPB - 1) / kWPB, (uint64_t)std::max(1, sms * std::max(1, per)));
+    k_inject<<<grid, kWPB * 32, smem, s>>>(make_emu_prog(p), image, t->warp_off, sites, n, out, log, log_cap, t->ckpt,
+                                           t->ckpt_off, ck_iv, order, counter, dev_status);
     return launch_status();
 }
 

@@ -101,7 +101,8 @@ def lib():
             "fi_build_site_index": (st, [vp, u32, vp, u64, vp, vp]),
             "fi_site_totals": (st, [vp, u32, vp, vp]),
             "fi_select_sites": (st, [vp, vp, vp, u32, u64, vp, vp, u64, u32, vp, vp, vp]),
-            "fi_inject": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, vp]),
+            "fi_inject_workspace": (sz, [u32]),
+            "fi_inject": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, sz, vp, vp]),
             "fi_classify": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, vp, vp]),
             "fi_write_params_txt": (st, [vp, C.c_char_p, C.c_char_p, sz]),
         }
@@ -326,7 +327,7 @@ def select_sites(idx: SiteIndex, sched: fi_schedule, j0: int, n: int, sites: tor
 
 
 def inject(gt: GoldenTrace, sites: torch.Tensor, n: int, log_cap: int, out: torch.Tensor | None = None,
-           log: torch.Tensor | None = None, status: DeviceStatus | None = None):
+           log: torch.Tensor | None = None, status: DeviceStatus | None = None, ws: torch.Tensor | None = None):
     """fi_inject (K4)."""
     dev = gt.dp.device
     if out is None:
@@ -334,8 +335,11 @@ def inject(gt: GoldenTrace, sites: torch.Tensor, n: int, log_cap: int, out: torc
     if log is None:
         log = torch.empty(max(n * log_cap, 1) * 16, dtype=torch.uint8, device=dev)
     st = status or DeviceStatus(dev)
+    ws_n = lib().fi_inject_workspace(n)
+    if ws is None or ws.numel() < ws_n:
+        ws = torch.empty(ws_n, dtype=torch.uint8, device=dev)
     _check(lib().fi_inject(C.byref(gt.dp.c), _p(gt.image), C.byref(gt.c), _p(sites), n, _p(out), _p(log), log_cap,
-                           st.ptr, _stream()), "fi_inject")
+                           _p(ws), ws_n, st.ptr, _stream()), "fi_inject")
     if status is None:
         st.check("fi_inject")
     return out, log
