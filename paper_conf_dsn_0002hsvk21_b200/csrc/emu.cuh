@@ -176,6 +176,25 @@ __device__ __forceinline__ uint32_t dev_lop3(uint32_t a, uint32_t b, uint32_t c,
     return r;
 }
 
+// Image data loads bypass L1 allocation: the small L1 left next to the register
+// files must keep the decoded code, granule map and buffer table resident.
+__device__ __forceinline__ uint32_t ld_img32(const uint8_t* p) {
+    uint32_t r;
+    asm volatile("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(r) : "l"(p));
+    return r;
+}
+__device__ __forceinline__ uint2 ld_img64(const uint8_t* p) {
+    uint2 r;
+    asm volatile("ld.global.nc.L1::no_allocate.v2.u32 {%0, %1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p));
+    return r;
+}
+__device__ __forceinline__ uint4 ld_img128(const uint8_t* p) {
+    uint4 r;
+    asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+    return r;
+}
+
 // Per-lane two-entry cache of buffer bounds (image offsets) for memory checks.
 struct BufCache {
     uint64_t lo0 = 1, hi0 = 0, lo1 = 1, hi1 = 0;   // empty ranges
@@ -428,12 +447,36 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
         if (conv) {
             // ---- straight-line run: no scheduling / control bookkeeping per step
             const uint32_t rw = __ldg(&runl[pcm]);
-            uint32_t run = rw & 0xFFFF, lr = rw >> 16;
+            uint32_t run = rw & 0xFFFF, lr = (rw >> 16) & 0xFF, fr = rw >> 24;
             uint32_t lim = watchdog - step;
             if (MODE == EMU_TRACE && use_ck) lim = min(lim, ck_interval - step % ck_interval);
             if (MODE == EMU_INJ && hook.step >= step) lim = min(lim, hook.step - step);
             run = min(run, lim);
             lr = min(min(lr, lim), (uint32_t)kLdgBatch);
+            fr = min(fr, lim);
+            if (fr) {
+                // ---- simple-FFMA run: unguarded, unmodified FFMAs (superinstruction loop)
+                const uint4* dp = dec + pcm;
+                uint4 nx = __ldg(&dp[0]);
+#pragma unroll 4
+                for (uint32_t j = 0; j < fr; ++j) {
+                    const uint4 cur = nx;
+                    nx = __ldg(&dp[min(j + 1, fr - 1)]);      // prefetch (branch-free)
+                    const float x = u2f(F.rd(cur.y & 0xFFFF)), y = u2f(F.rd(cur.y >> 16)), z = u2f(F.rd(cur.z & 0xFFFF));
+                    const float rf = __fmaf_rn(x, y, z);
+                    const uint32_t r = rf != rf ? kQNaN32 : __float_as_uint(rf);
+                    // simple FFMAs have a real destination (decode guarantees rd < zero row)
+                    if (live) *reinterpret_cast<uint32_t*>(F.Rb + (cur.z >> 16)) = r;
+                    if (MODE == EMU_TRACE) {
+                        const uint32_t s = step + j;
+                        if ((s & 31) == lane) recbuf = make_uint4(k, __ldg(&ins[pcm + j]), livem, kFull);
+                        if ((s & 31) == 31) reinterpret_cast<uint4*>(rec_out)[s - 31 + lane] = recbuf;
+                    }
+                }
+                step += fr;
+                upc = pcm + fr;
+                continue;
+            }
             if (lr >= 2) {
                 // ---- LDG batch: independent loads in flight together
                 uint4 vals[kLdgBatch];
@@ -462,9 +505,9 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
                         }
                         const uint8_t* src = img + (va - kVaBase);
                         if (ex && !c && !zero) {
-                            if (lw == 0) vals[b].x = __ldg(reinterpret_cast<const uint32_t*>(src));
-                            else if (lw == 1) { const uint2 t = __ldg(reinterpret_cast<const uint2*>(src)); vals[b].x = t.x; vals[b].y = t.y; }
-                            else vals[b] = __ldg(reinterpret_cast<const uint4*>(src));
+                            if (lw == 0) vals[b].x = ld_img32(src);
+                            else if (lw == 1) { const uint2 t = ld_img64(src); vals[b].x = t.x; vals[b].y = t.y; }
+                            else vals[b] = ld_img128(src);
                         }
                         exs[b] = ex;
                         dsts[b] = D.z >> 16;
@@ -500,7 +543,7 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
                 uint4 Dn = __ldg(&dec[pcm]);
                 for (uint32_t j = 0; j < run; ++j) {
                     const uint4 D = Dn;
-                    if (j + 1 < run) Dn = __ldg(&dec[pcm + j + 1]);
+                    Dn = __ldg(&dec[pcm + min(j + 1, run - 1)]);
                     const uint32_t guard = (D.x >> 8) & 0xFF;
                     bool pv = true;
                     uint32_t pred = kFull;
@@ -558,12 +601,12 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
                 if (ex) {
                     const uint8_t* src = img + (va - kVaBase);
                     if (lw == 0) {
-                        F.wr(id, zero ? 0u : __ldg(reinterpret_cast<const uint32_t*>(src)));
+                        F.wr(id, zero ? 0u : ld_img32(src));
                     } else if (lw == 1) {
-                        const uint2 v = zero ? make_uint2(0, 0) : __ldg(reinterpret_cast<const uint2*>(src));
+                        const uint2 v = zero ? make_uint2(0, 0) : ld_img64(src);
                         F.wr(id, v.x); F.wr(id + 128, v.y);
                     } else {
-                        const uint4 v = zero ? make_uint4(0, 0, 0, 0) : __ldg(reinterpret_cast<const uint4*>(src));
+                        const uint4 v = zero ? make_uint4(0, 0, 0, 0) : ld_img128(src);
                         F.wr(id, v.x); F.wr(id + 128, v.y); F.wr(id + 256, v.z); F.wr(id + 384, v.w);
                     }
                 }

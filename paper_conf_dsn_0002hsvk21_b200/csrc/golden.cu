@@ -102,7 +102,12 @@ __global__ void k_decode(const fi_insn* code, uint32_t n_code, const fi_kernel* 
         if (hazard) break;
         ++lr;
     }
-    run[i] = (r > 0xFFFF ? 0xFFFFu : r) | (lr << 16);
+    // simple-FFMA run: unguarded FFMAs without operand modifiers (GEMM / conv inner loops)
+    uint32_t fr = 0;
+    for (uint32_t j = i; j < end && fr < 0xFF && code[j].op == FFMA && code[j].guard == kPT && code[j].mod == 0 &&
+                         code[j].d0 < zr; ++j)
+        ++fr;
+    run[i] = (r > 0xFFFF ? 0xFFFFu : r) | (std::min<uint32_t>(lr, 0xFF) << 16) | (fr << 24);
 }
 
 __global__ void k_ckpt_counts(const uint64_t* warp_len, uint32_t n, uint32_t interval, uint64_t* cnt) {
