@@ -159,8 +159,11 @@ fi_status fi_profile(const fi_trace* t, uint64_t rec_begin, uint64_t rec_end, ui
                      uint64_t* inst_counts, uint32_t* chunk_counts, void* stream);
 #define FI_CHUNK 1024
 
-/* K2 — site index: exclusive prefix sums P_k[n_inst+1][8] of inst_counts and
- * P_c[n_chunks+1][8] of chunk_counts (u64), decoupled-lookback scan.
+/* K2 — site index ("1..N" of PAPER.md:78 as prefix sums): exclusive prefix
+ * sums P_k[n_inst+1][8] of inst_counts and P_t[T+1][8] of the chunk counts
+ * summed per tile of 64 chunks (T = ceil(n_chunks/64)), both u64 with the
+ * decoupled-lookback scan; the chunk level itself is resolved at selection time
+ * by a warp scan of the tile's chunk counts (no per-chunk prefix array).
  * `index` must hold fi_site_index_bytes(n_inst, n_chunks) bytes. */
 size_t fi_site_index_bytes(uint32_t n_inst, uint64_t n_chunks);
 fi_status fi_build_site_index(const uint64_t* inst_counts, uint32_t n_inst, const uint32_t* chunk_counts,
@@ -174,9 +177,10 @@ fi_status fi_site_totals(const void* index, uint32_t n_inst, uint64_t totals_hos
  * Replica j = j0 + i for i < n: s by Philox4x32-10 + Lemire,
  * then instance, chunk, record, lane, warp, step, slot and mask.
  * `sched` is a host pointer.  totals_host from fi_site_totals. */
-fi_status fi_select_sites(const fi_program* p, const fi_trace* t, const void* index, uint32_t n_inst,
-                          uint64_t n_chunks, const uint64_t totals_host[8], const fi_schedule* sched,
-                          uint64_t j0, uint32_t n, fi_site* sites, uint32_t* dev_status, void* stream);
+fi_status fi_select_sites(const fi_program* p, const fi_trace* t, const uint32_t* chunk_counts, const void* index,
+                          uint32_t n_inst, uint64_t n_chunks, const uint64_t totals_host[8],
+                          const fi_schedule* sched, uint64_t j0, uint32_t n, fi_site* sites, uint32_t* dev_status,
+                          void* stream);
 
 /* K4 — inject: one CUDA warp re-executes the site's
  * synthetic warp over the golden final image — from its first instruction, or

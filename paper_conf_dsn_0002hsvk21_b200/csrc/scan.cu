@@ -75,41 +75,54 @@ k_scan_rows(const Tin* __restrict__ in, uint64_t* __restrict__ out, uint64_t n_r
         }
     }
     __syncthreads();
-    if (threadIdx.x == 0) {
+    if (wid == 0) {
+        // decoupled lookback, one warp: publish this tile's aggregate, then look at
+        // 32 predecessors per probe; the nearest one with an inclusive prefix (P)
+        // ends the walk, the aggregate-only (A) ones in front of it are added.
         uint64_t agg[W];
 #pragma unroll
         for (int g = 0; g < W; ++g) agg[g] = s_warp[kThreads / 32 - 1][g];
-        volatile uint32_t* flags = &st[0].flag;
-        (void)flags;
         if (tile == 0) {
+            if (lane == 0) {
 #pragma unroll
-            for (int g = 0; g < W; ++g) { st[0].inc[g] = agg[g]; s_prefix[g] = 0; }
-            __threadfence();
-            *(volatile uint32_t*)&st[0].flag = 2u;
+                for (int g = 0; g < W; ++g) { st[0].inc[g] = agg[g]; s_prefix[g] = 0; }
+                __threadfence();
+                *(volatile uint32_t*)&st[0].flag = 2u;
+            }
         } else {
+            if (lane == 0) {
 #pragma unroll
-            for (int g = 0; g < W; ++g) st[tile].agg[g] = agg[g];
-            __threadfence();
-            *(volatile uint32_t*)&st[tile].flag = 1u;
+                for (int g = 0; g < W; ++g) st[tile].agg[g] = agg[g];
+                __threadfence();
+                *(volatile uint32_t*)&st[tile].flag = 1u;
+            }
             uint64_t pre[W];
 #pragma unroll
             for (int g = 0; g < W; ++g) pre[g] = 0;
-            for (int64_t p = (int64_t)tile - 1; p >= 0; --p) {
-                uint32_t f;
-                while ((f = *(volatile uint32_t*)&st[p].flag) == 0u) { }
+            for (int64_t base = (int64_t)tile - 1;; base -= 32) {
+                const int64_t p = base - (int64_t)lane;
+                uint32_t f = p >= 0 ? *(volatile uint32_t*)&st[p].flag : 2u;
+                while (__any_sync(0xFFFFFFFFu, f == 0u))
+                    if (f == 0u) f = *(volatile uint32_t*)&st[p].flag;
                 __threadfence();
-                if (f == 2u) {
+                const uint32_t pm = __ballot_sync(0xFFFFFFFFu, f == 2u);
+                const uint32_t stop = pm ? (uint32_t)(__ffs(pm) - 1) : 32u;
+                if (p >= 0 && lane <= stop) {
 #pragma unroll
-                    for (int g = 0; g < W; ++g) pre[g] += __ldcg(&st[p].inc[g]);
-                    break;
+                    for (int g = 0; g < W; ++g) pre[g] += lane == stop ? __ldcg(&st[p].inc[g]) : __ldcg(&st[p].agg[g]);
                 }
-#pragma unroll
-                for (int g = 0; g < W; ++g) pre[g] += __ldcg(&st[p].agg[g]);
+                if (pm) break;
             }
 #pragma unroll
-            for (int g = 0; g < W; ++g) { st[tile].inc[g] = pre[g] + agg[g]; s_prefix[g] = pre[g]; }
-            __threadfence();
-            *(volatile uint32_t*)&st[tile].flag = 2u;
+            for (int g = 0; g < W; ++g)
+#pragma unroll
+                for (int d = 16; d > 0; d >>= 1) pre[g] += __shfl_xor_sync(0xFFFFFFFFu, pre[g], d);
+            if (lane == 0) {
+#pragma unroll
+                for (int g = 0; g < W; ++g) { st[tile].inc[g] = pre[g] + agg[g]; s_prefix[g] = pre[g]; }
+                __threadfence();
+                *(volatile uint32_t*)&st[tile].flag = 2u;
+            }
         }
     }
     __syncthreads();

@@ -71,7 +71,9 @@ __device__ uint64_t warp_upper_search(const uint64_t* __restrict__ arr, uint64_t
 struct SelArgs {
     const fi_insn* code; const fi_kernel* kern; const fi_instance* inst;
     const uint4* rec; uint64_t n_rec; const uint64_t* warp_off; uint32_t n_warps;
-    const uint64_t* Pk; uint32_t n_inst; const uint64_t* Pc; uint64_t n_chunks;
+    const uint64_t* Pk; uint32_t n_inst;
+    const uint64_t* Pt; uint64_t n_tiles;         // prefix over 64-chunk tiles
+    const uint32_t* cc; uint64_t n_chunks;        // chunk counts [C][8]
     uint64_t totals[8];
     fi_schedule sched;
     uint64_t j0; uint32_t n;
@@ -79,6 +81,7 @@ struct SelArgs {
 };
 
 constexpr int kWarps = 4;
+constexpr uint32_t kTileChunks = 64;          // chunks per index tile (two-level chunk index)
 
 __global__ void __launch_bounds__(kWarps * 32) k_select(const SelArgs A) {
     const uint32_t lane = threadIdx.x & 31;
@@ -96,10 +99,30 @@ __global__ void __launch_bounds__(kWarps * 32) k_select(const SelArgs A) {
     u_dst = __shfl_sync(0xFFFFFFFFu, u_dst, 0);
     u_bit = __shfl_sync(0xFFFFFFFFu, u_bit, 0);
 
-    // instance: last k with P_k[k][g] <= s ; chunk: last c with P_c[c][g] <= s
+    // instance: last k with P_k[k][g] <= s ; tile: last t with P_t[t][g] <= s
     const uint32_t k = (uint32_t)warp_upper_search(A.Pk, A.n_inst, 8, g, s);
-    const uint64_t c = warp_upper_search(A.Pc, A.n_chunks, 8, g, s);
-    uint64_t r = s - __ldg(&A.Pc[c * 8 + g]);
+    const uint64_t t = warp_upper_search(A.Pt, A.n_tiles, 8, g, s);
+    uint64_t r = s - __ldg(&A.Pt[t * 8 + g]);
+    // chunk inside the tile: warp scan of its (up to 64) chunk counts of group g
+    uint64_t c = t * kTileChunks;
+    for (uint32_t half = 0; half < kTileChunks; half += 32) {
+        const uint64_t ci = t * kTileChunks + half + lane;
+        const uint32_t cnt = ci < A.n_chunks ? __ldg(&A.cc[ci * 8 + g]) : 0u;
+        uint32_t incl = cnt;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, incl, d);
+            if (lane >= (uint32_t)d) incl += y;
+        }
+        const uint32_t total = __shfl_sync(0xFFFFFFFFu, incl, 31);
+        if (r < total) {
+            const uint32_t L = __ffs(__ballot_sync(0xFFFFFFFFu, incl > r)) - 1;
+            r -= __shfl_sync(0xFFFFFFFFu, incl - cnt, L);
+            c = t * kTileChunks + half + L;
+            break;
+        }
+        r -= total;
+    }
 
     // scan the chunk's records for the r-th counted lane-instruction of group g
     const uint64_t base = c * FI_CHUNK;
@@ -176,17 +199,47 @@ __global__ void __launch_bounds__(kWarps * 32) k_select(const SelArgs A) {
 
 size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
 
+uint64_t n_tiles_of(uint64_t n_chunks) { return (n_chunks + kTileChunks - 1) / kTileChunks; }
+
 struct IndexLayout {
-    size_t pk, pc, ws_k, ws_c, total;
+    size_t pk, pt, tsum, ws_k, ws_t, total;
 };
 IndexLayout layout(uint32_t n_inst, uint64_t n_chunks) {
+    const uint64_t T = n_tiles_of(n_chunks);
     IndexLayout L;
     L.pk = 0;
-    L.pc = align256(((size_t)n_inst + 1) * 8 * sizeof(uint64_t));
-    L.ws_k = L.pc + align256(((size_t)n_chunks + 1) * 8 * sizeof(uint64_t));
-    L.ws_c = L.ws_k + align256(scan_rows_ws(n_inst, 8));
-    L.total = L.ws_c + align256(scan_rows_ws(n_chunks, 8));
+    L.pt = align256(((size_t)n_inst + 1) * 8 * sizeof(uint64_t));
+    L.tsum = L.pt + align256(((size_t)T + 1) * 8 * sizeof(uint64_t));
+    L.ws_k = L.tsum + align256((size_t)std::max<uint64_t>(T, 1) * 8 * sizeof(uint64_t));
+    L.ws_t = L.ws_k + align256(scan_rows_ws(n_inst, 8));
+    L.total = L.ws_t + align256(scan_rows_ws(T, 8));
     return L;
+}
+
+// per-tile sums of the chunk counts: one warp per 64-chunk tile
+__global__ void k_tile_sums(const uint32_t* __restrict__ cc, uint64_t n_chunks, uint64_t n_tiles,
+                            uint64_t* __restrict__ tsum) {
+    const uint64_t t = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t lane = threadIdx.x & 31;
+    if (t >= n_tiles) return;
+    uint64_t acc[8];
+#pragma unroll
+    for (int g = 0; g < 8; ++g) acc[g] = 0;
+#pragma unroll
+    for (uint32_t half = 0; half < kTileChunks; half += 32) {
+        const uint64_t ci = t * kTileChunks + half + lane;
+        if (ci < n_chunks) {
+            const uint4 a = __ldg(reinterpret_cast<const uint4*>(cc + ci * 8));
+            const uint4 b = __ldg(reinterpret_cast<const uint4*>(cc + ci * 8 + 4));
+            acc[0] += a.x; acc[1] += a.y; acc[2] += a.z; acc[3] += a.w;
+            acc[4] += b.x; acc[5] += b.y; acc[6] += b.z; acc[7] += b.w;
+        }
+    }
+#pragma unroll
+    for (int g = 0; g < 8; ++g) {
+        const uint64_t v = __reduce_add_sync(0xFFFFFFFFu, (uint32_t)acc[g]);  // per-tile sum < 2^32 (64 x 1024 x 32)
+        if (lane == (uint32_t)g) tsum[t * 8 + g] = v;
+    }
 }
 
 }  // namespace
@@ -203,10 +256,15 @@ extern "C" fi_status fi_build_site_index(const uint64_t* inst_counts, uint32_t n
     char* b = reinterpret_cast<char*>(index);
     cudaStream_t s = (cudaStream_t)stream;
     fi_status e = scan_rows_u64x8(inst_counts, reinterpret_cast<uint64_t*>(b + L.pk), n_inst, b + L.ws_k,
-                                  L.ws_c - L.ws_k, s);
+                                  L.ws_t - L.ws_k, s);
     if (e) return e;
-    return scan_rows_u32x8(chunk_counts, reinterpret_cast<uint64_t*>(b + L.pc), n_chunks, b + L.ws_c,
-                           L.total - L.ws_c, s);
+    const uint64_t T = n_tiles_of(n_chunks);
+    uint64_t* tsum = reinterpret_cast<uint64_t*>(b + L.tsum);
+    if (T) {
+        k_tile_sums<<<(unsigned)((T * 32 + 255) / 256), 256, 0, s>>>(chunk_counts, n_chunks, T, tsum);
+        if ((e = launch_status())) return e;
+    }
+    return scan_rows_u64x8(tsum, reinterpret_cast<uint64_t*>(b + L.pt), T, b + L.ws_t, L.total - L.ws_t, s);
 }
 
 extern "C" fi_status fi_site_totals(const void* index, uint32_t n_inst, uint64_t totals_host[8], void* stream) {
@@ -219,10 +277,11 @@ extern "C" fi_status fi_site_totals(const void* index, uint32_t n_inst, uint64_t
     return cuda_status(cudaStreamSynchronize(s));
 }
 
-extern "C" fi_status fi_select_sites(const fi_program* p, const fi_trace* t, const void* index, uint32_t n_inst,
-                                     uint64_t n_chunks, const uint64_t totals_host[8], const fi_schedule* sched,
-                                     uint64_t j0, uint32_t n, fi_site* sites, uint32_t* dev_status, void* stream) {
-    if (!p || !t || !index || !totals_host || !sched || !sites || !dev_status) return FI_E_ARG;
+extern "C" fi_status fi_select_sites(const fi_program* p, const fi_trace* t, const uint32_t* chunk_counts,
+                                     const void* index, uint32_t n_inst, uint64_t n_chunks,
+                                     const uint64_t totals_host[8], const fi_schedule* sched, uint64_t j0, uint32_t n,
+                                     fi_site* sites, uint32_t* dev_status, void* stream) {
+    if (!p || !t || !index || !chunk_counts || !totals_host || !sched || !sites || !dev_status) return FI_E_ARG;
     if (sched->n_groups == 0 || sched->n_groups > 8 || sched->n_bfms == 0 || sched->n_bfms > 4) return FI_E_ARG;
     for (uint32_t i = 0; i < sched->n_groups; ++i) {
         if (sched->groups[i] >= FI_NGROUPS) return FI_E_ARG;
@@ -238,7 +297,8 @@ extern "C" fi_status fi_select_sites(const fi_program* p, const fi_trace* t, con
     A.code = p->code; A.kern = p->kern; A.inst = p->inst;
     A.rec = reinterpret_cast<const uint4*>(t->rec); A.n_rec = t->n_rec; A.warp_off = t->warp_off; A.n_warps = t->n_warps;
     A.Pk = reinterpret_cast<const uint64_t*>(b + L.pk); A.n_inst = n_inst;
-    A.Pc = reinterpret_cast<const uint64_t*>(b + L.pc); A.n_chunks = n_chunks;
+    A.Pt = reinterpret_cast<const uint64_t*>(b + L.pt); A.n_tiles = n_tiles_of(n_chunks);
+    A.cc = chunk_counts; A.n_chunks = n_chunks;
     for (int g = 0; g < 8; ++g) A.totals[g] = totals_host[g];
     A.sched = *sched;
     A.j0 = j0; A.n = n; A.sites = sites; A.status = dev_status;

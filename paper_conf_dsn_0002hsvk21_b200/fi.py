@@ -100,7 +100,7 @@ def lib():
             "fi_site_index_bytes": (sz, [u32, u64]),
             "fi_build_site_index": (st, [vp, u32, vp, u64, vp, vp]),
             "fi_site_totals": (st, [vp, u32, vp, vp]),
-            "fi_select_sites": (st, [vp, vp, vp, u32, u64, vp, vp, u64, u32, vp, vp, vp]),
+            "fi_select_sites": (st, [vp, vp, vp, vp, u32, u64, vp, vp, u64, u32, vp, vp, vp]),
             "fi_inject_workspace": (sz, [u32]),
             "fi_inject": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, sz, vp, vp]),
             "fi_classify": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, vp, vp]),
@@ -282,10 +282,11 @@ def profile(gt: GoldenTrace, rec_begin: int = 0, rec_end: int | None = None,
 
 
 class SiteIndex:
-    """fi_build_site_index (K2): P_k and P_c prefix sums; totals N_g."""
+    """fi_build_site_index (K2): P_k and 64-chunk-tile prefix sums; totals N_g."""
 
     def __init__(self, gt: GoldenTrace, inst_counts: torch.Tensor, chunk_counts: torch.Tensor):
         self.gt = gt
+        self.chunk_counts = chunk_counts
         self.n_inst = gt.dp.n_inst
         self.n_chunks = gt.n_chunks
         nb = lib().fi_site_index_bytes(self.n_inst, self.n_chunks)
@@ -319,7 +320,8 @@ def select_sites(idx: SiteIndex, sched: fi_schedule, j0: int, n: int, sites: tor
     if sites is None:
         sites = torch.empty(max(n, 1) * 64, dtype=torch.uint8, device=gt.dp.device)
     st = status or DeviceStatus(gt.dp.device)
-    _check(lib().fi_select_sites(C.byref(gt.dp.c), C.byref(gt.c), _p(idx.buf), idx.n_inst, idx.n_chunks,
+    _check(lib().fi_select_sites(C.byref(gt.dp.c), C.byref(gt.c), _p(idx.chunk_counts), _p(idx.buf), idx.n_inst,
+                                 idx.n_chunks,
                                  idx._tot, C.byref(sched), j0, n, _p(sites), st.ptr, _stream()), "fi_select_sites")
     if status is None:
         st.check("fi_select_sites")

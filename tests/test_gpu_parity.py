@@ -184,3 +184,37 @@ def test_empty_and_ragged(F):
     ic, cc = F.profile(gt)
     idx = F.SiteIndex(gt, ic, cc)
     F.select_sites(idx, F.schedule(1, [F.G_GP], [0]), 0, 0)
+
+
+@pytest.mark.parametrize("n", [0, 1, 255, 256, 4096, 4097, 300001, 2_500_000])
+def test_scan_u64_and_rows(F, n):
+    """K2 scans (decoupled lookback) against numpy cumsum: width-1 u64 and width-8
+    u32 rows (the chunk index), many tiles and a ragged tail."""
+    rng = np.random.Generator(np.random.PCG64(n))
+    x = rng.integers(0, 2**40, n, dtype=np.uint64)
+    got = F.scan_u64(torch.from_numpy(x.view(np.int64)).cuda()).cpu().numpy().view(np.uint64)
+    want = np.concatenate([[0], np.cumsum(x, dtype=np.uint64)])
+    assert np.array_equal(got, want)
+    # width-8 u32 rows through the site index
+    cc = rng.integers(0, 32768, (max(n, 1), 8), dtype=np.int64).astype(np.int32)
+    ic = rng.integers(0, 2**40, (3, 8), dtype=np.int64)
+    L = F.lib()
+    import ctypes as C
+    nb = L.fi_site_index_bytes(3, n)
+    buf = torch.empty(nb, dtype=torch.uint8, device="cuda")
+    cct = torch.from_numpy(cc).cuda()
+    ict = torch.from_numpy(ic).cuda()
+    rc = L.fi_build_site_index(ict.data_ptr(), 3, cct.data_ptr(), n, buf.data_ptr(), torch.cuda.current_stream().cuda_stream)
+    assert rc == 0
+    torch.cuda.synchronize()
+    b = buf.cpu().numpy()
+    pk = b[: 4 * 64].view(np.uint64).reshape(4, 8)
+    assert np.array_equal(pk, np.concatenate([np.zeros((1, 8), np.uint64), np.cumsum(ic.astype(np.uint64), 0)]))
+    off = (4 * 64 + 255) // 256 * 256
+    T = (n + 63) // 64
+    pt = b[off: off + (T + 1) * 64].view(np.uint64).reshape(T + 1, 8)
+    tiles = np.zeros((T, 8), np.uint64)
+    for t in range(T):
+        tiles[t] = cc[t * 64: min(n, t * 64 + 64)].astype(np.uint64).sum(0)
+    wantt = np.concatenate([np.zeros((1, 8), np.uint64), np.cumsum(tiles, 0)])
+    assert np.array_equal(pt, wantt)
