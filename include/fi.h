@@ -33,7 +33,8 @@ typedef enum {
     FI_E_PROGRAM = 4,          /* golden run faulted / program violates DESIGN.md §3.5 */
     FI_E_CUDA = 5,
     FI_E_SITE = 6,             /* a site does not match the re-executed warp */
-    FI_E_CAPACITY = 8          /* faulty store log overflow (replica must be re-run with a larger log) */
+    FI_E_CAPACITY = 8,         /* faulty store log overflow (replica must be re-run with a larger log) */
+    FI_E_INVARIANT = 9         /* a Table II identity does not hold for a count row (§8 row a3) */
 } fi_status;
 
 /* Table II arch state ids [PAPER.md:94-104], 0-based (C-1) */
@@ -164,10 +165,13 @@ fi_status fi_profile(const fi_trace* t, uint64_t rec_begin, uint64_t rec_end, ui
  * summed per tile of 64 chunks (T = ceil(n_chunks/64)), both u64 with the
  * decoupled-lookback scan; the chunk level itself is resolved at selection time
  * by a warp scan of the tile's chunk counts (no per-chunk prefix array).
- * `index` must hold fi_site_index_bytes(n_inst, n_chunks) bytes. */
+ * `index` must hold fi_site_index_bytes(n_inst, n_chunks) bytes.
+ * §8 row a3: on the way it checks the Table II identities [PAPER.md:101-104]
+ * (GP = FP64+FP32+LD+OTHERS, GPPR = GP+PR) and count <= 32 x records on every
+ * instance row and every chunk row; a violation sets FI_E_INVARIANT. */
 size_t fi_site_index_bytes(uint32_t n_inst, uint64_t n_chunks);
 fi_status fi_build_site_index(const uint64_t* inst_counts, uint32_t n_inst, const uint32_t* chunk_counts,
-                              uint64_t n_chunks, void* index, void* stream);
+                              uint64_t n_chunks, void* index, uint32_t* dev_status, void* stream);
 /* Totals N_g (host, synchronizes): copies P_k[n_inst][*] */
 fi_status fi_site_totals(const void* index, uint32_t n_inst, uint64_t totals_host[8], void* stream);
 

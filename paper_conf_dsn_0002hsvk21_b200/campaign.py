@@ -110,7 +110,7 @@ class Campaign:
             allreduce_sum_(self.inst_counts, self.group)
             allreduce_sum_(self.chunk_counts, self.group)
         mark("exchange")
-        idx = fi.SiteIndex(self.gt, self.inst_counts, self.chunk_counts)
+        idx = fi.SiteIndex(self.gt, self.inst_counts, self.chunk_counts, self.status)
         mark("index")
         n = self.n_local
         fi.select_sites(idx, self.sched, self.j0, n, self.sites, self.status)

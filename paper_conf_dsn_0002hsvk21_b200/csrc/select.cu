@@ -216,9 +216,28 @@ IndexLayout layout(uint32_t n_inst, uint64_t n_chunks) {
     return L;
 }
 
-// per-tile sums of the chunk counts: one warp per 64-chunk tile
+// Table II identities [PAPER.md:101-104] (§8 row a3), checked on every count row:
+// GP = FP64 + FP32 + LD + OTHERS, GPPR = GP + PR, and no group exceeds 32 lanes per record.
+template <class T>
+__device__ __forceinline__ bool identities_hold(const T c[8], uint64_t max_count) {
+    bool ok = (uint64_t)c[FI_G_GP] == (uint64_t)c[FI_G_FP64] + c[FI_G_FP32] + c[FI_G_LD] + c[FI_G_OTHERS];
+    ok = ok && (uint64_t)c[FI_G_GPPR] == (uint64_t)c[FI_G_GP] + c[FI_G_PR];
+    for (int g = 0; g < 8; ++g) ok = ok && (uint64_t)c[g] <= max_count;
+    return ok;
+}
+
+__global__ void k_inst_identities(const uint64_t* __restrict__ ic, uint32_t n_inst, uint32_t* status) {
+    const uint32_t k = blockIdx.x * blockDim.x + threadIdx.x;
+    if (k >= n_inst) return;
+    uint64_t c[8];
+    for (int g = 0; g < 8; ++g) c[g] = ic[(uint64_t)k * 8 + g];
+    if (!identities_hold(c, ~0ull)) FI_DEV_ERR(status, FI_E_INVARIANT);
+}
+
+// per-tile sums of the chunk counts: one warp per 64-chunk tile (and the a3
+// identities of every chunk row on the way)
 __global__ void k_tile_sums(const uint32_t* __restrict__ cc, uint64_t n_chunks, uint64_t n_tiles,
-                            uint64_t* __restrict__ tsum) {
+                            uint64_t* __restrict__ tsum, uint32_t* status) {
     const uint64_t t = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t lane = threadIdx.x & 31;
     if (t >= n_tiles) return;
@@ -233,6 +252,8 @@ __global__ void k_tile_sums(const uint32_t* __restrict__ cc, uint64_t n_chunks, 
             const uint4 b = __ldg(reinterpret_cast<const uint4*>(cc + ci * 8 + 4));
             acc[0] += a.x; acc[1] += a.y; acc[2] += a.z; acc[3] += a.w;
             acc[4] += b.x; acc[5] += b.y; acc[6] += b.z; acc[7] += b.w;
+            const uint32_t row[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
+            if (!identities_hold(row, 32ull * FI_CHUNK)) FI_DEV_ERR(status, FI_E_INVARIANT);
         }
     }
 #pragma unroll
@@ -250,8 +271,8 @@ using namespace fi;
 extern "C" size_t fi_site_index_bytes(uint32_t n_inst, uint64_t n_chunks) { return layout(n_inst, n_chunks).total; }
 
 extern "C" fi_status fi_build_site_index(const uint64_t* inst_counts, uint32_t n_inst, const uint32_t* chunk_counts,
-                                         uint64_t n_chunks, void* index, void* stream) {
-    if (!inst_counts || !chunk_counts || !index) return FI_E_ARG;
+                                         uint64_t n_chunks, void* index, uint32_t* dev_status, void* stream) {
+    if (!inst_counts || !chunk_counts || !index || !dev_status) return FI_E_ARG;
     const IndexLayout L = layout(n_inst, n_chunks);
     char* b = reinterpret_cast<char*>(index);
     cudaStream_t s = (cudaStream_t)stream;
@@ -260,8 +281,12 @@ extern "C" fi_status fi_build_site_index(const uint64_t* inst_counts, uint32_t n
     if (e) return e;
     const uint64_t T = n_tiles_of(n_chunks);
     uint64_t* tsum = reinterpret_cast<uint64_t*>(b + L.tsum);
+    if (n_inst) {
+        k_inst_identities<<<(n_inst + 127) / 128, 128, 0, s>>>(inst_counts, n_inst, dev_status);
+        if ((e = launch_status())) return e;
+    }
     if (T) {
-        k_tile_sums<<<(unsigned)((T * 32 + 255) / 256), 256, 0, s>>>(chunk_counts, n_chunks, T, tsum);
+        k_tile_sums<<<(unsigned)((T * 32 + 255) / 256), 256, 0, s>>>(chunk_counts, n_chunks, T, tsum, dev_status);
         if ((e = launch_status())) return e;
     }
     return scan_rows_u64x8(tsum, reinterpret_cast<uint64_t*>(b + L.pt), T, b + L.ws_t, L.total - L.ws_t, s);

@@ -19,7 +19,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(HERE, "libfi.so")
 
 FI_OK, FI_E_ARG, FI_E_EMPTY_GROUP, FI_E_NOT_INJECTABLE, FI_E_PROGRAM, FI_E_CUDA, FI_E_SITE = 0, 1, 2, 3, 4, 5, 6
-FI_E_CAPACITY = 8
+FI_E_CAPACITY, FI_E_INVARIANT = 8, 9
 FI_CHUNK = 1024
 G_FP64, G_FP32, G_LD, G_PR, G_NODEST, G_OTHERS, G_GPPR, G_GP = range(8)
 GROUP_NAMES = ["G_FP64", "G_FP32", "G_LD", "G_PR", "G_NODEST", "G_OTHERS", "G_GPPR", "G_GP"]
@@ -98,7 +98,7 @@ def lib():
             "fi_golden_trace": (st, [vp, vp, vp, vp, vp]),
             "fi_profile": (st, [vp, u64, u64, u32, vp, vp, vp]),
             "fi_site_index_bytes": (sz, [u32, u64]),
-            "fi_build_site_index": (st, [vp, u32, vp, u64, vp, vp]),
+            "fi_build_site_index": (st, [vp, u32, vp, u64, vp, vp, vp]),
             "fi_site_totals": (st, [vp, u32, vp, vp]),
             "fi_select_sites": (st, [vp, vp, vp, vp, u32, u64, vp, vp, u64, u32, vp, vp, vp]),
             "fi_inject_workspace": (sz, [u32]),
@@ -284,19 +284,23 @@ def profile(gt: GoldenTrace, rec_begin: int = 0, rec_end: int | None = None,
 class SiteIndex:
     """fi_build_site_index (K2): P_k and 64-chunk-tile prefix sums; totals N_g."""
 
-    def __init__(self, gt: GoldenTrace, inst_counts: torch.Tensor, chunk_counts: torch.Tensor):
+    def __init__(self, gt: GoldenTrace, inst_counts: torch.Tensor, chunk_counts: torch.Tensor,
+                 status: DeviceStatus | None = None):
         self.gt = gt
         self.chunk_counts = chunk_counts
         self.n_inst = gt.dp.n_inst
         self.n_chunks = gt.n_chunks
         nb = lib().fi_site_index_bytes(self.n_inst, self.n_chunks)
         self.buf = torch.empty(nb, dtype=torch.uint8, device=gt.dp.device)
+        st = status or DeviceStatus(gt.dp.device)
         _check(lib().fi_build_site_index(_p(inst_counts), self.n_inst, _p(chunk_counts), self.n_chunks,
-                                         _p(self.buf), _stream()), "fi_build_site_index")
+                                         _p(self.buf), st.ptr, _stream()), "fi_build_site_index")
         tot = (C.c_uint64 * 8)()
         _check(lib().fi_site_totals(_p(self.buf), self.n_inst, tot, _stream()), "fi_site_totals")
         self.totals = [int(x) for x in tot]
         self._tot = tot
+        if status is None:
+            st.check("fi_build_site_index")      # totals already synchronized the stream
 
     def prefix_inst(self) -> torch.Tensor:
         return self.buf[: (self.n_inst + 1) * 64].view(torch.int64).view(self.n_inst + 1, 8)

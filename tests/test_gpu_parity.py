@@ -158,6 +158,23 @@ def test_profile_shards_sum(F):
     assert torch.equal(ca[:nc], cfull[:nc]) and torch.equal(cb[nc:], cfull[nc:])
 
 
+def test_invariant_violation_detected(F):
+    prog = P.c1()
+    dp, gt = _gpu_golden(F, prog)
+    ic, cc = F.profile(gt)
+    F.SiteIndex(gt, ic, cc)                      # consistent counts pass
+    bad = ic.clone()
+    bad[0, F.G_GP] += 1
+    with pytest.raises(F.FIError) as e:
+        F.SiteIndex(gt, bad, cc)
+    assert e.value.code == F.FI_E_INVARIANT
+    badc = cc.clone()
+    badc[0, F.G_GPPR] -= 1
+    with pytest.raises(F.FIError) as e:
+        F.SiteIndex(gt, ic, badc)
+    assert e.value.code == F.FI_E_INVARIANT
+
+
 def test_errors(F):
     prog = P.c1()
     dp, gt = _gpu_golden(F, prog)
@@ -204,8 +221,12 @@ def test_scan_u64_and_rows(F, n):
     buf = torch.empty(nb, dtype=torch.uint8, device="cuda")
     cct = torch.from_numpy(cc).cuda()
     ict = torch.from_numpy(ic).cuda()
-    rc = L.fi_build_site_index(ict.data_ptr(), 3, cct.data_ptr(), n, buf.data_ptr(), torch.cuda.current_stream().cuda_stream)
+    st = F.DeviceStatus("cuda")
+    rc = L.fi_build_site_index(ict.data_ptr(), 3, cct.data_ptr(), n, buf.data_ptr(), st.ptr,
+                               torch.cuda.current_stream().cuda_stream)
     assert rc == 0
+    torch.cuda.synchronize()
+    assert int(st.t.item()) == 1 << F.FI_E_INVARIANT        # random rows violate the Table II identities
     torch.cuda.synchronize()
     b = buf.cpu().numpy()
     pk = b[: 4 * 64].view(np.uint64).reshape(4, 8)
