@@ -100,7 +100,8 @@ typedef struct {
 
 typedef struct {
     uint32_t before, after, mask, fault_pc;          /* mask actually applied (ZERO_VALUE: = before) */
-    uint8_t fault_kind /*0 none, 1 misaligned, 2 unmapped, 3 watchdog, 4 illegal pc*/, outcome, overflow, pad;
+    uint8_t fault_kind /*0 none, 1 misaligned, 2 unmapped, 3 watchdog, 4 illegal pc*/, outcome, overflow,
+            flags /* bit0 FI_POTENTIAL_DUE: fault not fatal under FI_UNCHECKED (f4) */;
     uint32_t n_faulty_stores;                        /* faulty stores after the site (words) */
 } fi_inj;                                            /* 24 B */
 
@@ -206,10 +207,17 @@ fi_status fi_inject(const fi_program* p, const uint8_t* image, const fi_trace* t
  * DUE if a fault/watchdog ended the replica; else SDC if the final value of any
  * output-buffer word differs bitwise from the golden run; else Masked.
  * Writes out[i].outcome and adds 1 to hist[group][bfm][outcome] (u64 [8][4][3]).
- * Replicas with overflow set get outcome 0xFF and FI_E_CAPACITY in dev_status. */
+ * Replicas with overflow set get outcome 0xFF and FI_E_CAPACITY in dev_status.
+ * flags & FI_UNCHECKED (§8 row f4, "potential DUE" [PAPER.md:195-196], [PAPER.md:208]):
+ * the application does not check CUDA errors, so a memory fault or illegal
+ * instruction only ends the faulting warp — its earlier stores stand — and the
+ * replica is classified SDC/Masked by its outputs with FI_POTENTIAL_DUE set;
+ * a hang (watchdog) stays DUE. */
+#define FI_UNCHECKED 1u
+#define FI_POTENTIAL_DUE 1u
 fi_status fi_classify(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
                       uint32_t n, fi_inj* out, const fi_store* log, uint32_t log_cap, uint64_t* hist,
-                      uint32_t* dev_status, void* stream);
+                      uint32_t flags, uint32_t* dev_status, void* stream);
 
 /* Table II parameter file, one parameter per line in Table II order
  * [PAPER.md:88]: arch state id, bit-flip model, kernel name, kernel count,

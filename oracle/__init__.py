@@ -31,6 +31,8 @@ G_FP64, G_FP32, G_LD, G_PR, G_NODEST, G_OTHERS, G_GPPR, G_GP = range(8)
 GROUP_NAMES = ["G_FP64", "G_FP32", "G_LD", "G_PR", "G_NODEST", "G_OTHERS", "G_GPPR", "G_GP"]
 MASKED, SDC, DUE = 0, 1, 2
 MODE_FULL, MODE_WARP_LOCAL = 0, 1
+UNCHECKED = 0x100          # OR into mode: potential-DUE semantics (row f4)
+POTENTIAL_DUE = 1          # inj["flags"] bit
 
 RECORD_DTYPE = np.dtype([("instance", "<u4"), ("insn", "<u4"), ("active", "<u4"), ("pred", "<u4")])
 SITE_DTYPE = np.dtype([
@@ -41,7 +43,8 @@ SITE_DTYPE = np.dtype([
     ("n_elig", "u1"), ("pad", "u1"),
 ])
 INJ_DTYPE = np.dtype([("before", "<u4"), ("after", "<u4"), ("mask", "<u4"), ("fault_pc", "<u4"),
-                      ("fault_kind", "u1"), ("outcome", "u1"), ("pad", "u1", 2), ("n_faulty_stores", "<u4")])
+                      ("fault_kind", "u1"), ("outcome", "u1"), ("flags", "u1"), ("pad", "u1"),
+                      ("n_faulty_stores", "<u4")])
 assert SITE_DTYPE.itemsize == 64 and INJ_DTYPE.itemsize == 24
 
 

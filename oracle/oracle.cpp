@@ -507,12 +507,18 @@ void warp_coords(const orc_instance& in, uint32_t w, uint32_t& cta, uint32_t& wi
 struct FullRun {
     std::vector<uint8_t> mem;
     int fault = 0; uint32_t fault_pc = 0;
+    int pdue = 0; uint32_t pdue_pc = 0;        // unchecked mode: first non-fatal fault (potential DUE)
     uint64_t n_faulty_stores = 0;
 };
 
+// `unchecked` (§8 row f4): the application does not check
+// CUDA errors, so a memory fault or illegal instruction only ends the faulting
+// warp (its earlier stores stand) and the run goes on; a hang (watchdog) is
+// still detected by the monitor and ends the run.
 void run_program(const Golden* G, const Prog& P, Hook* hook, uint32_t hook_warp, int n_threads, FullRun& out,
                  std::vector<uint64_t>* wlen_out, std::vector<uint64_t>* wcounts, bool keep_trace,
-                 std::vector<std::vector<orc_record>>* wtraces, uint64_t* n_gstores, std::string* err) {
+                 std::vector<std::vector<orc_record>>* wtraces, uint64_t* n_gstores, std::string* err,
+                 bool unchecked = false) {
     out.mem.assign(P.p.init_image, P.p.init_image + P.p.image_bytes);
     for (uint32_t k = 0; k < P.p.n_inst && !out.fault; ++k) {
         const orc_instance& in = P.p.inst[k];
@@ -533,7 +539,14 @@ void run_program(const Golden* G, const Prog& P, Hook* hook, uint32_t hook_warp,
         };
         if (hook) for (uint32_t i = 0; i < nw; ++i) body(i);       // replica-level parallelism instead
         else parallel_for(nw, n_threads, body);
-        for (uint32_t i = 0; i < nw; ++i) if (rr[i].fault && !out.fault) { out.fault = rr[i].fault; out.fault_pc = rr[i].fault_pc; }
+        for (uint32_t i = 0; i < nw; ++i) {
+            if (!rr[i].fault) continue;
+            if (unchecked && rr[i].fault != 3) {
+                if (!out.pdue) { out.pdue = rr[i].fault; out.pdue_pc = rr[i].fault_pc; }
+                continue;
+            }
+            if (!out.fault) { out.fault = rr[i].fault; out.fault_pc = rr[i].fault_pc; }
+        }
         if (out.fault) {
             if (err) *err = "fault in golden run at instance " + std::to_string(k) + " pc " + std::to_string(out.fault_pc);
             break;
@@ -756,9 +769,12 @@ extern "C" int orc_locate(void* h, int group, const uint64_t* s, uint32_t n, orc
 // buffer with the golden run bitwise (C-12), DUE taking precedence (Table V).
 // WARP_LOCAL (single-instance programs): re-run only warp w, faulty and golden,
 // and compare the final value of every address either run stored to (C-14).
+// ORC_UNCHECKED in `mode` selects the potential-DUE semantics of row f4.
 extern "C" int orc_inject(void* h, const orc_site* sites, uint32_t n, int mode, int n_threads, orc_inj* out) {
     Golden* G = (Golden*)h;
     const Prog& P = G->P;
+    const bool unchecked = mode & ORC_UNCHECKED;
+    mode &= ~ORC_UNCHECKED;
     if (mode == ORC_MODE_WARP_LOCAL && !P.single_instance()) mode = ORC_MODE_FULL;
     std::atomic<int> status{0};
     std::mutex mu;
@@ -769,11 +785,12 @@ extern "C" int orc_inject(void* h, const orc_site* sites, uint32_t n, int mode, 
         Hook hk;
         hk.on = true; hk.step = S.step; hk.lane = S.lane; hk.kind = S.dst_kind; hk.reg = S.dst_reg;
         hk.bfm = S.bfm; hk.mask = S.mask; hk.pc = S.pc;
-        int fault = 0; uint32_t fpc = 0; bool sdc = false;
+        int fault = 0, pdue = 0; uint32_t fpc = 0; bool sdc = false;
         if (mode == ORC_MODE_FULL) {
             FullRun fr;
-            run_program(G, P, &hk, S.warp, 1, fr, nullptr, nullptr, false, nullptr, nullptr, nullptr);
+            run_program(G, P, &hk, S.warp, 1, fr, nullptr, nullptr, false, nullptr, nullptr, nullptr, unchecked);
             fault = fr.fault; fpc = fr.fault_pc;
+            if (!fault && fr.pdue) { pdue = fr.pdue; fpc = fr.pdue_pc; }
             R.n_faulty_stores = (uint32_t)fr.n_faulty_stores;
             if (!fault) sdc = output_differs(P, fr.mem, G->final_mem);
         } else {
@@ -784,6 +801,7 @@ extern "C" int orc_inject(void* h, const orc_site* sites, uint32_t n, int mode, 
             std::vector<StoreW> fst, gst;
             WarpResult fr = run_warp(P, pre, S.instance, cta, wic, &hk, 10 * G->wlen[S.warp] + 1024, &fst, nullptr, nullptr);
             fault = fr.fault; fpc = fr.fault_pc;
+            if (unchecked && fault && fault != 3) { pdue = fault; fault = 0; }   // the warp just stops (f4)
             R.n_faulty_stores = (uint32_t)fst.size();
             if (!fault) {
                 run_warp(P, pre, S.instance, cta, wic, nullptr, UINT64_MAX, &gst, nullptr, nullptr);
@@ -803,7 +821,8 @@ extern "C" int orc_inject(void* h, const orc_site* sites, uint32_t n, int mode, 
             status = 4;
         }
         R.before = hk.before; R.after = hk.after; R.mask = hk.applied_mask;
-        R.fault_kind = (uint8_t)fault; R.fault_pc = fpc;
+        R.fault_kind = (uint8_t)(fault ? fault : pdue); R.fault_pc = fpc;
+        R.flags = pdue ? ORC_POTENTIAL_DUE : 0;
         R.outcome = fault ? ORC_DUE : (sdc ? ORC_SDC : ORC_MASKED);
     });
     return status;

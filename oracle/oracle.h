@@ -52,14 +52,15 @@ typedef struct {
 
 typedef struct {
     uint32_t before, after, mask, fault_pc;
-    uint8_t fault_kind, outcome, pad[2];
+    uint8_t fault_kind, outcome, flags /* bit0: potential DUE (f4) */, pad;
     uint32_t n_faulty_stores;
 } orc_inj;                                            /* 24 B */
 
 /* groups (Table II order, C-1) and outcomes (Table V) */
 enum { ORC_G_FP64 = 0, ORC_G_FP32, ORC_G_LD, ORC_G_PR, ORC_G_NODEST, ORC_G_OTHERS, ORC_G_GPPR, ORC_G_GP };
 enum { ORC_MASKED = 0, ORC_SDC = 1, ORC_DUE = 2 };
-enum { ORC_MODE_FULL = 0, ORC_MODE_WARP_LOCAL = 1 };
+enum { ORC_MODE_FULL = 0, ORC_MODE_WARP_LOCAL = 1, ORC_UNCHECKED = 0x100 /* f4 potential-DUE semantics */ };
+enum { ORC_POTENTIAL_DUE = 1 };
 
 /* status: 0 ok; 1 arg; 2 empty group; 3 not injectable; 4 program error */
 const char* orc_error(void* h);

@@ -92,7 +92,7 @@ k_inject(EmuProg P, const uint8_t* img, const uint64_t* __restrict__ warp_off, c
     if (lane == 0) {
         fi_inj r;
         r.before = o.before; r.after = o.after; r.mask = o.mask; r.fault_pc = o.fault_pc;
-        r.fault_kind = (uint8_t)o.fault; r.outcome = 0; r.overflow = o.nstore > cap; r.pad = 0;
+        r.fault_kind = (uint8_t)o.fault; r.outcome = 0; r.overflow = o.nstore > cap; r.flags = 0;
         r.n_faulty_stores = o.nstore;
         out[i] = r;
         if (!o.fired || o.bad) FI_DEV_ERR(status, FI_E_SITE);
@@ -106,7 +106,7 @@ struct ClsArgs {
     const fi_store* gstore; const uint64_t* gstore_off;
     const fi_site* sites; fi_inj* inj; uint32_t n;
     const fi_store* log; uint32_t cap;
-    uint64_t* hist; uint32_t* status;
+    uint64_t* hist; uint32_t flags; uint32_t* status;
 };
 
 __device__ __forceinline__ uint32_t buf_of(const ClsArgs& A, uint64_t va) {
@@ -135,7 +135,9 @@ __global__ void __launch_bounds__(kClsWarps * 32) k_classify(const ClsArgs A) {
     const fi_site S = A.sites[i];
     const fi_inj R = A.inj[i];
     uint32_t outcome;
-    if (R.fault_kind) {
+    // f4: under FI_UNCHECKED only a hang is fatal; other faults just ended the warp
+    const bool pdue = (A.flags & FI_UNCHECKED) && R.fault_kind && R.fault_kind != 3;
+    if (R.fault_kind && !pdue) {
         outcome = FI_DUE;
     } else if (R.overflow) {
         outcome = 0xFF;
@@ -198,6 +200,7 @@ __global__ void __launch_bounds__(kClsWarps * 32) k_classify(const ClsArgs A) {
     }
     if (lane == 0) {
         A.inj[i].outcome = (uint8_t)outcome;
+        A.inj[i].flags = pdue ? FI_POTENTIAL_DUE : 0;
         if (outcome == 0xFF) FI_DEV_ERR(A.status, FI_E_CAPACITY);
         else atomicAdd((unsigned long long*)&A.hist[((uint32_t)S.group * 4 + S.bfm) * 3 + outcome], 1ull);
     }
@@ -239,11 +242,11 @@ extern "C" fi_status fi_inject(const fi_program* p, const uint8_t* image, const 
 
 extern "C" fi_status fi_classify(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
                                  uint32_t n, fi_inj* out, const fi_store* log, uint32_t log_cap, uint64_t* hist,
-                                 uint32_t* dev_status, void* stream) {
+                                 uint32_t flags, uint32_t* dev_status, void* stream) {
     if (!p || !image || !t || !sites || !out || !hist || !dev_status || !p->aux) return FI_E_ARG;
     if (n == 0) return FI_OK;
     const EmuProg P = make_emu_prog(p);
-    ClsArgs A{p->buf, P.gran, image, t->gstore, t->gstore_off, sites, out, n, log, log_cap, hist, dev_status};
+    ClsArgs A{p->buf, P.gran, image, t->gstore, t->gstore_off, sites, out, n, log, log_cap, hist, flags, dev_status};
     k_classify<<<(n + kClsWarps - 1) / kClsWarps, kClsWarps * 32, 0, (cudaStream_t)stream>>>(A);
     return launch_status();
 }

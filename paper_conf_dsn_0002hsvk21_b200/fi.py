@@ -21,6 +21,7 @@ LIB_PATH = os.path.join(HERE, "libfi.so")
 FI_OK, FI_E_ARG, FI_E_EMPTY_GROUP, FI_E_NOT_INJECTABLE, FI_E_PROGRAM, FI_E_CUDA, FI_E_SITE = 0, 1, 2, 3, 4, 5, 6
 FI_E_CAPACITY, FI_E_INVARIANT = 8, 9
 FI_CHUNK = 1024
+FI_UNCHECKED, FI_POTENTIAL_DUE = 1, 1
 G_FP64, G_FP32, G_LD, G_PR, G_NODEST, G_OTHERS, G_GPPR, G_GP = range(8)
 GROUP_NAMES = ["G_FP64", "G_FP32", "G_LD", "G_PR", "G_NODEST", "G_OTHERS", "G_GPPR", "G_GP"]
 BFM_NAMES = ["FLIP_SINGLE_BIT", "FLIP_TWO_BITS", "RANDOM_VALUE", "ZERO_VALUE"]
@@ -34,7 +35,7 @@ SITE_DTYPE = np.dtype([
     ("n_elig", "u1"), ("pad", "u1"),
 ])
 INJ_DTYPE = np.dtype([("before", "<u4"), ("after", "<u4"), ("mask", "<u4"), ("fault_pc", "<u4"),
-                      ("fault_kind", "u1"), ("outcome", "u1"), ("overflow", "u1"), ("pad", "u1"),
+                      ("fault_kind", "u1"), ("outcome", "u1"), ("overflow", "u1"), ("flags", "u1"),
                       ("n_faulty_stores", "<u4")])
 RECORD_DTYPE = np.dtype([("instance", "<u4"), ("insn", "<u4"), ("active", "<u4"), ("pred", "<u4")])
 STORE_DTYPE = np.dtype([("va", "<u8"), ("value", "<u4"), ("step", "<u4")])
@@ -103,7 +104,7 @@ def lib():
             "fi_select_sites": (st, [vp, vp, vp, vp, u32, u64, vp, vp, u64, u32, vp, vp, vp]),
             "fi_inject_workspace": (sz, [u32]),
             "fi_inject": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, sz, vp, vp]),
-            "fi_classify": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, vp, vp]),
+            "fi_classify": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, u32, vp, vp]),
             "fi_write_params_txt": (st, [vp, C.c_char_p, C.c_char_p, sz]),
         }
         for name, (res, args) in sig.items():
@@ -352,14 +353,16 @@ def inject(gt: GoldenTrace, sites: torch.Tensor, n: int, log_cap: int, out: torc
 
 
 def classify(gt: GoldenTrace, sites: torch.Tensor, n: int, out: torch.Tensor, log: torch.Tensor, log_cap: int,
-             hist: torch.Tensor | None = None, status: DeviceStatus | None = None) -> torch.Tensor:
-    """fi_classify (K5): fills out[].outcome, accumulates hist[8][4][3]."""
+             hist: torch.Tensor | None = None, status: DeviceStatus | None = None,
+             unchecked: bool = False) -> torch.Tensor:
+    """fi_classify (K5): fills out[].outcome, accumulates hist[8][4][3].
+    unchecked=True: potential-DUE semantics (FI_UNCHECKED, row f4)."""
     dev = gt.dp.device
     if hist is None:
         hist = torch.zeros((8, 4, 3), dtype=torch.int64, device=dev)
     st = status or DeviceStatus(dev)
     _check(lib().fi_classify(C.byref(gt.dp.c), _p(gt.image), C.byref(gt.c), _p(sites), n, _p(out), _p(log), log_cap,
-                             _p(hist), st.ptr, _stream()), "fi_classify")
+                             _p(hist), FI_UNCHECKED if unchecked else 0, st.ptr, _stream()), "fi_classify")
     if status is None:
         st.check("fi_classify")
     return hist

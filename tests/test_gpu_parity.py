@@ -64,7 +64,7 @@ def test_fuzz_trace_and_image(F, seed):
     assert np.array_equal(ic.cpu().numpy().astype(np.uint64), g.counts())
 
 
-def _campaign_parity(F, prog, seed, groups, bfms, n, mode, ckpt="auto"):
+def _campaign_parity(F, prog, seed, groups, bfms, n, mode, ckpt="auto", unchecked=False):
     g = O.Golden(prog)
     dp, gt = _gpu_golden(F, prog, ckpt)
     assert np.array_equal(_trace_np(F, gt), g.trace())
@@ -78,9 +78,10 @@ def _campaign_parity(F, prog, seed, groups, bfms, n, mode, ckpt="auto"):
     _assert_sites_equal(gs, os_)
     cap = F.log_capacity(gt)
     out, log = F.inject(gt, sites, n, cap)
-    hist = F.classify(gt, sites, n, out, log, cap)
+    hist = F.classify(gt, sites, n, out, log, cap, unchecked=unchecked)
     gi = F.as_numpy(out, F.INJ_DTYPE, n)
-    oi = g.inject(os_, mode)
+    oi = g.inject(os_, mode | (O.UNCHECKED if unchecked else 0))
+    assert (gi["flags"] == oi["flags"]).all()
     for f in ("before", "after", "mask", "fault_kind", "outcome"):
         bad = np.flatnonzero(gi[f] != oi[f])
         assert bad.size == 0, f"{f}: replica {bad[0]} gpu {gi[bad[0]]} oracle {oi[bad[0]]} site {os_[bad[0]]}"
@@ -110,6 +111,15 @@ def test_fuzz_campaign_parity(F, seed):
     # odd checkpoint intervals make replicas restart mid-divergence (seed % 3 == 0: no checkpoints)
     _campaign_parity(F, prog, 0xABC0 + seed, [F.G_GPPR, F.G_GP, F.G_PR, F.G_FP32, F.G_FP64, F.G_OTHERS][: 1 + seed % 6],
                      [0, 1, 2, 3], 300, O.MODE_FULL, ckpt=[0, 5, 13][seed % 3])
+
+
+@pytest.mark.parametrize("maker,mode", [(P.c1, O.MODE_FULL), (lambda: P.vector_add(n=1000), O.MODE_FULL),
+                                        (lambda: P.c2(full=False), O.MODE_WARP_LOCAL),
+                                        (lambda: P.fuzz_program(7, n_ops=90), O.MODE_FULL)])
+def test_unchecked_potential_due_parity(F, maker, mode):
+    """Row f4: potential-DUE semantics (FI_UNCHECKED) — outcome, flags and fault kinds match the oracle."""
+    gi, oi = _campaign_parity(F, maker(), 0xF4, [F.G_GP, F.G_OTHERS], [0, 1, 2, 3], 400, mode, unchecked=True)
+    assert not (gi["outcome"][gi["flags"] == 1] == F.DUE).any()
 
 
 def test_mini_c2_parity_checkpoints(F):

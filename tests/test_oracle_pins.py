@@ -322,6 +322,23 @@ def test_outcome_special_cases():
         assert r["after"] == 0 and r["outcome"] == O.MASKED
 
 
+def test_unchecked_fault_is_potential_due():
+    """Row f4 [PAPER.md:208]: with unchecked errors an unmapped load only ends the
+    faulting warp; its 32 outputs of c are never written (stay 0) -> SDC, flagged
+    potential DUE.  A hang stays DUE."""
+    prog = P.c1()
+    g = O.Golden(prog)
+    for mode in (O.MODE_FULL, O.MODE_WARP_LOCAL):
+        r = g.inject(_site(g, 8, warp=3, reg=5, mask=1 << 20), mode | O.UNCHECKED)[0]
+        assert r["outcome"] == O.SDC and r["flags"] == O.POTENTIAL_DUE and r["fault_kind"] == 2
+        r = g.inject(_site(g, 8, warp=3, reg=5, mask=1 << 20), mode)[0]
+        assert r["outcome"] == O.DUE and r["flags"] == 0
+    hang = P.sgemm(128, 128, 4)
+    gh = O.Golden(hang)
+    r = gh.inject(_site(gh, 87, reg=P.KCNT, mask=1 << 30), O.MODE_FULL | O.UNCHECKED)[0]
+    assert r["outcome"] == O.DUE and r["fault_kind"] == 3 and r["flags"] == 0
+
+
 def test_dead_register_is_masked():
     # MOV R5 <- 7 that nothing reads, inside an otherwise C1-like kernel
     s = isa.Asm()
