@@ -277,10 +277,13 @@ def fuzz_program(seed: int, n_ops: int = 120, grid: int = 2, block: int = 80, lo
     return pb.build(config="fuzz", seed=seed)
 
 
-def multi_instance_chain(n_inst: int = 3, n: int = 256, block: int = 64, seed: int = 77) -> Program:
+def multi_instance_chain(n_inst: int = 3, n: int = 256, block: int = 64, seed: int = 77, shrink: int = 0) -> Program:
     """y_{i+1} = y_i * s + x (FP32) over n_inst launches of one static kernel, each
     writing a new SSA buffer version.  Exercises multi-instance profiling,
-    kernel_count, and (oracle full mode) downstream propagation."""
+    kernel_count, and (oracle full mode) downstream propagation.  With shrink > 0
+    launch i only updates the first n - shrink*i elements (the rest exit early),
+    so instances of the same static kernel have different counts (approximate
+    profiling, PAPER.md:80)."""
     s = Asm()
     s.s2r(0, isa.SR_TID)
     s.s2r(1, isa.SR_CTAID)
@@ -309,6 +312,6 @@ def multi_instance_chain(n_inst: int = 3, n: int = 256, block: int = 64, seed: i
     grid = (n + block - 1) // block
     for i in range(n_inst):
         ynew = pb.add_buffer(f"y{i + 1}", 4 * n, writer=i, output=(i == n_inst - 1), dtype=isa.DT_F32)
-        pb.add_instance(k, grid, block, ptr_words(x) + ptr_words(y) + ptr_words(ynew) + [n, isa.f32_bits(0.5)])
+        pb.add_instance(k, grid, block, ptr_words(x) + ptr_words(y) + ptr_words(ynew) + [n - shrink * i, isa.f32_bits(0.5)])
         y = ynew
     return pb.build(config="chain", n_inst=n_inst, n=n)

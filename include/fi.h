@@ -43,7 +43,9 @@ typedef enum { FI_G_FP64 = 0, FI_G_FP32 = 1, FI_G_LD = 2, FI_G_PR = 3, FI_G_NODE
 /* Table II bit-flip models [PAPER.md:105-109], 0-based (C-1) */
 typedef enum { FI_FLIP_SINGLE_BIT = 0, FI_FLIP_TWO_BITS = 1, FI_RANDOM_VALUE = 2, FI_ZERO_VALUE = 3 } fi_bfm;
 /* Table V outcomes [PAPER.md:184-196] */
-typedef enum { FI_MASKED = 0, FI_SDC = 1, FI_DUE = 2 } fi_outcome;
+typedef enum { FI_MASKED = 0, FI_SDC = 1, FI_DUE = 2,
+               FI_NOT_INJECTED = 3 /* approximate profile named a site the instance does not have (C-17) */ } fi_outcome;
+#define FI_NOPS 32                                   /* opcode slots of the per-opcode profile */
 
 /* ---- program ------------------------------------------- */
 typedef struct { uint8_t op, guard, d0, d1, a, b, c, mod; uint32_t imm, ext; } fi_insn;          /* 16 B */
@@ -88,8 +90,10 @@ typedef struct {
     uint64_t s, instruction_count;                   /* s in [0, N_g) (C-4); instruction_count = s - P_k[instance] */
     uint32_t instance, kernel_id, kernel_count, warp, step, thread;   /* kernel_count: ordinal of the instance among its static kernel's */
     uint32_t pc, u_dst, u_bit, mask;                 /* mask = Table II pattern (0 for ZERO_VALUE: resolved at injection) */
-    uint8_t lane, group, bfm, slot, dst_kind /*0 GP, 1 PR*/, dst_reg, n_elig, pad;
+    uint8_t lane, group, bfm, slot, dst_kind /*0 GP, 1 PR*/, dst_reg, n_elig,
+            flags /* bit0 FI_SITE_NOT_INJECTED */;
 } fi_site;                                           /* 64 B */
+#define FI_SITE_NOT_INJECTED 1u
 
 typedef struct {
     uint64_t seed;                                   /* campaign seed (Philox key) */
@@ -117,7 +121,7 @@ uint32_t fi_program_regs(const fi_insn* code_host, uint32_t n_code);
 /* Prepared program data, built once per program into `aux` (then set
  * p->aux = aux): the granule map (buffer id per 256-B granule of the image,
  * for the C-15 access check) and the pre-decoded code the emulator executes. */
-size_t fi_program_aux_bytes(uint64_t image_bytes, uint32_t n_code);
+size_t fi_program_aux_bytes(uint64_t image_bytes, uint32_t n_code, uint32_t n_inst);
 fi_status fi_program_prepare(const fi_program* p, void* aux, void* stream);
 
 /* Golden run, pass 1 — PAPER.md:72 step (1)/(4) golden state.  Executes the
@@ -161,6 +165,24 @@ fi_status fi_profile(const fi_trace* t, uint64_t rec_begin, uint64_t rec_end, ui
                      uint64_t* inst_counts, uint32_t* chunk_counts, void* stream);
 #define FI_CHUNK 1024
 
+/* §8 row f1 — per-opcode profile, "a profile containing one line
+ * for every dynamic kernel and the total dynamic instruction counts for every
+ * opcode in every thread": op_counts[k][op] = sum over the records of instance k
+ * in [rec_begin, rec_end) with opcode op of popc(active & pred) (u64 [n_inst][32],
+ * zeroed by the call).  The executed-opcode set [PAPER.md:82] is its nonzero
+ * columns. */
+fi_status fi_profile_opcodes(const fi_trace* t, uint64_t rec_begin, uint64_t rec_end, uint32_t n_inst,
+                             uint64_t* op_counts, void* stream);
+
+/* §8 row f1 — approximate profiling: "only counts the dynamic
+ * instructions in the first instance of every static kernel and assumes that the
+ * instruction counts for subsequent instances of the same static kernel are the
+ * same".  Fills inst_counts[n_inst][8] that way (synchronizes once to upload the
+ * first-instance table).  Scratch: fi_profile_approx_workspace() bytes. */
+size_t fi_profile_approx_workspace(uint32_t n_kern, uint32_t n_inst);
+fi_status fi_profile_approx(const fi_program* p, const fi_trace* t, uint64_t* inst_counts, void* ws,
+                            size_t ws_bytes, void* stream);
+
 /* K2 — site index ("1..N" of PAPER.md:78 as prefix sums): exclusive prefix
  * sums P_k[n_inst+1][8] of inst_counts and P_t[T+1][8] of the chunk counts
  * summed per tile of 64 chunks (T = ceil(n_chunks/64)), both u64 with the
@@ -173,6 +195,10 @@ fi_status fi_profile(const fi_trace* t, uint64_t rec_begin, uint64_t rec_end, ui
 size_t fi_site_index_bytes(uint32_t n_inst, uint64_t n_chunks);
 fi_status fi_build_site_index(const uint64_t* inst_counts, uint32_t n_inst, const uint32_t* chunk_counts,
                               uint64_t n_chunks, void* index, uint32_t* dev_status, void* stream);
+/* The instance level alone (P_k + a3 identities), e.g. over approximate counts;
+ * `index` sized fi_site_index_bytes(n_inst, 0). */
+fi_status fi_build_instance_index(const uint64_t* inst_counts, uint32_t n_inst, void* index, uint32_t* dev_status,
+                                  void* stream);
 /* Totals N_g (host, synchronizes): copies P_k[n_inst][*] */
 fi_status fi_site_totals(const void* index, uint32_t n_inst, uint64_t totals_host[8], void* stream);
 
@@ -186,6 +212,16 @@ fi_status fi_select_sites(const fi_program* p, const fi_trace* t, const uint32_t
                           uint32_t n_inst, uint64_t n_chunks, const uint64_t totals_host[8],
                           const fi_schedule* sched, uint64_t j0, uint32_t n, fi_site* sites, uint32_t* dev_status,
                           void* stream);
+
+/* K3 with an approximate profile (row f1): s is drawn over the approximate
+ * totals and mapped to (instance k, instruction_count) by the approximate P_k;
+ * the site is then located like NVBitFI's injector does at run time — by
+ * counting group-g lane-instructions through instance k's records.  When
+ * instruction_count >= the instance's real count the site gets
+ * FI_SITE_NOT_INJECTED (C-17); K4/K5 skip it (outcome FI_NOT_INJECTED). */
+fi_status fi_select_sites_approx(const fi_program* p, const fi_trace* t, const void* index, uint32_t n_inst,
+                                 const uint64_t totals_host[8], const fi_schedule* sched, uint64_t j0, uint32_t n,
+                                 fi_site* sites, uint32_t* dev_status, void* stream);
 
 /* K4 — inject: one CUDA warp re-executes the site's
  * synthetic warp over the golden final image — from its first instruction, or
@@ -212,12 +248,20 @@ fi_status fi_inject(const fi_program* p, const uint8_t* image, const fi_trace* t
  * the application does not check CUDA errors, so a memory fault or illegal
  * instruction only ends the faulting warp — its earlier stores stand — and the
  * replica is classified SDC/Masked by its outputs with FI_POTENTIAL_DUE set;
- * a hang (watchdog) stays DUE. */
+ * a hang (watchdog) stays DUE.
+ * Multi-instance programs (K7): the faulty warp's effect in its instance is
+ * propagated through the later instances — every later instance that references
+ * a buffer holding a dirty word is re-executed against the replica's faulty
+ * overlay, its stores diffed against its golden store log — and the replica is
+ * classified on the whole program's outputs (PAPER.md:72 step (4), :206).
+ * Scratch: fi_classify_workspace(n_inst, n, log_cap) bytes (0 for one instance).
+ * Replicas whose overlay or update lists overflow get outcome 0xFF + FI_E_CAPACITY. */
 #define FI_UNCHECKED 1u
 #define FI_POTENTIAL_DUE 1u
+size_t fi_classify_workspace(uint32_t n_inst, uint32_t n, uint32_t log_cap);
 fi_status fi_classify(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
                       uint32_t n, fi_inj* out, const fi_store* log, uint32_t log_cap, uint64_t* hist,
-                      uint32_t flags, uint32_t* dev_status, void* stream);
+                      uint32_t flags, void* ws, size_t ws_bytes, uint32_t* dev_status, void* stream);
 
 /* Table II parameter file, one parameter per line in Table II order
  * [PAPER.md:88]: arch state id, bit-flip model, kernel name, kernel count,

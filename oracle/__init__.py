@@ -29,7 +29,7 @@ SRC = [os.path.join(HERE, "oracle.cpp"), os.path.join(HERE, "oracle.h")]
 
 G_FP64, G_FP32, G_LD, G_PR, G_NODEST, G_OTHERS, G_GPPR, G_GP = range(8)
 GROUP_NAMES = ["G_FP64", "G_FP32", "G_LD", "G_PR", "G_NODEST", "G_OTHERS", "G_GPPR", "G_GP"]
-MASKED, SDC, DUE = 0, 1, 2
+MASKED, SDC, DUE, NOT_INJECTED = 0, 1, 2, 3
 MODE_FULL, MODE_WARP_LOCAL = 0, 1
 UNCHECKED = 0x100          # OR into mode: potential-DUE semantics (row f4)
 POTENTIAL_DUE = 1          # inj["flags"] bit
@@ -40,7 +40,7 @@ SITE_DTYPE = np.dtype([
     ("instance", "<u4"), ("kernel_id", "<u4"), ("kernel_count", "<u4"), ("warp", "<u4"),
     ("step", "<u4"), ("thread", "<u4"), ("pc", "<u4"), ("u_dst", "<u4"), ("u_bit", "<u4"), ("mask", "<u4"),
     ("lane", "u1"), ("group", "u1"), ("bfm", "u1"), ("slot", "u1"), ("dst_kind", "u1"), ("dst_reg", "u1"),
-    ("n_elig", "u1"), ("pad", "u1"),
+    ("n_elig", "u1"), ("flags", "u1"),
 ])
 INJ_DTYPE = np.dtype([("before", "<u4"), ("after", "<u4"), ("mask", "<u4"), ("fault_pc", "<u4"),
                       ("fault_kind", "u1"), ("outcome", "u1"), ("flags", "u1"), ("pad", "u1"),
@@ -96,6 +96,9 @@ def lib():
             L.orc_count_warps.argtypes = [C.POINTER(_Program), u32, u32, i32, vp]
             L.orc_select.argtypes = [vp, u64, vp, u32, vp, u32, u64, u32, vp]
             L.orc_locate.argtypes = [vp, i32, vp, u32, vp]
+            L.orc_opcode_counts.argtypes = [vp, vp]
+            L.orc_approx_counts.argtypes = [vp, vp]
+            L.orc_select_approx.argtypes = [vp, u64, vp, u32, vp, u32, u64, u32, vp]
             L.orc_inject.argtypes = [vp, vp, u32, i32, i32, vp]
             L.orc_warp_site_rank.argtypes = [C.POINTER(_Program), u32, i32, u32, u32, C.POINTER(u64), C.POINTER(u64)]
             L.orc_inject_local.argtypes = [C.POINTER(_Program), vp, u32, i32, vp, vp]
@@ -184,6 +187,26 @@ class Golden:
         b = np.asarray(bfms, dtype=np.uint8)
         out = np.zeros(n, dtype=SITE_DTYPE)
         rc = lib().orc_select(self.h, seed, _ptr(g), len(g), _ptr(b), len(b), j0, n, _ptr(out))
+        if rc:
+            raise OracleError(rc, lib().orc_error(self.h).decode())
+        return out
+
+    def opcode_counts(self) -> np.ndarray:
+        out = np.zeros((len(self.prog.instances), 32), dtype=np.uint64)
+        if lib().orc_opcode_counts(self.h, _ptr(out)):
+            raise RuntimeError("trace not kept")
+        return out
+
+    def approx_counts(self) -> np.ndarray:
+        out = np.zeros((len(self.prog.instances), 8), dtype=np.uint64)
+        lib().orc_approx_counts(self.h, _ptr(out))
+        return out
+
+    def select_approx(self, seed: int, groups, bfms, j0: int, n: int) -> np.ndarray:
+        g = np.asarray(groups, dtype=np.uint8)
+        b = np.asarray(bfms, dtype=np.uint8)
+        out = np.zeros(n, dtype=SITE_DTYPE)
+        rc = lib().orc_select_approx(self.h, seed, _ptr(g), len(g), _ptr(b), len(b), j0, n, _ptr(out))
         if rc:
             raise OracleError(rc, lib().orc_error(self.h).decode())
         return out
@@ -322,5 +345,6 @@ def histogram(sites: np.ndarray, inj: np.ndarray) -> np.ndarray:
     """Outcome histogram [group][bfm][M,S,D] (u64), by plain counting."""
     h = np.zeros((8, 4, 3), dtype=np.uint64)
     for s, r in zip(sites, inj):
-        h[int(s["group"]), int(s["bfm"]), int(r["outcome"])] += 1
+        if int(r["outcome"]) < 3:                  # not-injected sites are not outcomes
+            h[int(s["group"]), int(s["bfm"]), int(r["outcome"])] += 1
     return h

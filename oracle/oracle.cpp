@@ -754,6 +754,104 @@ extern "C" int orc_select(void* h, uint64_t seed, const uint8_t* groups, uint32_
     return enumerate_sites(G, n, out);
 }
 
+// Row f1, per-opcode profile ("counts for every opcode"): the plain
+// sum of popc(active & pred) per (instance, opcode) over the trace.
+extern "C" int orc_opcode_counts(void* h, uint64_t* out /*[n_inst][32]*/) {
+    Golden* G = (Golden*)h;
+    if (!G->kept) return 1;
+    std::fill(out, out + (size_t)G->P.p.n_inst * 32, 0);
+    for (const orc_record& R : G->trace)
+        out[(size_t)R.instance * 32 + ((R.insn >> 16) & 31)] += (uint64_t)__builtin_popcount(R.active & R.pred);
+    return 0;
+}
+
+// Row f1, approximate profiling: every instance is assumed to have
+// the counts of the first instance of its static kernel.
+static void approx_counts(const Golden* G, std::vector<uint64_t>& a) {
+    const Prog& P = G->P;
+    a.assign((size_t)P.p.n_inst * 8, 0);
+    std::vector<int64_t> first(P.p.n_kern, -1);
+    for (uint32_t k = 0; k < P.p.n_inst; ++k) {
+        uint32_t kern = P.p.inst[k].kernel;
+        if (first[kern] < 0) first[kern] = k;
+        for (int g = 0; g < 8; ++g) a[8 * (size_t)k + g] = G->counts[8 * (size_t)first[kern] + g];
+    }
+}
+
+extern "C" int orc_approx_counts(void* h, uint64_t* out) {
+    std::vector<uint64_t> a;
+    approx_counts((Golden*)h, a);
+    std::copy(a.begin(), a.end(), out);
+    return 0;
+}
+
+// Selection over an approximate profile: s is drawn over the approximate totals
+// and read as (instance k, instruction_count) in launch order; the site is the
+// instruction_count-th group-g site of instance k itself (C-3), or does not
+// exist (C-17: flags = 1, "not injected").
+extern "C" int orc_select_approx(void* h, uint64_t seed, const uint8_t* groups, uint32_t n_groups,
+                                 const uint8_t* bfms, uint32_t n_bfms, uint64_t j0, uint32_t n, orc_site* out) {
+    Golden* G = (Golden*)h;
+    const Prog& P = G->P;
+    if (!G->kept) { G->err = "selection needs keep_trace"; return 1; }
+    if (n_groups == 0 || n_bfms == 0) { G->err = "empty schedule"; return 1; }
+    std::vector<uint64_t> a;
+    approx_counts(G, a);
+    std::vector<uint64_t> total(8, 0);
+    for (uint32_t k = 0; k < P.p.n_inst; ++k) for (int g = 0; g < 8; ++g) total[g] += a[8 * (size_t)k + g];
+    for (uint32_t i = 0; i < n; ++i) {
+        uint64_t j = j0 + i;
+        int g = groups[j % n_groups], b = bfms[(j / n_groups) % n_bfms];
+        if (g == ORC_G_NODEST) { G->err = "G_NODEST is not injectable (C-16)"; return 3; }
+        if (total[g] == 0) { G->err = "empty group"; return 2; }
+        orc_site& S = out[i];
+        memset(&S, 0, sizeof(S));
+        uint32_t att;
+        draw(seed, j, total[g], S.s, S.u_dst, S.u_bit, att);
+        S.group = (uint8_t)g; S.bfm = (uint8_t)b;
+        S.mask = mask_of(b, S.u_bit);
+        uint64_t cum = 0;
+        uint32_t k = 0;
+        for (k = 0; k < P.p.n_inst; ++k) {                // instance whose approximate range holds s
+            if (S.s < cum + a[8 * (size_t)k + g]) break;
+            cum += a[8 * (size_t)k + g];
+        }
+        const orc_instance& in = P.p.inst[k];
+        S.instance = k; S.kernel_id = in.kernel; S.kernel_count = in.kernel_count;
+        S.instruction_count = S.s - cum;
+        uint64_t seen = 0;
+        bool found = false;
+        for (uint32_t w = in.warp_begin; w < in.warp_end && !found; ++w) {
+            for (uint64_t r = G->woff[w]; r < G->woff[w + 1] && !found; ++r) {
+                const orc_record& R = G->trace[r];
+                if (!((R.insn >> (24 + g)) & 1)) continue;
+                uint32_t ex = R.active & R.pred;
+                for (int l = 0; l < 32 && !found; ++l) {
+                    if (!((ex >> l) & 1)) continue;
+                    if (seen == S.instruction_count) {
+                        uint32_t cta, wic;
+                        warp_coords(in, w, cta, wic);
+                        S.warp = w; S.step = (uint32_t)(r - G->woff[w]); S.lane = (uint8_t)l;
+                        S.thread = cta * in.block + wic * 32 + (uint32_t)l;
+                        S.pc = R.insn & 0xFFFF;
+                        const orc_insn& I = P.p.code[P.p.kern[in.kernel].code_off + S.pc];
+                        std::vector<std::pair<int, int>> sl;
+                        slots_for(I, g, sl);
+                        S.n_elig = (uint8_t)sl.size();
+                        S.slot = (uint8_t)(((uint64_t)sl.size() * S.u_dst) >> 32);
+                        S.dst_kind = (uint8_t)sl[S.slot].first;
+                        S.dst_reg = (uint8_t)sl[S.slot].second;
+                        found = true;
+                    }
+                    ++seen;
+                }
+            }
+        }
+        if (!found) S.flags = 1;
+    }
+    return 0;
+}
+
 // Locate given indices s (u_dst = 0, FLIP_SINGLE_BIT with u_bit = 0): the
 // enumeration alone, for the brute-force bijection pin.
 extern "C" int orc_locate(void* h, int group, const uint64_t* s, uint32_t n, orc_site* out) {
@@ -782,6 +880,7 @@ extern "C" int orc_inject(void* h, const orc_site* sites, uint32_t n, int mode, 
         const orc_site& S = sites[i];
         orc_inj& R = out[i];
         memset(&R, 0, sizeof(R));
+        if (S.flags & 1) { R.outcome = ORC_NOT_INJECTED; return; }      // C-17
         Hook hk;
         hk.on = true; hk.step = S.step; hk.lane = S.lane; hk.kind = S.dst_kind; hk.reg = S.dst_reg;
         hk.bfm = S.bfm; hk.mask = S.mask; hk.pc = S.pc;

@@ -47,7 +47,7 @@ typedef struct {
     uint64_t s, instruction_count;
     uint32_t instance, kernel_id, kernel_count, warp, step, thread;
     uint32_t pc, u_dst, u_bit, mask;
-    uint8_t lane, group, bfm, slot, dst_kind, dst_reg, n_elig, pad;
+    uint8_t lane, group, bfm, slot, dst_kind, dst_reg, n_elig, flags /* bit0: not injected (C-17) */;
 } orc_site;                                           /* 64 B */
 
 typedef struct {
@@ -58,7 +58,7 @@ typedef struct {
 
 /* groups (Table II order, C-1) and outcomes (Table V) */
 enum { ORC_G_FP64 = 0, ORC_G_FP32, ORC_G_LD, ORC_G_PR, ORC_G_NODEST, ORC_G_OTHERS, ORC_G_GPPR, ORC_G_GP };
-enum { ORC_MASKED = 0, ORC_SDC = 1, ORC_DUE = 2 };
+enum { ORC_MASKED = 0, ORC_SDC = 1, ORC_DUE = 2, ORC_NOT_INJECTED = 3 };
 enum { ORC_MODE_FULL = 0, ORC_MODE_WARP_LOCAL = 1, ORC_UNCHECKED = 0x100 /* f4 potential-DUE semantics */ };
 enum { ORC_POTENTIAL_DUE = 1 };
 
@@ -89,6 +89,12 @@ int orc_select(void* h, uint64_t seed, const uint8_t* groups, uint32_t n_groups,
                const uint8_t* bfms, uint32_t n_bfms, uint64_t j0, uint32_t n, orc_site* out);
 
 int orc_locate(void* h, int group, const uint64_t* s, uint32_t n, orc_site* out);
+
+/* row f1: per-opcode profile and approximate profiling */
+int orc_opcode_counts(void* h, uint64_t* out /*[n_inst][32]*/);
+int orc_approx_counts(void* h, uint64_t* out /*[n_inst][8]*/);
+int orc_select_approx(void* h, uint64_t seed, const uint8_t* groups, uint32_t n_groups,
+                      const uint8_t* bfms, uint32_t n_bfms, uint64_t j0, uint32_t n, orc_site* out);
 
 /* injection + classification; mode ORC_MODE_FULL re-runs the whole program */
 int orc_inject(void* h, const orc_site* sites, uint32_t n, int mode, int n_threads, orc_inj* out);

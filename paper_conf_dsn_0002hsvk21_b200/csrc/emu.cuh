@@ -41,18 +41,23 @@ namespace fi {
 
 constexpr uint32_t kFull = 0xFFFFFFFFu;
 constexpr int kLdgBatch = 4;          // independent LDGs issued together
-enum EmuMode { EMU_LEN = 0, EMU_TRACE = 1, EMU_INJ = 2 };
+enum EmuMode { EMU_LEN = 0, EMU_TRACE = 1, EMU_INJ = 2, EMU_PROP = 3 };
 
 // ---- prepared program data (fi_program.aux) --------------------------------
-struct AuxLayout { size_t gran, dec, ins, run, total; };
+// per instance: the buffers its constant bank points into (count, then ids;
+// count > kInstBufs = "unknown", never skipped by K7)
+constexpr uint32_t kInstBufs = 15;
+
+struct AuxLayout { size_t gran, dec, ins, run, ib, total; };
 __host__ __device__ inline size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
-__host__ __device__ inline AuxLayout aux_layout(uint64_t image_bytes, uint32_t n_code) {
+__host__ __device__ inline AuxLayout aux_layout(uint64_t image_bytes, uint32_t n_code, uint32_t n_inst) {
     AuxLayout L;
     L.gran = 0;
     L.dec = align256(((image_bytes + 255) >> 8) * sizeof(uint32_t));
     L.ins = L.dec + align256((size_t)n_code * 16);
     L.run = L.ins + align256((size_t)n_code * 4);
-    L.total = L.run + align256((size_t)n_code * 4);
+    L.ib = L.run + align256((size_t)n_code * 4);
+    L.total = L.ib + align256((size_t)n_inst * (kInstBufs + 1) * 4);
     return L;
 }
 
@@ -88,17 +93,19 @@ struct EmuProg {
     const uint32_t* cbank;
     const fi_buffer* buf;
     const uint32_t* gran;
+    const uint32_t* ib;        // per-instance referenced buffers [n_inst][kInstBufs+1]
     uint64_t image_bytes;
     uint32_t n_regs;
     uint32_t n_inst;
 };
 
 inline EmuProg make_emu_prog(const fi_program* p) {
-    const AuxLayout L = aux_layout(p->image_bytes, p->n_code);
+    const AuxLayout L = aux_layout(p->image_bytes, p->n_code, p->n_inst);
     const char* a = reinterpret_cast<const char*>(p->aux);
     return EmuProg{reinterpret_cast<const uint4*>(a + L.dec), reinterpret_cast<const uint32_t*>(a + L.ins),
                    reinterpret_cast<const uint32_t*>(a + L.run), p->kern, p->inst, p->cbank, p->buf,
-                   reinterpret_cast<const uint32_t*>(a + L.gran), p->image_bytes, p->n_regs, p->n_inst};
+                   reinterpret_cast<const uint32_t*>(a + L.gran), reinterpret_cast<const uint32_t*>(a + L.ib),
+                   p->image_bytes, p->n_regs, p->n_inst};
 }
 
 // checkpoint = (n_regs + 3) rows of 32 words: registers, then pc, predicates, live
@@ -379,12 +386,35 @@ __device__ __forceinline__ bool guard_of(uint32_t guard, uint32_t preds) {
     return (((gs == 7) ? 1u : ((preds >> gs) & 1u)) ^ ((guard >> 3) & 1u)) != 0;
 }
 
+// Faulty-memory overlay of one replica during downstream propagation (K7): an
+// open-addressing table of 32-bit words {va_lo, va_hi, value, used}; a word
+// present here holds the replica's current value, any other word has its
+// golden value (DESIGN.md §3.5 writer rule).
+struct Overlay {
+    uint4* tab;
+    uint32_t mask;                                   // capacity - 1 (power of two)
+};
+__device__ __forceinline__ uint32_t ov_hash(uint64_t va) {
+    return (uint32_t)(((va >> 2) * 0x9E3779B97F4A7C15ull) >> 32);
+}
+__device__ __forceinline__ bool ov_find(const Overlay& o, uint64_t va, uint32_t& v) {
+    uint32_t h = ov_hash(va) & o.mask;
+    for (uint32_t probes = 0; probes <= o.mask; ++probes) {
+        const uint4 e = __ldcg(&o.tab[h]);
+        if (!e.w) return false;
+        if (e.x == (uint32_t)va && e.y == (uint32_t)(va >> 32)) { v = e.z; return true; }
+        h = (h + 1) & o.mask;
+    }
+    return false;
+}
+
 template <int MODE>
 __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const uint8_t* img,
                                           uint32_t k, uint32_t cta, uint32_t wic, uint32_t* __restrict__ R,
                                           uint32_t watchdog, fi_record* __restrict__ rec_out,
                                           fi_store* __restrict__ st_out, uint32_t st_cap, HookIn hook,
-                                          uint32_t* __restrict__ ck, uint32_t ck_interval) {
+                                          uint32_t* __restrict__ ck, uint32_t ck_interval,
+                                          Overlay ov = Overlay{nullptr, 0}) {
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t lt_mask = (1u << lane) - 1u;
     const fi_instance in = P.inst[k];
@@ -509,6 +539,10 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
                             else if (lw == 1) { const uint2 t = ld_img64(src); vals[b].x = t.x; vals[b].y = t.y; }
                             else vals[b] = ld_img128(src);
                         }
+                        if (MODE == EMU_PROP && ex && !c) {  // the replica's overlay wins
+                            uint32_t* vw = &vals[b].x;
+                            for (uint32_t q = 0; q < (1u << lw); ++q) ov_find(ov, va + 4 * q, vw[q]);
+                        }
                         exs[b] = ex;
                         dsts[b] = D.z >> 16;
                         lws[b] = lw;
@@ -600,15 +634,19 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
             if (op == LDG) {
                 if (ex) {
                     const uint8_t* src = img + (va - kVaBase);
-                    if (lw == 0) {
-                        F.wr(id, zero ? 0u : ld_img32(src));
-                    } else if (lw == 1) {
-                        const uint2 v = zero ? make_uint2(0, 0) : ld_img64(src);
-                        F.wr(id, v.x); F.wr(id + 128, v.y);
-                    } else {
-                        const uint4 v = zero ? make_uint4(0, 0, 0, 0) : ld_img128(src);
-                        F.wr(id, v.x); F.wr(id + 128, v.y); F.wr(id + 256, v.z); F.wr(id + 384, v.w);
+                    uint4 v = make_uint4(0, 0, 0, 0);
+                    if (!zero) {
+                        if (lw == 0) v.x = ld_img32(src);
+                        else if (lw == 1) { const uint2 t = ld_img64(src); v.x = t.x; v.y = t.y; }
+                        else v = ld_img128(src);
                     }
+                    if (MODE == EMU_PROP) {                   // the replica's overlay wins
+                        uint32_t* vw = &v.x;
+                        for (uint32_t q = 0; q < nw; ++q) ov_find(ov, va + 4 * q, vw[q]);
+                    }
+                    F.wr(id, v.x);
+                    if (lw >= 1) F.wr(id + 128, v.y);
+                    if (lw >= 2) { F.wr(id + 256, v.z); F.wr(id + 384, v.w); }
                 }
             } else {
                 uint32_t v[4];
@@ -623,7 +661,7 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
                         else if (lw == 1) *reinterpret_cast<uint2*>(dst) = make_uint2(v[0], v[1]);
                         else *reinterpret_cast<uint4*>(dst) = make_uint4(v[0], v[1], v[2], v[3]);
                     }
-                } else if (MODE == EMU_TRACE || step > hook.step) {
+                } else if (MODE == EMU_TRACE || MODE == EMU_PROP || step > hook.step) {
                     if (ex) {
                         for (uint32_t i = 0; i < nw; ++i) {
                             const uint32_t e = nst + idx + i;

@@ -110,6 +110,29 @@ __global__ void k_decode(const fi_insn* code, uint32_t n_code, const fi_kernel* 
     run[i] = (r > 0xFFFF ? 0xFFFFu : r) | (std::min<uint32_t>(lr, 0xFF) << 16) | (fr << 24);
 }
 
+// Buffers an instance's constant bank points into (each adjacent word pair read as
+// a 64-bit VA): K7 skips a later instance when none of them holds dirty words.
+__global__ void k_inst_bufs(const fi_instance* inst, uint32_t n_inst, const uint32_t* cbank, const uint32_t* gran,
+                            uint64_t image_bytes, uint32_t* ib) {
+    const uint32_t k = blockIdx.x * blockDim.x + threadIdx.x;
+    if (k >= n_inst) return;
+    const fi_instance in = inst[k];
+    uint32_t* out = ib + (size_t)k * (kInstBufs + 1);
+    uint32_t n = 0;
+    for (uint32_t j = 0; j + 1 < in.cbank_len && n <= kInstBufs; ++j) {
+        const uint64_t va = (uint64_t)cbank[in.cbank_off + j] | ((uint64_t)cbank[in.cbank_off + j + 1] << 32);
+        if (va < kVaBase || va - kVaBase >= image_bytes) continue;
+        const uint32_t b = gran[(va - kVaBase) >> 8];
+        if (b == kNoBuf) continue;
+        bool have = false;
+        for (uint32_t q = 0; q < n && q < kInstBufs; ++q) have |= out[1 + q] == b;
+        if (have) continue;
+        if (n < kInstBufs) out[1 + n] = b;
+        ++n;
+    }
+    out[0] = n;                                       // > kInstBufs: too many, treat as unknown
+}
+
 __global__ void k_ckpt_counts(const uint64_t* warp_len, uint32_t n, uint32_t interval, uint64_t* cnt) {
     const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i < n) cnt[i] = (warp_len[i] + interval - 1) / interval;
@@ -133,14 +156,14 @@ extern "C" uint32_t fi_program_regs(const fi_insn* code, uint32_t n) {
     return std::min<uint32_t>(kRZ, mx + 4);        // +3: widest multi-register operand (LDG/STG.128)
 }
 
-extern "C" size_t fi_program_aux_bytes(uint64_t image_bytes, uint32_t n_code) {
-    return aux_layout(image_bytes, n_code).total;
+extern "C" size_t fi_program_aux_bytes(uint64_t image_bytes, uint32_t n_code, uint32_t n_inst) {
+    return aux_layout(image_bytes, n_code, n_inst).total;
 }
 
 extern "C" fi_status fi_program_prepare(const fi_program* p, void* aux, void* stream) {
     if (!p || !aux || p->n_regs == 0 || p->n_regs > kRZ) return FI_E_ARG;
     cudaStream_t s = (cudaStream_t)stream;
-    const AuxLayout L = aux_layout(p->image_bytes, p->n_code);
+    const AuxLayout L = aux_layout(p->image_bytes, p->n_code, p->n_inst);
     char* a = reinterpret_cast<char*>(aux);
     uint32_t* gran = reinterpret_cast<uint32_t*>(a + L.gran);
     const uint64_t n_gran = (p->image_bytes + 255) >> 8;
@@ -156,6 +179,11 @@ extern "C" fi_status fi_program_prepare(const fi_program* p, void* aux, void* st
                                                          reinterpret_cast<uint4*>(a + L.dec),
                                                          reinterpret_cast<uint32_t*>(a + L.ins),
                                                          reinterpret_cast<uint32_t*>(a + L.run));
+        if ((e = launch_status())) return e;
+    }
+    if (p->n_inst) {
+        k_inst_bufs<<<(p->n_inst + 127) / 128, 128, 0, s>>>(p->inst, p->n_inst, p->cbank, gran, p->image_bytes,
+                                                            reinterpret_cast<uint32_t*>(a + L.ib));
         if ((e = launch_status())) return e;
     }
     return FI_OK;

@@ -37,6 +37,7 @@ k_lpt_order(const fi_site* __restrict__ sites, const uint64_t* __restrict__ warp
     __shared__ uint32_t s_max;
     auto cost = [&](uint32_t i) -> uint64_t {
         const fi_site S = sites[i];
+        if (S.flags & FI_SITE_NOT_INJECTED) return 0;
         const uint64_t L = warp_off[S.warp + 1] - warp_off[S.warp];
         const uint64_t start = ck_interval ? (uint64_t)(S.step / ck_interval) * ck_interval : 0;
         return L > start ? L - start : 0;
@@ -79,6 +80,14 @@ k_inject(EmuProg P, const uint8_t* img, const uint64_t* __restrict__ warp_off, c
     if (p >= n) return;
     const uint32_t i = order[p];
     const fi_site S = sites[i];
+    if (S.flags & FI_SITE_NOT_INJECTED) {             // row f1 / C-17: nothing to inject
+        if (lane == 0) {
+            fi_inj r = {};
+            r.outcome = FI_NOT_INJECTED;
+            out[i] = r;
+        }
+        continue;
+    }
     const fi_instance in = P.inst[S.instance];
     const uint32_t wpc = (in.block + 31) / 32, lw = S.warp - in.warp_begin;
     const uint64_t L = warp_off[S.warp + 1] - warp_off[S.warp];
@@ -137,6 +146,10 @@ __global__ void __launch_bounds__(kClsWarps * 32) k_classify(const ClsArgs A) {
     uint32_t outcome;
     // f4: under FI_UNCHECKED only a hang is fatal; other faults just ended the warp
     const bool pdue = (A.flags & FI_UNCHECKED) && R.fault_kind && R.fault_kind != 3;
+    if (S.flags & FI_SITE_NOT_INJECTED) {
+        if (lane == 0) { A.inj[i].outcome = FI_NOT_INJECTED; A.inj[i].flags = 0; }
+        return;
+    }
     if (R.fault_kind && !pdue) {
         outcome = FI_DUE;
     } else if (R.overflow) {
@@ -240,11 +253,48 @@ extern "C" fi_status fi_inject(const fi_program* p, const uint8_t* image, const 
     return launch_status();
 }
 
+namespace fi {
+size_t propagate_slot_bytes(uint32_t ov_cap, uint32_t pend_cap);
+fi_status launch_propagate(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
+                           uint32_t n, fi_inj* out, const fi_store* log, uint32_t log_cap, uint64_t* hist,
+                           uint32_t flags, void* ws, size_t ws_bytes, const uint32_t* order, uint32_t* counter,
+                           uint32_t* dev_status, cudaStream_t s);
+namespace {
+__global__ void k_iota(uint32_t* order, uint32_t n, uint32_t* counter) {
+    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < n) order[i] = i;
+    if (i == 0) *counter = 0;
+}
+}  // namespace
+}  // namespace fi
+
+extern "C" size_t fi_classify_workspace(uint32_t n_inst, uint32_t n, uint32_t log_cap) {
+    if (n_inst <= 1 || n == 0) return 0;
+    uint32_t ov_cap = 1;
+    while (ov_cap < 4 * std::max<uint32_t>(log_cap, 4096)) ov_cap <<= 1;
+    const size_t sb = propagate_slot_bytes(ov_cap, 2 * std::max<uint32_t>(log_cap, 4096));
+    const uint64_t slots = std::min<uint64_t>(((uint64_t)n + 3) / 4 * 4, 148ull * 16);   // <= resident warps
+    return 256 + align256((size_t)n * 4) + slots * sb;
+}
+
 extern "C" fi_status fi_classify(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
                                  uint32_t n, fi_inj* out, const fi_store* log, uint32_t log_cap, uint64_t* hist,
-                                 uint32_t flags, uint32_t* dev_status, void* stream) {
+                                 uint32_t flags, void* ws, size_t ws_bytes, uint32_t* dev_status, void* stream) {
     if (!p || !image || !t || !sites || !out || !hist || !dev_status || !p->aux) return FI_E_ARG;
     if (n == 0) return FI_OK;
+    if (p->n_inst > 1) {
+        // K7: multi-instance programs propagate the faulty warp's effect downstream
+        if (!ws || ws_bytes < fi_classify_workspace(p->n_inst, n, log_cap)) return FI_E_ARG;
+        cudaStream_t s = (cudaStream_t)stream;
+        uint32_t* counter = reinterpret_cast<uint32_t*>(ws);
+        uint32_t* order = reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(ws) + 256);
+        const size_t head = 256 + align256((size_t)n * 4);
+        k_iota<<<(n + 255) / 256, 256, 0, s>>>(order, n, counter);
+        fi_status e = launch_status();
+        if (e) return e;
+        return launch_propagate(p, image, t, sites, n, out, log, log_cap, hist, flags, reinterpret_cast<char*>(ws) + head,
+                                ws_bytes - head, order, counter, dev_status, s);
+    }
     const EmuProg P = make_emu_prog(p);
     ClsArgs A{p->buf, P.gran, image, t->gstore, t->gstore_off, sites, out, n, log, log_cap, hist, flags, dev_status};
     k_classify<<<(n + kClsWarps - 1) / kClsWarps, kClsWarps * 32, 0, (cudaStream_t)stream>>>(A);

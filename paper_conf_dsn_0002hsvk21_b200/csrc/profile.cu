@@ -14,6 +14,7 @@
 // atomic per group per instance per warp).  Chunks that straddle instances
 // (rare: instance boundaries) attribute per record.
 #include <algorithm>
+#include <vector>
 
 #include "common.cuh"
 
@@ -96,6 +97,85 @@ k_profile(const uint4* __restrict__ rec, uint64_t r_begin, uint64_t r_end, uint6
 
 int g_grid = 0;
 
+// ---- §8 row f1: per-opcode profile ("counts for every opcode") ----
+// One warp per contiguous run of records; a per-warp shared-memory histogram over
+// the 32 opcode slots for the current instance, flushed with one u64 atomic per
+// nonzero opcode when the instance changes (records of a chunk that straddles an
+// instance boundary go straight to global atomics).
+constexpr int kOpThreads = 256;
+
+__global__ void __launch_bounds__(kOpThreads)
+k_profile_opcodes(const uint4* __restrict__ rec, uint64_t r_begin, uint64_t r_end, uint64_t* __restrict__ op_counts) {
+    __shared__ uint32_t hist[kOpThreads / 32][FI_NOPS];
+    const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    const uint64_t gw = ((uint64_t)blockIdx.x * kOpThreads + threadIdx.x) >> 5;
+    const uint64_t nwarps = ((uint64_t)gridDim.x * kOpThreads) >> 5;
+    const uint64_t n = r_end - r_begin;
+    const uint64_t per = ((n + nwarps - 1) / nwarps + 31) & ~31ull;
+    const uint64_t a = r_begin + gw * per, b = min(a + per, r_end);
+    uint32_t* h = hist[wib];
+    h[lane] = 0;
+    __syncwarp();
+    uint32_t cur = kNone;
+    for (uint64_t base = a; base < b; base += 32) {
+        const uint64_t r = base + lane;
+        const uint4 x = r < b ? ld_stream(rec + r) : make_uint4(kNone, 0, 0, 0);
+        const uint32_t k0 = __shfl_sync(0xFFFFFFFFu, x.x, 0);
+        if (k0 != cur) {                                  // flush the finished instance
+            __syncwarp();
+            if (cur != kNone && h[lane]) atomicAdd((unsigned long long*)&op_counts[(uint64_t)cur * FI_NOPS + lane], (unsigned long long)h[lane]);
+            h[lane] = 0;
+            __syncwarp();
+            cur = k0;
+        }
+        const uint32_t c = __popc(x.z & x.w);
+        const uint32_t op = (x.y >> 16) & (FI_NOPS - 1);
+        if (r < b && c) {
+            if (x.x == cur) atomicAdd(&h[op], c);
+            else atomicAdd((unsigned long long*)&op_counts[(uint64_t)x.x * FI_NOPS + op], (unsigned long long)c);
+        }
+    }
+    __syncwarp();
+    if (cur != kNone && h[lane]) atomicAdd((unsigned long long*)&op_counts[(uint64_t)cur * FI_NOPS + lane], (unsigned long long)h[lane]);
+}
+
+// ---- §8 row f1: approximate profiling ----------------------------
+// Count only the records of the first dynamic instance of each static kernel
+// (one instance's record range per blockIdx.y) ...
+__global__ void __launch_bounds__(kThreads)
+k_profile_first(const uint4* __restrict__ rec, const uint64_t* __restrict__ warp_off,
+                const fi_instance* __restrict__ inst, const uint32_t* __restrict__ firsts,
+                uint64_t* __restrict__ inst_counts) {
+    const uint32_t k = firsts[blockIdx.y];
+    const uint64_t r0 = warp_off[inst[k].warp_begin], r1 = warp_off[inst[k].warp_end];
+    const uint32_t lane = threadIdx.x & 31;
+    uint32_t cnt[8];
+#pragma unroll
+    for (int g = 0; g < 8; ++g) cnt[g] = 0;
+    for (uint64_t r = r0 + (uint64_t)blockIdx.x * kThreads + threadIdx.x; r < r1; r += (uint64_t)gridDim.x * kThreads) {
+        const uint4 x = ld_stream(rec + r);
+        const uint32_t c = __popc(x.z & x.w), gm = x.y >> 24;
+#pragma unroll
+        for (int g = 0; g < 8; ++g) cnt[g] += ((gm >> g) & 1u) ? c : 0u;
+    }
+#pragma unroll
+    for (int g = 0; g < 8; ++g) {
+        const uint32_t s = __reduce_add_sync(0xFFFFFFFFu, cnt[g]);
+        if (lane == 0 && s) atomicAdd((unsigned long long*)&inst_counts[(uint64_t)k * 8 + g], (unsigned long long)s);
+    }
+}
+
+// ... and assume every later instance of the same static kernel has the same counts.
+__global__ void k_expand_first(const fi_instance* __restrict__ inst, uint32_t n_inst,
+                               const uint32_t* __restrict__ first_of_kernel, uint64_t* __restrict__ counts,
+                               uint32_t width) {
+    const uint32_t k = blockIdx.x * blockDim.x + threadIdx.x;
+    if (k >= n_inst) return;
+    const uint32_t f = first_of_kernel[inst[k].kernel];
+    if (f == k) return;
+    for (uint32_t g = 0; g < width; ++g) counts[(uint64_t)k * width + g] = counts[(uint64_t)f * width + g];
+}
+
 }  // namespace
 }  // namespace fi
 
@@ -120,5 +200,53 @@ extern "C" fi_status fi_profile(const fi_trace* t, uint64_t rec_begin, uint64_t 
     const int grid = (int)std::min<uint64_t>((uint64_t)g_grid, (warps_needed * 32 + kThreads - 1) / kThreads);
     k_profile<<<grid, kThreads, 0, s>>>(reinterpret_cast<const uint4*>(t->rec), rec_begin, rec_end, c_begin, c_end,
                                          inst_counts, chunk_counts);
+    return launch_status();
+}
+
+extern "C" fi_status fi_profile_opcodes(const fi_trace* t, uint64_t rec_begin, uint64_t rec_end, uint32_t n_inst,
+                                        uint64_t* op_counts, void* stream) {
+    if (!t || !op_counts || rec_end > t->n_rec || rec_begin > rec_end) return FI_E_ARG;
+    cudaStream_t s = (cudaStream_t)stream;
+    fi_status e = cuda_status(cudaMemsetAsync(op_counts, 0, (size_t)n_inst * FI_NOPS * sizeof(uint64_t), s));
+    if (e || rec_begin == rec_end) return e;
+    int dev = 0, sms = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const uint64_t warps = (rec_end - rec_begin + 1023) / 1024;
+    const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)sms * 8, (warps * 32 + kOpThreads - 1) / kOpThreads));
+    k_profile_opcodes<<<grid, kOpThreads, 0, s>>>(reinterpret_cast<const uint4*>(t->rec), rec_begin, rec_end, op_counts);
+    return launch_status();
+}
+
+extern "C" size_t fi_profile_approx_workspace(uint32_t n_kern, uint32_t n_inst) {
+    (void)n_inst;
+    return 256 + 2 * (size_t)std::max<uint32_t>(n_kern, 1) * sizeof(uint32_t);
+}
+
+extern "C" fi_status fi_profile_approx(const fi_program* p, const fi_trace* t, uint64_t* inst_counts, void* ws,
+                                       size_t ws_bytes, void* stream) {
+    if (!p || !t || !inst_counts || !p->inst_host || !ws || ws_bytes < fi_profile_approx_workspace(p->n_kern, p->n_inst))
+        return FI_E_ARG;
+    cudaStream_t s = (cudaStream_t)stream;
+    std::vector<uint32_t> first_of(std::max<uint32_t>(p->n_kern, 1), 0xFFFFFFFFu), firsts;
+    for (uint32_t k = 0; k < p->n_inst; ++k) {
+        const fi_instance& in = p->inst_host[k];
+        if (in.kernel < p->n_kern && first_of[in.kernel] == 0xFFFFFFFFu) {
+            first_of[in.kernel] = k;
+            firsts.push_back(k);
+        }
+    }
+    uint32_t* d_first_of = reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(ws) + 256);
+    uint32_t* d_firsts = d_first_of + std::max<uint32_t>(p->n_kern, 1);
+    fi_status e = cuda_status(cudaMemsetAsync(inst_counts, 0, (size_t)p->n_inst * 8 * sizeof(uint64_t), s));
+    if (e || firsts.empty()) return e;
+    if ((e = cuda_status(cudaMemcpyAsync(d_first_of, first_of.data(), first_of.size() * 4, cudaMemcpyHostToDevice, s)))) return e;
+    if ((e = cuda_status(cudaMemcpyAsync(d_firsts, firsts.data(), firsts.size() * 4, cudaMemcpyHostToDevice, s)))) return e;
+    if ((e = cuda_status(cudaStreamSynchronize(s)))) return e;      // host vectors go out of scope
+    dim3 grid(64, (unsigned)firsts.size());
+    k_profile_first<<<grid, kThreads, 0, s>>>(reinterpret_cast<const uint4*>(t->rec), t->warp_off, p->inst, d_firsts,
+                                              inst_counts);
+    if ((e = launch_status())) return e;
+    k_expand_first<<<(p->n_inst + 127) / 128, 128, 0, s>>>(p->inst, p->n_inst, d_first_of, inst_counts, 8);
     return launch_status();
 }

@@ -83,6 +83,10 @@ struct SelArgs {
 constexpr int kWarps = 4;
 constexpr uint32_t kTileChunks = 64;          // chunks per index tile (two-level chunk index)
 
+__device__ void finish_site(const SelArgs& A, uint32_t i, uint32_t g, uint32_t bfm, uint64_t s, uint64_t ic,
+                            uint32_t k, uint32_t w, uint64_t rec_idx, uint32_t rinsn, uint32_t lane_sel,
+                            uint32_t u_dst, uint32_t u_bit);
+
 __global__ void __launch_bounds__(kWarps * 32) k_select(const SelArgs A) {
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t i = blockIdx.x * kWarps + (threadIdx.x >> 5);
@@ -162,6 +166,14 @@ __global__ void __launch_bounds__(kWarps * 32) k_select(const SelArgs A) {
     }
     const uint32_t w = (uint32_t)warp_upper_search(A.warp_off, A.n_warps, 1, 0, rec_idx);
     if (lane != 0) return;
+    finish_site(A, i, g, bfm, s, s - __ldg(&A.Pk[(uint64_t)k * 8 + g]), k, w, rec_idx, rinsn, lane_sel, u_dst, u_bit);
+}
+
+// Record the located site: warp-local step, thread, destination slot (C-6) and
+// Table II mask (C-5, C-8).  Lane 0 only.
+__device__ void finish_site(const SelArgs& A, uint32_t i, uint32_t g, uint32_t bfm, uint64_t s, uint64_t ic,
+                            uint32_t k, uint32_t w, uint64_t rec_idx, uint32_t rinsn, uint32_t lane_sel,
+                            uint32_t u_dst, uint32_t u_bit) {
     const fi_instance in = A.inst[k];
     const uint32_t wpc = (in.block + 31) / 32, lw = w - in.warp_begin;
     const uint32_t pc = rinsn & 0xFFFFu;
@@ -175,7 +187,7 @@ __global__ void __launch_bounds__(kWarps * 32) k_select(const SelArgs A) {
 
     fi_site S;
     S.s = s;
-    S.instruction_count = s - __ldg(&A.Pk[(uint64_t)k * 8 + g]);
+    S.instruction_count = ic;
     S.instance = k;
     S.kernel_id = in.kernel;
     S.kernel_count = in.kernel_count;
@@ -193,8 +205,69 @@ __global__ void __launch_bounds__(kWarps * 32) k_select(const SelArgs A) {
     S.dst_kind = (uint8_t)kind;
     S.dst_reg = (uint8_t)reg;
     S.n_elig = (uint8_t)ne;
-    S.pad = 0;
+    S.flags = 0;
     A.sites[i] = S;
+}
+
+// Row f1: the approximate profile's P_k names (instance, instruction_count); the
+// site is then found by counting through the instance's own records, as the
+// injector does at run time (C-17: not injected when the instance is shorter).
+__global__ void __launch_bounds__(kWarps * 32) k_select_approx(const SelArgs A) {
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t i = blockIdx.x * kWarps + (threadIdx.x >> 5);
+    if (i >= A.n) return;
+    const uint64_t j = A.j0 + i;
+    const uint32_t g = A.sched.groups[j % A.sched.n_groups];
+    const uint32_t bfm = A.sched.bfms[(j / A.sched.n_groups) % A.sched.n_bfms];
+    uint64_t s = 0;
+    uint32_t u_dst = 0, u_bit = 0;
+    if (lane == 0) draw(A.sched.seed, j, A.totals[g], s, u_dst, u_bit);
+    s = __shfl_sync(0xFFFFFFFFu, s, 0);
+    u_dst = __shfl_sync(0xFFFFFFFFu, u_dst, 0);
+    u_bit = __shfl_sync(0xFFFFFFFFu, u_bit, 0);
+    const uint32_t k = (uint32_t)warp_upper_search(A.Pk, A.n_inst, 8, g, s);
+    const uint64_t ic = s - __ldg(&A.Pk[(uint64_t)k * 8 + g]);
+    const fi_instance in = A.inst[k];
+    const uint64_t r0 = __ldg(&A.warp_off[in.warp_begin]), r1 = __ldg(&A.warp_off[in.warp_end]);
+    uint64_t r = ic, rec_idx = 0;
+    uint32_t rinsn = 0, lane_sel = 0;
+    bool found = false;
+    for (uint64_t base = r0; base < r1; base += 32) {
+        const uint64_t idx = base + lane;
+        const uint4 x = idx < r1 ? __ldg(&A.rec[idx]) : make_uint4(0, 0, 0, 0);
+        const uint32_t ex = x.z & x.w;
+        const uint32_t cnt = ((x.y >> (24 + g)) & 1u) ? __popc(ex) : 0u;
+        uint32_t incl = cnt;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, incl, d);
+            if (lane >= (uint32_t)d) incl += y;
+        }
+        const uint32_t total = __shfl_sync(0xFFFFFFFFu, incl, 31);
+        if (r < total) {
+            const uint32_t L = __ffs(__ballot_sync(0xFFFFFFFFu, incl > r)) - 1;
+            const uint32_t before = __shfl_sync(0xFFFFFFFFu, incl - cnt, L);
+            const uint32_t exL = __shfl_sync(0xFFFFFFFFu, ex, L);
+            rinsn = __shfl_sync(0xFFFFFFFFu, x.y, L);
+            lane_sel = __fns(exL, 0, (int)(r - before) + 1);
+            rec_idx = base + L;
+            found = true;
+            break;
+        }
+        r -= total;
+    }
+    if (!found) {                                      // C-17: the site does not exist in this instance
+        if (lane == 0) {
+            fi_site S = {};
+            S.s = s; S.instruction_count = ic; S.instance = k; S.kernel_id = in.kernel;
+            S.kernel_count = in.kernel_count; S.u_dst = u_dst; S.u_bit = u_bit; S.mask = bfm_mask(bfm, u_bit);
+            S.group = (uint8_t)g; S.bfm = (uint8_t)bfm; S.flags = FI_SITE_NOT_INJECTED;
+            A.sites[i] = S;
+        }
+        return;
+    }
+    const uint32_t w = (uint32_t)warp_upper_search(A.warp_off, A.n_warps, 1, 0, rec_idx);
+    if (lane == 0) finish_site(A, i, g, bfm, s, ic, k, w, rec_idx, rinsn, lane_sel, u_dst, u_bit);
 }
 
 size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
@@ -302,11 +375,7 @@ extern "C" fi_status fi_site_totals(const void* index, uint32_t n_inst, uint64_t
     return cuda_status(cudaStreamSynchronize(s));
 }
 
-extern "C" fi_status fi_select_sites(const fi_program* p, const fi_trace* t, const uint32_t* chunk_counts,
-                                     const void* index, uint32_t n_inst, uint64_t n_chunks,
-                                     const uint64_t totals_host[8], const fi_schedule* sched, uint64_t j0, uint32_t n,
-                                     fi_site* sites, uint32_t* dev_status, void* stream) {
-    if (!p || !t || !index || !chunk_counts || !totals_host || !sched || !sites || !dev_status) return FI_E_ARG;
+static fi_status check_schedule(const fi_schedule* sched, const uint64_t totals_host[8]) {
     if (sched->n_groups == 0 || sched->n_groups > 8 || sched->n_bfms == 0 || sched->n_bfms > 4) return FI_E_ARG;
     for (uint32_t i = 0; i < sched->n_groups; ++i) {
         if (sched->groups[i] >= FI_NGROUPS) return FI_E_ARG;
@@ -315,7 +384,48 @@ extern "C" fi_status fi_select_sites(const fi_program* p, const fi_trace* t, con
     }
     for (uint32_t i = 0; i < sched->n_bfms; ++i)
         if (sched->bfms[i] > FI_ZERO_VALUE) return FI_E_ARG;
-    if (n == 0) return FI_OK;
+    return FI_OK;
+}
+
+extern "C" fi_status fi_build_instance_index(const uint64_t* inst_counts, uint32_t n_inst, void* index,
+                                             uint32_t* dev_status, void* stream) {
+    if (!inst_counts || !index || !dev_status) return FI_E_ARG;
+    const IndexLayout L = layout(n_inst, 0);
+    char* b = reinterpret_cast<char*>(index);
+    cudaStream_t s = (cudaStream_t)stream;
+    if (n_inst) {
+        k_inst_identities<<<(n_inst + 127) / 128, 128, 0, s>>>(inst_counts, n_inst, dev_status);
+        fi_status e = launch_status();
+        if (e) return e;
+    }
+    return scan_rows_u64x8(inst_counts, reinterpret_cast<uint64_t*>(b + L.pk), n_inst, b + L.ws_k, L.ws_t - L.ws_k, s);
+}
+
+extern "C" fi_status fi_select_sites_approx(const fi_program* p, const fi_trace* t, const void* index, uint32_t n_inst,
+                                            const uint64_t totals_host[8], const fi_schedule* sched, uint64_t j0,
+                                            uint32_t n, fi_site* sites, uint32_t* dev_status, void* stream) {
+    if (!p || !t || !index || !totals_host || !sched || !sites || !dev_status) return FI_E_ARG;
+    fi_status e = check_schedule(sched, totals_host);
+    if (e || n == 0) return e;
+    const IndexLayout L = layout(n_inst, 0);
+    SelArgs A = {};
+    A.code = p->code; A.kern = p->kern; A.inst = p->inst;
+    A.rec = reinterpret_cast<const uint4*>(t->rec); A.n_rec = t->n_rec; A.warp_off = t->warp_off; A.n_warps = t->n_warps;
+    A.Pk = reinterpret_cast<const uint64_t*>(reinterpret_cast<const char*>(index) + L.pk); A.n_inst = n_inst;
+    for (int g = 0; g < 8; ++g) A.totals[g] = totals_host[g];
+    A.sched = *sched;
+    A.j0 = j0; A.n = n; A.sites = sites; A.status = dev_status;
+    k_select_approx<<<(n + kWarps - 1) / kWarps, kWarps * 32, 0, (cudaStream_t)stream>>>(A);
+    return launch_status();
+}
+
+extern "C" fi_status fi_select_sites(const fi_program* p, const fi_trace* t, const uint32_t* chunk_counts,
+                                     const void* index, uint32_t n_inst, uint64_t n_chunks,
+                                     const uint64_t totals_host[8], const fi_schedule* sched, uint64_t j0, uint32_t n,
+                                     fi_site* sites, uint32_t* dev_status, void* stream) {
+    if (!p || !t || !index || !chunk_counts || !totals_host || !sched || !sites || !dev_status) return FI_E_ARG;
+    fi_status e = check_schedule(sched, totals_host);
+    if (e || n == 0) return e;
     const IndexLayout L = layout(n_inst, n_chunks);
     const char* b = reinterpret_cast<const char*>(index);
     SelArgs A;

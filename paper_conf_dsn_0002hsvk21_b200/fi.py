@@ -25,14 +25,15 @@ FI_UNCHECKED, FI_POTENTIAL_DUE = 1, 1
 G_FP64, G_FP32, G_LD, G_PR, G_NODEST, G_OTHERS, G_GPPR, G_GP = range(8)
 GROUP_NAMES = ["G_FP64", "G_FP32", "G_LD", "G_PR", "G_NODEST", "G_OTHERS", "G_GPPR", "G_GP"]
 BFM_NAMES = ["FLIP_SINGLE_BIT", "FLIP_TWO_BITS", "RANDOM_VALUE", "ZERO_VALUE"]
-MASKED, SDC, DUE = 0, 1, 2
+MASKED, SDC, DUE, NOT_INJECTED = 0, 1, 2, 3
+FI_NOPS = 32
 
 SITE_DTYPE = np.dtype([
     ("s", "<u8"), ("instruction_count", "<u8"),
     ("instance", "<u4"), ("kernel_id", "<u4"), ("kernel_count", "<u4"), ("warp", "<u4"),
     ("step", "<u4"), ("thread", "<u4"), ("pc", "<u4"), ("u_dst", "<u4"), ("u_bit", "<u4"), ("mask", "<u4"),
     ("lane", "u1"), ("group", "u1"), ("bfm", "u1"), ("slot", "u1"), ("dst_kind", "u1"), ("dst_reg", "u1"),
-    ("n_elig", "u1"), ("pad", "u1"),
+    ("n_elig", "u1"), ("flags", "u1"),
 ])
 INJ_DTYPE = np.dtype([("before", "<u4"), ("after", "<u4"), ("mask", "<u4"), ("fault_pc", "<u4"),
                       ("fault_kind", "u1"), ("outcome", "u1"), ("overflow", "u1"), ("flags", "u1"),
@@ -88,7 +89,7 @@ def lib():
             "fi_last_cuda_error": (C.c_char_p, []),
             "fi_version": (C.c_char_p, []),
             "fi_program_regs": (u32, [vp, u32]),
-            "fi_program_aux_bytes": (sz, [u64, u32]),
+            "fi_program_aux_bytes": (sz, [u64, u32, u32]),
             "fi_program_prepare": (st, [vp, vp, vp]),
             "fi_golden_lengths": (st, [vp, vp, vp, vp, vp, vp]),
             "fi_scan_u64_workspace": (sz, [u64]),
@@ -104,8 +105,14 @@ def lib():
             "fi_select_sites": (st, [vp, vp, vp, vp, u32, u64, vp, vp, u64, u32, vp, vp, vp]),
             "fi_inject_workspace": (sz, [u32]),
             "fi_inject": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, sz, vp, vp]),
-            "fi_classify": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, u32, vp, vp]),
+            "fi_classify_workspace": (sz, [u32, u32, u32]),
+            "fi_classify": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, u32, vp, sz, vp, vp]),
             "fi_write_params_txt": (st, [vp, C.c_char_p, C.c_char_p, sz]),
+            "fi_profile_opcodes": (st, [vp, u64, u64, u32, vp, vp]),
+            "fi_profile_approx_workspace": (sz, [u32, u32]),
+            "fi_profile_approx": (st, [vp, vp, vp, vp, sz, vp]),
+            "fi_build_instance_index": (st, [vp, u32, vp, vp, vp]),
+            "fi_select_sites_approx": (st, [vp, vp, vp, u32, vp, vp, u64, u32, vp, vp, vp]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -178,7 +185,8 @@ class DeviceProgram:
         self.cbank = up("cbank", prog.cbank)
         self.buf = up("buffers", prog.buffers)
         self.init_image = up("init_image", prog.init_image)
-        self.aux = torch.empty(lib().fi_program_aux_bytes(prog.image_bytes, len(prog.code)), dtype=torch.uint8,
+        self.aux = torch.empty(lib().fi_program_aux_bytes(prog.image_bytes, len(prog.code), len(prog.instances)),
+                               dtype=torch.uint8,
                                device=self.device)
         self._code_host = np.ascontiguousarray(prog.code)
         self._inst_host = np.ascontiguousarray(prog.instances)
@@ -354,18 +362,74 @@ def inject(gt: GoldenTrace, sites: torch.Tensor, n: int, log_cap: int, out: torc
 
 def classify(gt: GoldenTrace, sites: torch.Tensor, n: int, out: torch.Tensor, log: torch.Tensor, log_cap: int,
              hist: torch.Tensor | None = None, status: DeviceStatus | None = None,
-             unchecked: bool = False) -> torch.Tensor:
+             unchecked: bool = False, ws: torch.Tensor | None = None) -> torch.Tensor:
     """fi_classify (K5): fills out[].outcome, accumulates hist[8][4][3].
     unchecked=True: potential-DUE semantics (FI_UNCHECKED, row f4)."""
     dev = gt.dp.device
     if hist is None:
         hist = torch.zeros((8, 4, 3), dtype=torch.int64, device=dev)
     st = status or DeviceStatus(dev)
+    ws_n = lib().fi_classify_workspace(gt.dp.n_inst, n, log_cap)
+    if ws_n and (ws is None or ws.numel() < ws_n):
+        ws = torch.empty(ws_n, dtype=torch.uint8, device=dev)
     _check(lib().fi_classify(C.byref(gt.dp.c), _p(gt.image), C.byref(gt.c), _p(sites), n, _p(out), _p(log), log_cap,
-                             _p(hist), FI_UNCHECKED if unchecked else 0, st.ptr, _stream()), "fi_classify")
+                             _p(hist), FI_UNCHECKED if unchecked else 0, _p(ws) if ws_n else None, ws_n, st.ptr,
+                             _stream()), "fi_classify")
     if status is None:
         st.check("fi_classify")
     return hist
+
+
+def profile_opcodes(gt: GoldenTrace, rec_begin: int = 0, rec_end: int | None = None) -> torch.Tensor:
+    """fi_profile_opcodes (row f1): per-instance, per-opcode thread-level counts [K][32]."""
+    rec_end = gt.n_rec if rec_end is None else rec_end
+    out = torch.empty((max(gt.dp.n_inst, 1), FI_NOPS), dtype=torch.int64, device=gt.dp.device)
+    _check(lib().fi_profile_opcodes(C.byref(gt.c), rec_begin, rec_end, gt.dp.n_inst, _p(out), _stream()),
+           "fi_profile_opcodes")
+    return out
+
+
+def profile_approx(gt: GoldenTrace) -> torch.Tensor:
+    """fi_profile_approx (row f1): counts of each static kernel's first instance reused."""
+    dp = gt.dp
+    out = torch.empty((max(dp.n_inst, 1), 8), dtype=torch.int64, device=dp.device)
+    ws_n = lib().fi_profile_approx_workspace(len(dp.prog.kernels), dp.n_inst)
+    ws = torch.empty(ws_n, dtype=torch.uint8, device=dp.device)
+    _check(lib().fi_profile_approx(C.byref(dp.c), C.byref(gt.c), _p(out), _p(ws), ws_n, _stream()), "fi_profile_approx")
+    return out
+
+
+class InstanceIndex:
+    """fi_build_instance_index: P_k only (e.g. over approximate counts) + totals."""
+
+    def __init__(self, gt: GoldenTrace, inst_counts: torch.Tensor, status: DeviceStatus | None = None):
+        self.gt = gt
+        self.n_inst = gt.dp.n_inst
+        nb = lib().fi_site_index_bytes(self.n_inst, 0)
+        self.buf = torch.empty(nb, dtype=torch.uint8, device=gt.dp.device)
+        st = status or DeviceStatus(gt.dp.device)
+        _check(lib().fi_build_instance_index(_p(inst_counts), self.n_inst, _p(self.buf), st.ptr, _stream()),
+               "fi_build_instance_index")
+        tot = (C.c_uint64 * 8)()
+        _check(lib().fi_site_totals(_p(self.buf), self.n_inst, tot, _stream()), "fi_site_totals")
+        self.totals = [int(x) for x in tot]
+        self._tot = tot
+        if status is None:
+            st.check("fi_build_instance_index")
+
+
+def select_sites_approx(idx: InstanceIndex, sched: fi_schedule, j0: int, n: int,
+                        sites: torch.Tensor | None = None, status: DeviceStatus | None = None) -> torch.Tensor:
+    """fi_select_sites_approx (row f1)."""
+    gt = idx.gt
+    if sites is None:
+        sites = torch.empty(max(n, 1) * 64, dtype=torch.uint8, device=gt.dp.device)
+    st = status or DeviceStatus(gt.dp.device)
+    _check(lib().fi_select_sites_approx(C.byref(gt.dp.c), C.byref(gt.c), _p(idx.buf), idx.n_inst, idx._tot,
+                                        C.byref(sched), j0, n, _p(sites), st.ptr, _stream()), "fi_select_sites_approx")
+    if status is None:
+        st.check("fi_select_sites_approx")
+    return sites
 
 
 def write_params_txt(site_row: np.ndarray, kernel_name: str) -> str:

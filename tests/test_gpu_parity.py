@@ -249,3 +249,58 @@ def test_scan_u64_and_rows(F, n):
         tiles[t] = cc[t * 64: min(n, t * 64 + 64)].astype(np.uint64).sum(0)
     wantt = np.concatenate([np.zeros((1, 8), np.uint64), np.cumsum(tiles, 0)])
     assert np.array_equal(pt, wantt)
+
+
+@pytest.mark.parametrize("maker", [P.c1, lambda: P.fuzz_program(3), lambda: P.multi_instance_chain(4, shrink=30),
+                                   lambda: P.c2(full=False)])
+def test_opcode_profile_parity(F, maker):
+    """Row f1: per-opcode profile equals the oracle's per-record sums, and
+    sharded profiles add up."""
+    prog = maker()
+    g = O.Golden(prog)
+    dp, gt = _gpu_golden(F, prog)
+    oc = F.profile_opcodes(gt).cpu().numpy().astype(np.uint64)[: len(prog.instances)]
+    assert np.array_equal(oc, g.opcode_counts())
+    cut = gt.n_rec // 2 + 7
+    a = F.profile_opcodes(gt, 0, cut) + F.profile_opcodes(gt, cut, gt.n_rec)
+    assert np.array_equal(a.cpu().numpy().astype(np.uint64)[: len(prog.instances)], oc)
+
+
+def test_approximate_profile_and_selection_parity(F):
+    """Row f1: approximate profiling and selection over it, including
+    the not-injected sites of C-17, bit-exact against the oracle; injection and
+    classification skip not-injected sites."""
+    prog = P.multi_instance_chain(n_inst=6, n=256, shrink=33)
+    g = O.Golden(prog)
+    dp, gt = _gpu_golden(F, prog)
+    ap = F.profile_approx(gt).cpu().numpy().astype(np.uint64)
+    assert np.array_equal(ap, g.approx_counts())
+    idx = F.InstanceIndex(gt, F.profile_approx(gt))
+    n = 500
+    sched = F.schedule(0xA11, [F.G_GP, F.G_FP32, F.G_LD], [0, 1, 2, 3])
+    sites = F.select_sites_approx(idx, sched, 0, n)
+    gs = F.as_numpy(sites, F.SITE_DTYPE, n)
+    os_ = g.select_approx(0xA11, [F.G_GP, F.G_FP32, F.G_LD], [0, 1, 2, 3], 0, n)
+    _assert_sites_equal(gs, os_)
+    assert 0 < (gs["flags"] == 1).sum() < n
+    cap = F.log_capacity(gt)
+    out, log = F.inject(gt, sites, n, cap)
+    hist = F.classify(gt, sites, n, out, log, cap)
+    gi = F.as_numpy(out, F.INJ_DTYPE, n)
+    oi = g.inject(os_, O.MODE_FULL)
+    assert (gi["outcome"] == oi["outcome"]).all()
+    ok = gs["flags"] == 0
+    for f in ("before", "after", "mask", "fault_kind"):
+        assert (gi[f][ok] == oi[f][ok]).all(), f
+    assert int(hist.sum()) == int(ok.sum())
+
+
+@pytest.mark.parametrize("maker,unchecked", [(lambda: P.multi_instance_chain(5), False),
+                                             (lambda: P.multi_instance_chain(6, shrink=29), False),
+                                             (lambda: P.multi_instance_chain(4, n=300, block=96), True)])
+def test_multi_instance_injection_parity(F, maker, unchecked):
+    """K7: faults in non-final instances propagate through the later launches; the
+    outcome is the whole program's (oracle full mode, the definition)."""
+    gi, oi = _campaign_parity(F, maker(), 0x7A7, [F.G_GP, F.G_LD, F.G_FP32, F.G_OTHERS], [0, 1, 2, 3], 400,
+                              O.MODE_FULL, unchecked=unchecked)
+    assert (oi["outcome"] == O.SDC).sum() > 0

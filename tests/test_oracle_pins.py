@@ -439,3 +439,43 @@ def test_watchdog_hang_is_due():
 def test_ci_margins():
     assert round(O.ci_margin(100, 0.90), 2) == 0.08          # "+-8%"
     assert round(O.ci_margin(1000, 0.95), 2) == 0.03         # "+-3%"
+
+
+# ---------------------------------------------------------------------------
+# Row f1: per-opcode profile and approximate profiling
+# ---------------------------------------------------------------------------
+def test_c1_opcode_profile_closed_form():
+    g = O.Golden(P.c1())
+    oc = g.opcode_counts()[0]
+    want = {isa.S2R: 3, isa.IMAD: 1, isa.LDC: 4, isa.ISETP: 1, isa.EXIT: 1, isa.IMAD_WIDE: 3, isa.LDG: 2,
+            isa.FADD: 1, isa.STG: 1}           # per thread; the @P0 EXIT is predicated off
+    for op in range(32):
+        assert int(oc[op]) == 1024 * want.get(op, 0), isa.OPNAMES[op] if op < len(isa.OPNAMES) else op
+    c = g.counts()[0]
+    assert int(oc.sum()) == int(c[GPPR] + c[NODEST])
+
+
+def test_approximate_profile_reuses_first_instance():
+    prog = P.multi_instance_chain(n_inst=5, n=256, shrink=40)
+    g = O.Golden(prog)
+    exact, approx = g.counts(), g.approx_counts()
+    assert (approx == exact[0]).all()                      # every instance assumed = the first
+    assert (exact[1:, GP] < exact[0, GP]).all()            # later launches really are shorter
+    s = g.select_approx(0xA9, [GP, FP32], [0, 1], 0, 400)
+    exact_first = np.concatenate([[0], np.cumsum(exact[:, GP])]), np.concatenate([[0], np.cumsum(exact[:, FP32])])
+    for site in s:
+        grp = int(site["group"])
+        k, ic = int(site["instance"]), int(site["instruction_count"])
+        col = GP if grp == GP else FP32
+        if ic >= exact[k, col]:
+            assert site["flags"] == 1                      # C-17: not injected
+            continue
+        assert site["flags"] == 0
+        # the same site as the exact enumeration's (instance-start + ic)-th
+        ref = g.locate(grp, [exact_first[0 if grp == GP else 1][k] + ic])[0]
+        for f in ("warp", "step", "lane", "pc", "thread"):
+            assert site[f] == ref[f]
+    assert 0 < (s["flags"] == 1).sum() < len(s)
+    r = g.inject(s, O.MODE_FULL)
+    assert (r["outcome"][s["flags"] == 1] == O.NOT_INJECTED).all()
+    assert (r["outcome"][s["flags"] == 0] != O.NOT_INJECTED).all()
