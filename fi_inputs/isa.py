@@ -29,12 +29,13 @@ import numpy as np
 NOP, EXIT, BRA, MOV, S2R, IADD3, IMAD, IMAD_WIDE, SHF, LOP3, SEL = range(11)
 ISETP, FSETP, DSETP, FADD, FMUL, FFMA, FMNMX, DADD, DMUL, DFMA = range(11, 21)
 LDG, LDC, STG, I2F, F2I, F2F_F64_F32, F2F_F32_F64, SHFL, IMNMX = range(21, 30)
-N_OPCODES = 30
+MUFU_RCP64 = 30
+N_OPCODES = 31
 
 OPNAMES = [
     "NOP", "EXIT", "BRA", "MOV", "S2R", "IADD3", "IMAD", "IMAD.WIDE", "SHF", "LOP3", "SEL",
     "ISETP", "FSETP", "DSETP", "FADD", "FMUL", "FFMA", "FMNMX", "DADD", "DMUL", "DFMA",
-    "LDG", "LDC", "STG", "I2F", "F2I", "F2F.F64.F32", "F2F.F32.F64", "SHFL", "IMNMX",
+    "LDG", "LDC", "STG", "I2F", "F2I", "F2F.F64.F32", "F2F.F32.F64", "SHFL", "IMNMX", "MUFU.RCP64",
 ]
 
 RZ = 127          # zero register: reads 0, writes discarded
@@ -215,6 +216,9 @@ class Asm:
     def imnmx(self, d, a, b, is_max=False, unsigned=False, guard=PT):
         mod = (MOD_MAX if is_max else 0) | (MOD_CMP_U32 if unsigned else 0)
         return self.emit(IMNMX, d0=d, a=a, b=b, mod=mod, guard=guard)
+
+    def mufu_rcp64(self, d, a, guard=PT):
+        return self.emit(MUFU_RCP64, d0=d, a=a, guard=guard)
 
     def assemble(self) -> np.ndarray:
         code = np.array(self.rows, dtype=INSN_DTYPE)

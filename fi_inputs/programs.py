@@ -315,3 +315,213 @@ def multi_instance_chain(n_inst: int = 3, n: int = 256, block: int = 64, seed: i
         pb.add_instance(k, grid, block, ptr_words(x) + ptr_words(y) + ptr_words(ynew) + [n - shrink * i, isa.f32_bits(0.5)])
         y = ynew
     return pb.build(config="chain", n_inst=n_inst, n=n)
+
+
+# ---------------------------------------------------------------------------
+# C3: library-style FP64 conjugate gradient on a 2-D 5-point Laplacian
+# (mirrors 354.cg's many small kernels, ~5,000 dynamic instances)
+# ---------------------------------------------------------------------------
+def _vec_prologue(s: Asm, n_off: int, exit_out: bool = True):
+    s.s2r(0, isa.SR_TID)
+    s.s2r(1, isa.SR_CTAID)
+    s.s2r(2, isa.SR_NTID)
+    s.imad(0, 1, 2, 0)                             # i = ctaid*ntid + tid
+    s.ldc(3, n_off)
+    if exit_out:
+        s.isetp(0, 0, 3, cmp=isa.GE)
+        s.exit(guard=0)
+
+
+def cg_spmv_code(nx: int) -> np.ndarray:
+    """Ap = A p, A = 4I - shifts (Dirichlet): neighbour loads predicated on the
+    boundary (partial active masks on boundary rows).  cbank: p, Ap, n, nx-1,
+    log2 nx, ny-1, 4.0."""
+    s = Asm()
+    _vec_prologue(s, 16)
+    s.ldc(5, 20)                                   # nx - 1
+    s.ldc(6, 24)                                   # log2 nx
+    s.lop3(7, 0, 5, RZ, 0xC0)                      # ix = i & (nx-1)
+    s.shf(8, 0, 6, mode=isa.SHF_R_U32)             # iy = i >> log2 nx
+    s.ldc(10, 0, wide=True)
+    s.imad_wide(10, 0, imm=8, c=10, unsigned=True)
+    s.ldg(12, 10, 0, isa.W64)
+    s.ldc(16, 32, wide=True)                       # 4.0
+    s.dmul(14, 12, 16)
+    s.isetp(1, 7, imm=0, cmp=isa.GT)
+    s.ldg(18, 10, -8, isa.W64, guard=1)
+    s.dadd(14, 14, 18, negb=True, guard=1)
+    s.isetp(2, 7, 5, cmp=isa.LT)
+    s.ldg(18, 10, 8, isa.W64, guard=2)
+    s.dadd(14, 14, 18, negb=True, guard=2)
+    s.isetp(3, 8, imm=0, cmp=isa.GT)
+    s.ldg(18, 10, -8 * nx, isa.W64, guard=3)
+    s.dadd(14, 14, 18, negb=True, guard=3)
+    s.ldc(9, 28)                                   # ny - 1
+    s.isetp(4, 8, 9, cmp=isa.LT)
+    s.ldg(18, 10, 8 * nx, isa.W64, guard=4)
+    s.dadd(14, 14, 18, negb=True, guard=4)
+    s.ldc(20, 8, wide=True)
+    s.imad_wide(20, 0, imm=8, c=20, unsigned=True)
+    s.stg(20, 14, 0, isa.W64)
+    s.exit()
+    return s.assemble()
+
+
+def cg_dot_partial_code() -> np.ndarray:
+    """part[warp] = sum over the warp of a[i]*b[i] (SHFL.BFLY tree on f64 pairs).
+    cbank: a, b, part, n."""
+    s = Asm()
+    _vec_prologue(s, 24, exit_out=False)
+    s.mov(10, imm=0)
+    s.mov(11, imm=0)
+    s.isetp(0, 0, 3, cmp=isa.LT)
+    s.ldc(12, 0, wide=True, guard=0)
+    s.imad_wide(12, 0, imm=8, c=12, unsigned=True, guard=0)
+    s.ldg(14, 12, 0, isa.W64, guard=0)
+    s.ldc(16, 8, wide=True, guard=0)
+    s.imad_wide(16, 0, imm=8, c=16, unsigned=True, guard=0)
+    s.ldg(18, 16, 0, isa.W64, guard=0)
+    s.dmul(10, 14, 18, guard=0)
+    for d in (16, 8, 4, 2, 1):
+        s.shfl(20, 10, imm=d, mode=isa.SHFL_BFLY)
+        s.shfl(21, 11, imm=d, mode=isa.SHFL_BFLY)
+        s.dadd(10, 10, 20)
+    s.s2r(4, isa.SR_LANEID)
+    s.isetp(1, 4, imm=0, cmp=isa.EQ)
+    s.shf(5, 0, imm=5, mode=isa.SHF_R_U32)         # global warp index
+    s.ldc(22, 16, wide=True)
+    s.imad_wide(22, 5, imm=8, c=22, unsigned=True, guard=1)
+    s.stg(22, 10, 0, isa.W64, guard=1)
+    s.exit()
+    return s.assemble()
+
+
+def cg_dot_final_code() -> np.ndarray:
+    """out = sum of np partials: one warp, strided loop (lanes leave it at
+    different trip counts), SHFL.BFLY tree.  cbank: part, out, np."""
+    s = Asm()
+    s.s2r(0, isa.SR_TID)
+    s.mov(10, imm=0)
+    s.mov(11, imm=0)
+    s.ldc(3, 16)
+    s.ldc(12, 0, wide=True)
+    s.label("loop")
+    s.isetp(0, 0, 3, cmp=isa.GE)
+    s.bra("done", guard=0)
+    s.imad_wide(14, 0, imm=8, c=12, unsigned=True)
+    s.ldg(16, 14, 0, isa.W64)
+    s.dadd(10, 10, 16)
+    s.iadd3(0, 0, imm=32)
+    s.bra("loop")
+    s.label("done")
+    for d in (16, 8, 4, 2, 1):
+        s.shfl(20, 10, imm=d, mode=isa.SHFL_BFLY)
+        s.shfl(21, 11, imm=d, mode=isa.SHFL_BFLY)
+        s.dadd(10, 10, 20)
+    s.s2r(4, isa.SR_LANEID)
+    s.isetp(1, 4, imm=0, cmp=isa.EQ)
+    s.ldc(18, 8, wide=True)
+    s.stg(18, 10, 0, isa.W64, guard=1)
+    s.exit()
+    return s.assemble()
+
+
+def cg_scalar_code() -> np.ndarray:
+    """out = num * rcp(den) in lane 0 (alpha = rr/pAp, beta = rr'/rr).
+    cbank: num, den, out."""
+    s = Asm()
+    s.s2r(0, isa.SR_LANEID)
+    s.isetp(0, 0, imm=0, cmp=isa.NE)
+    s.exit(guard=0)
+    s.ldc(2, 0, wide=True)
+    s.ldg(4, 2, 0, isa.W64)
+    s.ldc(6, 8, wide=True)
+    s.ldg(8, 6, 0, isa.W64)
+    s.mufu_rcp64(10, 8)
+    s.dmul(12, 4, 10)
+    s.ldc(14, 16, wide=True)
+    s.stg(14, 12, 0, isa.W64)
+    s.exit()
+    return s.assemble()
+
+
+def cg_axpy_code(neg: bool) -> np.ndarray:
+    """out = (+-alpha) * p + x.  cbank: x, p, alpha, out, n."""
+    s = Asm()
+    _vec_prologue(s, 32)
+    s.ldc(2, 16, wide=True)
+    s.ldg(4, 2, 0, isa.W64)
+    s.ldc(6, 0, wide=True)
+    s.imad_wide(6, 0, imm=8, c=6, unsigned=True)
+    s.ldg(8, 6, 0, isa.W64)
+    s.ldc(10, 8, wide=True)
+    s.imad_wide(10, 0, imm=8, c=10, unsigned=True)
+    s.ldg(12, 10, 0, isa.W64)
+    s.dfma(14, 4, 12, 8, nega=neg)
+    s.ldc(16, 24, wide=True)
+    s.imad_wide(16, 0, imm=8, c=16, unsigned=True)
+    s.stg(16, 14, 0, isa.W64)
+    s.exit()
+    return s.assemble()
+
+
+def _f64_words(x: float) -> list[int]:
+    b = int(np.array([x], dtype="<f8").view("<u8")[0])
+    return [b & 0xFFFFFFFF, b >> 32]
+
+
+def cg_program(nx: int = 512, ny: int = 256, iters: int = 500, seed: int = DATA_SEED[3]) -> Program:
+    """CG for A x = b (x0 = 0, r0 = p0 = b), 10 launches per iteration, every
+    vector / partial / scalar a new SSA buffer version; output = the final x."""
+    assert nx & (nx - 1) == 0 and (nx * ny) % 256 == 0
+    n = nx * ny
+    nparts = n // 32
+    pb = ProgramBuilder(f"cg_{nx}x{ny}_it{iters}")
+    K = {}
+    for name, code in (("spmv_lap5", cg_spmv_code(nx)), ("dot_partial_b", cg_dot_partial_code()),
+                       ("dot_final_b", cg_dot_final_code()), ("dot_partial_pAp", cg_dot_partial_code()),
+                       ("dot_final_pAp", cg_dot_final_code()), ("scalar_alpha", cg_scalar_code()),
+                       ("axpy_x", cg_axpy_code(False)), ("axpy_r", cg_axpy_code(True)),
+                       ("dot_partial_rr", cg_dot_partial_code()), ("dot_final_rr", cg_dot_final_code()),
+                       ("scalar_beta", cg_scalar_code()), ("xpay_p", cg_axpy_code(False))):
+        K[name] = pb.add_kernel(name, code, nregs=24)
+    grid = n // 256
+    lg = nx.bit_length() - 1
+
+    def newbuf(name, nbytes, output=False):
+        return pb.add_buffer(name, nbytes, writer=len(pb.instances), output=output, dtype=isa.DT_F64)
+
+    def dot(kp, kf, a, b, tag):
+        part = newbuf(f"part_{tag}", 8 * nparts)
+        pb.add_instance(K[kp], grid, 256, ptr_words(a) + ptr_words(b) + ptr_words(part) + [n])
+        out = newbuf(f"dot_{tag}", 8)
+        pb.add_instance(K[kf], 1, 32, ptr_words(part) + ptr_words(out) + [nparts])
+        return out
+
+    b = pb.add_buffer("b", 8 * n, f64_data(seed, n), dtype=isa.DT_F64)
+    x = pb.add_buffer("x0", 8 * n, dtype=isa.DT_F64)                 # zeros, never written
+    r = p = b
+    rr = dot("dot_partial_b", "dot_final_b", r, r, "rr0")
+    for it in range(iters):
+        ap = newbuf(f"Ap{it}", 8 * n)
+        pb.add_instance(K["spmv_lap5"], grid, 256, ptr_words(p) + ptr_words(ap) + [n, nx - 1, lg, ny - 1] +
+                        _f64_words(4.0))
+        pap = dot("dot_partial_pAp", "dot_final_pAp", p, ap, f"pAp{it}")
+        alpha = newbuf(f"alpha{it}", 8)
+        pb.add_instance(K["scalar_alpha"], 1, 32, ptr_words(rr) + ptr_words(pap) + ptr_words(alpha))
+        last = it == iters - 1
+        xn = newbuf(f"x{it + 1}", 8 * n, output=last)
+        pb.add_instance(K["axpy_x"], grid, 256, ptr_words(x) + ptr_words(p) + ptr_words(alpha) + ptr_words(xn) + [n])
+        rn = newbuf(f"r{it + 1}", 8 * n)
+        pb.add_instance(K["axpy_r"], grid, 256, ptr_words(r) + ptr_words(ap) + ptr_words(alpha) + ptr_words(rn) + [n])
+        rrn = dot("dot_partial_rr", "dot_final_rr", rn, rn, f"rr{it + 1}")
+        beta = newbuf(f"beta{it}", 8)
+        pb.add_instance(K["scalar_beta"], 1, 32, ptr_words(rrn) + ptr_words(rr) + ptr_words(beta))
+        pn = newbuf(f"p{it + 1}", 8 * n)
+        pb.add_instance(K["xpay_p"], grid, 256, ptr_words(rn) + ptr_words(p) + ptr_words(beta) + ptr_words(pn) + [n])
+        x, r, p, rr = xn, rn, pn, rrn
+    return pb.build(config="C3", nx=nx, ny=ny, iters=iters, n=n)
+
+
+def c3(full: bool = True) -> Program:
+    return cg_program(512, 256, 500) if full else cg_program(32, 16, 6)

@@ -31,7 +31,7 @@ namespace {
 enum Op {
     NOP = 0, EXIT, BRA, MOV, S2R, IADD3, IMAD, IMAD_WIDE, SHF, LOP3, SEL,
     ISETP, FSETP, DSETP, FADD, FMUL, FFMA, FMNMX, DADD, DMUL, DFMA,
-    LDG, LDC, STG, I2F, F2I, F2F_F64_F32, F2F_F32_F64, SHFL, IMNMX, N_OPS
+    LDG, LDC, STG, I2F, F2I, F2F_F64_F32, F2F_F32_F64, SHFL, IMNMX, MUFU_RCP64, N_OPS
 };
 const int RZ = 127, PT = 7;
 const uint64_t VA_BASE = 0x00007F0000000000ull;       // C-15
@@ -56,7 +56,7 @@ void dest_regs(const orc_insn& I, std::vector<int>& gp, std::vector<int>& pr) {
             gpn(1);
             if ((I.d1 & 7) != PT) pr.push_back(I.d1 & 7);   // predicate fields are 3 bits (§3.1)
             break;
-        case IMAD_WIDE: case DADD: case DMUL: case DFMA: case F2F_F64_F32:
+        case IMAD_WIDE: case DADD: case DMUL: case DFMA: case F2F_F64_F32: case MUFU_RCP64:
             gpn(2); break;
         case LDG: gpn(1 << std::min(I.mod & 3, 2)); break;
         case LDC: gpn((I.mod & 1) ? 2 : 1); break;
@@ -388,6 +388,10 @@ WarpResult run_warp(const Prog& P, const std::vector<uint8_t>& mem, uint32_t k, 
                     }
                     v[0] = rd(W, (int)src, I.a); break;
                 }
+                case MUFU_RCP64: {                              // 1/x in f64, round to nearest (§3.2)
+                    uint64_t rb = b64(1.0 / f64(rd2(W, l, I.a)));
+                    v[0] = (uint32_t)rb; v[1] = (uint32_t)(rb >> 32); break;
+                }
                 case IMNMX: {
                     bool mx = I.mod & 1;
                     if (I.mod & 8) v[0] = mx ? std::max(a, b) : std::min(a, b);
@@ -410,7 +414,7 @@ WarpResult run_warp(const Prog& P, const std::vector<uint8_t>& mem, uint32_t k, 
                 case F2F_F32_F64: case SHFL: case IMNMX: case FADD: case FMUL: case FFMA: case FMNMX:
                     wr(W, l, I.d0, v[0]); break;
                 case IADD3: wr(W, l, I.d0, v[0]); pwr(W, l, I.d1, v[1]); break;
-                case IMAD_WIDE: case DADD: case DMUL: case DFMA: case F2F_F64_F32:
+                case IMAD_WIDE: case DADD: case DMUL: case DFMA: case F2F_F64_F32: case MUFU_RCP64:
                     wr(W, l, I.d0, v[0]); wr(W, l, I.d0 + 1, v[1]); break;
                 case LDG: { uint32_t nw = 1u << std::min(I.mod & 3, 2); for (uint32_t i = 0; i < nw; ++i) wr(W, l, I.d0 + i, v[i]); break; }
                 case LDC: wr(W, l, I.d0, v[0]); if (I.mod & 1) wr(W, l, I.d0 + 1, v[1]); break;

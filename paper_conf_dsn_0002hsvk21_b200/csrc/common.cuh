@@ -11,7 +11,7 @@ namespace fi {
 enum Op : uint32_t {
     NOP = 0, EXIT, BRA, MOV, S2R, IADD3, IMAD, IMAD_WIDE, SHF, LOP3, SEL,
     ISETP, FSETP, DSETP, FADD, FMUL, FFMA, FMNMX, DADD, DMUL, DFMA,
-    LDG, LDC, STG, I2F, F2I, F2F_F64_F32, F2F_F32_F64, SHFL, IMNMX
+    LDG, LDC, STG, I2F, F2I, F2F_F64_F32, F2F_F32_F64, SHFL, IMNMX, MUFU_RCP64
 };
 constexpr uint32_t kRZ = 127, kPT = 7;
 constexpr uint64_t kVaBase = 0x00007F0000000000ull;          // C-15
@@ -30,7 +30,7 @@ __host__ __device__ inline Dests dests_of(uint32_t op, uint32_t d0, uint32_t d1,
         case MOV: case S2R: case IMAD: case SHF: case LOP3: case SEL: case I2F: case F2I:
         case F2F_F32_F64: case SHFL: case IMNMX: case FADD: case FMUL: case FFMA: case FMNMX: case IADD3:
             n = 1; break;
-        case IMAD_WIDE: case DADD: case DMUL: case DFMA: case F2F_F64_F32: n = 2; break;
+        case IMAD_WIDE: case DADD: case DMUL: case DFMA: case F2F_F64_F32: case MUFU_RCP64: n = 2; break;
         case LDG: n = 1u << ((mod & 3) > 2 ? 2 : (mod & 3)); break;
         case LDC: n = (mod & 1) ? 2 : 1; break;
         default: n = 0;

@@ -369,6 +369,11 @@ __device__ __forceinline__ void exec_plain(const RegFile& F, const LaneCtx& L, c
             if (ex) F.wr(id, v);
             break;
         }
+        case MUFU_RCP64: {                            // 1/x in f64, round to nearest (§3.2)
+            const uint64_t b = dbits(__drcp_rn(u2d(F.rd64(ia))));
+            if (ex) { F.wr(id, (uint32_t)b); F.wr(id + 128, (uint32_t)(b >> 32)); }
+            break;
+        }
         case IMNMX: {
             const uint32_t a = F.rd(ia);
             uint32_t v;

@@ -311,6 +311,18 @@ def cases(seed=0):
         add(f"DSETP.{c}", rows_of(lambda s, c=c: s.dsetp(5, 0, 2, cmp=c)), w2,
             lambda w, t, c=c: out_words(pw=(int(not (math.isnan(f64(_pair(w, 0))) or math.isnan(f64(_pair(w, 2))))
                                                  and _cmp(f64(_pair(w, 0)), f64(_pair(w, 2)), c)) << 5)))
+    # MUFU.RCP64: correctly rounded 1/x (Python float division is IEEE RN)
+    w2 = rand_words64(rng)
+    def rcp(w, t):
+        x = f64(_pair(w, 0))
+        if x == 0.0:
+            r = bits64(math.copysign(math.inf, x))
+        elif math.isnan(x):
+            r = QNAN64
+        else:
+            r = bits64(1.0 / x)
+        return out_words(r & M32, r >> 32)
+    add("MUFU.RCP64", rows_of(lambda s: s.mufu_rcp64(8, 0)), w2, rcp)
     # conversions
     w = rand_words(rng, p=0.5)
     w[:6, 0] = [0x7FFFFFFF, 0x80000000, 0xFFFFFFFF, 16777217, 0x4F000000, 0xCF000001]

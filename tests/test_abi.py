@@ -56,7 +56,7 @@ def test_header_constants_match_input_format():
     from fi_inputs import isa
     names = ["NOP", "EXIT", "BRA", "MOV", "S2R", "IADD3", "IMAD", "IMAD_WIDE", "SHF", "LOP3", "SEL",
              "ISETP", "FSETP", "DSETP", "FADD", "FMUL", "FFMA", "FMNMX", "DADD", "DMUL", "DFMA",
-             "LDG", "LDC", "STG", "I2F", "F2I", "F2F_F64_F32", "F2F_F32_F64", "SHFL", "IMNMX"]
+             "LDG", "LDC", "STG", "I2F", "F2I", "F2F_F64_F32", "F2F_F32_F64", "SHFL", "IMNMX", "MUFU_RCP64"]
     for i, n in enumerate(names):
         assert getattr(isa, n) == i
     for path in ("paper_conf_dsn_0002hsvk21_b200/csrc/common.cuh", "oracle/oracle.cpp"):

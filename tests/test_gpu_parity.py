@@ -304,3 +304,21 @@ def test_multi_instance_injection_parity(F, maker, unchecked):
     gi, oi = _campaign_parity(F, maker(), 0x7A7, [F.G_GP, F.G_LD, F.G_FP32, F.G_OTHERS], [0, 1, 2, 3], 400,
                               O.MODE_FULL, unchecked=unchecked)
     assert (oi["outcome"] == O.SDC).sum() > 0
+
+
+def test_c3_mini_campaign_parity(F):
+    """mini-C3 (62 instances, 12 static kernels, SHFL reductions, divergent loops,
+    boundary predication): trace, counts, sites and whole-program outcomes (K7)
+    bit-exact against the oracle's full-program mode."""
+    gi, oi = _campaign_parity(F, P.c3(full=False), P.CAMPAIGN_SEED[3], [F.G_GP, F.G_FP64, F.G_PR, F.G_LD],
+                              [0, 1, 2, 3], 300, O.MODE_FULL)
+    assert len(np.unique(oi["outcome"])) >= 2
+
+
+def test_c3_mini_approximate(F):
+    prog = P.c3(full=False)
+    g = O.Golden(prog)
+    dp, gt = _gpu_golden(F, prog)
+    ap = F.profile_approx(gt).cpu().numpy().astype(np.uint64)
+    assert np.array_equal(ap, g.approx_counts())
+    assert np.array_equal(ap, g.counts())          # no data-dependent control flow in CG kernels

@@ -479,3 +479,45 @@ def test_approximate_profile_reuses_first_instance():
     r = g.inject(s, O.MODE_FULL)
     assert (r["outcome"][s["flags"] == 1] == O.NOT_INJECTED).all()
     assert (r["outcome"][s["flags"] == 0] != O.NOT_INJECTED).all()
+
+
+def test_c3_cg_numerics_and_structure():
+    """mini-C3 (FP64 CG, 2-D Laplacian): the oracle's golden x equals an
+    independent numpy CG of the same recurrences to 1e-12 (different summation
+    order / no FMA), counts satisfy Table II per instance, and instances of one
+    static kernel have identical counts (no data-dependent control flow)."""
+    nx, ny, iters = 32, 16, 6
+    prog = P.cg_program(nx, ny, iters)
+    g = O.Golden(prog)
+    img = g.final_image()
+    b = prog.view(img, "b", "<f8").copy()
+
+    def A(v):
+        V = v.reshape(ny, nx)
+        out = 4 * V.copy()
+        out[:, 1:] -= V[:, :-1]
+        out[:, :-1] -= V[:, 1:]
+        out[1:, :] -= V[:-1, :]
+        out[:-1, :] -= V[1:, :]
+        return out.ravel()
+
+    x, r, p = np.zeros_like(b), b.copy(), b.copy()
+    rr = r @ r
+    for _ in range(iters):
+        ap = A(p)
+        alpha = rr * (1.0 / (p @ ap))
+        x = x + alpha * p
+        r = r - alpha * ap
+        rrn = r @ r
+        beta = rrn * (1.0 / rr)
+        p = r + beta * p
+        rr = rrn
+    xg = prog.view(img, f"x{iters}", "<f8")
+    assert np.allclose(xg, x, rtol=1e-12, atol=1e-12)
+    c = g.counts()
+    _invariants(c)
+    kern = prog.instances["kernel"]
+    for k in np.unique(kern):
+        rows = c[kern == k]
+        assert (rows == rows[0]).all()
+    assert (c[:, FP64] > 0).sum() >= 6 and len(np.unique(kern)) == 12
