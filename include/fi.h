@@ -263,6 +263,40 @@ fi_status fi_classify(const fi_program* p, const uint8_t* image, const fi_trace*
                       uint32_t n, fi_inj* out, const fi_store* log, uint32_t log_cap, uint64_t* hist,
                       uint32_t flags, void* ws, size_t ws_bytes, uint32_t* dev_status, void* stream);
 
+/* §8 rows f2/f3 — permanent faults (Table III
+ * [PAPER.md:128-134]) and intermittent faults.  A fault is
+ * {opcode id, SM id, lane id, XOR bit mask}: the destination registers of every
+ * dynamic instance of the opcode executed in that lane by the CTAs on that SM
+ * (CTA c of an instance runs on SM c mod n_sm, reading C-21) are XOR-ed with the
+ * same mask (a predicate destination flips iff mask bit 0 is set).  q32 != 0
+ * makes it intermittent: an instance is corrupted only when
+ * Philox4x32-10(ctr = {warp, step, replica, 0x46490002}, key = seed).x < q32
+ * (reading C-22).  Every run re-executes the affected warps of every instance
+ * (plus, as in K7, every later instance that may read corrupted words) and is
+ * classified on the whole program (Table V).  hist[3] (u64) accumulates
+ * op_weights[opcode] per outcome — the opcode-weighted outcomes of PAPER.md:228
+ * (1 per run when op_weights is NULL).
+ * A permanent fault can corrupt many words: ov_words bounds the distinct
+ * corrupted words one run may hold (e.g. image_bytes/4; 0 = the transient
+ * default, max(log_cap, 4096)); a run that exceeds it gets outcome 0xFF and
+ * FI_E_CAPACITY.  Scratch: fi_inject_permanent_workspace(n, log_cap, ov_words,
+ * max_slots) bytes — max_slots (0 = as many as can be resident, else >= 4)
+ * caps the replicas in flight and so the scratch; the call uses as many slots
+ * as ws_bytes holds (at least 4).  faults/op_weights/out/log/hist/ws/dev_status
+ * are device pointers; out[i].mask = faults[i].mask, fault_kind/fault_pc the
+ * first fault (DUE) or the first non-fatal one (FI_POTENTIAL_DUE). */
+typedef struct {
+    uint32_t opcode, sm, lane, mask;
+    uint32_t q32;                                    /* 0 = permanent; else activation probability * 2^32 */
+    uint32_t n_sm;                                   /* SMs of the modelled GPU (148 for B200) */
+    uint64_t seed;
+} fi_pfault;                                         /* 32 B */
+size_t fi_inject_permanent_workspace(uint32_t n, uint32_t log_cap, uint32_t ov_words, uint32_t max_slots);
+fi_status fi_inject_permanent(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_pfault* faults,
+                              uint32_t n, const uint64_t* op_weights, fi_inj* out, fi_store* log, uint32_t log_cap,
+                              uint32_t ov_words, uint64_t* hist, uint32_t flags, void* ws, size_t ws_bytes,
+                              uint32_t* dev_status, void* stream);
+
 /* Table II parameter file, one parameter per line in Table II order
  * [PAPER.md:88]: arch state id, bit-flip model, kernel name, kernel count,
  * instruction count, destination register value, bit-pattern value (the two

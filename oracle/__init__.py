@@ -45,7 +45,9 @@ SITE_DTYPE = np.dtype([
 INJ_DTYPE = np.dtype([("before", "<u4"), ("after", "<u4"), ("mask", "<u4"), ("fault_pc", "<u4"),
                       ("fault_kind", "u1"), ("outcome", "u1"), ("flags", "u1"), ("pad", "u1"),
                       ("n_faulty_stores", "<u4")])
-assert SITE_DTYPE.itemsize == 64 and INJ_DTYPE.itemsize == 24
+PFAULT_DTYPE = np.dtype([("opcode", "<u4"), ("sm", "<u4"), ("lane", "<u4"), ("mask", "<u4"), ("q32", "<u4"),
+                         ("n_sm", "<u4"), ("seed", "<u8")])
+assert SITE_DTYPE.itemsize == 64 and INJ_DTYPE.itemsize == 24 and PFAULT_DTYPE.itemsize == 32
 
 
 class _Program(C.Structure):
@@ -100,6 +102,8 @@ def lib():
             L.orc_approx_counts.argtypes = [vp, vp]
             L.orc_select_approx.argtypes = [vp, u64, vp, u32, vp, u32, u64, u32, vp]
             L.orc_inject.argtypes = [vp, vp, u32, i32, i32, vp]
+            L.orc_inject_permanent.argtypes = [vp, vp, u32, i32, i32, vp]
+            L.orc_permanent_image.argtypes = [vp, vp, u32, i32, vp]
             L.orc_warp_site_rank.argtypes = [C.POINTER(_Program), u32, i32, u32, u32, C.POINTER(u64), C.POINTER(u64)]
             L.orc_inject_local.argtypes = [C.POINTER(_Program), vp, u32, i32, vp, vp]
             L.orc_warp_site_at.argtypes = [C.POINTER(_Program), u32, i32, u64, C.POINTER(u32), C.POINTER(u32),
@@ -210,6 +214,20 @@ class Golden:
         if rc:
             raise OracleError(rc, lib().orc_error(self.h).decode())
         return out
+
+    def inject_permanent(self, faults: np.ndarray, mode: int = MODE_FULL, n_threads: int | None = None) -> np.ndarray:
+        """Rows f2/f3 by the definition: whole-program re-run per fault."""
+        faults = np.ascontiguousarray(faults, dtype=PFAULT_DTYPE)
+        out = np.zeros(len(faults), dtype=INJ_DTYPE)
+        lib().orc_inject_permanent(self.h, _ptr(faults), len(faults), mode, n_threads or n_threads_default(), _ptr(out))
+        return out
+
+    def permanent_image(self, fault, rep: int = 0, mode: int = MODE_FULL):
+        """(fault kind, faulty final image) of replica `rep` of one permanent fault."""
+        f = np.ascontiguousarray(np.asarray(fault, dtype=PFAULT_DTYPE).reshape(1))
+        img = np.zeros_like(self.final_image())
+        k = lib().orc_permanent_image(self.h, _ptr(f), rep, mode, _ptr(img))
+        return k, img
 
     def locate(self, group: int, s) -> np.ndarray:
         s = np.ascontiguousarray(s, dtype=np.uint64)

@@ -218,7 +218,15 @@ struct Hook {
     uint64_t step = 0; int lane = 0; int kind = 0; int reg = 0; int bfm = 0; uint32_t mask = 0; uint32_t pc = 0;
     bool fired = false, bad = false;
     uint32_t before = 0, after = 0, applied_mask = 0;
+    // permanent / intermittent fault (rows f2/f3): every executed instance of
+    // `perm_op` in lane `perm_lane` of this warp gets its destinations XOR-ed
+    bool perm = false;
+    uint32_t perm_op = 0, perm_lane = 0, perm_mask = 0, perm_q = 0, perm_rep = 0;
+    uint64_t perm_seed = 0;
 };
+
+// The permanent-fault spec of one run (Table III [PAPER.md:128-134]).
+struct PermSpec { uint32_t opcode, sm, lane, mask, q32, n_sm, rep; uint64_t seed; };
 
 // Find the allocation containing [va, va+w).  C-15: valid iff aligned to the
 // access width and fully inside one allocation.  Returns 0 ok, 1 misaligned, 2 unmapped.
@@ -450,6 +458,26 @@ WarpResult run_warp(const Prog& P, const std::vector<uint8_t>& mem, uint32_t k, 
                 pwr(W, l, hook->reg, after != 0);
             }
         }
+        // permanent fault: the same XOR mask on the destination
+        // registers of every dynamic instance of the opcode in the faulty lane;
+        // intermittent: only instances whose Philox draw is below q
+        if (hook && hook->perm && I.op == hook->perm_op && ((ex >> hook->perm_lane) & 1)) {
+            bool fire = true;
+            if (hook->perm_q) {
+                uint32_t wg = in.warp_begin + cta * ((in.block + 31) / 32) + wic;
+                uint32_t ctr[4] = {wg, (uint32_t)step, hook->perm_rep, 0x46490002u};
+                uint32_t key[2] = {(uint32_t)hook->perm_seed, (uint32_t)(hook->perm_seed >> 32)}, o[4];
+                philox(ctr, key, o);
+                fire = o[0] < hook->perm_q;
+            }
+            if (fire) {
+                std::vector<int> gp, pr;
+                dest_regs(I, gp, pr);
+                int l = hook->perm_lane;
+                for (int r : gp) wr(W, l, r, rd(W, l, r) ^ hook->perm_mask);
+                if (hook->perm_mask & 1) for (int p : pr) pwr(W, l, p, !prd(W, l, p));
+            }
+        }
         ++step;
     }
     res.steps = step;
@@ -522,7 +550,7 @@ struct FullRun {
 void run_program(const Golden* G, const Prog& P, Hook* hook, uint32_t hook_warp, int n_threads, FullRun& out,
                  std::vector<uint64_t>* wlen_out, std::vector<uint64_t>* wcounts, bool keep_trace,
                  std::vector<std::vector<orc_record>>* wtraces, uint64_t* n_gstores, std::string* err,
-                 bool unchecked = false) {
+                 bool unchecked = false, const PermSpec* perm = nullptr) {
     out.mem.assign(P.p.init_image, P.p.init_image + P.p.image_bytes);
     for (uint32_t k = 0; k < P.p.n_inst && !out.fault; ++k) {
         const orc_instance& in = P.p.inst[k];
@@ -536,12 +564,19 @@ void run_program(const Golden* G, const Prog& P, Hook* hook, uint32_t hook_warp,
             TraceSink ts;
             std::vector<orc_record> tr;
             if (keep_trace) ts.rec = &tr;
-            rr[i] = run_warp(P, out.mem, k, cta, wic, (hook && w == hook_warp) ? hook : nullptr, wd, &st[i],
+            Hook ph;                                     // permanent fault: CTAs on the faulty SM (C-21)
+            Hook* h = (hook && w == hook_warp) ? hook : nullptr;
+            if (perm && cta % perm->n_sm == perm->sm) {
+                ph.perm = true; ph.perm_op = perm->opcode; ph.perm_lane = perm->lane; ph.perm_mask = perm->mask;
+                ph.perm_q = perm->q32; ph.perm_rep = perm->rep; ph.perm_seed = perm->seed;
+                h = &ph;
+            }
+            rr[i] = run_warp(P, out.mem, k, cta, wic, h, wd, &st[i],
                              keep_trace ? &ts : nullptr, wcounts ? &(*wcounts)[8 * (size_t)w] : nullptr);
             if (wlen_out) (*wlen_out)[w] = rr[i].steps;
             if (keep_trace) (*wtraces)[w] = std::move(tr);
         };
-        if (hook) for (uint32_t i = 0; i < nw; ++i) body(i);       // replica-level parallelism instead
+        if (hook || perm) for (uint32_t i = 0; i < nw; ++i) body(i);   // replica-level parallelism instead
         else parallel_for(nw, n_threads, body);
         for (uint32_t i = 0; i < nw; ++i) {
             if (!rr[i].fault) continue;
@@ -1042,4 +1077,41 @@ extern "C" int orc_inject_local(const orc_program* p, const orc_site* sites, uin
         if (!sdc && unknown) decided[i] = 0;
     });
     return status;
+}
+
+// Rows f2/f3: permanent / intermittent faults by the definition — the whole
+// program re-run with the fault armed on every warp of every CTA mapped to the
+// faulty SM (CTA c on SM c mod n_sm, reading C-21), outputs compared bitwise
+// with the golden run (Table V), DUE taking precedence (C-9, C-10; f4 under
+// ORC_UNCHECKED).
+extern "C" int orc_inject_permanent(void* h, const orc_pfault* pf, uint32_t n, int mode, int n_threads, orc_inj* out) {
+    Golden* G = (Golden*)h;
+    const Prog& P = G->P;
+    const bool unchecked = mode & ORC_UNCHECKED;
+    parallel_for(n, n_threads, [&](uint32_t i) {
+        orc_inj& R = out[i];
+        memset(&R, 0, sizeof(R));
+        PermSpec ps{pf[i].opcode, pf[i].sm, pf[i].lane, pf[i].mask, pf[i].q32, pf[i].n_sm ? pf[i].n_sm : 148, i,
+                    pf[i].seed};
+        FullRun fr;
+        run_program(G, P, nullptr, 0, 1, fr, nullptr, nullptr, false, nullptr, nullptr, nullptr, unchecked, &ps);
+        R.mask = pf[i].mask;
+        if (fr.fault) { R.outcome = ORC_DUE; R.fault_kind = (uint8_t)fr.fault; R.fault_pc = fr.fault_pc; return; }
+        R.flags = fr.pdue ? ORC_POTENTIAL_DUE : 0;
+        R.fault_kind = (uint8_t)fr.pdue; R.fault_pc = fr.pdue_pc;
+        R.outcome = output_differs(P, fr.mem, G->final_mem) ? ORC_SDC : ORC_MASKED;
+    });
+    return 0;
+}
+
+// The faulty final image of one permanent / intermittent fault replica `rep`
+// (test pins of rows f2/f3).  Returns the fault kind (0 = none).
+extern "C" int orc_permanent_image(void* h, const orc_pfault* pf, uint32_t rep, int mode, uint8_t* out_image) {
+    Golden* G = (Golden*)h;
+    PermSpec ps{pf->opcode, pf->sm, pf->lane, pf->mask, pf->q32, pf->n_sm ? pf->n_sm : 148, rep, pf->seed};
+    FullRun fr;
+    run_program(G, G->P, nullptr, 0, 1, fr, nullptr, nullptr, false, nullptr, nullptr, nullptr,
+                (mode & ORC_UNCHECKED) != 0, &ps);
+    std::copy(fr.mem.begin(), fr.mem.end(), out_image);
+    return fr.fault ? fr.fault : fr.pdue;
 }

@@ -99,6 +99,11 @@ int orc_select_approx(void* h, uint64_t seed, const uint8_t* groups, uint32_t n_
 /* injection + classification; mode ORC_MODE_FULL re-runs the whole program */
 int orc_inject(void* h, const orc_site* sites, uint32_t n, int mode, int n_threads, orc_inj* out);
 
+/* rows f2/f3: permanent / intermittent faults (Table III) */
+typedef struct { uint32_t opcode, sm, lane, mask, q32, n_sm; uint64_t seed; } orc_pfault;   /* 32 B */
+int orc_inject_permanent(void* h, const orc_pfault* pf, uint32_t n, int mode, int n_threads, orc_inj* out);
+int orc_permanent_image(void* h, const orc_pfault* pf, uint32_t rep, int mode, uint8_t* out_image);
+
 /* single-instance, no golden handle (full-size sampled parity, CPU baselines) */
 int orc_warp_site_rank(const orc_program* p, uint32_t w, int g, uint32_t step, uint32_t lane,
                        uint64_t* rank, uint64_t* total);

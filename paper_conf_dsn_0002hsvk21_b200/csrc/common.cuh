@@ -75,6 +75,20 @@ __host__ __device__ inline uint32_t bfm_mask(uint32_t bfm, uint32_t u) {
     }
 }
 
+#ifdef __CUDACC__
+// Philox4x32-10 (Salmon et al. 2011), the counter-based RNG of every draw (C-5)
+__device__ __forceinline__ uint4 philox4x32_10(uint4 c, uint2 k) {
+#pragma unroll
+    for (int r = 0; r < 10; ++r) {
+        if (r) { k.x += 0x9E3779B9u; k.y += 0xBB67AE85u; }
+        const uint32_t hi0 = __umulhi(0xD2511F53u, c.x), lo0 = 0xD2511F53u * c.x;
+        const uint32_t hi1 = __umulhi(0xCD9E8D57u, c.z), lo1 = 0xCD9E8D57u * c.z;
+        c = make_uint4(hi1 ^ c.y ^ k.x, lo1, hi0 ^ c.w ^ k.y, lo0);
+    }
+    return c;
+}
+#endif
+
 }  // namespace fi
 
 // error plumbing for the host side of the ABI

@@ -111,7 +111,15 @@ inline EmuProg make_emu_prog(const fi_program* p) {
 // checkpoint = (n_regs + 3) rows of 32 words: registers, then pc, predicates, live
 __host__ __device__ inline size_t ckpt_bytes(uint32_t n_regs) { return (size_t)(n_regs + 3) * 128; }
 
-struct HookIn { uint32_t step, lane, kind, reg, bfm, mask, pc; };
+struct HookIn {
+    uint32_t step, lane, kind, reg, bfm, mask, pc;   // transient site (EMU_INJ)
+    // permanent / intermittent fault (EMU_PROP, rows f2/f3): every executed dynamic
+    // instance of perm_op in lane perm_lane has its destinations XOR-ed with
+    // perm_mask; intermittent: only when Philox(warp, step, rep) < perm_q
+    bool perm_on;
+    uint32_t perm_op, perm_lane, perm_mask, perm_q, perm_rep, perm_warp;
+    uint64_t perm_seed;
+};
 
 struct EmuOut {
     uint32_t steps = 0, fault = 0, fault_pc = 0, nstore = 0;
@@ -432,6 +440,9 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
     const RegFile F{reinterpret_cast<char*>(R + lane), R, zr * 128};
     const LaneCtx LC{lane, cta, wic, in.block, in.grid, in.cbank_len, P.cbank + in.cbank_off};
     const bool use_ck = ck != nullptr && ck_interval != 0;
+    // permanent / intermittent hook (row f2/f3): every step is inspected, so the
+    // straight-line fast paths are off while it is armed
+    const bool perm = MODE == EMU_PROP && hook.perm_on;
 
     uint32_t nl = in.block - wic * 32;
     bool live = lane < (nl > 32 ? 32u : nl);
@@ -479,7 +490,7 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
         if (step >= watchdog) { o.fault = 3; o.fault_pc = pcm; break; }
         if (pcm >= kn.code_len) { o.fault = 4; o.fault_pc = pcm; break; }
 
-        if (conv) {
+        if (conv && !perm) {
             // ---- straight-line run: no scheduling / control bookkeeping per step
             const uint32_t rw = __ldg(&runl[pcm]);
             uint32_t run = rw & 0xFFFF, lr = (rw >> 16) & 0xFF, fr = rw >> 24;
@@ -696,6 +707,22 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
             pc = ((taken >> lane) & 1u) ? imm : pcm + 1;
         }
 
+        if (perm && op == hook.perm_op && lane == hook.perm_lane && ex) {
+            // permanent fault: same XOR mask on the destination
+            // registers of every dynamic instance; intermittent: a
+            // random subset of them (reading C-21 / C-22)
+            bool fire = true;
+            if (hook.perm_q) {
+                const uint4 r = philox4x32_10(make_uint4(hook.perm_warp, step, hook.perm_rep, 0x46490002u),
+                                              make_uint2((uint32_t)hook.perm_seed, (uint32_t)(hook.perm_seed >> 32)));
+                fire = r.x < hook.perm_q;
+            }
+            if (fire) {
+                const Dests dd = dests_of(op, id == 0xFFFFu ? kRZ : id / 128, D.x >> 24, mod);
+                for (uint32_t q = 0; q < dd.n_gp; ++q) F.wr(id + 128 * q, F.rd(id + 128 * q) ^ hook.perm_mask);
+                if (dd.has_pr && (hook.perm_mask & 1u)) preds ^= 1u << dd.pr;
+            }
+        }
         if (MODE == EMU_INJ && step == hook.step) {
             // transient fault: corrupt one destination of this dynamic
             // instruction in one lane, after the instruction wrote it (C-7, C-8)

@@ -255,10 +255,12 @@ extern "C" fi_status fi_inject(const fi_program* p, const uint8_t* image, const 
 
 namespace fi {
 size_t propagate_slot_bytes(uint32_t ov_cap, uint32_t pend_cap);
+void propagate_caps(uint32_t log_cap, uint32_t ov_words, uint32_t& ov_cap, uint32_t& pend_cap);
 fi_status launch_propagate(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
                            uint32_t n, fi_inj* out, const fi_store* log, uint32_t log_cap, uint64_t* hist,
                            uint32_t flags, void* ws, size_t ws_bytes, const uint32_t* order, uint32_t* counter,
-                           uint32_t* dev_status, cudaStream_t s);
+                           uint32_t* dev_status, cudaStream_t s, const fi_pfault* pf, const uint64_t* opw,
+                           uint32_t ov_words);
 namespace {
 __global__ void k_iota(uint32_t* order, uint32_t n, uint32_t* counter) {
     const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
@@ -270,9 +272,9 @@ __global__ void k_iota(uint32_t* order, uint32_t n, uint32_t* counter) {
 
 extern "C" size_t fi_classify_workspace(uint32_t n_inst, uint32_t n, uint32_t log_cap) {
     if (n_inst <= 1 || n == 0) return 0;
-    uint32_t ov_cap = 1;
-    while (ov_cap < 4 * std::max<uint32_t>(log_cap, 4096)) ov_cap <<= 1;
-    const size_t sb = propagate_slot_bytes(ov_cap, 2 * std::max<uint32_t>(log_cap, 4096));
+    uint32_t ov_cap, pend_cap;
+    propagate_caps(log_cap, 0, ov_cap, pend_cap);
+    const size_t sb = propagate_slot_bytes(ov_cap, pend_cap);
     const uint64_t slots = std::min<uint64_t>(((uint64_t)n + 3) / 4 * 4, 148ull * 16);   // <= resident warps
     return 256 + align256((size_t)n * 4) + slots * sb;
 }
@@ -293,7 +295,7 @@ extern "C" fi_status fi_classify(const fi_program* p, const uint8_t* image, cons
         fi_status e = launch_status();
         if (e) return e;
         return launch_propagate(p, image, t, sites, n, out, log, log_cap, hist, flags, reinterpret_cast<char*>(ws) + head,
-                                ws_bytes - head, order, counter, dev_status, s);
+                                ws_bytes - head, order, counter, dev_status, s, nullptr, nullptr, 0);
     }
     const EmuProg P = make_emu_prog(p);
     ClsArgs A{p->buf, P.gran, image, t->gstore, t->gstore_off, sites, out, n, log, log_cap, hist, flags, dev_status};

@@ -42,6 +42,8 @@ struct PropArgs {
     uint32_t* dbuf;                                  // per warp-slot: [count, ids...]
     uint32_t* ov_list; uint32_t list_cap;            // per warp-slot: slots in use (for scans)
     uint64_t* hist; uint32_t flags; uint32_t* status;
+    const fi_pfault* pf;                             // permanent / intermittent faults (rows f2/f3), else null
+    const uint64_t* opw;                             // opcode weights [FI_NOPS] or null
 };
 
 __device__ __forceinline__ uint32_t buf_id(const EmuProg& P, uint64_t va) { return __ldg(&P.gran[(va - kVaBase) >> 8]); }
@@ -144,9 +146,12 @@ __global__ void __launch_bounds__(kWPB * 32) k_propagate(const PropArgs A) {
         if (p >= A.n) return;
         const uint32_t i = A.order[p];
         const uint32_t gen = p + 1;
-        const fi_site S = A.sites[i];
-        const fi_inj Rj = A.inj[i];
-        uint32_t outcome = FI_MASKED;
+        const bool permanent = A.pf != nullptr;
+        const fi_site S = permanent ? fi_site{} : A.sites[i];
+        const fi_inj Rj = permanent ? fi_inj{} : A.inj[i];
+        const fi_pfault PF = permanent ? A.pf[i] : fi_pfault{};
+        const uint32_t nsm = PF.n_sm ? PF.n_sm : 148u;      // CTA c runs on SM c mod n_sm (C-21)
+        uint32_t outcome = FI_MASKED, fkind = 0, fpc = 0;
         bool pdue = false, overflow = false;
         const bool unchecked = A.flags & FI_UNCHECKED;
         if (S.flags & FI_SITE_NOT_INJECTED) {
@@ -159,20 +164,24 @@ __global__ void __launch_bounds__(kWPB * 32) k_propagate(const PropArgs A) {
             pdue = Rj.fault_kind != 0;
             uint32_t ndb = 0, nlist = 0;
             bool db_over = false;
-            // ---- 1. the faulty warp's instance
-            const fi_store* G = A.gst + A.gst_off[S.warp];
-            const uint64_t nGall = A.gst_off[S.warp + 1] - A.gst_off[S.warp];
-            uint64_t gs = 0;
-            for (uint64_t b = 0; b < nGall; b += 32) {
-                const bool after = b + lane < nGall && G[b + lane].step > S.step;
-                const uint32_t m = __ballot_sync(kFull, after);
-                if (m) { gs = b + __ffs(m) - 1; break; }
-                gs = min(b + 32, nGall);
-            }
             uint32_t np = 0;
-            bool ok = warp_updates(A, ov, A.log + (uint64_t)i * A.cap, Rj.n_faulty_stores, G + gs, nGall - gs,
-                                   S.instance, pend, np);
-            int64_t t = S.instance;
+            bool ok = true;
+            int64_t t = -1;
+            if (!permanent) {
+                // ---- 1. the faulty warp's instance
+                const fi_store* G = A.gst + A.gst_off[S.warp];
+                const uint64_t nGall = A.gst_off[S.warp + 1] - A.gst_off[S.warp];
+                uint64_t gs = 0;
+                for (uint64_t b = 0; b < nGall; b += 32) {
+                    const bool after = b + lane < nGall && G[b + lane].step > S.step;
+                    const uint32_t m = __ballot_sync(kFull, after);
+                    if (m) { gs = b + __ffs(m) - 1; break; }
+                    gs = min(b + 32, nGall);
+                }
+                ok = warp_updates(A, ov, A.log + (uint64_t)i * A.cap, Rj.n_faulty_stores, G + gs, nGall - gs,
+                                  S.instance, pend, np);
+                t = S.instance;
+            }
             bool done = false;
             while (!done) {
                 // ---- apply the pending updates of instance t (end-of-instance visibility)
@@ -206,10 +215,13 @@ __global__ void __launch_bounds__(kWPB * 32) k_propagate(const PropArgs A) {
                     }
                     diff = __any_sync(kFull, d);
                 }
-                if (!diff) break;
-                // ---- next instance that references a dirty buffer
+                if (!diff && !permanent) break;              // a permanent fault keeps firing later
+                // ---- next instance that references a dirty buffer (or, for a
+                //      permanent fault, runs the opcode on the faulty SM)
                 int64_t nk = t + 1;
+                bool all = false;
                 for (; nk < (int64_t)A.n_inst; ++nk) {
+                    all = true;
                     if (db_over) break;
                     ibl = A.P.ib + (size_t)nk * (kInstBufs + 1);
                     const uint32_t cnt = __ldg(&ibl[0]);
@@ -220,23 +232,43 @@ __global__ void __launch_bounds__(kWPB * 32) k_propagate(const PropArgs A) {
                         hit = d < ndb && __ldg(&ibl[1 + a]) == dbuf[1 + d];
                     }
                     if (__any_sync(kFull, hit)) break;
+                    all = false;
+                    if (permanent) {
+                        const fi_instance ink = A.P.inst[nk];
+                        if (PF.sm >= nsm || PF.sm >= ink.grid) continue;              // no CTA of nk runs on the faulty SM
+                        const fi_kernel kn = A.P.kern[ink.kernel];
+                        bool has = false;
+                        for (uint32_t q = lane; q < kn.code_len && !has; q += 32)
+                            has = (__ldg(&A.P.dec[kn.code_off + q].x) & 0xFF) == PF.opcode;
+                        if (__any_sync(kFull, has)) break;
+                    }
                 }
                 if (nk >= (int64_t)A.n_inst) break;
-                // ---- re-execute every warp of instance nk against the overlay
+                // ---- re-execute the warps of instance nk against the overlay: all of
+                //      them when it may read dirty words, else the faulty SM's
                 t = nk;
                 const fi_instance in = A.P.inst[t];
                 const uint32_t wpc = (in.block + 31) / 32;
                 np = 0;
                 for (uint32_t w = in.warp_begin; w < in.warp_end && ok; ++w) {
                     const uint32_t lw = w - in.warp_begin;
+                    const bool hooked = permanent && (lw / wpc) % nsm == PF.sm;
+                    if (!all && !hooked) continue;
                     const uint64_t L = A.warp_off[w + 1] - A.warp_off[w];
                     const uint64_t wd = 10 * L + 1024;
                     const uint32_t watchdog = wd > 0xFFFFFFFFull ? 0xFFFFFFFFu : (uint32_t)wd;
                     HookIn h{};
+                    if (hooked) {
+                        h.perm_on = true; h.perm_op = PF.opcode; h.perm_lane = PF.lane; h.perm_mask = PF.mask;
+                        h.perm_q = PF.q32; h.perm_rep = i; h.perm_warp = w; h.perm_seed = PF.seed;
+                    }
                     fi_store* flog = A.log + (uint64_t)i * A.cap;
                     const EmuOut o = emulate<EMU_PROP>(A.P, nullptr, A.img, (uint32_t)t, lw / wpc, lw % wpc, R,
                                                        watchdog, nullptr, flog, A.cap, h, nullptr, 0, ov);
-                    if (o.fault && !(unchecked && o.fault != 3)) { outcome = FI_DUE; done = true; break; }
+                    if (o.fault && !fkind) { fkind = o.fault; fpc = o.fault_pc; }
+                    if (o.fault && !(unchecked && o.fault != 3)) {
+                        outcome = FI_DUE; fkind = o.fault; fpc = o.fault_pc; done = true; break;
+                    }
                     if (o.fault) pdue = true;
                     if (o.nstore > A.cap) { overflow = true; done = true; break; }
                     ok = warp_updates(A, ov, flog, o.nstore, A.gst + A.gst_off[w], A.gst_off[w + 1] - A.gst_off[w],
@@ -261,9 +293,19 @@ __global__ void __launch_bounds__(kWPB * 32) k_propagate(const PropArgs A) {
             }
         }
         if (lane == 0) {
+            if (permanent) {
+                fi_inj r = {};
+                r.mask = PF.mask;
+                r.fault_kind = (uint8_t)fkind;
+                r.fault_pc = fpc;
+                A.inj[i] = r;
+            }
             A.inj[i].outcome = (uint8_t)outcome;
             A.inj[i].flags = (pdue && outcome != FI_DUE && outcome != FI_NOT_INJECTED) ? FI_POTENTIAL_DUE : 0;
             if (outcome == 0xFF) FI_DEV_ERR(A.status, FI_E_CAPACITY);
+            else if (permanent)                     // opcode-weighted outcomes
+                atomicAdd((unsigned long long*)&A.hist[outcome],
+                          (unsigned long long)(A.opw ? A.opw[PF.opcode & (FI_NOPS - 1)] : 1ull));
             else if (outcome != FI_NOT_INJECTED)
                 atomicAdd((unsigned long long*)&A.hist[((uint32_t)S.group * 4 + S.bfm) * 3 + outcome], 1ull);
         }
@@ -273,6 +315,17 @@ __global__ void __launch_bounds__(kWPB * 32) k_propagate(const PropArgs A) {
 
 }  // namespace
 
+// Per replica slot: overlay of a power-of-two capacity (load <= 1/2 for
+// ov_words differing words; a transient fault's words are bounded by its log),
+// the pending-update list of one instance.
+void propagate_caps(uint32_t log_cap, uint32_t ov_words, uint32_t& ov_cap, uint32_t& pend_cap) {
+    const uint64_t words = std::max<uint64_t>({(uint64_t)log_cap, 4096ull, (uint64_t)ov_words});
+    uint64_t c = 1;
+    while (c < (ov_words ? 2 : 4) * words) c <<= 1;
+    ov_cap = (uint32_t)std::min<uint64_t>(c, 1ull << 31);
+    pend_cap = (uint32_t)std::min<uint64_t>(ov_words ? words + 2ull * log_cap : 2 * words, 0xFFFFFFFFull);
+}
+
 size_t propagate_slot_bytes(uint32_t ov_cap, uint32_t pend_cap) {
     return (size_t)ov_cap * 16 + (size_t)pend_cap * 16 + (kDirtyBufs + 1) * 4 + ((size_t)ov_cap + 1) * 4;
 }
@@ -280,7 +333,8 @@ size_t propagate_slot_bytes(uint32_t ov_cap, uint32_t pend_cap) {
 fi_status launch_propagate(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
                            uint32_t n, fi_inj* out, const fi_store* log, uint32_t log_cap, uint64_t* hist,
                            uint32_t flags, void* ws, size_t ws_bytes, const uint32_t* order, uint32_t* counter,
-                           uint32_t* dev_status, cudaStream_t s) {
+                           uint32_t* dev_status, cudaStream_t s, const fi_pfault* pf, const uint64_t* opw,
+                           uint32_t ov_words) {
     const size_t smem = golden_smem(p->n_regs);
     fi_status e = cuda_status(cudaFuncSetAttribute((const void*)k_propagate, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     if (e) return e;
@@ -288,10 +342,8 @@ fi_status launch_propagate(const fi_program* p, const uint8_t* image, const fi_t
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_propagate, kWPB * 32, smem);
-    // overlay capacity: a power of two; slots limited by the workspace
-    uint32_t ov_cap = 1;
-    while (ov_cap < 4 * std::max<uint32_t>(log_cap, 4096)) ov_cap <<= 1;
-    const uint32_t pend_cap = 2 * std::max<uint32_t>(log_cap, 4096);
+    uint32_t ov_cap, pend_cap;
+    propagate_caps(log_cap, ov_words, ov_cap, pend_cap);
     const size_t sb = propagate_slot_bytes(ov_cap, pend_cap);
     uint64_t slots = std::min<uint64_t>((uint64_t)std::max(1, sms * std::max(1, per)) * kWPB, ((uint64_t)n + kWPB - 1) / kWPB * kWPB);
     slots = std::min<uint64_t>(slots, ws_bytes / sb / kWPB * kWPB);
@@ -311,10 +363,49 @@ fi_status launch_propagate(const fi_program* p, const uint8_t* image, const fi_t
     A.ov_list = reinterpret_cast<uint32_t*>(b);
     A.list_cap = ov_cap;
     A.hist = hist; A.flags = flags; A.status = dev_status;
+    A.pf = pf; A.opw = opw;
     // generation tags restart at 1 for every call: clear the overlay tables once
     if ((e = cuda_status(cudaMemsetAsync(A.ov, 0, (size_t)slots * ov_cap * 16, s)))) return e;
     k_propagate<<<(unsigned)(slots / kWPB), kWPB * 32, smem, s>>>(A);
     return launch_status();
 }
 
+__global__ void k_iota_p(uint32_t* order, uint32_t n, uint32_t* counter) {
+    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < n) order[i] = i;
+    if (i == 0) *counter = 0;
+}
+
 }  // namespace fi
+
+using namespace fi;
+
+extern "C" size_t fi_inject_permanent_workspace(uint32_t n, uint32_t log_cap, uint32_t ov_words,
+                                                uint32_t max_slots) {
+    uint32_t ov_cap, pend_cap;
+    propagate_caps(log_cap, ov_words, ov_cap, pend_cap);
+    const size_t sb = propagate_slot_bytes(ov_cap, pend_cap);
+    uint64_t slots = std::min<uint64_t>(((uint64_t)n + 3) / 4 * 4, 148ull * 16);
+    if (max_slots) slots = std::min<uint64_t>(slots, ((uint64_t)std::max<uint32_t>(max_slots, 4) + 3) / 4 * 4);
+    return 256 + align256((size_t)n * 4) + slots * sb;
+}
+
+extern "C" fi_status fi_inject_permanent(const fi_program* p, const uint8_t* image, const fi_trace* t,
+                                         const fi_pfault* faults, uint32_t n, const uint64_t* op_weights, fi_inj* out,
+                                         fi_store* log, uint32_t log_cap, uint32_t ov_words, uint64_t* hist,
+                                         uint32_t flags, void* ws, size_t ws_bytes, uint32_t* dev_status,
+                                         void* stream) {
+    if (!p || !image || !t || !faults || !out || !log || !hist || !dev_status || !p->aux) return FI_E_ARG;
+    if (n == 0) return FI_OK;
+    if (!ws || ws_bytes < fi_inject_permanent_workspace(n, log_cap, ov_words, 4)) return FI_E_ARG;
+    cudaStream_t s = (cudaStream_t)stream;
+    uint32_t* counter = reinterpret_cast<uint32_t*>(ws);
+    uint32_t* order = reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(ws) + 256);
+    const size_t head = 256 + align256((size_t)n * 4);
+    k_iota_p<<<(n + 255) / 256, 256, 0, s>>>(order, n, counter);
+    fi_status e = launch_status();
+    if (e) return e;
+    return launch_propagate(p, image, t, nullptr, n, out, log, log_cap, hist, flags,
+                            reinterpret_cast<char*>(ws) + head, ws_bytes - head, order, counter, dev_status, s,
+                            faults, op_weights, ov_words);
+}

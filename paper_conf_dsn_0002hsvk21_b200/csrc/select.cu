@@ -16,18 +16,6 @@
 namespace fi {
 namespace {
 
-// ---- Philox4x32-10 (Salmon et al. 2011) ------------------------------------
-__device__ __forceinline__ uint4 philox4x32_10(uint4 c, uint2 k) {
-#pragma unroll
-    for (int r = 0; r < 10; ++r) {
-        if (r) { k.x += 0x9E3779B9u; k.y += 0xBB67AE85u; }
-        const uint32_t hi0 = __umulhi(0xD2511F53u, c.x), lo0 = 0xD2511F53u * c.x;
-        const uint32_t hi1 = __umulhi(0xCD9E8D57u, c.z), lo1 = 0xCD9E8D57u * c.z;
-        c = make_uint4(hi1 ^ c.y ^ k.x, lo1, hi0 ^ c.w ^ k.y, lo0);
-    }
-    return c;
-}
-
 // Lemire's nearly-divisionless unbiased draw of s in [0, n) for replica j (C-5).
 __device__ void draw(uint64_t seed, uint64_t j, uint64_t n, uint64_t& s, uint32_t& u_dst, uint32_t& u_bit) {
     const uint2 key = make_uint2((uint32_t)seed, (uint32_t)(seed >> 32));

@@ -40,7 +40,9 @@ INJ_DTYPE = np.dtype([("before", "<u4"), ("after", "<u4"), ("mask", "<u4"), ("fa
                       ("n_faulty_stores", "<u4")])
 RECORD_DTYPE = np.dtype([("instance", "<u4"), ("insn", "<u4"), ("active", "<u4"), ("pred", "<u4")])
 STORE_DTYPE = np.dtype([("va", "<u8"), ("value", "<u4"), ("step", "<u4")])
-assert SITE_DTYPE.itemsize == 64 and INJ_DTYPE.itemsize == 24
+PFAULT_DTYPE = np.dtype([("opcode", "<u4"), ("sm", "<u4"), ("lane", "<u4"), ("mask", "<u4"), ("q32", "<u4"),
+                         ("n_sm", "<u4"), ("seed", "<u8")])
+assert SITE_DTYPE.itemsize == 64 and INJ_DTYPE.itemsize == 24 and PFAULT_DTYPE.itemsize == 32
 
 
 class FIError(RuntimeError):
@@ -113,6 +115,8 @@ def lib():
             "fi_profile_approx": (st, [vp, vp, vp, vp, sz, vp]),
             "fi_build_instance_index": (st, [vp, u32, vp, vp, vp]),
             "fi_select_sites_approx": (st, [vp, vp, vp, u32, vp, vp, u64, u32, vp, vp, vp]),
+            "fi_inject_permanent_workspace": (sz, [u32, u32, u32, u32]),
+            "fi_inject_permanent": (st, [vp, vp, vp, vp, u32, vp, vp, vp, u32, u32, vp, u32, vp, sz, vp, vp]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -430,6 +434,35 @@ def select_sites_approx(idx: InstanceIndex, sched: fi_schedule, j0: int, n: int,
     if status is None:
         st.check("fi_select_sites_approx")
     return sites
+
+
+def inject_permanent(gt: GoldenTrace, faults: np.ndarray, op_weights: torch.Tensor | None = None,
+                     unchecked: bool = False, log_cap: int | None = None, ov_words: int | None = None,
+                     max_slots: int = 0):
+    """fi_inject_permanent (rows f2/f3).  Returns (inj [n*24] u8, weighted hist [3] i64).
+    ov_words defaults to every word of the image (a permanent fault may corrupt them all)."""
+    dev = gt.dp.device
+    f = np.ascontiguousarray(faults, dtype=PFAULT_DTYPE)
+    n = len(f)
+    cap = log_capacity(gt) if log_cap is None else log_cap
+    ft = torch.from_numpy(f.view(np.uint8).copy()).to(dev)
+    out = torch.zeros(max(n, 1) * 24, dtype=torch.uint8, device=dev)
+    log = torch.empty(max(n * cap, 1) * 16, dtype=torch.uint8, device=dev)
+    hist = torch.zeros(3, dtype=torch.int64, device=dev)
+    ovw = gt.dp.prog.image_bytes // 4 if ov_words is None else ov_words
+    ws_n = lib().fi_inject_permanent_workspace(n, cap, ovw, max_slots)
+    if not max_slots:                                 # keep the overlays within 16 GiB of HBM
+        ms = 2368
+        while ws_n > 16 << 30 and ms > 4:
+            ms //= 2
+            ws_n = lib().fi_inject_permanent_workspace(n, cap, ovw, ms)
+    ws = torch.empty(ws_n, dtype=torch.uint8, device=dev)
+    st = DeviceStatus(dev)
+    _check(lib().fi_inject_permanent(C.byref(gt.dp.c), _p(gt.image), C.byref(gt.c), _p(ft), n, _p(op_weights),
+                                     _p(out), _p(log), cap, ovw, _p(hist), FI_UNCHECKED if unchecked else 0, _p(ws), ws_n,
+                                     st.ptr, _stream()), "fi_inject_permanent")
+    st.check("fi_inject_permanent")
+    return out, hist
 
 
 def write_params_txt(site_row: np.ndarray, kernel_name: str) -> str:
