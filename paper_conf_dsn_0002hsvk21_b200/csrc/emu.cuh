@@ -461,8 +461,12 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
         for (uint32_t r = 0; r <= zr; ++r) R[r * 32 + lane] = 0u;
     }
     uint32_t livem = __ballot_sync(kFull, live);
-    bool conv = false;                                // recomputed at the first step
-    uint32_t upc = 0;
+    // Group mode (`conv`): the lanes of `amask` share pc `upc` and every other live
+    // lane is parked at a pc >= npc > upc, so by the min-pc rule (§3.3) the group
+    // keeps running alone, with no per-step scheduling, until it branches
+    // divergently, exits, or reaches npc (where parked lanes rejoin).
+    bool conv = false;
+    uint32_t upc = 0, amask = 0, npc = 0xFFFFFFFFu;
     EmuOut o;
     uint32_t nst = 0;
     uint4 recbuf = make_uint4(0, 0, 0, 0);
@@ -474,16 +478,18 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
         uint32_t pcm, active;
         if (conv) {
             pcm = upc;
-            active = livem;
+            active = amask;
         } else {
             pcm = __reduce_min_sync(kFull, live ? pc : 0xFFFFFFFFu);
             active = __ballot_sync(kFull, live && pc == pcm);
-            if (active == livem) { conv = true; upc = pcm; }
+            npc = active == livem ? 0xFFFFFFFFu : __reduce_min_sync(kFull, (live && pc != pcm) ? pc : 0xFFFFFFFFu);
+            conv = true; upc = pcm; amask = active;
         }
+        const bool inA = (amask >> lane) & 1u;
         if (MODE == EMU_TRACE && use_ck && (step % ck_interval) == 0) {
             uint32_t* dst = ck + (size_t)(step / ck_interval) * ckw;
             for (uint32_t r = 0; r < zr; ++r) dst[r * 32 + lane] = R[r * 32 + lane];
-            dst[zr * 32 + lane] = live ? (conv ? upc : pc) : 0u;
+            dst[zr * 32 + lane] = live ? (inA ? upc : pc) : 0u;
             dst[zr * 32 + 32 + lane] = preds;
             dst[zr * 32 + 64 + lane] = live ? 1u : 0u;
         }
@@ -494,7 +500,7 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
             // ---- straight-line run: no scheduling / control bookkeeping per step
             const uint32_t rw = __ldg(&runl[pcm]);
             uint32_t run = rw & 0xFFFF, lr = (rw >> 16) & 0xFF, fr = rw >> 24;
-            uint32_t lim = watchdog - step;
+            uint32_t lim = min(watchdog - step, npc - pcm);   // stop where parked lanes rejoin
             if (MODE == EMU_TRACE && use_ck) lim = min(lim, ck_interval - step % ck_interval);
             if (MODE == EMU_INJ && hook.step >= step) lim = min(lim, hook.step - step);
             run = min(run, lim);
@@ -512,15 +518,16 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
                     const float rf = __fmaf_rn(x, y, z);
                     const uint32_t r = rf != rf ? kQNaN32 : __float_as_uint(rf);
                     // simple FFMAs have a real destination (decode guarantees rd < zero row)
-                    if (live) *reinterpret_cast<uint32_t*>(F.Rb + (cur.z >> 16)) = r;
+                    if (inA) *reinterpret_cast<uint32_t*>(F.Rb + (cur.z >> 16)) = r;
                     if (MODE == EMU_TRACE) {
                         const uint32_t s = step + j;
-                        if ((s & 31) == lane) recbuf = make_uint4(k, __ldg(&ins[pcm + j]), livem, kFull);
+                        if ((s & 31) == lane) recbuf = make_uint4(k, __ldg(&ins[pcm + j]), amask, kFull);
                         if ((s & 31) == 31) reinterpret_cast<uint4*>(rec_out)[s - 31 + lane] = recbuf;
                     }
                 }
                 step += fr;
                 upc = pcm + fr;
+                if (upc >= npc) { conv = false; if (inA) pc = upc; }
                 continue;
             }
             if (lr >= 2) {
@@ -539,7 +546,7 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
                         const uint32_t guard = (D.x >> 8) & 0xFF, mod = (D.x >> 16) & 0xFF;
                         const bool pv = guard == 7 ? true : guard_of(guard, preds);
                         preds_b[b] = guard == 7 ? kFull : __ballot_sync(kFull, pv);
-                        const bool ex = live && pv;
+                        const bool ex = inA && pv;
                         const uint32_t lw = (mod & 3) > 2 ? 2 : (mod & 3);
                         const uint64_t va = F.rd64(D.y & 0xFFFF) + (uint64_t)(int64_t)(int32_t)D.w;
                         bool zero = false;
@@ -580,13 +587,14 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
                         }
                         if (MODE == EMU_TRACE) {
                             const uint32_t s = step + b;
-                            if ((s & 31) == lane) recbuf = make_uint4(k, __ldg(&ins[pcm + b]), livem, preds_b[b]);
+                            if ((s & 31) == lane) recbuf = make_uint4(k, __ldg(&ins[pcm + b]), amask, preds_b[b]);
                             if ((s & 31) == 31) reinterpret_cast<uint4*>(rec_out)[s - 31 + lane] = recbuf;
                         }
                     }
                 }
                 step += lr;
                 upc = pcm + lr;
+                if (upc >= npc) { conv = false; if (inA) pc = upc; }
                 continue;
             }
             if (run) {
@@ -603,13 +611,14 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
                     }
                     if (MODE == EMU_TRACE) {
                         const uint32_t s = step + j;
-                        if ((s & 31) == lane) recbuf = make_uint4(k, __ldg(&ins[pcm + j]), livem, pred);
+                        if ((s & 31) == lane) recbuf = make_uint4(k, __ldg(&ins[pcm + j]), amask, pred);
                         if ((s & 31) == 31) reinterpret_cast<uint4*>(rec_out)[s - 31 + lane] = recbuf;
                     }
-                    exec_plain(F, LC, D, live && pv, preds);
+                    exec_plain(F, LC, D, inA && pv, preds);
                 }
                 step += run;
                 upc = pcm + run;
+                if (upc >= npc) { conv = false; if (inA) pc = upc; }
                 continue;
             }
         }
@@ -634,6 +643,7 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
         if (op == EXIT) {
             if (ex) live = false;
             livem &= ~exm;
+            amask &= ~exm;
         } else if (op == BRA) {
             taken = exm;
         } else if (op == LDG || op == STG) {
@@ -696,15 +706,15 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
         }
 
         // control flow: advance / branch, tracking convergence
-        if (conv) {
-            if (taken == 0) upc = pcm + 1;
-            else if (taken == active) upc = imm;
-            else {
-                conv = false;
-                pc = ((taken >> lane) & 1u) ? imm : pcm + 1;
-            }
-        } else if (act) {
-            pc = ((taken >> lane) & 1u) ? imm : pcm + 1;
+        if (taken == 0) upc = pcm + 1;              // (always in group mode here: active = amask)
+        else if (taken == active) upc = imm;
+        else {
+            conv = false;
+            if (act) pc = ((taken >> lane) & 1u) ? imm : pcm + 1;
+        }
+        if (conv && (amask == 0 || upc >= npc)) {     // group exited / reached parked lanes
+            conv = false;
+            if ((amask >> lane) & 1u) pc = upc;
         }
 
         if (perm && op == hook.perm_op && lane == hook.perm_lane && ex) {
