@@ -227,6 +227,49 @@ def _fuzz_body(rng: np.random.Generator, s: Asm, n_ops: int, allow_branch=True):
         s.label(lbl[0])
 
 
+F32_SPECIALS = np.array([0x7FC00000, 0xFFC00000, 0x7F800001, 0xFF812345, 0x7FFFFFFF, 0x7FA5A5A5, 0x7F800000,
+                         0xFF800000, 0x00000000, 0x80000000, 0x00000001, 0x807FFFFF, 0x7F7FFFFF, 0x3F800000,
+                         0xBF800000, 0x00800000], dtype=np.uint32)
+
+
+def ffma_runs(seed: int = 5, grid: int = 2, block: int = 96) -> Program:
+    """Straight runs of unguarded FFMAs (the emulator's FFMA batch path) over
+    special f32 values: NaNs with payloads and both signs, infinities, signed
+    zeros, denormals, extremes.  Independent batches, dependent chains, and a
+    run that reads a register written earlier in it."""
+    s = Asm()
+    s.s2r(0, isa.SR_TID)
+    s.s2r(1, isa.SR_CTAID)
+    s.s2r(2, isa.SR_NTID)
+    s.imad(0, 1, 2, 0)
+    s.ldc(4, 0, wide=True)
+    s.imad_wide(4, 0, imm=64, c=4, unsigned=True)
+    s.ldc(6, 8, wide=True)
+    s.imad_wide(6, 0, imm=96, c=6, unsigned=True)
+    for q in range(4):
+        s.ldg(8 + 4 * q, 4, off=16 * q, width=isa.W128)
+    for q in range(8):                                 # independent: R24..R31
+        s.ffma(24 + q, 8 + q, 9 + q, 10 + q)
+    for q in range(8):                                 # chain through R32
+        s.ffma(32, 32 if q else 12, 16 + q, 24 + q)
+    for q in range(8):                                 # reads results of this run: R33..R39
+        s.ffma(33 + (q % 7), 24 + q, 32, 33 + ((q + 3) % 7))
+    for q in range(6):
+        s.stg(6, 24 + 4 * q, off=16 * q, width=isa.W128)
+    s.exit()
+    n = grid * block
+    rng = np.random.Generator(np.random.PCG64(seed))
+    x = rng.integers(0, 2**32, size=16 * n, dtype=np.uint64).astype(np.uint32)
+    pick = rng.random(16 * n) < 0.5
+    x[pick] = F32_SPECIALS[rng.integers(0, len(F32_SPECIALS), int(pick.sum()))]
+    pb = ProgramBuilder(f"ffma_runs_{seed}")
+    k = pb.add_kernel("ffma_runs", s.assemble(), nregs=44)
+    xb = pb.add_buffer("X", 64 * n, x.view(np.float32), dtype=isa.DT_U32)
+    yb = pb.add_buffer("Y", 96 * n, writer=0, output=True, dtype=isa.DT_U32)
+    pb.add_instance(k, grid, block, ptr_words(xb) + ptr_words(yb))
+    return pb.build(config="ffma_runs", n=n)
+
+
 def fuzz_program(seed: int, n_ops: int = 120, grid: int = 2, block: int = 80, loop_iters: int = 3) -> Program:
     """Random kernel: load 16 words per thread (special FP values mixed in), run
     a random op mix (optionally inside a counted loop), store the 16 registers

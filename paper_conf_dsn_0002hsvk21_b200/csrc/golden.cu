@@ -73,7 +73,7 @@ __global__ void k_gran(const fi_buffer* buf, uint32_t n_buf, uint32_t* gran, uin
 // decode every static instruction (register operands -> smem row offsets) and
 // precompute its trace insn word pc | op<<16 | groupmask<<24 (Table II, C-2)
 __global__ void k_decode(const fi_insn* code, uint32_t n_code, const fi_kernel* kern, uint32_t n_kern, uint32_t zr,
-                         uint4* dec, uint32_t* ins, uint32_t* run) {
+                         uint4* dec, uint4* fdec, uint32_t* ins, uint32_t* run) {
     const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= n_code) return;
     const fi_insn I = code[i];
@@ -108,6 +108,25 @@ __global__ void k_decode(const fi_insn* code, uint32_t n_code, const fi_kernel* 
                          code[j].d0 < zr; ++j)
         ++fr;
     run[i] = (r > 0xFFFF ? 0xFFFFu : r) | (std::min<uint32_t>(lr, 0xFF) << 16) | (fr << 24);
+    // independent batch inside the simple-FFMA run
+    uint32_t fb = 0;
+    for (uint32_t j = i; j < i + fr && fb < kFfmaBatch; ++j) {
+        bool hazard = false;
+        for (uint32_t q = i; q < j && !hazard; ++q) {
+            const uint32_t d = code[q].d0;
+            hazard = code[j].a == d || code[j].b == d || code[j].c == d || code[j].d0 == d;
+        }
+        if (hazard) break;
+        ++fb;
+    }
+    if (fr) {
+        const uint4 D = dec[i];
+        fdec[i] = make_uint4(D.y & 0xFFFF, D.y >> 16, D.z & 0xFFFF, (D.z >> 16) | (fb << 24));
+    } else {
+        fdec[i] = make_uint4(0, 0, 0, 0);
+    }
+    if (i + 1 == n_code)
+        for (uint32_t q = 0; q < kFfmaBatch; ++q) fdec[n_code + q] = make_uint4(0, 0, 0, 0);
 }
 
 // Buffers an instance's constant bank points into (each adjacent word pair read as
@@ -177,6 +196,7 @@ extern "C" fi_status fi_program_prepare(const fi_program* p, void* aux, void* st
     if (p->n_code) {
         k_decode<<<(p->n_code + 127) / 128, 128, 0, s>>>(p->code, p->n_code, p->kern, p->n_kern, p->n_regs,
                                                          reinterpret_cast<uint4*>(a + L.dec),
+                                                         reinterpret_cast<uint4*>(a + L.fdec),
                                                          reinterpret_cast<uint32_t*>(a + L.ins),
                                                          reinterpret_cast<uint32_t*>(a + L.run));
         if ((e = launch_status())) return e;

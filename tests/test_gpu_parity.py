@@ -64,6 +64,16 @@ def test_fuzz_trace_and_image(F, seed):
     assert np.array_equal(ic.cpu().numpy().astype(np.uint64), g.counts())
 
 
+@pytest.mark.parametrize("seed", [5, 6, 7])
+def test_ffma_runs_special_values(F, seed):
+    """The emulator's batched simple-FFMA path on NaN payloads, infinities, signed
+    zeros and denormals: images, traces and injected outcomes against the oracle
+    (which canonicalises NaN explicitly, C-13)."""
+    prog = P.ffma_runs(seed)
+    gi, oi = _campaign_parity(F, prog, seed, [F.G_FP32, F.G_GP, F.G_LD], [0, 1, 2, 3], 300, O.MODE_FULL)
+    assert len(np.unique(oi["outcome"])) >= 2
+
+
 def _campaign_parity(F, prog, seed, groups, bfms, n, mode, ckpt="auto", unchecked=False):
     g = O.Golden(prog)
     dp, gt = _gpu_golden(F, prog, ckpt)
