@@ -213,6 +213,7 @@ def main():
 
     stage_ms = {s: 0.0 for s in STAGES}
     step_ms = []
+    emulated_steps = 0
     clocks = ClockSampler(local)
     if world > 1:
         dist.barrier()
@@ -230,6 +231,7 @@ def main():
             stage_ms[s] += ev[prev].elapsed_time(ev[s])
             prev = s
         step_ms.append(ev["start"].elapsed_time(ev["end"]))
+        emulated_steps += int(camp.inj_ws[8:16].cpu().view(torch.int64).item())   # K4's own count (fi.h)
     clk = clocks.stop()
     if world > 1:
         dist.barrier()
@@ -263,6 +265,28 @@ def main():
         if d.get("config") == args.config:
             traffic = d.get("dram_bytes_per_launch")
 
+    # K4 (the dominant kernel of the step) is an interpreter: bound by the SM issue
+    # rate, not HBM.  achieved = SASS warp-instructions K4 issues
+    # per launch (ncu smsp__inst_executed.sum of the same workload, profiles/
+    # k4_counts.json) / its live CUDA-event duration; peak = 148 SMs x 4 schedulers
+    # x 1 warp-instruction/clock x the SM clock measured during the run.
+    k4_ms_local = stage_ms["inject"] / K
+    k4 = {"bound": "alu", "kernel": "k_inject (K4)", "unit": "warp-inst/s", "achieved": None, "peak": None,
+          "frac": None, "traffic": None}
+    kp = os.path.join(ROOT, "profiles", "k4_counts.json")
+    sm_mhz = clk.get("sm_mhz") or clk.get("sm_max_mhz") or 1965.0
+    k4["peak"] = 148 * 4 * sm_mhz * 1e6
+    k4["peak_source"] = f"148 SMs x 4 SMSPs x 1 issue/clk x {sm_mhz:.0f} MHz (measured SM clock under load)"
+    if os.path.exists(kp):
+        d = json.load(open(kp))
+        if d.get("config") == args.config and d.get("replicas") == n and world == 1:
+            k4["achieved"] = d["sass_warp_inst_per_launch"] / (k4_ms_local / 1e3)
+            k4["frac"] = k4["achieved"] / k4["peak"]
+            k4["traffic"] = d.get("dram_bytes_per_launch")
+            k4["sass_per_emulated_step"] = d["sass_warp_inst_per_launch"] / max(emulated_steps / K, 1)
+    k4["emulated_warp_steps_per_launch"] = emulated_steps / K
+    k4["emulated_warp_steps_per_s"] = emulated_steps / K / (k4_ms_local / 1e3)
+
     line = {
         "metric": "thread-dyn-instrs profiled/sec and injections/sec at 1/2/4/8 B200 (% HBM roofline)",
         "value": value, "unit": "thread-dyn-instrs/s", "n_gpus": world, "steps": K, "warmup": args.warmup,
@@ -275,11 +299,14 @@ def main():
         "injections_per_s": inj_rate,
         "stages_ms_per_step": {s: stage_ms[s] / K for s in STAGES},
         "outcomes": {"masked": int(hist[..., 0].sum()), "sdc": int(hist[..., 1].sum()), "due": int(hist[..., 2].sum())},
-        "roofline": {"bound": "hbm", "kernel": "k_profile (K1)", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                     "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
-                     "algorithmic_bytes_per_launch": algo_bytes},
+        "roofline": k4,
+        "roofline_profile": {"bound": "hbm", "kernel": "k_profile (K1)", "achieved": achieved, "peak": peak,
+                             "unit": "GB/s", "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
+                             "algorithmic_bytes_per_launch": algo_bytes},
         "clocks": clk,
-        "gpu_launches": 6 * K,
+        # per step: k_profile, 2 x k_scan_rows, k_inst_identities, k_tile_sums, k_select,
+        # k_lpt_order, k_inject, k_classify
+        "gpu_launches": 9 * K,
     }
 
     if not args.no_e2e:

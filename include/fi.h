@@ -233,7 +233,9 @@ fi_status fi_select_sites_approx(const fi_program* p, const fi_trace* t, const v
  * Memory faults and the watchdog (C-9, C-10) end the replica.
  * Scheduling only (results do not depend on it): persistent warps take
  * replicas from a queue ordered longest-expected-first (counting sort of the
- * steps left after the restart point); scratch: fi_inject_workspace(n) bytes. */
+ * steps left after the restart point); scratch: fi_inject_workspace(n) bytes.
+ * After the call, bytes 8..15 of ws hold the number of warp-instructions the
+ * replicas emulated (u64, from their restart points; measurement only). */
 size_t fi_inject_workspace(uint32_t n);
 fi_status fi_inject(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
                     uint32_t n, fi_inj* out, fi_store* log, uint32_t log_cap, void* ws, size_t ws_bytes,

@@ -48,7 +48,7 @@ enum EmuMode { EMU_LEN = 0, EMU_TRACE = 1, EMU_INJ = 2, EMU_PROP = 3 };
 // count > kInstBufs = "unknown", never skipped by K7)
 constexpr uint32_t kInstBufs = 15;
 
-struct AuxLayout { size_t gran, dec, fdec, ins, run, ib, total; };
+struct AuxLayout { size_t gran, dec, fdec, fbl, ins, run, ib, total; };
 constexpr uint32_t kFfmaBatch = 8;                   // independent simple FFMAs emulated together
 __host__ __device__ inline size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
 __host__ __device__ inline AuxLayout aux_layout(uint64_t image_bytes, uint32_t n_code, uint32_t n_inst) {
@@ -56,7 +56,8 @@ __host__ __device__ inline AuxLayout aux_layout(uint64_t image_bytes, uint32_t n
     L.gran = 0;
     L.dec = align256(((image_bytes + 255) >> 8) * sizeof(uint32_t));
     L.fdec = L.dec + align256((size_t)n_code * 16);
-    L.ins = L.fdec + align256(((size_t)n_code + kFfmaBatch) * 16);   // padded: batches load 8 entries
+    L.fbl = L.fdec + align256(((size_t)n_code + kFfmaBatch) * 16);   // padded: batches load 8 entries
+    L.ins = L.fbl + align256((size_t)n_code);
     L.run = L.ins + align256((size_t)n_code * 4);
     L.ib = L.run + align256((size_t)n_code * 4);
     L.total = L.ib + align256((size_t)n_inst * (kInstBufs + 1) * 4);
@@ -72,9 +73,9 @@ __host__ __device__ inline bool is_plain(uint32_t op) { return op != BRA && op !
 //   z = rc | rd << 16                               rd = 0xFFFF when the write is discarded
 //   w = imm
 // simple-FFMA entry (fdec, uint4): x, y, z = byte offsets of the a, b, c operand
-// rows; w = destination row offset | batch length << 24, the batch being the
-// longest run (<= kFfmaBatch) of simple FFMAs from here in which no FFMA reads
-// or writes a register written by an earlier one (all reads may go first).
+// rows, w = destination row offset; fbl (u8) = batch length: the longest run
+// (<= kFfmaBatch) of simple FFMAs from here in which no FFMA reads or writes a
+// register written by an earlier one (so all reads may go first).
 __host__ __device__ inline uint4 decode_insn(const fi_insn& I, uint32_t zr) {
     auto row = [&](uint32_t r) -> uint32_t { return (r < zr ? r : zr) * 128u; };
     uint32_t pb = 0;
@@ -92,7 +93,8 @@ __host__ __device__ inline uint4 decode_insn(const fi_insn& I, uint32_t zr) {
 
 struct EmuProg {
     const uint4* dec;          // decoded code
-    const uint4* fdec;         // simple-FFMA operand offsets + independent batch length
+    const uint4* fdec;         // simple-FFMA operand offsets
+    const uint8_t* fbl;        // simple-FFMA independent batch length
     const uint32_t* ins;       // trace insn word per static instruction: pc | op<<16 | groupmask<<24
     const uint32_t* run;       // straight-line run length starting at each static instruction
     const fi_kernel* kern;
@@ -110,7 +112,7 @@ inline EmuProg make_emu_prog(const fi_program* p) {
     const AuxLayout L = aux_layout(p->image_bytes, p->n_code, p->n_inst);
     const char* a = reinterpret_cast<const char*>(p->aux);
     return EmuProg{reinterpret_cast<const uint4*>(a + L.dec), reinterpret_cast<const uint4*>(a + L.fdec),
-                   reinterpret_cast<const uint32_t*>(a + L.ins),
+                   reinterpret_cast<const uint8_t*>(a + L.fbl), reinterpret_cast<const uint32_t*>(a + L.ins),
                    reinterpret_cast<const uint32_t*>(a + L.run), p->kern, p->inst, p->cbank, p->buf,
                    reinterpret_cast<const uint32_t*>(a + L.gran), reinterpret_cast<const uint32_t*>(a + L.ib),
                    p->image_bytes, p->n_regs, p->n_inst};
@@ -520,34 +522,53 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
                 //      then the writes.  No NaN canonicalisation is needed here: sm_100
                 //      FFMA returns 0x7FFFFFFF for every NaN result (C-13 holds as is;
                 //      pinned by the special-value parity tests).
-                const uint4* fp = P.fdec + kn.code_off + pcm;
-                for (uint32_t done = 0; done < fr;) {
+                const uint4* fq = P.fdec + kn.code_off + pcm;
+                const uint8_t* fl = P.fbl + kn.code_off + pcm;
+                uint32_t sb = step;
+                for (uint32_t left = fr; left;) {
+                    const uint32_t nb = min((uint32_t)__ldg(fl), left);
                     uint4 e[kFfmaBatch];
 #pragma unroll
-                    for (uint32_t b = 0; b < kFfmaBatch; ++b) e[b] = __ldg(&fp[done + b]);
-                    const uint32_t nb = min(e[0].w >> 24, fr - done);
+                    for (uint32_t b = 0; b < kFfmaBatch; ++b) e[b] = __ldg(fq + b);
                     float x[kFfmaBatch], y[kFfmaBatch], z[kFfmaBatch];
+                    if (nb == kFfmaBatch) {                   // full batch: no per-FFMA predication
 #pragma unroll
-                    for (uint32_t b = 0; b < kFfmaBatch; ++b) {
-                        if (b < nb) {
+                        for (uint32_t b = 0; b < kFfmaBatch; ++b) {
                             x[b] = u2f(F.rd(e[b].x));
                             y[b] = u2f(F.rd(e[b].y));
                             z[b] = u2f(F.rd(e[b].z));
                         }
-                    }
+                        if (inA) {
 #pragma unroll
-                    for (uint32_t b = 0; b < kFfmaBatch; ++b) {
-                        if (b < nb && inA)
-                            *reinterpret_cast<float*>(F.Rb + (e[b].w & 0xFFFFFFu)) = __fmaf_rn(x[b], y[b], z[b]);
+                            for (uint32_t b = 0; b < kFfmaBatch; ++b)
+                                *reinterpret_cast<float*>(F.Rb + e[b].w) = __fmaf_rn(x[b], y[b], z[b]);
+                        }
+                    } else {
+#pragma unroll
+                        for (uint32_t b = 0; b < kFfmaBatch; ++b) {
+                            if (b < nb) {
+                                x[b] = u2f(F.rd(e[b].x));
+                                y[b] = u2f(F.rd(e[b].y));
+                                z[b] = u2f(F.rd(e[b].z));
+                            }
+                        }
+#pragma unroll
+                        for (uint32_t b = 0; b < kFfmaBatch; ++b) {
+                            if (b < nb && inA)
+                                *reinterpret_cast<float*>(F.Rb + e[b].w) = __fmaf_rn(x[b], y[b], z[b]);
+                        }
                     }
                     if (MODE == EMU_TRACE) {
                         for (uint32_t b = 0; b < nb; ++b) {
-                            const uint32_t s = step + done + b;
-                            if ((s & 31) == lane) recbuf = make_uint4(k, __ldg(&ins[pcm + done + b]), amask, kFull);
+                            const uint32_t s = sb + b;
+                            if ((s & 31) == lane) recbuf = make_uint4(k, __ldg(&ins[pcm + (s - step)]), amask, kFull);
                             if ((s & 31) == 31) reinterpret_cast<uint4*>(rec_out)[s - 31 + lane] = recbuf;
                         }
                     }
-                    done += nb;
+                    fq += nb;
+                    fl += nb;
+                    sb += nb;
+                    left -= nb;
                 }
                 step += fr;
                 upc = pcm + fr;

@@ -73,7 +73,7 @@ __global__ void k_gran(const fi_buffer* buf, uint32_t n_buf, uint32_t* gran, uin
 // decode every static instruction (register operands -> smem row offsets) and
 // precompute its trace insn word pc | op<<16 | groupmask<<24 (Table II, C-2)
 __global__ void k_decode(const fi_insn* code, uint32_t n_code, const fi_kernel* kern, uint32_t n_kern, uint32_t zr,
-                         uint4* dec, uint4* fdec, uint32_t* ins, uint32_t* run) {
+                         uint4* dec, uint4* fdec, uint8_t* fbl, uint32_t* ins, uint32_t* run) {
     const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= n_code) return;
     const fi_insn I = code[i];
@@ -121,10 +121,11 @@ __global__ void k_decode(const fi_insn* code, uint32_t n_code, const fi_kernel* 
     }
     if (fr) {
         const uint4 D = dec[i];
-        fdec[i] = make_uint4(D.y & 0xFFFF, D.y >> 16, D.z & 0xFFFF, (D.z >> 16) | (fb << 24));
+        fdec[i] = make_uint4(D.y & 0xFFFF, D.y >> 16, D.z & 0xFFFF, D.z >> 16);
     } else {
         fdec[i] = make_uint4(0, 0, 0, 0);
     }
+    fbl[i] = (uint8_t)fb;
     if (i + 1 == n_code)
         for (uint32_t q = 0; q < kFfmaBatch; ++q) fdec[n_code + q] = make_uint4(0, 0, 0, 0);
 }
@@ -197,6 +198,7 @@ extern "C" fi_status fi_program_prepare(const fi_program* p, void* aux, void* st
         k_decode<<<(p->n_code + 127) / 128, 128, 0, s>>>(p->code, p->n_code, p->kern, p->n_kern, p->n_regs,
                                                          reinterpret_cast<uint4*>(a + L.dec),
                                                          reinterpret_cast<uint4*>(a + L.fdec),
+                                                         reinterpret_cast<uint8_t*>(a + L.fbl),
                                                          reinterpret_cast<uint32_t*>(a + L.ins),
                                                          reinterpret_cast<uint32_t*>(a + L.run));
         if ((e = launch_status())) return e;

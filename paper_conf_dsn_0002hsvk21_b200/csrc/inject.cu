@@ -43,7 +43,7 @@ k_lpt_order(const fi_site* __restrict__ sites, const uint64_t* __restrict__ warp
         return L > start ? L - start : 0;
     };
     for (uint32_t b = threadIdx.x; b < kBuckets; b += blockDim.x) hist[b] = 0;
-    if (threadIdx.x == 0) { s_max = 0; *counter = 0; }
+    if (threadIdx.x == 0) { s_max = 0; *counter = 0; *reinterpret_cast<unsigned long long*>(counter + 2) = 0; }
     __syncthreads();
     uint32_t mx = 0;
     for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) mx = max(mx, (uint32_t)min(cost(i), (uint64_t)0xFFFFFFFFu));
@@ -105,6 +105,8 @@ k_inject(EmuProg P, const uint8_t* img, const uint64_t* __restrict__ warp_off, c
         r.n_faulty_stores = o.nstore;
         out[i] = r;
         if (!o.fired || o.bad) FI_DEV_ERR(status, FI_E_SITE);
+        const uint32_t start = (ckpt && ck_interval) ? S.step / ck_interval * ck_interval : 0u;
+        atomicAdd(reinterpret_cast<unsigned long long*>(counter + 2), (unsigned long long)(o.steps - start));
     }
     __syncwarp();
     }
