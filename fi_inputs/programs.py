@@ -568,3 +568,48 @@ def cg_program(nx: int = 512, ny: int = 256, iters: int = 500, seed: int = DATA_
 
 def c3(full: bool = True) -> Program:
     return cg_program(512, 256, 500) if full else cg_program(32, 16, 6)
+
+
+def scatter_chain(n_inst: int = 4, n: int = 256, block: int = 64, seed: int = 91) -> Program:
+    """x_{i+1}[perm_i[j]] = 0.5 * x_i[j] + 1 and perm_{i+1}[j] = perm_i[j] over n_inst
+    launches: data-dependent store addresses, so a corrupted index makes a warp
+    store where another warp (or another buffer) does — wild stores whose order
+    C-14 fixes — or fault (DUE), in later launches too."""
+    s = Asm()
+    s.s2r(0, isa.SR_TID)
+    s.s2r(1, isa.SR_CTAID)
+    s.s2r(2, isa.SR_NTID)
+    s.imad(0, 1, 2, 0)
+    s.ldc(3, 32)
+    s.isetp(0, 0, 3, cmp=isa.GE)
+    s.exit(guard=0)
+    s.ldc(4, 0, wide=True)                             # perm_i
+    s.imad_wide(4, 0, imm=4, c=4, unsigned=True)
+    s.ldc(6, 8, wide=True)                             # x_i
+    s.imad_wide(6, 0, imm=4, c=6, unsigned=True)
+    s.ldg(12, 4)                                       # p = perm_i[j]
+    s.ldg(13, 6)                                       # v = x_i[j]
+    s.ldc(14, 36)                                      # 0.5
+    s.ldc(15, 40)                                      # 1.0
+    s.ffma(13, 13, 14, 15)
+    s.ldc(8, 16, wide=True)                            # x_{i+1}
+    s.imad_wide(8, 12, imm=4, c=8, unsigned=True)
+    s.stg(8, 13)
+    s.ldc(10, 24, wide=True)                           # perm_{i+1}
+    s.imad_wide(10, 0, imm=4, c=10, unsigned=True)
+    s.stg(10, 12)
+    s.exit()
+    rng = np.random.Generator(np.random.PCG64(seed))
+    pb = ProgramBuilder(f"scatter_chain_{n_inst}")
+    k = pb.add_kernel("scatter", s.assemble(), nregs=16)
+    perm = pb.add_buffer("perm0", 4 * n, rng.permutation(n).astype(np.uint32).view(np.float32), dtype=isa.DT_U32)
+    x = pb.add_buffer("x0", 4 * n, f32_data(seed, n), dtype=isa.DT_F32)
+    grid = (n + block - 1) // block
+    for i in range(n_inst):
+        last = i == n_inst - 1
+        xn = pb.add_buffer(f"x{i + 1}", 4 * n, writer=i, output=last, dtype=isa.DT_F32)
+        pn = pb.add_buffer(f"perm{i + 1}", 4 * n, writer=i, output=last, dtype=isa.DT_U32)
+        pb.add_instance(k, grid, block, ptr_words(perm) + ptr_words(x) + ptr_words(xn) + ptr_words(pn)
+                        + [n, isa.f32_bits(0.5), isa.f32_bits(1.0)])
+        perm, x = pn, xn
+    return pb.build(config="scatter_chain", n_inst=n_inst, n=n)

@@ -265,6 +265,26 @@ fi_status fi_classify(const fi_program* p, const uint8_t* image, const fi_trace*
                       uint32_t n, fi_inj* out, const fi_store* log, uint32_t log_cap, uint64_t* hist,
                       uint32_t flags, void* ws, size_t ws_bytes, uint32_t* dev_status, void* stream);
 
+/* K8 — fi_classify for long multi-instance programs (thousands of launches,
+ * SURVEY C3/C4/C5): same definition and result as fi_classify's K7 (C-12, C-14,
+ * C-19), computed instance-major over batches of `batch` replicas: for every
+ * later launch, the (replica, warp) pairs of the replicas whose corrupted words
+ * it may read are re-executed across the whole GPU.  Faulty memory lives in
+ * copy-on-write 4 KB pages from a pool of `pool_pages`; pages that equal the
+ * golden state are returned (a replica with none is Masked early) and pages of a
+ * buffer past its last launch reference are dropped.  pend_cap = update slots per
+ * replica and launch (>= the launch's golden stores, plus faulty extras).
+ * Replicas that exceed a capacity, or that later load a dropped corrupted word,
+ * get outcome 0xFF and FI_E_CAPACITY — never a wrong class.  Fills out[].outcome
+ * / flags (and fault_kind/fault_pc of the first downstream fault when K4 had
+ * none), accumulates hist[8][4][3].  Scratch: fi_classify_batched_workspace(). */
+size_t fi_classify_batched_workspace(const fi_program* p, uint32_t n, uint32_t log_cap, uint32_t batch,
+                                     uint32_t pool_pages, uint32_t pend_cap);
+fi_status fi_classify_batched(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
+                              uint32_t n, fi_inj* out, const fi_store* log, uint32_t log_cap, uint64_t* hist,
+                              uint32_t flags, uint32_t batch, uint32_t pool_pages, uint32_t pend_cap, void* ws,
+                              size_t ws_bytes, uint32_t* dev_status, void* stream);
+
 /* §8 rows f2/f3 — permanent faults (Table III
  * [PAPER.md:128-134]) and intermittent faults.  A fault is
  * {opcode id, SM id, lane id, XOR bit mask}: the destination registers of every

@@ -41,7 +41,7 @@ namespace fi {
 
 constexpr uint32_t kFull = 0xFFFFFFFFu;
 constexpr int kLdgBatch = 4;          // independent LDGs issued together
-enum EmuMode { EMU_LEN = 0, EMU_TRACE = 1, EMU_INJ = 2, EMU_PROP = 3 };
+enum EmuMode { EMU_LEN = 0, EMU_TRACE = 1, EMU_INJ = 2, EMU_PROP = 3, EMU_PAGE = 4 };
 
 // ---- prepared program data (fi_program.aux) --------------------------------
 // per instance: the buffers its constant bank points into (count, then ids;
@@ -431,13 +431,38 @@ __device__ __forceinline__ bool ov_find(const Overlay& o, uint64_t va, uint32_t&
     return false;
 }
 
+// Faulty memory of one replica slot in batched propagation (K8): copy-on-write
+// 4 KB pages per buffer (page p of buffer b = page_base[b] + offset/4096);
+// ptab[p] = pool page holding the replica's words, or >= kPageClaim when the
+// replica's word is the golden state.  A load from a buffer whose pages were
+// dropped after its last golden reference (a wild load) marks the slot inexact.
+constexpr uint32_t kPageWords = 1024;
+constexpr uint32_t kPageNone = 0xFFFFFFFFu, kPageClaim = 0xFFFFFFFEu;
+struct PageView {
+    const uint32_t* ptab;
+    const uint32_t* pool;
+    const uint32_t* page_base;
+    const uint32_t* last_ref;
+    const uint32_t* dropped;     // bit per buffer
+    uint32_t* inexact;
+    uint32_t t;
+};
+__device__ __forceinline__ void page_find(const EmuProg& P, const PageView& V, uint64_t va, uint32_t& v) {
+    const uint64_t off = va - kVaBase;
+    const uint32_t b = __ldg(&P.gran[off >> 8]);
+    const uint64_t rel = off - __ldg(&P.buf[b].off);
+    const uint32_t e = V.ptab[__ldg(&V.page_base[b]) + (uint32_t)(rel >> 12)];
+    if (e < kPageClaim) v = __ldcg(&V.pool[(size_t)e * kPageWords + ((rel >> 2) & (kPageWords - 1))]);
+    else if (__ldg(&V.last_ref[b]) < V.t && ((V.dropped[b >> 5] >> (b & 31)) & 1u)) *V.inexact = 1u;
+}
+
 template <int MODE>
 __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const uint8_t* img,
                                           uint32_t k, uint32_t cta, uint32_t wic, uint32_t* __restrict__ R,
                                           uint32_t watchdog, fi_record* __restrict__ rec_out,
                                           fi_store* __restrict__ st_out, uint32_t st_cap, HookIn hook,
                                           uint32_t* __restrict__ ck, uint32_t ck_interval,
-                                          Overlay ov = Overlay{nullptr, 0}) {
+                                          Overlay ov = Overlay{nullptr, 0}, PageView pg = PageView{}) {
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t lt_mask = (1u << lane) - 1u;
     const fi_instance in = P.inst[k];
@@ -611,6 +636,10 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
                             uint32_t* vw = &vals[b].x;
                             for (uint32_t q = 0; q < (1u << lw); ++q) ov_find(ov, va + 4 * q, vw[q]);
                         }
+                        if (MODE == EMU_PAGE && ex && !c) {  // the replica's pages win
+                            uint32_t* vw = &vals[b].x;
+                            for (uint32_t q = 0; q < (1u << lw); ++q) page_find(P, pg, va + 4 * q, vw[q]);
+                        }
                         exs[b] = ex;
                         dsts[b] = D.z >> 16;
                         lws[b] = lw;
@@ -715,6 +744,10 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
                         uint32_t* vw = &v.x;
                         for (uint32_t q = 0; q < nw; ++q) ov_find(ov, va + 4 * q, vw[q]);
                     }
+                    if (MODE == EMU_PAGE) {                   // the replica's pages win
+                        uint32_t* vw = &v.x;
+                        for (uint32_t q = 0; q < nw; ++q) page_find(P, pg, va + 4 * q, vw[q]);
+                    }
                     F.wr(id, v.x);
                     if (lw >= 1) F.wr(id + 128, v.y);
                     if (lw >= 2) { F.wr(id + 256, v.z); F.wr(id + 384, v.w); }
@@ -732,7 +765,7 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
                         else if (lw == 1) *reinterpret_cast<uint2*>(dst) = make_uint2(v[0], v[1]);
                         else *reinterpret_cast<uint4*>(dst) = make_uint4(v[0], v[1], v[2], v[3]);
                     }
-                } else if (MODE == EMU_TRACE || MODE == EMU_PROP || step > hook.step) {
+                } else if (MODE == EMU_TRACE || MODE == EMU_PROP || MODE == EMU_PAGE || step > hook.step) {
                     if (ex) {
                         for (uint32_t i = 0; i < nw; ++i) {
                             const uint32_t e = nst + idx + i;

@@ -299,6 +299,9 @@ __global__ void __launch_bounds__(kWPB * 32) k_propagate(const PropArgs A) {
                 r.fault_kind = (uint8_t)fkind;
                 r.fault_pc = fpc;
                 A.inj[i] = r;
+            } else if (!Rj.fault_kind && fkind) {        // first downstream fault, run order
+                A.inj[i].fault_kind = (uint8_t)fkind;
+                A.inj[i].fault_pc = fpc;
             }
             A.inj[i].outcome = (uint8_t)outcome;
             A.inj[i].flags = (pdue && outcome != FI_DUE && outcome != FI_NOT_INJECTED) ? FI_POTENTIAL_DUE : 0;

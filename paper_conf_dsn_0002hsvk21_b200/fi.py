@@ -116,6 +116,8 @@ def lib():
             "fi_build_instance_index": (st, [vp, u32, vp, vp, vp]),
             "fi_select_sites_approx": (st, [vp, vp, vp, u32, vp, vp, u64, u32, vp, vp, vp]),
             "fi_inject_permanent_workspace": (sz, [u32, u32, u32, u32]),
+            "fi_classify_batched_workspace": (sz, [vp, u32, u32, u32, u32, u32]),
+            "fi_classify_batched": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, u32, u32, u32, u32, vp, sz, vp, vp]),
             "fi_inject_permanent": (st, [vp, vp, vp, vp, u32, vp, vp, vp, u32, u32, vp, u32, vp, sz, vp, vp]),
         }
         for name, (res, args) in sig.items():
@@ -434,6 +436,41 @@ def select_sites_approx(idx: InstanceIndex, sched: fi_schedule, j0: int, n: int,
     if status is None:
         st.check("fi_select_sites_approx")
     return sites
+
+
+def pend_capacity(gt: GoldenTrace) -> int:
+    """Update slots per replica and launch for K8: 2x the largest launch's golden
+    stores + 4096 (faulty extras; exceeding it is reported, never mis-classified)."""
+    gs = gt.gstore_off.cpu().numpy()
+    wb = gt.dp.prog.instances["warp_begin"].astype(np.int64)
+    we = gt.dp.prog.instances["warp_end"].astype(np.int64)
+    mx = int((gs[we] - gs[wb]).max()) if len(wb) else 0
+    return 2 * mx + 4096
+
+
+def classify_batched(gt: GoldenTrace, sites: torch.Tensor, n: int, out: torch.Tensor, log: torch.Tensor,
+                     log_cap: int, hist: torch.Tensor | None = None, unchecked: bool = False, batch: int | None = None,
+                     pool_pages: int | None = None, pend_cap: int | None = None, mem_budget: int = 24 << 30,
+                     status: DeviceStatus | None = None) -> torch.Tensor:
+    """fi_classify_batched (K8): whole-program outcomes for long multi-instance
+    programs, replica batches in lockstep over the launches."""
+    dev = gt.dp.device
+    if hist is None:
+        hist = torch.zeros((8, 4, 3), dtype=torch.int64, device=dev)
+    pend_cap = pend_capacity(gt) if pend_cap is None else pend_cap
+    batch = min(n, 512) if batch is None else batch
+    if pool_pages is None:                             # the rest of the budget after the fixed parts
+        fixed = lib().fi_classify_batched_workspace(C.byref(gt.dp.c), n, log_cap, batch, 1, pend_cap)
+        pool_pages = max(1024, (mem_budget - fixed) // (4096 + 12))
+    ws_n = lib().fi_classify_batched_workspace(C.byref(gt.dp.c), n, log_cap, batch, pool_pages, pend_cap)
+    ws = torch.empty(ws_n, dtype=torch.uint8, device=dev)
+    st = status or DeviceStatus(dev)
+    _check(lib().fi_classify_batched(C.byref(gt.dp.c), _p(gt.image), C.byref(gt.c), _p(sites), n, _p(out), _p(log),
+                                     log_cap, _p(hist), FI_UNCHECKED if unchecked else 0, batch, pool_pages, pend_cap,
+                                     _p(ws), ws_n, st.ptr, _stream()), "fi_classify_batched")
+    if status is None:
+        st.check("fi_classify_batched")
+    return hist
 
 
 def inject_permanent(gt: GoldenTrace, faults: np.ndarray, op_weights: torch.Tensor | None = None,
