@@ -92,9 +92,39 @@ __device__ __forceinline__ uint32_t cur_value(const K8Args& A, uint32_t s, uint6
     return gstate(A.P, A.img, va, t - 1);
 }
 
+// Does pool page e differ from the golden state after t of page p (buffer b)?  All
+// words of a page belong to one buffer, so the writer rule is uniform; words past
+// the buffer's end are 0.  One warp, 16-B loads.
+__device__ __forceinline__ bool page_differs(const K8Args& A, uint32_t e, uint32_t b, uint32_t p, int64_t t) {
+    const uint32_t lane = threadIdx.x & 31;
+    const int32_t wr = __ldg(&A.P.buf[b].writer);
+    const bool zero = wr >= 0 && (int64_t)wr > t;
+    const uint64_t boff = __ldg(&A.P.buf[b].off), bsz = __ldg(&A.P.buf[b].size);
+    const uint64_t rel0 = (uint64_t)(p - __ldg(&A.page_base[b])) << 12;
+    const uint4* pg = reinterpret_cast<const uint4*>(A.pool + (size_t)e * kPageWords);
+    bool d = false;
+#pragma unroll 4
+    for (uint32_t q = lane; q < kPageWords / 4; q += 32) {
+        const uint64_t rel = rel0 + 16ull * q;
+        const uint4 v = __ldcg(&pg[q]);
+        uint4 g = make_uint4(0, 0, 0, 0);
+        if (!zero && rel < bsz) g = __ldg(reinterpret_cast<const uint4*>(A.img + boff + rel));
+        d |= (v.x != g.x) | (v.y != g.y) | (v.z != g.z) | (v.w != g.w);
+    }
+    return __any_sync(kFull, d);
+}
+
 __device__ __forceinline__ void set_err(const K8Args& A, uint32_t s, uint32_t code) {
     A.slot[s].overflow = 1;
     FI_DEV_ERR(A.status, code);
+}
+
+// An update that leaves a word without a page at its golden value after t changes
+// nothing (k8_foreign accounts for the dropped entry through the golden log).
+__device__ __forceinline__ bool no_change(const K8Args& A, uint32_t s, uint64_t va, uint32_t v, int64_t t) {
+    uint32_t b, w;
+    const uint32_t p = page_of(A, va, b, w);
+    return A.ptab[(size_t)s * A.total_pages + p] == kPageNone && v == gstate(A.P, A.img, va, t);
 }
 
 // Updates of one warp (F = its stores in program order, G = its golden stores):
@@ -104,6 +134,35 @@ __device__ void warp_updates8(const K8Args& A, uint32_t s, uint32_t w_idx, const
                               const fi_store* G, uint64_t nG, int64_t t, bool mark_foreign) {
     const uint32_t lane = threadIdx.x & 31;
     fi_store* pend = A.pend + (size_t)s * A.pend_cap;
+    // fast path: the faulty warp stored exactly the golden addresses in the golden
+    // order (a golden warp stores each word once), so the updates are F itself
+    bool same = nF == nG;
+    for (uint64_t b = 0; b < nF && same; b += 32) {
+        const uint64_t j = b + lane;
+        same = __all_sync(kFull, j >= nF || F[j].va == G[j].va);
+    }
+    if (same) {
+        for (uint64_t b = 0; b < nF; b += 32) {
+            const uint64_t j = b + lane;
+            fi_store f{};
+            bool keep = false;
+            if (j < nF) {
+                f = F[j];
+                f.step = w_idx;
+                keep = !no_change(A, s, f.va, f.value, t);
+            }
+            const uint32_t m = __ballot_sync(kFull, keep);
+            uint32_t base = 0;
+            if (lane == 0 && m) base = atomicAdd(&A.slot[s].pend_n, (uint32_t)__popc(m));
+            base = __shfl_sync(kFull, base, 0);
+            if (keep) {
+                const uint32_t pos = base + __popc(m & ((1u << lane) - 1));
+                if (pos < A.pend_cap) pend[(size_t)pos] = f;
+                else set_err(A, s, FI_E_CAPACITY);
+            }
+        }
+        return;
+    }
     for (uint64_t b = 0; b < nF; b += 32) {
         const uint64_t j = b + lane;
         bool keep = false, foreign = false;
@@ -116,6 +175,7 @@ __device__ void warp_updates8(const K8Args& A, uint32_t s, uint32_t w_idx, const
                 foreign = true;
                 for (uint64_t q = 0; q < nG && foreign; ++q) foreign = G[q].va != f.va;
             }
+            if (keep && !foreign && no_change(A, s, f.va, f.value, t)) keep = false;
         }
         const uint32_t m = __ballot_sync(kFull, keep);
         uint32_t base = 0;
@@ -142,10 +202,10 @@ __device__ void warp_updates8(const K8Args& A, uint32_t s, uint32_t w_idx, const
             bool inF = false;
             for (uint64_t q = 0; q < nF && !inF; ++q) inF = F[q].va == va;
             if (!inF) {
-                keep = true;
                 g.va = va;
                 g.value = cur_value(A, s, va, t);
                 g.step = w_idx;
+                keep = !no_change(A, s, va, g.value, t);
             }
         }
         const uint32_t m = __ballot_sync(kFull, keep);
@@ -323,10 +383,14 @@ __global__ void __launch_bounds__(256) k8_alloc(K8Args A, uint32_t t) {
         const uint32_t b = sb;
         const uint64_t boff = __ldg(&A.P.buf[b].off), bsz = __ldg(&A.P.buf[b].size);
         const uint64_t rel0 = (uint64_t)(p - __ldg(&A.page_base[b])) << 12;
-        for (uint32_t w = threadIdx.x; w < kPageWords; w += blockDim.x) {
-            const uint64_t rel = rel0 + 4ull * w;
-            A.pool[(size_t)page * kPageWords + w] =
-                rel < bsz ? gstate(A.P, A.img, kVaBase + boff + rel, t) : 0u;
+        const int32_t wr = __ldg(&A.P.buf[b].writer);
+        const bool zero = wr >= 0 && (int64_t)wr > (int64_t)t;            // writer rule, golden after t
+        uint4* dst = reinterpret_cast<uint4*>(A.pool + (size_t)page * kPageWords);
+        for (uint32_t q = threadIdx.x; q < kPageWords / 4; q += blockDim.x) {
+            const uint64_t rel = rel0 + 16ull * q;
+            uint4 g = make_uint4(0, 0, 0, 0);
+            if (!zero && rel < bsz) g = __ldg(reinterpret_cast<const uint4*>(A.img + boff + rel));
+            dst[q] = g;
         }
         __syncthreads();
         if (threadIdx.x == 0) {
@@ -355,19 +419,32 @@ __global__ void k8_apply(K8Args A) {
     }
 }
 
-// ---- foreign updates: the one from the highest warp index among all updates of the word wins (C-14)
-__global__ void __launch_bounds__(32) k8_foreign(K8Args A) {
+// ---- foreign updates: among all updates of the word — the pending ones and the
+//      golden warp's (which may have been dropped as a no-op) — the one from the
+//      highest warp index wins (C-14)
+__global__ void __launch_bounds__(32) k8_foreign(K8Args A, uint32_t t) {
     const uint32_t s = blockIdx.x, lane = threadIdx.x;
     const uint32_t nf = min(A.slot[s].for_n, kForeignCap);
     if (!nf) return;
     const uint32_t n = min(A.slot[s].pend_n, A.pend_cap);
     const fi_store* pend = A.pend + (size_t)s * A.pend_cap;
     const uint32_t* pt = A.ptab + (size_t)s * A.total_pages;
+    const fi_instance in = A.P.inst[t];
+    const uint64_t g0 = A.gst_off[in.warp_begin], g1 = A.gst_off[in.warp_end];
     for (uint32_t q = 0; q < nf; ++q) {
         const fi_store f = A.forn[(size_t)s * kForeignCap + q];
         uint32_t mx = 0;
         for (uint32_t j = lane; j < n; j += 32)
             if (pend[j].va == f.va) mx = max(mx, (pend[j].step & 0x7FFFFFFFu) + 1);
+        for (uint64_t j = g0 + lane; j < g1; j += 32)
+            if (A.gst[j].va == f.va) {                 // golden writer of the word: its warp
+                uint32_t lo = in.warp_begin, hi = in.warp_end;
+                while (hi - lo > 1) {
+                    const uint32_t mid = (lo + hi) / 2;
+                    if (A.gst_off[mid] <= j) lo = mid; else hi = mid;
+                }
+                mx = max(mx, lo - in.warp_begin + 1);
+            }
         mx = __reduce_max_sync(kFull, mx);
         if (lane == 0 && mx == (f.step & 0x7FFFFFFFu) + 1) {
             uint32_t b, w;
@@ -379,13 +456,14 @@ __global__ void __launch_bounds__(32) k8_foreign(K8Args A) {
     }
 }
 
-// ---- return pages equal to the golden state (buffers t references) and pages of
-//      buffers past their last reference; a slot without pages is Masked
-__global__ void __launch_bounds__(256) k8_gc(K8Args A, uint32_t t) {
+// ---- return pages equal to the golden state (buffers t writes) and the pages of
+//      buffers past their last reference; a slot without pages is Masked.  One
+//      warp per page.
+__global__ void __launch_bounds__(1024) k8_gc(K8Args A, uint32_t t) {
     const uint32_t s = blockIdx.x;
     Slot& z = A.slot[s];
     if (!z.alive || z.k0 > t) return;
-    __shared__ uint32_t any_diff, freed;
+    const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5, nwb = blockDim.x >> 5;
     uint32_t* pt = A.ptab + (size_t)s * A.total_pages;
     const uint32_t* ib = A.P.ib + (size_t)t * (kInstBufs + 1);
     const uint32_t nref = __ldg(&ib[0]) > kInstBufs ? 0u : __ldg(&ib[0]);
@@ -393,39 +471,23 @@ __global__ void __launch_bounds__(256) k8_gc(K8Args A, uint32_t t) {
     for (uint32_t q = 0; q < nref + (d1 - d0); ++q) {
         const bool dying = q >= nref;
         const uint32_t b = dying ? __ldg(&A.dying[d0 + q - nref]) : __ldg(&ib[1 + q]);
+        if (!dying && __ldg(&A.P.buf[b].writer) != (int32_t)t) continue;   // unchanged by t's golden stores
         if (A.bcount[(size_t)s * A.n_buf + b] == 0) continue;
         const uint32_t pb = __ldg(&A.page_base[b]), pe = __ldg(&A.page_base[b + 1]);
-        const uint64_t boff = __ldg(&A.P.buf[b].off), bsz = __ldg(&A.P.buf[b].size);
-        if (threadIdx.x == 0) freed = 0;
-        __syncthreads();
-        for (uint32_t p = pb; p < pe; ++p) {
+        for (uint32_t p = pb + wib; p < pe; p += nwb) {
             const uint32_t e = pt[p];
             if (e >= kPageClaim) continue;
-            if (threadIdx.x == 0) any_diff = 0;
-            __syncthreads();
-            {
-                const uint64_t rel0 = (uint64_t)(p - pb) << 12;
-                bool d = false;
-                for (uint32_t w = threadIdx.x; w < kPageWords && !d; w += blockDim.x) {
-                    const uint64_t rel = rel0 + 4ull * w;
-                    const uint32_t g = rel < bsz ? gstate(A.P, A.img, kVaBase + boff + rel, t) : 0u;
-                    d = __ldcg(&A.pool[(size_t)e * kPageWords + w]) != g;
-                }
-                if (d) atomicOr(&any_diff, 1u);
-            }
-            __syncthreads();
-            if (threadIdx.x == 0 && (dying || !any_diff)) {
+            const bool diff = page_differs(A, e, b, p, t);
+            if (lane == 0 && (dying || !diff)) {
                 pt[p] = kPageNone;
                 A.free_stack[atomicAdd(A.free_top, 1)] = e;
-                A.bcount[(size_t)s * A.n_buf + b] -= 1;
-                z.npages -= 1;
-                if (dying && any_diff) freed = 1;          // corrupted words dropped: later wild loads are inexact
+                atomicSub(&A.bcount[(size_t)s * A.n_buf + b], 1u);
+                atomicSub(&z.npages, 1u);
+                if (dying && diff) atomicOr(&A.dropped[(size_t)s * A.dwords + (b >> 5)], 1u << (b & 31));
             }
-            __syncthreads();
         }
-        if (threadIdx.x == 0 && dying && freed) A.dropped[(size_t)s * A.dwords + (b >> 5)] |= 1u << (b & 31);
-        __syncthreads();
     }
+    __syncthreads();
     if (threadIdx.x == 0) {
         if (z.fault_key != ~0ull) z.alive = 0;                       // DUE (C-9, C-10): nothing left to decide
         else if (z.npages == 0) z.alive = 0;                         // golden state again: Masked from here on
@@ -645,8 +707,8 @@ extern "C" fi_status fi_classify_batched(const fi_program* p, const uint8_t* ima
             k8_mark<<<dim3(std::max<uint32_t>(1, fix_grid / batch + 1), batch), 256, 0, s>>>(A);
             k8_alloc<<<fix_grid, 256, 0, s>>>(A, tt);
             k8_apply<<<dim3(std::max<uint32_t>(1, fix_grid / batch + 1), batch), 256, 0, s>>>(A);
-            k8_foreign<<<batch, 32, 0, s>>>(A);
-            k8_gc<<<batch, 256, 0, s>>>(A, tt);
+            k8_foreign<<<batch, 32, 0, s>>>(A, tt);
+            k8_gc<<<batch, 1024, 0, s>>>(A, tt);
             if ((e = launch_status())) return e;
         }
         k8_final<<<batch, 256, 0, s>>>(A);
