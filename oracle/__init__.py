@@ -154,7 +154,10 @@ class Golden:
 
     def __del__(self):
         if getattr(self, "h", None):
-            lib().orc_free(self.h)
+            try:
+                lib().orc_free(self.h)
+            except TypeError:                          # interpreter shutdown: module globals gone
+                pass
             self.h = None
 
     def counts(self) -> np.ndarray:
