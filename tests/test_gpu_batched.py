@@ -88,3 +88,17 @@ def test_k8_pool_exhaustion_is_reported(F):
     assert e.value.code == F.FI_E_CAPACITY
     gi = F.as_numpy(out, F.INJ_DTYPE, n)
     assert (gi["outcome"] == 0xFF).any()
+
+
+def test_k8_c4_mini(F):
+    """mini-C4 (ResNet-50 v1.5 shape, width 8, 32x32: 72 launches, 53 convolutions):
+    trace, counts and whole-program outcomes (K8 and K7) against the oracle."""
+    from fi_inputs import resnet as R
+    prog = R.c4(full=False)
+    g = O.Golden(prog)
+    dp = F.DeviceProgram(prog)
+    gt = F.golden_run(dp)
+    assert np.array_equal(F.as_numpy(gt.rec, F.RECORD_DTYPE, gt.n_rec), g.trace())
+    assert np.array_equal(gt.image.cpu().numpy(), g.final_image())
+    oi = _run(F, prog, R.C4_CAMPAIGN_SEED, [F.G_GP, F.G_FP32, F.G_LD, F.G_PR], [0, 1, 2, 3], 300)
+    assert (oi["outcome"] == O.SDC).any() and (oi["outcome"] == O.MASKED).any()
