@@ -102,3 +102,19 @@ def test_k8_c4_mini(F):
     assert np.array_equal(gt.image.cpu().numpy(), g.final_image())
     oi = _run(F, prog, R.C4_CAMPAIGN_SEED, [F.G_GP, F.G_FP32, F.G_LD, F.G_PR], [0, 1, 2, 3], 300)
     assert (oi["outcome"] == O.SDC).any() and (oi["outcome"] == O.MASKED).any()
+
+
+@pytest.mark.parametrize("which", range(5))
+def test_k8_c5_mini(F, which):
+    """mini C5 suite (stencil FP32, D3Q19 LBM FP64, LJ MD FP64 with divergent
+    cutoff branches, EP FP64+int, CG): golden trace and whole-program outcomes."""
+    from fi_inputs import hpc as H
+    prog = H.c5(full=False)[which]
+    g = O.Golden(prog)
+    dp = F.DeviceProgram(prog)
+    gt = F.golden_run(dp)
+    assert np.array_equal(F.as_numpy(gt.rec, F.RECORD_DTYPE, gt.n_rec), g.trace())
+    assert np.array_equal(gt.image.cpu().numpy(), g.final_image())
+    groups = [F.G_GP, F.G_GPPR, F.G_LD, F.G_PR, F.G_FP64 if which in (1, 2, 3, 4) else F.G_FP32]
+    oi = _run(F, prog, H.C5_CAMPAIGN_SEED + which, groups, [0, 1, 2, 3], 250)
+    assert (oi["outcome"] == O.SDC).any()
