@@ -65,7 +65,11 @@ class Campaign:
     program on this rank's GPU (all work in libfi kernels)."""
 
     def __init__(self, prog, seed: int, groups, bfms, n_replicas: int, rank: int = 0, world: int = 1,
-                 device="cuda", group=None, host_tensors: dict | None = None):
+                 device="cuda", group=None, host_tensors: dict | None = None, propagation: str = "auto"):
+        """propagation: how a multi-launch program's outcome is computed — "k7"
+        (fi_classify: one CUDA warp walks a replica's later launches), "k8"
+        (fi_classify_batched: replica batches in lockstep over the launches), or
+        "auto" (K8 from 64 launches on).  Both give identical results."""
         from . import fi
         self.fi = fi
         self.prog = prog
@@ -88,6 +92,7 @@ class Campaign:
         self.hist = torch.zeros((8, 4, 3), dtype=torch.int64, device=self.device)
         self.status = fi.DeviceStatus(self.device)
         self.inj_ws = torch.empty(fi.lib().fi_inject_workspace(nloc), dtype=torch.uint8, device=self.device)
+        self.batched = propagation == "k8" or (propagation == "auto" and self.dp.n_inst >= 64)
 
     @property
     def n_local(self):
@@ -118,7 +123,10 @@ class Campaign:
         fi.inject(self.gt, self.sites, n, self.cap, self.out, self.log, self.status, self.inj_ws)
         mark("inject")
         self.hist.zero_()
-        fi.classify(self.gt, self.sites, n, self.out, self.log, self.cap, self.hist, self.status)
+        if self.batched:
+            fi.classify_batched(self.gt, self.sites, n, self.out, self.log, self.cap, self.hist, status=self.status)
+        else:
+            fi.classify(self.gt, self.sites, n, self.out, self.log, self.cap, self.hist, self.status)
         mark("classify")
         allreduce_sum_(self.hist, self.group)
         mark("end")
