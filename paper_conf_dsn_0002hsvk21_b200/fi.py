@@ -458,7 +458,10 @@ def classify_batched(gt: GoldenTrace, sites: torch.Tensor, n: int, out: torch.Te
     if hist is None:
         hist = torch.zeros((8, 4, 3), dtype=torch.int64, device=dev)
     pend_cap = pend_capacity(gt) if pend_cap is None else pend_cap
-    batch = min(n, 512) if batch is None else batch
+    if batch is None:                                  # per-slot parts within half the budget
+        w1 = lib().fi_classify_batched_workspace(C.byref(gt.dp.c), n, log_cap, 1, 1, pend_cap)
+        w2 = lib().fi_classify_batched_workspace(C.byref(gt.dp.c), n, log_cap, 2, 1, pend_cap)
+        batch = int(max(1, min(n, 512, (mem_budget // 2 - w1) // max(w2 - w1, 1) + 1)))
     if pool_pages is None:                             # the rest of the budget after the fixed parts
         fixed = lib().fi_classify_batched_workspace(C.byref(gt.dp.c), n, log_cap, batch, 1, pend_cap)
         pool_pages = max(1024, (mem_budget - fixed) // (4096 + 12))
