@@ -319,6 +319,18 @@ fi_status fi_inject_permanent(const fi_program* p, const uint8_t* image, const f
                               uint32_t ov_words, uint64_t* hist, uint32_t flags, void* ws, size_t ws_bytes,
                               uint32_t* dev_status, void* stream);
 
+/* Rows f2/f3 on K8: fi_inject_permanent for long multi-launch programs — same
+ * faults, definition and outputs (out[i], opcode-weighted hist[3]); every replica
+ * runs from the first launch with the opcode hook armed on the faulty SM's CTAs,
+ * launches re-executed where the opcode runs on that SM or corrupted pages are
+ * referenced.  Scratch: fi_classify_batched_workspace(p, n, log_cap, batch,
+ * pool_pages, pend_cap); capacities as for fi_classify_batched. */
+fi_status fi_inject_permanent_batched(const fi_program* p, const uint8_t* image, const fi_trace* t,
+                                      const fi_pfault* faults, uint32_t n, const uint64_t* op_weights, fi_inj* out,
+                                      uint32_t log_cap, uint64_t* hist, uint32_t flags, uint32_t batch,
+                                      uint32_t pool_pages, uint32_t pend_cap, void* ws, size_t ws_bytes,
+                                      uint32_t* dev_status, void* stream);
+
 /* Table II parameter file, one parameter per line in Table II order
  * [PAPER.md:88]: arch state id, bit-flip model, kernel name, kernel count,
  * instruction count, destination register value, bit-pattern value (the two

@@ -477,7 +477,7 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
     const bool use_ck = ck != nullptr && ck_interval != 0;
     // permanent / intermittent hook (row f2/f3): every step is inspected, so the
     // straight-line fast paths are off while it is armed
-    const bool perm = MODE == EMU_PROP && hook.perm_on;
+    const bool perm = (MODE == EMU_PROP || MODE == EMU_PAGE) && hook.perm_on;
 
     uint32_t nl = in.block - wic * 32;
     bool live = lane < (nl > 32 ? 32u : nl);

@@ -42,7 +42,7 @@ constexpr uint32_t kNoRep = 0xFFFFFFFFu;
 struct Slot {
     uint32_t rep, k0, alive, outcome;
     uint32_t npages, inexact, overflow, pend_n;
-    uint32_t for_n, pdue, pad0, pad1;
+    uint32_t for_n, pdue, perm, pad1;                // perm: permanent / intermittent fault (rows f2/f3)
     unsigned long long fault_key;                    // (t << 43 | w << 19 | kind << 16 | pc), min = first
     unsigned long long pdue_key;
 };
@@ -65,6 +65,8 @@ struct K8Args {
     fi_store* scratch;                               // [resident warps][log_cap]
     const uint32_t* dying; const uint32_t* dying_off;   // CSR over instances
     uint32_t flags; uint32_t* status; uint64_t* hist;
+    const fi_pfault* pf; const uint64_t* opw;        // permanent mode (else null)
+    const uint32_t* kop;                             // per static kernel: bit op set iff the kernel has opcode op
 };
 
 __device__ __forceinline__ uint32_t buf_of(const EmuProg& P, uint64_t va) { return __ldg(&P.gran[(va - kVaBase) >> 8]); }
@@ -228,7 +230,12 @@ __global__ void k8_setup(K8Args A, const uint32_t* reps, uint32_t nb) {
     z.rep = kNoRep;
     z.fault_key = ~0ull;
     z.pdue_key = ~0ull;
-    if (s < nb) {
+    if (s < nb && A.pf) {                            // permanent: armed from the first launch
+        z.rep = reps[s];
+        z.alive = 1;
+        z.outcome = FI_MASKED;
+        z.perm = 1;
+    } else if (s < nb) {
         const uint32_t i = reps[s];
         const fi_site S = A.sites[i];
         const fi_inj R = A.inj[i];
@@ -263,11 +270,17 @@ __global__ void __launch_bounds__(1024) k8_activate(K8Args A, uint32_t t) {
         z.pend_n = 0;
         z.for_n = 0;
         bool act = false;
-        if (z.alive && z.k0 < t && !z.overflow) {
+        if (z.alive && (z.perm || z.k0 < t) && !z.overflow) {
             if (nref > kInstBufs) act = true;
             else
                 for (uint32_t q = 0; q < nref && !act; ++q)
                     act = A.bcount[(size_t)s * A.n_buf + __ldg(&ib[1 + q])] != 0;
+            if (z.perm && !act) {                    // the faulty SM runs the opcode in t
+                const fi_pfault F = A.pf[z.rep];
+                const fi_instance in = A.P.inst[t];
+                const uint32_t nsm = F.n_sm ? F.n_sm : 148u;
+                act = F.sm < nsm && F.sm < in.grid && ((__ldg(&A.kop[in.kernel]) >> (F.opcode & 31)) & 1u);
+            }
         }
         if (act) A.active[atomicAdd(&cnt, 1u)] = s;
     }
@@ -298,8 +311,17 @@ __global__ void __launch_bounds__(kWPB8 * 32) k8_exec(K8Args A, uint32_t t) {
         const uint32_t watchdog = wd > 0xFFFFFFFFull ? 0xFFFFFFFFu : (uint32_t)wd;
         PageView pv{A.ptab + (size_t)s * A.total_pages, A.pool, A.page_base, A.last_ref,
                     A.dropped + (size_t)s * A.dwords, &A.slot[s].inexact, t};
+        HookIn h{};
+        if (A.pf) {                                   // CTAs on the faulty SM (C-21)
+            const fi_pfault F = A.pf[A.slot[s].rep];
+            const uint32_t nsm = F.n_sm ? F.n_sm : 148u;
+            if ((lw / wpc) % nsm == F.sm) {
+                h.perm_on = true; h.perm_op = F.opcode; h.perm_lane = F.lane; h.perm_mask = F.mask;
+                h.perm_q = F.q32; h.perm_rep = A.slot[s].rep; h.perm_warp = w; h.perm_seed = F.seed;
+            }
+        }
         const EmuOut o = emulate<EMU_PAGE>(A.P, nullptr, A.img, t, lw / wpc, lw % wpc, R, watchdog, nullptr, scr,
-                                           A.log_cap, HookIn{}, nullptr, 0, Overlay{nullptr, 0}, pv);
+                                           A.log_cap, h, nullptr, 0, Overlay{nullptr, 0}, pv);
         if (o.fault) {
             if (lane == 0) {
                 const unsigned long long key = ((unsigned long long)t << 43) | ((unsigned long long)lw << 19) |
@@ -322,7 +344,7 @@ __global__ void __launch_bounds__(kWPB8 * 32) k8_k0(K8Args A, uint32_t t) {
     const uint32_t s = blockIdx.x * kWPB8 + (threadIdx.x >> 5);
     if (s >= A.B) return;
     const Slot z = A.slot[s];
-    if (!z.alive || z.k0 != t || z.overflow) return;
+    if (!z.alive || z.perm || z.k0 != t || z.overflow) return;
     const fi_site S = A.sites[z.rep];
     const fi_inj Rj = A.inj[z.rep];
     const fi_store* G = A.gst + A.gst_off[S.warp];
@@ -490,7 +512,7 @@ __global__ void __launch_bounds__(1024) k8_gc(K8Args A, uint32_t t) {
     __syncthreads();
     if (threadIdx.x == 0) {
         if (z.fault_key != ~0ull) z.alive = 0;                       // DUE (C-9, C-10): nothing left to decide
-        else if (z.npages == 0) z.alive = 0;                         // golden state again: Masked from here on
+        else if (z.npages == 0 && !z.perm) z.alive = 0;              // golden state again: Masked from here on
     }
 }
 
@@ -527,6 +549,7 @@ __global__ void __launch_bounds__(256) k8_final(K8Args A) {
     }
     if (threadIdx.x == 0) {
         fi_inj& r = A.inj[z.rep];
+        if (z.perm) { r = fi_inj{}; r.mask = A.pf[z.rep].mask; }
         const bool pdue = z.pdue || z.pdue_key != ~0ull;
         if (!r.fault_kind) {                                         // first downstream fault, run order
             const unsigned long long key = z.fault_key != ~0ull ? z.fault_key : z.pdue_key;
@@ -535,6 +558,9 @@ __global__ void __launch_bounds__(256) k8_final(K8Args A) {
         r.outcome = (uint8_t)outcome;
         r.flags = (pdue && outcome != FI_DUE && outcome != FI_NOT_INJECTED && outcome != 0xFF) ? FI_POTENTIAL_DUE : 0;
         if (outcome == 0xFF) FI_DEV_ERR(A.status, FI_E_CAPACITY);
+        else if (z.perm)                                             // opcode-weighted outcomes
+            atomicAdd((unsigned long long*)&A.hist[outcome],
+                      (unsigned long long)(A.opw ? A.opw[A.pf[z.rep].opcode & (FI_NOPS - 1)] : 1ull));
         else if (outcome != FI_NOT_INJECTED) {
             const fi_site S = A.sites[z.rep];
             atomicAdd((unsigned long long*)&A.hist[((uint32_t)S.group * 4 + S.bfm) * 3 + outcome], 1ull);
@@ -549,7 +575,7 @@ using namespace fi;
 
 namespace {
 struct K8Layout { size_t slot, ptab, bcount, dropped, pool, fstack, ftop, pend, forn, active, nact, work, need, nneed,
-                  scratch, page_base, last_ref, dying_off, dying, reps, total; };
+                  scratch, page_base, last_ref, dying_off, dying, reps, kop, total; };
 K8Layout k8_layout(uint64_t image_bytes, uint32_t n_buf, uint32_t n_inst, uint32_t n, uint32_t B, uint32_t pool_pages,
                    uint32_t pend_cap, uint32_t log_cap, uint32_t scratch_warps) {
     const uint64_t tp = image_bytes / 4096 + n_buf + 1;          // >= sum of per-buffer pages
@@ -577,6 +603,7 @@ K8Layout k8_layout(uint64_t image_bytes, uint32_t n_buf, uint32_t n_inst, uint32
     L.dying_off = take(((size_t)n_inst + 1) * 4);
     L.dying = take((size_t)n_buf * 4);
     L.reps = take((size_t)n * 4);
+    L.kop = take(4096);
     L.total = o;
     return L;
 }
@@ -595,12 +622,13 @@ extern "C" size_t fi_classify_batched_workspace(const fi_program* p, uint32_t n,
                      k8_scratch_warps()).total;
 }
 
-extern "C" fi_status fi_classify_batched(const fi_program* p, const uint8_t* image, const fi_trace* t,
-                                         const fi_site* sites, uint32_t n, fi_inj* out, const fi_store* log,
-                                         uint32_t log_cap, uint64_t* hist, uint32_t flags, uint32_t batch,
-                                         uint32_t pool_pages, uint32_t pend_cap, void* ws, size_t ws_bytes,
-                                         uint32_t* dev_status, void* stream) {
-    if (!p || !image || !t || !sites || !out || !hist || !dev_status || !p->aux || !p->inst_host) return FI_E_ARG;
+static fi_status k8_run(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
+                        const fi_pfault* pf, const uint64_t* opw, uint32_t n, fi_inj* out, const fi_store* log,
+                        uint32_t log_cap, uint64_t* hist, uint32_t flags, uint32_t batch, uint32_t pool_pages,
+                        uint32_t pend_cap, void* ws, size_t ws_bytes, uint32_t* dev_status, void* stream) {
+    if (!p || !image || !t || (!sites && !pf) || !out || !hist || !dev_status || !p->aux || !p->inst_host ||
+        !p->code_host)
+        return FI_E_ARG;
     if (n == 0) return FI_OK;
     if (!batch || !pool_pages || !pend_cap) return FI_E_ARG;
     const uint32_t sw = k8_scratch_warps();
@@ -611,12 +639,13 @@ extern "C" fi_status fi_classify_batched(const fi_program* p, const uint8_t* ima
     // ---- host-side tables: per-buffer page numbering, last reference, dying lists
     std::vector<fi_buffer> bufs(p->n_buf);
     std::vector<uint32_t> ib((size_t)p->n_inst * (kInstBufs + 1));
-    std::vector<fi_site> hs(n);
+    std::vector<fi_site> hs(sites ? n : 0);
     const AuxLayout AL = aux_layout(p->image_bytes, p->n_code, p->n_inst);
     if ((e = cuda_status(cudaMemcpyAsync(bufs.data(), p->buf, bufs.size() * sizeof(fi_buffer), cudaMemcpyDeviceToHost, s))) ||
         (e = cuda_status(cudaMemcpyAsync(ib.data(), reinterpret_cast<const char*>(p->aux) + AL.ib, ib.size() * 4,
                                          cudaMemcpyDeviceToHost, s))) ||
-        (e = cuda_status(cudaMemcpyAsync(hs.data(), sites, (size_t)n * sizeof(fi_site), cudaMemcpyDeviceToHost, s))) ||
+        (sites && (e = cuda_status(cudaMemcpyAsync(hs.data(), sites, (size_t)n * sizeof(fi_site),
+                                                   cudaMemcpyDeviceToHost, s)))) ||
         (e = cuda_status(cudaStreamSynchronize(s))))
         return e;
     std::vector<uint32_t> page_base(p->n_buf + 1, 0), last_ref(p->n_buf, 0);
@@ -645,7 +674,19 @@ extern "C" fi_status fi_classify_batched(const fi_program* p, const uint8_t* ima
     // replicas in order of their faulty instance, batched
     std::vector<uint32_t> order(n);
     for (uint32_t i = 0; i < n; ++i) order[i] = i;
-    std::stable_sort(order.begin(), order.end(), [&](uint32_t a, uint32_t b) { return hs[a].instance < hs[b].instance; });
+    if (sites)
+        std::stable_sort(order.begin(), order.end(), [&](uint32_t a, uint32_t b) { return hs[a].instance < hs[b].instance; });
+    // per static kernel: which opcodes it contains (permanent faults arm only where the opcode runs)
+    if (p->n_kern > 1024) return FI_E_ARG;
+    std::vector<uint32_t> kop(std::max<uint32_t>(p->n_kern, 1), 0);
+    {
+        std::vector<fi_kernel> kh(p->n_kern);
+        if (p->n_kern &&
+            (e = cuda_status(cudaMemcpy(kh.data(), p->kern, kh.size() * sizeof(fi_kernel), cudaMemcpyDeviceToHost))))
+            return e;
+        for (uint32_t k = 0; k < p->n_kern; ++k)
+            for (uint32_t q = 0; q < kh[k].code_len; ++q) kop[k] |= 1u << (p->code_host[kh[k].code_off + q].op & 31);
+    }
 
     char* w = reinterpret_cast<char*>(ws);
     K8Args A;
@@ -671,12 +712,16 @@ extern "C" fi_status fi_classify_batched(const fi_program* p, const uint8_t* ima
     A.dying_off = reinterpret_cast<uint32_t*>(w + L.dying_off);
     A.dying = reinterpret_cast<uint32_t*>(w + L.dying);
     A.flags = flags; A.status = dev_status; A.hist = hist;
+    A.pf = pf; A.opw = opw;
+    A.kop = reinterpret_cast<uint32_t*>(w + L.kop);
     uint32_t* d_reps = reinterpret_cast<uint32_t*>(w + L.reps);
     if ((e = cuda_status(cudaMemcpyAsync(const_cast<uint32_t*>(A.page_base), page_base.data(), page_base.size() * 4, cudaMemcpyHostToDevice, s))) ||
         (e = cuda_status(cudaMemcpyAsync(const_cast<uint32_t*>(A.last_ref), last_ref.data(), last_ref.size() * 4, cudaMemcpyHostToDevice, s))) ||
         (e = cuda_status(cudaMemcpyAsync(const_cast<uint32_t*>(A.dying_off), dying_off.data(), dying_off.size() * 4, cudaMemcpyHostToDevice, s))) ||
         (!dying.empty() &&
          (e = cuda_status(cudaMemcpyAsync(const_cast<uint32_t*>(A.dying), dying.data(), dying.size() * 4, cudaMemcpyHostToDevice, s)))) ||
+        (e = cuda_status(cudaMemcpyAsync(const_cast<uint32_t*>(A.kop), kop.data(), kop.size() * 4,
+                                         cudaMemcpyHostToDevice, s))) ||
         (e = cuda_status(cudaMemcpyAsync(d_reps, order.data(), (size_t)n * 4, cudaMemcpyHostToDevice, s))))
         return e;
 
@@ -692,7 +737,7 @@ extern "C" fi_status fi_classify_batched(const fi_program* p, const uint8_t* ima
 
     for (uint32_t b0 = 0; b0 < n; b0 += batch) {
         const uint32_t nb = std::min(batch, n - b0);
-        const uint32_t kmin = hs[order[b0]].instance;
+        const uint32_t kmin = sites ? hs[order[b0]].instance : 0u;
         if ((e = cuda_status(cudaMemsetAsync(A.ptab, 0xFF, (size_t)batch * A.total_pages * 4, s))) ||
             (e = cuda_status(cudaMemsetAsync(A.bcount, 0, (size_t)batch * p->n_buf * 4, s))) ||
             (e = cuda_status(cudaMemsetAsync(A.dropped, 0, (size_t)batch * A.dwords * 4, s))))
@@ -702,7 +747,7 @@ extern "C" fi_status fi_classify_batched(const fi_program* p, const uint8_t* ima
         if ((e = launch_status())) return e;
         for (uint32_t tt = kmin; tt < p->n_inst; ++tt) {
             k8_activate<<<1, 1024, 0, s>>>(A, tt);
-            if (tt > kmin) k8_exec<<<exec_grid, kWPB8 * 32, smem, s>>>(A, tt);
+            if (tt > kmin || pf) k8_exec<<<exec_grid, kWPB8 * 32, smem, s>>>(A, tt);
             k8_k0<<<(batch + kWPB8 - 1) / kWPB8, kWPB8 * 32, 0, s>>>(A, tt);
             k8_mark<<<dim3(std::max<uint32_t>(1, fix_grid / batch + 1), batch), 256, 0, s>>>(A);
             k8_alloc<<<fix_grid, 256, 0, s>>>(A, tt);
@@ -715,4 +760,24 @@ extern "C" fi_status fi_classify_batched(const fi_program* p, const uint8_t* ima
         if ((e = launch_status())) return e;
     }
     return FI_OK;
+}
+
+extern "C" fi_status fi_classify_batched(const fi_program* p, const uint8_t* image, const fi_trace* t,
+                                         const fi_site* sites, uint32_t n, fi_inj* out, const fi_store* log,
+                                         uint32_t log_cap, uint64_t* hist, uint32_t flags, uint32_t batch,
+                                         uint32_t pool_pages, uint32_t pend_cap, void* ws, size_t ws_bytes,
+                                         uint32_t* dev_status, void* stream) {
+    if (!sites) return FI_E_ARG;
+    return k8_run(p, image, t, sites, nullptr, nullptr, n, out, log, log_cap, hist, flags, batch, pool_pages,
+                  pend_cap, ws, ws_bytes, dev_status, stream);
+}
+
+extern "C" fi_status fi_inject_permanent_batched(const fi_program* p, const uint8_t* image, const fi_trace* t,
+                                                 const fi_pfault* faults, uint32_t n, const uint64_t* op_weights,
+                                                 fi_inj* out, uint32_t log_cap, uint64_t* hist, uint32_t flags,
+                                                 uint32_t batch, uint32_t pool_pages, uint32_t pend_cap, void* ws,
+                                                 size_t ws_bytes, uint32_t* dev_status, void* stream) {
+    if (!faults) return FI_E_ARG;
+    return k8_run(p, image, t, nullptr, faults, op_weights, n, out, nullptr, log_cap, hist, flags, batch, pool_pages,
+                  pend_cap, ws, ws_bytes, dev_status, stream);
 }

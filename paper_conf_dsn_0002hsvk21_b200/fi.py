@@ -117,6 +117,8 @@ def lib():
             "fi_select_sites_approx": (st, [vp, vp, vp, u32, vp, vp, u64, u32, vp, vp, vp]),
             "fi_inject_permanent_workspace": (sz, [u32, u32, u32, u32]),
             "fi_classify_batched_workspace": (sz, [vp, u32, u32, u32, u32, u32]),
+            "fi_inject_permanent_batched": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, u32, u32, u32, u32, vp, sz,
+                                                 vp, vp]),
             "fi_classify_batched": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, u32, u32, u32, u32, vp, sz, vp, vp]),
             "fi_inject_permanent": (st, [vp, vp, vp, vp, u32, vp, vp, vp, u32, u32, vp, u32, vp, sz, vp, vp]),
         }
@@ -474,6 +476,36 @@ def classify_batched(gt: GoldenTrace, sites: torch.Tensor, n: int, out: torch.Te
     if status is None:
         st.check("fi_classify_batched")
     return hist
+
+
+def inject_permanent_batched(gt: GoldenTrace, faults: np.ndarray, op_weights: torch.Tensor | None = None,
+                             unchecked: bool = False, batch: int | None = None, pool_pages: int | None = None,
+                             pend_cap: int | None = None, mem_budget: int = 24 << 30):
+    """fi_inject_permanent_batched (rows f2/f3 on K8).  Returns (inj [n*24] u8, weighted hist [3] i64)."""
+    dev = gt.dp.device
+    f = np.ascontiguousarray(faults, dtype=PFAULT_DTYPE)
+    n = len(f)
+    ft = torch.from_numpy(f.view(np.uint8).copy()).to(dev)
+    out = torch.zeros(max(n, 1) * 24, dtype=torch.uint8, device=dev)
+    hist = torch.zeros(3, dtype=torch.int64, device=dev)
+    cap = log_capacity(gt)
+    pend_cap = pend_capacity(gt) if pend_cap is None else pend_cap
+    if batch is None:
+        w1 = lib().fi_classify_batched_workspace(C.byref(gt.dp.c), n, cap, 1, 1, pend_cap)
+        w2 = lib().fi_classify_batched_workspace(C.byref(gt.dp.c), n, cap, 2, 1, pend_cap)
+        batch = int(max(1, min(n, 512, (mem_budget // 2 - w1) // max(w2 - w1, 1) + 1)))
+    if pool_pages is None:
+        fixed = lib().fi_classify_batched_workspace(C.byref(gt.dp.c), n, cap, batch, 1, pend_cap)
+        pool_pages = max(1024, (mem_budget - fixed) // (4096 + 12))
+    ws_n = lib().fi_classify_batched_workspace(C.byref(gt.dp.c), n, cap, batch, pool_pages, pend_cap)
+    ws = torch.empty(ws_n, dtype=torch.uint8, device=dev)
+    st = DeviceStatus(dev)
+    _check(lib().fi_inject_permanent_batched(C.byref(gt.dp.c), _p(gt.image), C.byref(gt.c), _p(ft), n,
+                                             _p(op_weights), _p(out), cap, _p(hist),
+                                             FI_UNCHECKED if unchecked else 0, batch, pool_pages, pend_cap, _p(ws),
+                                             ws_n, st.ptr, _stream()), "fi_inject_permanent_batched")
+    st.check("fi_inject_permanent_batched")
+    return out, hist
 
 
 def inject_permanent(gt: GoldenTrace, faults: np.ndarray, op_weights: torch.Tensor | None = None,

@@ -46,13 +46,14 @@ def _faults(prog, n, seed, intermittent):
     return f
 
 
-def _parity(F, prog, n, seed, intermittent=False, unchecked=False):
+def _parity(F, prog, n, seed, intermittent=False, unchecked=False, batched=False):
     g = O.Golden(prog)
     dp = F.DeviceProgram(prog)
     gt = F.golden_run(dp)
     f = _faults(prog, n, seed, intermittent)
     opw = np.arange(1, F.FI_NOPS + 1, dtype=np.int64) * 3
-    out, hist = F.inject_permanent(gt, f, op_weights=torch.from_numpy(opw).cuda(), unchecked=unchecked)
+    inj = F.inject_permanent_batched if batched else F.inject_permanent
+    out, hist = inj(gt, f, op_weights=torch.from_numpy(opw).cuda(), unchecked=unchecked)
     gi = F.as_numpy(out, F.INJ_DTYPE, n)
     oi = g.inject_permanent(f, mode=O.MODE_FULL | (O.UNCHECKED if unchecked else 0))
     bad = np.nonzero(gi["outcome"] != oi["outcome"])[0]
@@ -90,4 +91,22 @@ def test_permanent_parity_sgemm_mini(F):
 
 def test_permanent_parity_c3_mini(F):
     oi = _parity(F, P.c3(full=False), 64, 17)
+    assert (oi["outcome"] == O.SDC).any()
+
+
+@pytest.mark.parametrize("maker,intermittent,unchecked", [
+    (lambda: P.vector_add(n=1000), False, False),
+    (lambda: P.multi_instance_chain(5), False, False),
+    (lambda: P.multi_instance_chain(4, n=300, block=96), True, True),
+    (lambda: P.scatter_chain(), False, False),
+    (lambda: P.c3(full=False), False, False),
+])
+def test_permanent_parity_k8(F, maker, intermittent, unchecked):
+    """Rows f2/f3 on K8 (fi_inject_permanent_batched) against the oracle."""
+    _parity(F, maker(), 120, 21, intermittent=intermittent, unchecked=unchecked, batched=True)
+
+
+def test_permanent_parity_k8_c4_mini(F):
+    from fi_inputs import resnet as R
+    oi = _parity(F, R.c4(full=False), 64, 22, batched=True)
     assert (oi["outcome"] == O.SDC).any()
