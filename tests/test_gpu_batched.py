@@ -17,7 +17,7 @@ def F():
     return fi
 
 
-def _run(F, prog, seed, groups, bfms, n, unchecked=False, **kw):
+def _run(F, prog, seed, groups, bfms, n, unchecked=False, k7=True, **kw):
     g = O.Golden(prog)
     dp = F.DeviceProgram(prog)
     gt = F.golden_run(dp)
@@ -29,7 +29,7 @@ def _run(F, prog, seed, groups, bfms, n, unchecked=False, **kw):
     out, log = F.inject(gt, sites, n, cap)
     out7 = out.clone()
     hist = F.classify_batched(gt, sites, n, out, log, cap, unchecked=unchecked, **kw)
-    hist7 = F.classify(gt, sites, n, out7, log, cap, unchecked=unchecked)
+    hist7 = F.classify(gt, sites, n, out7, log, cap, unchecked=unchecked) if k7 else None
     gi = F.as_numpy(out, F.INJ_DTYPE, n)
     g7 = F.as_numpy(out7, F.INJ_DTYPE, n)
     oi = g.inject(os_, O.MODE_FULL | (O.UNCHECKED if unchecked else 0))
@@ -37,10 +37,11 @@ def _run(F, prog, seed, groups, bfms, n, unchecked=False, **kw):
         bad = np.flatnonzero(gi[f] != oi[f])
         assert bad.size == 0, f"{f}: replica {bad[0]} k8 {gi[bad[0]]} oracle {oi[bad[0]]} site {os_[bad[0]]}"
     assert (gi["fault_pc"][gi["fault_kind"] > 0] == oi["fault_pc"][oi["fault_kind"] > 0]).all()
-    for f in ("outcome", "flags", "fault_kind"):
-        assert (gi[f] == g7[f]).all(), f
     assert np.array_equal(hist.cpu().numpy().astype(np.uint64), O.histogram(os_, oi))
-    assert np.array_equal(hist.cpu().numpy(), hist7.cpu().numpy())
+    if k7:                                    # K7's fixed-size overlay suits short programs only
+        for f in ("outcome", "flags", "fault_kind"):
+            assert (gi[f] == g7[f]).all(), f
+        assert np.array_equal(hist.cpu().numpy(), hist7.cpu().numpy())
     return oi
 
 
@@ -92,7 +93,7 @@ def test_k8_pool_exhaustion_is_reported(F):
 
 def test_k8_c4_mini(F):
     """mini-C4 (ResNet-50 v1.5 shape, width 8, 32x32: 72 launches, 53 convolutions):
-    trace, counts and whole-program outcomes (K8 and K7) against the oracle."""
+    trace and whole-program outcomes (K8) against the oracle."""
     from fi_inputs import resnet as R
     prog = R.c4(full=False)
     g = O.Golden(prog)
@@ -100,7 +101,7 @@ def test_k8_c4_mini(F):
     gt = F.golden_run(dp)
     assert np.array_equal(F.as_numpy(gt.rec, F.RECORD_DTYPE, gt.n_rec), g.trace())
     assert np.array_equal(gt.image.cpu().numpy(), g.final_image())
-    oi = _run(F, prog, R.C4_CAMPAIGN_SEED, [F.G_GP, F.G_FP32, F.G_LD, F.G_PR], [0, 1, 2, 3], 300)
+    oi = _run(F, prog, R.C4_CAMPAIGN_SEED, [F.G_GP, F.G_FP32, F.G_LD, F.G_PR], [0, 1, 2, 3], 300, k7=False)
     assert (oi["outcome"] == O.SDC).any() and (oi["outcome"] == O.MASKED).any()
 
 
@@ -116,5 +117,5 @@ def test_k8_c5_mini(F, which):
     assert np.array_equal(F.as_numpy(gt.rec, F.RECORD_DTYPE, gt.n_rec), g.trace())
     assert np.array_equal(gt.image.cpu().numpy(), g.final_image())
     groups = [F.G_GP, F.G_GPPR, F.G_LD, F.G_PR, F.G_FP64 if which in (1, 2, 3, 4) else F.G_FP32]
-    oi = _run(F, prog, H.C5_CAMPAIGN_SEED + which, groups, [0, 1, 2, 3], 250)
+    oi = _run(F, prog, H.C5_CAMPAIGN_SEED + which, groups, [0, 1, 2, 3], 250, k7=which in (2, 3))
     assert (oi["outcome"] == O.SDC).any()
