@@ -260,6 +260,11 @@ fi_status fi_inject(const fi_program* p, const uint8_t* image, const fi_trace* t
  * Replicas whose overlay or update lists overflow get outcome 0xFF + FI_E_CAPACITY. */
 #define FI_UNCHECKED 1u
 #define FI_POTENTIAL_DUE 1u
+/* K8 outcome 0xFF (not classified) reasons in fi_inj.flags: a capacity was
+ * exceeded (also FI_E_CAPACITY), or the replica loaded a corrupted word of a
+ * buffer whose pages were dropped after its last launch reference (wild load) */
+#define FI_UNCLASSIFIED_CAPACITY 2u
+#define FI_UNCLASSIFIED_WILD 4u
 size_t fi_classify_workspace(uint32_t n_inst, uint32_t n, uint32_t log_cap);
 fi_status fi_classify(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
                       uint32_t n, fi_inj* out, const fi_store* log, uint32_t log_cap, uint64_t* hist,

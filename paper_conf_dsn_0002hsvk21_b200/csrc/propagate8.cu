@@ -245,7 +245,7 @@ __global__ void k8_setup(K8Args A, const uint32_t* reps, uint32_t nb) {
         z.alive = 1;
         z.outcome = FI_MASKED;
         if (S.flags & FI_SITE_NOT_INJECTED) { z.alive = 0; z.outcome = FI_NOT_INJECTED; }
-        else if (R.overflow) { z.alive = 0; z.outcome = 0xFF; }
+        else if (R.overflow) { z.alive = 0; z.outcome = 0xFF; z.overflow = 1; }
         else if (R.fault_kind && !(unchecked && R.fault_kind != 3)) { z.alive = 0; z.outcome = FI_DUE; }
         else if (R.fault_kind) z.pdue = 1;
     }
@@ -557,7 +557,10 @@ __global__ void __launch_bounds__(256) k8_final(K8Args A) {
         }
         r.outcome = (uint8_t)outcome;
         r.flags = (pdue && outcome != FI_DUE && outcome != FI_NOT_INJECTED && outcome != 0xFF) ? FI_POTENTIAL_DUE : 0;
-        if (outcome == 0xFF) FI_DEV_ERR(A.status, FI_E_CAPACITY);
+        if (outcome == 0xFF) {
+            r.flags = (z.overflow ? FI_UNCLASSIFIED_CAPACITY : 0u) | (z.inexact ? FI_UNCLASSIFIED_WILD : 0u);
+            if (z.overflow) FI_DEV_ERR(A.status, FI_E_CAPACITY);
+        }
         else if (z.perm)                                             // opcode-weighted outcomes
             atomicAdd((unsigned long long*)&A.hist[outcome],
                       (unsigned long long)(A.opw ? A.opw[A.pf[z.rep].opcode & (FI_NOPS - 1)] : 1ull));

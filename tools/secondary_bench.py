@@ -48,14 +48,16 @@ def run(name, prog, seed, n, batch):
     (out, log), k4_ms = timed(lambda: fi.inject(gt, sites, n, cap))
     hist, k8_ms = timed(lambda: fi.classify_batched(gt, sites, n, out, log, cap, batch=batch))
     inj = fi.as_numpy(out, fi.INJ_DTYPE, n)
-    oc = np.bincount(inj["outcome"], minlength=4)
+    oc = np.bincount(np.minimum(inj["outcome"], 4), minlength=5)
     line = {"program": name, "instances": dp.n_inst, "static_kernels": len(prog.kernels), "warps": dp.n_warps,
             "records": gt.n_rec, "counted_thread_instrs": counted, "golden_s": golden_s,
             "profile_ms": prof_ms, "profile_thread_instrs_per_s": counted / (prof_ms / 1e3),
             "profile_hbm_gbs": algo / (prof_ms / 1e3) / 1e9, "index_ms": idx_ms, "select_ms": sel_ms,
             "replicas": n, "k4_ms": k4_ms, "k8_ms": k8_ms,
             "injections_per_s": n / ((sel_ms + k4_ms + k8_ms) / 1e3),
-            "outcomes": {"masked": int(oc[0]), "sdc": int(oc[1]), "due": int(oc[2])},
+            "outcomes": {"masked": int(oc[0]), "sdc": int(oc[1]), "due": int(oc[2]),
+                         "unclassified_wild_load": int(((inj["outcome"] == 0xFF) & (inj["flags"] & 4 > 0)).sum()),
+                         "unclassified_capacity": int(((inj["outcome"] == 0xFF) & (inj["flags"] & 2 > 0)).sum())},
             "group": "G_GP", "bfm": "FLIP_SINGLE_BIT"}
     print(json.dumps(line), flush=True)
     del gt, dp
@@ -65,7 +67,7 @@ def run(name, prog, seed, n, batch):
 def main():
     cfg = sys.argv[1] if len(sys.argv) > 1 else "C3"
     n = int(sys.argv[2]) if len(sys.argv) > 2 else 200
-    batch = int(sys.argv[3]) if len(sys.argv) > 3 else 512
+    batch = int(sys.argv[3]) if len(sys.argv) > 3 else None          # None: sized to the memory budget
     if cfg == "C3":
         run("C3 CG 512x256, 500 iterations", P.c3(full=True), P.CAMPAIGN_SEED[3], n, batch)
     elif cfg == "C4":
