@@ -49,6 +49,8 @@ def parse():
     ap.add_argument("--impl", default="fi", choices=["fi", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-secondary", action="store_true",
+                    help="skip the C4 (ResNet-50-shaped, 72 launches) multi-launch campaign sample")
     return ap.parse_args()
 
 
@@ -311,12 +313,51 @@ def main():
 
     if not args.no_e2e:
         line["e2e"] = e2e(args, prog, seed, groups, bfms, n, rank, world, dev, camp)
+    if rank == 0 and world == 1 and not args.no_secondary:
+        line["secondary"] = secondary_c4(dev)
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(prog, camp.sites_np())
     if rank == 0:
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
+
+
+def secondary_c4(dev, n=256):
+    """BASELINE configs[3]'s program (ResNet-50 v1.5 inference shape, 72 launches)
+    on one GPU: golden run, exact profile, select, K4, K8 whole-program outcomes
+    for a bounded replica sample (the 100 k campaign shards these over ranks).
+    CUDA events on the launching stream; not part of `value`."""
+    import torch
+    from fi_inputs import resnet as R
+    from paper_conf_dsn_0002hsvk21_b200 import fi
+    prog = R.c4(full=True)
+    dp = fi.DeviceProgram(prog, dev)
+    gt = fi.golden_run(dp)
+    ev = [torch.cuda.Event(enable_timing=True) for _ in range(5)]
+    torch.cuda.synchronize()
+    ev[0].record()
+    ic, cc = fi.profile(gt)
+    ev[1].record()
+    idx = fi.SiteIndex(gt, ic, cc)
+    sites = fi.select_sites(idx, fi.schedule(R.C4_CAMPAIGN_SEED, [fi.G_GP], [0]), 0, n)
+    ev[2].record()
+    cap = fi.log_capacity(gt)
+    out, log = fi.inject(gt, sites, n, cap)
+    ev[3].record()
+    hist = fi.classify_batched(gt, sites, n, out, log, cap)
+    ev[4].record()
+    torch.cuda.synchronize()
+    ms = [ev[i].elapsed_time(ev[i + 1]) for i in range(4)]
+    counts = ic.cpu().numpy()
+    counted = int(counts[:, 4].sum() + counts[:, 6].sum())
+    h = hist.cpu().numpy()
+    return {"workload": "C4 ResNet-50 v1.5 inference, 224x224, batch 1: 72 launches, 265,696 warps; "
+                        f"{n} replicas G_GP FLIP_SINGLE_BIT, whole-program outcomes (K8)",
+            "records": gt.n_rec, "profile_thread_instrs_per_s": counted / (ms[0] / 1e3),
+            "injections_per_s": n / ((ms[1] + ms[2] + ms[3]) / 1e3),
+            "ms": {"profile": ms[0], "index_select": ms[1], "inject_k4": ms[2], "propagate_classify_k8": ms[3]},
+            "outcomes": {"masked": int(h[..., 0].sum()), "sdc": int(h[..., 1].sum()), "due": int(h[..., 2].sum())}}
 
 
 def e2e(args, prog, seed, groups, bfms, n, rank, world, dev, camp):
