@@ -34,7 +34,8 @@ typedef enum {
     FI_E_CUDA = 5,
     FI_E_SITE = 6,             /* a site does not match the re-executed warp */
     FI_E_CAPACITY = 8,         /* faulty store log overflow (replica must be re-run with a larger log) */
-    FI_E_INVARIANT = 9         /* a Table II identity does not hold for a count row (§8 row a3) */
+    FI_E_INVARIANT = 9,        /* a Table II identity does not hold for a count row (§8 row a3) */
+    FI_E_COLLECTIVE = 10       /* fi_campaign: the caller's all-reduce callback failed */
 } fi_status;
 
 /* Table II arch state ids [PAPER.md:94-104], 0-based (C-1) */
@@ -341,6 +342,90 @@ fi_status fi_inject_permanent_batched(const fi_program* p, const uint8_t* image,
  * instruction count, destination register value, bit-pattern value (the two
  * [0,1) values printed as u/2^32 with 10 digits).  Host only. */
 fi_status fi_write_params_txt(const fi_site* site_host, const char* kernel_name, char* buf, size_t buf_bytes);
+
+/* The profile file of PAPER.md:78 ("a profile containing one line for every
+ * dynamic kernel"): one line per dynamic kernel instance k, in launch order,
+ *   <kernel_name>; kernel_count: <c>; <G_FP64> <G_FP32> <G_LD> <G_PR> <G_NODEST> <G_OTHERS> <G_GPPR> <G_GP>
+ * with the eight Table II counts of inst_counts_host[k][0..7] (u64, host).
+ * kernel_names[n_kern] (host) names the static kernels; inst_host[n_inst] gives
+ * each instance's static kernel and kernel_count.  Writes at most buf_bytes
+ * (NUL-terminated); *needed (if not NULL) receives the full length + 1, so a
+ * call with buf = NULL, buf_bytes = 0 sizes the buffer.  FI_E_ARG if it does
+ * not fit.  Host only. */
+fi_status fi_write_profile_txt(const uint64_t* inst_counts_host, const fi_instance* inst_host, uint32_t n_inst,
+                               const char* const* kernel_names, uint32_t n_kern, char* buf, size_t buf_bytes,
+                               size_t* needed);
+
+/* ---- fi_campaign: the whole campaign of one rank, host buffers in and out ----
+ * PAPER.md:72 Fig. 1 steps (1)-(4) end to end, as the driver of SURVEY §8(e):
+ * H2D of the program (from HOST arrays), golden run (passes 1 + 2, golden
+ * checkpoints), K1 profile of this rank's chunk-aligned record shard
+ * [chunk r*C/G, (r+1)*C/G), all-reduce(SUM) of inst_counts (u64) and
+ * chunk_counts (u32) through `allreduce`, K2 index (+ a3 identities), K3 select
+ * / K4 inject / K5|K7|K8 classify of this rank's replica block
+ * [r*n/G, (r+1)*n/G) (replica RNG keyed by the global index j, so results do
+ * not depend on G), all-reduce(SUM) of the u64 histogram, D2H of the results.
+ * With cfg->approximate the profile is PAPER.md:80's approximate one
+ * (fi_profile_approx, first instance per static kernel; no record sharding,
+ * no count all-reduce) and sites come from fi_select_sites_approx (C-17).
+ *
+ * allreduce(dev, count, elem_bytes, ctx, stream): in-place SUM over the ranks of
+ * `count` integers of elem_bytes (4 or 8) at device pointer dev, ordered on
+ * `stream`; returns 0 on success.  May be NULL when world == 1.  Typically
+ * torch.distributed all_reduce on NCCL (paper_conf_dsn_0002hsvk21_b200.fi.campaign).
+ *
+ * Memory: unlike the other calls, fi_campaign allocates its device memory itself
+ * (cudaMalloc on cfg->device, all freed before it returns) and SYNCHRONIZES.
+ * Host arrays in cfg are read only; result arrays marked optional may be NULL.
+ * Errors: FI_E_ARG (bad cfg), FI_E_PROGRAM / FI_E_INVARIANT / FI_E_SITE /
+ * FI_E_CAPACITY from device status, FI_E_EMPTY_GROUP / FI_E_NOT_INJECTABLE from
+ * selection, FI_E_CUDA, FI_E_COLLECTIVE when allreduce returns non-zero. */
+typedef int (*fi_allreduce_fn)(void* dev, uint64_t count, uint32_t elem_bytes, void* ctx, void* stream);
+#define FI_PROPAGATION_AUTO 0u      /* K8 from 64 launches on, else K5/K7 (fi_classify) */
+#define FI_PROPAGATION_K7 1u        /* fi_classify */
+#define FI_PROPAGATION_K8 2u        /* fi_classify_batched */
+#define FI_CKPT_AUTO 0xFFFFFFFFu    /* 4096 steps, doubled until the checkpoints fit 20% of free HBM */
+typedef struct {
+    /* the program, HOST arrays */
+    const fi_insn* code;         uint32_t n_code;
+    const fi_kernel* kern;       uint32_t n_kern;
+    const fi_instance* inst;     uint32_t n_inst;
+    const uint32_t* cbank;       uint32_t n_cbank;
+    const fi_buffer* buf;        uint32_t n_buf;
+    const uint8_t* init_image;   uint64_t image_bytes;
+    uint32_t n_warps;
+    /* the campaign */
+    fi_schedule sched;           /* seed + per-replica group / bit-flip model */
+    uint64_t n_replicas;         /* whole campaign, all ranks */
+    uint32_t flags;              /* FI_UNCHECKED (row f4) */
+    uint32_t propagation;        /* FI_PROPAGATION_* */
+    uint32_t approximate;        /* 1 = approximate profile (row f1) */
+    uint32_t ckpt_interval;      /* steps between golden checkpoints, 0 = none, FI_CKPT_AUTO */
+    uint64_t k8_mem_budget;      /* device bytes for K8 scratch (0 = 24 GiB) */
+    int device;                  /* CUDA device ordinal (< 0 = current) */
+    void* stream;                /* cudaStream_t (NULL = a stream fi_campaign creates) */
+} fi_campaign_cfg;
+
+typedef struct {
+    uint64_t hist[8][4][3];      /* [group][bfm][Masked, SDC, DUE], summed over all ranks */
+    uint64_t totals[8];          /* N_g over the whole trace (exact or approximate) */
+    uint64_t n_rec;              /* trace records (warp-instructions) */
+    uint64_t counted;            /* thread-level dynamic instructions counted (NODEST + GPPR) */
+    uint64_t j0, n_local;        /* this rank's replica block */
+    uint64_t rec_begin, rec_end; /* this rank's profile shard */
+    uint64_t n_unclassified;     /* replicas with outcome 0xFF (capacity), this rank */
+    uint64_t n_not_injected;     /* approximate sites that do not exist (C-17), this rank */
+    /* CUDA-event times on the stream, ms: H2D + prepare, golden run, profile,
+     * count exchange, index, select, inject, classify + histogram exchange, D2H */
+    float ms_h2d, ms_golden, ms_profile, ms_exchange, ms_index, ms_select, ms_inject, ms_classify, ms_d2h;
+    /* optional host outputs (NULL = not returned) */
+    fi_site* sites;              /* [n_local] */
+    fi_inj* inj;                 /* [n_local] */
+    uint64_t* inst_counts;       /* [n_inst][8] (after the exchange) */
+} fi_campaign_result;
+
+fi_status fi_campaign(const fi_campaign_cfg* cfg, int rank, int world, fi_allreduce_fn allreduce, void* ctx,
+                      fi_campaign_result* res);
 
 #ifdef __cplusplus
 }

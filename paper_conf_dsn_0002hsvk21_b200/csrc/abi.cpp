@@ -29,6 +29,7 @@ extern "C" const char* fi_status_str(fi_status s) {
         case FI_E_SITE: return "site does not match the re-executed warp / trace";
         case FI_E_CAPACITY: return "faulty store log overflow";
         case FI_E_INVARIANT: return "Table II identity violated by a count row (GP = FP64+FP32+LD+OTHERS, GPPR = GP+PR)";
+        case FI_E_COLLECTIVE: return "all-reduce callback failed";
     }
     return "unknown status";
 }

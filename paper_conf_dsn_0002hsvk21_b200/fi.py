@@ -75,6 +75,37 @@ class fi_schedule(C.Structure):
                 ("groups", C.c_uint8 * 8), ("bfms", C.c_uint8 * 4)]
 
 
+class fi_campaign_cfg(C.Structure):
+    _fields_ = [("code", C.c_void_p), ("n_code", C.c_uint32),
+                ("kern", C.c_void_p), ("n_kern", C.c_uint32),
+                ("inst", C.c_void_p), ("n_inst", C.c_uint32),
+                ("cbank", C.c_void_p), ("n_cbank", C.c_uint32),
+                ("buf", C.c_void_p), ("n_buf", C.c_uint32),
+                ("init_image", C.c_void_p), ("image_bytes", C.c_uint64),
+                ("n_warps", C.c_uint32),
+                ("sched", fi_schedule),
+                ("n_replicas", C.c_uint64),
+                ("flags", C.c_uint32), ("propagation", C.c_uint32), ("approximate", C.c_uint32),
+                ("ckpt_interval", C.c_uint32), ("k8_mem_budget", C.c_uint64),
+                ("device", C.c_int), ("stream", C.c_void_p)]
+
+
+class fi_campaign_result(C.Structure):
+    _fields_ = [("hist", C.c_uint64 * 96), ("totals", C.c_uint64 * 8),
+                ("n_rec", C.c_uint64), ("counted", C.c_uint64), ("j0", C.c_uint64), ("n_local", C.c_uint64),
+                ("rec_begin", C.c_uint64), ("rec_end", C.c_uint64),
+                ("n_unclassified", C.c_uint64), ("n_not_injected", C.c_uint64),
+                ("ms_h2d", C.c_float), ("ms_golden", C.c_float), ("ms_profile", C.c_float),
+                ("ms_exchange", C.c_float), ("ms_index", C.c_float), ("ms_select", C.c_float),
+                ("ms_inject", C.c_float), ("ms_classify", C.c_float), ("ms_d2h", C.c_float),
+                ("sites", C.c_void_p), ("inj", C.c_void_p), ("inst_counts", C.c_void_p)]
+
+
+# int allreduce(void* dev, uint64_t count, uint32_t elem_bytes, void* ctx, void* stream)
+ALLREDUCE_FN = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_uint64, C.c_uint32, C.c_void_p, C.c_void_p)
+FI_PROPAGATION = {"auto": 0, "k7": 1, "k8": 2}
+FI_CKPT_AUTO = 0xFFFFFFFF
+
 _lib = None
 
 
@@ -121,6 +152,9 @@ def lib():
                                                  vp, vp]),
             "fi_classify_batched": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, u32, u32, u32, u32, vp, sz, vp, vp]),
             "fi_inject_permanent": (st, [vp, vp, vp, vp, u32, vp, vp, vp, u32, u32, vp, u32, vp, sz, vp, vp]),
+            "fi_write_profile_txt": (st, [vp, vp, u32, vp, u32, vp, sz, C.POINTER(C.c_size_t)]),
+            "fi_campaign": (st, [C.POINTER(fi_campaign_cfg), C.c_int, C.c_int, ALLREDUCE_FN, vp,
+                                 C.POINTER(fi_campaign_result)]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -542,6 +576,122 @@ def write_params_txt(site_row: np.ndarray, kernel_name: str) -> str:
     buf = C.create_string_buffer(1024)
     _check(lib().fi_write_params_txt(a.ctypes.data, kernel_name.encode(), buf, 1024), "fi_write_params_txt")
     return buf.value.decode()
+
+
+def write_profile_txt(inst_counts: np.ndarray, prog) -> str:
+    """fi_write_profile_txt: PAPER.md:78's profile, one line per dynamic kernel."""
+    ic = np.ascontiguousarray(inst_counts, dtype=np.uint64)
+    inst = np.ascontiguousarray(prog.instances)
+    names = [n.encode() for n in prog.kernel_names]
+    arr = (C.c_char_p * max(len(names), 1))(*names)
+    need = C.c_size_t(0)
+    _check(lib().fi_write_profile_txt(ic.ctypes.data, inst.ctypes.data, len(inst), arr, len(names), None, 0,
+                                      C.byref(need)), "fi_write_profile_txt")
+    buf = C.create_string_buffer(need.value)
+    _check(lib().fi_write_profile_txt(ic.ctypes.data, inst.ctypes.data, len(inst), arr, len(names), buf, need.value,
+                                      None), "fi_write_profile_txt")
+    return buf.value.decode()
+
+
+class _DevArray:
+    """A device pointer seen through __cuda_array_interface__ (zero-copy into torch)."""
+
+    def __init__(self, ptr: int, n: int, typestr: str):
+        self.__cuda_array_interface__ = {"shape": (n,), "typestr": typestr, "data": (ptr, False), "version": 3,
+                                         "strides": None, "stream": None}
+
+
+def device_view(ptr: int, n: int, elem_bytes: int, device) -> torch.Tensor:
+    return torch.as_tensor(_DevArray(ptr, n, "<i8" if elem_bytes == 8 else "<i4"), device=device)
+
+
+def torch_allreduce(group=None):
+    """An fi_allreduce_fn over torch.distributed (NCCL on the GPU box): in-place
+    SUM of the device integers, ordered on fi_campaign's stream."""
+    import torch.distributed as dist
+
+    def cb(dev, count, elem_bytes, ctx, stream):
+        try:
+            d = torch.device("cuda", torch.cuda.current_device())
+            t = device_view(dev, count, elem_bytes, d)
+            with torch.cuda.stream(torch.cuda.ExternalStream(stream, device=d)):
+                dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
+            return 0
+        except Exception as e:                          # never raise across the C ABI
+            import sys
+            print(f"fi allreduce callback failed: {e!r}", file=sys.stderr)
+            return 1
+    return ALLREDUCE_FN(cb)
+
+
+@dataclass
+class CampaignResult:
+    hist: np.ndarray             # [8][4][3] u64, all ranks
+    totals: list
+    n_rec: int
+    counted: int
+    j0: int
+    n_local: int
+    rec_range: tuple
+    n_unclassified: int
+    n_not_injected: int
+    ms: dict
+    sites: np.ndarray | None
+    inj: np.ndarray | None
+    inst_counts: np.ndarray | None
+
+
+def campaign(prog, seed: int, groups, bfms, n_replicas: int, rank: int = 0, world: int = 1, allreduce=None,
+             unchecked: bool = False, propagation: str = "auto", approximate: bool = False, ckpt="auto",
+             k8_mem_budget: int = 0, device: int | None = None, host: dict | None = None,
+             return_arrays: bool = True) -> CampaignResult:
+    """fi_campaign: the whole campaign of this rank from HOST arrays (golden run,
+    sharded profile, count exchange, index, select, inject, classify, histogram
+    exchange, D2H).  `host`: optional pinned uint8 tensors keyed code / kernels /
+    instances / cbank / buffers / init_image (else the numpy arrays are used).
+    allreduce: an ALLREDUCE_FN (torch_allreduce() by default when world > 1)."""
+    arrs = {k: np.ascontiguousarray(getattr(prog, k)) for k in
+            ("code", "kernels", "instances", "cbank", "buffers", "init_image")}
+
+    def hp(k):
+        if host is not None and host[k].numel():
+            return host[k].data_ptr()
+        return arrs[k].ctypes.data if arrs[k].size else None
+    cfg = fi_campaign_cfg()
+    cfg.code, cfg.n_code = hp("code"), len(arrs["code"])
+    cfg.kern, cfg.n_kern = hp("kernels"), len(arrs["kernels"])
+    cfg.inst, cfg.n_inst = hp("instances"), len(arrs["instances"])
+    cfg.cbank, cfg.n_cbank = hp("cbank"), len(arrs["cbank"])
+    cfg.buf, cfg.n_buf = hp("buffers"), len(arrs["buffers"])
+    cfg.init_image, cfg.image_bytes = hp("init_image"), prog.image_bytes
+    cfg.n_warps = prog.n_warps
+    cfg.sched = schedule(seed, groups, bfms)
+    cfg.n_replicas = n_replicas
+    cfg.flags = FI_UNCHECKED if unchecked else 0
+    cfg.propagation = FI_PROPAGATION[propagation]
+    cfg.approximate = 1 if approximate else 0
+    cfg.ckpt_interval = FI_CKPT_AUTO if ckpt == "auto" else int(ckpt)
+    cfg.k8_mem_budget = k8_mem_budget
+    cfg.device = torch.cuda.current_device() if device is None else device
+    cfg.stream = torch.cuda.current_stream(cfg.device).cuda_stream or None
+    n_loc = n_replicas * (rank + 1) // world - n_replicas * rank // world
+    res = fi_campaign_result()
+    sites = inj = ic = None
+    if return_arrays:
+        sites = np.zeros(max(n_loc, 1), dtype=SITE_DTYPE)
+        inj = np.zeros(max(n_loc, 1), dtype=INJ_DTYPE)
+        ic = np.zeros((max(len(prog.instances), 1), 8), dtype=np.uint64)
+        res.sites, res.inj, res.inst_counts = sites.ctypes.data, inj.ctypes.data, ic.ctypes.data
+    if world > 1 and allreduce is None:
+        allreduce = torch_allreduce()
+    cb = allreduce if allreduce is not None else ALLREDUCE_FN()
+    _check(lib().fi_campaign(C.byref(cfg), rank, world, cb, None, C.byref(res)), "fi_campaign")
+    ms = {k: float(getattr(res, "ms_" + k)) for k in
+          ("h2d", "golden", "profile", "exchange", "index", "select", "inject", "classify", "d2h")}
+    return CampaignResult(np.array(res.hist, dtype=np.uint64).reshape(8, 4, 3), [int(x) for x in res.totals],
+                          int(res.n_rec), int(res.counted), int(res.j0), int(res.n_local),
+                          (int(res.rec_begin), int(res.rec_end)), int(res.n_unclassified), int(res.n_not_injected),
+                          ms, None if sites is None else sites[:n_loc], None if inj is None else inj[:n_loc], ic)
 
 
 def as_numpy(t: torch.Tensor, dtype: np.dtype, n: int | None = None) -> np.ndarray:

@@ -65,3 +65,31 @@ def test_header_constants_match_input_format():
         listed = ("NOP, " + m.group(1) + " " + m.group(2) + " " + m.group(3)).replace("\n", " ")
         got = [x.strip() for x in listed.split(",") if x.strip()]
         assert got[:len(names)] == names, path
+
+
+def test_profile_txt_one_line_per_dynamic_kernel():
+    """the profile has one line per dynamic kernel (name, kernel
+    count, the eight Table II counts in order)."""
+    from paper_conf_dsn_0002hsvk21_b200 import fi
+    prog = P.multi_instance_chain(5)
+    ic = (np.arange(5 * 8, dtype=np.uint64).reshape(5, 8) * np.uint64(1 << 33))
+    txt = fi.write_profile_txt(ic, prog).splitlines()
+    assert len(txt) == 5
+    for k, line in enumerate(txt):
+        name, kc, counts = line.split("; ")
+        inst = prog.instances[k]
+        assert name == prog.kernel_names[inst["kernel"]]
+        assert kc == f"kernel_count: {inst['kernel_count']}"
+        assert [int(x) for x in counts.split()] == [int(x) for x in ic[k]]
+
+
+def test_campaign_argument_errors_without_gpu():
+    """fi_campaign validates its host arguments before touching the device."""
+    from paper_conf_dsn_0002hsvk21_b200 import fi
+    res = fi.fi_campaign_result()
+    cfg = fi.fi_campaign_cfg()
+    L = fi.lib()
+    assert L.fi_campaign(None, 0, 1, fi.ALLREDUCE_FN(), None, C.byref(res)) == fi.FI_E_ARG
+    assert L.fi_campaign(C.byref(cfg), 0, 1, fi.ALLREDUCE_FN(), None, C.byref(res)) == fi.FI_E_ARG   # empty program
+    assert L.fi_campaign(C.byref(cfg), 2, 2, fi.ALLREDUCE_FN(), None, C.byref(res)) == fi.FI_E_ARG   # rank >= world
+    assert L.fi_campaign(C.byref(cfg), 0, 2, fi.ALLREDUCE_FN(), None, C.byref(res)) == fi.FI_E_ARG   # no callback
