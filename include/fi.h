@@ -337,6 +337,33 @@ fi_status fi_inject_permanent_batched(const fi_program* p, const uint8_t* image,
                                       uint32_t pool_pages, uint32_t pend_cap, void* ws, size_t ws_bytes,
                                       uint32_t* dev_status, void* stream);
 
+/* ---- JIT-specialised emulator (K4 on per-program generated code) --------
+ * fi_jit_build generates CUDA source from the program's code (p->code_host and
+ * the HOST kernel table kern_host[p->n_kern]) — every static instruction
+ * becomes straight-line device code with the synthetic registers in hardware
+ * registers — compiles it with NVRTC for sm_100a (libnvrtc.so.12, loaded at
+ * run time) and loads it into the current device's primary context.  The
+ * semantics are DESIGN.md §3, identical to the interpreter behind fi_inject.
+ * Synchronous; FI_E_PROGRAM if NVRTC rejects the source (fi_jit_log() has the
+ * log), FI_E_CUDA if NVRTC / the driver is unavailable.  Free with fi_jit_free.
+ * fi_jit_compile_check compiles without loading (no GPU needed); fi_jit_source
+ * returns the generated source (buf may be NULL; returns the bytes needed, 0 on
+ * bad arguments). */
+typedef struct fi_jit fi_jit;
+fi_status fi_jit_build(const fi_program* p, const fi_kernel* kern_host, fi_jit** out);
+void fi_jit_free(fi_jit* j);
+double fi_jit_compile_seconds(const fi_jit* j);
+const char* fi_jit_log(void);
+fi_status fi_jit_compile_check(const fi_insn* code_host, uint32_t n_code, const fi_kernel* kern_host, uint32_t n_kern,
+                               uint32_t n_regs, size_t* cubin_bytes);
+size_t fi_jit_source(const fi_insn* code_host, uint32_t n_code, const fi_kernel* kern_host, uint32_t n_kern,
+                     uint32_t n_regs, char* buf, size_t buf_bytes);
+/* K4 on the JIT module `j` built for p: same arguments, scratch, scheduling and
+ * results as fi_inject (bit-identical outputs), asynchronous on `stream`. */
+fi_status fi_inject_jit(const fi_jit* j, const fi_program* p, const uint8_t* image, const fi_trace* t,
+                        const fi_site* sites, uint32_t n, fi_inj* out, fi_store* log, uint32_t log_cap, void* ws,
+                        size_t ws_bytes, uint32_t* dev_status, void* stream);
+
 /* Table II parameter file, one parameter per line in Table II order
  * [PAPER.md:88]: arch state id, bit-flip model, kernel name, kernel count,
  * instruction count, destination register value, bit-pattern value (the two

@@ -17,8 +17,8 @@ ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2", "--expt-relaxed-constexpr",
          "-Xptxas", "-v,-warn-spills"] + ARCH
 SOURCES = ["abi.cpp", "golden.cu", "scan.cu", "profile.cu", "select.cu", "inject.cu", "propagate.cu", "propagate8.cu",
-           "campaign.cpp"]
-HEADERS = ["common.cuh", "emu.cuh", "scan.cuh"]
+           "campaign.cpp", "jit.cpp"]
+HEADERS = ["common.cuh", "emu.cuh", "scan.cuh", "jit_prelude.cuh"]
 
 
 def _stale(obj: str, deps: list[str]) -> bool:
@@ -29,13 +29,19 @@ def build(force: bool = False, verbose: bool = False) -> str:
     objdir = os.path.join(HERE, "_obj")
     os.makedirs(objdir, exist_ok=True)
     hdrs = [os.path.join(CSRC, h) for h in HEADERS] + [os.path.join(ROOT, "include", "fi.h")]
+    # the JIT prelude is embedded into libfi.so as a string (NVRTC compiles it per program)
+    inc = os.path.join(objdir, "jit_prelude.inc")
+    pre = os.path.join(CSRC, "jit_prelude.cuh")
+    if force or _stale(inc, [pre]):
+        with open(pre) as f, open(inc, "w") as g:
+            g.write('R"FIJITPRELUDE(' + f.read() + ')FIJITPRELUDE"\n')
     objs = []
     for src in SOURCES:
         s = os.path.join(CSRC, src)
         o = os.path.join(objdir, src + ".o")
         objs.append(o)
         if force or _stale(o, [s] + hdrs):
-            cmd = [NVCC, *FLAGS, "-c", s, "-o", o]
+            cmd = [NVCC, *FLAGS, "-I", objdir, "-c", s, "-o", o]
             r = subprocess.run(cmd, capture_output=True, text=True)
             if r.returncode:
                 sys.stderr.write(r.stdout + r.stderr)

@@ -222,6 +222,11 @@ __global__ void __launch_bounds__(kClsWarps * 32) k_classify(const ClsArgs A) {
 }
 
 }  // namespace
+
+void launch_lpt_order(const fi_site* sites, const uint64_t* warp_off, uint32_t ck_interval, uint32_t n,
+                      uint32_t* order, uint32_t* counter, cudaStream_t s) {
+    k_lpt_order<<<1, 1024, 0, s>>>(sites, warp_off, ck_interval, n, order, counter);
+}
 }  // namespace fi
 
 using namespace fi;

@@ -1,0 +1,784 @@
+// jit.cpp — the JIT-specialised emulator: per-program CUDA generated from the
+// mini-SASS code and compiled by NVRTC for sm_100a (fi_jit_build), and K4 on it
+// (fi_inject_jit).
+//
+// Why: the interpreter (emu.cuh) keeps the synthetic register file in shared
+// memory and decodes every emulated instruction, ~26 SASS per emulated step on
+// C2.  Here every static instruction becomes straight-line device code with the
+// synthetic registers in real registers (R0..R{n_regs-1} are C++ locals with
+// constant indices), so an FFMA is one predicated FFMA.  Semantics are those of
+// DESIGN.md §3 and identical to emu.cuh's EMU_INJ mode step for step:
+//   * min-pc scheduling with the same group-mode rule (a group of lanes sharing
+//     pc runs alone until it branches divergently, exits or reaches parked lanes);
+//   * a "block" (from any pc to the next BRA/EXIT or the end of the kernel code)
+//     runs without per-step bookkeeping when it cannot reach parked lanes, the
+//     watchdog or the injection site; otherwise instructions run one step at a
+//     time through the same generated bodies (`S_i` labels);
+//   * the site's corruption, store logging after the site, memory faults
+//     (first faulting instruction in program order, C-9), watchdog (C-10), and
+//     the restart from the golden checkpoint at or before the site.
+// All generated control flow is warp-uniform (switch on the warp's pc, ballots);
+// per-lane effects are predicated, so SHFL sees every lane's register.
+#include <dlfcn.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include "../../include/fi.h"
+#include "common.cuh"
+
+namespace {
+
+const char* const kPrelude =
+#include "jit_prelude.inc"
+    ;
+
+// ---------------------------------------------------------------- generator
+struct Src {
+    std::string s;
+    void operator()(const char* fmt, ...) __attribute__((format(printf, 2, 3))) {
+        char buf[4096];
+        va_list ap;
+        va_start(ap, fmt);
+        int n = std::vsnprintf(buf, sizeof buf, fmt, ap);
+        va_end(ap);
+        if (n > 0) s.append(buf, std::min<size_t>((size_t)n, sizeof buf - 1));
+    }
+};
+
+struct Gen {
+    uint32_t NR;                                      // register rows (fi_program.n_regs)
+    std::string R(uint32_t j) const { return j < NR ? "R" + std::to_string(j) : std::string("0u"); }
+    std::string R64(uint32_t j) const { return "jpair(" + R(j) + ", " + R(j + 1) + ")"; }
+    bool W(uint32_t j) const { return j < NR; }
+    static std::string guard(uint32_t g) {
+        if (g == 7) return "true";
+        const uint32_t gs = g & 7, neg = (g >> 3) & 1;
+        if (gs == 7) return neg ? "false" : "true";
+        char b[96];
+        std::snprintf(b, sizeof b, "((((preds >> %uu) & 1u) ^ %uu) != 0u)", gs, neg);
+        return b;
+    }
+    std::string bv(const fi_insn& I) const {
+        if (I.mod & 0x80) {
+            char b[32];
+            std::snprintf(b, sizeof b, "0x%08Xu", I.imm);
+            return b;
+        }
+        return R(I.b);
+    }
+    static std::string hex(uint32_t v) {
+        char b[32];
+        std::snprintf(b, sizeof b, "0x%08Xu", v);
+        return b;
+    }
+    // writes of n consecutive registers from d0 under `ex` (values v0..)
+    void wr(Src& o, uint32_t d0, const char* const* vals, uint32_t n) const {
+        if (d0 == fi::kRZ) return;
+        for (uint32_t q = 0; q < n; ++q)
+            if (W(d0 + q)) o("if (ex) R%u = %s; ", d0 + q, vals[q]);
+    }
+
+    // a plain instruction (emu.cuh exec_plain): `ex` is declared
+    void plain(Src& o, const fi_insn& I) const {
+        using namespace fi;
+        const uint32_t op = I.op, mod = I.mod;
+        const std::string a = R(I.a), c = R(I.c), b = bv(I);
+        switch (op) {
+            case FFMA: {
+                // sm_100 FFMA returns the canonical 0x7FFFFFFF for every NaN (C-13 as is;
+                // emu.cuh's batched FFMA path relies on the same, pinned by parity tests)
+                o("{ const float x = ju2f(%s ^ %s), y = ju2f(%s ^ %s), z = ju2f(%s ^ %s); "
+                  "const u32 v = __float_as_uint(__fmaf_rn(x, y, z)); ",
+                  a.c_str(), hex((mod & 1u) << 31).c_str(), b.c_str(), hex((mod & 2u) << 30).c_str(), c.c_str(),
+                  hex((mod & 4u) << 29).c_str());
+                const char* v[] = {"v"};
+                wr(o, I.d0, v, 1);
+                o("}\n");
+                return;
+            }
+            case MOV: { o("{ const u32 v = %s; ", b.c_str()); const char* v[] = {"v"}; wr(o, I.d0, v, 1); o("}\n"); return; }
+            case S2R: {
+                const char* e = "0u";
+                switch (I.imm) {
+                    case 0: e = "wic * 32u + lane"; break;
+                    case 1: e = "cta"; break;
+                    case 2: e = "in.block"; break;
+                    case 3: e = "in.grid"; break;
+                    case 4: e = "lane"; break;
+                    case 5: e = "wic"; break;
+                }
+                const char* v[] = {e};
+                o("{ ");
+                wr(o, I.d0, v, 1);
+                o("}\n");
+                return;
+            }
+            case IADD3: {
+                const uint32_t pb = I.d1 & 7;
+                o("{ const u32 a_ = %s, c_ = %s, b_ = %s; const u32 x = %s, y = %s; const u64 s_ = (u64)x + y + c_; "
+                  "const u32 v = (u32)s_; ",
+                  a.c_str(), c.c_str(), b.c_str(), (mod & 1) ? "0u - a_" : "a_", (mod & 2) ? "0u - b_" : "b_");
+                const char* v[] = {"v"};
+                wr(o, I.d0, v, 1);
+                if (pb != 7) o("if (ex) preds = (preds & ~(1u << %uu)) | ((u32)((s_ >> 32) != 0ull) << %uu); ", pb, pb);
+                o("}\n");
+                return;
+            }
+            case IMAD: {
+                o("{ const u32 v = %s * %s + %s; ", a.c_str(), b.c_str(), c.c_str());
+                const char* v[] = {"v"};
+                wr(o, I.d0, v, 1);
+                o("}\n");
+                return;
+            }
+            case IMAD_WIDE: {
+                o("{ const u32 a_ = %s, b_ = %s; const u64 p_ = %s; const u64 r_ = p_ + %s; "
+                  "const u32 v0 = (u32)r_, v1 = (u32)(r_ >> 32); ",
+                  a.c_str(), b.c_str(),
+                  (mod & 1) ? "(u64)a_ * (u64)b_" : "(u64)((i64)(i32)a_ * (i64)(i32)b_)", R64(I.c).c_str());
+                const char* v[] = {"v0", "v1"};
+                wr(o, I.d0, v, 2);
+                o("}\n");
+                return;
+            }
+            case SHF: {
+                o("{ const u32 v = jshf(%s, %s, %uu); ", a.c_str(), b.c_str(), mod & 3u);
+                const char* v[] = {"v"};
+                wr(o, I.d0, v, 1);
+                o("}\n");
+                return;
+            }
+            case LOP3: {
+                o("{ const u32 v = jlop3<%uu>(%s, %s, %s); ", I.ext & 0xFFu, a.c_str(), b.c_str(), c.c_str());
+                const char* v[] = {"v"};
+                wr(o, I.d0, v, 1);
+                o("}\n");
+                return;
+            }
+            case SEL: {
+                const uint32_t pb = I.c & 0xF, p = pb & 7;
+                std::string cond = p == 7 ? "1u" : ("((preds >> " + std::to_string(p) + "u) & 1u)");
+                o("{ const bool s_ = ((%s) ^ %uu) != 0u; const u32 v = s_ ? %s : %s; ", cond.c_str(), (pb >> 3) & 1u,
+                  a.c_str(), b.c_str());
+                const char* v[] = {"v"};
+                wr(o, I.d0, v, 1);
+                o("}\n");
+                return;
+            }
+            case ISETP: case FSETP: case DSETP: {
+                const uint32_t pb = I.d0 & 7, cc = mod & 7;
+                if (op == ISETP)
+                    o("{ const bool v = %s(%s, %s, %uu); ", (mod & 8) ? "jcmp_u" : "jcmp_s",
+                      (mod & 8) ? a.c_str() : ("(i32)" + a).c_str(), (mod & 8) ? b.c_str() : ("(i32)" + b).c_str(), cc);
+                else if (op == FSETP)
+                    o("{ const bool v = jcmp_f((double)ju2f(%s), (double)ju2f(%s), %uu); ", a.c_str(), R(I.b).c_str(), cc);
+                else
+                    o("{ const bool v = jcmp_f(ju2d(%s), ju2d(%s), %uu); ", R64(I.a).c_str(), R64(I.b).c_str(), cc);
+                if (pb != 7) o("if (ex) preds = (preds & ~(1u << %uu)) | ((u32)v << %uu); ", pb, pb);
+                o("}\n");
+                return;
+            }
+            case FADD: case FMUL: {
+                o("{ const float x = ju2f(%s ^ %s), y = ju2f(%s ^ %s); const u32 v = jfbits(%s(x, y)); ", a.c_str(),
+                  hex((mod & 1u) << 31).c_str(), b.c_str(), hex((mod & 2u) << 30).c_str(),
+                  op == FADD ? "__fadd_rn" : "__fmul_rn");
+                const char* v[] = {"v"};
+                wr(o, I.d0, v, 1);
+                o("}\n");
+                return;
+            }
+            case FMNMX: {
+                o("{ const u32 v = jfmnmx(%s, %s, %s); ", a.c_str(), b.c_str(), (mod & 1) ? "true" : "false");
+                const char* v[] = {"v"};
+                wr(o, I.d0, v, 1);
+                o("}\n");
+                return;
+            }
+            case DADD: case DMUL: case DFMA: {
+                o("{ const double x = ju2d(%s ^ %s), y = ju2d(%s ^ %s), z = ju2d(%s ^ %s); ", R64(I.a).c_str(),
+                  (mod & 1) ? "0x8000000000000000ull" : "0ull", R64(I.b).c_str(),
+                  (mod & 2) ? "0x8000000000000000ull" : "0ull", R64(I.c).c_str(),
+                  (mod & 4) ? "0x8000000000000000ull" : "0ull");
+                o("const u64 r_ = jdbits(%s); const u32 v0 = (u32)r_, v1 = (u32)(r_ >> 32); ",
+                  op == DADD ? "__dadd_rn(x, y)" : op == DMUL ? "__dmul_rn(x, y)" : "__fma_rn(x, y, z)");
+                (void)0;
+                const char* v[] = {"v0", "v1"};
+                wr(o, I.d0, v, 2);
+                o("}\n");
+                return;
+            }
+            case LDC: {
+                const uint32_t w0 = I.imm >> 2;
+                o("{ const u32 v0 = %uu < cbank_len ? __ldg(&cb[%uu]) : 0u; ", w0, w0);
+                if (mod & 1) {
+                    o("const u32 v1 = %uu < cbank_len ? __ldg(&cb[%uu]) : 0u; ", w0 + 1, w0 + 1);
+                    const char* v[] = {"v0", "v1"};
+                    wr(o, I.d0, v, 2);
+                } else {
+                    const char* v[] = {"v0"};
+                    wr(o, I.d0, v, 1);
+                }
+                o("}\n");
+                return;
+            }
+            case I2F: {
+                o("{ const u32 v = jfbits(%s); ", (mod & 1) ? ("__uint2float_rn(" + a + ")").c_str()
+                                                            : ("__int2float_rn((int)" + a + ")").c_str());
+                const char* v[] = {"v"};
+                wr(o, I.d0, v, 1);
+                o("}\n");
+                return;
+            }
+            case F2I: { o("{ const u32 v = jf2i(%s); ", a.c_str()); const char* v[] = {"v"}; wr(o, I.d0, v, 1); o("}\n"); return; }
+            case F2F_F64_F32: {
+                o("{ const u64 r_ = jdbits((double)ju2f(%s)); const u32 v0 = (u32)r_, v1 = (u32)(r_ >> 32); ", a.c_str());
+                const char* v[] = {"v0", "v1"};
+                wr(o, I.d0, v, 2);
+                o("}\n");
+                return;
+            }
+            case F2F_F32_F64: {
+                o("{ const u32 v = jfbits(__double2float_rn(ju2d(%s))); ", R64(I.a).c_str());
+                const char* v[] = {"v"};
+                wr(o, I.d0, v, 1);
+                o("}\n");
+                return;
+            }
+            case SHFL: {
+                o("{ const u32 src_ = jshfl_src(lane, %s, %uu); const u32 v = __shfl_sync(JFULL, %s, src_); ", b.c_str(),
+                  mod & 3u, a.c_str());
+                const char* v[] = {"v"};
+                wr(o, I.d0, v, 1);
+                o("}\n");
+                return;
+            }
+            case MUFU_RCP64: {
+                o("{ const u64 r_ = jdbits(__drcp_rn(ju2d(%s))); const u32 v0 = (u32)r_, v1 = (u32)(r_ >> 32); ",
+                  R64(I.a).c_str());
+                const char* v[] = {"v0", "v1"};
+                wr(o, I.d0, v, 2);
+                o("}\n");
+                return;
+            }
+            case IMNMX: {
+                if (mod & 8)
+                    o("{ const u32 a_ = %s, b_ = %s; const u32 v = %s; ", a.c_str(), b.c_str(),
+                      (mod & 1) ? "max(a_, b_)" : "min(a_, b_)");
+                else
+                    o("{ const i32 a_ = (i32)%s, b_ = (i32)%s; const u32 v = (u32)%s; ", a.c_str(), b.c_str(),
+                      (mod & 1) ? "max(a_, b_)" : "min(a_, b_)");
+                const char* v[] = {"v"};
+                wr(o, I.d0, v, 1);
+                o("}\n");
+                return;
+            }
+            default: o("/* nop */\n"); return;
+        }
+    }
+
+    // LDG / STG.  `stepx` = this instruction's step.
+    void mem(Src& o, const fi_insn& I, uint32_t pc, const char* stepx) const {
+        using namespace fi;
+        const uint32_t lw = (I.mod & 3) > 2 ? 2 : (I.mod & 3), nw = 1u << lw;
+        o("{ const bool pv = %s; const bool ex = inA && pv; ", guard(I.guard).c_str());
+        o("const u64 va = %s + (u64)(i64)(i32)%s; ", R64(I.a).c_str(), hex(I.imm).c_str());
+        if (I.op == LDG) {
+            o("uint4 v_; const u32 c_ = jldg<%uu>(A, bc, va, k, ex, v_); ", lw);
+            o("if (__ballot_sync(JFULL, c_ != 0u)) { fault = __ballot_sync(JFULL, c_ == 1u) ? 1u : 2u; fault_pc = %uu; "
+              "step = %s; goto finish; } ", pc, stepx);
+            const char* v[] = {"v_.x", "v_.y", "v_.z", "v_.w"};
+            wr(o, I.d0, v, nw);
+            o("}\n");
+        } else {
+            o("const u32 exm_ = amask & __ballot_sync(JFULL, pv); bool z_ = false; "
+              "const u32 c_ = ex ? jcheck(A, bc, va, %uu, k, &z_) : 0u; ", 4u << lw);
+            o("if (__ballot_sync(JFULL, c_ != 0u)) { fault = __ballot_sync(JFULL, c_ == 1u) ? 1u : 2u; fault_pc = %uu; "
+              "step = %s; goto finish; } ", pc, stepx);
+            o("const u32 sst_ = %s; if (sst_ > hstep) { if (ex) { const u32 idx_ = __popc(exm_ & lt_mask) * %uu; ",
+              stepx, nw);
+            for (uint32_t q = 0; q < nw; ++q)
+                o("if (nst + idx_ + %uu < st_cap) { jfi_store e_; e_.va = va + %uu; e_.value = %s; e_.step = sst_; "
+                  "st_out[nst + idx_ + %uu] = e_; } ",
+                  q, 4 * q, (I.b == kRZ ? std::string("0u") : R(I.b + q)).c_str(), q);
+            o("} nst += __popc(exm_) * %uu; } }\n", nw);
+        }
+    }
+
+    // m consecutive independent LDGs (block mode): all address checks first, one
+    // fault ballot (the first faulting load in program order wins, C-9), then all
+    // loads in flight together, then the register writes in program order.
+    void ldg_batch(Src& o, const fi_insn* code, uint32_t i0, uint32_t m) const {
+        o(" { // LDG batch %u..%u\n", i0, i0 + m - 1);
+        for (uint32_t j = 0; j < m; ++j) {
+            const fi_insn& I = code[i0 + j];
+            const uint32_t lw = (I.mod & 3) > 2 ? 2 : (I.mod & 3);
+            o("  const bool ex%u = inA && %s; const u64 va%u = %s + (u64)(i64)(i32)%s; bool z%u = false; "
+              "const u32 c%u = ex%u ? jcheck(A, bc, va%u, %uu, k, &z%u) : 0u;\n",
+              j, guard(I.guard).c_str(), j, R64(I.a).c_str(), hex(I.imm).c_str(), j, j, j, j, 4u << lw, j);
+        }
+        o("  if (__ballot_sync(JFULL, 0u");
+        for (uint32_t j = 0; j < m; ++j) o(" | c%u", j);
+        o(")) {\n");
+        for (uint32_t j = 0; j < m; ++j)
+            o("   if (__ballot_sync(JFULL, c%u != 0u)) { fault = __ballot_sync(JFULL, c%u == 1u) ? 1u : 2u; "
+              "fault_pc = %uu; step = step + (%uu - pcm); goto finish; }\n",
+              j, j, i0 + j, i0 + j);
+        o("  }\n");
+        for (uint32_t j = 0; j < m; ++j) {
+            const fi_insn& I = code[i0 + j];
+            const uint32_t lw = (I.mod & 3) > 2 ? 2 : (I.mod & 3);
+            o("  uint4 v%u = make_uint4(0u, 0u, 0u, 0u); if (ex%u && !z%u) { const u8* p_ = A.img + (va%u - JVA_BASE); ",
+              j, j, j, j);
+            if (lw == 0) o("v%u.x = jld32(p_); }\n", j);
+            else if (lw == 1) o("const uint2 t_ = jld64(p_); v%u.x = t_.x; v%u.y = t_.y; }\n", j, j);
+            else o("v%u = jld128(p_); }\n", j);
+        }
+        for (uint32_t j = 0; j < m; ++j) {
+            const fi_insn& I = code[i0 + j];
+            const uint32_t lw = (I.mod & 3) > 2 ? 2 : (I.mod & 3), nw = 1u << lw;
+            if (I.d0 == fi::kRZ) continue;
+            for (uint32_t q = 0; q < nw; ++q)
+                if (W(I.d0 + q)) o("  if (ex%u) R%u = v%u.%c;\n", j, I.d0 + q, j, "xyzw"[q]);
+        }
+        o(" }\n");
+    }
+};
+
+// consecutive LDGs from i0 that may be batched: none crosses a leader (a jump
+// target) and none's address pair is written by an earlier LDG of the batch
+static uint32_t ldg_batch_len(const fi_insn* code, uint32_t n, uint32_t i0, const std::vector<uint8_t>& leader) {
+    using namespace fi;
+    uint32_t m = 0;
+    for (uint32_t j = i0; j < n && code[j].op == LDG && m < 8 && (j == i0 || !leader[j]); ++j) {
+        bool hazard = false;
+        for (uint32_t q = i0; q < j && !hazard; ++q) {
+            const Dests d = dests_of(code[q].op, code[q].d0, code[q].d1, code[q].mod);
+            for (uint32_t x = 0; x < 2; ++x) {
+                const uint32_t a = code[j].a + x;
+                if (code[j].a != kRZ && a >= d.gp_base && a < d.gp_base + d.n_gp) hazard = true;
+            }
+        }
+        if (hazard) break;
+        ++m;
+    }
+    return m;
+}
+
+// Generate the device function of one static kernel (EMU_INJ mode).
+void gen_kernel(Src& o, const Gen& G, uint32_t kid, const fi_insn* code, uint32_t n) {
+    using namespace fi;
+    const uint32_t NR = G.NR;
+    // block length from each pc: to the next BRA/EXIT inclusive, or the code end
+    std::vector<uint32_t> blen(n);
+    for (int64_t i = (int64_t)n - 1; i >= 0; --i) {
+        const uint32_t op = code[i].op;
+        blen[i] = (op == BRA || op == EXIT || i + 1 == (int64_t)n) ? 1u : blen[i + 1] + 1u;
+    }
+    o("__device__ __noinline__ void kern_%u(const JArgs& A, const u32 hstep, const u32 hpc, const u32 hlane, "
+      "const u32 hkind, const u32 hreg, const u32 hbfm, const u32 hmask, const u32 k, const u32 cta, "
+      "const u32 wic, const u32 watchdog, const u32* __restrict__ ck, const u32 ck_interval, "
+      "jfi_store* __restrict__ st_out, const u32 st_cap, JOut& out) {\n", kid);
+    o("const u32 lane = threadIdx.x & 31u, lt_mask = (1u << lane) - 1u;\n");
+    o("const jfi_instance in = A.inst[k];\nconst u32 cbank_len = in.cbank_len; const u32* __restrict__ cb = A.cbank + "
+      "in.cbank_off;\n(void)cbank_len; (void)cb; (void)lt_mask;\n");
+    for (uint32_t j = 0; j < NR; ++j) o("u32 R%u;%s", j, (j % 16 == 15) ? "\n" : " ");
+    o("\nconst u32 nl_ = in.block - wic * 32u; bool live = lane < (nl_ > 32u ? 32u : nl_);\n");
+    o("u32 pc = 0u, preds = 0u, step = 0u;\n");
+    o("if (ck) {\n  const u32 c_ = hstep / ck_interval; const u32* __restrict__ src = ck + (u64)c_ * %uu;\n",
+      (NR + 3) * 32);
+    for (uint32_t j = 0; j < NR; ++j) o("  R%u = __ldg(&src[%uu + lane]);\n", j, j * 32);
+    o("  pc = __ldg(&src[%uu + lane]); preds = __ldg(&src[%uu + lane]); live = __ldg(&src[%uu + lane]) != 0u; "
+      "step = c_ * ck_interval;\n} else {\n",
+      NR * 32, NR * 32 + 32, NR * 32 + 64);
+    for (uint32_t j = 0; j < NR; ++j) o("R%u = 0u;%s", j, (j % 16 == 15) ? "\n" : " ");
+    o("\n}\n");
+    o("u32 livem = __ballot_sync(JFULL, live);\nbool conv = false; u32 upc = 0u, amask = 0u, npc = 0xFFFFFFFFu;\n"
+      "u32 nst = 0u, fault = 0u, fault_pc = 0u, before = 0u, after = 0u, msk = 0u; bool fired = false, bad = false;\n"
+      "JBufCache bc;\n");
+    o("for (;;) {\n if (!livem) break;\n u32 pcm, active;\n"
+      " if (conv) { pcm = upc; active = amask; }\n"
+      " else { pcm = __reduce_min_sync(JFULL, live ? pc : 0xFFFFFFFFu); active = __ballot_sync(JFULL, live && pc == pcm);\n"
+      "   npc = active == livem ? 0xFFFFFFFFu : __reduce_min_sync(JFULL, (live && pc != pcm) ? pc : 0xFFFFFFFFu);\n"
+      "   conv = true; upc = pcm; amask = active; }\n"
+      " const bool inA = (amask >> lane) & 1u;\n"
+      " if (step >= watchdog) { fault = 3u; fault_pc = pcm; break; }\n"
+      " if (pcm >= %uu) { fault = 4u; fault_pc = pcm; break; }\n"
+      " u32 taken = 0u, exm = 0u, tgt = 0u;\n",
+      n);
+    // leaders: pc 0, branch targets, and the pc after every BRA / EXIT.  Blocks
+    // are entered only at leaders (few merge points keep the block code
+    // straight-line for the compiler); any other pc runs single steps until a
+    // leader is reached (after a checkpoint restart or the injection site).
+    std::vector<uint8_t> leader(n + 1, 0);
+    leader[0] = 1;
+    for (uint32_t i = 0; i < n; ++i) {
+        if (code[i].op == BRA && code[i].imm < n) leader[code[i].imm] = 1;
+        if ((code[i].op == BRA || code[i].op == EXIT) && i + 1 < n) leader[i + 1] = 1;
+    }
+    // dispatch: a whole block when it fits, else one step
+    o(" switch (pcm) {\n");
+    for (uint32_t i = 0; i < n; ++i)
+        if (leader[i])
+            o("  case %u: if (%uu <= npc && step + %uu <= watchdog && (u32)(hstep - step) >= %uu) goto B%u; goto S_any;\n",
+              i, i + blen[i], blen[i], blen[i], i);
+    o("  default: goto S_any;\n }\n");
+    // ---- block code (fallthrough from a leader to the block's BRA / EXIT)
+    char stepx[64];
+    uint32_t batch_end = 0;                           // LDGs [.., batch_end) already emitted as a batch
+    for (uint32_t i = 0; i < n; ++i) {
+        const fi_insn& I = code[i];
+        std::snprintf(stepx, sizeof stepx, "step + (%uu - pcm)", i);
+        if (leader[i]) o(" B%u:\n", i);
+        if (i < batch_end) {
+            if (i + 1 == n)
+                o(" { step += %uu - pcm; upc = %uu; if (upc >= npc) { conv = false; if (inA) pc = upc; } continue; }\n",
+                  n, n);
+            continue;
+        }
+        if (I.op == LDG) {
+            const uint32_t m = ldg_batch_len(code, n, i, leader);
+            if (m >= 2) {
+                G.ldg_batch(o, code, i, m);
+                batch_end = i + m;
+                if (i + m == n)
+                    o(" { step += %uu - pcm; upc = %uu; if (upc >= npc) { conv = false; if (inA) pc = upc; } continue; }\n",
+                      n, n);
+                continue;
+            }
+        }
+        if (I.op == BRA) {
+            o(" { const bool pv = %s; const u32 exm_ = amask & __ballot_sync(JFULL, pv); step += %uu - pcm;\n"
+              "   if (exm_ == 0u) upc = %uu; else if (exm_ == amask) upc = %uu;\n"
+              "   else { conv = false; if (inA) pc = ((exm_ >> lane) & 1u) ? %uu : %uu; }\n"
+              "   if (conv && (amask == 0u || upc >= npc)) { conv = false; if ((amask >> lane) & 1u) pc = upc; }\n"
+              "   continue; }\n",
+              G.guard(I.guard).c_str(), i + 1, i + 1, I.imm, I.imm, i + 1);
+        } else if (I.op == EXIT) {
+            o(" { const bool pv = %s; const u32 exm_ = amask & __ballot_sync(JFULL, pv); step += %uu - pcm;\n"
+              "   if (inA && pv) live = false; livem &= ~exm_; amask &= ~exm_; upc = %uu;\n"
+              "   if (conv && (amask == 0u || upc >= npc)) { conv = false; if ((amask >> lane) & 1u) pc = upc; }\n"
+              "   continue; }\n",
+              G.guard(I.guard).c_str(), i + 1, i + 1);
+        } else {
+            if (I.op == LDG || I.op == STG) {
+                G.mem(o, I, i, stepx);
+            } else {
+                o(" { const bool ex = inA && %s; ", G.guard(I.guard).c_str());
+                G.plain(o, I);
+                o(" }\n");
+            }
+            if (i + 1 == n)
+                o(" { step += %uu - pcm; upc = %uu; if (upc >= npc) { conv = false; if (inA) pc = upc; } continue; }\n",
+                  n, n);
+        }
+    }
+    // ---- single steps
+    o(" S_any:\n switch (pcm) {\n");
+    for (uint32_t i = 0; i < n; ++i) {
+        const fi_insn& I = code[i];
+        o("  case %u: { const bool pv = %s; const u32 pred_ = __ballot_sync(JFULL, pv); const bool ex = inA && pv; "
+          "exm = active & pred_; (void)ex;\n",
+          i, G.guard(I.guard).c_str());
+        if (I.op == BRA) {
+            o("  taken = exm; tgt = %uu;\n", I.imm);
+        } else if (I.op == EXIT) {
+            o("  if (ex) live = false; livem &= ~exm; amask &= ~exm;\n");
+        } else if (I.op == LDG || I.op == STG) {
+            o("  ");
+            G.mem(o, I, i, "step");
+        } else {
+            o("  ");
+            G.plain(o, I);
+        }
+        o("  } break;\n");
+    }
+    o("  default: break;\n }\n");
+    o(" // Sdone\n"
+      " if (taken == 0u) upc = pcm + 1u; else if (taken == active) upc = tgt;\n"
+      " else { conv = false; if (inA) pc = ((taken >> lane) & 1u) ? tgt : pcm + 1u; }\n"
+      " if (conv && (amask == 0u || upc >= npc)) { conv = false; if ((amask >> lane) & 1u) pc = upc; }\n");
+    // the transient fault (C-7, C-8), after the instruction wrote its destinations
+    o(" if (step == hstep) {\n  fired = true;\n  if (pcm != hpc || !((exm >> hlane) & 1u)) bad = true;\n"
+      "  if (lane == hlane) {\n   if (hkind == 0) {\n    switch (hreg) {\n");
+    for (uint32_t j = 0; j < NR; ++j)
+        o("     case %u: before = R%u; msk = hbfm == 3 ? before : hmask; after = before ^ msk; R%u = after; break;\n",
+          j, j, j);
+    o("     default: before = 0u; msk = hbfm == 3 ? 0u : hmask; after = msk; break;\n    }\n   } else {\n"
+      "    const u32 p_ = hreg & 7u; const u32 b_ = (p_ == 7u) ? 1u : ((preds >> p_) & 1u); u32 m_ = hmask, a_;\n"
+      "    if (hbfm == 0 || hbfm == 1) a_ = b_ ^ 1u; else if (hbfm == 2) a_ = (m_ >> 31) & 1u; else { m_ = b_; a_ = 0u; }\n"
+      "    before = b_; msk = m_; after = a_; if (p_ != 7u) preds = (preds & ~(1u << p_)) | (a_ << p_);\n   }\n  }\n }\n"
+      " ++step;\n}\n");
+    o("finish:\n out.steps = step; out.fault = fault; out.fault_pc = fault_pc; out.nstore = nst;\n"
+      " out.before = __shfl_sync(JFULL, before, hlane); out.after = __shfl_sync(JFULL, after, hlane);\n"
+      " out.mask = __shfl_sync(JFULL, msk, hlane); out.fired = fired; out.bad = bad;\n}\n\n");
+}
+
+std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern, uint32_t n_regs) {
+    Src o;
+    o.s = kPrelude;
+    Gen G{n_regs};
+    for (uint32_t k = 0; k < n_kern; ++k) gen_kernel(o, G, k, code + kern[k].code_off, kern[k].code_len);
+    // K4 on the generated kernels: persistent warps over the LPT-ordered replicas
+    // (same scheduling and outputs as inject.cu's k_inject)
+    o("extern \"C\" __global__ void __launch_bounds__(128) k_inject_jit(const JArgs A, const u64* __restrict__ warp_off, "
+      "const jfi_site* __restrict__ sites, const u32 n, jfi_inj* __restrict__ out, jfi_store* __restrict__ log, "
+      "const u32 cap, const u32* ckpt, const u64* __restrict__ ck_off, const u32 ck_interval, "
+      "const u32* __restrict__ order, u32* counter, u32* status) {\n"
+      " const u32 lane = threadIdx.x & 31u;\n"
+      " for (;;) {\n  u32 p = 0u; if (lane == 0u) p = atomicAdd(counter, 1u); p = __shfl_sync(JFULL, p, 0);\n"
+      "  if (p >= n) return;\n  const u32 i = order[p]; const jfi_site S = sites[i];\n"
+      "  if (S.flags & 1u) { if (lane == 0u) { jfi_inj r; r.before = r.after = r.mask = r.fault_pc = 0u; "
+      "r.fault_kind = 0; r.outcome = 3; r.overflow = 0; r.flags = 0; r.n_faulty_stores = 0u; out[i] = r; } continue; }\n"
+      "  const jfi_instance in = A.inst[S.instance]; const u32 wpc = (in.block + 31u) / 32u, lw = S.warp - in.warp_begin;\n"
+      "  const u64 L = warp_off[S.warp + 1] - warp_off[S.warp]; const u64 wd = 10ull * L + 1024ull;\n"
+      "  const u32 watchdog = wd > 0xFFFFFFFFull ? 0xFFFFFFFFu : (u32)wd;\n"
+      "  const u32* ck = ckpt ? ckpt + ck_off[S.warp] * %uull : (const u32*)0;\n"
+      "  JOut o;\n  switch (in.kernel) {\n",
+      (n_regs + 3) * 32);
+    for (uint32_t k = 0; k < n_kern; ++k)
+        o("   case %u: kern_%u(A, S.step, S.pc, S.lane, S.dst_kind, S.dst_reg, S.bfm, S.mask, S.instance, lw / wpc, lw %% wpc, watchdog, ck, ck ? ck_interval : 0u, "
+          "log + (u64)i * cap, cap, o); break;\n", k, k);
+    o("   default: o.steps = 0; o.fired = false; o.bad = true; o.fault = 0; o.fault_pc = 0; o.nstore = 0; "
+      "o.before = o.after = o.mask = 0; break;\n  }\n"
+      "  if (lane == 0u) {\n   jfi_inj r; r.before = o.before; r.after = o.after; r.mask = o.mask; r.fault_pc = o.fault_pc;\n"
+      "   r.fault_kind = (u8)o.fault; r.outcome = 0; r.overflow = o.nstore > cap; r.flags = 0; r.n_faulty_stores = o.nstore;\n"
+      "   out[i] = r;\n   if (!o.fired || o.bad) atomicOr(status, 1u << 6);\n"
+      "   const u32 start = ck ? S.step / ck_interval * ck_interval : 0u;\n"
+      "   atomicAdd((unsigned long long*)(counter + 2), (unsigned long long)(o.steps - start));\n  }\n  __syncwarp();\n }\n}\n");
+    return o.s;
+}
+
+// ---------------------------------------------------------------- NVRTC + driver
+typedef int (*nvrtcCreateProgram_t)(void**, const char*, const char*, int, const char* const*, const char* const*);
+typedef int (*nvrtcCompileProgram_t)(void*, int, const char* const*);
+typedef int (*nvrtcGetSize_t)(void*, size_t*);
+typedef int (*nvrtcGetData_t)(void*, char*);
+typedef int (*nvrtcDestroyProgram_t)(void**);
+
+struct Nvrtc {
+    void* h = nullptr;
+    nvrtcCreateProgram_t create = nullptr;
+    nvrtcCompileProgram_t compile = nullptr;
+    nvrtcGetSize_t log_size = nullptr, cubin_size = nullptr;
+    nvrtcGetData_t log = nullptr, cubin = nullptr;
+    nvrtcDestroyProgram_t destroy = nullptr;
+    bool ok = false;
+};
+
+Nvrtc& nvrtc() {
+    static Nvrtc N;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        const char* cands[] = {"libnvrtc.so.12", "/usr/local/cuda/lib64/libnvrtc.so.12", "libnvrtc.so"};
+        for (const char* c : cands)
+            if ((N.h = dlopen(c, RTLD_NOW | RTLD_LOCAL))) break;
+        if (!N.h) return;
+        N.create = (nvrtcCreateProgram_t)dlsym(N.h, "nvrtcCreateProgram");
+        N.compile = (nvrtcCompileProgram_t)dlsym(N.h, "nvrtcCompileProgram");
+        N.log_size = (nvrtcGetSize_t)dlsym(N.h, "nvrtcGetProgramLogSize");
+        N.log = (nvrtcGetData_t)dlsym(N.h, "nvrtcGetProgramLog");
+        N.cubin_size = (nvrtcGetSize_t)dlsym(N.h, "nvrtcGetCUBINSize");
+        N.cubin = (nvrtcGetData_t)dlsym(N.h, "nvrtcGetCUBIN");
+        N.destroy = (nvrtcDestroyProgram_t)dlsym(N.h, "nvrtcDestroyProgram");
+        N.ok = N.create && N.compile && N.log_size && N.log && N.cubin_size && N.cubin && N.destroy;
+    });
+    return N;
+}
+
+typedef CUresult (*cuModuleLoadData_t)(CUmodule*, const void*);
+typedef CUresult (*cuModuleGetFunction_t)(CUfunction*, CUmodule, const char*);
+typedef CUresult (*cuModuleUnload_t)(CUmodule);
+typedef CUresult (*cuLaunchKernel_t)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned,
+                                     CUstream, void**, void**);
+typedef CUresult (*cuOccupancy_t)(int*, CUfunction, int, size_t);
+
+struct Drv {
+    cuModuleLoadData_t load = nullptr;
+    cuModuleGetFunction_t get = nullptr;
+    cuModuleUnload_t unload = nullptr;
+    cuLaunchKernel_t launch = nullptr;
+    cuOccupancy_t occ = nullptr;
+    bool ok = false;
+};
+
+Drv& drv() {
+    static Drv D;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        cudaDriverEntryPointQueryResult q;
+        cudaGetDriverEntryPoint("cuModuleLoadData", (void**)&D.load, cudaEnableDefault, &q);
+        cudaGetDriverEntryPoint("cuModuleGetFunction", (void**)&D.get, cudaEnableDefault, &q);
+        cudaGetDriverEntryPoint("cuModuleUnload", (void**)&D.unload, cudaEnableDefault, &q);
+        cudaGetDriverEntryPoint("cuLaunchKernel", (void**)&D.launch, cudaEnableDefault, &q);
+        cudaGetDriverEntryPoint("cuOccupancyMaxActiveBlocksPerMultiprocessor", (void**)&D.occ, cudaEnableDefault, &q);
+        D.ok = D.load && D.get && D.unload && D.launch && D.occ;
+    });
+    return D;
+}
+
+thread_local std::string g_jit_log;
+
+}  // namespace
+
+struct fi_jit {
+    CUmodule mod = nullptr;
+    CUfunction inject = nullptr;
+    uint32_t n_regs = 0, n_code = 0;
+    double compile_s = 0;
+    size_t src_bytes = 0, cubin_bytes = 0;
+};
+
+namespace fi {
+void launch_lpt_order(const fi_site* sites, const uint64_t* warp_off, uint32_t ck_interval, uint32_t n,
+                      uint32_t* order, uint32_t* counter, cudaStream_t s);
+}
+
+extern "C" const char* fi_jit_log(void) { return g_jit_log.c_str(); }
+
+extern "C" size_t fi_jit_source(const fi_insn* code_host, uint32_t n_code, const fi_kernel* kern_host, uint32_t n_kern,
+                                uint32_t n_regs, char* buf, size_t buf_bytes) {
+    if (!code_host || !kern_host || !n_kern || n_regs == 0 || n_regs > fi::kRZ) return 0;
+    for (uint32_t k = 0; k < n_kern; ++k)
+        if ((uint64_t)kern_host[k].code_off + kern_host[k].code_len > n_code) return 0;
+    const std::string s = generate(code_host, kern_host, n_kern, n_regs);
+    if (buf && buf_bytes) {
+        const size_t m = std::min(buf_bytes - 1, s.size());
+        std::memcpy(buf, s.data(), m);
+        buf[m] = 0;
+    }
+    return s.size() + 1;
+}
+
+namespace {
+fi_status compile_cubin(const fi_insn* code, uint32_t n_code, const fi_kernel* kern, uint32_t n_kern, uint32_t n_regs,
+                        std::string& src, std::vector<char>& cubin) {
+    (void)n_code;
+    Nvrtc& N = nvrtc();
+    if (!N.ok) { g_jit_log = "libnvrtc.so.12 not found"; return FI_E_CUDA; }
+    src = generate(code, kern, n_kern, n_regs);
+    void* prog = nullptr;
+    if (N.create(&prog, src.c_str(), "fi_jit.cu", 0, nullptr, nullptr)) { g_jit_log = "nvrtcCreateProgram failed"; return FI_E_CUDA; }
+    const char* opts[] = {"--gpu-architecture=sm_100a", "--std=c++17", "--fmad=false", "-lineinfo"};
+    const int rc = N.compile(prog, 4, opts);
+    size_t ls = 0;
+    N.log_size(prog, &ls);
+    std::string lg(ls, '\0');
+    if (ls) N.log(prog, &lg[0]);
+    g_jit_log = lg;
+    if (rc) { N.destroy(&prog); return FI_E_PROGRAM; }
+    size_t cs = 0;
+    N.cubin_size(prog, &cs);
+    cubin.resize(cs);
+    N.cubin(prog, cubin.data());
+    N.destroy(&prog);
+    return FI_OK;
+}
+}  // namespace
+
+extern "C" fi_status fi_jit_compile_check(const fi_insn* code_host, uint32_t n_code, const fi_kernel* kern_host,
+                                          uint32_t n_kern, uint32_t n_regs, size_t* cubin_bytes) {
+    if (!code_host || !kern_host || !n_kern || n_regs == 0 || n_regs > fi::kRZ) return FI_E_ARG;
+    for (uint32_t k = 0; k < n_kern; ++k)
+        if ((uint64_t)kern_host[k].code_off + kern_host[k].code_len > n_code) return FI_E_ARG;
+    std::string src;
+    std::vector<char> cubin;
+    fi_status e = compile_cubin(code_host, n_code, kern_host, n_kern, n_regs, src, cubin);
+    if (cubin_bytes) *cubin_bytes = cubin.size();
+    return e;
+}
+
+extern "C" fi_status fi_jit_build(const fi_program* p, const fi_kernel* kern_host, fi_jit** out) {
+    if (!p || !kern_host || !out || !p->code_host || !p->n_kern || p->n_regs == 0 || p->n_regs > fi::kRZ)
+        return FI_E_ARG;
+    for (uint32_t k = 0; k < p->n_kern; ++k)
+        if ((uint64_t)kern_host[k].code_off + kern_host[k].code_len > p->n_code) return FI_E_ARG;
+    *out = nullptr;
+    Drv& D = drv();
+    if (!D.ok) { g_jit_log = "CUDA driver entry points unavailable"; return FI_E_CUDA; }
+    const auto t0 = std::chrono::steady_clock::now();
+    fi_status e0 = fi::cuda_status(cudaFree(0));       // bind the device's primary context to this thread
+    if (e0) return e0;
+    std::string src;
+    std::vector<char> cubin;
+    fi_status e = compile_cubin(p->code_host, p->n_code, kern_host, p->n_kern, p->n_regs, src, cubin);
+    if (e) return e;
+    const size_t cs = cubin.size();
+    fi_jit* j = new fi_jit();
+    if (D.load(&j->mod, cubin.data()) != CUDA_SUCCESS || D.get(&j->inject, j->mod, "k_inject_jit") != CUDA_SUCCESS) {
+        g_jit_log += "\ncuModuleLoadData/cuModuleGetFunction failed";
+        if (j->mod) D.unload(j->mod);
+        delete j;
+        return FI_E_CUDA;
+    }
+    j->n_regs = p->n_regs;
+    j->n_code = p->n_code;
+    j->src_bytes = src.size();
+    j->cubin_bytes = cs;
+    j->compile_s = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+    *out = j;
+    return FI_OK;
+}
+
+extern "C" double fi_jit_compile_seconds(const fi_jit* j) { return j ? j->compile_s : 0.0; }
+
+extern "C" void fi_jit_free(fi_jit* j) {
+    if (!j) return;
+    if (j->mod) drv().unload(j->mod);
+    delete j;
+}
+
+struct JArgsHost {
+    const uint8_t* img;
+    const uint32_t* gran;
+    const fi_buffer* buf;
+    const fi_instance* inst;
+    const uint32_t* cbank;
+    uint64_t image_bytes;
+};
+
+
+extern "C" fi_status fi_inject_jit(const fi_jit* j, const fi_program* p, const uint8_t* image, const fi_trace* t,
+                                   const fi_site* sites, uint32_t n, fi_inj* out, fi_store* log, uint32_t log_cap,
+                                   void* ws, size_t ws_bytes, uint32_t* dev_status, void* stream) {
+    if (!j || !p || !image || !t || !sites || !out || !dev_status || (log_cap && !log) || !p->aux) return FI_E_ARG;
+    if (j->n_regs != p->n_regs || j->n_code != p->n_code) return FI_E_ARG;
+    if (t->ckpt && (!t->ckpt_off || !t->ckpt_interval)) return FI_E_ARG;
+    if (n == 0) return FI_OK;
+    if (!ws || ws_bytes < fi_inject_workspace(n)) return FI_E_ARG;
+    cudaStream_t s = (cudaStream_t)stream;
+    uint32_t* counter = reinterpret_cast<uint32_t*>(ws);
+    uint32_t* order = reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(ws) + 256);
+    const uint32_t ck_iv = t->ckpt ? t->ckpt_interval : 0;
+    fi::launch_lpt_order(sites, t->warp_off, ck_iv, n, order, counter, s);
+    fi_status e = fi::launch_status();
+    if (e) return e;
+    Drv& D = drv();
+    int dev = 0, sms = 0, per = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    D.occ(&per, j->inject, 128, 0);
+    const uint32_t grid =
+        (uint32_t)std::min<uint64_t>((n + 3) / 4, (uint64_t)std::max(1, sms * std::max(1, per)));
+    JArgsHost A{image, reinterpret_cast<const uint32_t*>(p->aux)   /* granule map at aux offset 0 */, p->buf, p->inst, p->cbank, p->image_bytes};
+    const uint64_t* warp_off = t->warp_off;
+    const uint32_t* ckpt = t->ckpt;
+    const uint64_t* ck_off = t->ckpt_off;
+    void* args[] = {&A, (void*)&warp_off, (void*)&sites, &n, &out, &log, &log_cap, (void*)&ckpt, (void*)&ck_off,
+                    (void*)&ck_iv, &order, &counter, &dev_status};
+    const CUresult r = D.launch(j->inject, grid, 1, 1, 128, 1, 1, 0, (CUstream)s, args, nullptr);
+    if (r != CUDA_SUCCESS) {
+        g_jit_log = "cuLaunchKernel failed: " + std::to_string((int)r);
+        return FI_E_CUDA;
+    }
+    return fi::launch_status();
+}

@@ -152,6 +152,13 @@ def lib():
                                                  vp, vp]),
             "fi_classify_batched": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, u32, u32, u32, u32, vp, sz, vp, vp]),
             "fi_inject_permanent": (st, [vp, vp, vp, vp, u32, vp, vp, vp, u32, u32, vp, u32, vp, sz, vp, vp]),
+            "fi_jit_build": (st, [vp, vp, C.POINTER(vp)]),
+            "fi_jit_free": (None, [vp]),
+            "fi_jit_compile_seconds": (C.c_double, [vp]),
+            "fi_jit_log": (C.c_char_p, []),
+            "fi_jit_compile_check": (st, [vp, u32, vp, u32, u32, C.POINTER(C.c_size_t)]),
+            "fi_jit_source": (sz, [vp, u32, vp, u32, u32, vp, sz]),
+            "fi_inject_jit": (st, [vp, vp, vp, vp, vp, u32, vp, vp, u32, vp, sz, vp, vp]),
             "fi_write_profile_txt": (st, [vp, vp, u32, vp, u32, vp, sz, C.POINTER(C.c_size_t)]),
             "fi_campaign": (st, [C.POINTER(fi_campaign_cfg), C.c_int, C.c_int, ALLREDUCE_FN, vp,
                                  C.POINTER(fi_campaign_result)]),
@@ -232,6 +239,8 @@ class DeviceProgram:
                                device=self.device)
         self._code_host = np.ascontiguousarray(prog.code)
         self._inst_host = np.ascontiguousarray(prog.instances)
+        self._kern_host = np.ascontiguousarray(prog.kernels)
+        self._jit = None
         self.n_regs = int(lib().fi_program_regs(self._code_host.ctypes.data, len(self._code_host)))
         self.c = fi_program(
             _p(self.code), len(prog.code), _p(self.kern), len(prog.kernels), _p(self.inst), len(prog.instances),
@@ -243,9 +252,64 @@ class DeviceProgram:
     def n_inst(self):
         return len(self.prog.instances)
 
+    def jit(self) -> "Jit":
+        """The program's JIT-specialised emulator module (fi_jit_build), built once
+        per (code, kernel table, register rows, device) in this process."""
+        if self._jit is None:
+            import hashlib
+            key = (hashlib.sha1(self._code_host.tobytes() + self._kern_host.tobytes()).hexdigest(), self.n_regs,
+                   self.device.index if self.device.index is not None else torch.cuda.current_device())
+            if key not in _JIT_CACHE:
+                _JIT_CACHE[key] = Jit(self)
+            self._jit = _JIT_CACHE[key]
+        return self._jit
+
     @property
     def n_warps(self):
         return self.prog.n_warps
+
+
+_JIT_CACHE: dict = {}
+
+
+class Jit:
+    """fi_jit_build: per-program generated CUDA, NVRTC-compiled for sm_100a."""
+
+    def __init__(self, dp: "DeviceProgram"):
+        h = C.c_void_p()
+        rc = lib().fi_jit_build(C.byref(dp.c), dp._kern_host.ctypes.data, C.byref(h))
+        if rc != FI_OK:
+            raise FIError(rc, "fi_jit_build", lib().fi_jit_log().decode()[-4000:])
+        self.h = h
+        self.compile_seconds = float(lib().fi_jit_compile_seconds(h))
+
+    def __del__(self):
+        try:
+            if self.h:
+                lib().fi_jit_free(self.h)
+                self.h = None
+        except Exception:
+            pass
+
+
+def jit_source(prog, n_regs: int | None = None) -> str:
+    code, kern = np.ascontiguousarray(prog.code), np.ascontiguousarray(prog.kernels)
+    nr = n_regs or int(lib().fi_program_regs(code.ctypes.data, len(code)))
+    n = lib().fi_jit_source(code.ctypes.data, len(code), kern.ctypes.data, len(kern), nr, None, 0)
+    buf = C.create_string_buffer(n)
+    lib().fi_jit_source(code.ctypes.data, len(code), kern.ctypes.data, len(kern), nr, buf, n)
+    return buf.value.decode()
+
+
+def jit_compile_check(prog) -> int:
+    """NVRTC-compile the program's generated emulator without loading it (no GPU); returns cubin bytes."""
+    code, kern = np.ascontiguousarray(prog.code), np.ascontiguousarray(prog.kernels)
+    nr = int(lib().fi_program_regs(code.ctypes.data, len(code)))
+    cb = C.c_size_t(0)
+    rc = lib().fi_jit_compile_check(code.ctypes.data, len(code), kern.ctypes.data, len(kern), nr, C.byref(cb))
+    if rc != FI_OK:
+        raise FIError(rc, "fi_jit_compile_check", lib().fi_jit_log().decode()[-4000:])
+    return int(cb.value)
 
 
 @dataclass
@@ -384,8 +448,11 @@ def select_sites(idx: SiteIndex, sched: fi_schedule, j0: int, n: int, sites: tor
 
 
 def inject(gt: GoldenTrace, sites: torch.Tensor, n: int, log_cap: int, out: torch.Tensor | None = None,
-           log: torch.Tensor | None = None, status: DeviceStatus | None = None, ws: torch.Tensor | None = None):
-    """fi_inject (K4)."""
+           log: torch.Tensor | None = None, status: DeviceStatus | None = None, ws: torch.Tensor | None = None,
+           engine: str = "jit"):
+    """fi_inject (K4).  engine "jit": fi_inject_jit on the program's generated
+    emulator (built on first use); "interp": fi_inject (the shared-memory
+    interpreter).  Both give bit-identical results."""
     dev = gt.dp.device
     if out is None:
         out = torch.empty(max(n, 1) * 24, dtype=torch.uint8, device=dev)
@@ -395,8 +462,14 @@ def inject(gt: GoldenTrace, sites: torch.Tensor, n: int, log_cap: int, out: torc
     ws_n = lib().fi_inject_workspace(n)
     if ws is None or ws.numel() < ws_n:
         ws = torch.empty(ws_n, dtype=torch.uint8, device=dev)
-    _check(lib().fi_inject(C.byref(gt.dp.c), _p(gt.image), C.byref(gt.c), _p(sites), n, _p(out), _p(log), log_cap,
-                           _p(ws), ws_n, st.ptr, _stream()), "fi_inject")
+    if engine == "jit":
+        _check(lib().fi_inject_jit(gt.dp.jit().h, C.byref(gt.dp.c), _p(gt.image), C.byref(gt.c), _p(sites), n, _p(out),
+                                   _p(log), log_cap, _p(ws), ws_n, st.ptr, _stream()), "fi_inject_jit")
+    elif engine == "interp":
+        _check(lib().fi_inject(C.byref(gt.dp.c), _p(gt.image), C.byref(gt.c), _p(sites), n, _p(out), _p(log), log_cap,
+                               _p(ws), ws_n, st.ptr, _stream()), "fi_inject")
+    else:
+        raise ValueError(engine)
     if status is None:
         st.check("fi_inject")
     return out, log

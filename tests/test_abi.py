@@ -93,3 +93,13 @@ def test_campaign_argument_errors_without_gpu():
     assert L.fi_campaign(C.byref(cfg), 0, 1, fi.ALLREDUCE_FN(), None, C.byref(res)) == fi.FI_E_ARG   # empty program
     assert L.fi_campaign(C.byref(cfg), 2, 2, fi.ALLREDUCE_FN(), None, C.byref(res)) == fi.FI_E_ARG   # rank >= world
     assert L.fi_campaign(C.byref(cfg), 0, 2, fi.ALLREDUCE_FN(), None, C.byref(res)) == fi.FI_E_ARG   # no callback
+
+
+def test_jit_source_compiles_for_sm100a():
+    """The JIT-specialised emulator's generated CUDA compiles with NVRTC for
+    sm_100a (no GPU needed) for programs exercising every opcode."""
+    from paper_conf_dsn_0002hsvk21_b200 import fi
+    for prog in (P.c1(), P.fuzz_program(3, n_ops=120), P.multi_instance_chain(3), P.scatter_chain()):
+        assert fi.jit_compile_check(prog) > 1000
+    src = fi.jit_source(P.c1())
+    assert "k_inject_jit" in src and "kern_0" in src

@@ -1,0 +1,87 @@
+"""The JIT-specialised emulator (fi_jit_build / fi_inject_jit): per-program
+generated CUDA compiled by NVRTC must give results bit-identical to the
+shared-memory interpreter (fi_inject) — every fi_inj field and every logged
+faulty store — and to the CPU oracle (the oracle comparisons of
+test_gpu_parity.py run on the JIT path, fi.inject's default engine)."""
+import numpy as np
+import pytest
+import torch
+
+import oracle as O
+from fi_inputs import hpc as H
+from fi_inputs import programs as P
+from fi_inputs import resnet as RN
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def F():
+    from paper_conf_dsn_0002hsvk21_b200 import fi
+    return fi
+
+
+def _both(F, prog, seed, groups, bfms, n, ckpt="auto", approx=False):
+    dp = F.DeviceProgram(prog)
+    gt = F.golden_run(dp, ckpt_interval=ckpt)
+    if approx:
+        idx = F.InstanceIndex(gt, F.profile_approx(gt))
+        sites = F.select_sites_approx(idx, F.schedule(seed, groups, bfms), 0, n)
+    else:
+        ic, cc = F.profile(gt)
+        sites = F.select_sites(F.SiteIndex(gt, ic, cc), F.schedule(seed, groups, bfms), 0, n)
+    cap = F.log_capacity(gt)
+    res = {}
+    for eng in ("interp", "jit"):
+        out, log = F.inject(gt, sites, n, cap, engine=eng)
+        torch.cuda.synchronize()
+        res[eng] = (F.as_numpy(out, F.INJ_DTYPE, n).copy(), log.view(-1, 16).cpu().numpy().copy())
+    a, b = res["interp"][0], res["jit"][0]
+    for f in a.dtype.names:
+        bad = np.flatnonzero(a[f] != b[f])
+        assert bad.size == 0, f"{f}: replica {bad[0]} interp {a[bad[0]]} jit {b[bad[0]]}"
+    la, lb = res["interp"][1].reshape(n, cap, 16), res["jit"][1].reshape(n, cap, 16)
+    for i in range(n):
+        k = min(int(a["n_faulty_stores"][i]), cap)
+        assert np.array_equal(la[i, :k], lb[i, :k]), f"faulty store log of replica {i}"
+    return a, F.as_numpy(sites, F.SITE_DTYPE, n)
+
+
+def test_jit_c1(F):
+    a, s = _both(F, P.c1(), P.CAMPAIGN_SEED[1], [F.G_GP, F.G_PR, F.G_GPPR], [0, 1, 2, 3], 400)
+    assert len(np.unique(a["outcome"] * 0 + a["fault_kind"])) >= 2
+
+
+@pytest.mark.parametrize("seed", range(24))
+def test_jit_fuzz(F, seed):
+    prog = P.fuzz_program(300 + seed, n_ops=int(60 + seed * 11 % 140), block=[80, 64, 96, 33][seed % 4])
+    _both(F, prog, 0xBEE0 + seed, [F.G_GPPR, F.G_GP, F.G_PR, F.G_FP32, F.G_FP64, F.G_OTHERS][: 1 + seed % 6],
+          [0, 1, 2, 3], 300, ckpt=[0, 5, 13, "auto"][seed % 4])
+
+
+def test_jit_mini_c2(F):
+    a, _ = _both(F, P.c2(full=False), 0x77, [F.G_GP, F.G_LD, F.G_PR, F.G_OTHERS], [0, 1, 2, 3], 600)
+    assert (a["fault_kind"] == 3).sum() + (a["fault_kind"] == 2).sum() > 0
+
+
+@pytest.mark.parametrize("seed", [5, 6, 7])
+def test_jit_ffma_special_values(F, seed):
+    _both(F, P.ffma_runs(seed), seed, [F.G_FP32, F.G_GP, F.G_LD], [0, 1, 2, 3], 300)
+
+
+@pytest.mark.parametrize("maker", [lambda: P.multi_instance_chain(6, shrink=29), P.scatter_chain,
+                                   lambda: P.c3(full=False), lambda: RN.c4(full=False)])
+def test_jit_multi_launch(F, maker):
+    _both(F, maker(), 0x4A11, [F.G_GP, F.G_LD, F.G_GPPR, F.G_OTHERS], [0, 1, 2, 3], 400)
+
+
+def test_jit_approximate_not_injected(F):
+    a, s = _both(F, P.multi_instance_chain(n_inst=6, n=256, shrink=33), 0xA11, [F.G_GP, F.G_FP32], [0, 1, 2, 3], 300,
+                 approx=True)
+    assert ((s["flags"] == 1) == (a["outcome"] == F.NOT_INJECTED)).all()
+
+
+@pytest.mark.parametrize("which", range(5))
+def test_jit_c5_minis(F, which):
+    prog = H.c5(full=False)[which]
+    _both(F, prog, 0xC5, [F.G_GP, F.G_GPPR, F.G_PR], [0, 1, 2, 3], 300)
