@@ -25,6 +25,7 @@
 #include <chrono>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <string>
@@ -334,21 +335,19 @@ struct Gen {
               "fault_pc = %uu; step = step + (%uu - pcm); goto finish; }\n",
               j, j, i0 + j, i0 + j);
         o("  }\n");
-        for (uint32_t j = 0; j < m; ++j) {
-            const fi_insn& I = code[i0 + j];
-            const uint32_t lw = (I.mod & 3) > 2 ? 2 : (I.mod & 3);
-            o("  uint4 v%u = make_uint4(0u, 0u, 0u, 0u); if (ex%u && !z%u) { const u8* p_ = A.img + (va%u - JVA_BASE); ",
-              j, j, j, j);
-            if (lw == 0) o("v%u.x = jld32(p_); }\n", j);
-            else if (lw == 1) o("const uint2 t_ = jld64(p_); v%u.x = t_.x; v%u.y = t_.y; }\n", j, j);
-            else o("v%u = jld128(p_); }\n", j);
-        }
+        // loads straight into the destination registers (predicated, program order)
         for (uint32_t j = 0; j < m; ++j) {
             const fi_insn& I = code[i0 + j];
             const uint32_t lw = (I.mod & 3) > 2 ? 2 : (I.mod & 3), nw = 1u << lw;
-            if (I.d0 == fi::kRZ) continue;
-            for (uint32_t q = 0; q < nw; ++q)
-                if (W(I.d0 + q)) o("  if (ex%u) R%u = v%u.%c;\n", j, I.d0 + q, j, "xyzw"[q]);
+            o("  if (ex%u) { uint4 v_ = make_uint4(0u, 0u, 0u, 0u); if (!z%u) { const u8* p_ = A.img + (va%u - JVA_BASE); ",
+              j, j, j);
+            if (lw == 0) o("v_.x = jld32(p_); } ");
+            else if (lw == 1) o("const uint2 t_ = jld64(p_); v_.x = t_.x; v_.y = t_.y; } ");
+            else o("v_ = jld128(p_); } ");
+            if (I.d0 != fi::kRZ)
+                for (uint32_t q = 0; q < nw; ++q)
+                    if (W(I.d0 + q)) o("R%u = v_.%c; ", I.d0 + q, "xyzw"[q]);
+            o("}\n");
         }
         o(" }\n");
     }
@@ -384,10 +383,11 @@ void gen_kernel(Src& o, const Gen& G, uint32_t kid, const fi_insn* code, uint32_
         const uint32_t op = code[i].op;
         blen[i] = (op == BRA || op == EXIT || i + 1 == (int64_t)n) ? 1u : blen[i + 1] + 1u;
     }
-    o("__device__ __noinline__ void kern_%u(const JArgs& A, const u32 hstep, const u32 hpc, const u32 hlane, "
+    o("__device__ __noinline__ void kern_%u(const JArgs& A_, const u32 hstep, const u32 hpc, const u32 hlane, "
       "const u32 hkind, const u32 hreg, const u32 hbfm, const u32 hmask, const u32 k, const u32 cta, "
       "const u32 wic, const u32 watchdog, const u32* __restrict__ ck, const u32 ck_interval, "
       "jfi_store* __restrict__ st_out, const u32 st_cap, JOut& out) {\n", kid);
+    o("const JArgs A = A_;                 // kernel arguments in registers for the whole run\n");
     o("const u32 lane = threadIdx.x & 31u, lt_mask = (1u << lane) - 1u;\n");
     o("const jfi_instance in = A.inst[k];\nconst u32 cbank_len = in.cbank_len; const u32* __restrict__ cb = A.cbank + "
       "in.cbank_off;\n(void)cbank_len; (void)cb; (void)lt_mask;\n");
@@ -457,12 +457,23 @@ void gen_kernel(Src& o, const Gen& G, uint32_t kid, const fi_insn* code, uint32_
             }
         }
         if (I.op == BRA) {
+            // block chaining: a uniform branch to a block that fits goes straight to
+            // its code (the loop-top checks it skips cannot fire: see `fits`)
+            auto chain = [&](uint32_t L) -> std::string {
+                if (L >= n || !leader[L]) return "";
+                char b[256];
+                std::snprintf(b, sizeof b,
+                              "if (%uu <= npc && step + %uu <= watchdog && (u32)(hstep - step) >= %uu) { pcm = %uu; "
+                              "goto B%u; } ",
+                              L + blen[L], blen[L], blen[L], L, L);
+                return b;
+            };
             o(" { const bool pv = %s; const u32 exm_ = amask & __ballot_sync(JFULL, pv); step += %uu - pcm;\n"
-              "   if (exm_ == 0u) upc = %uu; else if (exm_ == amask) upc = %uu;\n"
+              "   if (exm_ == 0u) { %supc = %uu; } else if (exm_ == amask) { %supc = %uu; }\n"
               "   else { conv = false; if (inA) pc = ((exm_ >> lane) & 1u) ? %uu : %uu; }\n"
               "   if (conv && (amask == 0u || upc >= npc)) { conv = false; if ((amask >> lane) & 1u) pc = upc; }\n"
               "   continue; }\n",
-              G.guard(I.guard).c_str(), i + 1, i + 1, I.imm, I.imm, i + 1);
+              G.guard(I.guard).c_str(), i + 1, chain(i + 1).c_str(), i + 1, chain(I.imm).c_str(), I.imm, I.imm, i + 1);
         } else if (I.op == EXIT) {
             o(" { const bool pv = %s; const u32 exm_ = amask & __ballot_sync(JFULL, pv); step += %uu - pcm;\n"
               "   if (inA && pv) live = false; livem &= ~exm_; amask &= ~exm_; upc = %uu;\n"
@@ -524,13 +535,17 @@ void gen_kernel(Src& o, const Gen& G, uint32_t kid, const fi_insn* code, uint32_
 }
 
 std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern, uint32_t n_regs) {
+    // resident 128-thread CTAs per SM the register budget targets (3: <= 168 registers)
+    uint32_t min_blocks = 3;
+    if (const char* e = std::getenv("FI_JIT_MIN_BLOCKS")) min_blocks = (uint32_t)std::max(1, std::atoi(e));
     Src o;
     o.s = kPrelude;
     Gen G{n_regs};
     for (uint32_t k = 0; k < n_kern; ++k) gen_kernel(o, G, k, code + kern[k].code_off, kern[k].code_len);
     // K4 on the generated kernels: persistent warps over the LPT-ordered replicas
     // (same scheduling and outputs as inject.cu's k_inject)
-    o("extern \"C\" __global__ void __launch_bounds__(128) k_inject_jit(const JArgs A, const u64* __restrict__ warp_off, "
+    o("extern \"C\" __global__ void __launch_bounds__(128, %u) k_inject_jit(", min_blocks);
+    o("const JArgs A, const u64* __restrict__ warp_off, "
       "const jfi_site* __restrict__ sites, const u32 n, jfi_inj* __restrict__ out, jfi_store* __restrict__ log, "
       "const u32 cap, const u32* ckpt, const u64* __restrict__ ck_off, const u32 ck_interval, "
       "const u32* __restrict__ order, u32* counter, u32* status) {\n"
