@@ -231,8 +231,9 @@ __device__ __forceinline__ uint32_t check_access(const EmuProg& P, BufCache& C, 
                                                  bool* zero) {
     if (va & (w - 1)) return 1;
     const uint64_t off = va - kVaBase;
-    if (off >= C.lo0 && off + w <= C.hi0) { *zero = C.z0; return 0; }
-    if (off >= C.lo1 && off + w <= C.hi1) { *zero = C.z1; return 0; }
+    // (off < hi first: an address just below the VA base wraps off + w around)
+    if (off >= C.lo0 && off < C.hi0 && off + w <= C.hi0) { *zero = C.z0; return 0; }
+    if (off >= C.lo1 && off < C.hi1 && off + w <= C.hi1) { *zero = C.z1; return 0; }
     if (va < kVaBase || off >= P.image_bytes) return 2;
     const uint32_t b = __ldg(&P.gran[off >> 8]);
     if (b == kNoBuf) return 2;

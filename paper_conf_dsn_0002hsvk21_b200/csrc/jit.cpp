@@ -66,7 +66,7 @@ struct Gen {
         const uint32_t gs = g & 7, neg = (g >> 3) & 1;
         if (gs == 7) return neg ? "false" : "true";
         char b[96];
-        std::snprintf(b, sizeof b, "((((preds >> %uu) & 1u) ^ %uu) != 0u)", gs, neg);
+        std::snprintf(b, sizeof b, neg ? "(!Q%u)" : "Q%u", gs);
         return b;
     }
     std::string bv(const fi_insn& I) const {
@@ -131,7 +131,7 @@ struct Gen {
                   a.c_str(), c.c_str(), b.c_str(), (mod & 1) ? "0u - a_" : "a_", (mod & 2) ? "0u - b_" : "b_");
                 const char* v[] = {"v"};
                 wr(o, I.d0, v, 1);
-                if (pb != 7) o("if (ex) preds = (preds & ~(1u << %uu)) | ((u32)((s_ >> 32) != 0ull) << %uu); ", pb, pb);
+                if (pb != 7) o("if (ex) Q%u = (s_ >> 32) != 0ull; ", pb);
                 o("}\n");
                 return;
             }
@@ -168,8 +168,8 @@ struct Gen {
             }
             case SEL: {
                 const uint32_t pb = I.c & 0xF, p = pb & 7;
-                std::string cond = p == 7 ? "1u" : ("((preds >> " + std::to_string(p) + "u) & 1u)");
-                o("{ const bool s_ = ((%s) ^ %uu) != 0u; const u32 v = s_ ? %s : %s; ", cond.c_str(), (pb >> 3) & 1u,
+                std::string cond = p == 7 ? "true" : ("Q" + std::to_string(p));
+                o("{ const bool s_ = %s%s; const u32 v = s_ ? %s : %s; ", (pb >> 3) & 1u ? "!" : "", cond.c_str(),
                   a.c_str(), b.c_str());
                 const char* v[] = {"v"};
                 wr(o, I.d0, v, 1);
@@ -185,7 +185,7 @@ struct Gen {
                     o("{ const bool v = jcmp_f((double)ju2f(%s), (double)ju2f(%s), %uu); ", a.c_str(), R(I.b).c_str(), cc);
                 else
                     o("{ const bool v = jcmp_f(ju2d(%s), ju2d(%s), %uu); ", R64(I.a).c_str(), R64(I.b).c_str(), cc);
-                if (pb != 7) o("if (ex) preds = (preds & ~(1u << %uu)) | ((u32)v << %uu); ", pb, pb);
+                if (pb != 7) o("if (ex) Q%u = v; ", pb);
                 o("}\n");
                 return;
             }
@@ -322,11 +322,24 @@ struct Gen {
         o(" { // LDG batch %u..%u\n", i0, i0 + m - 1);
         for (uint32_t j = 0; j < m; ++j) {
             const fi_insn& I = code[i0 + j];
-            const uint32_t lw = (I.mod & 3) > 2 ? 2 : (I.mod & 3);
-            o("  const bool ex%u = inA && %s; const u64 va%u = %s + (u64)(i64)(i32)%s; bool z%u = false; "
-              "const u32 c%u = ex%u ? jcheck(A, bc, va%u, %uu, k, &z%u) : 0u;\n",
-              j, guard(I.guard).c_str(), j, R64(I.a).c_str(), hex(I.imm).c_str(), j, j, j, j, 4u << lw, j);
+            o("  const bool ex%u = inA && %s; const u64 va%u = %s + (u64)(i64)(i32)%s; bool z%u = false; u32 c%u = 0u;\n",
+              j, guard(I.guard).c_str(), j, R64(I.a).c_str(), hex(I.imm).c_str(), j, j);
         }
+        // fast path: every executing lane hits its buffer cache (no table lookups, no
+        // cache updates); otherwise the full checks in program order
+        o("  if (__ballot_sync(JFULL, !(true");
+        for (uint32_t j = 0; j < m; ++j) {
+            const fi_insn& I = code[i0 + j];
+            const uint32_t lw = (I.mod & 3) > 2 ? 2 : (I.mod & 3);
+            o(" && (!ex%u || jhit(bc, va%u, %uu, &z%u))", j, j, 4u << lw, j);
+        }
+        o("))) {\n");
+        for (uint32_t j = 0; j < m; ++j) {
+            const fi_insn& I = code[i0 + j];
+            const uint32_t lw = (I.mod & 3) > 2 ? 2 : (I.mod & 3);
+            o("   c%u = ex%u ? jcheck(A, bc, va%u, %uu, k, &z%u) : 0u;\n", j, j, j, 4u << lw, j);
+        }
+        o("  }\n");
         o("  if (__ballot_sync(JFULL, 0u");
         for (uint32_t j = 0; j < m; ++j) o(" | c%u", j);
         o(")) {\n");
@@ -393,18 +406,22 @@ void gen_kernel(Src& o, const Gen& G, uint32_t kid, const fi_insn* code, uint32_
       "in.cbank_off;\n(void)cbank_len; (void)cb; (void)lt_mask;\n");
     for (uint32_t j = 0; j < NR; ++j) o("u32 R%u;%s", j, (j % 16 == 15) ? "\n" : " ");
     o("\nconst u32 nl_ = in.block - wic * 32u; bool live = lane < (nl_ > 32u ? 32u : nl_);\n");
-    o("u32 pc = 0u, preds = 0u, step = 0u;\n");
+    o("u32 pc = 0u, step = 0u; bool Q0 = false, Q1 = false, Q2 = false, Q3 = false, Q4 = false, Q5 = false, "
+      "Q6 = false;\n");
     o("if (ck) {\n  const u32 c_ = hstep / ck_interval; const u32* __restrict__ src = ck + (u64)c_ * %uu;\n",
       (NR + 3) * 32);
     for (uint32_t j = 0; j < NR; ++j) o("  R%u = __ldg(&src[%uu + lane]);\n", j, j * 32);
-    o("  pc = __ldg(&src[%uu + lane]); preds = __ldg(&src[%uu + lane]); live = __ldg(&src[%uu + lane]) != 0u; "
-      "step = c_ * ck_interval;\n} else {\n",
+    o("  pc = __ldg(&src[%uu + lane]); const u32 pw_ = __ldg(&src[%uu + lane]); live = __ldg(&src[%uu + lane]) != 0u; "
+      "step = c_ * ck_interval;\n  Q0 = pw_ & 1u; Q1 = (pw_ >> 1) & 1u; Q2 = (pw_ >> 2) & 1u; Q3 = (pw_ >> 3) & 1u; "
+      "Q4 = (pw_ >> 4) & 1u; Q5 = (pw_ >> 5) & 1u; Q6 = (pw_ >> 6) & 1u;\n} else {\n",
       NR * 32, NR * 32 + 32, NR * 32 + 64);
     for (uint32_t j = 0; j < NR; ++j) o("R%u = 0u;%s", j, (j % 16 == 15) ? "\n" : " ");
     o("\n}\n");
     o("u32 livem = __ballot_sync(JFULL, live);\nbool conv = false; u32 upc = 0u, amask = 0u, npc = 0xFFFFFFFFu;\n"
       "u32 nst = 0u, fault = 0u, fault_pc = 0u, before = 0u, after = 0u, msk = 0u; bool fired = false, bad = false;\n"
-      "JBufCache bc;\n");
+      "JBufCache bc;\n"
+      "// blocks run only within [step, lim): lim = the watchdog, or the injection step while it is pending\n"
+      "u32 lim = (hstep >= step && hstep < watchdog) ? hstep : watchdog;\n");
     o("for (;;) {\n if (!livem) break;\n u32 pcm, active;\n"
       " if (conv) { pcm = upc; active = amask; }\n"
       " else { pcm = __reduce_min_sync(JFULL, live ? pc : 0xFFFFFFFFu); active = __ballot_sync(JFULL, live && pc == pcm);\n"
@@ -429,8 +446,7 @@ void gen_kernel(Src& o, const Gen& G, uint32_t kid, const fi_insn* code, uint32_
     o(" switch (pcm) {\n");
     for (uint32_t i = 0; i < n; ++i)
         if (leader[i])
-            o("  case %u: if (%uu <= npc && step + %uu <= watchdog && (u32)(hstep - step) >= %uu) goto B%u; goto S_any;\n",
-              i, i + blen[i], blen[i], blen[i], i);
+            o("  case %u: if (%uu <= npc && step + %uu <= lim) goto B%u; goto S_any;\n", i, i + blen[i], blen[i], i);
     o("  default: goto S_any;\n }\n");
     // ---- block code (fallthrough from a leader to the block's BRA / EXIT)
     char stepx[64];
@@ -462,10 +478,8 @@ void gen_kernel(Src& o, const Gen& G, uint32_t kid, const fi_insn* code, uint32_
             auto chain = [&](uint32_t L) -> std::string {
                 if (L >= n || !leader[L]) return "";
                 char b[256];
-                std::snprintf(b, sizeof b,
-                              "if (%uu <= npc && step + %uu <= watchdog && (u32)(hstep - step) >= %uu) { pcm = %uu; "
-                              "goto B%u; } ",
-                              L + blen[L], blen[L], blen[L], L, L);
+                std::snprintf(b, sizeof b, "if (%uu <= npc && step + %uu <= lim) { pcm = %uu; goto B%u; } ", L + blen[L],
+                              blen[L], L, L);
                 return b;
             };
             o(" { const bool pv = %s; const u32 exm_ = amask & __ballot_sync(JFULL, pv); step += %uu - pcm;\n"
@@ -525,10 +539,14 @@ void gen_kernel(Src& o, const Gen& G, uint32_t kid, const fi_insn* code, uint32_
         o("     case %u: before = R%u; msk = hbfm == 3 ? before : hmask; after = before ^ msk; R%u = after; break;\n",
           j, j, j);
     o("     default: before = 0u; msk = hbfm == 3 ? 0u : hmask; after = msk; break;\n    }\n   } else {\n"
-      "    const u32 p_ = hreg & 7u; const u32 b_ = (p_ == 7u) ? 1u : ((preds >> p_) & 1u); u32 m_ = hmask, a_;\n"
+      "    const u32 p_ = hreg & 7u;\n"
+      "    const u32 b_ = p_ == 0u ? Q0 : p_ == 1u ? Q1 : p_ == 2u ? Q2 : p_ == 3u ? Q3 : p_ == 4u ? Q4 : p_ == 5u ? Q5 : "
+      "p_ == 6u ? Q6 : 1u;\n    u32 m_ = hmask, a_;\n"
       "    if (hbfm == 0 || hbfm == 1) a_ = b_ ^ 1u; else if (hbfm == 2) a_ = (m_ >> 31) & 1u; else { m_ = b_; a_ = 0u; }\n"
-      "    before = b_; msk = m_; after = a_; if (p_ != 7u) preds = (preds & ~(1u << p_)) | (a_ << p_);\n   }\n  }\n }\n"
-      " ++step;\n}\n");
+      "    before = b_; msk = m_; after = a_;\n"
+      "    switch (p_) { case 0: Q0 = a_; break; case 1: Q1 = a_; break; case 2: Q2 = a_; break; case 3: Q3 = a_; break; "
+      "case 4: Q4 = a_; break; case 5: Q5 = a_; break; case 6: Q6 = a_; break; default: break; }\n   }\n  }\n }\n"
+      " ++step;\n if (step > hstep) lim = watchdog;\n}\n");
     o("finish:\n out.steps = step; out.fault = fault; out.fault_pc = fault_pc; out.nstore = nst;\n"
       " out.before = __shfl_sync(JFULL, before, hlane); out.after = __shfl_sync(JFULL, after, hlane);\n"
       " out.mask = __shfl_sync(JFULL, msk, hlane); out.fired = fired; out.bad = bad;\n}\n\n");

@@ -154,8 +154,9 @@ struct JBufCache {
 __device__ __forceinline__ u32 jcheck(const JArgs& A, JBufCache& C, u64 va, u32 w, u32 k, bool* zero) {
     if (va & (w - 1)) return 1;
     const u64 off = va - JVA_BASE;
-    if (off >= C.lo0 && off + w <= C.hi0) { *zero = C.z0; return 0; }
-    if (off >= C.lo1 && off + w <= C.hi1) { *zero = C.z1; return 0; }
+    // (off < hi first: an address just below the VA base wraps off + w around)
+    if (off >= C.lo0 && off < C.hi0 && off + w <= C.hi0) { *zero = C.z0; return 0; }
+    if (off >= C.lo1 && off < C.hi1 && off + w <= C.hi1) { *zero = C.z1; return 0; }
     if (va < JVA_BASE || off >= A.image_bytes) return 2;
     const u32 b = __ldg(&A.gran[off >> 8]);
     if (b == JNOBUF) return 2;
@@ -166,6 +167,16 @@ __device__ __forceinline__ u32 jcheck(const JArgs& A, JBufCache& C, u64 va, u32 
     C.lo0 = lo; C.hi0 = hi; C.z0 = wr >= 0 && (u32)wr >= k;
     *zero = C.z0;
     return 0;
+}
+
+// cache-only check: true iff the access is aligned and inside one of the two
+// cached buffers (then *zero is that buffer's writer-rule flag); no state change
+__device__ __forceinline__ bool jhit(const JBufCache& C, u64 va, u32 w, bool* zero) {
+    const u64 off = va - JVA_BASE;
+    const bool h0 = off >= C.lo0 && off < C.hi0 && off + w <= C.hi0;
+    const bool h1 = off >= C.lo1 && off < C.hi1 && off + w <= C.hi1;
+    *zero = h0 ? C.z0 : C.z1;
+    return ((va & (w - 1)) == 0) && (h0 || h1);
 }
 
 // one LDG of 1/2/4 words for this lane; returns the fault code (0 ok)
