@@ -411,7 +411,9 @@ typedef int (*fi_allreduce_fn)(void* dev, uint64_t count, uint32_t elem_bytes, v
 #define FI_PROPAGATION_AUTO 0u      /* K8 from 64 launches on, else K5/K7 (fi_classify) */
 #define FI_PROPAGATION_K7 1u        /* fi_classify */
 #define FI_PROPAGATION_K8 2u        /* fi_classify_batched */
-#define FI_CKPT_AUTO 0xFFFFFFFFu    /* 4096 steps, doubled until the checkpoints fit 20% of free HBM */
+#define FI_CKPT_AUTO 0xFFFFFFFFu
+#define FI_ENGINE_INTERP 0u
+#define FI_ENGINE_JIT 1u    /* 4096 steps, doubled until the checkpoints fit 20% of free HBM */
 typedef struct {
     /* the program, HOST arrays */
     const fi_insn* code;         uint32_t n_code;
@@ -428,6 +430,8 @@ typedef struct {
     uint32_t propagation;        /* FI_PROPAGATION_* */
     uint32_t approximate;        /* 1 = approximate profile (row f1) */
     uint32_t ckpt_interval;      /* steps between golden checkpoints, 0 = none, FI_CKPT_AUTO */
+    uint32_t engine;             /* K4 engine: FI_ENGINE_INTERP, or FI_ENGINE_JIT (fi_inject_jit; the module is
+                                    built once per program and device and cached for the process) */
     uint64_t k8_mem_budget;      /* device bytes for K8 scratch (0 = 24 GiB) */
     int device;                  /* CUDA device ordinal (< 0 = current) */
     void* stream;                /* cudaStream_t (NULL = a stream fi_campaign creates) */
@@ -445,6 +449,7 @@ typedef struct {
     /* CUDA-event times on the stream, ms: H2D + prepare, golden run, profile,
      * count exchange, index, select, inject, classify + histogram exchange, D2H */
     float ms_h2d, ms_golden, ms_profile, ms_exchange, ms_index, ms_select, ms_inject, ms_classify, ms_d2h;
+    float ms_jit;                /* host time building the JIT module (0 when cached or not used) */
     /* optional host outputs (NULL = not returned) */
     fi_site* sites;              /* [n_local] */
     fi_inj* inj;                 /* [n_local] */

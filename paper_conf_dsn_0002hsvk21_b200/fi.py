@@ -86,7 +86,7 @@ class fi_campaign_cfg(C.Structure):
                 ("sched", fi_schedule),
                 ("n_replicas", C.c_uint64),
                 ("flags", C.c_uint32), ("propagation", C.c_uint32), ("approximate", C.c_uint32),
-                ("ckpt_interval", C.c_uint32), ("k8_mem_budget", C.c_uint64),
+                ("ckpt_interval", C.c_uint32), ("engine", C.c_uint32), ("k8_mem_budget", C.c_uint64),
                 ("device", C.c_int), ("stream", C.c_void_p)]
 
 
@@ -97,7 +97,7 @@ class fi_campaign_result(C.Structure):
                 ("n_unclassified", C.c_uint64), ("n_not_injected", C.c_uint64),
                 ("ms_h2d", C.c_float), ("ms_golden", C.c_float), ("ms_profile", C.c_float),
                 ("ms_exchange", C.c_float), ("ms_index", C.c_float), ("ms_select", C.c_float),
-                ("ms_inject", C.c_float), ("ms_classify", C.c_float), ("ms_d2h", C.c_float),
+                ("ms_inject", C.c_float), ("ms_classify", C.c_float), ("ms_d2h", C.c_float), ("ms_jit", C.c_float),
                 ("sites", C.c_void_p), ("inj", C.c_void_p), ("inst_counts", C.c_void_p)]
 
 
@@ -717,7 +717,7 @@ class CampaignResult:
 def campaign(prog, seed: int, groups, bfms, n_replicas: int, rank: int = 0, world: int = 1, allreduce=None,
              unchecked: bool = False, propagation: str = "auto", approximate: bool = False, ckpt="auto",
              k8_mem_budget: int = 0, device: int | None = None, host: dict | None = None,
-             return_arrays: bool = True) -> CampaignResult:
+             return_arrays: bool = True, engine: str = "jit") -> CampaignResult:
     """fi_campaign: the whole campaign of this rank from HOST arrays (golden run,
     sharded profile, count exchange, index, select, inject, classify, histogram
     exchange, D2H).  `host`: optional pinned uint8 tensors keyed code / kernels /
@@ -744,6 +744,7 @@ def campaign(prog, seed: int, groups, bfms, n_replicas: int, rank: int = 0, worl
     cfg.propagation = FI_PROPAGATION[propagation]
     cfg.approximate = 1 if approximate else 0
     cfg.ckpt_interval = FI_CKPT_AUTO if ckpt == "auto" else int(ckpt)
+    cfg.engine = {"interp": 0, "jit": 1}[engine]
     cfg.k8_mem_budget = k8_mem_budget
     cfg.device = torch.cuda.current_device() if device is None else device
     cfg.stream = torch.cuda.current_stream(cfg.device).cuda_stream or None
@@ -760,7 +761,7 @@ def campaign(prog, seed: int, groups, bfms, n_replicas: int, rank: int = 0, worl
     cb = allreduce if allreduce is not None else ALLREDUCE_FN()
     _check(lib().fi_campaign(C.byref(cfg), rank, world, cb, None, C.byref(res)), "fi_campaign")
     ms = {k: float(getattr(res, "ms_" + k)) for k in
-          ("h2d", "golden", "profile", "exchange", "index", "select", "inject", "classify", "d2h")}
+          ("h2d", "golden", "profile", "exchange", "index", "select", "inject", "classify", "d2h", "jit")}
     return CampaignResult(np.array(res.hist, dtype=np.uint64).reshape(8, 4, 3), [int(x) for x in res.totals],
                           int(res.n_rec), int(res.counted), int(res.j0), int(res.n_local),
                           (int(res.rec_begin), int(res.rec_end)), int(res.n_unclassified), int(res.n_not_injected),
