@@ -396,10 +396,25 @@ void gen_kernel(Src& o, const Gen& G, uint32_t kid, const fi_insn* code, uint32_
         const uint32_t op = code[i].op;
         blen[i] = (op == BRA || op == EXIT || i + 1 == (int64_t)n) ? 1u : blen[i + 1] + 1u;
     }
+    // leaders: pc 0, branch targets, and the pc after every BRA / EXIT.  Blocks
+    // are entered only at leaders (few merge points keep the block code
+    // straight-line for the compiler); any other pc runs in step mode
+    // (jinterp_inj) until a leader is reached.
+    std::vector<uint8_t> leader(n + 1, 0);
+    leader[0] = 1;
+    for (uint32_t i = 0; i < n; ++i) {
+        if (code[i].op == BRA && code[i].imm < n) leader[code[i].imm] = 1;
+        if ((code[i].op == BRA || code[i].op == EXIT) && i + 1 < n) leader[i + 1] = 1;
+    }
+    // per pc: the block length if pc is a leader, else 0 (step mode's exit test)
+    o("__device__ const unsigned short kblen_%u[%u] = {", kid, n);
+    for (uint32_t i = 0; i < n; ++i) o("%u%s", leader[i] ? std::min<uint32_t>(blen[i], 0xFFFF) : 0u, i + 1 < n ? "," : "");
+    o("};\n");
     o("__device__ __noinline__ void kern_%u(const JArgs& A_, const u32 hstep, const u32 hpc, const u32 hlane, "
       "const u32 hkind, const u32 hreg, const u32 hbfm, const u32 hmask, const u32 k, const u32 cta, "
       "const u32 wic, const u32 watchdog, const u32* __restrict__ ck, const u32 ck_interval, "
-      "jfi_store* __restrict__ st_out, const u32 st_cap, JOut& out) {\n", kid);
+      "jfi_store* __restrict__ st_out, const u32 st_cap, JOut& out, u32* __restrict__ Rs, "
+      "const uint4* __restrict__ dec) {\n", kid);
     o("const JArgs A = A_;                 // kernel arguments in registers for the whole run\n");
     o("const u32 lane = threadIdx.x & 31u, lt_mask = (1u << lane) - 1u;\n");
     o("const jfi_instance in = A.inst[k];\nconst u32 cbank_len = in.cbank_len; const u32* __restrict__ cb = A.cbank + "
@@ -429,19 +444,8 @@ void gen_kernel(Src& o, const Gen& G, uint32_t kid, const fi_insn* code, uint32_
       "   conv = true; upc = pcm; amask = active; }\n"
       " const bool inA = (amask >> lane) & 1u;\n"
       " if (step >= watchdog) { fault = 3u; fault_pc = pcm; break; }\n"
-      " if (pcm >= %uu) { fault = 4u; fault_pc = pcm; break; }\n"
-      " u32 taken = 0u, exm = 0u, tgt = 0u;\n",
+      " if (pcm >= %uu) { fault = 4u; fault_pc = pcm; break; }\n",
       n);
-    // leaders: pc 0, branch targets, and the pc after every BRA / EXIT.  Blocks
-    // are entered only at leaders (few merge points keep the block code
-    // straight-line for the compiler); any other pc runs single steps until a
-    // leader is reached (after a checkpoint restart or the injection site).
-    std::vector<uint8_t> leader(n + 1, 0);
-    leader[0] = 1;
-    for (uint32_t i = 0; i < n; ++i) {
-        if (code[i].op == BRA && code[i].imm < n) leader[code[i].imm] = 1;
-        if ((code[i].op == BRA || code[i].op == EXIT) && i + 1 < n) leader[i + 1] = 1;
-    }
     // dispatch: a whole block when it fits, else one step
     o(" switch (pcm) {\n");
     for (uint32_t i = 0; i < n; ++i)
@@ -507,46 +511,26 @@ void gen_kernel(Src& o, const Gen& G, uint32_t kid, const fi_insn* code, uint32_
                   n, n);
         }
     }
-    // ---- single steps
-    o(" S_any:\n switch (pcm) {\n");
-    for (uint32_t i = 0; i < n; ++i) {
-        const fi_insn& I = code[i];
-        o("  case %u: { const bool pv = %s; const u32 pred_ = __ballot_sync(JFULL, pv); const bool ex = inA && pv; "
-          "exm = active & pred_; (void)ex;\n",
-          i, G.guard(I.guard).c_str());
-        if (I.op == BRA) {
-            o("  taken = exm; tgt = %uu;\n", I.imm);
-        } else if (I.op == EXIT) {
-            o("  if (ex) live = false; livem &= ~exm; amask &= ~exm;\n");
-        } else if (I.op == LDG || I.op == STG) {
-            o("  ");
-            G.mem(o, I, i, "step");
-        } else {
-            o("  ");
-            G.plain(o, I);
-        }
-        o("  } break;\n");
-    }
-    o("  default: break;\n }\n");
-    o(" // Sdone\n"
-      " if (taken == 0u) upc = pcm + 1u; else if (taken == active) upc = tgt;\n"
-      " else { conv = false; if (inA) pc = ((taken >> lane) & 1u) ? tgt : pcm + 1u; }\n"
-      " if (conv && (amask == 0u || upc >= npc)) { conv = false; if ((amask >> lane) & 1u) pc = upc; }\n");
-    // the transient fault (C-7, C-8), after the instruction wrote its destinations
-    o(" if (step == hstep) {\n  fired = true;\n  if (pcm != hpc || !((exm >> hlane) & 1u)) bad = true;\n"
-      "  if (lane == hlane) {\n   if (hkind == 0) {\n    switch (hreg) {\n");
-    for (uint32_t j = 0; j < NR; ++j)
-        o("     case %u: before = R%u; msk = hbfm == 3 ? before : hmask; after = before ^ msk; R%u = after; break;\n",
-          j, j, j);
-    o("     default: before = 0u; msk = hbfm == 3 ? 0u : hmask; after = msk; break;\n    }\n   } else {\n"
-      "    const u32 p_ = hreg & 7u;\n"
-      "    const u32 b_ = p_ == 0u ? Q0 : p_ == 1u ? Q1 : p_ == 2u ? Q2 : p_ == 3u ? Q3 : p_ == 4u ? Q4 : p_ == 5u ? Q5 : "
-      "p_ == 6u ? Q6 : 1u;\n    u32 m_ = hmask, a_;\n"
-      "    if (hbfm == 0 || hbfm == 1) a_ = b_ ^ 1u; else if (hbfm == 2) a_ = (m_ >> 31) & 1u; else { m_ = b_; a_ = 0u; }\n"
-      "    before = b_; msk = m_; after = a_;\n"
-      "    switch (p_) { case 0: Q0 = a_; break; case 1: Q1 = a_; break; case 2: Q2 = a_; break; case 3: Q3 = a_; break; "
-      "case 4: Q4 = a_; break; case 5: Q5 = a_; break; case 6: Q6 = a_; break; default: break; }\n   }\n  }\n }\n"
-      " ++step;\n if (step > hstep) lim = watchdog;\n}\n");
+    // ---- step mode: registers to the warp's shared-memory file, interpreter, back
+    o(" S_any: {\n");
+    for (uint32_t j = 0; j < NR; ++j) o("  Rs[%uu + lane] = R%u;%s", j * 32, j, (j % 8 == 7) ? "\n" : "");
+    o("\n  JState st_; st_.pc = pc; st_.live = live; st_.step = step; st_.livem = livem; st_.conv = conv; "
+      "st_.upc = upc; st_.amask = amask; st_.npc = npc; st_.nst = nst; st_.fault = fault; st_.fault_pc = fault_pc; "
+      "st_.before = before; st_.after = after; st_.msk = msk; st_.fired = fired; st_.bad = bad; st_.lim = lim;\n"
+      "  st_.preds = (u32)Q0 | ((u32)Q1 << 1) | ((u32)Q2 << 2) | ((u32)Q3 << 3) | ((u32)Q4 << 4) | ((u32)Q5 << 5) | "
+      "((u32)Q6 << 6);\n"
+      "  __syncwarp();\n"
+      "  const u32 done_ = jinterp_inj(A, st_, bc, Rs, dec, kblen_%u, %uu, k, cta, wic, watchdog, hstep, hpc, hlane, "
+      "hkind, hreg, hbfm, hmask, st_out, st_cap, %uu);\n"
+      "  __syncwarp();\n",
+      kid, n, NR);
+    for (uint32_t j = 0; j < NR; ++j) o("  R%u = Rs[%uu + lane];%s", j, j * 32, (j % 8 == 7) ? "\n" : "");
+    o("\n  pc = st_.pc; live = st_.live; step = st_.step; livem = st_.livem; conv = st_.conv; upc = st_.upc; "
+      "amask = st_.amask; npc = st_.npc; nst = st_.nst; fault = st_.fault; fault_pc = st_.fault_pc; "
+      "before = st_.before; after = st_.after; msk = st_.msk; fired = st_.fired; bad = st_.bad; lim = st_.lim;\n"
+      "  Q0 = st_.preds & 1u; Q1 = (st_.preds >> 1) & 1u; Q2 = (st_.preds >> 2) & 1u; Q3 = (st_.preds >> 3) & 1u; "
+      "Q4 = (st_.preds >> 4) & 1u; Q5 = (st_.preds >> 5) & 1u; Q6 = (st_.preds >> 6) & 1u;\n"
+      "  if (done_) goto finish;\n  continue;\n }\n}\n");
     o("finish:\n out.steps = step; out.fault = fault; out.fault_pc = fault_pc; out.nstore = nst;\n"
       " out.before = __shfl_sync(JFULL, before, hlane); out.after = __shfl_sync(JFULL, after, hlane);\n"
       " out.mask = __shfl_sync(JFULL, msk, hlane); out.fired = fired; out.bad = bad;\n}\n\n");
@@ -567,7 +551,10 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
       "const jfi_site* __restrict__ sites, const u32 n, jfi_inj* __restrict__ out, jfi_store* __restrict__ log, "
       "const u32 cap, const u32* ckpt, const u64* __restrict__ ck_off, const u32 ck_interval, "
       "const u32* __restrict__ order, u32* counter, u32* status) {\n"
+      " extern __shared__ u32 jsmem[];\n"
       " const u32 lane = threadIdx.x & 31u;\n"
+      " u32* Rs = jsmem + (threadIdx.x >> 5) * %uu;\n"
+      " Rs[%uu + lane] = 0u;                     // the zero row (RZ, indices >= n_regs)\n"
       " for (;;) {\n  u32 p = 0u; if (lane == 0u) p = atomicAdd(counter, 1u); p = __shfl_sync(JFULL, p, 0);\n"
       "  if (p >= n) return;\n  const u32 i = order[p]; const jfi_site S = sites[i];\n"
       "  if (S.flags & 1u) { if (lane == 0u) { jfi_inj r; r.before = r.after = r.mask = r.fault_pc = 0u; "
@@ -577,10 +564,11 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
       "  const u32 watchdog = wd > 0xFFFFFFFFull ? 0xFFFFFFFFu : (u32)wd;\n"
       "  const u32* ck = ckpt ? ckpt + ck_off[S.warp] * %uull : (const u32*)0;\n"
       "  JOut o;\n  switch (in.kernel) {\n",
-      (n_regs + 3) * 32);
+      (n_regs + 1) * 32, n_regs * 32, (n_regs + 3) * 32);
     for (uint32_t k = 0; k < n_kern; ++k)
-        o("   case %u: kern_%u(A, S.step, S.pc, S.lane, S.dst_kind, S.dst_reg, S.bfm, S.mask, S.instance, lw / wpc, lw %% wpc, watchdog, ck, ck ? ck_interval : 0u, "
-          "log + (u64)i * cap, cap, o); break;\n", k, k);
+        o("   case %u: kern_%u(A, S.step, S.pc, S.lane, S.dst_kind, S.dst_reg, S.bfm, S.mask, S.instance, lw / wpc, "
+          "lw %% wpc, watchdog, ck, ck ? ck_interval : 0u, log + (u64)i * cap, cap, o, Rs, A.dec + %uu); break;\n",
+          k, k, kern[k].code_off);
     o("   default: o.steps = 0; o.fired = false; o.bad = true; o.fault = 0; o.fault_pc = 0; o.nstore = 0; "
       "o.before = o.after = o.mask = 0; break;\n  }\n"
       "  if (lane == 0u) {\n   jfi_inj r; r.before = o.before; r.after = o.after; r.mask = o.mask; r.fault_pc = o.fault_pc;\n"
@@ -634,6 +622,7 @@ typedef CUresult (*cuModuleUnload_t)(CUmodule);
 typedef CUresult (*cuLaunchKernel_t)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned,
                                      CUstream, void**, void**);
 typedef CUresult (*cuOccupancy_t)(int*, CUfunction, int, size_t);
+typedef CUresult (*cuFuncSetAttribute_t)(CUfunction, CUfunction_attribute, int);
 
 struct Drv {
     cuModuleLoadData_t load = nullptr;
@@ -641,6 +630,7 @@ struct Drv {
     cuModuleUnload_t unload = nullptr;
     cuLaunchKernel_t launch = nullptr;
     cuOccupancy_t occ = nullptr;
+    cuFuncSetAttribute_t set_attr = nullptr;
     bool ok = false;
 };
 
@@ -654,7 +644,8 @@ Drv& drv() {
         cudaGetDriverEntryPoint("cuModuleUnload", (void**)&D.unload, cudaEnableDefault, &q);
         cudaGetDriverEntryPoint("cuLaunchKernel", (void**)&D.launch, cudaEnableDefault, &q);
         cudaGetDriverEntryPoint("cuOccupancyMaxActiveBlocksPerMultiprocessor", (void**)&D.occ, cudaEnableDefault, &q);
-        D.ok = D.load && D.get && D.unload && D.launch && D.occ;
+        cudaGetDriverEntryPoint("cuFuncSetAttribute", (void**)&D.set_attr, cudaEnableDefault, &q);
+        D.ok = D.load && D.get && D.unload && D.launch && D.occ && D.set_attr;
     });
     return D;
 }
@@ -663,7 +654,11 @@ thread_local std::string g_jit_log;
 
 }  // namespace
 
+// step mode's shared-memory register files: 4 warps x (n_regs + 1) rows x 32 lanes
+static size_t jit_smem(uint32_t n_regs) { return (size_t)4 * (n_regs + 1) * 128; }
+
 struct fi_jit {
+    size_t smem = 0;
     CUmodule mod = nullptr;
     CUfunction inject = nullptr;
     uint32_t n_regs = 0, n_code = 0;
@@ -672,6 +667,7 @@ struct fi_jit {
 };
 
 namespace fi {
+size_t aux_dec_offset(const fi_program* p);
 void launch_lpt_order(const fi_site* sites, const uint64_t* warp_off, uint32_t ck_interval, uint32_t n,
                       uint32_t* order, uint32_t* counter, cudaStream_t s);
 }
@@ -755,6 +751,13 @@ extern "C" fi_status fi_jit_build(const fi_program* p, const fi_kernel* kern_hos
     }
     j->n_regs = p->n_regs;
     j->n_code = p->n_code;
+    j->smem = jit_smem(p->n_regs);
+    if (D.set_attr(j->inject, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)j->smem) != CUDA_SUCCESS) {
+        g_jit_log = "cuFuncSetAttribute(MAX_DYNAMIC_SHARED_SIZE_BYTES) failed";
+        D.unload(j->mod);
+        delete j;
+        return FI_E_CUDA;
+    }
     j->src_bytes = src.size();
     j->cubin_bytes = cs;
     j->compile_s = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
@@ -770,12 +773,13 @@ extern "C" void fi_jit_free(fi_jit* j) {
     delete j;
 }
 
-struct JArgsHost {
+struct JArgsHost {                                   // = JArgs of jit_prelude.cuh
     const uint8_t* img;
     const uint32_t* gran;
     const fi_buffer* buf;
     const fi_instance* inst;
     const uint32_t* cbank;
+    const uint4* dec;
     uint64_t image_bytes;
 };
 
@@ -799,16 +803,20 @@ extern "C" fi_status fi_inject_jit(const fi_jit* j, const fi_program* p, const u
     int dev = 0, sms = 0, per = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    D.occ(&per, j->inject, 128, 0);
+    D.occ(&per, j->inject, 128, j->smem);
     const uint32_t grid =
         (uint32_t)std::min<uint64_t>((n + 3) / 4, (uint64_t)std::max(1, sms * std::max(1, per)));
-    JArgsHost A{image, reinterpret_cast<const uint32_t*>(p->aux)   /* granule map at aux offset 0 */, p->buf, p->inst, p->cbank, p->image_bytes};
+    JArgsHost A{image,
+                reinterpret_cast<const uint32_t*>(p->aux),   // granule map at aux offset 0
+                p->buf, p->inst, p->cbank,
+                reinterpret_cast<const uint4*>(reinterpret_cast<const char*>(p->aux) + fi::aux_dec_offset(p)),
+                p->image_bytes};
     const uint64_t* warp_off = t->warp_off;
     const uint32_t* ckpt = t->ckpt;
     const uint64_t* ck_off = t->ckpt_off;
     void* args[] = {&A, (void*)&warp_off, (void*)&sites, &n, &out, &log, &log_cap, (void*)&ckpt, (void*)&ck_off,
                     (void*)&ck_iv, &order, &counter, &dev_status};
-    const CUresult r = D.launch(j->inject, grid, 1, 1, 128, 1, 1, 0, (CUstream)s, args, nullptr);
+    const CUresult r = D.launch(j->inject, grid, 1, 1, 128, 1, 1, (unsigned)j->smem, (CUstream)s, args, nullptr);
     if (r != CUDA_SUCCESS) {
         g_jit_log = "cuLaunchKernel failed: " + std::to_string((int)r);
         return FI_E_CUDA;

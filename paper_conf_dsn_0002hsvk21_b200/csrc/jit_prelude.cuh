@@ -39,6 +39,7 @@ struct JArgs {
     const jfi_buffer* buf;
     const jfi_instance* inst;
     const u32* cbank;
+    const uint4* dec;            // pre-decoded code (fi_program_prepare), for step mode
     u64 image_bytes;
 };
 
@@ -192,4 +193,273 @@ __device__ __forceinline__ u32 jldg(const JArgs& A, JBufCache& C, u64 va, u32 k,
         else v = jld128(src);
     }
     return c;
+}
+
+// ---------------------------------------------------------------------------
+// Step-at-a-time mode of the JIT module.  Whenever a block cannot run (entry
+// off a leader, divergent groups, the injection step, the watchdog's last
+// steps) the generated code spills its registers to the warp's shared-memory
+// register file ([n_regs+1][32] words, row n_regs all zero) and this
+// interpreter runs single steps from the pre-decoded code (fi_program_prepare's
+// layout, emu.cuh) until the warp reaches a leader whose block fits again, ends
+// or faults.  Same semantics as emu.cuh's general step.
+struct JState {
+    u32 pc, live, step, livem, conv, upc, amask, npc, nst, fault, fault_pc, before, after, msk, fired, bad, lim, preds;
+};
+
+__device__ __forceinline__ bool jguard(u32 guard, u32 preds) {
+    const u32 gs = guard & 7;
+    return (((gs == 7) ? 1u : ((preds >> gs) & 1u)) ^ ((guard >> 3) & 1u)) != 0;
+}
+
+struct JRegs {                                      // this lane's column of the smem register file
+    char* Rb; u32* R; u32 zb;
+    __device__ __forceinline__ u32 rd(u32 o) const { return *reinterpret_cast<const u32*>(Rb + o); }
+    __device__ __forceinline__ u64 rd64(u32 o) const { return (u64)rd(o) | ((u64)rd(min(o + 128u, zb)) << 32); }
+    __device__ __forceinline__ void wr(u32 o, u32 v) const { if (o < zb) *reinterpret_cast<u32*>(Rb + o) = v; }
+};
+
+// one plain instruction (not BRA / EXIT / LDG / STG), all lanes together
+__device__ __forceinline__ void jexec_plain(const JRegs& F, const uint4 D, const bool ex, u32& preds, u32 lane, u32 cta,
+                                            u32 wic, const jfi_instance& in, const u32* cb) {
+    const u32 op = D.x & 0xFF, mod = (D.x >> 16) & 0xFF, pb = D.x >> 24;
+    const u32 ia = D.y & 0xFFFF, ib = D.y >> 16, ic = D.z & 0xFFFF, id = D.z >> 16;
+    const u32 imm = D.w;
+    const u32 bv = (mod & 0x80) ? imm : F.rd(ib);
+    switch (op) {
+        case 16: {                                    // FFMA
+            const float x = ju2f(F.rd(ia) ^ (mod << 31)), y = ju2f(bv ^ ((mod & 2) << 30)), z = ju2f(F.rd(ic) ^ ((mod & 4) << 29));
+            const u32 r = jfbits(__fmaf_rn(x, y, z));
+            if (ex) F.wr(id, r);
+            break;
+        }
+        case 3: if (ex) F.wr(id, bv); break;          // MOV
+        case 4: {                                     // S2R
+            u32 v = 0;
+            switch (imm) {
+                case 0: v = wic * 32 + lane; break; case 1: v = cta; break; case 2: v = in.block; break;
+                case 3: v = in.grid; break; case 4: v = lane; break; case 5: v = wic; break;
+            }
+            if (ex) F.wr(id, v);
+            break;
+        }
+        case 5: {                                     // IADD3
+            const u32 a = F.rd(ia), c = F.rd(ic);
+            const u32 x = (mod & 1) ? 0u - a : a, y = (mod & 2) ? 0u - bv : bv;
+            const u64 s = (u64)x + y + c;
+            if (ex) {
+                F.wr(id, (u32)s);
+                if (pb != 7) preds = (preds & ~(1u << pb)) | ((u32)((s >> 32) != 0) << pb);
+            }
+            break;
+        }
+        case 6: if (ex) F.wr(id, F.rd(ia) * bv + F.rd(ic)); break;      // IMAD
+        case 7: {                                     // IMAD.WIDE
+            const u32 a = F.rd(ia);
+            const u64 prod = (mod & 1) ? (u64)a * (u64)bv : (u64)((i64)(i32)a * (i64)(i32)bv);
+            const u64 r = prod + F.rd64(ic);
+            if (ex) { F.wr(id, (u32)r); F.wr(id + 128, (u32)(r >> 32)); }
+            break;
+        }
+        case 8: { const u32 v = jshf(F.rd(ia), bv, mod & 3); if (ex) F.wr(id, v); break; }     // SHF
+        case 9: {                                     // LOP3 (lut = pb)
+            const u32 a = F.rd(ia), c = F.rd(ic);
+            u32 r = 0;
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                const u32 t = ((i & 4) ? a : ~a) & ((i & 2) ? bv : ~bv) & ((i & 1) ? c : ~c);
+                r |= ((pb >> i) & 1u) ? t : 0u;
+            }
+            if (ex) F.wr(id, r);
+            break;
+        }
+        case 10: {                                    // SEL
+            const u32 p = pb & 7;
+            const bool s = (((p == 7) ? 1u : ((preds >> p) & 1u)) ^ ((pb >> 3) & 1u)) != 0;
+            if (ex) F.wr(id, s ? F.rd(ia) : bv);
+            break;
+        }
+        case 11: case 12: case 13: {                  // ISETP / FSETP / DSETP
+            bool v;
+            const u32 c = mod & 7;
+            if (op == 11) v = (mod & 8) ? jcmp_u(F.rd(ia), bv, c) : jcmp_s((i32)F.rd(ia), (i32)bv, c);
+            else if (op == 12) v = jcmp_f((double)ju2f(F.rd(ia)), (double)ju2f(F.rd(ib)), c);
+            else v = jcmp_f(ju2d(F.rd64(ia)), ju2d(F.rd64(ib)), c);
+            if (ex && pb != 7) preds = (preds & ~(1u << pb)) | ((u32)v << pb);
+            break;
+        }
+        case 14: case 15: {                           // FADD / FMUL
+            const float x = ju2f(F.rd(ia) ^ (mod << 31)), y = ju2f(bv ^ ((mod & 2) << 30));
+            const float r = op == 14 ? __fadd_rn(x, y) : __fmul_rn(x, y);
+            if (ex) F.wr(id, jfbits(r));
+            break;
+        }
+        case 17: if (ex) F.wr(id, jfmnmx(F.rd(ia), bv, mod & 1)); break;  // FMNMX
+        case 18: case 19: case 20: {                  // DADD / DMUL / DFMA
+            const double x = ju2d(F.rd64(ia) ^ ((u64)(mod & 1) << 63));
+            const double y = ju2d(F.rd64(ib) ^ ((u64)(mod & 2) << 62));
+            const double z = ju2d(F.rd64(ic) ^ ((u64)(mod & 4) << 61));
+            const double r = op == 18 ? __dadd_rn(x, y) : op == 19 ? __dmul_rn(x, y) : __fma_rn(x, y, z);
+            const u64 b = jdbits(r);
+            if (ex) { F.wr(id, (u32)b); F.wr(id + 128, (u32)(b >> 32)); }
+            break;
+        }
+        case 22: {                                    // LDC
+            const u32 w0 = imm >> 2;
+            if (ex) {
+                F.wr(id, w0 < in.cbank_len ? __ldg(&cb[w0]) : 0u);
+                if (mod & 1) F.wr(id + 128, w0 + 1 < in.cbank_len ? __ldg(&cb[w0 + 1]) : 0u);
+            }
+            break;
+        }
+        case 24: if (ex) F.wr(id, jfbits((mod & 1) ? __uint2float_rn(F.rd(ia)) : __int2float_rn((int)F.rd(ia)))); break;
+        case 25: if (ex) F.wr(id, jf2i(F.rd(ia))); break;
+        case 26: {                                    // F2F.F64.F32
+            const u64 b = jdbits((double)ju2f(F.rd(ia)));
+            if (ex) { F.wr(id, (u32)b); F.wr(id + 128, (u32)(b >> 32)); }
+            break;
+        }
+        case 27: if (ex) F.wr(id, jfbits(__double2float_rn(ju2d(F.rd64(ia))))); break;     // F2F.F32.F64
+        case 28: {                                    // SHFL: reads the source lane's register even if inactive
+            const u32 src = jshfl_src(lane, bv, mod & 3);
+            __syncwarp();
+            const u32 v = *reinterpret_cast<const u32*>(reinterpret_cast<const char*>(F.R + src) + ia);
+            __syncwarp();
+            if (ex) F.wr(id, v);
+            break;
+        }
+        case 30: {                                    // MUFU.RCP64
+            const u64 b = jdbits(__drcp_rn(ju2d(F.rd64(ia))));
+            if (ex) { F.wr(id, (u32)b); F.wr(id + 128, (u32)(b >> 32)); }
+            break;
+        }
+        case 29: {                                    // IMNMX
+            const u32 a = F.rd(ia);
+            u32 v;
+            if (mod & 8) v = (mod & 1) ? max(a, bv) : min(a, bv);
+            else v = (u32)((mod & 1) ? max((i32)a, (i32)bv) : min((i32)a, (i32)bv));
+            if (ex) F.wr(id, v);
+            break;
+        }
+        default: break;                               // NOP
+    }
+}
+
+// Injection-mode steps (EMU_INJ of emu.cuh).  Returns 1 when the warp is done
+// (finished or faulted), 0 when it stands at a leader whose block fits.
+__device__ __noinline__ u32 jinterp_inj(const JArgs& A, JState& S, JBufCache& bc, u32* R, const uint4* __restrict__ dec,
+                                        const unsigned short* __restrict__ blen, const u32 code_len, const u32 k,
+                                        const u32 cta, const u32 wic, const u32 watchdog, const u32 hstep, const u32 hpc,
+                                        const u32 hlane, const u32 hkind, const u32 hreg, const u32 hbfm,
+                                        const u32 hmask, jfi_store* __restrict__ st_out, const u32 st_cap,
+                                        const u32 zr) {
+    const u32 lane = threadIdx.x & 31, lt_mask = (1u << lane) - 1u;
+    const JRegs F{reinterpret_cast<char*>(R + lane), R, zr * 128};
+    const jfi_instance in = A.inst[k];
+    const u32* cb = A.cbank + in.cbank_off;
+    bool live = S.live != 0, conv = S.conv != 0;
+    u32 pc = S.pc, step = S.step, livem = S.livem, upc = S.upc, amask = S.amask, npc = S.npc, nst = S.nst;
+    u32 preds = S.preds, lim = S.lim;
+    u32 done = 0;
+    for (;;) {
+        if (!livem) { done = 1; break; }
+        u32 pcm, active;
+        if (conv) { pcm = upc; active = amask; }
+        else {
+            pcm = __reduce_min_sync(JFULL, live ? pc : 0xFFFFFFFFu);
+            active = __ballot_sync(JFULL, live && pc == pcm);
+            npc = active == livem ? 0xFFFFFFFFu : __reduce_min_sync(JFULL, (live && pc != pcm) ? pc : 0xFFFFFFFFu);
+            conv = true; upc = pcm; amask = active;
+        }
+        if (step >= watchdog) { S.fault = 3; S.fault_pc = pcm; done = 1; break; }
+        if (pcm >= code_len) { S.fault = 4; S.fault_pc = pcm; done = 1; break; }
+        const u32 bl = blen[pcm];                     // 0 unless pcm is a leader
+        if (bl && pcm + bl <= npc && step + bl <= lim) break;      // the generated block runs from here
+        const uint4 D = __ldg(&dec[pcm]);
+        const u32 op = D.x & 0xFF, guard = (D.x >> 8) & 0xFF, mod = (D.x >> 16) & 0xFF;
+        const u32 ia = D.y & 0xFFFF, ib = D.y >> 16, id = D.z >> 16, imm = D.w;
+        const bool act = (active >> lane) & 1u;
+        const bool pv = guard == 7 ? true : jguard(guard, preds);
+        const u32 pred = guard == 7 ? JFULL : __ballot_sync(JFULL, pv);
+        const bool ex = act && pv;
+        const u32 exm = active & pred;
+        u32 taken = 0;
+        if (op == 1) {                                // EXIT
+            if (ex) live = false;
+            livem &= ~exm;
+            amask &= ~exm;
+        } else if (op == 2) {                         // BRA
+            taken = exm;
+        } else if (op == 21 || op == 23) {            // LDG / STG
+            const u32 lw = (mod & 3) > 2 ? 2 : (mod & 3), nw = 1u << lw, w = 4u << lw;
+            const u64 va = F.rd64(ia) + (u64)(i64)(i32)imm;
+            bool zero = false;
+            const u32 c = ex ? jcheck(A, bc, va, w, k, &zero) : 0u;
+            if (__ballot_sync(JFULL, c != 0u)) {      // memory fault: DUE (C-9); the step has no effect
+                S.fault = __ballot_sync(JFULL, c == 1u) ? 1u : 2u;
+                S.fault_pc = pcm;
+                done = 1;
+                break;
+            }
+            if (op == 21) {
+                if (ex) {
+                    uint4 v = make_uint4(0, 0, 0, 0);
+                    if (!zero) {
+                        const u8* src = A.img + (va - JVA_BASE);
+                        if (lw == 0) v.x = jld32(src);
+                        else if (lw == 1) { const uint2 t = jld64(src); v.x = t.x; v.y = t.y; }
+                        else v = jld128(src);
+                    }
+                    F.wr(id, v.x);
+                    if (lw >= 1) F.wr(id + 128, v.y);
+                    if (lw >= 2) { F.wr(id + 256, v.z); F.wr(id + 384, v.w); }
+                }
+            } else if (step > hstep) {                // stores after the site are logged
+                u32 v[4];
+#pragma unroll
+                for (int i = 0; i < 4; ++i) v[i] = (u32)i < nw ? F.rd(min(ib + 128u * i, F.zb)) : 0u;
+                if (ex) {
+                    const u32 idx = __popc(exm & lt_mask) * nw;
+                    for (u32 i = 0; i < nw; ++i) {
+                        const u32 e = nst + idx + i;
+                        if (e < st_cap) { jfi_store s_; s_.va = va + 4 * i; s_.value = v[i]; s_.step = step; st_out[e] = s_; }
+                    }
+                }
+                nst += __popc(exm) * nw;
+            }
+        } else {
+            jexec_plain(F, D, ex, preds, lane, cta, wic, in, cb);
+        }
+        if (taken == 0) upc = pcm + 1;
+        else if (taken == active) upc = imm;
+        else { conv = false; if (act) pc = ((taken >> lane) & 1u) ? imm : pcm + 1; }
+        if (conv && (amask == 0 || upc >= npc)) { conv = false; if ((amask >> lane) & 1u) pc = upc; }
+        if (step == hstep) {                          // the transient fault (C-7, C-8)
+            S.fired = 1;
+            if (pcm != hpc || !((exm >> hlane) & 1u)) S.bad = 1;
+            if (lane == hlane) {
+                if (hkind == 0) {
+                    const u32 ri = min(hreg, zr) * 128;
+                    const u32 b = F.rd(ri);
+                    const u32 m = hbfm == 3 ? b : hmask;
+                    S.before = b; S.msk = m; S.after = b ^ m;
+                    F.wr(ri, S.after);
+                } else {
+                    const u32 p = hreg & 7;
+                    const u32 b = (p == 7) ? 1u : ((preds >> p) & 1u);
+                    u32 m = hmask, a;
+                    if (hbfm == 0 || hbfm == 1) a = b ^ 1u;
+                    else if (hbfm == 2) a = (m >> 31) & 1u;
+                    else { m = b; a = 0u; }
+                    S.before = b; S.msk = m; S.after = a;
+                    if (p != 7) preds = (preds & ~(1u << p)) | (a << p);
+                }
+            }
+        }
+        ++step;
+        if (step > hstep) lim = watchdog;
+    }
+    S.pc = pc; S.live = live; S.step = step; S.livem = livem; S.conv = conv; S.upc = upc; S.amask = amask;
+    S.npc = npc; S.nst = nst; S.preds = preds; S.lim = lim;
+    return done;
 }
