@@ -350,19 +350,28 @@ fi_status fi_inject_permanent_batched(const fi_program* p, const uint8_t* image,
  * returns the generated source (buf may be NULL; returns the bytes needed, 0 on
  * bad arguments). */
 typedef struct fi_jit fi_jit;
-fi_status fi_jit_build(const fi_program* p, const fi_kernel* kern_host, fi_jit** out);
+#define FI_JIT_INJECT 1u                            /* k_inject_jit (fi_inject_jit) */
+#define FI_JIT_GOLDEN 2u                            /* golden passes (fi_golden_lengths_jit, fi_golden_trace_jit) */
+fi_status fi_jit_build(const fi_program* p, const fi_kernel* kern_host, uint32_t modes, fi_jit** out);
 void fi_jit_free(fi_jit* j);
 double fi_jit_compile_seconds(const fi_jit* j);
 const char* fi_jit_log(void);
 fi_status fi_jit_compile_check(const fi_insn* code_host, uint32_t n_code, const fi_kernel* kern_host, uint32_t n_kern,
-                               uint32_t n_regs, size_t* cubin_bytes);
+                               uint32_t n_regs, uint32_t modes, size_t* cubin_bytes);
 size_t fi_jit_source(const fi_insn* code_host, uint32_t n_code, const fi_kernel* kern_host, uint32_t n_kern,
-                     uint32_t n_regs, char* buf, size_t buf_bytes);
+                     uint32_t n_regs, uint32_t modes, char* buf, size_t buf_bytes);
 /* K4 on the JIT module `j` built for p: same arguments, scratch, scheduling and
  * results as fi_inject (bit-identical outputs), asynchronous on `stream`. */
 fi_status fi_inject_jit(const fi_jit* j, const fi_program* p, const uint8_t* image, const fi_trace* t,
                         const fi_site* sites, uint32_t n, fi_inj* out, fi_store* log, uint32_t log_cap, void* ws,
                         size_t ws_bytes, uint32_t* dev_status, void* stream);
+/* The golden passes on a module built with FI_JIT_GOLDEN: same arguments and
+ * results (trace records, store log, checkpoints, final image, lengths) as
+ * fi_golden_lengths / fi_golden_trace, bit for bit. */
+fi_status fi_golden_lengths_jit(const fi_jit* j, const fi_program* p, uint8_t* image, uint64_t* warp_len,
+                                uint64_t* warp_nstore, uint32_t* dev_status, void* stream);
+fi_status fi_golden_trace_jit(const fi_jit* j, const fi_program* p, const uint8_t* image, const fi_trace* t,
+                              uint32_t* dev_status, void* stream);
 
 /* Table II parameter file, one parameter per line in Table II order
  * [PAPER.md:88]: arch state id, bit-flip model, kernel name, kernel count,

@@ -162,6 +162,7 @@ __global__ void k_ckpt_counts(const uint64_t* warp_len, uint32_t n, uint32_t int
 
 size_t golden_smem(uint32_t n_regs) { return emu_smem(n_regs); }
 size_t aux_dec_offset(const fi_program* p) { return aux_layout(p->image_bytes, p->n_code, p->n_inst).dec; }
+size_t aux_ins_offset(const fi_program* p) { return aux_layout(p->image_bytes, p->n_code, p->n_inst).ins; }
 
 }  // namespace fi
 

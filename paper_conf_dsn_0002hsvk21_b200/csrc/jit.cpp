@@ -288,10 +288,20 @@ struct Gen {
     }
 
     // LDG / STG.  `stepx` = this instruction's step.
+    uint32_t mode = 0;                               // JM_INJ / JM_LEN / JM_TRACE of jit_prelude.cuh
+    // trace record of the instruction at pc (App. A.3): written only in JM_TRACE
+    void rec(Src& o, const fi_insn& I, uint32_t pc, const char* stepx, const char* pv) const {
+        if (mode != 2) return;
+        const uint32_t insw = pc | ((uint32_t)I.op << 16) | (fi::groupmask_of(I.op, I.d0, I.d1, I.mod) << 24);
+        o("{ const u32 s_ = %s; const u32 pr_ = %s; if ((s_ & 31u) == lane) recbuf = make_uint4(k, %uu, amask, pr_); "
+          "if ((s_ & 31u) == 31u) rec_out[s_ - 31u + lane] = recbuf; } ",
+          stepx, I.guard == 7 ? "JFULL" : (std::string("__ballot_sync(JFULL, ") + pv + ")").c_str(), insw);
+    }
     void mem(Src& o, const fi_insn& I, uint32_t pc, const char* stepx) const {
         using namespace fi;
         const uint32_t lw = (I.mod & 3) > 2 ? 2 : (I.mod & 3), nw = 1u << lw;
         o("{ const bool pv = %s; const bool ex = inA && pv; ", guard(I.guard).c_str());
+        rec(o, I, pc, stepx, "pv");
         o("const u64 va = %s + (u64)(i64)(i32)%s; ", R64(I.a).c_str(), hex(I.imm).c_str());
         if (I.op == LDG) {
             o("uint4 v_; const u32 c_ = jldg<%uu>(A, bc, va, k, ex, v_); ", lw);
@@ -305,12 +315,27 @@ struct Gen {
               "const u32 c_ = ex ? jcheck(A, bc, va, %uu, k, &z_) : 0u; ", 4u << lw);
             o("if (__ballot_sync(JFULL, c_ != 0u)) { fault = __ballot_sync(JFULL, c_ == 1u) ? 1u : 2u; fault_pc = %uu; "
               "step = %s; goto finish; } ", pc, stepx);
-            o("const u32 sst_ = %s; if (sst_ > hstep) { if (ex) { const u32 idx_ = __popc(exm_ & lt_mask) * %uu; ",
-              stepx, nw);
-            for (uint32_t q = 0; q < nw; ++q)
-                o("if (nst + idx_ + %uu < st_cap) { jfi_store e_; e_.va = va + %uu; e_.value = %s; e_.step = sst_; "
-                  "st_out[nst + idx_ + %uu] = e_; } ",
-                  q, 4 * q, (I.b == kRZ ? std::string("0u") : R(I.b + q)).c_str(), q);
+            if (mode == 1) {                           // golden pass 1: into the image
+                o("if (ex) { u8* d_ = img_w + (va - JVA_BASE); ");
+                if (lw == 0) o("*reinterpret_cast<u32*>(d_) = %s; ", R(I.b).c_str());
+                else if (lw == 1) o("*reinterpret_cast<uint2*>(d_) = make_uint2(%s, %s); ", R(I.b).c_str(), R(I.b + 1).c_str());
+                else
+                    o("*reinterpret_cast<uint4*>(d_) = make_uint4(%s, %s, %s, %s); ", R(I.b).c_str(), R(I.b + 1).c_str(),
+                      R(I.b + 2).c_str(), R(I.b + 3).c_str());
+                o("} nst += __popc(exm_) * %uu; }\n", nw);
+                return;
+            }
+            o("const u32 sst_ = %s; if (%s) { if (ex) { const u32 idx_ = __popc(exm_ & lt_mask) * %uu; ",
+              stepx, mode == 2 ? "true" : "sst_ > hstep", nw);
+            for (uint32_t q = 0; q < nw; ++q) {
+                if (mode == 2)
+                    o("{ jfi_store e_; e_.va = va + %uu; e_.value = %s; e_.step = sst_; st_out[nst + idx_ + %uu] = e_; } ",
+                      4 * q, R(I.b + q).c_str(), q);
+                else
+                    o("if (nst + idx_ + %uu < st_cap) { jfi_store e_; e_.va = va + %uu; e_.value = %s; e_.step = sst_; "
+                      "st_out[nst + idx_ + %uu] = e_; } ",
+                      q, 4 * q, R(I.b + q).c_str(), q);
+            }
             o("} nst += __popc(exm_) * %uu; } }\n", nw);
         }
     }
@@ -322,8 +347,9 @@ struct Gen {
         o(" { // LDG batch %u..%u\n", i0, i0 + m - 1);
         for (uint32_t j = 0; j < m; ++j) {
             const fi_insn& I = code[i0 + j];
-            o("  const bool ex%u = inA && %s; const u64 va%u = %s + (u64)(i64)(i32)%s; bool z%u = false; u32 c%u = 0u;\n",
-              j, guard(I.guard).c_str(), j, R64(I.a).c_str(), hex(I.imm).c_str(), j, j);
+            o("  const bool pv%u = %s; const bool ex%u = inA && pv%u; const u64 va%u = %s + (u64)(i64)(i32)%s; "
+              "bool z%u = false; u32 c%u = 0u;\n",
+              j, guard(I.guard).c_str(), j, j, j, R64(I.a).c_str(), hex(I.imm).c_str(), j, j);
         }
         // fast path: every executing lane hits its buffer cache (no table lookups, no
         // cache updates); otherwise the full checks in program order
@@ -348,6 +374,12 @@ struct Gen {
               "fault_pc = %uu; step = step + (%uu - pcm); goto finish; }\n",
               j, j, i0 + j, i0 + j);
         o("  }\n");
+        for (uint32_t j = 0; j < m; ++j) {
+            char sx[64], pvn[16];
+            std::snprintf(sx, sizeof sx, "step + (%uu - pcm)", i0 + j);
+            std::snprintf(pvn, sizeof pvn, "pv%u", j);
+            if (mode == 2) { o("  "); rec(o, code[i0 + j], i0 + j, sx, pvn); o("\n"); }
+        }
         // loads straight into the destination registers (predicated, program order)
         for (uint32_t j = 0; j < m; ++j) {
             const fi_insn& I = code[i0 + j];
@@ -387,9 +419,14 @@ static uint32_t ldg_batch_len(const fi_insn* code, uint32_t n, uint32_t i0, cons
 }
 
 // Generate the device function of one static kernel (EMU_INJ mode).
-void gen_kernel(Src& o, const Gen& G, uint32_t kid, const fi_insn* code, uint32_t n) {
+// Generate the device function of one static kernel in mode `mode` (JM_INJ,
+// JM_LEN, JM_TRACE); `blen`/leader tables are emitted once (with_tables).
+void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32_t n, uint32_t mode, bool with_tables) {
     using namespace fi;
+    Gen G = G0;
+    G.mode = mode;
     const uint32_t NR = G.NR;
+    static const char* const mname[] = {"inj", "len", "trace"};
     // block length from each pc: to the next BRA/EXIT inclusive, or the code end
     std::vector<uint32_t> blen(n);
     for (int64_t i = (int64_t)n - 1; i >= 0; --i) {
@@ -407,14 +444,19 @@ void gen_kernel(Src& o, const Gen& G, uint32_t kid, const fi_insn* code, uint32_
         if ((code[i].op == BRA || code[i].op == EXIT) && i + 1 < n) leader[i + 1] = 1;
     }
     // per pc: the block length if pc is a leader, else 0 (step mode's exit test)
-    o("__device__ const unsigned short kblen_%u[%u] = {", kid, n);
-    for (uint32_t i = 0; i < n; ++i) o("%u%s", leader[i] ? std::min<uint32_t>(blen[i], 0xFFFF) : 0u, i + 1 < n ? "," : "");
-    o("};\n");
-    o("__device__ __noinline__ void kern_%u(const JArgs& A_, const u32 hstep, const u32 hpc, const u32 hlane, "
+    if (with_tables) {
+        o("__device__ const unsigned short kblen_%u[%u] = {", kid, n);
+        for (uint32_t i = 0; i < n; ++i)
+            o("%u%s", leader[i] ? std::min<uint32_t>(blen[i], 0xFFFF) : 0u, i + 1 < n ? "," : "");
+        o("};\n");
+    }
+    o("__device__ __noinline__ void kern_%u_%s(const JArgs& A_, const u32 hstep, const u32 hpc, const u32 hlane, "
       "const u32 hkind, const u32 hreg, const u32 hbfm, const u32 hmask, const u32 k, const u32 cta, "
-      "const u32 wic, const u32 watchdog, const u32* __restrict__ ck, const u32 ck_interval, "
+      "const u32 wic, const u32 watchdog, u32* __restrict__ ck, const u32 ck_interval, "
       "jfi_store* __restrict__ st_out, const u32 st_cap, JOut& out, u32* __restrict__ Rs, "
-      "const uint4* __restrict__ dec) {\n", kid);
+      "const uint4* __restrict__ dec, const u32* __restrict__ ins, u8* __restrict__ img_w, "
+      "uint4* __restrict__ rec_out) {\n", kid, mname[mode]);
+    o("(void)img_w; (void)rec_out; (void)ins;\n");
     o("const JArgs A = A_;                 // kernel arguments in registers for the whole run\n");
     o("const u32 lane = threadIdx.x & 31u, lt_mask = (1u << lane) - 1u;\n");
     o("const jfi_instance in = A.inst[k];\nconst u32 cbank_len = in.cbank_len; const u32* __restrict__ cb = A.cbank + "
@@ -423,8 +465,8 @@ void gen_kernel(Src& o, const Gen& G, uint32_t kid, const fi_insn* code, uint32_
     o("\nconst u32 nl_ = in.block - wic * 32u; bool live = lane < (nl_ > 32u ? 32u : nl_);\n");
     o("u32 pc = 0u, step = 0u; bool Q0 = false, Q1 = false, Q2 = false, Q3 = false, Q4 = false, Q5 = false, "
       "Q6 = false;\n");
-    o("if (ck) {\n  const u32 c_ = hstep / ck_interval; const u32* __restrict__ src = ck + (u64)c_ * %uu;\n",
-      (NR + 3) * 32);
+    o("if (%s) {\n  const u32 c_ = hstep / ck_interval; const u32* __restrict__ src = ck + (u64)c_ * %uu;\n",
+      mode == 0 ? "ck" : "false", (NR + 3) * 32);
     for (uint32_t j = 0; j < NR; ++j) o("  R%u = __ldg(&src[%uu + lane]);\n", j, j * 32);
     o("  pc = __ldg(&src[%uu + lane]); const u32 pw_ = __ldg(&src[%uu + lane]); live = __ldg(&src[%uu + lane]) != 0u; "
       "step = c_ * ck_interval;\n  Q0 = pw_ & 1u; Q1 = (pw_ >> 1) & 1u; Q2 = (pw_ >> 2) & 1u; Q3 = (pw_ >> 3) & 1u; "
@@ -434,16 +476,27 @@ void gen_kernel(Src& o, const Gen& G, uint32_t kid, const fi_insn* code, uint32_
     o("\n}\n");
     o("u32 livem = __ballot_sync(JFULL, live);\nbool conv = false; u32 upc = 0u, amask = 0u, npc = 0xFFFFFFFFu;\n"
       "u32 nst = 0u, fault = 0u, fault_pc = 0u, before = 0u, after = 0u, msk = 0u; bool fired = false, bad = false;\n"
-      "JBufCache bc;\n"
-      "// blocks run only within [step, lim): lim = the watchdog, or the injection step while it is pending\n"
-      "u32 lim = (hstep >= step && hstep < watchdog) ? hstep : watchdog;\n");
+      "JBufCache bc; uint4 recbuf = make_uint4(0u, 0u, 0u, 0u); (void)recbuf;\n"
+      "// blocks run only within [step, lim): lim = the watchdog, or the injection step while it is pending,\n"
+      "// or the next checkpoint step (golden trace pass)\n"
+      "u32 lim = %s;\n", mode == 0 ? "(hstep >= step && hstep < watchdog) ? hstep : watchdog" : "watchdog");
     o("for (;;) {\n if (!livem) break;\n u32 pcm, active;\n"
       " if (conv) { pcm = upc; active = amask; }\n"
       " else { pcm = __reduce_min_sync(JFULL, live ? pc : 0xFFFFFFFFu); active = __ballot_sync(JFULL, live && pc == pcm);\n"
       "   npc = active == livem ? 0xFFFFFFFFu : __reduce_min_sync(JFULL, (live && pc != pcm) ? pc : 0xFFFFFFFFu);\n"
       "   conv = true; upc = pcm; amask = active; }\n"
-      " const bool inA = (amask >> lane) & 1u;\n"
-      " if (step >= watchdog) { fault = 3u; fault_pc = pcm; break; }\n"
+      " const bool inA = (amask >> lane) & 1u;\n");
+    if (mode == 2) {                                  // golden checkpoint every ck_interval steps (from registers)
+        o(" if (ck) {\n  if (step %% ck_interval == 0u) {\n   u32* dst_ = ck + (u64)(step / ck_interval) * %uu;\n",
+          (NR + 3) * 32);
+        for (uint32_t j = 0; j < NR; ++j) o("   dst_[%uu + lane] = R%u;%s", j * 32, j, (j % 8 == 7) ? "\n" : "");
+        o("\n   dst_[%uu + lane] = live ? (inA ? upc : pc) : 0u;\n"
+          "   dst_[%uu + lane] = (u32)Q0 | ((u32)Q1 << 1) | ((u32)Q2 << 2) | ((u32)Q3 << 3) | ((u32)Q4 << 4) | "
+          "((u32)Q5 << 5) | ((u32)Q6 << 6);\n   dst_[%uu + lane] = live ? 1u : 0u;\n  }\n"
+          "  lim = min(watchdog, (step / ck_interval + 1u) * ck_interval);\n }\n",
+          NR * 32, NR * 32 + 32, NR * 32 + 64);
+    }
+    o(" if (step >= watchdog) { fault = 3u; fault_pc = pcm; break; }\n"
       " if (pcm >= %uu) { fault = 4u; fault_pc = pcm; break; }\n",
       n);
     // dispatch: a whole block when it fits, else one step
@@ -486,23 +539,28 @@ void gen_kernel(Src& o, const Gen& G, uint32_t kid, const fi_insn* code, uint32_
                               blen[L], L, L);
                 return b;
             };
-            o(" { const bool pv = %s; const u32 exm_ = amask & __ballot_sync(JFULL, pv); step += %uu - pcm;\n"
+            o(" { const bool pv = %s; ", G.guard(I.guard).c_str());
+            G.rec(o, I, i, stepx, "pv");
+            o("const u32 exm_ = amask & __ballot_sync(JFULL, pv); step += %uu - pcm;\n"
               "   if (exm_ == 0u) { %supc = %uu; } else if (exm_ == amask) { %supc = %uu; }\n"
               "   else { conv = false; if (inA) pc = ((exm_ >> lane) & 1u) ? %uu : %uu; }\n"
               "   if (conv && (amask == 0u || upc >= npc)) { conv = false; if ((amask >> lane) & 1u) pc = upc; }\n"
               "   continue; }\n",
-              G.guard(I.guard).c_str(), i + 1, chain(i + 1).c_str(), i + 1, chain(I.imm).c_str(), I.imm, I.imm, i + 1);
+              i + 1, chain(i + 1).c_str(), i + 1, chain(I.imm).c_str(), I.imm, I.imm, i + 1);
         } else if (I.op == EXIT) {
-            o(" { const bool pv = %s; const u32 exm_ = amask & __ballot_sync(JFULL, pv); step += %uu - pcm;\n"
+            o(" { const bool pv = %s; ", G.guard(I.guard).c_str());
+            G.rec(o, I, i, stepx, "pv");
+            o("const u32 exm_ = amask & __ballot_sync(JFULL, pv); step += %uu - pcm;\n"
               "   if (inA && pv) live = false; livem &= ~exm_; amask &= ~exm_; upc = %uu;\n"
               "   if (conv && (amask == 0u || upc >= npc)) { conv = false; if ((amask >> lane) & 1u) pc = upc; }\n"
               "   continue; }\n",
-              G.guard(I.guard).c_str(), i + 1, i + 1);
+              i + 1, i + 1);
         } else {
             if (I.op == LDG || I.op == STG) {
                 G.mem(o, I, i, stepx);
             } else {
-                o(" { const bool ex = inA && %s; ", G.guard(I.guard).c_str());
+                o(" { const bool pv = %s; const bool ex = inA && pv; (void)pv; ", G.guard(I.guard).c_str());
+                G.rec(o, I, i, stepx, "pv");
                 G.plain(o, I);
                 o(" }\n");
             }
@@ -518,32 +576,44 @@ void gen_kernel(Src& o, const Gen& G, uint32_t kid, const fi_insn* code, uint32_
       "st_.upc = upc; st_.amask = amask; st_.npc = npc; st_.nst = nst; st_.fault = fault; st_.fault_pc = fault_pc; "
       "st_.before = before; st_.after = after; st_.msk = msk; st_.fired = fired; st_.bad = bad; st_.lim = lim;\n"
       "  st_.preds = (u32)Q0 | ((u32)Q1 << 1) | ((u32)Q2 << 2) | ((u32)Q3 << 3) | ((u32)Q4 << 4) | ((u32)Q5 << 5) | "
-      "((u32)Q6 << 6);\n"
+      "((u32)Q6 << 6); st_.recbuf = recbuf;\n"
       "  __syncwarp();\n"
-      "  const u32 done_ = jinterp_inj(A, st_, bc, Rs, dec, kblen_%u, %uu, k, cta, wic, watchdog, hstep, hpc, hlane, "
-      "hkind, hreg, hbfm, hmask, st_out, st_cap, %uu);\n"
+      "  const u32 done_ = jinterp<%u>(A, st_, bc, Rs, dec, kblen_%u, %uu, k, cta, wic, watchdog, hstep, hpc, hlane, "
+      "hkind, hreg, hbfm, hmask, st_out, st_cap, %uu, img_w, rec_out, ck, ck_interval, ins);\n"
       "  __syncwarp();\n",
-      kid, n, NR);
+      mode, kid, n, NR);
     for (uint32_t j = 0; j < NR; ++j) o("  R%u = Rs[%uu + lane];%s", j, j * 32, (j % 8 == 7) ? "\n" : "");
     o("\n  pc = st_.pc; live = st_.live; step = st_.step; livem = st_.livem; conv = st_.conv; upc = st_.upc; "
       "amask = st_.amask; npc = st_.npc; nst = st_.nst; fault = st_.fault; fault_pc = st_.fault_pc; "
-      "before = st_.before; after = st_.after; msk = st_.msk; fired = st_.fired; bad = st_.bad; lim = st_.lim;\n"
+      "before = st_.before; after = st_.after; msk = st_.msk; fired = st_.fired; bad = st_.bad; lim = st_.lim; "
+      "recbuf = st_.recbuf;\n"
       "  Q0 = st_.preds & 1u; Q1 = (st_.preds >> 1) & 1u; Q2 = (st_.preds >> 2) & 1u; Q3 = (st_.preds >> 3) & 1u; "
       "Q4 = (st_.preds >> 4) & 1u; Q5 = (st_.preds >> 5) & 1u; Q6 = (st_.preds >> 6) & 1u;\n"
       "  if (done_) goto finish;\n  continue;\n }\n}\n");
-    o("finish:\n out.steps = step; out.fault = fault; out.fault_pc = fault_pc; out.nstore = nst;\n"
+    if (mode == 2) o("finish:\n { const u32 rem_ = step & 31u; if (rem_ && lane < rem_) rec_out[step - rem_ + lane] = recbuf; }\n");
+    else o("finish:\n");
+    o(" out.steps = step; out.fault = fault; out.fault_pc = fault_pc; out.nstore = nst;\n"
       " out.before = __shfl_sync(JFULL, before, hlane); out.after = __shfl_sync(JFULL, after, hlane);\n"
       " out.mask = __shfl_sync(JFULL, msk, hlane); out.fired = fired; out.bad = bad;\n}\n\n");
 }
 
-std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern, uint32_t n_regs) {
+std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern, uint32_t n_regs, uint32_t modes) {
     // resident 128-thread CTAs per SM the register budget targets (3: <= 168 registers)
     uint32_t min_blocks = 3;
     if (const char* e = std::getenv("FI_JIT_MIN_BLOCKS")) min_blocks = (uint32_t)std::max(1, std::atoi(e));
     Src o;
     o.s = kPrelude;
     Gen G{n_regs};
-    for (uint32_t k = 0; k < n_kern; ++k) gen_kernel(o, G, k, code + kern[k].code_off, kern[k].code_len);
+    for (uint32_t k = 0; k < n_kern; ++k) {
+        bool tables = true;
+        if (modes & FI_JIT_INJECT) { gen_kernel(o, G, k, code + kern[k].code_off, kern[k].code_len, 0, tables); tables = false; }
+        if (modes & FI_JIT_GOLDEN) {
+            gen_kernel(o, G, k, code + kern[k].code_off, kern[k].code_len, 1, tables);
+            gen_kernel(o, G, k, code + kern[k].code_off, kern[k].code_len, 2, false);
+        }
+    }
+    const uint32_t rs = (n_regs + 1) * 32, zrow = n_regs * 32, ckw = (n_regs + 3) * 32;
+    if (modes & FI_JIT_INJECT) {
     // K4 on the generated kernels: persistent warps over the LPT-ordered replicas
     // (same scheduling and outputs as inject.cu's k_inject)
     o("extern \"C\" __global__ void __launch_bounds__(128, %u) k_inject_jit(", min_blocks);
@@ -562,13 +632,14 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
       "  const jfi_instance in = A.inst[S.instance]; const u32 wpc = (in.block + 31u) / 32u, lw = S.warp - in.warp_begin;\n"
       "  const u64 L = warp_off[S.warp + 1] - warp_off[S.warp]; const u64 wd = 10ull * L + 1024ull;\n"
       "  const u32 watchdog = wd > 0xFFFFFFFFull ? 0xFFFFFFFFu : (u32)wd;\n"
-      "  const u32* ck = ckpt ? ckpt + ck_off[S.warp] * %uull : (const u32*)0;\n"
+      "  u32* ck = ckpt ? (u32*)ckpt + ck_off[S.warp] * %uull : (u32*)0;\n"
       "  JOut o;\n  switch (in.kernel) {\n",
-      (n_regs + 1) * 32, n_regs * 32, (n_regs + 3) * 32);
+      rs, zrow, ckw);
     for (uint32_t k = 0; k < n_kern; ++k)
-        o("   case %u: kern_%u(A, S.step, S.pc, S.lane, S.dst_kind, S.dst_reg, S.bfm, S.mask, S.instance, lw / wpc, "
-          "lw %% wpc, watchdog, ck, ck ? ck_interval : 0u, log + (u64)i * cap, cap, o, Rs, A.dec + %uu); break;\n",
-          k, k, kern[k].code_off);
+        o("   case %u: kern_%u_inj(A, S.step, S.pc, S.lane, S.dst_kind, S.dst_reg, S.bfm, S.mask, S.instance, lw / wpc, "
+          "lw %% wpc, watchdog, ck, ck ? ck_interval : 0u, log + (u64)i * cap, cap, o, Rs, A.dec + %uu, A.ins + %uu, "
+          "(u8*)0, (uint4*)0); break;\n",
+          k, k, kern[k].code_off, kern[k].code_off);
     o("   default: o.steps = 0; o.fired = false; o.bad = true; o.fault = 0; o.fault_pc = 0; o.nstore = 0; "
       "o.before = o.after = o.mask = 0; break;\n  }\n"
       "  if (lane == 0u) {\n   jfi_inj r; r.before = o.before; r.after = o.after; r.mask = o.mask; r.fault_pc = o.fault_pc;\n"
@@ -576,6 +647,46 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
       "   out[i] = r;\n   if (!o.fired || o.bad) atomicOr(status, 1u << 6);\n"
       "   const u32 start = ck ? S.step / ck_interval * ck_interval : 0u;\n"
       "   atomicAdd((unsigned long long*)(counter + 2), (unsigned long long)(o.steps - start));\n  }\n  __syncwarp();\n }\n}\n");
+    }
+    if (modes & FI_JIT_GOLDEN) {
+        // golden pass 1 (one launch per instance k, golden.cu k_golden_len) and pass 2
+        // (every warp in one launch, golden.cu k_golden_trace) on the generated kernels
+        o("extern \"C\" __global__ void __launch_bounds__(128, %u) k_golden_len_jit(const JArgs A, const u32 k, "
+          "u8* img_w, u64* warp_len, u64* warp_nst, u32* status) {\n"
+          " extern __shared__ u32 jsmem[];\n const u32 lane = threadIdx.x & 31u;\n"
+          " u32* Rs = jsmem + (threadIdx.x >> 5) * %uu;\n Rs[%uu + lane] = 0u;\n"
+          " const jfi_instance in = A.inst[k];\n const u32 lw = blockIdx.x * 4u + (threadIdx.x >> 5);\n"
+          " if (lw >= in.warp_end - in.warp_begin) return;\n const u32 wpc = (in.block + 31u) / 32u;\n"
+          " JOut o;\n switch (in.kernel) {\n",
+          min_blocks, rs, zrow);
+        for (uint32_t k = 0; k < n_kern; ++k)
+            o("  case %u: kern_%u_len(A, 0xFFFFFFFFu, 0u, 0u, 0u, 0u, 0u, 0u, k, lw / wpc, lw %% wpc, 0xFFFFFFFFu, (u32*)0, "
+              "0u, (jfi_store*)0, 0u, o, Rs, A.dec + %uu, A.ins + %uu, img_w, (uint4*)0); break;\n",
+              k, k, kern[k].code_off, kern[k].code_off);
+        o("  default: o.steps = 0; o.fault = 9; o.nstore = 0; break;\n }\n"
+          " if (lane == 0u) { warp_len[in.warp_begin + lw] = o.steps; warp_nst[in.warp_begin + lw] = o.nstore; "
+          "if (o.fault) atomicOr(status, 1u << 4); }\n}\n");
+        o("extern \"C\" __global__ void __launch_bounds__(128, %u) k_golden_trace_jit(const JArgs A, const u32 n_warps, "
+          "const u64* __restrict__ warp_off, const u64* __restrict__ gst_off, uint4* rec, jfi_store* gst, u32* ckpt, "
+          "const u64* __restrict__ ck_off, const u32 ck_interval, u32* status) {\n"
+          " extern __shared__ u32 jsmem[];\n const u32 lane = threadIdx.x & 31u;\n"
+          " u32* Rs = jsmem + (threadIdx.x >> 5) * %uu;\n Rs[%uu + lane] = 0u;\n"
+          " const u32 w = blockIdx.x * 4u + (threadIdx.x >> 5);\n if (w >= n_warps) return;\n"
+          " u32 lo = 0, hi = A.n_inst;\n while (hi - lo > 1) { const u32 mid = (lo + hi) >> 1; "
+          "if (__ldg(&A.inst[mid].warp_begin) <= w) lo = mid; else hi = mid; }\n const u32 k = lo;\n"
+          " const jfi_instance in = A.inst[k];\n const u32 wpc = (in.block + 31u) / 32u, lw = w - in.warp_begin;\n"
+          " const u64 r0 = warp_off[w], g0 = gst_off[w];\n"
+          " u32* ck = ckpt ? ckpt + ck_off[w] * %uull : (u32*)0;\n"
+          " JOut o;\n switch (in.kernel) {\n",
+          min_blocks, rs, zrow, ckw);
+        for (uint32_t k = 0; k < n_kern; ++k)
+            o("  case %u: kern_%u_trace(A, 0xFFFFFFFFu, 0u, 0u, 0u, 0u, 0u, 0u, k, lw / wpc, lw %% wpc, 0xFFFFFFFFu, ck, "
+              "ck ? ck_interval : 0u, gst + g0, 0xFFFFFFFFu, o, Rs, A.dec + %uu, A.ins + %uu, (u8*)0, rec + r0); break;\n",
+              k, k, kern[k].code_off, kern[k].code_off);
+        o("  default: o.steps = 0; o.fault = 9; o.nstore = 0; break;\n }\n"
+          " if (lane == 0u && (o.fault || o.steps != warp_off[w + 1] - r0 || o.nstore != gst_off[w + 1] - g0)) "
+          "atomicOr(status, 1u << 4);\n}\n");
+    }
     return o.s;
 }
 
@@ -659,8 +770,9 @@ static size_t jit_smem(uint32_t n_regs) { return (size_t)4 * (n_regs + 1) * 128;
 
 struct fi_jit {
     size_t smem = 0;
+    uint32_t modes = 0;
     CUmodule mod = nullptr;
-    CUfunction inject = nullptr;
+    CUfunction inject = nullptr, glen = nullptr, gtrace = nullptr;
     uint32_t n_regs = 0, n_code = 0;
     double compile_s = 0;
     size_t src_bytes = 0, cubin_bytes = 0;
@@ -668,6 +780,7 @@ struct fi_jit {
 
 namespace fi {
 size_t aux_dec_offset(const fi_program* p);
+size_t aux_ins_offset(const fi_program* p);
 void launch_lpt_order(const fi_site* sites, const uint64_t* warp_off, uint32_t ck_interval, uint32_t n,
                       uint32_t* order, uint32_t* counter, cudaStream_t s);
 }
@@ -675,11 +788,11 @@ void launch_lpt_order(const fi_site* sites, const uint64_t* warp_off, uint32_t c
 extern "C" const char* fi_jit_log(void) { return g_jit_log.c_str(); }
 
 extern "C" size_t fi_jit_source(const fi_insn* code_host, uint32_t n_code, const fi_kernel* kern_host, uint32_t n_kern,
-                                uint32_t n_regs, char* buf, size_t buf_bytes) {
-    if (!code_host || !kern_host || !n_kern || n_regs == 0 || n_regs > fi::kRZ) return 0;
+                                uint32_t n_regs, uint32_t modes, char* buf, size_t buf_bytes) {
+    if (!code_host || !kern_host || !n_kern || n_regs == 0 || n_regs > fi::kRZ || !modes || modes > 3) return 0;
     for (uint32_t k = 0; k < n_kern; ++k)
         if ((uint64_t)kern_host[k].code_off + kern_host[k].code_len > n_code) return 0;
-    const std::string s = generate(code_host, kern_host, n_kern, n_regs);
+    const std::string s = generate(code_host, kern_host, n_kern, n_regs, modes);
     if (buf && buf_bytes) {
         const size_t m = std::min(buf_bytes - 1, s.size());
         std::memcpy(buf, s.data(), m);
@@ -689,12 +802,11 @@ extern "C" size_t fi_jit_source(const fi_insn* code_host, uint32_t n_code, const
 }
 
 namespace {
-fi_status compile_cubin(const fi_insn* code, uint32_t n_code, const fi_kernel* kern, uint32_t n_kern, uint32_t n_regs,
+fi_status compile_cubin(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern, uint32_t n_regs, uint32_t modes,
                         std::string& src, std::vector<char>& cubin) {
-    (void)n_code;
     Nvrtc& N = nvrtc();
     if (!N.ok) { g_jit_log = "libnvrtc.so.12 not found"; return FI_E_CUDA; }
-    src = generate(code, kern, n_kern, n_regs);
+    src = generate(code, kern, n_kern, n_regs, modes);
     void* prog = nullptr;
     if (N.create(&prog, src.c_str(), "fi_jit.cu", 0, nullptr, nullptr)) { g_jit_log = "nvrtcCreateProgram failed"; return FI_E_CUDA; }
     const char* opts[] = {"--gpu-architecture=sm_100a", "--std=c++17", "--fmad=false", "-lineinfo"};
@@ -712,25 +824,30 @@ fi_status compile_cubin(const fi_insn* code, uint32_t n_code, const fi_kernel* k
     N.destroy(&prog);
     return FI_OK;
 }
+
+bool valid_kernels(const fi_kernel* kern, uint32_t n_kern, uint32_t n_code) {
+    for (uint32_t k = 0; k < n_kern; ++k)
+        if ((uint64_t)kern[k].code_off + kern[k].code_len > n_code) return false;
+    return true;
+}
 }  // namespace
 
 extern "C" fi_status fi_jit_compile_check(const fi_insn* code_host, uint32_t n_code, const fi_kernel* kern_host,
-                                          uint32_t n_kern, uint32_t n_regs, size_t* cubin_bytes) {
-    if (!code_host || !kern_host || !n_kern || n_regs == 0 || n_regs > fi::kRZ) return FI_E_ARG;
-    for (uint32_t k = 0; k < n_kern; ++k)
-        if ((uint64_t)kern_host[k].code_off + kern_host[k].code_len > n_code) return FI_E_ARG;
+                                          uint32_t n_kern, uint32_t n_regs, uint32_t modes, size_t* cubin_bytes) {
+    if (!code_host || !kern_host || !n_kern || n_regs == 0 || n_regs > fi::kRZ || !modes || modes > 3) return FI_E_ARG;
+    if (!valid_kernels(kern_host, n_kern, n_code)) return FI_E_ARG;
     std::string src;
     std::vector<char> cubin;
-    fi_status e = compile_cubin(code_host, n_code, kern_host, n_kern, n_regs, src, cubin);
+    fi_status e = compile_cubin(code_host, kern_host, n_kern, n_regs, modes, src, cubin);
     if (cubin_bytes) *cubin_bytes = cubin.size();
     return e;
 }
 
-extern "C" fi_status fi_jit_build(const fi_program* p, const fi_kernel* kern_host, fi_jit** out) {
-    if (!p || !kern_host || !out || !p->code_host || !p->n_kern || p->n_regs == 0 || p->n_regs > fi::kRZ)
+extern "C" fi_status fi_jit_build(const fi_program* p, const fi_kernel* kern_host, uint32_t modes, fi_jit** out) {
+    if (!p || !kern_host || !out || !p->code_host || !p->n_kern || p->n_regs == 0 || p->n_regs > fi::kRZ || !modes ||
+        modes > 3)
         return FI_E_ARG;
-    for (uint32_t k = 0; k < p->n_kern; ++k)
-        if ((uint64_t)kern_host[k].code_off + kern_host[k].code_len > p->n_code) return FI_E_ARG;
+    if (!valid_kernels(kern_host, p->n_kern, p->n_code)) return FI_E_ARG;
     *out = nullptr;
     Drv& D = drv();
     if (!D.ok) { g_jit_log = "CUDA driver entry points unavailable"; return FI_E_CUDA; }
@@ -739,27 +856,28 @@ extern "C" fi_status fi_jit_build(const fi_program* p, const fi_kernel* kern_hos
     if (e0) return e0;
     std::string src;
     std::vector<char> cubin;
-    fi_status e = compile_cubin(p->code_host, p->n_code, kern_host, p->n_kern, p->n_regs, src, cubin);
+    fi_status e = compile_cubin(p->code_host, kern_host, p->n_kern, p->n_regs, modes, src, cubin);
     if (e) return e;
-    const size_t cs = cubin.size();
     fi_jit* j = new fi_jit();
-    if (D.load(&j->mod, cubin.data()) != CUDA_SUCCESS || D.get(&j->inject, j->mod, "k_inject_jit") != CUDA_SUCCESS) {
-        g_jit_log += "\ncuModuleLoadData/cuModuleGetFunction failed";
+    j->smem = jit_smem(p->n_regs);
+    bool ok = D.load(&j->mod, cubin.data()) == CUDA_SUCCESS;
+    auto get = [&](CUfunction* f, const char* name) {
+        ok = ok && D.get(f, j->mod, name) == CUDA_SUCCESS &&
+             D.set_attr(*f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)j->smem) == CUDA_SUCCESS;
+    };
+    if (modes & FI_JIT_INJECT) get(&j->inject, "k_inject_jit");
+    if (modes & FI_JIT_GOLDEN) { get(&j->glen, "k_golden_len_jit"); get(&j->gtrace, "k_golden_trace_jit"); }
+    if (!ok) {
+        g_jit_log += "\ncuModuleLoadData / cuModuleGetFunction / cuFuncSetAttribute failed";
         if (j->mod) D.unload(j->mod);
         delete j;
         return FI_E_CUDA;
     }
+    j->modes = modes;
     j->n_regs = p->n_regs;
     j->n_code = p->n_code;
-    j->smem = jit_smem(p->n_regs);
-    if (D.set_attr(j->inject, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)j->smem) != CUDA_SUCCESS) {
-        g_jit_log = "cuFuncSetAttribute(MAX_DYNAMIC_SHARED_SIZE_BYTES) failed";
-        D.unload(j->mod);
-        delete j;
-        return FI_E_CUDA;
-    }
     j->src_bytes = src.size();
-    j->cubin_bytes = cs;
+    j->cubin_bytes = cubin.size();
     j->compile_s = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
     *out = j;
     return FI_OK;
@@ -773,6 +891,7 @@ extern "C" void fi_jit_free(fi_jit* j) {
     delete j;
 }
 
+namespace {
 struct JArgsHost {                                   // = JArgs of jit_prelude.cuh
     const uint8_t* img;
     const uint32_t* gran;
@@ -780,15 +899,36 @@ struct JArgsHost {                                   // = JArgs of jit_prelude.c
     const fi_instance* inst;
     const uint32_t* cbank;
     const uint4* dec;
+    const uint32_t* ins;
     uint64_t image_bytes;
+    uint32_t n_inst;
 };
 
+JArgsHost jargs(const fi_program* p, const uint8_t* image) {
+    const char* aux = reinterpret_cast<const char*>(p->aux);
+    return JArgsHost{image,
+                     reinterpret_cast<const uint32_t*>(aux),   // granule map at aux offset 0
+                     p->buf, p->inst, p->cbank,
+                     reinterpret_cast<const uint4*>(aux + fi::aux_dec_offset(p)),
+                     reinterpret_cast<const uint32_t*>(aux + fi::aux_ins_offset(p)),
+                     p->image_bytes, p->n_inst};
+}
+
+fi_status launch(CUfunction f, uint32_t grid, size_t smem, cudaStream_t s, void** args) {
+    const CUresult r = drv().launch(f, grid, 1, 1, 128, 1, 1, (unsigned)smem, (CUstream)s, args, nullptr);
+    if (r != CUDA_SUCCESS) {
+        g_jit_log = "cuLaunchKernel failed: " + std::to_string((int)r);
+        return FI_E_CUDA;
+    }
+    return fi::launch_status();
+}
+}  // namespace
 
 extern "C" fi_status fi_inject_jit(const fi_jit* j, const fi_program* p, const uint8_t* image, const fi_trace* t,
                                    const fi_site* sites, uint32_t n, fi_inj* out, fi_store* log, uint32_t log_cap,
                                    void* ws, size_t ws_bytes, uint32_t* dev_status, void* stream) {
     if (!j || !p || !image || !t || !sites || !out || !dev_status || (log_cap && !log) || !p->aux) return FI_E_ARG;
-    if (j->n_regs != p->n_regs || j->n_code != p->n_code) return FI_E_ARG;
+    if (!(j->modes & FI_JIT_INJECT) || j->n_regs != p->n_regs || j->n_code != p->n_code) return FI_E_ARG;
     if (t->ckpt && (!t->ckpt_off || !t->ckpt_interval)) return FI_E_ARG;
     if (n == 0) return FI_OK;
     if (!ws || ws_bytes < fi_inject_workspace(n)) return FI_E_ARG;
@@ -799,27 +939,51 @@ extern "C" fi_status fi_inject_jit(const fi_jit* j, const fi_program* p, const u
     fi::launch_lpt_order(sites, t->warp_off, ck_iv, n, order, counter, s);
     fi_status e = fi::launch_status();
     if (e) return e;
-    Drv& D = drv();
     int dev = 0, sms = 0, per = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    D.occ(&per, j->inject, 128, j->smem);
-    const uint32_t grid =
-        (uint32_t)std::min<uint64_t>((n + 3) / 4, (uint64_t)std::max(1, sms * std::max(1, per)));
-    JArgsHost A{image,
-                reinterpret_cast<const uint32_t*>(p->aux),   // granule map at aux offset 0
-                p->buf, p->inst, p->cbank,
-                reinterpret_cast<const uint4*>(reinterpret_cast<const char*>(p->aux) + fi::aux_dec_offset(p)),
-                p->image_bytes};
+    drv().occ(&per, j->inject, 128, j->smem);
+    const uint32_t grid = (uint32_t)std::min<uint64_t>((n + 3) / 4, (uint64_t)std::max(1, sms * std::max(1, per)));
+    JArgsHost A = jargs(p, image);
     const uint64_t* warp_off = t->warp_off;
     const uint32_t* ckpt = t->ckpt;
     const uint64_t* ck_off = t->ckpt_off;
     void* args[] = {&A, (void*)&warp_off, (void*)&sites, &n, &out, &log, &log_cap, (void*)&ckpt, (void*)&ck_off,
                     (void*)&ck_iv, &order, &counter, &dev_status};
-    const CUresult r = D.launch(j->inject, grid, 1, 1, 128, 1, 1, (unsigned)j->smem, (CUstream)s, args, nullptr);
-    if (r != CUDA_SUCCESS) {
-        g_jit_log = "cuLaunchKernel failed: " + std::to_string((int)r);
-        return FI_E_CUDA;
+    return launch(j->inject, grid, j->smem, s, args);
+}
+
+extern "C" fi_status fi_golden_lengths_jit(const fi_jit* j, const fi_program* p, uint8_t* image, uint64_t* warp_len,
+                                           uint64_t* warp_nstore, uint32_t* dev_status, void* stream) {
+    if (!j || !p || !image || !warp_len || !warp_nstore || !dev_status || !p->inst_host || !p->aux) return FI_E_ARG;
+    if (!(j->modes & FI_JIT_GOLDEN) || j->n_regs != p->n_regs || j->n_code != p->n_code) return FI_E_ARG;
+    cudaStream_t s = (cudaStream_t)stream;
+    JArgsHost A = jargs(p, image);
+    for (uint32_t k = 0; k < p->n_inst; ++k) {
+        const uint32_t nw = p->inst_host[k].warp_end - p->inst_host[k].warp_begin;
+        if (!nw) continue;
+        uint32_t kk = k;
+        void* args[] = {&A, &kk, &image, &warp_len, &warp_nstore, &dev_status};
+        fi_status e = launch(j->glen, (nw + 3) / 4, j->smem, s, args);
+        if (e) return e;
     }
-    return fi::launch_status();
+    return FI_OK;
+}
+
+extern "C" fi_status fi_golden_trace_jit(const fi_jit* j, const fi_program* p, const uint8_t* image, const fi_trace* t,
+                                         uint32_t* dev_status, void* stream) {
+    if (!j || !p || !image || !t || !t->warp_off || !t->gstore_off || !t->rec || !dev_status || !p->aux) return FI_E_ARG;
+    if (!(j->modes & FI_JIT_GOLDEN) || j->n_regs != p->n_regs || j->n_code != p->n_code) return FI_E_ARG;
+    if (t->ckpt && (!t->ckpt_off || !t->ckpt_interval)) return FI_E_ARG;
+    if (!p->n_warps) return FI_OK;
+    JArgsHost A = jargs(p, image);
+    uint32_t nw = p->n_warps, iv = t->ckpt ? t->ckpt_interval : 0;
+    const uint64_t* woff = t->warp_off;
+    const uint64_t* goff = t->gstore_off;
+    const uint64_t* ckoff = t->ckpt_off;
+    fi_record* rec = t->rec;
+    fi_store* gst = t->gstore;
+    uint32_t* ck = t->ckpt;
+    void* args[] = {&A, &nw, (void*)&woff, (void*)&goff, &rec, &gst, &ck, (void*)&ckoff, &iv, &dev_status};
+    return launch(j->gtrace, (nw + 3) / 4, j->smem, (cudaStream_t)stream, args);
 }

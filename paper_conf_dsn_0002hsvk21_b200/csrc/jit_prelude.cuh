@@ -40,7 +40,9 @@ struct JArgs {
     const jfi_instance* inst;
     const u32* cbank;
     const uint4* dec;            // pre-decoded code (fi_program_prepare), for step mode
+    const u32* ins;              // trace insn word per static instruction (pc | op << 16 | groups << 24)
     u64 image_bytes;
+    u32 n_inst;
 };
 
 struct JOut {
@@ -205,7 +207,11 @@ __device__ __forceinline__ u32 jldg(const JArgs& A, JBufCache& C, u64 va, u32 k,
 // or faults.  Same semantics as emu.cuh's general step.
 struct JState {
     u32 pc, live, step, livem, conv, upc, amask, npc, nst, fault, fault_pc, before, after, msk, fired, bad, lim, preds;
+    uint4 recbuf;                                    // golden trace pass: this lane's record of the 32-step window
 };
+#define JM_INJ 0                                     // injection replica (K4): hook, stores after the site logged
+#define JM_LEN 1                                     // golden pass 1: stores into the image, steps / stores counted
+#define JM_TRACE 2                                   // golden pass 2: trace records, store log, checkpoints
 
 __device__ __forceinline__ bool jguard(u32 guard, u32 preds) {
     const u32 gs = guard & 7;
@@ -345,14 +351,17 @@ __device__ __forceinline__ void jexec_plain(const JRegs& F, const uint4 D, const
     }
 }
 
-// Injection-mode steps (EMU_INJ of emu.cuh).  Returns 1 when the warp is done
-// (finished or faulted), 0 when it stands at a leader whose block fits.
-__device__ __noinline__ u32 jinterp_inj(const JArgs& A, JState& S, JBufCache& bc, u32* R, const uint4* __restrict__ dec,
-                                        const unsigned short* __restrict__ blen, const u32 code_len, const u32 k,
-                                        const u32 cta, const u32 wic, const u32 watchdog, const u32 hstep, const u32 hpc,
-                                        const u32 hlane, const u32 hkind, const u32 hreg, const u32 hbfm,
-                                        const u32 hmask, jfi_store* __restrict__ st_out, const u32 st_cap,
-                                        const u32 zr) {
+// Step mode (emu.cuh's general step; MODE = JM_INJ / JM_LEN / JM_TRACE).  Returns
+// 1 when the warp is done (finished or faulted), 0 when it stands at a leader
+// whose block fits.  `ck` (JM_TRACE): the warp's checkpoint destination, or 0.
+template <int MODE>
+__device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u32* R, const uint4* __restrict__ dec,
+                                    const unsigned short* __restrict__ blen, const u32 code_len, const u32 k,
+                                    const u32 cta, const u32 wic, const u32 watchdog, const u32 hstep, const u32 hpc,
+                                    const u32 hlane, const u32 hkind, const u32 hreg, const u32 hbfm,
+                                    const u32 hmask, jfi_store* __restrict__ st_out, const u32 st_cap,
+                                    const u32 zr, u8* __restrict__ img_w, uint4* __restrict__ rec_out,
+                                    u32* __restrict__ ck, const u32 ck_interval, const u32* __restrict__ ins) {
     const u32 lane = threadIdx.x & 31, lt_mask = (1u << lane) - 1u;
     const JRegs F{reinterpret_cast<char*>(R + lane), R, zr * 128};
     const jfi_instance in = A.inst[k];
@@ -360,6 +369,7 @@ __device__ __noinline__ u32 jinterp_inj(const JArgs& A, JState& S, JBufCache& bc
     bool live = S.live != 0, conv = S.conv != 0;
     u32 pc = S.pc, step = S.step, livem = S.livem, upc = S.upc, amask = S.amask, npc = S.npc, nst = S.nst;
     u32 preds = S.preds, lim = S.lim;
+    uint4 recbuf = S.recbuf;
     u32 done = 0;
     for (;;) {
         if (!livem) { done = 1; break; }
@@ -370,6 +380,17 @@ __device__ __noinline__ u32 jinterp_inj(const JArgs& A, JState& S, JBufCache& bc
             active = __ballot_sync(JFULL, live && pc == pcm);
             npc = active == livem ? 0xFFFFFFFFu : __reduce_min_sync(JFULL, (live && pc != pcm) ? pc : 0xFFFFFFFFu);
             conv = true; upc = pcm; amask = active;
+        }
+        if (MODE == JM_TRACE && ck) {                 // golden register-file checkpoint every ck_interval steps
+            if (step % ck_interval == 0) {
+                const bool inA = (amask >> lane) & 1u;
+                u32* dst = ck + (u64)(step / ck_interval) * (zr + 3) * 32;
+                for (u32 r = 0; r < zr; ++r) dst[r * 32 + lane] = R[r * 32 + lane];
+                dst[zr * 32 + lane] = live ? (inA ? upc : pc) : 0u;
+                dst[zr * 32 + 32 + lane] = preds;
+                dst[zr * 32 + 64 + lane] = live ? 1u : 0u;
+            }
+            lim = min(watchdog, (step / ck_interval + 1) * ck_interval);
         }
         if (step >= watchdog) { S.fault = 3; S.fault_pc = pcm; done = 1; break; }
         if (pcm >= code_len) { S.fault = 4; S.fault_pc = pcm; done = 1; break; }
@@ -383,6 +404,10 @@ __device__ __noinline__ u32 jinterp_inj(const JArgs& A, JState& S, JBufCache& bc
         const u32 pred = guard == 7 ? JFULL : __ballot_sync(JFULL, pv);
         const bool ex = act && pv;
         const u32 exm = active & pred;
+        if (MODE == JM_TRACE) {                       // one trace record per step (App. A.3)
+            if ((step & 31) == lane) recbuf = make_uint4(k, __ldg(&ins[pcm]), active, pred);
+            if ((step & 31) == 31) rec_out[step - 31 + lane] = recbuf;
+        }
         u32 taken = 0;
         if (op == 1) {                                // EXIT
             if (ex) live = false;
@@ -414,18 +439,30 @@ __device__ __noinline__ u32 jinterp_inj(const JArgs& A, JState& S, JBufCache& bc
                     if (lw >= 1) F.wr(id + 128, v.y);
                     if (lw >= 2) { F.wr(id + 256, v.z); F.wr(id + 384, v.w); }
                 }
-            } else if (step > hstep) {                // stores after the site are logged
+            } else {
                 u32 v[4];
 #pragma unroll
                 for (int i = 0; i < 4; ++i) v[i] = (u32)i < nw ? F.rd(min(ib + 128u * i, F.zb)) : 0u;
-                if (ex) {
-                    const u32 idx = __popc(exm & lt_mask) * nw;
-                    for (u32 i = 0; i < nw; ++i) {
-                        const u32 e = nst + idx + i;
-                        if (e < st_cap) { jfi_store s_; s_.va = va + 4 * i; s_.value = v[i]; s_.step = step; st_out[e] = s_; }
+                if (MODE == JM_LEN) {                 // golden pass 1: stores go to the image
+                    if (ex) {
+                        u8* dst = img_w + (va - JVA_BASE);
+                        if (lw == 0) *reinterpret_cast<u32*>(dst) = v[0];
+                        else if (lw == 1) *reinterpret_cast<uint2*>(dst) = make_uint2(v[0], v[1]);
+                        else *reinterpret_cast<uint4*>(dst) = make_uint4(v[0], v[1], v[2], v[3]);
                     }
+                    nst += __popc(exm) * nw;
+                } else if (MODE == JM_TRACE || step > hstep) {   // golden store log / stores after the site
+                    if (ex) {
+                        const u32 idx = __popc(exm & lt_mask) * nw;
+                        for (u32 i = 0; i < nw; ++i) {
+                            const u32 e = nst + idx + i;
+                            if (MODE == JM_TRACE || e < st_cap) {
+                                jfi_store s_; s_.va = va + 4 * i; s_.value = v[i]; s_.step = step; st_out[e] = s_;
+                            }
+                        }
+                    }
+                    nst += __popc(exm) * nw;
                 }
-                nst += __popc(exm) * nw;
             }
         } else {
             jexec_plain(F, D, ex, preds, lane, cta, wic, in, cb);
@@ -434,7 +471,7 @@ __device__ __noinline__ u32 jinterp_inj(const JArgs& A, JState& S, JBufCache& bc
         else if (taken == active) upc = imm;
         else { conv = false; if (act) pc = ((taken >> lane) & 1u) ? imm : pcm + 1; }
         if (conv && (amask == 0 || upc >= npc)) { conv = false; if ((amask >> lane) & 1u) pc = upc; }
-        if (step == hstep) {                          // the transient fault (C-7, C-8)
+        if (MODE == JM_INJ && step == hstep) {        // the transient fault (C-7, C-8)
             S.fired = 1;
             if (pcm != hpc || !((exm >> hlane) & 1u)) S.bad = 1;
             if (lane == hlane) {
@@ -457,9 +494,9 @@ __device__ __noinline__ u32 jinterp_inj(const JArgs& A, JState& S, JBufCache& bc
             }
         }
         ++step;
-        if (step > hstep) lim = watchdog;
+        if (MODE == JM_INJ && step > hstep) lim = watchdog;
     }
     S.pc = pc; S.live = live; S.step = step; S.livem = livem; S.conv = conv; S.upc = upc; S.amask = amask;
-    S.npc = npc; S.nst = nst; S.preds = preds; S.lim = lim;
+    S.npc = npc; S.nst = nst; S.preds = preds; S.lim = lim; S.recbuf = recbuf;
     return done;
 }

@@ -105,6 +105,7 @@ class fi_campaign_result(C.Structure):
 ALLREDUCE_FN = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_uint64, C.c_uint32, C.c_void_p, C.c_void_p)
 FI_PROPAGATION = {"auto": 0, "k7": 1, "k8": 2}
 FI_CKPT_AUTO = 0xFFFFFFFF
+FI_JIT_INJECT, FI_JIT_GOLDEN = 1, 2
 
 _lib = None
 
@@ -152,12 +153,14 @@ def lib():
                                                  vp, vp]),
             "fi_classify_batched": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, u32, u32, u32, u32, vp, sz, vp, vp]),
             "fi_inject_permanent": (st, [vp, vp, vp, vp, u32, vp, vp, vp, u32, u32, vp, u32, vp, sz, vp, vp]),
-            "fi_jit_build": (st, [vp, vp, C.POINTER(vp)]),
+            "fi_jit_build": (st, [vp, vp, u32, C.POINTER(vp)]),
             "fi_jit_free": (None, [vp]),
             "fi_jit_compile_seconds": (C.c_double, [vp]),
             "fi_jit_log": (C.c_char_p, []),
-            "fi_jit_compile_check": (st, [vp, u32, vp, u32, u32, C.POINTER(C.c_size_t)]),
-            "fi_jit_source": (sz, [vp, u32, vp, u32, u32, vp, sz]),
+            "fi_jit_compile_check": (st, [vp, u32, vp, u32, u32, u32, C.POINTER(C.c_size_t)]),
+            "fi_jit_source": (sz, [vp, u32, vp, u32, u32, u32, vp, sz]),
+            "fi_golden_lengths_jit": (st, [vp, vp, vp, vp, vp, vp, vp]),
+            "fi_golden_trace_jit": (st, [vp, vp, vp, vp, vp, vp]),
             "fi_inject_jit": (st, [vp, vp, vp, vp, vp, u32, vp, vp, u32, vp, sz, vp, vp]),
             "fi_write_profile_txt": (st, [vp, vp, u32, vp, u32, vp, sz, C.POINTER(C.c_size_t)]),
             "fi_campaign": (st, [C.POINTER(fi_campaign_cfg), C.c_int, C.c_int, ALLREDUCE_FN, vp,
@@ -240,7 +243,7 @@ class DeviceProgram:
         self._code_host = np.ascontiguousarray(prog.code)
         self._inst_host = np.ascontiguousarray(prog.instances)
         self._kern_host = np.ascontiguousarray(prog.kernels)
-        self._jit = None
+        self._jit = {}
         self.n_regs = int(lib().fi_program_regs(self._code_host.ctypes.data, len(self._code_host)))
         self.c = fi_program(
             _p(self.code), len(prog.code), _p(self.kern), len(prog.kernels), _p(self.inst), len(prog.instances),
@@ -252,17 +255,17 @@ class DeviceProgram:
     def n_inst(self):
         return len(self.prog.instances)
 
-    def jit(self) -> "Jit":
-        """The program's JIT-specialised emulator module (fi_jit_build), built once
-        per (code, kernel table, register rows, device) in this process."""
-        if self._jit is None:
+    def jit(self, modes: int = FI_JIT_INJECT) -> "Jit":
+        """The program's JIT-specialised emulator module (fi_jit_build) for `modes`,
+        built once per (code, kernel table, register rows, modes, device) in this process."""
+        if modes not in self._jit:
             import hashlib
-            key = (hashlib.sha1(self._code_host.tobytes() + self._kern_host.tobytes()).hexdigest(), self.n_regs,
+            key = (hashlib.sha1(self._code_host.tobytes() + self._kern_host.tobytes()).hexdigest(), self.n_regs, modes,
                    self.device.index if self.device.index is not None else torch.cuda.current_device())
             if key not in _JIT_CACHE:
-                _JIT_CACHE[key] = Jit(self)
-            self._jit = _JIT_CACHE[key]
-        return self._jit
+                _JIT_CACHE[key] = Jit(self, modes)
+            self._jit[modes] = _JIT_CACHE[key]
+        return self._jit[modes]
 
     @property
     def n_warps(self):
@@ -275,9 +278,9 @@ _JIT_CACHE: dict = {}
 class Jit:
     """fi_jit_build: per-program generated CUDA, NVRTC-compiled for sm_100a."""
 
-    def __init__(self, dp: "DeviceProgram"):
+    def __init__(self, dp: "DeviceProgram", modes: int = FI_JIT_INJECT):
         h = C.c_void_p()
-        rc = lib().fi_jit_build(C.byref(dp.c), dp._kern_host.ctypes.data, C.byref(h))
+        rc = lib().fi_jit_build(C.byref(dp.c), dp._kern_host.ctypes.data, modes, C.byref(h))
         if rc != FI_OK:
             raise FIError(rc, "fi_jit_build", lib().fi_jit_log().decode()[-4000:])
         self.h = h
@@ -292,21 +295,21 @@ class Jit:
             pass
 
 
-def jit_source(prog, n_regs: int | None = None) -> str:
+def jit_source(prog, modes: int = FI_JIT_INJECT, n_regs: int | None = None) -> str:
     code, kern = np.ascontiguousarray(prog.code), np.ascontiguousarray(prog.kernels)
     nr = n_regs or int(lib().fi_program_regs(code.ctypes.data, len(code)))
-    n = lib().fi_jit_source(code.ctypes.data, len(code), kern.ctypes.data, len(kern), nr, None, 0)
+    n = lib().fi_jit_source(code.ctypes.data, len(code), kern.ctypes.data, len(kern), nr, modes, None, 0)
     buf = C.create_string_buffer(n)
-    lib().fi_jit_source(code.ctypes.data, len(code), kern.ctypes.data, len(kern), nr, buf, n)
+    lib().fi_jit_source(code.ctypes.data, len(code), kern.ctypes.data, len(kern), nr, modes, buf, n)
     return buf.value.decode()
 
 
-def jit_compile_check(prog) -> int:
+def jit_compile_check(prog, modes: int = FI_JIT_INJECT) -> int:
     """NVRTC-compile the program's generated emulator without loading it (no GPU); returns cubin bytes."""
     code, kern = np.ascontiguousarray(prog.code), np.ascontiguousarray(prog.kernels)
     nr = int(lib().fi_program_regs(code.ctypes.data, len(code)))
     cb = C.c_size_t(0)
-    rc = lib().fi_jit_compile_check(code.ctypes.data, len(code), kern.ctypes.data, len(kern), nr, C.byref(cb))
+    rc = lib().fi_jit_compile_check(code.ctypes.data, len(code), kern.ctypes.data, len(kern), nr, modes, C.byref(cb))
     if rc != FI_OK:
         raise FIError(rc, "fi_jit_compile_check", lib().fi_jit_log().decode()[-4000:])
     return int(cb.value)
@@ -342,17 +345,26 @@ def scan_u64(x: torch.Tensor) -> torch.Tensor:
     return out
 
 
-def golden_run(dp: DeviceProgram, ckpt_interval: int | str = "auto", ckpt_budget_frac: float = 0.2) -> GoldenTrace:
+def golden_run(dp: DeviceProgram, ckpt_interval: int | str = "auto", ckpt_budget_frac: float = 0.2,
+               engine: str = "interp") -> GoldenTrace:
     """fi_golden_lengths (pass 1) -> scans + checkpoint layout -> fi_golden_trace (pass 2).
 
     ckpt_interval: steps between golden register-file checkpoints (0 = none);
-    "auto" = 4096, doubled until the checkpoints fit ckpt_budget_frac of free HBM."""
+    "auto" = 4096, doubled until the checkpoints fit ckpt_budget_frac of free HBM.
+    engine: "interp" (emu.cuh) or "jit" (fi_golden_*_jit on the program's JIT
+    module built with FI_JIT_GOLDEN): bit-identical results."""
+    jit = dp.jit(FI_JIT_GOLDEN) if engine == "jit" else None
     st = DeviceStatus(dp.device)
     image = dp.init_image.clone()
     W = dp.n_warps
     wl = torch.zeros(max(W, 1), dtype=torch.int64, device=dp.device)
     wn = torch.zeros(max(W, 1), dtype=torch.int64, device=dp.device)
-    _check(lib().fi_golden_lengths(C.byref(dp.c), _p(image), _p(wl), _p(wn), st.ptr, _stream()), "fi_golden_lengths")
+    if jit is not None:
+        _check(lib().fi_golden_lengths_jit(jit.h, C.byref(dp.c), _p(image), _p(wl), _p(wn), st.ptr, _stream()),
+               "fi_golden_lengths_jit")
+    else:
+        _check(lib().fi_golden_lengths(C.byref(dp.c), _p(image), _p(wl), _p(wn), st.ptr, _stream()),
+               "fi_golden_lengths")
     woff = scan_u64(wl[:W])
     goff = scan_u64(wn[:W])
     st.check("fi_golden_lengths")
@@ -377,7 +389,11 @@ def golden_run(dp: DeviceProgram, ckpt_interval: int | str = "auto", ckpt_budget
             interval *= 2
         ck = torch.empty(max(total, 16), dtype=torch.uint8, device=dp.device)
     tc = fi_trace(_p(rec), n_rec, _p(woff), _p(gst), _p(goff), _p(ck), _p(ckoff), interval, W)
-    _check(lib().fi_golden_trace(C.byref(dp.c), _p(image), C.byref(tc), st.ptr, _stream()), "fi_golden_trace")
+    if jit is not None:
+        _check(lib().fi_golden_trace_jit(jit.h, C.byref(dp.c), _p(image), C.byref(tc), st.ptr, _stream()),
+               "fi_golden_trace_jit")
+    else:
+        _check(lib().fi_golden_trace(C.byref(dp.c), _p(image), C.byref(tc), st.ptr, _stream()), "fi_golden_trace")
     st.check("fi_golden_trace")
     return GoldenTrace(dp, image, wl[:W], woff, goff, rec, gst, n_rec, n_gst, tc, ck, ckoff, interval)
 
@@ -463,7 +479,7 @@ def inject(gt: GoldenTrace, sites: torch.Tensor, n: int, log_cap: int, out: torc
     if ws is None or ws.numel() < ws_n:
         ws = torch.empty(ws_n, dtype=torch.uint8, device=dev)
     if engine == "jit":
-        _check(lib().fi_inject_jit(gt.dp.jit().h, C.byref(gt.dp.c), _p(gt.image), C.byref(gt.c), _p(sites), n, _p(out),
+        _check(lib().fi_inject_jit(gt.dp.jit(FI_JIT_INJECT).h, C.byref(gt.dp.c), _p(gt.image), C.byref(gt.c), _p(sites), n, _p(out),
                                    _p(log), log_cap, _p(ws), ws_n, st.ptr, _stream()), "fi_inject_jit")
     elif engine == "interp":
         _check(lib().fi_inject(C.byref(gt.dp.c), _p(gt.image), C.byref(gt.c), _p(sites), n, _p(out), _p(log), log_cap,

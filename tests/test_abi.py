@@ -101,5 +101,6 @@ def test_jit_source_compiles_for_sm100a():
     from paper_conf_dsn_0002hsvk21_b200 import fi
     for prog in (P.c1(), P.fuzz_program(3, n_ops=120), P.multi_instance_chain(3), P.scatter_chain()):
         assert fi.jit_compile_check(prog) > 1000
+    assert fi.jit_compile_check(P.c1(), fi.FI_JIT_INJECT | fi.FI_JIT_GOLDEN) > 1000
     src = fi.jit_source(P.c1())
     assert "k_inject_jit" in src and "kern_0" in src

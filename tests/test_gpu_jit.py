@@ -85,3 +85,34 @@ def test_jit_approximate_not_injected(F):
 def test_jit_c5_minis(F, which):
     prog = H.c5(full=False)[which]
     _both(F, prog, 0xC5, [F.G_GP, F.G_GPPR, F.G_PR], [0, 1, 2, 3], 300)
+
+
+def _golden_both(F, prog, ckpt):
+    dp = F.DeviceProgram(prog)
+    a = F.golden_run(dp, ckpt_interval=ckpt, engine="interp")
+    b = F.golden_run(dp, ckpt_interval=ckpt, engine="jit")
+    torch.cuda.synchronize()
+    assert a.n_rec == b.n_rec and a.n_gstore == b.n_gstore
+    assert torch.equal(a.warp_len, b.warp_len)
+    assert torch.equal(a.image, b.image), "golden final image"
+    assert torch.equal(a.rec[: a.n_rec * 16], b.rec[: b.n_rec * 16]), "trace records"
+    assert torch.equal(a.gstore[: a.n_gstore * 16], b.gstore[: b.n_gstore * 16]), "golden store log"
+    assert a.ckpt_interval == b.ckpt_interval
+    if a.ckpt is not None:
+        assert torch.equal(a.ckpt, b.ckpt), "register-file checkpoints"
+    return a
+
+
+@pytest.mark.parametrize("ckpt", [0, 5, 13, "auto"])
+@pytest.mark.parametrize("maker", [P.c1, lambda: P.fuzz_program(3, n_ops=120), lambda: P.fuzz_program(8, block=33),
+                                   lambda: P.c2(full=False), lambda: P.multi_instance_chain(6, shrink=29),
+                                   P.scatter_chain, lambda: P.c3(full=False), lambda: P.ffma_runs(5)])
+def test_jit_golden_passes(F, maker, ckpt):
+    """Golden passes 1 and 2 on the JIT module: lengths, final image, trace records,
+    store log and checkpoints byte-identical to the interpreter's."""
+    _golden_both(F, maker(), ckpt)
+
+
+@pytest.mark.parametrize("which", range(5))
+def test_jit_golden_c5_minis(F, which):
+    _golden_both(F, H.c5(full=False)[which], 7)
