@@ -352,6 +352,7 @@ fi_status fi_inject_permanent_batched(const fi_program* p, const uint8_t* image,
 typedef struct fi_jit fi_jit;
 #define FI_JIT_INJECT 1u                            /* k_inject_jit (fi_inject_jit) */
 #define FI_JIT_GOLDEN 2u                            /* golden passes (fi_golden_lengths_jit, fi_golden_trace_jit) */
+#define FI_JIT_PAGE 4u                              /* K8 re-execution over replica pages (fi_classify_batched_jit) */
 fi_status fi_jit_build(const fi_program* p, const fi_kernel* kern_host, uint32_t modes, fi_jit** out);
 void fi_jit_free(fi_jit* j);
 double fi_jit_compile_seconds(const fi_jit* j);
@@ -372,6 +373,12 @@ fi_status fi_golden_lengths_jit(const fi_jit* j, const fi_program* p, uint8_t* i
                                 uint64_t* warp_nstore, uint32_t* dev_status, void* stream);
 fi_status fi_golden_trace_jit(const fi_jit* j, const fi_program* p, const uint8_t* image, const fi_trace* t,
                               uint32_t* dev_status, void* stream);
+/* fi_classify_batched with K8's per-launch re-execution on a module built with
+ * FI_JIT_PAGE: same arguments, scratch and results (transient faults). */
+fi_status fi_classify_batched_jit(const fi_jit* j, const fi_program* p, const uint8_t* image, const fi_trace* t,
+                                  const fi_site* sites, uint32_t n, fi_inj* out, const fi_store* log, uint32_t log_cap,
+                                  uint64_t* hist, uint32_t flags, uint32_t batch, uint32_t pool_pages,
+                                  uint32_t pend_cap, void* ws, size_t ws_bytes, uint32_t* dev_status, void* stream);
 
 /* Table II parameter file, one parameter per line in Table II order
  * [PAPER.md:88]: arch state id, bit-flip model, kernel name, kernel count,

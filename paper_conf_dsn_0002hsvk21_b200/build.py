@@ -18,7 +18,7 @@ FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2", "--expt-re
          "-Xptxas", "-v,-warn-spills"] + ARCH
 SOURCES = ["abi.cpp", "golden.cu", "scan.cu", "profile.cu", "select.cu", "inject.cu", "propagate.cu", "propagate8.cu",
            "campaign.cpp", "jit.cpp"]
-HEADERS = ["common.cuh", "emu.cuh", "scan.cuh", "jit_prelude.cuh"]
+HEADERS = ["common.cuh", "emu.cuh", "scan.cuh", "jit_prelude.cuh", "jit_k8.h"]
 
 
 def _stale(obj: str, deps: list[str]) -> bool:

@@ -36,6 +36,7 @@
 
 #include "../../include/fi.h"
 #include "common.cuh"
+#include "jit_k8.h"
 
 namespace {
 
@@ -307,6 +308,7 @@ struct Gen {
             o("uint4 v_; const u32 c_ = jldg<%uu>(A, bc, va, k, ex, v_); ", lw);
             o("if (__ballot_sync(JFULL, c_ != 0u)) { fault = __ballot_sync(JFULL, c_ == 1u) ? 1u : 2u; fault_pc = %uu; "
               "step = %s; goto finish; } ", pc, stepx);
+            if (mode == 3) o("if (ex) jpage<%uu>(A, PG, va, v_); ", nw);
             const char* v[] = {"v_.x", "v_.y", "v_.z", "v_.w"};
             wr(o, I.d0, v, nw);
             o("}\n");
@@ -326,7 +328,7 @@ struct Gen {
                 return;
             }
             o("const u32 sst_ = %s; if (%s) { if (ex) { const u32 idx_ = __popc(exm_ & lt_mask) * %uu; ",
-              stepx, mode == 2 ? "true" : "sst_ > hstep", nw);
+              stepx, (mode == 2 || mode == 3) ? "true" : "sst_ > hstep", nw);
             for (uint32_t q = 0; q < nw; ++q) {
                 if (mode == 2)
                     o("{ jfi_store e_; e_.va = va + %uu; e_.value = %s; e_.step = sst_; st_out[nst + idx_ + %uu] = e_; } ",
@@ -389,6 +391,7 @@ struct Gen {
             if (lw == 0) o("v_.x = jld32(p_); } ");
             else if (lw == 1) o("const uint2 t_ = jld64(p_); v_.x = t_.x; v_.y = t_.y; } ");
             else o("v_ = jld128(p_); } ");
+            if (mode == 3) o("jpage<%uu>(A, PG, va%u, v_); ", nw, j);
             if (I.d0 != fi::kRZ)
                 for (uint32_t q = 0; q < nw; ++q)
                     if (W(I.d0 + q)) o("R%u = v_.%c; ", I.d0 + q, "xyzw"[q]);
@@ -426,7 +429,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
     Gen G = G0;
     G.mode = mode;
     const uint32_t NR = G.NR;
-    static const char* const mname[] = {"inj", "len", "trace"};
+    static const char* const mname[] = {"inj", "len", "trace", "page"};
     // block length from each pc: to the next BRA/EXIT inclusive, or the code end
     std::vector<uint32_t> blen(n);
     for (int64_t i = (int64_t)n - 1; i >= 0; --i) {
@@ -455,8 +458,9 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "const u32 wic, const u32 watchdog, u32* __restrict__ ck, const u32 ck_interval, "
       "jfi_store* __restrict__ st_out, const u32 st_cap, JOut& out, u32* __restrict__ Rs, "
       "const uint4* __restrict__ dec, const u32* __restrict__ ins, u8* __restrict__ img_w, "
-      "uint4* __restrict__ rec_out) {\n", kid, mname[mode]);
+      "uint4* __restrict__ rec_out, const JPage* __restrict__ pgp) {\n", kid, mname[mode]);
     o("(void)img_w; (void)rec_out; (void)ins;\n");
+    if (mode == 3) o("const JPage PG = *pgp;               // the replica slot's pages (K8)\n");
     o("const JArgs A = A_;                 // kernel arguments in registers for the whole run\n");
     o("const u32 lane = threadIdx.x & 31u, lt_mask = (1u << lane) - 1u;\n");
     o("const jfi_instance in = A.inst[k];\nconst u32 cbank_len = in.cbank_len; const u32* __restrict__ cb = A.cbank + "
@@ -579,7 +583,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "((u32)Q6 << 6); st_.recbuf = recbuf;\n"
       "  __syncwarp();\n"
       "  const u32 done_ = jinterp<%u>(A, st_, bc, Rs, dec, kblen_%u, %uu, k, cta, wic, watchdog, hstep, hpc, hlane, "
-      "hkind, hreg, hbfm, hmask, st_out, st_cap, %uu, img_w, rec_out, ck, ck_interval, ins);\n"
+      "hkind, hreg, hbfm, hmask, st_out, st_cap, %uu, img_w, rec_out, ck, ck_interval, ins, pgp);\n"
       "  __syncwarp();\n",
       mode, kid, n, NR);
     for (uint32_t j = 0; j < NR; ++j) o("  R%u = Rs[%uu + lane];%s", j, j * 32, (j % 8 == 7) ? "\n" : "");
@@ -610,7 +614,9 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
         if (modes & FI_JIT_GOLDEN) {
             gen_kernel(o, G, k, code + kern[k].code_off, kern[k].code_len, 1, tables);
             gen_kernel(o, G, k, code + kern[k].code_off, kern[k].code_len, 2, false);
+            tables = false;
         }
+        if (modes & FI_JIT_PAGE) gen_kernel(o, G, k, code + kern[k].code_off, kern[k].code_len, 3, tables);
     }
     const uint32_t rs = (n_regs + 1) * 32, zrow = n_regs * 32, ckw = (n_regs + 3) * 32;
     if (modes & FI_JIT_INJECT) {
@@ -638,7 +644,7 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
     for (uint32_t k = 0; k < n_kern; ++k)
         o("   case %u: kern_%u_inj(A, S.step, S.pc, S.lane, S.dst_kind, S.dst_reg, S.bfm, S.mask, S.instance, lw / wpc, "
           "lw %% wpc, watchdog, ck, ck ? ck_interval : 0u, log + (u64)i * cap, cap, o, Rs, A.dec + %uu, A.ins + %uu, "
-          "(u8*)0, (uint4*)0); break;\n",
+          "(u8*)0, (uint4*)0, (const JPage*)0); break;\n",
           k, k, kern[k].code_off, kern[k].code_off);
     o("   default: o.steps = 0; o.fired = false; o.bad = true; o.fault = 0; o.fault_pc = 0; o.nstore = 0; "
       "o.before = o.after = o.mask = 0; break;\n  }\n"
@@ -647,6 +653,38 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
       "   out[i] = r;\n   if (!o.fired || o.bad) atomicOr(status, 1u << 6);\n"
       "   const u32 start = ck ? S.step / ck_interval * ck_interval : 0u;\n"
       "   atomicAdd((unsigned long long*)(counter + 2), (unsigned long long)(o.steps - start));\n  }\n  __syncwarp();\n }\n}\n");
+    }
+    if (modes & FI_JIT_PAGE) {
+        // K8's re-execution of instance t (propagate8.cu k8_exec) on the generated kernels
+        o("extern \"C\" __global__ void __launch_bounds__(128, %u) k8_exec_jit(const JArgs A, const JK8 K, const u32 t) {\n"
+          " extern __shared__ u32 jsmem[];\n const u32 lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;\n"
+          " u32* Rs = jsmem + wib * %uu;\n Rs[%uu + lane] = 0u;\n"
+          " jfi_store* scr = K.scratch + (u64)(blockIdx.x * 4u + wib) * K.log_cap;\n"
+          " const jfi_instance in = A.inst[t];\n const u32 nw = in.warp_end - in.warp_begin, wpc = (in.block + 31u) / 32u;\n"
+          " const u64 items = (u64)(*K.n_active) * nw;\n const bool unchecked = K.flags & 1u;\n"
+          " for (;;) {\n  u32 it = 0u; if (lane == 0u) it = atomicAdd(K.work, 1u); it = __shfl_sync(JFULL, it, 0);\n"
+          "  if (it >= items) return;\n  const u32 s = K.active[it / nw], lw = it %% nw, w = in.warp_begin + lw;\n"
+          "  if (K.slot[s].overflow) continue;\n"
+          "  const u64 L = K.warp_off[w + 1] - K.warp_off[w]; const u64 wd = 10ull * L + 1024ull;\n"
+          "  const u32 watchdog = wd > 0xFFFFFFFFull ? 0xFFFFFFFFu : (u32)wd;\n"
+          "  JPage pg; pg.ptab = K.ptab + (u64)s * K.total_pages; pg.pool = K.pool; pg.page_base = K.page_base; "
+          "pg.last_ref = K.last_ref; pg.dropped = K.dropped + (u64)s * K.dwords; pg.inexact = &K.slot[s].inexact; pg.t = t;\n"
+          "  JOut o;\n  switch (in.kernel) {\n",
+          min_blocks, rs, zrow);
+        for (uint32_t k = 0; k < n_kern; ++k)
+            o("   case %u: kern_%u_page(A, 0xFFFFFFFFu, 0u, 0u, 0u, 0u, 0u, 0u, t, lw / wpc, lw %% wpc, watchdog, (u32*)0, "
+              "0u, scr, K.log_cap, o, Rs, A.dec + %uu, A.ins + %uu, (u8*)0, (uint4*)0, &pg); break;\n",
+              k, k, kern[k].code_off, kern[k].code_off);
+        o("   default: o.steps = 0; o.fault = 4; o.fault_pc = 0; o.nstore = 0; break;\n  }\n"
+          "  if (o.fault) {\n   if (lane == 0u) {\n"
+          "    const unsigned long long key = ((unsigned long long)t << 43) | ((unsigned long long)lw << 19) | "
+          "((unsigned long long)o.fault << 16) | (o.fault_pc & 0xFFFFu);\n"
+          "    if (!(unchecked && o.fault != 3u)) atomicMin(&K.slot[s].fault_key, key); "
+          "else atomicMin(&K.slot[s].pdue_key, key);\n   }\n"
+          "   if (!(unchecked && o.fault != 3u)) continue;\n  }\n"
+          "  if (o.nstore > K.log_cap) { if (lane == 0u) jk8_err(K, s, 8); continue; }\n"
+          "  jk8_updates(A, K, s, lw, scr, o.nstore, K.gst + K.gst_off[w], K.gst_off[w + 1] - K.gst_off[w], (i64)t);\n"
+          " }\n}\n");
     }
     if (modes & FI_JIT_GOLDEN) {
         // golden pass 1 (one launch per instance k, golden.cu k_golden_len) and pass 2
@@ -661,7 +699,7 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
           min_blocks, rs, zrow);
         for (uint32_t k = 0; k < n_kern; ++k)
             o("  case %u: kern_%u_len(A, 0xFFFFFFFFu, 0u, 0u, 0u, 0u, 0u, 0u, k, lw / wpc, lw %% wpc, 0xFFFFFFFFu, (u32*)0, "
-              "0u, (jfi_store*)0, 0u, o, Rs, A.dec + %uu, A.ins + %uu, img_w, (uint4*)0); break;\n",
+              "0u, (jfi_store*)0, 0u, o, Rs, A.dec + %uu, A.ins + %uu, img_w, (uint4*)0, (const JPage*)0); break;\n",
               k, k, kern[k].code_off, kern[k].code_off);
         o("  default: o.steps = 0; o.fault = 9; o.nstore = 0; break;\n }\n"
           " if (lane == 0u) { warp_len[in.warp_begin + lw] = o.steps; warp_nst[in.warp_begin + lw] = o.nstore; "
@@ -681,7 +719,8 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
           min_blocks, rs, zrow, ckw);
         for (uint32_t k = 0; k < n_kern; ++k)
             o("  case %u: kern_%u_trace(A, 0xFFFFFFFFu, 0u, 0u, 0u, 0u, 0u, 0u, k, lw / wpc, lw %% wpc, 0xFFFFFFFFu, ck, "
-              "ck ? ck_interval : 0u, gst + g0, 0xFFFFFFFFu, o, Rs, A.dec + %uu, A.ins + %uu, (u8*)0, rec + r0); break;\n",
+              "ck ? ck_interval : 0u, gst + g0, 0xFFFFFFFFu, o, Rs, A.dec + %uu, A.ins + %uu, (u8*)0, rec + r0, "
+              "(const JPage*)0); break;\n",
               k, k, kern[k].code_off, kern[k].code_off);
         o("  default: o.steps = 0; o.fault = 9; o.nstore = 0; break;\n }\n"
           " if (lane == 0u && (o.fault || o.steps != warp_off[w + 1] - r0 || o.nstore != gst_off[w + 1] - g0)) "
@@ -772,7 +811,7 @@ struct fi_jit {
     size_t smem = 0;
     uint32_t modes = 0;
     CUmodule mod = nullptr;
-    CUfunction inject = nullptr, glen = nullptr, gtrace = nullptr;
+    CUfunction inject = nullptr, glen = nullptr, gtrace = nullptr, k8exec = nullptr;
     uint32_t n_regs = 0, n_code = 0;
     double compile_s = 0;
     size_t src_bytes = 0, cubin_bytes = 0;
@@ -789,7 +828,7 @@ extern "C" const char* fi_jit_log(void) { return g_jit_log.c_str(); }
 
 extern "C" size_t fi_jit_source(const fi_insn* code_host, uint32_t n_code, const fi_kernel* kern_host, uint32_t n_kern,
                                 uint32_t n_regs, uint32_t modes, char* buf, size_t buf_bytes) {
-    if (!code_host || !kern_host || !n_kern || n_regs == 0 || n_regs > fi::kRZ || !modes || modes > 3) return 0;
+    if (!code_host || !kern_host || !n_kern || n_regs == 0 || n_regs > fi::kRZ || !modes || modes > 7) return 0;
     for (uint32_t k = 0; k < n_kern; ++k)
         if ((uint64_t)kern_host[k].code_off + kern_host[k].code_len > n_code) return 0;
     const std::string s = generate(code_host, kern_host, n_kern, n_regs, modes);
@@ -834,7 +873,7 @@ bool valid_kernels(const fi_kernel* kern, uint32_t n_kern, uint32_t n_code) {
 
 extern "C" fi_status fi_jit_compile_check(const fi_insn* code_host, uint32_t n_code, const fi_kernel* kern_host,
                                           uint32_t n_kern, uint32_t n_regs, uint32_t modes, size_t* cubin_bytes) {
-    if (!code_host || !kern_host || !n_kern || n_regs == 0 || n_regs > fi::kRZ || !modes || modes > 3) return FI_E_ARG;
+    if (!code_host || !kern_host || !n_kern || n_regs == 0 || n_regs > fi::kRZ || !modes || modes > 7) return FI_E_ARG;
     if (!valid_kernels(kern_host, n_kern, n_code)) return FI_E_ARG;
     std::string src;
     std::vector<char> cubin;
@@ -845,7 +884,7 @@ extern "C" fi_status fi_jit_compile_check(const fi_insn* code_host, uint32_t n_c
 
 extern "C" fi_status fi_jit_build(const fi_program* p, const fi_kernel* kern_host, uint32_t modes, fi_jit** out) {
     if (!p || !kern_host || !out || !p->code_host || !p->n_kern || p->n_regs == 0 || p->n_regs > fi::kRZ || !modes ||
-        modes > 3)
+        modes > 7)
         return FI_E_ARG;
     if (!valid_kernels(kern_host, p->n_kern, p->n_code)) return FI_E_ARG;
     *out = nullptr;
@@ -867,6 +906,7 @@ extern "C" fi_status fi_jit_build(const fi_program* p, const fi_kernel* kern_hos
     };
     if (modes & FI_JIT_INJECT) get(&j->inject, "k_inject_jit");
     if (modes & FI_JIT_GOLDEN) { get(&j->glen, "k_golden_len_jit"); get(&j->gtrace, "k_golden_trace_jit"); }
+    if (modes & FI_JIT_PAGE) get(&j->k8exec, "k8_exec_jit");
     if (!ok) {
         g_jit_log += "\ncuModuleLoadData / cuModuleGetFunction / cuFuncSetAttribute failed";
         if (j->mod) D.unload(j->mod);
@@ -952,6 +992,24 @@ extern "C" fi_status fi_inject_jit(const fi_jit* j, const fi_program* p, const u
                     (void*)&ck_iv, &order, &counter, &dev_status};
     return launch(j->inject, grid, j->smem, s, args);
 }
+
+namespace fi {
+// propagate8.cu's k8 loop: k8_exec of instance t on the JIT module (K = JK8 layout, jit_k8.h)
+fi_status jit_k8_exec(const fi_jit* j, const fi_program* p, const uint8_t* image, const JK8Host& K, uint32_t t,
+                      uint32_t max_grid, cudaStream_t s) {
+    if (!j || !(j->modes & FI_JIT_PAGE) || j->n_regs != p->n_regs || j->n_code != p->n_code) return FI_E_ARG;
+    int dev = 0, sms = 0, per = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    drv().occ(&per, j->k8exec, 128, j->smem);
+    const uint32_t grid = std::max<uint32_t>(1, std::min<uint32_t>((uint32_t)std::max(1, sms * std::max(1, per)), max_grid));
+    JArgsHost A = jargs(p, image);
+    JK8Host KK = K;
+    uint32_t tt = t;
+    void* args[] = {&A, &KK, &tt};
+    return launch(j->k8exec, grid, j->smem, s, args);
+}
+}  // namespace fi
 
 extern "C" fi_status fi_golden_lengths_jit(const fi_jit* j, const fi_program* p, uint8_t* image, uint64_t* warp_len,
                                            uint64_t* warp_nstore, uint32_t* dev_status, void* stream) {

@@ -351,6 +351,62 @@ __device__ __forceinline__ void jexec_plain(const JRegs& F, const uint4 D, const
     }
 }
 
+// ---------------------------------------------------------------------------
+// K8 (propagate8.cu) on the JIT module: re-execution of instance t for every
+// active replica slot over its copy-on-write pages.  Layouts mirror
+// propagate8.cu's Slot and the K8Args fields k8_exec uses.
+#define JM_PAGE 3
+#define JPAGE_WORDS 1024u
+#define JPAGE_CLAIM 0xFFFFFFFEu
+struct JSlot {
+    u32 rep, k0, alive, outcome;
+    u32 npages, inexact, overflow, pend_n;
+    u32 for_n, pdue, perm, pad1;
+    unsigned long long fault_key, pdue_key;
+};
+struct JK8 {
+    const u64* warp_off; const u64* gst_off; const jfi_store* gst;
+    JSlot* slot;
+    const u32* ptab; u32 total_pages;
+    const u32* pool; const u32* page_base; const u32* last_ref; const u32* dropped; u32 dwords;
+    jfi_store* pend; u32 pend_cap;
+    jfi_store* forn; u32 foreign_cap;
+    const u32* active; const u32* n_active; u32* work;
+    jfi_store* scratch; u32 log_cap;
+    u32 flags; u32* status;
+};
+// the replica slot's view of memory during instance t
+struct JPage {
+    const u32* ptab;             // the slot's page table
+    const u32* pool; const u32* page_base; const u32* last_ref; const u32* dropped;
+    u32* inexact; u32 t;
+};
+
+// The replica's words of an aligned access of NW words (one 4 KB page): its page
+// if it has one, else the golden value already in v.  A load from a buffer whose
+// pages were dropped after its last golden reference marks the slot inexact.
+template <u32 NW>
+__device__ __forceinline__ void jpage(const JArgs& A, const JPage& G, u64 va, uint4& v) {
+    const u64 off = va - JVA_BASE;
+    const u32 b = __ldg(&A.gran[off >> 8]);
+    const u64 rel = off - __ldg(&A.buf[b].off);
+    const u32 e = G.ptab[__ldg(&G.page_base[b]) + (u32)(rel >> 12)];
+    if (e < JPAGE_CLAIM) {
+        const u32* src = G.pool + (u64)e * JPAGE_WORDS + ((rel >> 2) & (JPAGE_WORDS - 1));
+        if (NW == 1) v.x = __ldcg(src);
+        else if (NW == 2) { const uint2 t = __ldcg(reinterpret_cast<const uint2*>(src)); v.x = t.x; v.y = t.y; }
+        else v = __ldcg(reinterpret_cast<const uint4*>(src));
+    } else if (__ldg(&G.last_ref[b]) < G.t && ((G.dropped[b >> 5] >> (b & 31)) & 1u)) {
+        *G.inexact = 1u;
+    }
+}
+__device__ __forceinline__ void jpage_n(const JArgs& A, const JPage& G, u64 va, u32 nw, uint4& v) {
+    if (nw == 1) jpage<1>(A, G, va, v);
+    else if (nw == 2) jpage<2>(A, G, va, v);
+    else jpage<4>(A, G, va, v);
+}
+
+
 // Step mode (emu.cuh's general step; MODE = JM_INJ / JM_LEN / JM_TRACE).  Returns
 // 1 when the warp is done (finished or faulted), 0 when it stands at a leader
 // whose block fits.  `ck` (JM_TRACE): the warp's checkpoint destination, or 0.
@@ -361,7 +417,8 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
                                     const u32 hlane, const u32 hkind, const u32 hreg, const u32 hbfm,
                                     const u32 hmask, jfi_store* __restrict__ st_out, const u32 st_cap,
                                     const u32 zr, u8* __restrict__ img_w, uint4* __restrict__ rec_out,
-                                    u32* __restrict__ ck, const u32 ck_interval, const u32* __restrict__ ins) {
+                                    u32* __restrict__ ck, const u32 ck_interval, const u32* __restrict__ ins,
+                                    const JPage* __restrict__ pg) {
     const u32 lane = threadIdx.x & 31, lt_mask = (1u << lane) - 1u;
     const JRegs F{reinterpret_cast<char*>(R + lane), R, zr * 128};
     const jfi_instance in = A.inst[k];
@@ -435,6 +492,7 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
                         else if (lw == 1) { const uint2 t = jld64(src); v.x = t.x; v.y = t.y; }
                         else v = jld128(src);
                     }
+                    if (MODE == JM_PAGE) jpage_n(A, *pg, va, nw, v);   // the replica's pages win
                     F.wr(id, v.x);
                     if (lw >= 1) F.wr(id + 128, v.y);
                     if (lw >= 2) { F.wr(id + 256, v.z); F.wr(id + 384, v.w); }
@@ -451,7 +509,7 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
                         else *reinterpret_cast<uint4*>(dst) = make_uint4(v[0], v[1], v[2], v[3]);
                     }
                     nst += __popc(exm) * nw;
-                } else if (MODE == JM_TRACE || step > hstep) {   // golden store log / stores after the site
+                } else if (MODE == JM_TRACE || MODE == JM_PAGE || step > hstep) {   // store logs
                     if (ex) {
                         const u32 idx = __popc(exm & lt_mask) * nw;
                         for (u32 i = 0; i < nw; ++i) {
@@ -499,4 +557,123 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
     S.pc = pc; S.live = live; S.step = step; S.livem = livem; S.conv = conv; S.upc = upc; S.amask = amask;
     S.npc = npc; S.nst = nst; S.preds = preds; S.lim = lim; S.recbuf = recbuf;
     return done;
+}
+
+__device__ __forceinline__ u32 jk8_page_of(const JArgs& A, const JK8& K, u64 va, u32& b, u32& word) {
+    const u64 off = va - JVA_BASE;
+    b = __ldg(&A.gran[off >> 8]);
+    const u64 rel = off - __ldg(&A.buf[b].off);
+    word = (u32)(rel >> 2) & (JPAGE_WORDS - 1);
+    return __ldg(&K.page_base[b]) + (u32)(rel >> 12);
+}
+// golden value of word va after instance t (t = -1: initial image)
+__device__ __forceinline__ u32 jk8_gstate(const JArgs& A, u64 va, i64 t) {
+    const i32 wr = __ldg(&A.buf[__ldg(&A.gran[(va - JVA_BASE) >> 8])].writer);
+    return (wr >= 0 && (i64)wr > t) ? 0u : __ldg(reinterpret_cast<const u32*>(A.img + (va - JVA_BASE)));
+}
+__device__ __forceinline__ u32 jk8_cur(const JArgs& A, const JK8& K, u32 s, u64 va, i64 t) {
+    u32 b, w;
+    const u32 p = jk8_page_of(A, K, va, b, w);
+    const u32 e = K.ptab[(u64)s * K.total_pages + p];
+    if (e < JPAGE_CLAIM) return __ldcg(&K.pool[(u64)e * JPAGE_WORDS + w]);
+    return jk8_gstate(A, va, t - 1);
+}
+__device__ __forceinline__ bool jk8_no_change(const JArgs& A, const JK8& K, u32 s, u64 va, u32 v, i64 t) {
+    u32 b, w;
+    const u32 p = jk8_page_of(A, K, va, b, w);
+    return K.ptab[(u64)s * K.total_pages + p] == 0xFFFFFFFFu && v == jk8_gstate(A, va, t);
+}
+__device__ __forceinline__ void jk8_err(const JK8& K, u32 s, u32 code) {
+    K.slot[s].overflow = 1;
+    atomicOr(K.status, 1u << code);
+}
+// propagate8.cu warp_updates8 with mark_foreign = true (a re-executed warp):
+// F deduplicated (last write wins) and G \ F with the replica's old values, appended
+// to the slot's pending list; F entries outside G are also "foreign" (C-14)
+__device__ void jk8_updates(const JArgs& A, const JK8& K, u32 s, u32 w_idx, const jfi_store* F, u64 nF,
+                            const jfi_store* G, u64 nG, i64 t) {
+    const u32 lane = threadIdx.x & 31;
+    jfi_store* pend = K.pend + (u64)s * K.pend_cap;
+    bool same = nF == nG;
+    for (u64 b = 0; b < nF && same; b += 32) {
+        const u64 j = b + lane;
+        same = __all_sync(JFULL, j >= nF || F[j].va == G[j].va);
+    }
+    if (same) {
+        for (u64 b = 0; b < nF; b += 32) {
+            const u64 j = b + lane;
+            jfi_store f; f.va = 0; f.value = 0; f.step = 0;
+            bool keep = false;
+            if (j < nF) {
+                f = F[j];
+                f.step = w_idx;
+                keep = !jk8_no_change(A, K, s, f.va, f.value, t);
+            }
+            const u32 m = __ballot_sync(JFULL, keep);
+            u32 base = 0;
+            if (lane == 0 && m) base = atomicAdd(&K.slot[s].pend_n, (u32)__popc(m));
+            base = __shfl_sync(JFULL, base, 0);
+            if (keep) {
+                const u32 pos = base + __popc(m & ((1u << lane) - 1));
+                if (pos < K.pend_cap) pend[pos] = f;
+                else jk8_err(K, s, 8);
+            }
+        }
+        return;
+    }
+    for (u64 b = 0; b < nF; b += 32) {
+        const u64 j = b + lane;
+        bool keep = false, foreign = false;
+        jfi_store f; f.va = 0; f.value = 0; f.step = 0;
+        if (j < nF) {
+            f = F[j];
+            keep = true;
+            for (u64 q = j + 1; q < nF && keep; ++q) keep = F[q].va != f.va;
+            if (keep) {
+                foreign = true;
+                for (u64 q = 0; q < nG && foreign; ++q) foreign = G[q].va != f.va;
+            }
+            if (keep && !foreign && jk8_no_change(A, K, s, f.va, f.value, t)) keep = false;
+        }
+        const u32 m = __ballot_sync(JFULL, keep);
+        u32 base = 0;
+        if (lane == 0 && m) base = atomicAdd(&K.slot[s].pend_n, (u32)__popc(m));
+        base = __shfl_sync(JFULL, base, 0);
+        if (keep) {
+            const u32 pos = base + __popc(m & ((1u << lane) - 1));
+            f.step = w_idx | (foreign ? 0x80000000u : 0u);
+            if (pos < K.pend_cap) pend[pos] = f;
+            else jk8_err(K, s, 8);
+            if (foreign) {
+                const u32 fp = atomicAdd(&K.slot[s].for_n, 1u);
+                if (fp < K.foreign_cap) K.forn[(u64)s * K.foreign_cap + fp] = f;
+                else jk8_err(K, s, 8);
+            }
+        }
+    }
+    for (u64 b = 0; b < nG; b += 32) {
+        const u64 j = b + lane;
+        bool keep = false;
+        jfi_store g; g.va = 0; g.value = 0; g.step = 0;
+        if (j < nG) {
+            const u64 va = G[j].va;
+            bool inF = false;
+            for (u64 q = 0; q < nF && !inF; ++q) inF = F[q].va == va;
+            if (!inF) {
+                g.va = va;
+                g.value = jk8_cur(A, K, s, va, t);
+                g.step = w_idx;
+                keep = !jk8_no_change(A, K, s, va, g.value, t);
+            }
+        }
+        const u32 m = __ballot_sync(JFULL, keep);
+        u32 base = 0;
+        if (lane == 0 && m) base = atomicAdd(&K.slot[s].pend_n, (u32)__popc(m));
+        base = __shfl_sync(JFULL, base, 0);
+        if (keep) {
+            const u32 pos = base + __popc(m & ((1u << lane) - 1));
+            if (pos < K.pend_cap) pend[pos] = g;
+            else jk8_err(K, s, 8);
+        }
+    }
 }

@@ -30,6 +30,7 @@
 #include <vector>
 
 #include "emu.cuh"
+#include "jit_k8.h"
 
 namespace fi {
 size_t golden_smem(uint32_t n_regs);
@@ -628,7 +629,9 @@ extern "C" size_t fi_classify_batched_workspace(const fi_program* p, uint32_t n,
 static fi_status k8_run(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
                         const fi_pfault* pf, const uint64_t* opw, uint32_t n, fi_inj* out, const fi_store* log,
                         uint32_t log_cap, uint64_t* hist, uint32_t flags, uint32_t batch, uint32_t pool_pages,
-                        uint32_t pend_cap, void* ws, size_t ws_bytes, uint32_t* dev_status, void* stream) {
+                        uint32_t pend_cap, void* ws, size_t ws_bytes, uint32_t* dev_status, void* stream,
+                        const fi_jit* jit = nullptr) {
+    if (jit && pf) return FI_E_ARG;                  // the JIT engine serves transient faults
     if (!p || !image || !t || (!sites && !pf) || !out || !hist || !dev_status || !p->aux || !p->inst_host ||
         !p->code_host)
         return FI_E_ARG;
@@ -737,6 +740,9 @@ static fi_status k8_run(const fi_program* p, const uint8_t* image, const fi_trac
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k8_exec, kWPB8 * 32, smem);
     const uint32_t exec_grid = std::min<uint32_t>((uint32_t)std::max(1, sms * std::max(1, per)), sw / kWPB8);
     const uint32_t fix_grid = (uint32_t)std::max(1, sms * 4);
+    JK8Host JK{A.warp_off, A.gst_off, A.gst, A.slot, A.ptab, A.total_pages, A.pool, A.page_base, A.last_ref,
+               A.dropped, A.dwords, A.pend, A.pend_cap, A.forn, kForeignCap, A.active, A.n_active, A.work,
+               A.scratch, A.log_cap, A.flags, A.status};
 
     for (uint32_t b0 = 0; b0 < n; b0 += batch) {
         const uint32_t nb = std::min(batch, n - b0);
@@ -750,7 +756,13 @@ static fi_status k8_run(const fi_program* p, const uint8_t* image, const fi_trac
         if ((e = launch_status())) return e;
         for (uint32_t tt = kmin; tt < p->n_inst; ++tt) {
             k8_activate<<<1, 1024, 0, s>>>(A, tt);
-            if (tt > kmin || pf) k8_exec<<<exec_grid, kWPB8 * 32, smem, s>>>(A, tt);
+            if (tt > kmin || pf) {
+                if (jit) {
+                    if ((e = jit_k8_exec(jit, p, image, JK, tt, sw / kWPB8, s))) return e;
+                } else {
+                    k8_exec<<<exec_grid, kWPB8 * 32, smem, s>>>(A, tt);
+                }
+            }
             k8_k0<<<(batch + kWPB8 - 1) / kWPB8, kWPB8 * 32, 0, s>>>(A, tt);
             k8_mark<<<dim3(std::max<uint32_t>(1, fix_grid / batch + 1), batch), 256, 0, s>>>(A);
             k8_alloc<<<fix_grid, 256, 0, s>>>(A, tt);
@@ -773,6 +785,16 @@ extern "C" fi_status fi_classify_batched(const fi_program* p, const uint8_t* ima
     if (!sites) return FI_E_ARG;
     return k8_run(p, image, t, sites, nullptr, nullptr, n, out, log, log_cap, hist, flags, batch, pool_pages,
                   pend_cap, ws, ws_bytes, dev_status, stream);
+}
+
+extern "C" fi_status fi_classify_batched_jit(const fi_jit* j, const fi_program* p, const uint8_t* image,
+                                             const fi_trace* t, const fi_site* sites, uint32_t n, fi_inj* out,
+                                             const fi_store* log, uint32_t log_cap, uint64_t* hist, uint32_t flags,
+                                             uint32_t batch, uint32_t pool_pages, uint32_t pend_cap, void* ws,
+                                             size_t ws_bytes, uint32_t* dev_status, void* stream) {
+    if (!sites || !j) return FI_E_ARG;
+    return k8_run(p, image, t, sites, nullptr, nullptr, n, out, log, log_cap, hist, flags, batch, pool_pages,
+                  pend_cap, ws, ws_bytes, dev_status, stream, j);
 }
 
 extern "C" fi_status fi_inject_permanent_batched(const fi_program* p, const uint8_t* image, const fi_trace* t,

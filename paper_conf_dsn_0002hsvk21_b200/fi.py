@@ -105,7 +105,7 @@ class fi_campaign_result(C.Structure):
 ALLREDUCE_FN = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_uint64, C.c_uint32, C.c_void_p, C.c_void_p)
 FI_PROPAGATION = {"auto": 0, "k7": 1, "k8": 2}
 FI_CKPT_AUTO = 0xFFFFFFFF
-FI_JIT_INJECT, FI_JIT_GOLDEN = 1, 2
+FI_JIT_INJECT, FI_JIT_GOLDEN, FI_JIT_PAGE = 1, 2, 4
 
 _lib = None
 
@@ -152,6 +152,8 @@ def lib():
             "fi_inject_permanent_batched": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, u32, u32, u32, u32, vp, sz,
                                                  vp, vp]),
             "fi_classify_batched": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, u32, u32, u32, u32, vp, sz, vp, vp]),
+            "fi_classify_batched_jit": (st, [vp, vp, vp, vp, vp, u32, vp, vp, u32, vp, u32, u32, u32, u32, vp, sz, vp,
+                                             vp]),
             "fi_inject_permanent": (st, [vp, vp, vp, vp, u32, vp, vp, vp, u32, u32, vp, u32, vp, sz, vp, vp]),
             "fi_jit_build": (st, [vp, vp, u32, C.POINTER(vp)]),
             "fi_jit_free": (None, [vp]),
@@ -576,9 +578,10 @@ def pend_capacity(gt: GoldenTrace) -> int:
 def classify_batched(gt: GoldenTrace, sites: torch.Tensor, n: int, out: torch.Tensor, log: torch.Tensor,
                      log_cap: int, hist: torch.Tensor | None = None, unchecked: bool = False, batch: int | None = None,
                      pool_pages: int | None = None, pend_cap: int | None = None, mem_budget: int = 24 << 30,
-                     status: DeviceStatus | None = None) -> torch.Tensor:
+                     status: DeviceStatus | None = None, engine: str = "interp") -> torch.Tensor:
     """fi_classify_batched (K8): whole-program outcomes for long multi-instance
-    programs, replica batches in lockstep over the launches."""
+    programs, replica batches in lockstep over the launches.  engine "jit":
+    fi_classify_batched_jit (re-execution on the program's JIT module)."""
     dev = gt.dp.device
     if hist is None:
         hist = torch.zeros((8, 4, 3), dtype=torch.int64, device=dev)
@@ -593,9 +596,15 @@ def classify_batched(gt: GoldenTrace, sites: torch.Tensor, n: int, out: torch.Te
     ws_n = lib().fi_classify_batched_workspace(C.byref(gt.dp.c), n, log_cap, batch, pool_pages, pend_cap)
     ws = torch.empty(ws_n, dtype=torch.uint8, device=dev)
     st = status or DeviceStatus(dev)
-    _check(lib().fi_classify_batched(C.byref(gt.dp.c), _p(gt.image), C.byref(gt.c), _p(sites), n, _p(out), _p(log),
-                                     log_cap, _p(hist), FI_UNCHECKED if unchecked else 0, batch, pool_pages, pend_cap,
-                                     _p(ws), ws_n, st.ptr, _stream()), "fi_classify_batched")
+    if engine == "jit":
+        _check(lib().fi_classify_batched_jit(gt.dp.jit(FI_JIT_PAGE).h, C.byref(gt.dp.c), _p(gt.image), C.byref(gt.c),
+                                             _p(sites), n, _p(out), _p(log), log_cap, _p(hist),
+                                             FI_UNCHECKED if unchecked else 0, batch, pool_pages, pend_cap, _p(ws),
+                                             ws_n, st.ptr, _stream()), "fi_classify_batched_jit")
+    else:
+        _check(lib().fi_classify_batched(C.byref(gt.dp.c), _p(gt.image), C.byref(gt.c), _p(sites), n, _p(out),
+                                         _p(log), log_cap, _p(hist), FI_UNCHECKED if unchecked else 0, batch,
+                                         pool_pages, pend_cap, _p(ws), ws_n, st.ptr, _stream()), "fi_classify_batched")
     if status is None:
         st.check("fi_classify_batched")
     return hist

@@ -116,3 +116,41 @@ def test_jit_golden_passes(F, maker, ckpt):
 @pytest.mark.parametrize("which", range(5))
 def test_jit_golden_c5_minis(F, which):
     _golden_both(F, H.c5(full=False)[which], 7)
+
+
+def _k8_both(F, prog, seed, groups, bfms, n, unchecked=False, **kw):
+    dp = F.DeviceProgram(prog)
+    gt = F.golden_run(dp)
+    ic, cc = F.profile(gt)
+    sites = F.select_sites(F.SiteIndex(gt, ic, cc), F.schedule(seed, groups, bfms), 0, n)
+    cap = F.log_capacity(gt)
+    out, log = F.inject(gt, sites, n, cap)
+    res = {}
+    for eng in ("interp", "jit"):
+        o = out.clone()
+        h = F.classify_batched(gt, sites, n, o, log, cap, unchecked=unchecked, engine=eng, **kw)
+        torch.cuda.synchronize()
+        res[eng] = (F.as_numpy(o, F.INJ_DTYPE, n).copy(), h.cpu().numpy())
+    a, b = res["interp"][0], res["jit"][0]
+    for f in a.dtype.names:
+        bad = np.flatnonzero(a[f] != b[f])
+        assert bad.size == 0, f"{f}: replica {bad[0]} interp {a[bad[0]]} jit {b[bad[0]]}"
+    assert np.array_equal(res["interp"][1], res["jit"][1])
+    return a
+
+
+@pytest.mark.parametrize("maker,unchecked", [(lambda: P.multi_instance_chain(6, shrink=29), False),
+                                             (lambda: P.multi_instance_chain(4, n=300, block=96), True),
+                                             (P.scatter_chain, False), (P.scatter_chain, True),
+                                             (lambda: P.c3(full=False), False), (lambda: RN.c4(full=False), False)])
+def test_jit_k8(F, maker, unchecked):
+    """K8's per-launch re-execution on the JIT module (fi_classify_batched_jit):
+    outcomes, flags, first downstream faults and histograms identical to the
+    interpreter's K8 (which test_gpu_batched.py pins to the oracle)."""
+    a = _k8_both(F, maker(), 0x5A5, [F.G_GP, F.G_LD, F.G_OTHERS], [0, 1, 2, 3], 300, unchecked)
+    assert (a["outcome"] == F.SDC).sum() > 0
+
+
+@pytest.mark.parametrize("which", range(5))
+def test_jit_k8_c5_minis(F, which):
+    _k8_both(F, H.c5(full=False)[which], 0xC5C5, [F.G_GP, F.G_GPPR], [0], 200, batch=64)
