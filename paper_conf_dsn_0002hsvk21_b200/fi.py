@@ -258,16 +258,23 @@ class DeviceProgram:
         return len(self.prog.instances)
 
     def jit(self, modes: int = FI_JIT_INJECT) -> "Jit":
-        """The program's JIT-specialised emulator module (fi_jit_build) for `modes`,
-        built once per (code, kernel table, register rows, modes, device) in this process."""
-        if modes not in self._jit:
-            import hashlib
-            key = (hashlib.sha1(self._code_host.tobytes() + self._kern_host.tobytes()).hexdigest(), self.n_regs, modes,
-                   self.device.index if self.device.index is not None else torch.cuda.current_device())
-            if key not in _JIT_CACHE:
-                _JIT_CACHE[key] = Jit(self, modes)
-            self._jit[modes] = _JIT_CACHE[key]
-        return self._jit[modes]
+        """The program's JIT-specialised emulator module (fi_jit_build) holding
+        `modes` — any module already built with a superset is reused; else one is
+        built and cached per (code, kernel table, register rows, modes, device)."""
+        for m, j in self._jit.items():
+            if m & modes == modes:
+                return j
+        import hashlib
+        base = (hashlib.sha1(self._code_host.tobytes() + self._kern_host.tobytes()).hexdigest(), self.n_regs,
+                self.device.index if self.device.index is not None else torch.cuda.current_device())
+        for (b, m), j in _JIT_CACHE.items():
+            if b == base and m & modes == modes:
+                self._jit[m] = j
+                return j
+        j = Jit(self, modes)
+        _JIT_CACHE[(base, modes)] = j
+        self._jit[modes] = j
+        return j
 
     @property
     def n_warps(self):

@@ -31,10 +31,18 @@ def timed(f, reps=1):
     return r, best
 
 
+ENGINE = os.environ.get("FI_ENGINE", "jit")        # jit | interp
+
+
 def run(name, prog, seed, n, batch):
-    t0 = time.time()
     dp = fi.DeviceProgram(prog)
-    gt = fi.golden_run(dp)
+    jit_s = 0.0
+    if ENGINE == "jit":                               # one module: golden passes, K4, K8 (setup, reported)
+        t0 = time.time()
+        dp.jit(fi.FI_JIT_INJECT | fi.FI_JIT_GOLDEN | fi.FI_JIT_PAGE)
+        jit_s = time.time() - t0
+    t0 = time.time()
+    gt = fi.golden_run(dp, engine=ENGINE)
     torch.cuda.synchronize()
     golden_s = time.time() - t0
     (ic, cc), prof_ms = timed(lambda: fi.profile(gt), reps=3)
@@ -45,8 +53,8 @@ def run(name, prog, seed, n, batch):
     idx, idx_ms = timed(lambda: fi.SiteIndex(gt, ic, cc))
     sites, sel_ms = timed(lambda: fi.select_sites(idx, fi.schedule(seed, [fi.G_GP], [0]), 0, n))
     cap = fi.log_capacity(gt)
-    (out, log), k4_ms = timed(lambda: fi.inject(gt, sites, n, cap))
-    hist, k8_ms = timed(lambda: fi.classify_batched(gt, sites, n, out, log, cap, batch=batch))
+    (out, log), k4_ms = timed(lambda: fi.inject(gt, sites, n, cap, engine=ENGINE))
+    hist, k8_ms = timed(lambda: fi.classify_batched(gt, sites, n, out, log, cap, batch=batch, engine=ENGINE))
     inj = fi.as_numpy(out, fi.INJ_DTYPE, n)
     oc = np.bincount(np.minimum(inj["outcome"], 4), minlength=5)
     line = {"program": name, "instances": dp.n_inst, "static_kernels": len(prog.kernels), "warps": dp.n_warps,
@@ -58,7 +66,7 @@ def run(name, prog, seed, n, batch):
             "outcomes": {"masked": int(oc[0]), "sdc": int(oc[1]), "due": int(oc[2]),
                          "unclassified_wild_load": int(((inj["outcome"] == 0xFF) & (inj["flags"] & 4 > 0)).sum()),
                          "unclassified_capacity": int(((inj["outcome"] == 0xFF) & (inj["flags"] & 2 > 0)).sum())},
-            "group": "G_GP", "bfm": "FLIP_SINGLE_BIT"}
+            "group": "G_GP", "bfm": "FLIP_SINGLE_BIT", "engine": ENGINE, "jit_compile_s": jit_s}
     print(json.dumps(line), flush=True)
     del gt, dp
     torch.cuda.empty_cache()
