@@ -65,11 +65,14 @@ class Campaign:
     program on this rank's GPU (all work in libfi kernels)."""
 
     def __init__(self, prog, seed: int, groups, bfms, n_replicas: int, rank: int = 0, world: int = 1,
-                 device="cuda", group=None, host_tensors: dict | None = None, propagation: str = "auto"):
+                 device="cuda", group=None, host_tensors: dict | None = None, propagation: str = "auto",
+                 engine: str = "jit"):
         """propagation: how a multi-launch program's outcome is computed — "k7"
         (fi_classify: one CUDA warp walks a replica's later launches), "k8"
         (fi_classify_batched: replica batches in lockstep over the launches), or
-        "auto" (K8 from 64 launches on).  Both give identical results."""
+        "auto" (K8 from 64 launches on).  Both give identical results.
+        engine: "jit" (golden passes, K4 and K8 on the program's JIT module, built
+        once here) or "interp" (the shared-memory interpreter); identical results."""
         from . import fi
         self.fi = fi
         self.prog = prog
@@ -79,7 +82,11 @@ class Campaign:
         self.n = n_replicas
         self.j0, self.j1 = replica_block(n_replicas, rank, world)
         self.dp = fi.DeviceProgram(prog, self.device, host_tensors)
-        self.gt = fi.golden_run(self.dp)
+        self.engine = engine
+        self.batched = propagation == "k8" or (propagation == "auto" and self.dp.n_inst >= 64)
+        if engine == "jit":
+            self.dp.jit(fi.FI_JIT_INJECT | fi.FI_JIT_GOLDEN | (fi.FI_JIT_PAGE if self.batched else 0))
+        self.gt = fi.golden_run(self.dp, engine=engine)
         self.r0, self.r1 = record_shard(self.gt.n_rec, rank, world)
         self.cap = fi.log_capacity(self.gt)
         nloc = max(self.j1 - self.j0, 1)
@@ -92,7 +99,6 @@ class Campaign:
         self.hist = torch.zeros((8, 4, 3), dtype=torch.int64, device=self.device)
         self.status = fi.DeviceStatus(self.device)
         self.inj_ws = torch.empty(fi.lib().fi_inject_workspace(nloc), dtype=torch.uint8, device=self.device)
-        self.batched = propagation == "k8" or (propagation == "auto" and self.dp.n_inst >= 64)
 
     @property
     def n_local(self):
@@ -120,11 +126,12 @@ class Campaign:
         n = self.n_local
         fi.select_sites(idx, self.sched, self.j0, n, self.sites, self.status)
         mark("select")
-        fi.inject(self.gt, self.sites, n, self.cap, self.out, self.log, self.status, self.inj_ws)
+        fi.inject(self.gt, self.sites, n, self.cap, self.out, self.log, self.status, self.inj_ws, engine=self.engine)
         mark("inject")
         self.hist.zero_()
         if self.batched:
-            fi.classify_batched(self.gt, self.sites, n, self.out, self.log, self.cap, self.hist, status=self.status)
+            fi.classify_batched(self.gt, self.sites, n, self.out, self.log, self.cap, self.hist, status=self.status,
+                                engine=self.engine)
         else:
             fi.classify(self.gt, self.sites, n, self.out, self.log, self.cap, self.hist, self.status)
         mark("classify")

@@ -85,19 +85,21 @@ struct OwnedStream {
 
 // JIT modules built by fi_campaign, per (program code, kernel table, register
 // rows, device): compiled once per process, reused by later campaigns.
-fi_status cached_jit(const fi_program& p, const fi_kernel* kern_host, int dev, fi_jit** out, float* ms) {
+fi_status cached_jit(const fi_program& p, const fi_kernel* kern_host, int dev, uint32_t modes, fi_jit** out,
+                     float* ms) {
     static std::mutex mu;
     static std::map<std::string, fi_jit*> cache;
     std::string key((const char*)p.code_host, sizeof(fi_insn) * p.n_code);
     key.append((const char*)kern_host, sizeof(fi_kernel) * p.n_kern);
     key.append((const char*)&p.n_regs, 4);
     key.append((const char*)&dev, sizeof dev);
+    key.append((const char*)&modes, sizeof modes);
     std::lock_guard<std::mutex> g(mu);
     auto it = cache.find(key);
     if (it != cache.end()) { *out = it->second; *ms = 0.f; return FI_OK; }
     const auto t0 = std::chrono::steady_clock::now();
     fi_jit* j = nullptr;
-    FI_TRY(fi_jit_build(&p, kern_host, FI_JIT_INJECT | FI_JIT_GOLDEN, &j));
+    FI_TRY(fi_jit_build(&p, kern_host, modes, &j));
     *ms = std::chrono::duration<float, std::milli>(std::chrono::steady_clock::now() - t0).count();
     cache[key] = j;
     *out = j;
@@ -161,10 +163,11 @@ extern "C" fi_status fi_campaign(const fi_campaign_cfg* cfg, int rank, int world
     // JIT engine: the program's module (golden passes + K4), built once per process
     fi_jit* jit = nullptr;
     float ms_jit = 0.f;
+    const bool k8 = cfg->propagation == FI_PROPAGATION_K8 || (cfg->propagation == FI_PROPAGATION_AUTO && K >= 64);
     if (cfg->engine == FI_ENGINE_JIT) {
         int dev = 0;
         FI_TRY(cu(cudaGetDevice(&dev)));
-        FI_TRY(cached_jit(p, cfg->kern, dev, &jit, &ms_jit));
+        FI_TRY(cached_jit(p, cfg->kern, dev, FI_JIT_INJECT | FI_JIT_GOLDEN | (k8 ? FI_JIT_PAGE : 0u), &jit, &ms_jit));
     }
     FI_TRY(ev.mark(s));                                                    // 1
 
@@ -303,7 +306,6 @@ extern "C" fi_status fi_campaign(const fi_campaign_cfg* cfg, int rank, int world
     uint64_t* hist;
     FI_TRY(A.alloc(&hist, sizeof(res->hist)));
     FI_TRY(cu(cudaMemsetAsync(hist, 0, sizeof(res->hist), s)));
-    const bool k8 = cfg->propagation == FI_PROPAGATION_K8 || (cfg->propagation == FI_PROPAGATION_AUTO && K >= 64);
     if (n && k8) {
         // pend_cap: 2x the largest launch's golden stores + 4096 (fi.py pend_capacity)
         uint64_t mx_l = 0;
@@ -321,8 +323,12 @@ extern "C" fi_status fi_campaign(const fi_campaign_cfg* cfg, int rank, int world
         const size_t kws = fi_classify_batched_workspace(&p, n, log_cap, batch, pool, pend);
         void* kw;
         FI_TRY(A.alloc(&kw, kws));
-        FI_TRY(fi_classify_batched(&p, image, &t, sites, n, inj, log, log_cap, hist, cfg->flags, batch, pool, pend,
-                                   kw, kws, st, s));
+        if (jit)
+            FI_TRY(fi_classify_batched_jit(jit, &p, image, &t, sites, n, inj, log, log_cap, hist, cfg->flags, batch,
+                                           pool, pend, kw, kws, st, s));
+        else
+            FI_TRY(fi_classify_batched(&p, image, &t, sites, n, inj, log, log_cap, hist, cfg->flags, batch, pool,
+                                       pend, kw, kws, st, s));
     } else if (n) {
         const size_t cws = fi_classify_workspace(K, n, log_cap);
         void* cw = nullptr;

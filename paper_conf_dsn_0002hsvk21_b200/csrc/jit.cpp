@@ -305,16 +305,16 @@ struct Gen {
         rec(o, I, pc, stepx, "pv");
         o("const u64 va = %s + (u64)(i64)(i32)%s; ", R64(I.a).c_str(), hex(I.imm).c_str());
         if (I.op == LDG) {
-            o("uint4 v_; const u32 c_ = jldg<%uu>(A, bc, va, k, ex, v_); ", lw);
+            o("uint4 v_; const u32 c_ = jldg<%uu>(A, bc, va, k, ex, v_%s); ", lw, mode == 3 ? ", PG.page_base" : "");
             o("if (__ballot_sync(JFULL, c_ != 0u)) { fault = __ballot_sync(JFULL, c_ == 1u) ? 1u : 2u; fault_pc = %uu; "
               "step = %s; goto finish; } ", pc, stepx);
-            if (mode == 3) o("if (ex) jpage<%uu>(A, PG, va, v_); ", nw);
+            if (mode == 3) o("if (ex) jpage_c<%uu>(bc, PG, va, v_); ", nw);
             const char* v[] = {"v_.x", "v_.y", "v_.z", "v_.w"};
             wr(o, I.d0, v, nw);
             o("}\n");
         } else {
             o("const u32 exm_ = amask & __ballot_sync(JFULL, pv); bool z_ = false; "
-              "const u32 c_ = ex ? jcheck(A, bc, va, %uu, k, &z_) : 0u; ", 4u << lw);
+              "const u32 c_ = ex ? jcheck(A, bc, va, %uu, k, &z_%s) : 0u; ", 4u << lw, mode == 3 ? ", PG.page_base" : "");
             o("if (__ballot_sync(JFULL, c_ != 0u)) { fault = __ballot_sync(JFULL, c_ == 1u) ? 1u : 2u; fault_pc = %uu; "
               "step = %s; goto finish; } ", pc, stepx);
             if (mode == 1) {                           // golden pass 1: into the image
@@ -365,7 +365,8 @@ struct Gen {
         for (uint32_t j = 0; j < m; ++j) {
             const fi_insn& I = code[i0 + j];
             const uint32_t lw = (I.mod & 3) > 2 ? 2 : (I.mod & 3);
-            o("   c%u = ex%u ? jcheck(A, bc, va%u, %uu, k, &z%u) : 0u;\n", j, j, j, 4u << lw, j);
+            o("   c%u = ex%u ? jcheck(A, bc, va%u, %uu, k, &z%u%s) : 0u;\n", j, j, j, 4u << lw, j,
+              mode == 3 ? ", PG.page_base" : "");
         }
         o("  }\n");
         o("  if (__ballot_sync(JFULL, 0u");
@@ -391,7 +392,7 @@ struct Gen {
             if (lw == 0) o("v_.x = jld32(p_); } ");
             else if (lw == 1) o("const uint2 t_ = jld64(p_); v_.x = t_.x; v_.y = t_.y; } ");
             else o("v_ = jld128(p_); } ");
-            if (mode == 3) o("jpage<%uu>(A, PG, va%u, v_); ", nw, j);
+            if (mode == 3) o("jpage_c<%uu>(bc, PG, va%u, v_); ", nw, j);
             if (I.d0 != fi::kRZ)
                 for (uint32_t q = 0; q < nw; ++q)
                     if (W(I.d0 + q)) o("R%u = v_.%c; ", I.d0 + q, "xyzw"[q]);

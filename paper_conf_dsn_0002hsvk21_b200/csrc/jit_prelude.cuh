@@ -150,11 +150,14 @@ __device__ __forceinline__ uint4 jld128(const u8* p) {
 struct JBufCache {
     u64 lo0, hi0, lo1, hi1;
     bool z0, z1;
-    __device__ __forceinline__ JBufCache() : lo0(1), hi0(0), lo1(1), hi1(0), z0(false), z1(false) {}
+    u32 b0, b1, pb0, pb1;        // buffer ids and their first page index (K8 page tables; 0 elsewhere)
+    __device__ __forceinline__ JBufCache()
+        : lo0(1), hi0(0), lo1(1), hi1(0), z0(false), z1(false), b0(0), b1(0), pb0(0), pb1(0) {}
 };
 
 // 0 ok, 1 misaligned, 2 unmapped (C-15); *zero = writer rule for instance k
-__device__ __forceinline__ u32 jcheck(const JArgs& A, JBufCache& C, u64 va, u32 w, u32 k, bool* zero) {
+__device__ __forceinline__ u32 jcheck(const JArgs& A, JBufCache& C, u64 va, u32 w, u32 k, bool* zero,
+                                      const u32* page_base = nullptr) {
     if (va & (w - 1)) return 1;
     const u64 off = va - JVA_BASE;
     // (off < hi first: an address just below the VA base wraps off + w around)
@@ -166,8 +169,9 @@ __device__ __forceinline__ u32 jcheck(const JArgs& A, JBufCache& C, u64 va, u32 
     const u64 lo = __ldg(&A.buf[b].off), hi = lo + __ldg(&A.buf[b].size);
     if (off + w > hi) return 2;
     const i32 wr = __ldg(&A.buf[b].writer);
-    C.lo1 = C.lo0; C.hi1 = C.hi0; C.z1 = C.z0;
-    C.lo0 = lo; C.hi0 = hi; C.z0 = wr >= 0 && (u32)wr >= k;
+    C.lo1 = C.lo0; C.hi1 = C.hi0; C.z1 = C.z0; C.b1 = C.b0; C.pb1 = C.pb0;
+    C.lo0 = lo; C.hi0 = hi; C.z0 = wr >= 0 && (u32)wr >= k; C.b0 = b;
+    C.pb0 = page_base ? __ldg(&page_base[b]) : 0u;
     *zero = C.z0;
     return 0;
 }
@@ -184,9 +188,10 @@ __device__ __forceinline__ bool jhit(const JBufCache& C, u64 va, u32 w, bool* ze
 
 // one LDG of 1/2/4 words for this lane; returns the fault code (0 ok)
 template <u32 LW>
-__device__ __forceinline__ u32 jldg(const JArgs& A, JBufCache& C, u64 va, u32 k, bool ex, uint4& v) {
+__device__ __forceinline__ u32 jldg(const JArgs& A, JBufCache& C, u64 va, u32 k, bool ex, uint4& v,
+                                    const u32* page_base = nullptr) {
     bool zero = false;
-    const u32 c = ex ? jcheck(A, C, va, 4u << LW, k, &zero) : 0u;
+    const u32 c = ex ? jcheck(A, C, va, 4u << LW, k, &zero, page_base) : 0u;
     v = make_uint4(0, 0, 0, 0);
     if (ex && !c && !zero) {
         const u8* src = A.img + (va - JVA_BASE);
@@ -400,6 +405,23 @@ __device__ __forceinline__ void jpage(const JArgs& A, const JPage& G, u64 va, ui
         *G.inexact = 1u;
     }
 }
+// the same through the lane's buffer cache (entry of the checked access): one page-table load
+template <u32 NW>
+__device__ __forceinline__ void jpage_c(const JBufCache& C, const JPage& G, u64 va, uint4& v) {
+    const u64 off = va - JVA_BASE;
+    const bool e0 = off >= C.lo0 && off < C.hi0;
+    const u64 rel = off - (e0 ? C.lo0 : C.lo1);
+    const u32 b = e0 ? C.b0 : C.b1;
+    const u32 e = G.ptab[(e0 ? C.pb0 : C.pb1) + (u32)(rel >> 12)];
+    if (e < JPAGE_CLAIM) {
+        const u32* src = G.pool + (u64)e * JPAGE_WORDS + ((rel >> 2) & (JPAGE_WORDS - 1));
+        if (NW == 1) v.x = __ldcg(src);
+        else if (NW == 2) { const uint2 t = __ldcg(reinterpret_cast<const uint2*>(src)); v.x = t.x; v.y = t.y; }
+        else v = __ldcg(reinterpret_cast<const uint4*>(src));
+    } else if (__ldg(&G.last_ref[b]) < G.t && ((G.dropped[b >> 5] >> (b & 31)) & 1u)) {
+        *G.inexact = 1u;
+    }
+}
 __device__ __forceinline__ void jpage_n(const JArgs& A, const JPage& G, u64 va, u32 nw, uint4& v) {
     if (nw == 1) jpage<1>(A, G, va, v);
     else if (nw == 2) jpage<2>(A, G, va, v);
@@ -476,7 +498,7 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
             const u32 lw = (mod & 3) > 2 ? 2 : (mod & 3), nw = 1u << lw, w = 4u << lw;
             const u64 va = F.rd64(ia) + (u64)(i64)(i32)imm;
             bool zero = false;
-            const u32 c = ex ? jcheck(A, bc, va, w, k, &zero) : 0u;
+            const u32 c = ex ? jcheck(A, bc, va, w, k, &zero, MODE == JM_PAGE ? pg->page_base : nullptr) : 0u;
             if (__ballot_sync(JFULL, c != 0u)) {      // memory fault: DUE (C-9); the step has no effect
                 S.fault = __ballot_sync(JFULL, c == 1u) ? 1u : 2u;
                 S.fault_pc = pcm;
@@ -492,7 +514,11 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
                         else if (lw == 1) { const uint2 t = jld64(src); v.x = t.x; v.y = t.y; }
                         else v = jld128(src);
                     }
-                    if (MODE == JM_PAGE) jpage_n(A, *pg, va, nw, v);   // the replica's pages win
+                    if (MODE == JM_PAGE) {            // the replica's pages win
+                        if (nw == 1) jpage_c<1>(bc, *pg, va, v);
+                        else if (nw == 2) jpage_c<2>(bc, *pg, va, v);
+                        else jpage_c<4>(bc, *pg, va, v);
+                    }
                     F.wr(id, v.x);
                     if (lw >= 1) F.wr(id + 128, v.y);
                     if (lw >= 2) { F.wr(id + 256, v.z); F.wr(id + 384, v.w); }
