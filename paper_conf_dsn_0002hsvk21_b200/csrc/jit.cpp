@@ -305,10 +305,10 @@ struct Gen {
         rec(o, I, pc, stepx, "pv");
         o("const u64 va = %s + (u64)(i64)(i32)%s; ", R64(I.a).c_str(), hex(I.imm).c_str());
         if (I.op == LDG) {
-            o("uint4 v_; const u32 c_ = jldg<%uu>(A, bc, va, k, ex, v_%s); ", lw, mode == 3 ? ", PG.page_base" : "");
+            o("uint4 v_; const u32 c_ = jldg<%uu>(A, jimg, bc, va, k, ex, v_%s); ", lw, mode == 3 ? ", PG.page_base" : "");
             o("if (__ballot_sync(JFULL, c_ != 0u)) { fault = __ballot_sync(JFULL, c_ == 1u) ? 1u : 2u; fault_pc = %uu; "
               "step = %s; goto finish; } ", pc, stepx);
-            if (mode == 3) o("if (ex) jpage_c<%uu>(bc, PG, va, v_); ", nw);
+            if (mode == 3) o("if (ex) jpage_c<%uu>(A, bc, PG, va, v_); ", nw);
             const char* v[] = {"v_.x", "v_.y", "v_.z", "v_.w"};
             wr(o, I.d0, v, nw);
             o("}\n");
@@ -355,11 +355,12 @@ struct Gen {
         }
         // fast path: every executing lane hits its buffer cache (no table lookups, no
         // cache updates); otherwise the full checks in program order
+        // (bitwise, not short-circuit: every test is evaluated, no branches)
         o("  if (__ballot_sync(JFULL, !(true");
         for (uint32_t j = 0; j < m; ++j) {
             const fi_insn& I = code[i0 + j];
             const uint32_t lw = (I.mod & 3) > 2 ? 2 : (I.mod & 3);
-            o(" && (!ex%u || jhit(bc, va%u, %uu, &z%u))", j, j, 4u << lw, j);
+            o(" & (!ex%u | jhit(bc, va%u, %uu, &z%u))", j, j, 4u << lw, j);
         }
         o("))) {\n");
         for (uint32_t j = 0; j < m; ++j) {
@@ -387,12 +388,14 @@ struct Gen {
         for (uint32_t j = 0; j < m; ++j) {
             const fi_insn& I = code[i0 + j];
             const uint32_t lw = (I.mod & 3) > 2 ? 2 : (I.mod & 3), nw = 1u << lw;
-            o("  if (ex%u) { uint4 v_ = make_uint4(0u, 0u, 0u, 0u); if (!z%u) { const u8* p_ = A.img + (va%u - JVA_BASE); ",
+            // (a word the writer rule zeroes is read from a zero line: one unconditional load)
+            o("  if (ex%u) { uint4 v_ = make_uint4(0u, 0u, 0u, 0u); "
+              "const u8* p_ = z%u ? reinterpret_cast<const u8*>(jzero16) : jimg + (va%u - JVA_BASE); ",
               j, j, j);
-            if (lw == 0) o("v_.x = jld32(p_); } ");
-            else if (lw == 1) o("const uint2 t_ = jld64(p_); v_.x = t_.x; v_.y = t_.y; } ");
-            else o("v_ = jld128(p_); } ");
-            if (mode == 3) o("jpage_c<%uu>(bc, PG, va%u, v_); ", nw, j);
+            if (lw == 0) o("v_.x = jld32(p_); ");
+            else if (lw == 1) o("const uint2 t_ = jld64(p_); v_.x = t_.x; v_.y = t_.y; ");
+            else o("v_ = jld128(p_); ");
+            if (mode == 3) o("jpage_c<%uu>(A, bc, PG, va%u, v_); ", nw, j);
             if (I.d0 != fi::kRZ)
                 for (uint32_t q = 0; q < nw; ++q)
                     if (W(I.d0 + q)) o("R%u = v_.%c; ", I.d0 + q, "xyzw"[q]);
@@ -462,7 +465,9 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "uint4* __restrict__ rec_out, const JPage* __restrict__ pgp) {\n", kid, mname[mode]);
     o("(void)img_w; (void)rec_out; (void)ins;\n");
     if (mode == 3) o("const JPage PG = *pgp;               // the replica slot's pages (K8)\n");
-    o("const JArgs A = A_;                 // kernel arguments in registers for the whole run\n");
+    // the image base in a register; the other kernel arguments are read where they
+    // are used (cold paths), so they do not hold registers across the block code
+    o("const JArgs& A = A_; const u8* __restrict__ const jimg = A_.img;\n");
     o("const u32 lane = threadIdx.x & 31u, lt_mask = (1u << lane) - 1u;\n");
     o("const jfi_instance in = A.inst[k];\nconst u32 cbank_len = in.cbank_len; const u32* __restrict__ cb = A.cbank + "
       "in.cbank_off;\n(void)cbank_len; (void)cb; (void)lt_mask;\n");
@@ -583,7 +588,8 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "  st_.preds = (u32)Q0 | ((u32)Q1 << 1) | ((u32)Q2 << 2) | ((u32)Q3 << 3) | ((u32)Q4 << 4) | ((u32)Q5 << 5) | "
       "((u32)Q6 << 6); st_.recbuf = recbuf;\n"
       "  __syncwarp();\n"
-      "  const u32 done_ = jinterp<%u>(A, st_, bc, Rs, dec, kblen_%u, %uu, k, cta, wic, watchdog, hstep, hpc, hlane, "
+      "  JBufCache bcs_ = bc;                // (a copy: bc's address never escapes, so it stays in registers)\n"
+      "  const u32 done_ = jinterp<%u>(A, st_, bcs_, Rs, dec, kblen_%u, %uu, k, cta, wic, watchdog, hstep, hpc, hlane, "
       "hkind, hreg, hbfm, hmask, st_out, st_cap, %uu, img_w, rec_out, ck, ck_interval, ins, pgp);\n"
       "  __syncwarp();\n",
       mode, kid, n, NR);
@@ -591,7 +597,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
     o("\n  pc = st_.pc; live = st_.live; step = st_.step; livem = st_.livem; conv = st_.conv; upc = st_.upc; "
       "amask = st_.amask; npc = st_.npc; nst = st_.nst; fault = st_.fault; fault_pc = st_.fault_pc; "
       "before = st_.before; after = st_.after; msk = st_.msk; fired = st_.fired; bad = st_.bad; lim = st_.lim; "
-      "recbuf = st_.recbuf;\n"
+      "recbuf = st_.recbuf; bc = bcs_;\n"
       "  Q0 = st_.preds & 1u; Q1 = (st_.preds >> 1) & 1u; Q2 = (st_.preds >> 2) & 1u; Q3 = (st_.preds >> 3) & 1u; "
       "Q4 = (st_.preds >> 4) & 1u; Q5 = (st_.preds >> 5) & 1u; Q6 = (st_.preds >> 6) & 1u;\n"
       "  if (done_) goto finish;\n  continue;\n }\n}\n");
@@ -862,6 +868,10 @@ fi_status compile_cubin(const fi_insn* code, const fi_kernel* kern, uint32_t n_k
     cubin.resize(cs);
     N.cubin(prog, cubin.data());
     N.destroy(&prog);
+    if (const char* d = std::getenv("FI_JIT_DUMP")) {     // profiling aid: the module's source and cubin
+        if (FILE* f = std::fopen((std::string(d) + ".cu").c_str(), "wb")) { std::fwrite(src.data(), 1, src.size(), f); std::fclose(f); }
+        if (FILE* f = std::fopen((std::string(d) + ".cubin").c_str(), "wb")) { std::fwrite(cubin.data(), 1, cubin.size(), f); std::fclose(f); }
+    }
     return FI_OK;
 }
 

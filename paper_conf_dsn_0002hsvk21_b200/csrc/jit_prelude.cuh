@@ -146,55 +146,65 @@ __device__ __forceinline__ uint4 jld128(const u8* p) {
     return r;
 }
 
-// per-lane two-entry cache of buffer bounds (image offsets)
+// per-lane two-entry cache of buffer bounds, 32-bit: image offset `lo` and the
+// size floored to 16 B (`sz`; 0 = empty entry).  Only buffers with lo % 16 == 0
+// and lo + size <= 2^31 are cached (others always take jcheck's full path), so
+// for an aligned address va = JVA_BASE + off: off is in the entry iff
+// hi32(va) == hi32(JVA_BASE) and (u32)(lo32(va) - lo) < sz — an offset below lo
+// wraps to >= 2^31 > sz, and d < sz with d, sz multiples of the access width w
+// gives d + w <= sz <= size.  A miss is never wrong, only slower.
+static_assert((JVA_BASE & 0xFFFFFFFFull) == 0, "the cache tests the low word of va only");
+#define JVA_HI ((u32)(JVA_BASE >> 32))
 struct JBufCache {
-    u64 lo0, hi0, lo1, hi1;
+    u32 lo0, sz0, lo1, sz1;
     bool z0, z1;
     u32 b0, b1, pb0, pb1;        // buffer ids and their first page index (K8 page tables; 0 elsewhere)
     __device__ __forceinline__ JBufCache()
-        : lo0(1), hi0(0), lo1(1), hi1(0), z0(false), z1(false), b0(0), b1(0), pb0(0), pb1(0) {}
+        : lo0(0), sz0(0), lo1(0), sz1(0), z0(false), z1(false), b0(0), b1(0), pb0(0), pb1(0) {}
 };
+
+// cache-only check: true iff the access is aligned and inside one of the two
+// cached buffers (then *zero is that buffer's writer-rule flag); no state change
+__device__ __forceinline__ bool jhit(const JBufCache& C, u64 va, u32 w, bool* zero) {
+    const u32 vlo = (u32)va;
+    const bool h0 = vlo - C.lo0 < C.sz0;
+    const bool h1 = vlo - C.lo1 < C.sz1;
+    *zero = h0 ? C.z0 : C.z1;
+    return ((u32)(va >> 32) == JVA_HI) & ((vlo & (w - 1)) == 0) & (h0 | h1);
+}
+__device__ const uint4 jzero16[1] = {{0u, 0u, 0u, 0u}};   // the zero line of writer-rule loads
 
 // 0 ok, 1 misaligned, 2 unmapped (C-15); *zero = writer rule for instance k
 __device__ __forceinline__ u32 jcheck(const JArgs& A, JBufCache& C, u64 va, u32 w, u32 k, bool* zero,
                                       const u32* page_base = nullptr) {
     if (va & (w - 1)) return 1;
+    if (jhit(C, va, w, zero)) return 0;
     const u64 off = va - JVA_BASE;
-    // (off < hi first: an address just below the VA base wraps off + w around)
-    if (off >= C.lo0 && off < C.hi0 && off + w <= C.hi0) { *zero = C.z0; return 0; }
-    if (off >= C.lo1 && off < C.hi1 && off + w <= C.hi1) { *zero = C.z1; return 0; }
     if (va < JVA_BASE || off >= A.image_bytes) return 2;
     const u32 b = __ldg(&A.gran[off >> 8]);
     if (b == JNOBUF) return 2;
-    const u64 lo = __ldg(&A.buf[b].off), hi = lo + __ldg(&A.buf[b].size);
-    if (off + w > hi) return 2;
+    const u64 lo = __ldg(&A.buf[b].off), size = __ldg(&A.buf[b].size);
+    if (off + w > lo + size) return 2;
     const i32 wr = __ldg(&A.buf[b].writer);
-    C.lo1 = C.lo0; C.hi1 = C.hi0; C.z1 = C.z0; C.b1 = C.b0; C.pb1 = C.pb0;
-    C.lo0 = lo; C.hi0 = hi; C.z0 = wr >= 0 && (u32)wr >= k; C.b0 = b;
-    C.pb0 = page_base ? __ldg(&page_base[b]) : 0u;
-    *zero = C.z0;
+    const bool z = wr >= 0 && (u32)wr >= k;
+    *zero = z;
+    if ((lo & 15u) == 0 && lo + size <= 0x80000000ull && size >= 16) {
+        C.lo1 = C.lo0; C.sz1 = C.sz0; C.z1 = C.z0; C.b1 = C.b0; C.pb1 = C.pb0;
+        C.lo0 = (u32)lo; C.sz0 = (u32)size & ~15u; C.z0 = z; C.b0 = b;
+        C.pb0 = page_base ? __ldg(&page_base[b]) : 0u;
+    }
     return 0;
-}
-
-// cache-only check: true iff the access is aligned and inside one of the two
-// cached buffers (then *zero is that buffer's writer-rule flag); no state change
-__device__ __forceinline__ bool jhit(const JBufCache& C, u64 va, u32 w, bool* zero) {
-    const u64 off = va - JVA_BASE;
-    const bool h0 = off >= C.lo0 && off < C.hi0 && off + w <= C.hi0;
-    const bool h1 = off >= C.lo1 && off < C.hi1 && off + w <= C.hi1;
-    *zero = h0 ? C.z0 : C.z1;
-    return ((va & (w - 1)) == 0) && (h0 || h1);
 }
 
 // one LDG of 1/2/4 words for this lane; returns the fault code (0 ok)
 template <u32 LW>
-__device__ __forceinline__ u32 jldg(const JArgs& A, JBufCache& C, u64 va, u32 k, bool ex, uint4& v,
-                                    const u32* page_base = nullptr) {
+__device__ __forceinline__ u32 jldg(const JArgs& A, const u8* __restrict__ img, JBufCache& C, u64 va, u32 k, bool ex,
+                                    uint4& v, const u32* page_base = nullptr) {
     bool zero = false;
     const u32 c = ex ? jcheck(A, C, va, 4u << LW, k, &zero, page_base) : 0u;
     v = make_uint4(0, 0, 0, 0);
     if (ex && !c && !zero) {
-        const u8* src = A.img + (va - JVA_BASE);
+        const u8* src = img + (va - JVA_BASE);
         if (LW == 0) v.x = jld32(src);
         else if (LW == 1) { const uint2 t = jld64(src); v.x = t.x; v.y = t.y; }
         else v = jld128(src);
@@ -405,14 +415,16 @@ __device__ __forceinline__ void jpage(const JArgs& A, const JPage& G, u64 va, ui
         *G.inexact = 1u;
     }
 }
-// the same through the lane's buffer cache (entry of the checked access): one page-table load
+// the same through the lane's buffer cache when one of its entries holds the
+// access (one page-table load), else jpage's full lookup
 template <u32 NW>
-__device__ __forceinline__ void jpage_c(const JBufCache& C, const JPage& G, u64 va, uint4& v) {
-    const u64 off = va - JVA_BASE;
-    const bool e0 = off >= C.lo0 && off < C.hi0;
-    const u64 rel = off - (e0 ? C.lo0 : C.lo1);
+__device__ __forceinline__ void jpage_c(const JArgs& A, const JBufCache& C, const JPage& G, u64 va, uint4& v) {
+    const u32 vlo = (u32)va, d0 = vlo - C.lo0, d1 = vlo - C.lo1;
+    const bool e0 = d0 < C.sz0;
+    if (!e0 && !(d1 < C.sz1)) { jpage<NW>(A, G, va, v); return; }
+    const u32 rel = e0 ? d0 : d1;
     const u32 b = e0 ? C.b0 : C.b1;
-    const u32 e = G.ptab[(e0 ? C.pb0 : C.pb1) + (u32)(rel >> 12)];
+    const u32 e = G.ptab[(e0 ? C.pb0 : C.pb1) + (rel >> 12)];
     if (e < JPAGE_CLAIM) {
         const u32* src = G.pool + (u64)e * JPAGE_WORDS + ((rel >> 2) & (JPAGE_WORDS - 1));
         if (NW == 1) v.x = __ldcg(src);
@@ -515,9 +527,9 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
                         else v = jld128(src);
                     }
                     if (MODE == JM_PAGE) {            // the replica's pages win
-                        if (nw == 1) jpage_c<1>(bc, *pg, va, v);
-                        else if (nw == 2) jpage_c<2>(bc, *pg, va, v);
-                        else jpage_c<4>(bc, *pg, va, v);
+                        if (nw == 1) jpage_c<1>(A, bc, *pg, va, v);
+                        else if (nw == 2) jpage_c<2>(A, bc, *pg, va, v);
+                        else jpage_c<4>(A, bc, *pg, va, v);
                     }
                     F.wr(id, v.x);
                     if (lw >= 1) F.wr(id + 128, v.y);
