@@ -345,7 +345,8 @@ struct Gen {
     // m consecutive independent LDGs (block mode): all address checks first, one
     // fault ballot (the first faulting load in program order wins, C-9), then all
     // loads in flight together, then the register writes in program order.
-    void ldg_batch(Src& o, const fi_insn* code, uint32_t i0, uint32_t m) const {
+    void ldg_batch(Src& o, const fi_insn* code, uint32_t i0, uint32_t m,
+                   const std::vector<std::string>& stride = {}) const {
         o(" { // LDG batch %u..%u\n", i0, i0 + m - 1);
         for (uint32_t j = 0; j < m; ++j) {
             const fi_insn& I = code[i0 + j];
@@ -401,6 +402,16 @@ struct Gen {
                     if (W(I.d0 + q)) o("R%u = v_.%c; ", I.d0 + q, "xyzw"[q]);
             o("}\n");
         }
+        // the next iteration's lines of a loop-carried pointer (address + loop-invariant
+        // stride) into L1 while this iteration computes; a hint only (no architectural
+        // effect), issued only for addresses inside a cached buffer
+        // (one per address pair: the batch's other loads off the same pointer are
+        // usually in the same lines)
+        for (uint32_t j = 0; j < m && j < stride.size(); ++j) {
+            bool first = !stride[j].empty();
+            for (uint32_t q = 0; q < j && first; ++q) first = code[i0 + q].a != code[i0 + j].a;
+            if (first) o("  if (ex%u) jprefetch(jimg, bc, va%u + (%s));\n", j, j, stride[j].c_str());
+        }
         o(" }\n");
     }
 };
@@ -423,6 +434,43 @@ static uint32_t ldg_batch_len(const fi_insn* code, uint32_t n, uint32_t i0, cons
         ++m;
     }
     return m;
+}
+
+// Per load of the LDG batch at i0 (length m) inside the self-looping block
+// [L, E] (code[E] = BRA to L): the change of its address over one iteration as
+// a C++ expression of the current registers, or "" if not a plain pointer walk.
+// The address pair (a, a+1) must be written in the block by exactly one
+// unguarded IMAD.WIDE d = a * b + (a, a+1) whose a/b operands the block never
+// writes (so the stride is loop-invariant and readable at the batch).
+static std::vector<std::string> batch_strides(const Gen& G, const fi_insn* code, uint32_t L, uint32_t E, uint32_t i0,
+                                              uint32_t m) {
+    using namespace fi;
+    std::vector<std::string> st(m);
+    auto writes = [&](uint32_t q, uint32_t r) {
+        const Dests d = dests_of(code[q].op, code[q].d0, code[q].d1, code[q].mod);
+        return r >= d.gp_base && r < d.gp_base + d.n_gp;
+    };
+    for (uint32_t j = 0; j < m; ++j) {
+        const uint32_t a = code[i0 + j].a;
+        if (a == kRZ || a + 1 >= G.NR) continue;
+        int w = -1, nw = 0;
+        for (uint32_t q = L; q <= E; ++q) {
+            if (q >= i0 && q < i0 + m) continue;
+            if (writes(q, a) || writes(q, a + 1)) { w = (int)q; ++nw; }
+        }
+        if (nw != 1) continue;
+        const fi_insn& W = code[w];
+        if (W.op != IMAD_WIDE || W.guard != 7 || W.d0 != a || W.c != a) continue;
+        bool inv = true;
+        for (uint32_t q = L; q <= E && inv; ++q) {
+            if (W.a != kRZ && writes(q, W.a)) inv = false;
+            if (!(W.mod & 0x80) && W.b != kRZ && writes(q, W.b)) inv = false;
+        }
+        if (!inv) continue;
+        const std::string x = G.R(W.a), y = G.bv(W);
+        st[j] = (W.mod & 1) ? "(u64)" + x + " * (u64)" + y : "(u64)((i64)(i32)" + x + " * (i64)(i32)" + y + ")";
+    }
+    return st;
 }
 
 // Generate the device function of one static kernel (EMU_INJ mode).
@@ -531,7 +579,12 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
         if (I.op == LDG) {
             const uint32_t m = ldg_batch_len(code, n, i, leader);
             if (m >= 2) {
-                G.ldg_batch(o, code, i, m);
+                // the block holding the batch: from its leader L to its BRA / EXIT E
+                uint32_t L = i;
+                while (L > 0 && !leader[L]) --L;
+                const uint32_t E = L + blen[L] - 1;
+                const bool self_loop = code[E].op == BRA && code[E].imm == L && (mode == 0 || mode == 3);
+                G.ldg_batch(o, code, i, m, self_loop ? batch_strides(G, code, L, E, i, m) : std::vector<std::string>());
                 batch_end = i + m;
                 if (i + m == n)
                     o(" { step += %uu - pcm; upc = %uu; if (upc >= npc) { conv = false; if (inA) pc = upc; } continue; }\n",
@@ -613,7 +666,8 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
     uint32_t min_blocks = 3;
     if (const char* e = std::getenv("FI_JIT_MIN_BLOCKS")) min_blocks = (uint32_t)std::max(1, std::atoi(e));
     Src o;
-    o.s = kPrelude;
+    if (std::getenv("FI_JIT_LDALLOC")) o.s = "#define JLD_L1 \"\"\n";
+    o.s += kPrelude;
     Gen G{n_regs};
     for (uint32_t k = 0; k < n_kern; ++k) {
         bool tables = true;

@@ -129,19 +129,22 @@ __device__ __forceinline__ u32 jshfl_src(u32 lane, u32 bv, u32 m) {
     return (u32)src;
 }
 
+#ifndef JLD_L1
+#define JLD_L1 ".L1::no_allocate"                    // image loads do not allocate in L1 (override: FI_JIT_LDALLOC)
+#endif
 __device__ __forceinline__ u32 jld32(const u8* p) {
     u32 r;
-    asm volatile("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(r) : "l"(p));
+    asm volatile("ld.global.nc" JLD_L1 ".u32 %0, [%1];" : "=r"(r) : "l"(p));
     return r;
 }
 __device__ __forceinline__ uint2 jld64(const u8* p) {
     uint2 r;
-    asm volatile("ld.global.nc.L1::no_allocate.v2.u32 {%0, %1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p));
+    asm volatile("ld.global.nc" JLD_L1 ".v2.u32 {%0, %1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p));
     return r;
 }
 __device__ __forceinline__ uint4 jld128(const u8* p) {
     uint4 r;
-    asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0, %1, %2, %3}, [%4];"
+    asm volatile("ld.global.nc" JLD_L1 ".v4.u32 {%0, %1, %2, %3}, [%4];"
                  : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
     return r;
 }
@@ -173,6 +176,12 @@ __device__ __forceinline__ bool jhit(const JBufCache& C, u64 va, u32 w, bool* ze
     return ((u32)(va >> 32) == JVA_HI) & ((vlo & (w - 1)) == 0) & (h0 | h1);
 }
 __device__ const uint4 jzero16[1] = {{0u, 0u, 0u, 0u}};   // the zero line of writer-rule loads
+// L1 prefetch of an address inside one of the lane's cached buffers (else nothing)
+__device__ __forceinline__ void jprefetch(const u8* __restrict__ img, const JBufCache& C, u64 va) {
+    const u32 vlo = (u32)va;
+    if (((u32)(va >> 32) == JVA_HI) & ((vlo - C.lo0 < C.sz0) | (vlo - C.lo1 < C.sz1)))
+        asm volatile("prefetch.global.L1 [%0];" ::"l"(img + (va - JVA_BASE)));
+}
 
 // 0 ok, 1 misaligned, 2 unmapped (C-15); *zero = writer rule for instance k
 __device__ __forceinline__ u32 jcheck(const JArgs& A, JBufCache& C, u64 va, u32 w, u32 k, bool* zero,
