@@ -310,8 +310,8 @@ def main():
                              "algorithmic_bytes_per_launch": algo_bytes},
         "clocks": clk,
         # per step: k_profile, 2 x k_scan_rows, k_inst_identities, k_tile_sums, k_select,
-        # k_lpt_order, k_inject_jit, k_classify
-        "gpu_launches": 9 * K,
+        # k_lpt_order, k_inject_jit, k_classify, k_classify_slow
+        "gpu_launches": 10 * K,
     }
 
     if not args.no_e2e:

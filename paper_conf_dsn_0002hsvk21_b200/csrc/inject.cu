@@ -138,6 +138,16 @@ __device__ __forceinline__ uint32_t pre_word(const ClsArgs& A, uint64_t va, uint
 }
 
 constexpr int kClsWarps = 4;
+constexpr uint8_t kSlow = 0xFE;                      // k_classify -> k_classify_slow hand-off outcome
+
+// a 16-B log entry through the read-only path (both logs are read-only here)
+__device__ __forceinline__ fi_store ld_store_nc(const fi_store* p) {
+    const uint4 w = __ldg(reinterpret_cast<const uint4*>(p));
+    fi_store s;
+    static_assert(sizeof(fi_store) == 16, "fi_store is 16 B");
+    memcpy(&s, &w, 16);
+    return s;
+}
 
 __global__ void __launch_bounds__(kClsWarps * 32) k_classify(const ClsArgs A) {
     const uint32_t lane = threadIdx.x & 31;
@@ -170,54 +180,115 @@ __global__ void __launch_bounds__(kClsWarps * 32) k_classify(const ClsArgs A) {
         const fi_store* Gs = G + gs;
         const uint64_t nG = nGall - gs, nF = R.n_faulty_stores;
         const fi_store* F = A.log + (uint64_t)i * A.cap;
-        bool same_addr = nF == nG;
-        for (uint64_t b = 0; same_addr && b < nF; b += 32) {
-            const bool d = b + lane < nF && F[b + lane].va != Gs[b + lane].va;
-            same_addr = !__any_sync(kFull, d);
-        }
-        bool sdc = false;
-        if (same_addr) {
-            // fast path: same store addresses in the same order; golden words are
-            // stored once per warp so the golden value is Gs[j]
-            for (uint64_t b = 0; b < nF && !sdc; b += 32) {
-                bool d = false;
-                if (b + lane < nF) {
-                    const fi_store f = F[b + lane];
-                    d = f.value != Gs[b + lane].value && is_output(A, f.va);
-                }
-                sdc = __any_sync(kFull, d);
+        // fast path: same store addresses in the same order; golden words are stored
+        // once per warp, so then the golden value of F[j] is Gs[j].
+        // One pass over both logs, 4 entries per lane in flight: address equality
+        // and "an output word differs" together (the latter decides only if every
+        // address matched)
+        bool same_addr = nF == nG, vdiff = false;
+        for (uint64_t b = 0; same_addr && b < nF; b += 128) {
+            fi_store f[4], g[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                const uint64_t j = b + u * 32 + lane;
+                if (j < nF) { f[u] = ld_store_nc(F + j); g[u] = ld_store_nc(Gs + j); }
             }
-        } else {
-            for (uint64_t b = 0; b < nF && !sdc; b += 32) {            // faulty stores: last write wins
-                bool d = false;
-                const uint64_t j = b + lane;
+            bool d = false, v = false;
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                const uint64_t j = b + u * 32 + lane;
                 if (j < nF) {
-                    const fi_store f = F[j];
-                    bool last = true;
-                    for (uint64_t q = j + 1; q < nF && last; ++q) last = F[q].va != f.va;
-                    d = last && is_output(A, f.va) && f.value != golden_word(A, f.va);
+                    d |= f[u].va != g[u].va;
+                    v |= f[u].va == g[u].va && f[u].value != g[u].value && is_output(A, f[u].va);
                 }
-                sdc = __any_sync(kFull, d);
             }
-            for (uint64_t b = 0; b < nG && !sdc; b += 32) {            // golden stores the faulty run skipped
-                bool d = false;
-                const uint64_t j = b + lane;
-                if (j < nG) {
-                    const uint64_t va = Gs[j].va;
-                    bool inF = false;
-                    for (uint64_t q = 0; q < nF && !inF; ++q) inF = F[q].va == va;
-                    d = !inF && is_output(A, va) && pre_word(A, va, S.instance) != golden_word(A, va);
-                }
-                sdc = __any_sync(kFull, d);
-            }
+            same_addr = !__any_sync(kFull, d);
+            vdiff |= v;
         }
-        outcome = sdc ? FI_SDC : FI_MASKED;
+        // different store addresses: k_classify_slow decides (outcome kSlow meanwhile)
+        outcome = !same_addr ? kSlow : __any_sync(kFull, vdiff) ? FI_SDC : FI_MASKED;
     }
     if (lane == 0) {
         A.inj[i].outcome = (uint8_t)outcome;
         A.inj[i].flags = pdue ? FI_POTENTIAL_DUE : 0;
         if (outcome == 0xFF) FI_DEV_ERR(A.status, FI_E_CAPACITY);
-        else atomicAdd((unsigned long long*)&A.hist[((uint32_t)S.group * 4 + S.bfm) * 3 + outcome], 1ull);
+        else if (outcome != kSlow) atomicAdd((unsigned long long*)&A.hist[((uint32_t)S.group * 4 + S.bfm) * 3 + outcome], 1ull);
+    }
+}
+
+// first golden store-log entry of warp w after step `step` (entries are in step order)
+__device__ uint64_t golden_suffix(const ClsArgs& A, uint32_t w, uint32_t step, uint32_t lane) {
+    const fi_store* G = A.gstore + A.gstore_off[w];
+    const uint64_t nGall = A.gstore_off[w + 1] - A.gstore_off[w];
+    uint64_t gs = 0;
+    for (uint64_t b = 0; b < nGall; b += 32) {
+        const uint32_t m = __ballot_sync(kFull, b + lane < nGall && G[b + lane].step > step);
+        if (m) { gs = b + __ffs(m) - 1; break; }
+        gs = min(b + 32, nGall);
+    }
+    return gs;
+}
+
+// K5's general case (faulty and golden store sequences differ in addresses), one
+// CTA per such replica (persistent over the replicas k_classify marked kSlow):
+//   SDC <=> some output word's final faulty value differs from its golden final value
+//   (a) a faulty store that is the last faulty write to its address and differs, or
+//   (b) a golden store after the site the faulty run never wrote, whose value before
+//       the instance differs from the golden final value (C-12).
+// The pairwise "any later write to the same address" / "any faulty write to this
+// address" tests run over 256-entry smem tiles of the faulty log (broadcast reads).
+constexpr int kSlowThreads = 256;
+__global__ void __launch_bounds__(kSlowThreads) k_classify_slow(const ClsArgs A) {
+    __shared__ uint64_t tva[kSlowThreads];
+    __shared__ uint64_t s_gs;
+    const uint32_t t = threadIdx.x, lane = t & 31;
+    for (uint32_t i = blockIdx.x; i < A.n; i += gridDim.x) {
+        if (A.inj[i].outcome != kSlow) continue;
+        const fi_site S = A.sites[i];
+        const fi_inj R = A.inj[i];
+        const bool pdue = (A.flags & FI_UNCHECKED) && R.fault_kind && R.fault_kind != 3;
+        if (t < 32) { const uint64_t gs = golden_suffix(A, S.warp, S.step, lane); if (t == 0) s_gs = gs; }
+        __syncthreads();
+        const uint64_t gs = s_gs;
+        const fi_store* Gs = A.gstore + A.gstore_off[S.warp] + gs;
+        const uint64_t nG = A.gstore_off[S.warp + 1] - A.gstore_off[S.warp] - gs, nF = R.n_faulty_stores;
+        const fi_store* F = A.log + (uint64_t)i * A.cap;
+        bool sdc = false;
+        for (uint64_t jb = 0; jb < nF && !sdc; jb += kSlowThreads) {           // (a)
+            const uint64_t j = jb + t;
+            const bool have = j < nF;
+            const fi_store f = have ? F[j] : fi_store{0, 0, 0};
+            bool last = have;
+            for (uint64_t qb = jb; qb < nF; qb += kSlowThreads) {
+                __syncthreads();
+                if (qb + t < nF) tva[t] = F[qb + t].va;
+                __syncthreads();
+                const uint32_t qn = (uint32_t)(nF - qb < (uint64_t)kSlowThreads ? nF - qb : (uint64_t)kSlowThreads);
+                for (uint32_t q = 0; q < qn; ++q) last &= !(qb + q > j && tva[q] == f.va);
+            }
+            sdc = __syncthreads_or(last && is_output(A, f.va) && f.value != golden_word(A, f.va));
+        }
+        for (uint64_t jb = 0; jb < nG && !sdc; jb += kSlowThreads) {           // (b)
+            const uint64_t j = jb + t;
+            const bool have = j < nG;
+            const uint64_t va = have ? Gs[j].va : 0;
+            bool inF = false;
+            for (uint64_t qb = 0; qb < nF; qb += kSlowThreads) {
+                __syncthreads();
+                if (qb + t < nF) tva[t] = F[qb + t].va;
+                __syncthreads();
+                const uint32_t qn = (uint32_t)(nF - qb < (uint64_t)kSlowThreads ? nF - qb : (uint64_t)kSlowThreads);
+                for (uint32_t q = 0; q < qn; ++q) inF |= tva[q] == va;
+            }
+            sdc = __syncthreads_or(have && !inF && is_output(A, va) && pre_word(A, va, S.instance) != golden_word(A, va));
+        }
+        if (t == 0) {
+            const uint32_t outcome = sdc ? FI_SDC : FI_MASKED;
+            A.inj[i].outcome = (uint8_t)outcome;
+            A.inj[i].flags = pdue ? FI_POTENTIAL_DUE : 0;
+            atomicAdd((unsigned long long*)&A.hist[((uint32_t)S.group * 4 + S.bfm) * 3 + outcome], 1ull);
+        }
+        __syncthreads();
     }
 }
 
@@ -307,5 +378,6 @@ extern "C" fi_status fi_classify(const fi_program* p, const uint8_t* image, cons
     const EmuProg P = make_emu_prog(p);
     ClsArgs A{p->buf, P.gran, image, t->gstore, t->gstore_off, sites, out, n, log, log_cap, hist, flags, dev_status};
     k_classify<<<(n + kClsWarps - 1) / kClsWarps, kClsWarps * 32, 0, (cudaStream_t)stream>>>(A);
+    k_classify_slow<<<std::min<uint32_t>(n, 148u * 8u), kSlowThreads, 0, (cudaStream_t)stream>>>(A);
     return launch_status();
 }
