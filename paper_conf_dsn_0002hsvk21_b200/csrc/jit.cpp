@@ -476,6 +476,11 @@ static std::vector<std::string> batch_strides(const Gen& G, const fi_insn* code,
 // Generate the device function of one static kernel (EMU_INJ mode).
 // Generate the device function of one static kernel in mode `mode` (JM_INJ,
 // JM_LEN, JM_TRACE); `blen`/leader tables are emitted once (with_tables).
+// kern_* arguments kept in the warp's JCtx (shared memory) instead of registers
+const char* const kCtxNames[] = {"hstep", "hpc", "hlane", "hkind", "hreg", "hbfm", "hmask", "k", "cta", "wic",
+                                 "watchdog", "ck", "ck_interval", "st_out", "st_cap", "Rs", "dec", "ins",
+                                 "img_w", "rec_out", "pgp"};
+
 void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32_t n, uint32_t mode, bool with_tables) {
     using namespace fi;
     Gen G = G0;
@@ -505,12 +510,24 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
             o("%u%s", leader[i] ? std::min<uint32_t>(blen[i], 0xFFFF) : 0u, i + 1 < n ? "," : "");
         o("};\n");
     }
-    o("__device__ __noinline__ void kern_%u_%s(const JArgs& A_, const u32 hstep, const u32 hpc, const u32 hlane, "
-      "const u32 hkind, const u32 hreg, const u32 hbfm, const u32 hmask, const u32 k, const u32 cta, "
-      "const u32 wic, const u32 watchdog, u32* __restrict__ ck, const u32 ck_interval, "
-      "jfi_store* __restrict__ st_out, const u32 st_cap, JOut& out, u32* __restrict__ Rs, "
-      "const uint4* __restrict__ dec, const u32* __restrict__ ins, u8* __restrict__ img_w, "
-      "uint4* __restrict__ rec_out, const JPage* __restrict__ pgp) {\n", kid, mname[mode]);
+    o("__device__ __noinline__ void kern_%u_%s(const JArgs& A_, const u32 hstep_p, const u32 hpc_p, const u32 hlane_p, "
+      "const u32 hkind_p, const u32 hreg_p, const u32 hbfm_p, const u32 hmask_p, const u32 k_p, const u32 cta_p, "
+      "const u32 wic_p, const u32 watchdog_p, u32* __restrict__ ck_p, const u32 ck_interval_p, "
+      "jfi_store* __restrict__ st_out_p, const u32 st_cap_p, JOut& out_p, u32* __restrict__ Rs_p, "
+      "const uint4* __restrict__ dec_p, const u32* __restrict__ ins_p, u8* __restrict__ img_w_p, "
+      "uint4* __restrict__ rec_out_p, const JPage* __restrict__ pgp_p) {\n", kid, mname[mode]);
+    // The arguments go to this warp's context in shared memory and are read where
+    // they are used (mostly cold paths): held in registers they would compete with
+    // the synthetic registers across the block code.
+    o("extern __shared__ u32 jsmem[];\nJCtx* const jx = reinterpret_cast<JCtx*>(jsmem + %uu + (threadIdx.x >> 5) * "
+      "(JCTX_BYTES / 4u));\n", 4u * (NR + 1) * 32u);
+    o("if ((threadIdx.x & 31u) == 0u) { jx->hstep = hstep_p; jx->hpc = hpc_p; jx->hlane = hlane_p; jx->hkind = hkind_p; "
+      "jx->hreg = hreg_p; jx->hbfm = hbfm_p; jx->hmask = hmask_p; jx->k = k_p; jx->cta = cta_p; jx->wic = wic_p; "
+      "jx->watchdog = watchdog_p; jx->ck = ck_p; jx->ck_interval = ck_interval_p; jx->st_out = st_out_p; "
+      "jx->st_cap = st_cap_p; jx->out = &out_p; jx->Rs = Rs_p; jx->dec = dec_p; jx->ins = ins_p; jx->img_w = img_w_p; "
+      "jx->rec_out = rec_out_p; jx->pgp = pgp_p; }\n__syncwarp();\n");
+    for (const char* nm : kCtxNames) o("#define %s (jx->%s)\n", nm, nm);
+    o("#define out (*jx->out)\n");
     o("(void)img_w; (void)rec_out; (void)ins;\n");
     if (mode == 3) o("const JPage PG = *pgp;               // the replica slot's pages (K8)\n");
     // the image base in a register; the other kernel arguments are read where they
@@ -658,7 +675,9 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
     else o("finish:\n");
     o(" out.steps = step; out.fault = fault; out.fault_pc = fault_pc; out.nstore = nst;\n"
       " out.before = __shfl_sync(JFULL, before, hlane); out.after = __shfl_sync(JFULL, after, hlane);\n"
-      " out.mask = __shfl_sync(JFULL, msk, hlane); out.fired = fired; out.bad = bad;\n}\n\n");
+      " out.mask = __shfl_sync(JFULL, msk, hlane); out.fired = fired; out.bad = bad;\n}\n");
+    for (const char* nm : kCtxNames) o("#undef %s\n", nm);
+    o("#undef out\n\n");
 }
 
 std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern, uint32_t n_regs, uint32_t modes) {
@@ -866,7 +885,8 @@ thread_local std::string g_jit_log;
 }  // namespace
 
 // step mode's shared-memory register files: 4 warps x (n_regs + 1) rows x 32 lanes
-static size_t jit_smem(uint32_t n_regs) { return (size_t)4 * (n_regs + 1) * 128; }
+// + 4 warps' JCtx (JCTX_BYTES of jit_prelude.cuh)
+static size_t jit_smem(uint32_t n_regs) { return (size_t)4 * (n_regs + 1) * 128 + 4 * 256; }
 
 struct fi_jit {
     size_t smem = 0;

@@ -49,6 +49,16 @@ struct JOut {
     u32 steps, fault, fault_pc, nstore, before, after, mask;
     bool fired, bad;
 };
+// a generated kern_*'s arguments, per warp in shared memory after the 4 warps'
+// step-mode register files (jit.cpp kCtxNames, jit_smem)
+struct JPage;
+struct JCtx {
+    u32 hstep, hpc, hlane, hkind, hreg, hbfm, hmask, k, cta, wic, watchdog, ck_interval, st_cap;
+    u32* ck; jfi_store* st_out; JOut* out; u32* Rs; const uint4* dec; const u32* ins; u8* img_w; uint4* rec_out;
+    const JPage* pgp;
+};
+#define JCTX_BYTES 256u
+static_assert(sizeof(JCtx) <= JCTX_BYTES, "JCtx fits its smem slot");
 
 __device__ __forceinline__ float ju2f(u32 x) { return __uint_as_float(x); }
 __device__ __forceinline__ u32 jfbits(float f) { return f != f ? JQNAN32 : __float_as_uint(f); }
