@@ -480,6 +480,9 @@ static std::vector<std::string> batch_strides(const Gen& G, const fi_insn* code,
 const char* const kCtxNames[] = {"hstep", "hpc", "hlane", "hkind", "hreg", "hbfm", "hmask", "k", "cta", "wic",
                                  "watchdog", "ck", "ck_interval", "st_out", "st_cap", "Rs", "dec", "ins",
                                  "img_w", "rec_out", "pgp"};
+// warp state that block code rarely touches (store count, fault, the site's values):
+// per lane in the context (JCtx arrays), not in registers
+const char* const kCtxLaneNames[] = {"nst", "fault", "fault_pc", "before", "after", "msk", "fired", "bad"};
 
 void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32_t n, uint32_t mode, bool with_tables) {
     using namespace fi;
@@ -527,6 +530,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "jx->st_cap = st_cap_p; jx->out = &out_p; jx->Rs = Rs_p; jx->dec = dec_p; jx->ins = ins_p; jx->img_w = img_w_p; "
       "jx->rec_out = rec_out_p; jx->pgp = pgp_p; }\n__syncwarp();\n");
     for (const char* nm : kCtxNames) o("#define %s (jx->%s)\n", nm, nm);
+    for (const char* nm : kCtxLaneNames) o("#define %s (jx->%s_[threadIdx.x & 31u])\n", nm, nm);
     o("#define out (*jx->out)\n");
     o("(void)img_w; (void)rec_out; (void)ins;\n");
     if (mode == 3) o("const JPage PG = *pgp;               // the replica slot's pages (K8)\n");
@@ -550,7 +554,8 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
     for (uint32_t j = 0; j < NR; ++j) o("R%u = 0u;%s", j, (j % 16 == 15) ? "\n" : " ");
     o("\n}\n");
     o("u32 livem = __ballot_sync(JFULL, live);\nbool conv = false; u32 upc = 0u, amask = 0u, npc = 0xFFFFFFFFu;\n"
-      "u32 nst = 0u, fault = 0u, fault_pc = 0u, before = 0u, after = 0u, msk = 0u; bool fired = false, bad = false;\n"
+      "jx->nst_[lane] = 0u; jx->fault_[lane] = 0u; jx->fault_pc_[lane] = 0u; jx->before_[lane] = 0u; "
+      "jx->after_[lane] = 0u; jx->msk_[lane] = 0u; jx->fired_[lane] = 0u; jx->bad_[lane] = 0u;\n"
       "JBufCache bc; uint4 recbuf = make_uint4(0u, 0u, 0u, 0u); (void)recbuf;\n"
       "// blocks run only within [step, lim): lim = the watchdog, or the injection step while it is pending,\n"
       "// or the next checkpoint step (golden trace pass)\n"
@@ -650,11 +655,14 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
         }
     }
     // ---- step mode: registers to the warp's shared-memory file, interpreter, back
+    // (the per-lane context names are member names of JState / JOut too: spelled out below)
+    for (const char* nm : kCtxLaneNames) o("#undef %s\n", nm);
     o(" S_any: {\n");
     for (uint32_t j = 0; j < NR; ++j) o("  Rs[%uu + lane] = R%u;%s", j * 32, j, (j % 8 == 7) ? "\n" : "");
     o("\n  JState st_; st_.pc = pc; st_.live = live; st_.step = step; st_.livem = livem; st_.conv = conv; "
-      "st_.upc = upc; st_.amask = amask; st_.npc = npc; st_.nst = nst; st_.fault = fault; st_.fault_pc = fault_pc; "
-      "st_.before = before; st_.after = after; st_.msk = msk; st_.fired = fired; st_.bad = bad; st_.lim = lim;\n"
+      "st_.upc = upc; st_.amask = amask; st_.npc = npc; st_.nst = jx->nst_[lane]; st_.fault = jx->fault_[lane]; "
+      "st_.fault_pc = jx->fault_pc_[lane]; st_.before = jx->before_[lane]; st_.after = jx->after_[lane]; "
+      "st_.msk = jx->msk_[lane]; st_.fired = jx->fired_[lane]; st_.bad = jx->bad_[lane]; st_.lim = lim;\n"
       "  st_.preds = (u32)Q0 | ((u32)Q1 << 1) | ((u32)Q2 << 2) | ((u32)Q3 << 3) | ((u32)Q4 << 4) | ((u32)Q5 << 5) | "
       "((u32)Q6 << 6); st_.recbuf = recbuf;\n"
       "  __syncwarp();\n"
@@ -665,19 +673,22 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       mode, kid, n, NR);
     for (uint32_t j = 0; j < NR; ++j) o("  R%u = Rs[%uu + lane];%s", j, j * 32, (j % 8 == 7) ? "\n" : "");
     o("\n  pc = st_.pc; live = st_.live; step = st_.step; livem = st_.livem; conv = st_.conv; upc = st_.upc; "
-      "amask = st_.amask; npc = st_.npc; nst = st_.nst; fault = st_.fault; fault_pc = st_.fault_pc; "
-      "before = st_.before; after = st_.after; msk = st_.msk; fired = st_.fired; bad = st_.bad; lim = st_.lim; "
+      "amask = st_.amask; npc = st_.npc; jx->nst_[lane] = st_.nst; jx->fault_[lane] = st_.fault; "
+      "jx->fault_pc_[lane] = st_.fault_pc; jx->before_[lane] = st_.before; jx->after_[lane] = st_.after; "
+      "jx->msk_[lane] = st_.msk; jx->fired_[lane] = st_.fired; jx->bad_[lane] = st_.bad; lim = st_.lim; "
       "recbuf = st_.recbuf; bc = bcs_;\n"
       "  Q0 = st_.preds & 1u; Q1 = (st_.preds >> 1) & 1u; Q2 = (st_.preds >> 2) & 1u; Q3 = (st_.preds >> 3) & 1u; "
       "Q4 = (st_.preds >> 4) & 1u; Q5 = (st_.preds >> 5) & 1u; Q6 = (st_.preds >> 6) & 1u;\n"
       "  if (done_) goto finish;\n  continue;\n }\n}\n");
     if (mode == 2) o("finish:\n { const u32 rem_ = step & 31u; if (rem_ && lane < rem_) rec_out[step - rem_ + lane] = recbuf; }\n");
     else o("finish:\n");
-    o(" out.steps = step; out.fault = fault; out.fault_pc = fault_pc; out.nstore = nst;\n"
-      " out.before = __shfl_sync(JFULL, before, hlane); out.after = __shfl_sync(JFULL, after, hlane);\n"
-      " out.mask = __shfl_sync(JFULL, msk, hlane); out.fired = fired; out.bad = bad;\n}\n");
+    o("#undef out\n");
+    o(" { JOut& out_ = *jx->out; out_.steps = step; out_.fault = jx->fault_[lane]; out_.fault_pc = jx->fault_pc_[lane]; "
+      "out_.nstore = jx->nst_[lane];\n"
+      " out_.before = __shfl_sync(JFULL, jx->before_[lane], hlane); out_.after = __shfl_sync(JFULL, jx->after_[lane], hlane);\n"
+      " out_.mask = __shfl_sync(JFULL, jx->msk_[lane], hlane); out_.fired = jx->fired_[lane]; out_.bad = jx->bad_[lane]; }\n}\n");
     for (const char* nm : kCtxNames) o("#undef %s\n", nm);
-    o("#undef out\n\n");
+    o("\n");
 }
 
 std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern, uint32_t n_regs, uint32_t modes) {
@@ -886,7 +897,7 @@ thread_local std::string g_jit_log;
 
 // step mode's shared-memory register files: 4 warps x (n_regs + 1) rows x 32 lanes
 // + 4 warps' JCtx (JCTX_BYTES of jit_prelude.cuh)
-static size_t jit_smem(uint32_t n_regs) { return (size_t)4 * (n_regs + 1) * 128 + 4 * 256; }
+static size_t jit_smem(uint32_t n_regs) { return (size_t)4 * (n_regs + 1) * 128 + 4 * 1280; }
 
 struct fi_jit {
     size_t smem = 0;

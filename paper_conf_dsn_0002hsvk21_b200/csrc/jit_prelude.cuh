@@ -56,8 +56,10 @@ struct JCtx {
     u32 hstep, hpc, hlane, hkind, hreg, hbfm, hmask, k, cta, wic, watchdog, ck_interval, st_cap;
     u32* ck; jfi_store* st_out; JOut* out; u32* Rs; const uint4* dec; const u32* ins; u8* img_w; uint4* rec_out;
     const JPage* pgp;
+    // per lane: warp state block code rarely touches (jit.cpp kCtxLaneNames)
+    u32 nst_[32], fault_[32], fault_pc_[32], before_[32], after_[32], msk_[32], fired_[32], bad_[32];
 };
-#define JCTX_BYTES 256u
+#define JCTX_BYTES 1280u
 static_assert(sizeof(JCtx) <= JCTX_BYTES, "JCtx fits its smem slot");
 
 __device__ __forceinline__ float ju2f(u32 x) { return __uint_as_float(x); }
