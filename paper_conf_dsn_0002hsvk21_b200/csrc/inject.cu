@@ -29,21 +29,55 @@ constexpr int kWPB = 4;
 constexpr int kBuckets = 1024;
 
 // Longest-expected-first replica order (LPT scheduling): counting sort, one CTA,
-// of the steps each replica must emulate after its restart point.
+// of the steps each replica must emulate after its restart point.  The golden
+// remaining length is the estimate, except for a replica whose corrupted
+// register is a loop-control operand (read by an ISETP whose predicate guards a
+// backward BRA of the same static kernel): its loop may run longer than the
+// golden one, so it goes first (estimate 2x its warp length).  Order only:
+// results do not depend on it.
+constexpr uint32_t kLptMaxKern = 256;
 __global__ void __launch_bounds__(1024)
 k_lpt_order(const fi_site* __restrict__ sites, const uint64_t* __restrict__ warp_off, uint32_t ck_interval,
-            uint32_t n, uint32_t* __restrict__ order, uint32_t* __restrict__ counter) {
+            uint32_t n, uint32_t* __restrict__ order, uint32_t* __restrict__ counter, const fi_insn* __restrict__ code,
+            const fi_kernel* __restrict__ kern, uint32_t n_kern) {
     __shared__ uint32_t hist[kBuckets];
     __shared__ uint32_t s_max;
+    __shared__ uint32_t ctl[kLptMaxKern][4];         // per static kernel: loop-control registers (bit mask)
+    const bool use_ctl = code && kern && n_kern <= kLptMaxKern;
     auto cost = [&](uint32_t i) -> uint64_t {
         const fi_site S = sites[i];
         if (S.flags & FI_SITE_NOT_INJECTED) return 0;
         const uint64_t L = warp_off[S.warp + 1] - warp_off[S.warp];
+        if (use_ctl && S.dst_kind == 0 && S.kernel_id < n_kern && S.dst_reg < 128 &&
+            ((ctl[S.kernel_id][S.dst_reg >> 5] >> (S.dst_reg & 31)) & 1u))
+            return 2 * L;
         const uint64_t start = ck_interval ? (uint64_t)(S.step / ck_interval) * ck_interval : 0;
         return L > start ? L - start : 0;
     };
     for (uint32_t b = threadIdx.x; b < kBuckets; b += blockDim.x) hist[b] = 0;
     if (threadIdx.x == 0) { s_max = 0; *counter = 0; *reinterpret_cast<unsigned long long*>(counter + 2) = 0; }
+    if (use_ctl) {
+        for (uint32_t q = threadIdx.x; q < n_kern * 4; q += blockDim.x) ctl[q >> 2][q & 3] = 0;
+        __syncthreads();
+        // one warp per static kernel: each lane takes ISETPs, then scans for a backward
+        // BRA guarded by the ISETP's predicate
+        const uint32_t lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+        for (uint32_t k = w; k < n_kern; k += blockDim.x >> 5) {
+            const fi_kernel K = kern[k];
+            for (uint32_t pc = lane; pc < K.code_len; pc += 32) {
+                const fi_insn I = code[K.code_off + pc];
+                if (I.op != ISETP || (I.d0 & 7) == kPT) continue;
+                bool loop = false;
+                for (uint32_t q = 0; q < K.code_len && !loop; ++q) {
+                    const fi_insn B = code[K.code_off + q];
+                    loop = B.op == BRA && (B.guard & 7) == (I.d0 & 7) && B.imm <= q;
+                }
+                if (!loop) continue;
+                if (I.a < 128) atomicOr(&ctl[k][I.a >> 5], 1u << (I.a & 31));
+                if (!(I.mod & 0x80) && I.b < 128) atomicOr(&ctl[k][I.b >> 5], 1u << (I.b & 31));
+            }
+        }
+    }
     __syncthreads();
     uint32_t mx = 0;
     for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) mx = max(mx, (uint32_t)min(cost(i), (uint64_t)0xFFFFFFFFu));
@@ -294,9 +328,9 @@ __global__ void __launch_bounds__(kSlowThreads) k_classify_slow(const ClsArgs A)
 
 }  // namespace
 
-void launch_lpt_order(const fi_site* sites, const uint64_t* warp_off, uint32_t ck_interval, uint32_t n,
-                      uint32_t* order, uint32_t* counter, cudaStream_t s) {
-    k_lpt_order<<<1, 1024, 0, s>>>(sites, warp_off, ck_interval, n, order, counter);
+void launch_lpt_order(const fi_program* p, const fi_site* sites, const uint64_t* warp_off, uint32_t ck_interval,
+                      uint32_t n, uint32_t* order, uint32_t* counter, cudaStream_t s) {
+    k_lpt_order<<<1, 1024, 0, s>>>(sites, warp_off, ck_interval, n, order, counter, p->code, p->kern, p->n_kern);
 }
 }  // namespace fi
 
@@ -315,7 +349,7 @@ extern "C" fi_status fi_inject(const fi_program* p, const uint8_t* image, const 
     uint32_t* counter = reinterpret_cast<uint32_t*>(ws);
     uint32_t* order = reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(ws) + 256);
     const uint32_t ck_iv = t->ckpt ? t->ckpt_interval : 0;
-    k_lpt_order<<<1, 1024, 0, s>>>(sites, t->warp_off, ck_iv, n, order, counter);
+    k_lpt_order<<<1, 1024, 0, s>>>(sites, t->warp_off, ck_iv, n, order, counter, p->code, p->kern, p->n_kern);
     fi_status e = launch_status();
     if (e) return e;
     const size_t smem = golden_smem(p->n_regs);

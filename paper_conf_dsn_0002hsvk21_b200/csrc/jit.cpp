@@ -912,8 +912,8 @@ struct fi_jit {
 namespace fi {
 size_t aux_dec_offset(const fi_program* p);
 size_t aux_ins_offset(const fi_program* p);
-void launch_lpt_order(const fi_site* sites, const uint64_t* warp_off, uint32_t ck_interval, uint32_t n,
-                      uint32_t* order, uint32_t* counter, cudaStream_t s);
+void launch_lpt_order(const fi_program* p, const fi_site* sites, const uint64_t* warp_off, uint32_t ck_interval,
+                      uint32_t n, uint32_t* order, uint32_t* counter, cudaStream_t s);
 }
 
 extern "C" const char* fi_jit_log(void) { return g_jit_log.c_str(); }
@@ -1072,7 +1072,7 @@ extern "C" fi_status fi_inject_jit(const fi_jit* j, const fi_program* p, const u
     uint32_t* counter = reinterpret_cast<uint32_t*>(ws);
     uint32_t* order = reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(ws) + 256);
     const uint32_t ck_iv = t->ckpt ? t->ckpt_interval : 0;
-    fi::launch_lpt_order(sites, t->warp_off, ck_iv, n, order, counter, s);
+    fi::launch_lpt_order(p, sites, t->warp_off, ck_iv, n, order, counter, s);
     fi_status e = fi::launch_status();
     if (e) return e;
     int dev = 0, sms = 0, per = 0;
