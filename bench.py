@@ -378,7 +378,7 @@ def e2e(args, prog, seed, groups, bfms, n, rank, world, dev, camp):
     del camp
     torch.cuda.empty_cache()
     times, r, jit_ms = [], None, []
-    for it in range(2):
+    for it in range(4):
         if world > 1:
             import torch.distributed as dist
             dist.barrier()
@@ -387,16 +387,18 @@ def e2e(args, prog, seed, groups, bfms, n, rank, world, dev, camp):
         r = fi.campaign(prog, seed, groups, bfms, n, rank, world, host=host, engine="jit")
         times.append(time.perf_counter() - t0)
         jit_ms.append(r.ms["jit"])
+    fi.campaign_release_memory(dev.index if dev.index is not None else -1)
     assert int(r.hist.sum()) == n
     n_loc = r.n_local
     d2h = r.hist.nbytes + n_loc * (fi.SITE_DTYPE.itemsize + fi.INJ_DTYPE.itemsize) + r.inst_counts.nbytes
-    T = allreduce_max(min(times), dev)
+    T = allreduce_max(min(times[1:]), dev)
     return {"value": r.counted / T, "unit": "thread-dyn-instrs/s", "h2d_bytes_per_step": h2d,
             "d2h_bytes_per_step": d2h, "injections_per_s": n / T, "seconds": T,
             "api": "fi_campaign (C ABI) via paper_conf_dsn_0002hsvk21_b200.fi.campaign, K4 engine JIT",
             "cold_seconds": times[0], "jit_compile_s": jit_ms[0] / 1e3,
-            "timing": "value/seconds from the second call (JIT module cached in-process by the first, which "
-                      "also reports cold_seconds including the one-time NVRTC compile)",
+            "timing": "value/seconds: the fastest of calls 2-4 (JIT module cached in-process and device memory "
+                      "kept in the pool by the first call, which reports cold_seconds including the one-time NVRTC "
+                      "compile and the first allocations)", "warm_seconds": times[1:],
             "stages_ms": r.ms,
             "includes": "H2D program+image (pinned), golden run passes 1+2 (trace generation + checkpoints), "
                         "profile, count exchange, index, select, inject, classify, histogram exchange, "

@@ -418,7 +418,9 @@ fi_status fi_write_profile_txt(const uint64_t* inst_counts_host, const fi_instan
  * torch.distributed all_reduce on NCCL (paper_conf_dsn_0002hsvk21_b200.fi.campaign).
  *
  * Memory: unlike the other calls, fi_campaign allocates its device memory itself
- * (cudaMalloc on cfg->device, all freed before it returns) and SYNCHRONIZES.
+ * (stream-ordered, from cfg->device's default memory pool; all freed before it
+ * returns, but the pool keeps the memory reserved for the next call — see
+ * fi_campaign_release_memory) and SYNCHRONIZES.
  * Host arrays in cfg are read only; result arrays marked optional may be NULL.
  * Errors: FI_E_ARG (bad cfg), FI_E_PROGRAM / FI_E_INVARIANT / FI_E_SITE /
  * FI_E_CAPACITY from device status, FI_E_EMPTY_GROUP / FI_E_NOT_INJECTABLE from
@@ -474,6 +476,10 @@ typedef struct {
 
 fi_status fi_campaign(const fi_campaign_cfg* cfg, int rank, int world, fi_allreduce_fn allreduce, void* ctx,
                       fi_campaign_result* res);
+/* Return the device memory fi_campaign's calls left reserved in `device`'s default
+ * memory pool (device < 0: the current device) to the driver.  Synchronizes the
+ * device.  FI_E_CUDA on failure. */
+fi_status fi_campaign_release_memory(int device);
 
 #ifdef __cplusplus
 }

@@ -167,6 +167,7 @@ def lib():
             "fi_write_profile_txt": (st, [vp, vp, u32, vp, u32, vp, sz, C.POINTER(C.c_size_t)]),
             "fi_campaign": (st, [C.POINTER(fi_campaign_cfg), C.c_int, C.c_int, ALLREDUCE_FN, vp,
                                  C.POINTER(fi_campaign_result)]),
+            "fi_campaign_release_memory": (st, [C.c_int]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -798,6 +799,12 @@ def campaign(prog, seed: int, groups, bfms, n_replicas: int, rank: int = 0, worl
                           int(res.n_rec), int(res.counted), int(res.j0), int(res.n_local),
                           (int(res.rec_begin), int(res.rec_end)), int(res.n_unclassified), int(res.n_not_injected),
                           ms, None if sites is None else sites[:n_loc], None if inj is None else inj[:n_loc], ic)
+
+
+def campaign_release_memory(device: int = -1) -> None:
+    """fi_campaign_release_memory: give back the device memory fi_campaign keeps
+    reserved in the device's default pool between calls."""
+    _check(lib().fi_campaign_release_memory(device), "fi_campaign_release_memory")
 
 
 def as_numpy(t: torch.Tensor, dtype: np.dtype, n: int | None = None) -> np.ndarray:
