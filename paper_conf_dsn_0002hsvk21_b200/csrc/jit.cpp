@@ -291,12 +291,23 @@ struct Gen {
     // LDG / STG.  `stepx` = this instruction's step.
     uint32_t mode = 0;                               // JM_INJ / JM_LEN / JM_TRACE of jit_prelude.cuh
     // trace record of the instruction at pc (App. A.3): written only in JM_TRACE
+    // Block code writes the records of a whole block when it leaves it (flush_recs);
+    // here only a guarded instruction's predicate mask is kept for that.
     void rec(Src& o, const fi_insn& I, uint32_t pc, const char* stepx, const char* pv) const {
+        (void)stepx;
+        if (mode != 2 || I.guard == 7) return;
+        o("gb_%u = __ballot_sync(JFULL, %s); ", pc, pv);
+    }
+    // the trace records of block steps [pcm, E] (App. A.3), lanes striding over them:
+    // {instance, trace-insn word, active mask, guard-predicate mask}; call before the
+    // step counter moves past the block
+    void flush_recs(Src& o, const fi_insn* code, uint32_t L, uint32_t E) const {
         if (mode != 2) return;
-        const uint32_t insw = pc | ((uint32_t)I.op << 16) | (fi::groupmask_of(I.op, I.d0, I.d1, I.mod) << 24);
-        o("{ const u32 s_ = %s; const u32 pr_ = %s; if ((s_ & 31u) == lane) recbuf = make_uint4(k, %uu, amask, pr_); "
-          "if ((s_ & 31u) == 31u) rec_out[s_ - 31u + lane] = recbuf; } ",
-          stepx, I.guard == 7 ? "JFULL" : (std::string("__ballot_sync(JFULL, ") + pv + ")").c_str(), insw);
+        o("   { const u32 n_ = %uu - pcm; for (u32 j_ = lane; j_ < n_; j_ += 32u) { const u32 p_ = pcm + j_; u32 pr_ = JFULL; ",
+          E + 1);
+        for (uint32_t q = L; q <= E; ++q)
+            if (code[q].guard != 7) o("if (p_ == %uu) pr_ = gb_%u; ", q, q);
+        o("rec_out[step + j_] = make_uint4(k, __ldg(&ins[p_]), amask, pr_); } }\n");
     }
     void mem(Src& o, const fi_insn& I, uint32_t pc, const char* stepx) const {
         using namespace fi;
@@ -579,6 +590,9 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
     o(" if (step >= watchdog) { fault = 3u; fault_pc = pcm; break; }\n"
       " if (pcm >= %uu) { fault = 4u; fault_pc = pcm; break; }\n",
       n);
+    if (mode == 2)                                    // guard masks of this block's predicated steps (flush_recs)
+        for (uint32_t q = 0; q < n; ++q)
+            if (code[q].guard != 7) o("u32 gb_%u = 0u; (void)gb_%u;\n", q, q);
     // dispatch: a whole block when it fits, else one step
     o(" switch (pcm) {\n");
     for (uint32_t i = 0; i < n; ++i)
@@ -587,15 +601,23 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
     o("  default: goto S_any;\n }\n");
     // ---- block code (fallthrough from a leader to the block's BRA / EXIT)
     char stepx[64];
+    auto run_start = [&](uint32_t E) {               // first pc of the straight-line run ending at E
+        uint32_t q = E;
+        while (q > 0 && code[q - 1].op != BRA && code[q - 1].op != EXIT) --q;
+        return q;
+    };
+    auto flush_end = [&]() { G.flush_recs(o, code, run_start(n - 1), n - 1); };
     uint32_t batch_end = 0;                           // LDGs [.., batch_end) already emitted as a batch
     for (uint32_t i = 0; i < n; ++i) {
         const fi_insn& I = code[i];
         std::snprintf(stepx, sizeof stepx, "step + (%uu - pcm)", i);
         if (leader[i]) o(" B%u:\n", i);
         if (i < batch_end) {
-            if (i + 1 == n)
+            if (i + 1 == n) {
+                flush_end();
                 o(" { step += %uu - pcm; upc = %uu; if (upc >= npc) { conv = false; if (inA) pc = upc; } continue; }\n",
                   n, n);
+            }
             continue;
         }
         if (I.op == LDG) {
@@ -605,12 +627,14 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
                 uint32_t L = i;
                 while (L > 0 && !leader[L]) --L;
                 const uint32_t E = L + blen[L] - 1;
-                const bool self_loop = code[E].op == BRA && code[E].imm == L && (mode == 0 || mode == 3);
+                const bool self_loop = code[E].op == BRA && code[E].imm == L;
                 G.ldg_batch(o, code, i, m, self_loop ? batch_strides(G, code, L, E, i, m) : std::vector<std::string>());
                 batch_end = i + m;
-                if (i + m == n)
+                if (i + m == n) {
+                    flush_end();
                     o(" { step += %uu - pcm; upc = %uu; if (upc >= npc) { conv = false; if (inA) pc = upc; } continue; }\n",
                       n, n);
+                }
                 continue;
             }
         }
@@ -626,6 +650,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
             };
             o(" { const bool pv = %s; ", G.guard(I.guard).c_str());
             G.rec(o, I, i, stepx, "pv");
+            G.flush_recs(o, code, run_start(i), i);
             o("const u32 exm_ = amask & __ballot_sync(JFULL, pv); step += %uu - pcm;\n"
               "   if (exm_ == 0u) { %supc = %uu; } else if (exm_ == amask) { %supc = %uu; }\n"
               "   else { conv = false; if (inA) pc = ((exm_ >> lane) & 1u) ? %uu : %uu; }\n"
@@ -635,6 +660,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
         } else if (I.op == EXIT) {
             o(" { const bool pv = %s; ", G.guard(I.guard).c_str());
             G.rec(o, I, i, stepx, "pv");
+            G.flush_recs(o, code, run_start(i), i);
             o("const u32 exm_ = amask & __ballot_sync(JFULL, pv); step += %uu - pcm;\n"
               "   if (inA && pv) live = false; livem &= ~exm_; amask &= ~exm_; upc = %uu;\n"
               "   if (conv && (amask == 0u || upc >= npc)) { conv = false; if ((amask >> lane) & 1u) pc = upc; }\n"
@@ -649,9 +675,11 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
                 G.plain(o, I);
                 o(" }\n");
             }
-            if (i + 1 == n)
+            if (i + 1 == n) {
+                flush_end();
                 o(" { step += %uu - pcm; upc = %uu; if (upc >= npc) { conv = false; if (inA) pc = upc; } continue; }\n",
                   n, n);
+            }
         }
     }
     // ---- step mode: registers to the warp's shared-memory file, interpreter, back
@@ -680,8 +708,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "  Q0 = st_.preds & 1u; Q1 = (st_.preds >> 1) & 1u; Q2 = (st_.preds >> 2) & 1u; Q3 = (st_.preds >> 3) & 1u; "
       "Q4 = (st_.preds >> 4) & 1u; Q5 = (st_.preds >> 5) & 1u; Q6 = (st_.preds >> 6) & 1u;\n"
       "  if (done_) goto finish;\n  continue;\n }\n}\n");
-    if (mode == 2) o("finish:\n { const u32 rem_ = step & 31u; if (rem_ && lane < rem_) rec_out[step - rem_ + lane] = recbuf; }\n");
-    else o("finish:\n");
+    o("finish:\n");
     o("#undef out\n");
     o(" { JOut& out_ = *jx->out; out_.steps = step; out_.fault = jx->fault_[lane]; out_.fault_pc = jx->fault_pc_[lane]; "
       "out_.nstore = jx->nst_[lane];\n"

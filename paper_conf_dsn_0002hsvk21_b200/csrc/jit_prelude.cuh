@@ -516,10 +516,8 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
         const u32 pred = guard == 7 ? JFULL : __ballot_sync(JFULL, pv);
         const bool ex = act && pv;
         const u32 exm = active & pred;
-        if (MODE == JM_TRACE) {                       // one trace record per step (App. A.3)
-            if ((step & 31) == lane) recbuf = make_uint4(k, __ldg(&ins[pcm]), active, pred);
-            if ((step & 31) == 31) rec_out[step - 31 + lane] = recbuf;
-        }
+        if (MODE == JM_TRACE && lane == 0)            // one trace record per step (App. A.3)
+            rec_out[step] = make_uint4(k, __ldg(&ins[pcm]), active, pred);
         u32 taken = 0;
         if (op == 1) {                                // EXIT
             if (ex) live = false;
