@@ -967,8 +967,10 @@ fi_status compile_cubin(const fi_insn* code, const fi_kernel* kern, uint32_t n_k
     src = generate(code, kern, n_kern, n_regs, modes);
     void* prog = nullptr;
     if (N.create(&prog, src.c_str(), "fi_jit.cu", 0, nullptr, nullptr)) { g_jit_log = "nvrtcCreateProgram failed"; return FI_E_CUDA; }
-    const char* opts[] = {"--gpu-architecture=sm_100a", "--std=c++17", "--fmad=false", "-lineinfo"};
-    const int rc = N.compile(prog, 4, opts);
+    std::vector<const char*> opts = {"--gpu-architecture=sm_100a", "--std=c++17", "--fmad=false", "-lineinfo"};
+    std::string extra;                                // experiments: one more NVRTC option
+    if (const char* e = std::getenv("FI_JIT_NVRTC_OPT")) if (*e) { extra = e; opts.push_back(extra.c_str()); }
+    const int rc = N.compile(prog, (int)opts.size(), opts.data());
     size_t ls = 0;
     N.log_size(prog, &ls);
     std::string lg(ls, '\0');
