@@ -27,7 +27,9 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <atomic>
 #include <mutex>
+#include <thread>
 #include <string>
 #include <vector>
 
@@ -718,7 +720,10 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
     o("\n");
 }
 
-std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern, uint32_t n_regs, uint32_t modes) {
+// The module source of static kernel `only` (its device functions, and entry kernels
+// that serve only it), or of every kernel (only < 0: fi_jit_source's combined view).
+std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern, uint32_t n_regs, uint32_t modes,
+                     int only = -1) {
     // resident 128-thread CTAs per SM the register budget targets (3: <= 168 registers)
     uint32_t min_blocks = 3;
     if (const char* e = std::getenv("FI_JIT_MIN_BLOCKS")) min_blocks = (uint32_t)std::max(1, std::atoi(e));
@@ -726,7 +731,9 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
     if (std::getenv("FI_JIT_LDALLOC")) o.s = "#define JLD_L1 \"\"\n";
     o.s += kPrelude;
     Gen G{n_regs};
+    auto mine = [&](uint32_t k) { return only < 0 || (uint32_t)only == k; };
     for (uint32_t k = 0; k < n_kern; ++k) {
+        if (!mine(k)) continue;
         bool tables = true;
         if (modes & FI_JIT_INJECT) { gen_kernel(o, G, k, code + kern[k].code_off, kern[k].code_len, 0, tables); tables = false; }
         if (modes & FI_JIT_GOLDEN) {
@@ -751,16 +758,18 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
       " Rs[%uu + lane] = 0u;                     // the zero row (RZ, indices >= n_regs)\n"
       " for (;;) {\n  u32 p = 0u; if (lane == 0u) p = atomicAdd(counter, 1u); p = __shfl_sync(JFULL, p, 0);\n"
       "  if (p >= n) return;\n  const u32 i = order[p]; const jfi_site S = sites[i];\n"
-      "  if (S.flags & 1u) { if (lane == 0u) { jfi_inj r; r.before = r.after = r.mask = r.fault_pc = 0u; "
+      "  if (S.flags & 1u) { if (%s && lane == 0u) { jfi_inj r; r.before = r.after = r.mask = r.fault_pc = 0u; "
       "r.fault_kind = 0; r.outcome = 3; r.overflow = 0; r.flags = 0; r.n_faulty_stores = 0u; out[i] = r; } continue; }\n"
       "  const jfi_instance in = A.inst[S.instance]; const u32 wpc = (in.block + 31u) / 32u, lw = S.warp - in.warp_begin;\n"
+      "  if (%s) continue;                       // another module's replica\n"
       "  const u64 L = warp_off[S.warp + 1] - warp_off[S.warp]; const u64 wd = 10ull * L + 1024ull;\n"
       "  const u32 watchdog = wd > 0xFFFFFFFFull ? 0xFFFFFFFFu : (u32)wd;\n"
       "  u32* ck = ckpt ? (u32*)ckpt + ck_off[S.warp] * %uull : (u32*)0;\n"
       "  JOut o;\n  switch (in.kernel) {\n",
-      rs, zrow, ckw);
+      rs, zrow, only <= 0 ? "true" : "false", only < 0 ? "false" : ("in.kernel != " + std::to_string(only) + "u").c_str(),
+      ckw);
     for (uint32_t k = 0; k < n_kern; ++k)
-        o("   case %u: kern_%u_inj(A, S.step, S.pc, S.lane, S.dst_kind, S.dst_reg, S.bfm, S.mask, S.instance, lw / wpc, "
+        if (mine(k)) o("   case %u: kern_%u_inj(A, S.step, S.pc, S.lane, S.dst_kind, S.dst_reg, S.bfm, S.mask, S.instance, lw / wpc, "
           "lw %% wpc, watchdog, ck, ck ? ck_interval : 0u, log + (u64)i * cap, cap, o, Rs, A.dec + %uu, A.ins + %uu, "
           "(u8*)0, (uint4*)0, (const JPage*)0); break;\n",
           k, k, kern[k].code_off, kern[k].code_off);
@@ -790,7 +799,7 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
           "  JOut o;\n  switch (in.kernel) {\n",
           min_blocks, rs, zrow);
         for (uint32_t k = 0; k < n_kern; ++k)
-            o("   case %u: kern_%u_page(A, 0xFFFFFFFFu, 0u, 0u, 0u, 0u, 0u, 0u, t, lw / wpc, lw %% wpc, watchdog, (u32*)0, "
+            if (mine(k)) o("   case %u: kern_%u_page(A, 0xFFFFFFFFu, 0u, 0u, 0u, 0u, 0u, 0u, t, lw / wpc, lw %% wpc, watchdog, (u32*)0, "
               "0u, scr, K.log_cap, o, Rs, A.dec + %uu, A.ins + %uu, (u8*)0, (uint4*)0, &pg); break;\n",
               k, k, kern[k].code_off, kern[k].code_off);
         o("   default: o.steps = 0; o.fault = 4; o.fault_pc = 0; o.nstore = 0; break;\n  }\n"
@@ -816,27 +825,26 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
           " JOut o;\n switch (in.kernel) {\n",
           min_blocks, rs, zrow);
         for (uint32_t k = 0; k < n_kern; ++k)
-            o("  case %u: kern_%u_len(A, 0xFFFFFFFFu, 0u, 0u, 0u, 0u, 0u, 0u, k, lw / wpc, lw %% wpc, 0xFFFFFFFFu, (u32*)0, "
+            if (mine(k)) o("  case %u: kern_%u_len(A, 0xFFFFFFFFu, 0u, 0u, 0u, 0u, 0u, 0u, k, lw / wpc, lw %% wpc, 0xFFFFFFFFu, (u32*)0, "
               "0u, (jfi_store*)0, 0u, o, Rs, A.dec + %uu, A.ins + %uu, img_w, (uint4*)0, (const JPage*)0); break;\n",
               k, k, kern[k].code_off, kern[k].code_off);
         o("  default: o.steps = 0; o.fault = 9; o.nstore = 0; break;\n }\n"
           " if (lane == 0u) { warp_len[in.warp_begin + lw] = o.steps; warp_nst[in.warp_begin + lw] = o.nstore; "
           "if (o.fault) atomicOr(status, 1u << 4); }\n}\n");
-        o("extern \"C\" __global__ void __launch_bounds__(128, %u) k_golden_trace_jit(const JArgs A, const u32 n_warps, "
+        // (one launch per instance k, like pass 1: each module serves its own kernel's instances)
+        o("extern \"C\" __global__ void __launch_bounds__(128, %u) k_golden_trace_jit(const JArgs A, const u32 k, "
           "const u64* __restrict__ warp_off, const u64* __restrict__ gst_off, uint4* rec, jfi_store* gst, u32* ckpt, "
           "const u64* __restrict__ ck_off, const u32 ck_interval, u32* status) {\n"
           " extern __shared__ u32 jsmem[];\n const u32 lane = threadIdx.x & 31u;\n"
           " u32* Rs = jsmem + (threadIdx.x >> 5) * %uu;\n Rs[%uu + lane] = 0u;\n"
-          " const u32 w = blockIdx.x * 4u + (threadIdx.x >> 5);\n if (w >= n_warps) return;\n"
-          " u32 lo = 0, hi = A.n_inst;\n while (hi - lo > 1) { const u32 mid = (lo + hi) >> 1; "
-          "if (__ldg(&A.inst[mid].warp_begin) <= w) lo = mid; else hi = mid; }\n const u32 k = lo;\n"
-          " const jfi_instance in = A.inst[k];\n const u32 wpc = (in.block + 31u) / 32u, lw = w - in.warp_begin;\n"
+          " const jfi_instance in = A.inst[k];\n const u32 lw = blockIdx.x * 4u + (threadIdx.x >> 5);\n"
+          " if (lw >= in.warp_end - in.warp_begin) return;\n const u32 w = in.warp_begin + lw, wpc = (in.block + 31u) / 32u;\n"
           " const u64 r0 = warp_off[w], g0 = gst_off[w];\n"
           " u32* ck = ckpt ? ckpt + ck_off[w] * %uull : (u32*)0;\n"
           " JOut o;\n switch (in.kernel) {\n",
           min_blocks, rs, zrow, ckw);
         for (uint32_t k = 0; k < n_kern; ++k)
-            o("  case %u: kern_%u_trace(A, 0xFFFFFFFFu, 0u, 0u, 0u, 0u, 0u, 0u, k, lw / wpc, lw %% wpc, 0xFFFFFFFFu, ck, "
+            if (mine(k)) o("  case %u: kern_%u_trace(A, 0xFFFFFFFFu, 0u, 0u, 0u, 0u, 0u, 0u, k, lw / wpc, lw %% wpc, 0xFFFFFFFFu, ck, "
               "ck ? ck_interval : 0u, gst + g0, 0xFFFFFFFFu, o, Rs, A.dec + %uu, A.ins + %uu, (u8*)0, rec + r0, "
               "(const JPage*)0); break;\n",
               k, k, kern[k].code_off, kern[k].code_off);
@@ -926,11 +934,17 @@ thread_local std::string g_jit_log;
 // + 4 warps' JCtx (JCTX_BYTES of jit_prelude.cuh)
 static size_t jit_smem(uint32_t n_regs) { return (size_t)4 * (n_regs + 1) * 128 + 4 * 1280; }
 
+// one CUmodule per static kernel (compiled in parallel: ptxas time grows faster
+// than linearly with the size of one program), each with the entry kernels of
+// its own kernel
+struct fi_jit_mod {
+    CUmodule mod = nullptr;
+    CUfunction inject = nullptr, glen = nullptr, gtrace = nullptr, k8exec = nullptr;
+};
 struct fi_jit {
     size_t smem = 0;
     uint32_t modes = 0;
-    CUmodule mod = nullptr;
-    CUfunction inject = nullptr, glen = nullptr, gtrace = nullptr, k8exec = nullptr;
+    std::vector<fi_jit_mod> m;                        // [static kernel]
     uint32_t n_regs = 0, n_code = 0;
     double compile_s = 0;
     size_t src_bytes = 0, cubin_bytes = 0;
@@ -961,10 +975,10 @@ extern "C" size_t fi_jit_source(const fi_insn* code_host, uint32_t n_code, const
 
 namespace {
 fi_status compile_cubin(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern, uint32_t n_regs, uint32_t modes,
-                        std::string& src, std::vector<char>& cubin) {
+                        std::string& src, std::vector<char>& cubin, int only = -1) {
     Nvrtc& N = nvrtc();
     if (!N.ok) { g_jit_log = "libnvrtc.so.12 not found"; return FI_E_CUDA; }
-    src = generate(code, kern, n_kern, n_regs, modes);
+    src = generate(code, kern, n_kern, n_regs, modes, only);
     void* prog = nullptr;
     if (N.create(&prog, src.c_str(), "fi_jit.cu", 0, nullptr, nullptr)) { g_jit_log = "nvrtcCreateProgram failed"; return FI_E_CUDA; }
     std::vector<const char*> opts = {"--gpu-architecture=sm_100a", "--std=c++17", "--fmad=false", "-lineinfo"};
@@ -983,8 +997,9 @@ fi_status compile_cubin(const fi_insn* code, const fi_kernel* kern, uint32_t n_k
     N.cubin(prog, cubin.data());
     N.destroy(&prog);
     if (const char* d = std::getenv("FI_JIT_DUMP")) {     // profiling aid: the module's source and cubin
-        if (FILE* f = std::fopen((std::string(d) + ".cu").c_str(), "wb")) { std::fwrite(src.data(), 1, src.size(), f); std::fclose(f); }
-        if (FILE* f = std::fopen((std::string(d) + ".cubin").c_str(), "wb")) { std::fwrite(cubin.data(), 1, cubin.size(), f); std::fclose(f); }
+        const std::string b = std::string(d) + (only > 0 ? "_k" + std::to_string(only) : std::string());
+        if (FILE* f = std::fopen((b + ".cu").c_str(), "wb")) { std::fwrite(src.data(), 1, src.size(), f); std::fclose(f); }
+        if (FILE* f = std::fopen((b + ".cubin").c_str(), "wb")) { std::fwrite(cubin.data(), 1, cubin.size(), f); std::fclose(f); }
     }
     return FI_OK;
 }
@@ -994,16 +1009,50 @@ bool valid_kernels(const fi_kernel* kern, uint32_t n_kern, uint32_t n_code) {
         if ((uint64_t)kern[k].code_off + kern[k].code_len > n_code) return false;
     return true;
 }
+
+// every static kernel's module, NVRTC programs compiled by a pool of threads
+fi_status compile_all(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern, uint32_t n_regs, uint32_t modes,
+                      std::vector<std::vector<char>>& cubins, size_t& src_bytes) {
+    cubins.assign(n_kern, {});
+    std::vector<fi_status> st(n_kern, FI_OK);
+    std::vector<std::string> logs(n_kern);
+    std::vector<size_t> sb(n_kern, 0);
+    std::atomic<uint32_t> next{0};
+    auto work = [&] {
+        for (uint32_t k; (k = next.fetch_add(1)) < n_kern;) {
+            std::string src;
+            st[k] = compile_cubin(code, kern, n_kern, n_regs, modes, src, cubins[k], (int)k);
+            logs[k] = g_jit_log;                      // (thread_local: carried back to the caller)
+            sb[k] = src.size();
+        }
+    };
+    uint32_t nt = std::max(1u, std::min<uint32_t>(n_kern, std::thread::hardware_concurrency()));
+    if (const char* e = std::getenv("FI_JIT_THREADS")) nt = std::max(1, std::atoi(e));
+    std::vector<std::thread> pool;
+    for (uint32_t t = 1; t < nt; ++t) pool.emplace_back(work);
+    work();
+    for (auto& t : pool) t.join();
+    src_bytes = 0;
+    for (uint32_t k = 0; k < n_kern; ++k) {
+        src_bytes += sb[k];
+        if (st[k]) { g_jit_log = "static kernel " + std::to_string(k) + ": " + logs[k]; return st[k]; }
+    }
+    g_jit_log = logs.empty() ? std::string() : logs[0];
+    return FI_OK;
+}
 }  // namespace
 
 extern "C" fi_status fi_jit_compile_check(const fi_insn* code_host, uint32_t n_code, const fi_kernel* kern_host,
                                           uint32_t n_kern, uint32_t n_regs, uint32_t modes, size_t* cubin_bytes) {
     if (!code_host || !kern_host || !n_kern || n_regs == 0 || n_regs > fi::kRZ || !modes || modes > 7) return FI_E_ARG;
     if (!valid_kernels(kern_host, n_kern, n_code)) return FI_E_ARG;
-    std::string src;
-    std::vector<char> cubin;
-    fi_status e = compile_cubin(code_host, kern_host, n_kern, n_regs, modes, src, cubin);
-    if (cubin_bytes) *cubin_bytes = cubin.size();
+    std::vector<std::vector<char>> cubins;
+    size_t sb = 0;
+    fi_status e = compile_all(code_host, kern_host, n_kern, n_regs, modes, cubins, sb);
+    if (cubin_bytes) {
+        *cubin_bytes = 0;
+        for (auto& c : cubins) *cubin_bytes += c.size();
+    }
     return e;
 }
 
@@ -1018,31 +1067,38 @@ extern "C" fi_status fi_jit_build(const fi_program* p, const fi_kernel* kern_hos
     const auto t0 = std::chrono::steady_clock::now();
     fi_status e0 = fi::cuda_status(cudaFree(0));       // bind the device's primary context to this thread
     if (e0) return e0;
-    std::string src;
-    std::vector<char> cubin;
-    fi_status e = compile_cubin(p->code_host, kern_host, p->n_kern, p->n_regs, modes, src, cubin);
+    std::vector<std::vector<char>> cubins;
+    size_t src_bytes = 0;
+    fi_status e = compile_all(p->code_host, kern_host, p->n_kern, p->n_regs, modes, cubins, src_bytes);
     if (e) return e;
     fi_jit* j = new fi_jit();
     j->smem = jit_smem(p->n_regs);
-    bool ok = D.load(&j->mod, cubin.data()) == CUDA_SUCCESS;
-    auto get = [&](CUfunction* f, const char* name) {
-        ok = ok && D.get(f, j->mod, name) == CUDA_SUCCESS &&
-             D.set_attr(*f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)j->smem) == CUDA_SUCCESS;
-    };
-    if (modes & FI_JIT_INJECT) get(&j->inject, "k_inject_jit");
-    if (modes & FI_JIT_GOLDEN) { get(&j->glen, "k_golden_len_jit"); get(&j->gtrace, "k_golden_trace_jit"); }
-    if (modes & FI_JIT_PAGE) get(&j->k8exec, "k8_exec_jit");
+    j->m.resize(p->n_kern);
+    bool ok = true;
+    size_t cubin_bytes = 0;
+    for (uint32_t k = 0; k < p->n_kern && ok; ++k) {
+        fi_jit_mod& M = j->m[k];
+        cubin_bytes += cubins[k].size();
+        ok = D.load(&M.mod, cubins[k].data()) == CUDA_SUCCESS;
+        auto get = [&](CUfunction* f, const char* name) {
+            ok = ok && D.get(f, M.mod, name) == CUDA_SUCCESS &&
+                 D.set_attr(*f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)j->smem) == CUDA_SUCCESS;
+        };
+        if (modes & FI_JIT_INJECT) get(&M.inject, "k_inject_jit");
+        if (modes & FI_JIT_GOLDEN) { get(&M.glen, "k_golden_len_jit"); get(&M.gtrace, "k_golden_trace_jit"); }
+        if (modes & FI_JIT_PAGE) get(&M.k8exec, "k8_exec_jit");
+    }
     if (!ok) {
         g_jit_log += "\ncuModuleLoadData / cuModuleGetFunction / cuFuncSetAttribute failed";
-        if (j->mod) D.unload(j->mod);
+        for (auto& M : j->m) if (M.mod) D.unload(M.mod);
         delete j;
         return FI_E_CUDA;
     }
     j->modes = modes;
     j->n_regs = p->n_regs;
     j->n_code = p->n_code;
-    j->src_bytes = src.size();
-    j->cubin_bytes = cubin.size();
+    j->src_bytes = src_bytes;
+    j->cubin_bytes = cubin_bytes;
     j->compile_s = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
     *out = j;
     return FI_OK;
@@ -1052,7 +1108,7 @@ extern "C" double fi_jit_compile_seconds(const fi_jit* j) { return j ? j->compil
 
 extern "C" void fi_jit_free(fi_jit* j) {
     if (!j) return;
-    if (j->mod) drv().unload(j->mod);
+    for (auto& M : j->m) if (M.mod) drv().unload(M.mod);
     delete j;
 }
 
@@ -1107,15 +1163,25 @@ extern "C" fi_status fi_inject_jit(const fi_jit* j, const fi_program* p, const u
     int dev = 0, sms = 0, per = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    drv().occ(&per, j->inject, 128, j->smem);
-    const uint32_t grid = (uint32_t)std::min<uint64_t>((n + 3) / 4, (uint64_t)std::max(1, sms * std::max(1, per)));
     JArgsHost A = jargs(p, image);
     const uint64_t* warp_off = t->warp_off;
     const uint32_t* ckpt = t->ckpt;
     const uint64_t* ck_off = t->ckpt_off;
     void* args[] = {&A, (void*)&warp_off, (void*)&sites, &n, &out, &log, &log_cap, (void*)&ckpt, (void*)&ck_off,
                     (void*)&ck_iv, &order, &counter, &dev_status};
-    return launch(j->inject, grid, j->smem, s, args);
+    // each static kernel's module takes its own replicas off the LPT queue (k_lpt_order
+    // reset the queue counter; it is reset again before every later module)
+    for (size_t k = 0; k < j->m.size(); ++k) {
+        if (k) {
+            e = fi::cuda_status(cudaMemsetAsync(counter, 0, 4, s));
+            if (e) return e;
+        }
+        drv().occ(&per, j->m[k].inject, 128, j->smem);
+        const uint32_t grid = (uint32_t)std::min<uint64_t>((n + 3) / 4, (uint64_t)std::max(1, sms * std::max(1, per)));
+        e = launch(j->m[k].inject, grid, j->smem, s, args);
+        if (e) return e;
+    }
+    return FI_OK;
 }
 
 namespace fi {
@@ -1123,16 +1189,18 @@ namespace fi {
 fi_status jit_k8_exec(const fi_jit* j, const fi_program* p, const uint8_t* image, const JK8Host& K, uint32_t t,
                       uint32_t max_grid, cudaStream_t s) {
     if (!j || !(j->modes & FI_JIT_PAGE) || j->n_regs != p->n_regs || j->n_code != p->n_code) return FI_E_ARG;
+    if (!p->inst_host || t >= p->n_inst || p->inst_host[t].kernel >= j->m.size()) return FI_E_ARG;
+    CUfunction f = j->m[p->inst_host[t].kernel].k8exec;
     int dev = 0, sms = 0, per = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    drv().occ(&per, j->k8exec, 128, j->smem);
+    drv().occ(&per, f, 128, j->smem);
     const uint32_t grid = std::max<uint32_t>(1, std::min<uint32_t>((uint32_t)std::max(1, sms * std::max(1, per)), max_grid));
     JArgsHost A = jargs(p, image);
     JK8Host KK = K;
     uint32_t tt = t;
     void* args[] = {&A, &KK, &tt};
-    return launch(j->k8exec, grid, j->smem, s, args);
+    return launch(f, grid, j->smem, s, args);
 }
 }  // namespace fi
 
@@ -1147,7 +1215,8 @@ extern "C" fi_status fi_golden_lengths_jit(const fi_jit* j, const fi_program* p,
         if (!nw) continue;
         uint32_t kk = k;
         void* args[] = {&A, &kk, &image, &warp_len, &warp_nstore, &dev_status};
-        fi_status e = launch(j->glen, (nw + 3) / 4, j->smem, s, args);
+        if (p->inst_host[k].kernel >= j->m.size()) return FI_E_ARG;
+        fi_status e = launch(j->m[p->inst_host[k].kernel].glen, (nw + 3) / 4, j->smem, s, args);
         if (e) return e;
     }
     return FI_OK;
@@ -1159,14 +1228,23 @@ extern "C" fi_status fi_golden_trace_jit(const fi_jit* j, const fi_program* p, c
     if (!(j->modes & FI_JIT_GOLDEN) || j->n_regs != p->n_regs || j->n_code != p->n_code) return FI_E_ARG;
     if (t->ckpt && (!t->ckpt_off || !t->ckpt_interval)) return FI_E_ARG;
     if (!p->n_warps) return FI_OK;
+    if (!p->inst_host) return FI_E_ARG;
     JArgsHost A = jargs(p, image);
-    uint32_t nw = p->n_warps, iv = t->ckpt ? t->ckpt_interval : 0;
+    uint32_t iv = t->ckpt ? t->ckpt_interval : 0;
     const uint64_t* woff = t->warp_off;
     const uint64_t* goff = t->gstore_off;
     const uint64_t* ckoff = t->ckpt_off;
     fi_record* rec = t->rec;
     fi_store* gst = t->gstore;
     uint32_t* ck = t->ckpt;
-    void* args[] = {&A, &nw, (void*)&woff, (void*)&goff, &rec, &gst, &ck, (void*)&ckoff, &iv, &dev_status};
-    return launch(j->gtrace, (nw + 3) / 4, j->smem, (cudaStream_t)stream, args);
+    for (uint32_t k = 0; k < p->n_inst; ++k) {        // one launch per instance, on its kernel's module
+        const uint32_t nw = p->inst_host[k].warp_end - p->inst_host[k].warp_begin;
+        if (!nw) continue;
+        if (p->inst_host[k].kernel >= j->m.size()) return FI_E_ARG;
+        uint32_t kk = k;
+        void* args[] = {&A, &kk, (void*)&woff, (void*)&goff, &rec, &gst, &ck, (void*)&ckoff, &iv, &dev_status};
+        fi_status e = launch(j->m[p->inst_host[k].kernel].gtrace, (nw + 3) / 4, j->smem, (cudaStream_t)stream, args);
+        if (e) return e;
+    }
+    return FI_OK;
 }
