@@ -334,9 +334,17 @@ def secondary_c4(dev, n=256):
     import torch
     from fi_inputs import resnet as R
     from paper_conf_dsn_0002hsvk21_b200 import fi
+    import time as _t
     prog = R.c4(full=True)
     dp = fi.DeviceProgram(prog, dev)
-    gt = fi.golden_run(dp)
+    t0 = _t.perf_counter()
+    dp.jit(fi.FI_JIT_INJECT | fi.FI_JIT_GOLDEN | fi.FI_JIT_PAGE)     # one module per static kernel, compiled in parallel
+    jit_s = _t.perf_counter() - t0
+    torch.cuda.synchronize()
+    t0 = _t.perf_counter()
+    gt = fi.golden_run(dp, engine="jit")
+    torch.cuda.synchronize()
+    golden_s = _t.perf_counter() - t0
     ev = [torch.cuda.Event(enable_timing=True) for _ in range(5)]
     torch.cuda.synchronize()
     ev[0].record()
@@ -346,9 +354,9 @@ def secondary_c4(dev, n=256):
     sites = fi.select_sites(idx, fi.schedule(R.C4_CAMPAIGN_SEED, [fi.G_GP], [0]), 0, n)
     ev[2].record()
     cap = fi.log_capacity(gt)
-    out, log = fi.inject(gt, sites, n, cap, engine="interp")      # 29 kernels: K4 is 1 % here, not worth a JIT build
+    out, log = fi.inject(gt, sites, n, cap, engine="jit")
     ev[3].record()
-    hist = fi.classify_batched(gt, sites, n, out, log, cap)
+    hist = fi.classify_batched(gt, sites, n, out, log, cap, engine="jit")
     ev[4].record()
     torch.cuda.synchronize()
     ms = [ev[i].elapsed_time(ev[i + 1]) for i in range(4)]
@@ -360,7 +368,8 @@ def secondary_c4(dev, n=256):
             "records": gt.n_rec, "profile_thread_instrs_per_s": counted / (ms[0] / 1e3),
             "injections_per_s": n / ((ms[1] + ms[2] + ms[3]) / 1e3),
             "ms": {"profile": ms[0], "index_select": ms[1], "inject_k4": ms[2], "propagate_classify_k8": ms[3]},
-            "outcomes": {"masked": int(h[..., 0].sum()), "sdc": int(h[..., 1].sum()), "due": int(h[..., 2].sum())}}
+            "outcomes": {"masked": int(h[..., 0].sum()), "sdc": int(h[..., 1].sum()), "due": int(h[..., 2].sum())},
+            "engine": "jit", "jit_compile_s": jit_s, "golden_run_s": golden_s}
 
 
 def e2e(args, prog, seed, groups, bfms, n, rank, world, dev, camp):
