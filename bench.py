@@ -195,10 +195,19 @@ def main():
 
     import torch
     import torch.distributed as dist
+    # (FI_BENCH_SHARE_GPU=1: ranks share the visible GPUs, e.g. a 2-rank run on a
+    # 1-GPU box to exercise the multi-rank path; FI_BENCH_BACKEND=gloo there, since
+    # NCCL refuses two ranks on one GPU)
+    if os.environ.get("FI_BENCH_SHARE_GPU"):
+        local = local % torch.cuda.device_count()
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        backend = os.environ.get("FI_BENCH_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
     from paper_conf_dsn_0002hsvk21_b200 import fi
     from paper_conf_dsn_0002hsvk21_b200.campaign import Campaign, allreduce_max
 
