@@ -8,6 +8,7 @@ import subprocess
 import sys
 
 src_csv, dump = sys.argv[1], sys.argv[2]
+KERNEL = __import__("os").environ.get("JIT_KERNEL", "k_inject_jit")
 top = int(sys.argv[3]) if len(sys.argv) > 3 else 30
 rows = list(csv.reader(open(src_csv)))
 h = rows[1]
@@ -25,7 +26,7 @@ for line in subprocess.run(["nvdisasm", "-g", "-c", dump + ".cubin"], capture_ou
         cur = int(m.group(2))
         continue
     m = re.search(r"/\*([0-9a-f]{4,})\*/", line)
-    if m and cur and fn == "k_inject_jit":
+    if m and cur and fn == KERNEL:
         loc[int(m.group(1), 16)] = cur
 src = open(dump + ".cu").read().split("\n")
 agg = collections.defaultdict(lambda: [0, 0])
