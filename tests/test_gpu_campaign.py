@@ -163,3 +163,18 @@ def test_campaign_errors(F):
     with pytest.raises(F.FIError) as e:
         F.campaign(prog0, 1, [F.G_FP64], [0], 10)
     assert e.value.code == F.FI_E_EMPTY_GROUP
+
+
+def test_campaign_repeat_reuses_pool_then_release(F):
+    """fi_campaign's device memory comes from the device's default pool and stays
+    reserved between calls: a repeated campaign gives identical results, and
+    fi_campaign_release_memory hands the memory back."""
+    prog = P.c2(full=False)
+    r1 = F.campaign(prog, 11, [F.G_GP], [0, 1, 2, 3], 64)
+    r2 = F.campaign(prog, 11, [F.G_GP], [0, 1, 2, 3], 64)
+    assert np.array_equal(r1.hist, r2.hist)
+    assert np.array_equal(_site_rows(r1.sites), _site_rows(r2.sites))
+    assert np.array_equal(r1.inj["outcome"], r2.inj["outcome"])
+    F.campaign_release_memory()
+    r3 = F.campaign(prog, 11, [F.G_GP], [0, 1, 2, 3], 64)
+    assert np.array_equal(r1.hist, r3.hist)
