@@ -2,7 +2,7 @@
 exchanges the path has:
 
   1. after the sharded profile: all_reduce(SUM) of inst_counts [K][8] (u64 as
-     int64) and of chunk_counts [C][8] (each rank filled only its own chunks,
+     int64) and an all-gather of chunk_counts [C][8] (each rank filled only its own chunks,
      so the sum is an all-gather);
   2. at the end: all_reduce(SUM) of the outcome histogram [8][4][3].
 
@@ -41,6 +41,33 @@ def allreduce_sum_(t: torch.Tensor, group=None) -> torch.Tensor:
     if dist.is_available() and dist.is_initialized() and dist.get_world_size(group) > 1:
         dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
     return t
+
+
+def allgather_chunks_(cc: torch.Tensor, n_rec: int, group=None) -> torch.Tensor:
+    """In place: every rank's chunk_counts rows [c0_r, c1_r) (its record shard,
+    record_shard) gathered into every rank's [C][8] array — the same result as the
+    SUM all-reduce (each rank wrote only its own chunks, the rest are zero) with
+    half the bytes of a ring all-reduce: rank slices padded to ceil(C/G) rows,
+    one all_gather_into_tensor, then the slices copied into place."""
+    import torch.distributed as dist
+    if not (dist.is_available() and dist.is_initialized()):
+        return cc
+    world, rank = dist.get_world_size(group), dist.get_rank(group)
+    if world == 1:
+        return cc
+    C = cc.shape[0]
+    per = (C + world - 1) // world
+    bounds = [(C * r // world, C * (r + 1) // world) for r in range(world)]
+    c0, c1 = bounds[rank]
+    send = torch.zeros((per,) + tuple(cc.shape[1:]), dtype=cc.dtype, device=cc.device)
+    send[: c1 - c0] = cc[c0:c1]
+    recv = torch.empty((world * per,) + tuple(cc.shape[1:]), dtype=cc.dtype, device=cc.device)
+    dist.all_gather_into_tensor(recv, send, group=group)
+    for r, (a, b) in enumerate(bounds):
+        if r != rank and b > a:
+            cc[a:b] = recv[r * per: r * per + (b - a)]
+    assert (n_rec + FI_CHUNK - 1) // FI_CHUNK == C
+    return cc
 
 
 def allreduce_max(x: float, device, group=None) -> float:
@@ -119,7 +146,7 @@ class Campaign:
         mark("profile")
         if self.world > 1:
             allreduce_sum_(self.inst_counts, self.group)
-            allreduce_sum_(self.chunk_counts, self.group)
+            allgather_chunks_(self.chunk_counts, self.gt.n_rec, self.group)
         mark("exchange")
         idx = fi.SiteIndex(self.gt, self.inst_counts, self.chunk_counts, self.status)
         mark("index")

@@ -14,7 +14,8 @@ import torch.multiprocessing as mp
 
 import oracle as O
 from fi_inputs import programs as P
-from paper_conf_dsn_0002hsvk21_b200.campaign import allreduce_max, allreduce_sum_, record_shard, replica_block
+from paper_conf_dsn_0002hsvk21_b200.campaign import (allgather_chunks_, allreduce_max, allreduce_sum_, record_shard,
+                                                     replica_block)
 
 
 def _free_port():
@@ -48,8 +49,10 @@ def _worker(rank, world, port, prog_name, q):
     r0, r1 = record_shard(len(t), rank, world)
     c, ch = _partial_counts(t, r0, r1, len(prog.instances))
     ct, cht = torch.from_numpy(c), torch.from_numpy(ch)
+    chg = cht.clone()
     allreduce_sum_(ct)
     allreduce_sum_(cht)
+    allgather_chunks_(chg, len(t))                   # the bench's exchange: all-gather of the owned rows
     # replica block of a small campaign, oracle outcomes, histogram all-reduce
     n = 37
     j0, j1 = replica_block(n, rank, world)
@@ -63,7 +66,7 @@ def _worker(rank, world, port, prog_name, q):
         full_hist = O.histogram(full_sites, g.inject(full_sites, O.MODE_FULL, n_threads=1))
         fc, fch = _partial_counts(t, 0, len(t), len(prog.instances))
         q.put(dict(counts_ok=bool((ct.numpy() == fc).all() and (ct.numpy().astype(np.uint64) == g.counts()).all()),
-                   chunks_ok=bool((cht.numpy() == fch).all()),
+                   chunks_ok=bool((cht.numpy() == fch).all() and (chg.numpy() == fch).all()),
                    hist_ok=bool((h.numpy() == full_hist.astype(np.int64)).all()),
                    max_ok=(mx == float(world))))
     dist.barrier()
