@@ -218,7 +218,11 @@ def main():
 
     prog, seed, groups, bfms, n = make_program(args.config)
     n = args.replicas or n
-    camp = Campaign(prog, seed, groups, bfms, n, rank, world, dev)
+    # N > 1: the profile fused with its exchange (fi_profile_peers: chunk rows stored
+    # into the peers' memory by the profile kernel itself); FI_BENCH_EXCHANGE=collective
+    # for fi_profile + torch.distributed collectives instead
+    camp = Campaign(prog, seed, groups, bfms, n, rank, world, dev,
+                    exchange=os.environ.get("FI_BENCH_EXCHANGE", "peers"))
     torch.cuda.synchronize()
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
 
@@ -328,6 +332,8 @@ def main():
         "gpu_launches": 10 * K,
     }
 
+    if camp.peers is not None:
+        camp.peers.close()
     if not args.no_e2e:
         line["e2e"] = e2e(args, prog, seed, groups, bfms, n, rank, world, dev, camp)
     if rank == 0 and world == 1 and not args.no_secondary:

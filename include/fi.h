@@ -172,6 +172,43 @@ fi_status fi_profile(const fi_trace* t, uint64_t rec_begin, uint64_t rec_end, ui
  * in [rec_begin, rec_end) with opcode op of popc(active & pred) (u64 [n_inst][32],
  * zeroed by the call).  The executed-opcode set [PAPER.md:82] is its nonzero
  * columns. */
+/* ---- multi-GPU profile fused with its exchange ------------------
+ * One rank of G (<= FI_MAX_PEERS) GPUs: K1 over this rank's chunk-aligned record
+ * shard that ALSO stores every finished chunk-count row straight into each peer's
+ * chunk_counts (peer memory mapped over NVLink with fi_ipc_open), then pushes its
+ * partial instance counts into slot [rank] of every peer's partials, signals every
+ * peer's flag (system-scope release), waits until its own flag reaches
+ * epoch * G (all ranks' rows and partials arrived), sums the G partial slots
+ * into inst_counts [K][8] and copies the completed rows into chunk_counts [C][8]
+ * (caller's device arrays, as fi_profile's).  Replaces fi_profile + two all-reduces with one
+ * stream-ordered call: no host round trip, no separate collective.
+ * peers (host struct): chunk_counts[r] ([C][8] u32), partials[r] ([G][K][8] u64),
+ * flags[r] (u32, zero-initialised, never reset) of every rank r, this rank's own
+ * at [rank]; part_local: [K][8] u64 scratch of this rank; epoch: 1, 2, ... — the
+ * number of fi_profile_peers calls this rank has made, the same on every rank.
+ * Every rank must call it for every epoch (the wait spins on the device until the
+ * others do).  A rank must not start epoch e+1 before every rank has consumed the
+ * chunk_counts / partials of epoch e (the bench's per-step barrier).
+ * Errors: FI_E_ARG, FI_E_CUDA. */
+#define FI_MAX_PEERS 8
+typedef struct {
+    uint32_t* chunk_counts[FI_MAX_PEERS];
+    uint64_t* partials[FI_MAX_PEERS];
+    uint32_t* flags[FI_MAX_PEERS];
+    uint32_t world, rank;
+} fi_peers;
+fi_status fi_profile_peers(const fi_trace* t, uint64_t rec_begin, uint64_t rec_end, uint32_t n_inst,
+                           const fi_peers* peers, uint64_t* part_local, uint32_t epoch, uint64_t* inst_counts,
+                           uint32_t* chunk_counts, void* stream);
+/* Device memory shareable with the other ranks' processes (cudaMalloc +
+ * cudaIpcGetMemHandle): *dev_ptr (zero-filled) and its 64-B handle; fi_ipc_open
+ * maps a peer's handle into this process (peer access enabled lazily);
+ * fi_ipc_close unmaps it, fi_ipc_free frees this process's allocation. */
+fi_status fi_ipc_alloc(size_t bytes, void** dev_ptr, void* handle /* 64 B out */);
+fi_status fi_ipc_open(const void* handle /* 64 B */, void** dev_ptr);
+fi_status fi_ipc_close(void* dev_ptr);
+fi_status fi_ipc_free(void* dev_ptr);
+
 fi_status fi_profile_opcodes(const fi_trace* t, uint64_t rec_begin, uint64_t rec_end, uint32_t n_inst,
                              uint64_t* op_counts, void* stream);
 

@@ -93,13 +93,17 @@ class Campaign:
 
     def __init__(self, prog, seed: int, groups, bfms, n_replicas: int, rank: int = 0, world: int = 1,
                  device="cuda", group=None, host_tensors: dict | None = None, propagation: str = "auto",
-                 engine: str = "jit"):
+                 engine: str = "jit", exchange: str = "collective"):
         """propagation: how a multi-launch program's outcome is computed — "k7"
         (fi_classify: one CUDA warp walks a replica's later launches), "k8"
         (fi_classify_batched: replica batches in lockstep over the launches), or
         "auto" (K8 from 64 launches on).  Both give identical results.
         engine: "jit" (golden passes, K4 and K8 on the program's JIT module, built
-        once here) or "interp" (the shared-memory interpreter); identical results."""
+        once here) or "interp" (the shared-memory interpreter); identical results.
+        exchange (world > 1): "collective" (fi_profile, then torch.distributed
+        all-reduce / all-gather) or "peers" (fi_profile_peers: the profile kernel
+        stores its chunk rows straight into the peers' memory over NVLink and the
+        ranks synchronise on device flags — no separate collective); identical results."""
         from . import fi
         self.fi = fi
         self.prog = prog
@@ -120,6 +124,12 @@ class Campaign:
         K, C = self.dp.n_inst, max(self.gt.n_chunks, 1)
         self.inst_counts = torch.zeros((K, 8), dtype=torch.int64, device=self.device)
         self.chunk_counts = torch.zeros((C, 8), dtype=torch.int32, device=self.device)
+        self.peers = None
+        if exchange == "peers" and world > 1:
+            self.peers = fi.PeerExchange(C, K, rank, world, self.device, group)
+            self.chunk_counts = self.peers.chunk_counts   # (its rows arrive from the peers' profile kernels)
+        elif exchange not in ("collective", "peers"):
+            raise ValueError(exchange)
         self.sites = torch.empty(nloc * 64, dtype=torch.uint8, device=self.device)
         self.out = torch.empty(nloc * 24, dtype=torch.uint8, device=self.device)
         self.log = torch.empty(nloc * self.cap * 16, dtype=torch.uint8, device=self.device)
@@ -140,13 +150,19 @@ class Campaign:
                 ev[name].record()
 
         mark("start")
-        if self.world > 1:
-            self.chunk_counts.zero_()
-        fi.profile(self.gt, self.r0, self.r1, self.inst_counts, self.chunk_counts)
-        mark("profile")
-        if self.world > 1:
-            allreduce_sum_(self.inst_counts, self.group)
-            allgather_chunks_(self.chunk_counts, self.gt.n_rec, self.group)
+        if self.peers is not None:
+            # K1 with its rows stored into every peer, partial counts pushed, device-side
+            # flag wait, partial sum: one stream-ordered call, the exchange inside it
+            self.peers.profile(self.gt, self.r0, self.r1, self.inst_counts)
+            mark("profile")
+        else:
+            if self.world > 1:
+                self.chunk_counts.zero_()
+            fi.profile(self.gt, self.r0, self.r1, self.inst_counts, self.chunk_counts)
+            mark("profile")
+            if self.world > 1:
+                allreduce_sum_(self.inst_counts, self.group)
+                allgather_chunks_(self.chunk_counts, self.gt.n_rec, self.group)
         mark("exchange")
         idx = fi.SiteIndex(self.gt, self.inst_counts, self.chunk_counts, self.status)
         mark("index")

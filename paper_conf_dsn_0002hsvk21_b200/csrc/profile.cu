@@ -14,6 +14,7 @@
 // atomic per group per instance per warp).  Chunks that straddle instances
 // (rare: instance boundaries) attribute per record.
 #include <algorithm>
+#include <cstring>
 #include <vector>
 
 #include "common.cuh"
@@ -32,9 +33,18 @@ __device__ __forceinline__ uint4 ld_stream(const uint4* p) {
     return r;
 }
 
+// PEERS (fi_profile_peers, the multi-GPU path fused with its exchange): every
+// chunk-count row also goes straight into each peer rank's chunk_counts over
+// NVLink (P.cc[r], IPC-mapped), as the chunk is finished
+struct PeerOut {
+    uint32_t* cc[FI_MAX_PEERS];
+    uint32_t world, rank;
+};
+
+template <bool PEERS>
 __global__ void __launch_bounds__(kThreads)
 k_profile(const uint4* __restrict__ rec, uint64_t r_begin, uint64_t r_end, uint64_t c_begin, uint64_t c_end,
-          uint64_t* __restrict__ inst_counts, uint32_t* __restrict__ chunk_counts) {
+          uint64_t* __restrict__ inst_counts, uint32_t* __restrict__ chunk_counts, const PeerOut P) {
     const uint32_t lane = threadIdx.x & 31;
     const uint64_t gw = ((uint64_t)blockIdx.x * kThreads + threadIdx.x) >> 5;
     const uint64_t nwarps = ((uint64_t)gridDim.x * kThreads) >> 5;
@@ -73,7 +83,12 @@ k_profile(const uint4* __restrict__ rec, uint64_t r_begin, uint64_t r_end, uint6
             const uint32_t s = __reduce_add_sync(0xFFFFFFFFu, cnt[g]);
             if (lane == (uint32_t)g) mine = s;
         }
-        if (lane < 8) chunk_counts[c * 8 + lane] = mine;
+        if (lane < 8) {
+            chunk_counts[c * 8 + lane] = mine;
+            if (PEERS)
+                for (uint32_t r = 0; r < P.world; ++r)
+                    if (r != P.rank) P.cc[r][c * 8 + lane] = mine;
+        }
         if (kf == kl) {
             if (kf != cur_k) {
                 if (cur_k != kNone && lane < 8 && acc) atomicAdd((unsigned long long*)&inst_counts[(uint64_t)cur_k * 8 + lane], acc);
@@ -192,15 +207,111 @@ extern "C" fi_status fi_profile(const fi_trace* t, uint64_t rec_begin, uint64_t 
         int dev = 0, sms = 0, per = 0;
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_profile, kThreads, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_profile<false>, kThreads, 0);
         g_grid = std::max(1, sms * std::max(1, per));
     }
     const uint64_t c_begin = rec_begin / FI_CHUNK, c_end = (rec_end + FI_CHUNK - 1) / FI_CHUNK;
     const uint64_t warps_needed = c_end - c_begin;
     const int grid = (int)std::min<uint64_t>((uint64_t)g_grid, (warps_needed * 32 + kThreads - 1) / kThreads);
-    k_profile<<<grid, kThreads, 0, s>>>(reinterpret_cast<const uint4*>(t->rec), rec_begin, rec_end, c_begin, c_end,
-                                         inst_counts, chunk_counts);
+    k_profile<false><<<grid, kThreads, 0, s>>>(reinterpret_cast<const uint4*>(t->rec), rec_begin, rec_end, c_begin,
+                                                c_end, inst_counts, chunk_counts, PeerOut{});
     return launch_status();
+}
+
+// ---- multi-GPU profile fused with its exchange -------------------
+namespace fi {
+namespace {
+// this rank's partial instance counts into slot [rank] of every rank's partials
+__global__ void k_push_partials(const uint64_t* __restrict__ part, uint64_t n, fi_peers P) {
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t v = part[i];
+        for (uint32_t r = 0; r < P.world; ++r) P.partials[r][(uint64_t)P.rank * n + i] = v;
+    }
+}
+// release: everything this rank wrote to its peers is visible before its flag
+// increment reaches them (system scope)
+__global__ void k_signal(fi_peers P) {
+    __threadfence_system();
+    for (uint32_t r = 0; r < P.world; ++r) atomicAdd_system(P.flags[r], 1u);
+}
+// acquire: wait until every rank's increment of this epoch arrived
+__global__ void k_wait(const uint32_t* flag, uint32_t target) {
+    while (*reinterpret_cast<const volatile uint32_t*>(flag) < target) __nanosleep(200);
+    __threadfence_system();
+}
+__global__ void k_sum_partials(const uint64_t* __restrict__ part, uint64_t n, uint32_t world, uint64_t* __restrict__ out) {
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+        uint64_t s = 0;
+        for (uint32_t r = 0; r < world; ++r) s += part[(uint64_t)r * n + i];
+        out[i] = s;
+    }
+}
+}  // namespace
+}  // namespace fi
+
+extern "C" fi_status fi_ipc_alloc(size_t bytes, void** dev_ptr, void* handle) {
+    if (!dev_ptr || !handle) return FI_E_ARG;
+    void* p = nullptr;
+    fi_status e = cuda_status(cudaMalloc(&p, std::max<size_t>(bytes, 256)));
+    if (e) return e;
+    if ((e = cuda_status(cudaMemset(p, 0, std::max<size_t>(bytes, 256))))) { cudaFree(p); return e; }
+    cudaIpcMemHandle_t h;
+    if ((e = cuda_status(cudaIpcGetMemHandle(&h, p)))) { cudaFree(p); return e; }
+    std::memcpy(handle, &h, sizeof h);
+    *dev_ptr = p;
+    return FI_OK;
+}
+extern "C" fi_status fi_ipc_open(const void* handle, void** dev_ptr) {
+    if (!handle || !dev_ptr) return FI_E_ARG;
+    cudaIpcMemHandle_t h;
+    std::memcpy(&h, handle, sizeof h);
+    return cuda_status(cudaIpcOpenMemHandle(dev_ptr, h, cudaIpcMemLazyEnablePeerAccess));
+}
+extern "C" fi_status fi_ipc_close(void* dev_ptr) { return cuda_status(cudaIpcCloseMemHandle(dev_ptr)); }
+extern "C" fi_status fi_ipc_free(void* dev_ptr) { return cuda_status(cudaFree(dev_ptr)); }
+
+extern "C" fi_status fi_profile_peers(const fi_trace* t, uint64_t rec_begin, uint64_t rec_end, uint32_t n_inst,
+                                      const fi_peers* peers, uint64_t* part_local, uint32_t epoch,
+                                      uint64_t* inst_counts, uint32_t* chunk_counts, void* stream) {
+    if (!t || !peers || !part_local || !inst_counts || !chunk_counts || rec_end > t->n_rec || rec_begin > rec_end)
+        return FI_E_ARG;
+    if (rec_begin % FI_CHUNK || peers->world < 1 || peers->world > FI_MAX_PEERS || peers->rank >= peers->world ||
+        epoch == 0)
+        return FI_E_ARG;
+    const fi_peers P = *peers;
+    for (uint32_t r = 0; r < P.world; ++r)
+        if (!P.chunk_counts[r] || !P.partials[r] || !P.flags[r]) return FI_E_ARG;
+    cudaStream_t s = (cudaStream_t)stream;
+    const uint64_t n = (uint64_t)n_inst * 8;
+    fi_status e = cuda_status(cudaMemsetAsync(part_local, 0, n * sizeof(uint64_t), s));
+    if (e) return e;
+    if (rec_begin < rec_end) {
+        if (!g_grid) {
+            int dev = 0, sms = 0, per = 0;
+            cudaGetDevice(&dev);
+            cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_profile<false>, kThreads, 0);
+            g_grid = std::max(1, sms * std::max(1, per));
+        }
+        const uint64_t c_begin = rec_begin / FI_CHUNK, c_end = (rec_end + FI_CHUNK - 1) / FI_CHUNK;
+        const int grid = (int)std::min<uint64_t>((uint64_t)g_grid, ((c_end - c_begin) * 32 + kThreads - 1) / kThreads);
+        PeerOut po{};
+        for (uint32_t r = 0; r < P.world; ++r) po.cc[r] = P.chunk_counts[r];
+        po.world = P.world;
+        po.rank = P.rank;
+        k_profile<true><<<grid, kThreads, 0, s>>>(reinterpret_cast<const uint4*>(t->rec), rec_begin, rec_end, c_begin,
+                                                   c_end, part_local, P.chunk_counts[P.rank], po);
+        if ((e = launch_status())) return e;
+    }
+    const uint32_t pg = (uint32_t)std::min<uint64_t>(std::max<uint64_t>(1, (n + 255) / 256), 1184);
+    k_push_partials<<<pg, 256, 0, s>>>(part_local, n, P);
+    k_signal<<<1, 1, 0, s>>>(P);
+    k_wait<<<1, 1, 0, s>>>(P.flags[P.rank], epoch * P.world);
+    k_sum_partials<<<pg, 256, 0, s>>>(P.partials[P.rank], n, P.world, inst_counts);
+    if ((e = launch_status())) return e;
+    const uint64_t C = (t->n_rec + FI_CHUNK - 1) / FI_CHUNK;  // every rank's rows, now complete, to the caller's array
+    return cuda_status(cudaMemcpyAsync(chunk_counts, P.chunk_counts[P.rank], C * 8 * sizeof(uint32_t),
+                                       cudaMemcpyDeviceToDevice, s));
 }
 
 extern "C" fi_status fi_profile_opcodes(const fi_trace* t, uint64_t rec_begin, uint64_t rec_end, uint32_t n_inst,

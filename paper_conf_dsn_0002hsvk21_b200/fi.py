@@ -75,6 +75,14 @@ class fi_schedule(C.Structure):
                 ("groups", C.c_uint8 * 8), ("bfms", C.c_uint8 * 4)]
 
 
+FI_MAX_PEERS = 8
+
+
+class fi_peers(C.Structure):
+    _fields_ = [("chunk_counts", C.c_void_p * FI_MAX_PEERS), ("partials", C.c_void_p * FI_MAX_PEERS),
+                ("flags", C.c_void_p * FI_MAX_PEERS), ("world", C.c_uint32), ("rank", C.c_uint32)]
+
+
 class fi_campaign_cfg(C.Structure):
     _fields_ = [("code", C.c_void_p), ("n_code", C.c_uint32),
                 ("kern", C.c_void_p), ("n_kern", C.c_uint32),
@@ -168,6 +176,11 @@ def lib():
             "fi_campaign": (st, [C.POINTER(fi_campaign_cfg), C.c_int, C.c_int, ALLREDUCE_FN, vp,
                                  C.POINTER(fi_campaign_result)]),
             "fi_campaign_release_memory": (st, [C.c_int]),
+            "fi_profile_peers": (st, [vp, u64, u64, u32, vp, vp, u32, vp, vp, vp]),
+            "fi_ipc_alloc": (st, [sz, C.POINTER(C.c_void_p), vp]),
+            "fi_ipc_open": (st, [vp, C.POINTER(C.c_void_p)]),
+            "fi_ipc_close": (st, [vp]),
+            "fi_ipc_free": (st, [vp]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -420,6 +433,62 @@ def profile(gt: GoldenTrace, rec_begin: int = 0, rec_end: int | None = None,
     _check(lib().fi_profile(C.byref(gt.c), rec_begin, rec_end, K, _p(inst_counts), _p(chunk_counts), _stream()),
            "fi_profile")
     return inst_counts, chunk_counts
+
+
+class PeerExchange:
+    """The buffers of fi_profile_peers for one rank: this rank's
+    chunk_counts [C][8] u32, partials [G][K][8] u64 and flag, allocated shareable
+    (fi_ipc_alloc), their handles exchanged through torch.distributed
+    (all_gather_object), every peer's mapped here (fi_ipc_open)."""
+
+    def __init__(self, n_chunks: int, n_inst: int, rank: int, world: int, device, group=None):
+        import torch.distributed as dist
+        assert 1 <= world <= FI_MAX_PEERS
+        self.world, self.rank, self.n_inst, self.device = world, rank, n_inst, torch.device(device)
+        self.epoch = 0
+        sizes = (max(n_chunks, 1) * 8 * 4, world * max(n_inst, 1) * 8 * 8, 256)
+        self.own, handles = [], []
+        for b in sizes:
+            ptr, h = C.c_void_p(), C.create_string_buffer(64)
+            _check(lib().fi_ipc_alloc(b, C.byref(ptr), h), "fi_ipc_alloc")
+            self.own.append(ptr.value)
+            handles.append(h.raw)
+        allh = [None] * world
+        dist.all_gather_object(allh, handles, group=group)
+        self.opened = []
+        self.peers = fi_peers()
+        self.peers.world, self.peers.rank = world, rank
+        for r in range(world):
+            for q, arr in enumerate((self.peers.chunk_counts, self.peers.partials, self.peers.flags)):
+                if r == rank:
+                    arr[r] = self.own[q]
+                else:
+                    ptr = C.c_void_p()
+                    _check(lib().fi_ipc_open(C.create_string_buffer(allh[r][q], 64), C.byref(ptr)), "fi_ipc_open")
+                    self.opened.append(ptr.value)
+                    arr[r] = ptr.value
+        self.part_local = torch.empty((max(n_inst, 1), 8), dtype=torch.int64, device=self.device)
+        self.chunk_counts = torch.zeros((max(n_chunks, 1), 8), dtype=torch.int32, device=self.device)
+
+    def profile(self, gt: "GoldenTrace", rec_begin: int, rec_end: int, inst_counts: torch.Tensor) -> None:
+        self.epoch += 1
+        _check(lib().fi_profile_peers(C.byref(gt.c), rec_begin, rec_end, gt.dp.n_inst, C.byref(self.peers),
+                                      _p(self.part_local), self.epoch, _p(inst_counts), _p(self.chunk_counts),
+                                      _stream()), "fi_profile_peers")
+
+    def close(self, group=None):
+        """Unmap the peers' buffers, wait for every rank to have done the same, then
+        free this rank's (collective: every rank calls it)."""
+        import torch.distributed as dist
+        torch.cuda.synchronize(self.device)
+        for p in self.opened:
+            lib().fi_ipc_close(p)
+        self.opened = []
+        if dist.is_available() and dist.is_initialized():
+            dist.barrier(group=group)
+        for p in self.own:
+            lib().fi_ipc_free(p)
+        self.own = []
 
 
 class SiteIndex:
