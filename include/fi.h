@@ -187,7 +187,7 @@ fi_status fi_profile(const fi_trace* t, uint64_t rec_begin, uint64_t rec_end, ui
  * at [rank]; part_local: [K][8] u64 scratch of this rank; epoch: 1, 2, ... — the
  * number of fi_profile_peers calls this rank has made, the same on every rank.
  * Every rank must call it for every epoch (the wait spins on the device until the
- * others do).  A rank must not start epoch e+1 before every rank has consumed the
+ * others do; after 60 s without them it traps: a CUDA error, not a hung GPU).  A rank must not start epoch e+1 before every rank has consumed the
  * chunk_counts / partials of epoch e (the bench's per-step barrier).
  * Errors: FI_E_ARG, FI_E_CUDA. */
 #define FI_MAX_PEERS 8

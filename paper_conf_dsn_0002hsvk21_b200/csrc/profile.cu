@@ -234,9 +234,20 @@ __global__ void k_signal(fi_peers P) {
     __threadfence_system();
     for (uint32_t r = 0; r < P.world; ++r) atomicAdd_system(P.flags[r], 1u);
 }
-// acquire: wait until every rank's increment of this epoch arrived
+// acquire: wait until every rank's increment of this epoch arrived.  Bounded: a
+// rank that never signals (it died) turns into a device trap after 60 s — a loud
+// CUDA error in this process instead of a GPU spinning forever.
+__device__ __forceinline__ uint64_t globaltimer_ns() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
 __global__ void k_wait(const uint32_t* flag, uint32_t target) {
-    while (*reinterpret_cast<const volatile uint32_t*>(flag) < target) __nanosleep(200);
+    const uint64_t t0 = globaltimer_ns();
+    while (*reinterpret_cast<const volatile uint32_t*>(flag) < target) {
+        __nanosleep(200);
+        if (globaltimer_ns() - t0 > 60ull * 1000000000ull) __trap();
+    }
     __threadfence_system();
 }
 __global__ void k_sum_partials(const uint64_t* __restrict__ part, uint64_t n, uint32_t world, uint64_t* __restrict__ out) {
