@@ -1,7 +1,7 @@
 """fi_profile_peers: the multi-GPU profile fused with its exchange —
 K1 stores its chunk-count rows straight into the peer ranks' memory (IPC-mapped),
-pushes partial instance counts, and the ranks meet on device flags.  Two ranks
-share the one GPU here (two processes, IPC on the same device, gloo only for the
+pushes partial instance counts, and the ranks meet on device flags.  Two or three
+ranks share the one GPU here (processes, IPC on the same device, gloo only for the
 handle exchange); counts, chunk counts, histograms and per-replica outcomes must
 equal the single-rank campaign's, over several epochs."""
 import os
@@ -47,7 +47,8 @@ def _worker(rank, world, port, q):
     dist.destroy_process_group()
 
 
-def test_profile_peers_equals_single_rank():
+@pytest.mark.parametrize("world", [2, 3])
+def test_profile_peers_equals_single_rank(world):
     from fi_inputs import programs as P
     from paper_conf_dsn_0002hsvk21_b200 import fi
     from paper_conf_dsn_0002hsvk21_b200.campaign import Campaign
@@ -56,7 +57,6 @@ def test_profile_peers_equals_single_rank():
     torch.cuda.synchronize()
     ic, cc, hist = ref.inst_counts.cpu().numpy(), ref.chunk_counts.cpu().numpy(), ref.hist.cpu().numpy()
     ref_out = ref.inj_np()["outcome"]
-    world = 2
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
