@@ -59,6 +59,8 @@ struct Src {
     }
 };
 
+constexpr int kJbcSlots = 4;                        // JBC_SLOTS of jit_prelude.cuh
+
 struct Gen {
     uint32_t NR;                                      // register rows (fi_program.n_regs)
     std::string R(uint32_t j) const { return j < NR ? "R" + std::to_string(j) : std::string("0u"); }
@@ -292,6 +294,9 @@ struct Gen {
 
     // LDG / STG.  `stepx` = this instruction's step.
     uint32_t mode = 0;                               // JM_INJ / JM_LEN / JM_TRACE of jit_prelude.cuh
+    // buffer-cache entry (JBufCache slot) of each address register of the kernel being generated
+    std::vector<int> slot_of = std::vector<int>(256, 0);
+    int slot(const fi_insn& I) const { return slot_of[I.a & 0xFF]; }
     // trace record of the instruction at pc (App. A.3): written only in JM_TRACE
     // Block code writes the records of a whole block when it leaves it (flush_recs);
     // here only a guarded instruction's predicate mask is kept for that.
@@ -318,16 +323,18 @@ struct Gen {
         rec(o, I, pc, stepx, "pv");
         o("const u64 va = %s + (u64)(i64)(i32)%s; ", R64(I.a).c_str(), hex(I.imm).c_str());
         if (I.op == LDG) {
-            o("uint4 v_; const u32 c_ = jldg<%uu>(A, jimg, bc, va, k, ex, v_%s); ", lw, mode == 3 ? ", PG.page_base" : "");
+            o("uint4 v_; const u32 c_ = jldg<%uu, %d>(A, jimg, bc, va, k, ex, v_%s); ", lw, slot(I),
+              mode == 3 ? ", PG.page_base" : "");
             o("if (__ballot_sync(JFULL, c_ != 0u)) { fault = __ballot_sync(JFULL, c_ == 1u) ? 1u : 2u; fault_pc = %uu; "
               "step = %s; goto finish; } ", pc, stepx);
-            if (mode == 3) o("if (ex) jpage_c<%uu>(A, bc, PG, va, v_); ", nw);
+            if (mode == 3) o("if (ex) jpage_c<%uu, %d>(A, bc, PG, va, v_); ", nw, slot(I));
             const char* v[] = {"v_.x", "v_.y", "v_.z", "v_.w"};
             wr(o, I.d0, v, nw);
             o("}\n");
         } else {
             o("const u32 exm_ = amask & __ballot_sync(JFULL, pv); bool z_ = false; "
-              "const u32 c_ = ex ? jcheck(A, bc, va, %uu, k, &z_%s) : 0u; ", 4u << lw, mode == 3 ? ", PG.page_base" : "");
+              "const u32 c_ = ex ? jcheck<%d>(A, bc, va, %uu, k, &z_%s) : 0u; ", slot(I), 4u << lw,
+              mode == 3 ? ", PG.page_base" : "");
             o("if (__ballot_sync(JFULL, c_ != 0u)) { fault = __ballot_sync(JFULL, c_ == 1u) ? 1u : 2u; fault_pc = %uu; "
               "step = %s; goto finish; } ", pc, stepx);
             if (mode == 1) {                           // golden pass 1: into the image
@@ -374,13 +381,13 @@ struct Gen {
         for (uint32_t j = 0; j < m; ++j) {
             const fi_insn& I = code[i0 + j];
             const uint32_t lw = (I.mod & 3) > 2 ? 2 : (I.mod & 3);
-            o(" & (!ex%u | jhit(bc, va%u, %uu, &z%u))", j, j, 4u << lw, j);
+            o(" & (!ex%u | jhit<%d>(bc, va%u, %uu, &z%u))", j, slot(I), j, 4u << lw, j);
         }
         o("))) {\n");
         for (uint32_t j = 0; j < m; ++j) {
             const fi_insn& I = code[i0 + j];
             const uint32_t lw = (I.mod & 3) > 2 ? 2 : (I.mod & 3);
-            o("   c%u = ex%u ? jcheck(A, bc, va%u, %uu, k, &z%u%s) : 0u;\n", j, j, j, 4u << lw, j,
+            o("   c%u = ex%u ? jcheck<%d>(A, bc, va%u, %uu, k, &z%u%s) : 0u;\n", j, j, slot(I), j, 4u << lw, j,
               mode == 3 ? ", PG.page_base" : "");
         }
         o("  }\n");
@@ -409,7 +416,7 @@ struct Gen {
             if (lw == 0) o("v_.x = jld32(p_); ");
             else if (lw == 1) o("const uint2 t_ = jld64(p_); v_.x = t_.x; v_.y = t_.y; ");
             else o("v_ = jld128(p_); ");
-            if (mode == 3) o("jpage_c<%uu>(A, bc, PG, va%u, v_); ", nw, j);
+            if (mode == 3) o("jpage_c<%uu, %d>(A, bc, PG, va%u, v_); ", nw, slot(I), j);
             if (I.d0 != fi::kRZ)
                 for (uint32_t q = 0; q < nw; ++q)
                     if (W(I.d0 + q)) o("R%u = v_.%c; ", I.d0 + q, "xyzw"[q]);
@@ -423,7 +430,7 @@ struct Gen {
         for (uint32_t j = 0; j < m && j < stride.size(); ++j) {
             bool first = !stride[j].empty();
             for (uint32_t q = 0; q < j && first; ++q) first = code[i0 + q].a != code[i0 + j].a;
-            if (first) o("  if (ex%u) jprefetch(jimg, bc, va%u + (%s));\n", j, j, stride[j].c_str());
+            if (first) o("  if (ex%u) jprefetch<%d>(jimg, bc, va%u + (%s));\n", j, slot(code[i0 + j]), j, stride[j].c_str());
         }
         o(" }\n");
     }
@@ -501,6 +508,17 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
     using namespace fi;
     Gen G = G0;
     G.mode = mode;
+    // one cache entry per address register, in order of first use (wrapping beyond JBC_SLOTS)
+    {
+        std::vector<int> seen(256, -1);
+        int next = 0;
+        for (uint32_t i = 0; i < n; ++i) {
+            if (code[i].op != LDG && code[i].op != STG) continue;
+            const uint32_t a = code[i].a & 0xFF;
+            if (seen[a] < 0) seen[a] = next++ % kJbcSlots;
+            G.slot_of[a] = seen[a];
+        }
+    }
     const uint32_t NR = G.NR;
     static const char* const mname[] = {"inj", "len", "trace", "page"};
     // block length from each pc: to the next BRA/EXIT inclusive, or the code end
@@ -696,7 +714,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "  st_.preds = (u32)Q0 | ((u32)Q1 << 1) | ((u32)Q2 << 2) | ((u32)Q3 << 3) | ((u32)Q4 << 4) | ((u32)Q5 << 5) | "
       "((u32)Q6 << 6); st_.recbuf = recbuf;\n"
       "  __syncwarp();\n"
-      "  JBufCache bcs_ = bc;                // (a copy: bc's address never escapes, so it stays in registers)\n"
+      "  JBufCache bcs_;                     // (step mode's own cache: bc's address never escapes, so it stays in registers)\n"
       "  const u32 done_ = jinterp<%u>(A, st_, bcs_, Rs, dec, kblen_%u, %uu, k, cta, wic, watchdog, hstep, hpc, hlane, "
       "hkind, hreg, hbfm, hmask, st_out, st_cap, %uu, img_w, rec_out, ck, ck_interval, ins, pgp);\n"
       "  __syncwarp();\n",
@@ -706,7 +724,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "amask = st_.amask; npc = st_.npc; jx->nst_[lane] = st_.nst; jx->fault_[lane] = st_.fault; "
       "jx->fault_pc_[lane] = st_.fault_pc; jx->before_[lane] = st_.before; jx->after_[lane] = st_.after; "
       "jx->msk_[lane] = st_.msk; jx->fired_[lane] = st_.fired; jx->bad_[lane] = st_.bad; lim = st_.lim; "
-      "recbuf = st_.recbuf; bc = bcs_;\n"
+      "recbuf = st_.recbuf;\n"
       "  Q0 = st_.preds & 1u; Q1 = (st_.preds >> 1) & 1u; Q2 = (st_.preds >> 2) & 1u; Q3 = (st_.preds >> 3) & 1u; "
       "Q4 = (st_.preds >> 4) & 1u; Q5 = (st_.preds >> 5) & 1u; Q6 = (st_.preds >> 6) & 1u;\n"
       "  if (done_) goto finish;\n  continue;\n }\n}\n");

@@ -161,45 +161,53 @@ __device__ __forceinline__ uint4 jld128(const u8* p) {
     return r;
 }
 
-// per-lane two-entry cache of buffer bounds, 32-bit: image offset `lo` and the
-// size floored to 16 B (`sz`; 0 = empty entry).  Only buffers with lo % 16 == 0
-// and lo + size <= 2^31 are cached (others always take jcheck's full path), so
-// for an aligned address va = JVA_BASE + off: off is in the entry iff
-// hi32(va) == hi32(JVA_BASE) and (u32)(lo32(va) - lo) < sz — an offset below lo
-// wraps to >= 2^31 > sz, and d < sz with d, sz multiples of the access width w
+// per-lane cache of buffer bounds, JBC_SLOTS entries, 32-bit: image offset `lo`
+// and the size floored to 16 B (`sz`; 0 = empty entry).  The generator gives each
+// memory instruction a fixed entry (slot) by its address register, so a loop that
+// walks several buffers through different pointers keeps one entry per pointer;
+// the step-mode interpreter uses entry 0 of its own cache.  Only buffers with
+// lo % 16 == 0 and lo + size <= 2^31 are cached (others always take jcheck's
+// full path), so for an aligned address va = JVA_BASE + off: off is in the entry
+// iff hi32(va) == hi32(JVA_BASE) and (u32)(lo32(va) - lo) < sz — an offset below
+// lo wraps to >= 2^31 > sz, and d < sz with d, sz multiples of the access width w
 // gives d + w <= sz <= size.  A miss is never wrong, only slower.
 static_assert((JVA_BASE & 0xFFFFFFFFull) == 0, "the cache tests the low word of va only");
 #define JVA_HI ((u32)(JVA_BASE >> 32))
+#define JBC_SLOTS 4
 struct JBufCache {
-    u32 lo0, sz0, lo1, sz1;
-    bool z0, z1;
-    u32 b0, b1, pb0, pb1;        // buffer ids and their first page index (K8 page tables; 0 elsewhere)
-    __device__ __forceinline__ JBufCache()
-        : lo0(0), sz0(0), lo1(0), sz1(0), z0(false), z1(false), b0(0), b1(0), pb0(0), pb1(0) {}
+    u32 lo[JBC_SLOTS], sz[JBC_SLOTS];
+    bool z[JBC_SLOTS];
+    u32 b[JBC_SLOTS], pb[JBC_SLOTS];   // buffer ids and their first page index (K8 page tables; 0 elsewhere)
+    __device__ __forceinline__ JBufCache() {
+#pragma unroll
+        for (int i = 0; i < JBC_SLOTS; ++i) { lo[i] = 0; sz[i] = 0; z[i] = false; b[i] = 0; pb[i] = 0; }
+    }
 };
 
-// cache-only check: true iff the access is aligned and inside one of the two
-// cached buffers (then *zero is that buffer's writer-rule flag); no state change
+// cache-only check against entry S: true iff the access is aligned and inside the
+// buffer cached there (then *zero is that buffer's writer-rule flag); no state change
+template <int S>
 __device__ __forceinline__ bool jhit(const JBufCache& C, u64 va, u32 w, bool* zero) {
     const u32 vlo = (u32)va;
-    const bool h0 = vlo - C.lo0 < C.sz0;
-    const bool h1 = vlo - C.lo1 < C.sz1;
-    *zero = h0 ? C.z0 : C.z1;
-    return ((u32)(va >> 32) == JVA_HI) & ((vlo & (w - 1)) == 0) & (h0 | h1);
+    *zero = C.z[S];
+    return ((u32)(va >> 32) == JVA_HI) & ((vlo & (w - 1)) == 0) & (vlo - C.lo[S] < C.sz[S]);
 }
 __device__ const uint4 jzero16[1] = {{0u, 0u, 0u, 0u}};   // the zero line of writer-rule loads
-// L1 prefetch of an address inside one of the lane's cached buffers (else nothing)
+// L1 prefetch of an address inside the buffer cached in entry S (else nothing)
+template <int S>
 __device__ __forceinline__ void jprefetch(const u8* __restrict__ img, const JBufCache& C, u64 va) {
     const u32 vlo = (u32)va;
-    if (((u32)(va >> 32) == JVA_HI) & ((vlo - C.lo0 < C.sz0) | (vlo - C.lo1 < C.sz1)))
+    if (((u32)(va >> 32) == JVA_HI) & (vlo - C.lo[S] < C.sz[S]))
         asm volatile("prefetch.global.L1 [%0];" ::"l"(img + (va - JVA_BASE)));
 }
 
-// 0 ok, 1 misaligned, 2 unmapped (C-15); *zero = writer rule for instance k
+// 0 ok, 1 misaligned, 2 unmapped (C-15); *zero = writer rule for instance k.
+// A miss refills entry S.
+template <int S>
 __device__ __forceinline__ u32 jcheck(const JArgs& A, JBufCache& C, u64 va, u32 w, u32 k, bool* zero,
                                       const u32* page_base = nullptr) {
     if (va & (w - 1)) return 1;
-    if (jhit(C, va, w, zero)) return 0;
+    if (jhit<S>(C, va, w, zero)) return 0;
     const u64 off = va - JVA_BASE;
     if (va < JVA_BASE || off >= A.image_bytes) return 2;
     const u32 b = __ldg(&A.gran[off >> 8]);
@@ -210,19 +218,18 @@ __device__ __forceinline__ u32 jcheck(const JArgs& A, JBufCache& C, u64 va, u32 
     const bool z = wr >= 0 && (u32)wr >= k;
     *zero = z;
     if ((lo & 15u) == 0 && lo + size <= 0x80000000ull && size >= 16) {
-        C.lo1 = C.lo0; C.sz1 = C.sz0; C.z1 = C.z0; C.b1 = C.b0; C.pb1 = C.pb0;
-        C.lo0 = (u32)lo; C.sz0 = (u32)size & ~15u; C.z0 = z; C.b0 = b;
-        C.pb0 = page_base ? __ldg(&page_base[b]) : 0u;
+        C.lo[S] = (u32)lo; C.sz[S] = (u32)size & ~15u; C.z[S] = z; C.b[S] = b;
+        C.pb[S] = page_base ? __ldg(&page_base[b]) : 0u;
     }
     return 0;
 }
 
 // one LDG of 1/2/4 words for this lane; returns the fault code (0 ok)
-template <u32 LW>
+template <u32 LW, int S>
 __device__ __forceinline__ u32 jldg(const JArgs& A, const u8* __restrict__ img, JBufCache& C, u64 va, u32 k, bool ex,
                                     uint4& v, const u32* page_base = nullptr) {
     bool zero = false;
-    const u32 c = ex ? jcheck(A, C, va, 4u << LW, k, &zero, page_base) : 0u;
+    const u32 c = ex ? jcheck<S>(A, C, va, 4u << LW, k, &zero, page_base) : 0u;
     v = make_uint4(0, 0, 0, 0);
     if (ex && !c && !zero) {
         const u8* src = img + (va - JVA_BASE);
@@ -436,16 +443,14 @@ __device__ __forceinline__ void jpage(const JArgs& A, const JPage& G, u64 va, ui
         *G.inexact = 1u;
     }
 }
-// the same through the lane's buffer cache when one of its entries holds the
-// access (one page-table load), else jpage's full lookup
-template <u32 NW>
+// the same through entry S of the lane's buffer cache when it holds the access
+// (one page-table load), else jpage's full lookup
+template <u32 NW, int S>
 __device__ __forceinline__ void jpage_c(const JArgs& A, const JBufCache& C, const JPage& G, u64 va, uint4& v) {
-    const u32 vlo = (u32)va, d0 = vlo - C.lo0, d1 = vlo - C.lo1;
-    const bool e0 = d0 < C.sz0;
-    if (!e0 && !(d1 < C.sz1)) { jpage<NW>(A, G, va, v); return; }
-    const u32 rel = e0 ? d0 : d1;
-    const u32 b = e0 ? C.b0 : C.b1;
-    const u32 e = G.ptab[(e0 ? C.pb0 : C.pb1) + (rel >> 12)];
+    const u32 rel = (u32)va - C.lo[S];
+    if (!(rel < C.sz[S])) { jpage<NW>(A, G, va, v); return; }
+    const u32 b = C.b[S];
+    const u32 e = G.ptab[C.pb[S] + (rel >> 12)];
     if (e < JPAGE_CLAIM) {
         const u32* src = G.pool + (u64)e * JPAGE_WORDS + ((rel >> 2) & (JPAGE_WORDS - 1));
         if (NW == 1) v.x = __ldcg(src);
@@ -529,7 +534,7 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
             const u32 lw = (mod & 3) > 2 ? 2 : (mod & 3), nw = 1u << lw, w = 4u << lw;
             const u64 va = F.rd64(ia) + (u64)(i64)(i32)imm;
             bool zero = false;
-            const u32 c = ex ? jcheck(A, bc, va, w, k, &zero, MODE == JM_PAGE ? pg->page_base : nullptr) : 0u;
+            const u32 c = ex ? jcheck<0>(A, bc, va, w, k, &zero, MODE == JM_PAGE ? pg->page_base : nullptr) : 0u;
             if (__ballot_sync(JFULL, c != 0u)) {      // memory fault: DUE (C-9); the step has no effect
                 S.fault = __ballot_sync(JFULL, c == 1u) ? 1u : 2u;
                 S.fault_pc = pcm;
@@ -546,9 +551,9 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
                         else v = jld128(src);
                     }
                     if (MODE == JM_PAGE) {            // the replica's pages win
-                        if (nw == 1) jpage_c<1>(A, bc, *pg, va, v);
-                        else if (nw == 2) jpage_c<2>(A, bc, *pg, va, v);
-                        else jpage_c<4>(A, bc, *pg, va, v);
+                        if (nw == 1) jpage_c<1, 0>(A, bc, *pg, va, v);
+                        else if (nw == 2) jpage_c<2, 0>(A, bc, *pg, va, v);
+                        else jpage_c<4, 0>(A, bc, *pg, va, v);
                     }
                     F.wr(id, v.x);
                     if (lw >= 1) F.wr(id + 128, v.y);
