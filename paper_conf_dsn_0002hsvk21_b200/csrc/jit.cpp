@@ -28,6 +28,8 @@
 #include <cstdlib>
 #include <cstring>
 #include <atomic>
+#include <bitset>
+#include <cctype>
 #include <mutex>
 #include <thread>
 #include <string>
@@ -51,11 +53,18 @@ struct Src {
     std::string s;
     void operator()(const char* fmt, ...) __attribute__((format(printf, 2, 3))) {
         char buf[4096];
-        va_list ap;
+        va_list ap, ap2;
         va_start(ap, fmt);
+        va_copy(ap2, ap);
         int n = std::vsnprintf(buf, sizeof buf, fmt, ap);
         va_end(ap);
-        if (n > 0) s.append(buf, std::min<size_t>((size_t)n, sizeof buf - 1));
+        if (n > 0 && (size_t)n < sizeof buf) s.append(buf, (size_t)n);
+        else if (n > 0) {                              // long lines (register kill lists)
+            std::string big((size_t)n + 1, '\0');
+            std::vsnprintf(&big[0], big.size(), fmt, ap2);
+            s.append(big.data(), (size_t)n);
+        }
+        va_end(ap2);
     }
 };
 
@@ -537,6 +546,69 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
         if (code[i].op == BRA && code[i].imm < n) leader[code[i].imm] = 1;
         if ((code[i].op == BRA || code[i].op == EXIT) && i + 1 < n) leader[i + 1] = 1;
     }
+    // ---- per-thread register liveness (every mode but the trace pass, whose checkpoints
+    // copy the whole register file).  The dispatch loop reaches step mode, which spills
+    // every register, from every block exit, and a lane-predicated write `if (ex) R = v`
+    // keeps the old value of the lanes that do not execute: to the compiler every
+    // synthetic register is live everywhere.  `kills(keep)` zeroes, on the entries and
+    // exits of the block code, the registers no lane can read again there: the active
+    // lanes go to the path's targets, the parked ones wait at pcs >= npc >= the block's
+    // end (the `fits` rule), so keep = live_in(targets) | live_from[end].  The values
+    // are unobservable (outcomes come from stores; the site's before/after from the
+    // instruction that writes them); SHFL sources are never zeroed (SHFL reads parked
+    // and exited lanes).  Reads are over-approximated (operand fields and every register
+    // the instruction's own code mentions); only an unguarded `if (ex) R = v` kills.
+    typedef std::bitset<256> RSet;
+    std::vector<RSet> lin(n + 1), lfrom(n + 2);     // live-in per pc; lfrom[e] = union of lin[q], q >= e
+    RSet shfl;
+    const bool use_kill = mode != 2 && !std::getenv("FI_JIT_NO_KILL");
+    if (use_kill) {
+        std::vector<RSet> rd(n), kl(n);
+        for (uint32_t i = 0; i < n; ++i) {
+            const fi_insn& I = code[i];
+            auto add = [&](uint32_t j) { if (j < NR && j < 256) rd[i].set(j); };
+            if (I.op != NOP && I.op != EXIT && I.op != BRA && I.op != S2R && I.op != LDC) {
+                add(I.a); add(I.a + 1u); add(I.c); add(I.c + 1u);
+                if (!(I.mod & 0x80)) for (uint32_t q = 0; q < 4; ++q) add(I.b + q);
+            }
+            if (I.op == BRA || I.op == EXIT) continue;
+            Src t;
+            if (I.op == LDG || I.op == STG) G.mem(t, I, i, "step");
+            else { t("{ const bool ex = true; "); G.plain(t, I); t("}"); }
+            const std::string& s = t.s;
+            const bool uncond = G.guard(I.guard) == "true";
+            for (size_t p = 0; p < s.size(); ++p) {
+                if (s[p] != 'R' || (p > 0 && (std::isalnum((unsigned char)s[p - 1]) || s[p - 1] == '_'))) continue;
+                size_t q = p + 1;
+                if (q >= s.size() || !std::isdigit((unsigned char)s[q])) continue;
+                uint32_t v = 0;
+                while (q < s.size() && std::isdigit((unsigned char)s[q])) v = v * 10 + (uint32_t)(s[q++] - '0');
+                if (q < s.size() && (std::isalnum((unsigned char)s[q]) || s[q] == '_')) continue;
+                const bool w = s.compare(q, 3, " = ") == 0 && (q + 3 >= s.size() || s[q + 3] != '=');
+                if (!w) add(v);
+                else if (uncond && p >= 8 && s.compare(p - 8, 8, "if (ex) ") == 0 && v < 256) kl[i].set(v);
+            }
+            if (I.op == SHFL) shfl |= rd[i];
+        }
+        for (bool ch = true; ch;) {
+            ch = false;
+            for (int64_t i = (int64_t)n - 1; i >= 0; --i) {
+                RSet out = lin[i + 1];
+                if (code[i].op == BRA && code[i].imm < n) out |= lin[code[i].imm];
+                const RSet in = rd[i] | (out & ~kl[i]);
+                if (in != lin[i]) { lin[i] = in; ch = true; }
+            }
+        }
+        for (int64_t e = (int64_t)n; e >= 0; --e) lfrom[e] = lin[e] | lfrom[e + 1];
+    }
+    auto kills = [&](const RSet& keep) -> std::string {
+        std::string s;
+        if (!use_kill) return s;
+        for (uint32_t j = 0; j < NR && j < 256; ++j)
+            if (!keep[j] && !shfl[j]) s += "R" + std::to_string(j) + " = 0u; ";
+        return s;
+    };
+    auto entry_kills = [&](uint32_t L) { return kills(lin[L] | lfrom[std::min(n, L + blen[L])]); };
     // per pc: the block length if pc is a leader, else 0 (step mode's exit test)
     if (with_tables) {
         o("__device__ const unsigned short kblen_%u[%u] = {", kid, n);
@@ -617,7 +689,8 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
     o(" switch (pcm) {\n");
     for (uint32_t i = 0; i < n; ++i)
         if (leader[i])
-            o("  case %u: if (%uu <= npc && step + %uu <= lim) goto B%u; goto S_any;\n", i, i + blen[i], blen[i], i);
+            o("  case %u: if (%uu <= npc && step + %uu <= lim) { %sgoto B%u; } goto S_any;\n", i, i + blen[i], blen[i],
+              entry_kills(i).c_str(), i);
     o("  default: goto S_any;\n }\n");
     // ---- block code (fallthrough from a leader to the block's BRA / EXIT)
     char stepx[64];
@@ -635,8 +708,8 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
         if (i < batch_end) {
             if (i + 1 == n) {
                 flush_end();
-                o(" { step += %uu - pcm; upc = %uu; if (upc >= npc) { conv = false; if (inA) pc = upc; } continue; }\n",
-                  n, n);
+                o(" { %sstep += %uu - pcm; upc = %uu; if (upc >= npc) { conv = false; if (inA) pc = upc; } continue; }\n",
+                  kills(RSet()).c_str(), n, n);
             }
             continue;
         }
@@ -664,28 +737,30 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
             auto chain = [&](uint32_t L) -> std::string {
                 if (L >= n || !leader[L]) return "";
                 char b[256];
-                std::snprintf(b, sizeof b, "if (%uu <= npc && step + %uu <= lim) { pcm = %uu; goto B%u; } ", L + blen[L],
-                              blen[L], L, L);
-                return b;
+                std::snprintf(b, sizeof b, "if (%uu <= npc && step + %uu <= lim) { pcm = %uu; ", L + blen[L], blen[L], L);
+                return b + entry_kills(L) + "goto B" + std::to_string(L) + "; } ";
             };
             o(" { const bool pv = %s; ", G.guard(I.guard).c_str());
             G.rec(o, I, i, stepx, "pv");
             G.flush_recs(o, code, run_start(i), i);
+            const RSet keep_ft = use_kill ? lfrom[i + 1] : RSet();
+            const RSet keep_tk = use_kill ? (I.imm < n ? lin[I.imm] : RSet()) | lfrom[i + 1] : RSet();
             o("const u32 exm_ = amask & __ballot_sync(JFULL, pv); step += %uu - pcm;\n"
-              "   if (exm_ == 0u) { %supc = %uu; } else if (exm_ == amask) { %supc = %uu; }\n"
-              "   else { conv = false; if (inA) pc = ((exm_ >> lane) & 1u) ? %uu : %uu; }\n"
+              "   if (exm_ == 0u) { %s%supc = %uu; } else if (exm_ == amask) { %s%supc = %uu; }\n"
+              "   else { %sconv = false; if (inA) pc = ((exm_ >> lane) & 1u) ? %uu : %uu; }\n"
               "   if (conv && (amask == 0u || upc >= npc)) { conv = false; if ((amask >> lane) & 1u) pc = upc; }\n"
               "   continue; }\n",
-              i + 1, chain(i + 1).c_str(), i + 1, chain(I.imm).c_str(), I.imm, I.imm, i + 1);
+              i + 1, chain(i + 1).c_str(), kills(keep_ft).c_str(), i + 1, chain(I.imm).c_str(),
+              kills(keep_tk).c_str(), I.imm, kills(keep_tk).c_str(), I.imm, i + 1);
         } else if (I.op == EXIT) {
             o(" { const bool pv = %s; ", G.guard(I.guard).c_str());
             G.rec(o, I, i, stepx, "pv");
             G.flush_recs(o, code, run_start(i), i);
             o("const u32 exm_ = amask & __ballot_sync(JFULL, pv); step += %uu - pcm;\n"
-              "   if (inA && pv) live = false; livem &= ~exm_; amask &= ~exm_; upc = %uu;\n"
+              "   if (inA && pv) live = false; livem &= ~exm_; amask &= ~exm_; upc = %uu; %s\n"
               "   if (conv && (amask == 0u || upc >= npc)) { conv = false; if ((amask >> lane) & 1u) pc = upc; }\n"
               "   continue; }\n",
-              i + 1, i + 1);
+              i + 1, i + 1, kills(use_kill ? lfrom[i + 1] : RSet()).c_str());
         } else {
             if (I.op == LDG || I.op == STG) {
                 G.mem(o, I, i, stepx);
@@ -697,8 +772,8 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
             }
             if (i + 1 == n) {
                 flush_end();
-                o(" { step += %uu - pcm; upc = %uu; if (upc >= npc) { conv = false; if (inA) pc = upc; } continue; }\n",
-                  n, n);
+                o(" { %sstep += %uu - pcm; upc = %uu; if (upc >= npc) { conv = false; if (inA) pc = upc; } continue; }\n",
+                  kills(RSet()).c_str(), n, n);
             }
         }
     }
