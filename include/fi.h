@@ -466,9 +466,9 @@ typedef int (*fi_allreduce_fn)(void* dev, uint64_t count, uint32_t elem_bytes, v
 #define FI_PROPAGATION_AUTO 0u      /* K8 from 64 launches on, else K5/K7 (fi_classify) */
 #define FI_PROPAGATION_K7 1u        /* fi_classify */
 #define FI_PROPAGATION_K8 2u        /* fi_classify_batched */
-#define FI_CKPT_AUTO 0xFFFFFFFFu
+#define FI_CKPT_AUTO 0xFFFFFFFFu    /* 8192 steps, doubled until the checkpoints fit 20% of free HBM */
 #define FI_ENGINE_INTERP 0u
-#define FI_ENGINE_JIT 1u    /* 4096 steps, doubled until the checkpoints fit 20% of free HBM */
+#define FI_ENGINE_JIT 1u
 typedef struct {
     /* the program, HOST arrays */
     const fi_insn* code;         uint32_t n_code;

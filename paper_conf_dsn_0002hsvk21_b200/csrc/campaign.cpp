@@ -226,7 +226,7 @@ extern "C" fi_status fi_campaign(const fi_campaign_cfg* cfg, int rank, int world
     uint64_t* ckoff = nullptr;
     uint32_t interval = 0;
     if (cfg->ckpt_interval) {
-        interval = cfg->ckpt_interval == FI_CKPT_AUTO ? 4096u : cfg->ckpt_interval;
+        interval = cfg->ckpt_interval == FI_CKPT_AUTO ? 8192u : cfg->ckpt_interval;
         const size_t ck_bytes = fi_ckpt_bytes(p.n_regs);
         const size_t lws = fi_ckpt_layout_workspace(W);
         void* lw;

@@ -373,7 +373,8 @@ def golden_run(dp: DeviceProgram, ckpt_interval: int | str = "auto", ckpt_budget
     """fi_golden_lengths (pass 1) -> scans + checkpoint layout -> fi_golden_trace (pass 2).
 
     ckpt_interval: steps between golden register-file checkpoints (0 = none);
-    "auto" = 4096, doubled until the checkpoints fit ckpt_budget_frac of free HBM.
+    "auto" = 8192 (the trace pass runs in step mode around every
+    checkpoint, a replica restarts from the one at or before its site), doubled until the checkpoints fit ckpt_budget_frac of free HBM.
     engine: "interp" (emu.cuh) or "jit" (fi_golden_*_jit on the program's JIT
     module built with FI_JIT_GOLDEN): bit-identical results."""
     jit = dp.jit(FI_JIT_GOLDEN) if engine == "jit" else None
@@ -399,7 +400,7 @@ def golden_run(dp: DeviceProgram, ckpt_interval: int | str = "auto", ckpt_budget
     interval = 0
     ck_bytes = lib().fi_ckpt_bytes(dp.n_regs)
     if ckpt_interval and W:
-        interval = 4096 if ckpt_interval == "auto" else int(ckpt_interval)
+        interval = 8192 if ckpt_interval == "auto" else int(ckpt_interval)
         free = torch.cuda.mem_get_info(dp.device)[0]
         ws_n = lib().fi_ckpt_layout_workspace(W)
         ws = torch.empty(ws_n, dtype=torch.uint8, device=dp.device)
