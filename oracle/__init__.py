@@ -104,6 +104,7 @@ def lib():
             L.orc_inject.argtypes = [vp, vp, u32, i32, i32, vp]
             L.orc_inject_permanent.argtypes = [vp, vp, u32, i32, i32, vp]
             L.orc_permanent_image.argtypes = [vp, vp, u32, i32, vp]
+            L.orc_inject_image.argtypes = [vp, vp, i32, vp]
             L.orc_warp_site_rank.argtypes = [C.POINTER(_Program), u32, i32, u32, u32, C.POINTER(u64), C.POINTER(u64)]
             L.orc_inject_local.argtypes = [C.POINTER(_Program), vp, u32, i32, vp, vp]
             L.orc_warp_site_at.argtypes = [C.POINTER(_Program), u32, i32, u64, C.POINTER(u32), C.POINTER(u32),
@@ -230,6 +231,15 @@ class Golden:
         f = np.ascontiguousarray(np.asarray(fault, dtype=PFAULT_DTYPE).reshape(1))
         img = np.zeros_like(self.final_image())
         k = lib().orc_permanent_image(self.h, _ptr(f), rep, mode, _ptr(img))
+        return k, img
+
+    def inject_image(self, site, mode: int = MODE_FULL):
+        """(fault kind, faulty final image) of one transient site, full mode."""
+        s = np.ascontiguousarray(np.asarray(site, dtype=SITE_DTYPE).reshape(1))
+        img = np.zeros(self.prog.image_bytes, dtype=np.uint8)
+        k = lib().orc_inject_image(self.h, _ptr(s), mode, _ptr(img))
+        if k < 0:
+            raise OracleError(4, "injection site not reached as selected")
         return k, img
 
     def locate(self, group: int, s) -> np.ndarray:

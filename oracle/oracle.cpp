@@ -718,9 +718,11 @@ extern "C" uint32_t orc_dest_slots(const orc_insn* I, int g, uint8_t* kind, uint
 // lane-instruction of group g in canonical order (C-3): warps in trace order,
 // dynamic order within a warp, lanes ascending within a record.  `out[i]` must
 // already hold s, group, u_dst (and bfm/mask); this fills the location.
+static int enumerate_sites_by_warp(Golden* G, uint32_t n, orc_site* out);
+
 static int enumerate_sites(Golden* G, uint32_t n, orc_site* out) {
     const Prog& P = G->P;
-    if (!G->kept) { G->err = "selection needs keep_trace"; return 1; }
+    if (!G->kept) return enumerate_sites_by_warp(G, n, out);
     struct Want { uint64_t s; uint32_t idx; };
     std::vector<std::vector<Want>> per_g(8);
     for (uint32_t i = 0; i < n; ++i) per_g[out[i].group & 7].push_back({out[i].s, i});
@@ -768,6 +770,82 @@ static int enumerate_sites(Golden* G, uint32_t n, orc_site* out) {
         }
         if (q != v.size()) { G->err = "s beyond the group's site count"; return 4; }
     }
+    return 0;
+}
+
+// Selection without a kept trace (single-instance programs at full size, whose
+// App. A.3 trace does not fit in host RAM): the same canonical order (C-3).  The
+// warp holding site s is the first whose cumulative group-g count — warps in
+// trace order, per-warp counts of the golden run — exceeds s; the rank inside
+// it is found by re-interpreting that warp from the memory before the instance
+// (the initial image of a single-instance program) and walking its records
+// exactly as enumerate_sites walks the kept trace.
+static int enumerate_sites_by_warp(Golden* G, uint32_t n, orc_site* out) {
+    const Prog& P = G->P;
+    if (!P.single_instance()) { G->err = "selection without a kept trace needs a single-instance program"; return 1; }
+    std::vector<uint64_t> rank(n, 0);
+    std::map<uint32_t, std::vector<uint32_t>> by_warp;      // warp -> indices into out
+    for (int g = 0; g < 8; ++g) {
+        std::vector<std::pair<uint64_t, uint32_t>> v;
+        for (uint32_t i = 0; i < n; ++i) if ((out[i].group & 7) == g) v.push_back({out[i].s, i});
+        if (v.empty()) continue;
+        std::sort(v.begin(), v.end());
+        uint64_t cum = 0;
+        size_t q = 0;
+        for (uint32_t w = 0; w < P.n_warps && q < v.size(); ++w) {
+            uint64_t c = G->wcounts[8 * (size_t)w + g];
+            while (q < v.size() && v[q].first < cum + c) {
+                rank[v[q].second] = v[q].first - cum;
+                by_warp[w].push_back(v[q].second);
+                ++q;
+            }
+            cum += c;
+        }
+        if (q != v.size()) { G->err = "s beyond the group's site count"; return 4; }
+    }
+    std::vector<std::pair<uint32_t, std::vector<uint32_t>>> jobs(by_warp.begin(), by_warp.end());
+    const std::vector<uint8_t> pre(P.p.init_image, P.p.init_image + P.p.image_bytes);
+    const orc_instance& in = P.p.inst[0];
+    std::atomic<int> status{0};
+    parallel_for((uint32_t)jobs.size(), (int)std::max(1u, std::thread::hardware_concurrency()), [&](uint32_t jb) {
+        uint32_t w = jobs[jb].first, cta, wic;
+        warp_coords(in, w, cta, wic);
+        std::vector<orc_record> tr;
+        TraceSink ts;
+        ts.rec = &tr;
+        std::vector<StoreW> st;
+        run_warp(P, pre, 0, cta, wic, nullptr, UINT64_MAX, &st, &ts, nullptr);
+        for (uint32_t i : jobs[jb].second) {
+            orc_site& S = out[i];
+            const int g = S.group & 7;
+            uint64_t seen = 0;
+            bool found = false;
+            for (size_t r = 0; r < tr.size() && !found; ++r) {
+                if (!((tr[r].insn >> (24 + g)) & 1)) continue;
+                uint32_t ex = tr[r].active & tr[r].pred;
+                for (int l = 0; l < 32 && !found; ++l) {
+                    if (!((ex >> l) & 1)) continue;
+                    if (seen++ != rank[i]) continue;
+                    S.instance = 0; S.kernel_id = in.kernel; S.kernel_count = in.kernel_count;
+                    S.warp = w; S.step = (uint32_t)r; S.lane = (uint8_t)l;
+                    S.thread = cta * in.block + wic * 32 + (uint32_t)l;
+                    S.pc = tr[r].insn & 0xFFFF;
+                    S.instruction_count = S.s;
+                    const orc_insn& I = P.p.code[P.p.kern[in.kernel].code_off + S.pc];
+                    std::vector<std::pair<int, int>> sl;
+                    slots_for(I, g, sl);
+                    if (sl.empty()) { status = 4; return; }
+                    S.n_elig = (uint8_t)sl.size();
+                    S.slot = (uint8_t)(((uint64_t)sl.size() * S.u_dst) >> 32);   // floor(n x value), C-5
+                    S.dst_kind = (uint8_t)sl[S.slot].first;
+                    S.dst_reg = (uint8_t)sl[S.slot].second;
+                    found = true;
+                }
+            }
+            if (!found) status = 4;
+        }
+    });
+    if (status) { G->err = "warp re-run disagrees with the golden per-warp counts"; return 4; }
     return 0;
 }
 
@@ -1113,5 +1191,23 @@ extern "C" int orc_permanent_image(void* h, const orc_pfault* pf, uint32_t rep, 
     run_program(G, G->P, nullptr, 0, 1, fr, nullptr, nullptr, false, nullptr, nullptr, nullptr,
                 (mode & ORC_UNCHECKED) != 0, &ps);
     std::copy(fr.mem.begin(), fr.mem.end(), out_image);
+    return fr.fault ? fr.fault : fr.pdue;
+}
+
+// The faulty final image of one transient site by the definition (full mode:
+// the whole program re-run with the corruption, PAPER.md:72 step (4), :78,
+// :138) — for the multi-launch propagation pins.  Returns the fault kind
+// (0 = none), or -1 if the site was not reached as selected.
+extern "C" int orc_inject_image(void* h, const orc_site* site, int mode, uint8_t* out_image) {
+    Golden* G = (Golden*)h;
+    const orc_site& S = *site;
+    Hook hk;
+    hk.on = true; hk.step = S.step; hk.lane = S.lane; hk.kind = S.dst_kind; hk.reg = S.dst_reg;
+    hk.bfm = S.bfm; hk.mask = S.mask; hk.pc = S.pc;
+    FullRun fr;
+    run_program(G, G->P, &hk, S.warp, 1, fr, nullptr, nullptr, false, nullptr, nullptr, nullptr,
+                (mode & ORC_UNCHECKED) != 0);
+    std::copy(fr.mem.begin(), fr.mem.end(), out_image);
+    if (!hk.fired || hk.bad) return -1;
     return fr.fault ? fr.fault : fr.pdue;
 }

@@ -84,7 +84,9 @@ uint64_t orc_n_golden_stores(void* h);
  * baselines.  Returns records interpreted. */
 uint64_t orc_count_warps(const orc_program* p, uint32_t w0, uint32_t w1, int n_threads, uint64_t* counts8);
 
-/* selection by enumeration (C-3..C-6) */
+/* selection by enumeration (C-3..C-6).  With keep_trace=0 (single-
+ * instance programs only) the site's warp comes from the per-warp counts and the
+ * rank inside it from a re-interpretation of that warp — the same canonical order. */
 int orc_select(void* h, uint64_t seed, const uint8_t* groups, uint32_t n_groups,
                const uint8_t* bfms, uint32_t n_bfms, uint64_t j0, uint32_t n, orc_site* out);
 
@@ -103,6 +105,10 @@ int orc_inject(void* h, const orc_site* sites, uint32_t n, int mode, int n_threa
 typedef struct { uint32_t opcode, sm, lane, mask, q32, n_sm; uint64_t seed; } orc_pfault;   /* 32 B */
 int orc_inject_permanent(void* h, const orc_pfault* pf, uint32_t n, int mode, int n_threads, orc_inj* out);
 int orc_permanent_image(void* h, const orc_pfault* pf, uint32_t rep, int mode, uint8_t* out_image);
+
+/* faulty final image of one transient site, full mode (multi-launch propagation pins);
+ * returns the fault kind, -1 if the site was not reached */
+int orc_inject_image(void* h, const orc_site* site, int mode, uint8_t* out_image);
 
 /* single-instance, no golden handle (full-size sampled parity, CPU baselines) */
 int orc_warp_site_rank(const orc_program* p, uint32_t w, int g, uint32_t step, uint32_t lane,

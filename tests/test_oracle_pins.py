@@ -169,23 +169,6 @@ def test_predicated_off_lanes_not_counted():
     assert g.n_records == 576
 
 
-def _unused_sgemm_closed_form(M, N, K):
-    """Per-thread counts of the C2 kernel (fi_inputs.programs.sgemm_code), by
-    hand from the listing: prologue 17 insns, 73 per k-iteration (4 LDG.128,
-    64 FFMA, 2 IMAD.WIDE + IADD3, ISETP, BRA — the last BRA predicated off),
-    epilogue 29 insns (LDC.64, LDC, IMAD, IMAD.WIDE, 8 x (2 STG.128 + IMAD.WIDE), EXIT)."""
-    per = [0] * 8
-    per[LD] = 5 + 4 * K + 2
-    per[FP32] = 64 * K
-    per[OTHERS] = 12 + 3 * K + 2 + 8
-    per[PR] = K
-    per[NODEST] = (K - 1) + 16 + 1
-    per[GP] = per[FP32] + per[LD] + per[OTHERS]
-    per[GPPR] = per[GP] + per[PR]
-    threads = M * N // 64
-    return [x * threads for x in per], (M * N // 64 // 32) * (17 + 73 * K + 29)
-
-
 def test_mini_c2_closed_form_and_numerics():
     prog = P.c2(full=False)
     g = O.Golden(prog, keep_trace=False)
