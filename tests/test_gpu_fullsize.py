@@ -1,13 +1,20 @@
 """Parity at BASELINE.json's full size (C2: SGEMM 4096^3, 10,000 replicas) in
 the launch configuration bench.py times (campaign.Campaign.step).
 
-The oracle cannot re-run all 8,192 warps in a test, so it checks:
+Checks:
   * counts and record totals against the hand-derived closed form;
   * every one of the 10,000 draws (s, u_dst, u_bit) against its own Philox+Lemire;
   * every site's warp against the closed-form per-warp count, and its mask;
-  * a stratified sample of replicas fully: the oracle selects the site itself
-    (draw -> warp -> enumeration inside the warp) and injects it warp-locally;
-    site fields, before/after/mask, fault kind and outcome must be identical.
+  * ALL 10,000 replicas against the oracle: its own golden run of the whole
+    C2 program (orc_golden_run without a kept trace: per-warp counts and the
+    golden final image, PAPER.md:72 step (1)), its own selection (the warp from
+    the per-warp counts, the rank inside it by re-interpreting that warp, C-3)
+    and warp-local injection classified against that golden image
+    (C-14) — every site field, before/after/mask, fault kind/pc
+    and outcome identical, no replica left undecided;
+  * the GPU golden final image equals the oracle's byte for byte;
+  * a stratified sample again through build_site / inject_local (the checker
+    without a golden handle, pinned in tests/test_oracle_pins_local.py).
 """
 import numpy as np
 import pytest
@@ -26,6 +33,38 @@ def camp():
     c.step()
     c.check()
     return c
+
+
+@pytest.fixture(scope="module")
+def oracle_c2(camp):
+    return O.Golden(camp.prog, keep_trace=False)
+
+
+def test_c2_oracle_golden_run(camp, oracle_c2):
+    want, nrec = sgemm_closed_form(4096, 4096, 4096)
+    assert oracle_c2.counts()[0].tolist() == want and oracle_c2.n_records == nrec
+    assert np.array_equal(camp.gt.image.cpu().numpy(), oracle_c2.final_image())
+    assert np.array_equal(camp.gt.warp_len.cpu().numpy().astype(np.uint64), oracle_c2.warp_len())
+
+
+def test_c2_all_10000_replicas_vs_oracle(camp, oracle_c2):
+    """Every replica of the headline campaign, element by element (no sample,
+    no undecided escape): sites, injected values, faults and outcomes."""
+    sites = camp.sites_np()
+    inj = camp.inj_np()
+    osites = oracle_c2.select(P.CAMPAIGN_SEED[2], [GP], [0, 1, 2, 3], 0, 10000)
+    for n in osites.dtype.names:
+        assert (osites[n] == sites[n]).all(), n
+    oi = oracle_c2.inject(osites, O.MODE_WARP_LOCAL)
+    for f in ("before", "after", "mask", "fault_kind", "outcome", "flags"):
+        bad = np.flatnonzero(oi[f] != inj[f])
+        assert bad.size == 0, (f, bad[:10].tolist())
+    fk = oi["fault_kind"] > 0
+    assert (oi["fault_pc"][fk] == inj["fault_pc"][fk]).all()
+    assert (inj["overflow"] == 0).all()
+    h = camp.hist.cpu().numpy()
+    assert (h == O.histogram(osites, oi).astype(np.int64)).all()
+    assert set(np.unique(oi["outcome"]).tolist()) == {0, 1, 2}
 
 
 def test_c2_counts_closed_form(camp):
