@@ -59,6 +59,37 @@ def c1() -> Program:
     return vector_add()
 
 
+def vector_add_f64(n: int = 512, grid: int = 2, block: int = 256, seed: int = DATA_SEED[1] + 64) -> Program:
+    """c = a + b in FP64 (LDG.64, DADD, STG.64): an f64 output buffer for the
+    C-12 secondary numeric classification (an element is a register pair)."""
+    s = Asm()
+    s.s2r(0, isa.SR_TID)                      # 0
+    s.s2r(1, isa.SR_CTAID)                    # 1
+    s.s2r(2, isa.SR_NTID)                     # 2
+    s.imad(0, 1, 2, 0)                        # 3  gid
+    s.ldc(3, 24)                              # 4  n
+    s.isetp(0, 0, 3, cmp=isa.GE)              # 5
+    s.exit(guard=0)                           # 6
+    s.ldc(4, 0, wide=True)                    # 7  a
+    s.imad_wide(4, 0, imm=8, c=4)             # 8
+    s.ldc(6, 8, wide=True)                    # 9  b
+    s.imad_wide(6, 0, imm=8, c=6)             # 10
+    s.ldg(8, 4, width=isa.W64)                # 11 R8:R9
+    s.ldg(10, 6, width=isa.W64)               # 12 R10:R11
+    s.ldc(12, 16, wide=True)                  # 13 c
+    s.imad_wide(12, 0, imm=8, c=12)           # 14
+    s.dadd(8, 8, 10)                          # 15 R8:R9
+    s.stg(12, 8, width=isa.W64)               # 16
+    s.exit()                                  # 17
+    pb = ProgramBuilder(f"vecadd_f64_n{n}")
+    k = pb.add_kernel("vecadd_f64", s.assemble(), nregs=14)
+    a = pb.add_buffer("a", 8 * n, f64_data(seed, n), dtype=isa.DT_F64)
+    b = pb.add_buffer("b", 8 * n, f64_data(seed + 1, n), dtype=isa.DT_F64)
+    c = pb.add_buffer("c", 8 * n, writer=0, output=True, dtype=isa.DT_F64)
+    pb.add_instance(k, grid, block, ptr_words(a) + ptr_words(b) + ptr_words(c) + [n])
+    return pb.build(config="vecadd_f64", n=n, grid=grid, block=block)
+
+
 # ---------------------------------------------------------------------------
 # C2: SGEMM, 128x128 CTA tile, 8x8 per thread (App. A.5, SURVEY §8(d))
 # ---------------------------------------------------------------------------

@@ -303,10 +303,22 @@ fi_status fi_inject(const fi_program* p, const uint8_t* image, const fi_trace* t
  * buffer whose pages were dropped after its last launch reference (wild load) */
 #define FI_UNCLASSIFIED_CAPACITY 2u
 #define FI_UNCLASSIFIED_WILD 4u
+/* C-12 secondary numeric classification ("rtol = 1e-6, atol = 0,
+ * NaN != number", reported beside the graded bitwise one; the paper leaves the
+ * SDC check to the user, "Output file is different" [PAPER.md:189], "both
+ * application and user dependent" [PAPER.md:204]).  With rtol > 0 the classify
+ * calls also set FI_SDC_WITHIN_TOL in fi_inj.flags of every bitwise SDC whose
+ * differing output ELEMENTS (buffer dtype, fi_buffer.flags bits 8..15: 0 u32,
+ * 1 f32, 2 f64) all satisfy: both finite and |f - g| <= rtol * |g| (IEEE double,
+ * round to nearest; u32 elements never do), and, when hist_tol is not NULL,
+ * accumulate hist_tol[8][4][3] with those replicas counted as Masked.  The
+ * graded outcome and hist are unchanged.  rtol = 0 (hist_tol ignored): bitwise only. */
+#define FI_SDC_WITHIN_TOL 8u
 size_t fi_classify_workspace(uint32_t n_inst, uint32_t n, uint32_t log_cap);
 fi_status fi_classify(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
                       uint32_t n, fi_inj* out, const fi_store* log, uint32_t log_cap, uint64_t* hist,
-                      uint32_t flags, void* ws, size_t ws_bytes, uint32_t* dev_status, void* stream);
+                      uint32_t flags, double rtol, uint64_t* hist_tol, void* ws, size_t ws_bytes,
+                      uint32_t* dev_status, void* stream);
 
 /* K8 — fi_classify for long multi-instance programs (thousands of launches,
  * SURVEY C3/C4/C5): same definition and result as fi_classify's K7 (C-12, C-14,
@@ -325,8 +337,8 @@ size_t fi_classify_batched_workspace(const fi_program* p, uint32_t n, uint32_t l
                                      uint32_t pool_pages, uint32_t pend_cap);
 fi_status fi_classify_batched(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
                               uint32_t n, fi_inj* out, const fi_store* log, uint32_t log_cap, uint64_t* hist,
-                              uint32_t flags, uint32_t batch, uint32_t pool_pages, uint32_t pend_cap, void* ws,
-                              size_t ws_bytes, uint32_t* dev_status, void* stream);
+                              uint32_t flags, double rtol, uint64_t* hist_tol, uint32_t batch, uint32_t pool_pages,
+                              uint32_t pend_cap, void* ws, size_t ws_bytes, uint32_t* dev_status, void* stream);
 
 /* §8 rows f2/f3 — permanent faults (Table III
  * [PAPER.md:128-134]) and intermittent faults.  A fault is
@@ -414,8 +426,35 @@ fi_status fi_golden_trace_jit(const fi_jit* j, const fi_program* p, const uint8_
  * FI_JIT_PAGE: same arguments, scratch and results (transient faults). */
 fi_status fi_classify_batched_jit(const fi_jit* j, const fi_program* p, const uint8_t* image, const fi_trace* t,
                                   const fi_site* sites, uint32_t n, fi_inj* out, const fi_store* log, uint32_t log_cap,
-                                  uint64_t* hist, uint32_t flags, uint32_t batch, uint32_t pool_pages,
-                                  uint32_t pend_cap, void* ws, size_t ws_bytes, uint32_t* dev_status, void* stream);
+                                  uint64_t* hist, uint32_t flags, double rtol, uint64_t* hist_tol, uint32_t batch,
+                                  uint32_t pool_pages, uint32_t pend_cap, void* ws, size_t ws_bytes,
+                                  uint32_t* dev_status, void* stream);
+
+/* fi_golden_run — the golden run as ONE call: Fig. 1 step (1) (the
+ * run whose dynamic instructions the profiler counts) and the golden
+ * output state step (4) compares against.  Runs pass 1
+ * (per-warp lengths and stored-word counts, golden final image), the scans, the
+ * checkpoint layout and pass 2 (App. A.3 trace records, golden store log,
+ * register-file checkpoints) on `jit` (a module built with FI_JIT_GOLDEN) or, with
+ * jit = NULL, on the shared-memory interpreter — bit-identical results.
+ *   image         device, caller's: in = the initial image, out = golden final image
+ *   ckpt_interval 0 = no checkpoints, FI_CKPT_AUTO = 8192 steps doubled while the
+ *                 checkpoints exceed ckpt_budget_frac (<= 0: 0.2) of free HBM
+ *   *out          the trace: fi_golden_trace_of(*out) is the fi_trace every later
+ *                 call reads (fi_profile, fi_select_sites, fi_inject*, fi_classify*)
+ * Memory: UNLIKE the calls above, the trace arrays (records, store log,
+ * checkpoints, offsets) are sized by pass 1 and allocated by this call,
+ * stream-ordered from the current device's default memory pool; *out owns them
+ * until fi_golden_free(*out, stream).  SYNCHRONIZES (the record totals size the
+ * allocations).  Errors: FI_E_ARG, FI_E_PROGRAM (the golden run faulted: the
+ * program violates DESIGN.md §3.5), FI_E_CUDA; nothing is allocated on error. */
+typedef struct fi_golden fi_golden;
+fi_status fi_golden_run(const fi_program* p, const fi_jit* jit, uint8_t* image, uint32_t ckpt_interval,
+                        double ckpt_budget_frac, fi_golden** out, void* stream);
+const fi_trace* fi_golden_trace_of(const fi_golden* g);          /* host struct of device pointers */
+const uint64_t* fi_golden_warp_len(const fi_golden* g);          /* device [n_warps] golden steps per warp */
+const uint64_t* fi_golden_gstore_off_host(const fi_golden* g);   /* HOST [n_warps+1] copy of gstore_off */
+fi_status fi_golden_free(fi_golden* g, void* stream);            /* stream-ordered release; NULL g is a no-op */
 
 /* Table II parameter file, one parameter per line in Table II order
  * [PAPER.md:88]: arch state id, bit-flip model, kernel name, kernel count,
@@ -490,6 +529,7 @@ typedef struct {
     uint64_t k8_mem_budget;      /* device bytes for K8 scratch (0 = 24 GiB) */
     int device;                  /* CUDA device ordinal (< 0 = current) */
     void* stream;                /* cudaStream_t (NULL = a stream fi_campaign creates) */
+    double rtol;                 /* > 0: also the C-12 secondary numeric classification (hist_tol) */
 } fi_campaign_cfg;
 
 typedef struct {
@@ -509,6 +549,7 @@ typedef struct {
     fi_site* sites;              /* [n_local] */
     fi_inj* inj;                 /* [n_local] */
     uint64_t* inst_counts;       /* [n_inst][8] (after the exchange) */
+    uint64_t hist_tol[8][4][3];  /* cfg->rtol > 0: secondary histogram (FI_SDC_WITHIN_TOL counted Masked), all ranks */
 } fi_campaign_result;
 
 fi_status fi_campaign(const fi_campaign_cfg* cfg, int rank, int world, fi_allreduce_fn allreduce, void* ctx,

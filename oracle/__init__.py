@@ -33,6 +33,7 @@ MASKED, SDC, DUE, NOT_INJECTED = 0, 1, 2, 3
 MODE_FULL, MODE_WARP_LOCAL = 0, 1
 UNCHECKED = 0x100          # OR into mode: potential-DUE semantics (row f4)
 POTENTIAL_DUE = 1          # inj["flags"] bit
+SDC_WITHIN_TOL = 8         # inj["flags"] bit: C-12 secondary numeric mode
 
 RECORD_DTYPE = np.dtype([("instance", "<u4"), ("insn", "<u4"), ("active", "<u4"), ("pred", "<u4")])
 SITE_DTYPE = np.dtype([
@@ -101,7 +102,7 @@ def lib():
             L.orc_opcode_counts.argtypes = [vp, vp]
             L.orc_approx_counts.argtypes = [vp, vp]
             L.orc_select_approx.argtypes = [vp, u64, vp, u32, vp, u32, u64, u32, vp]
-            L.orc_inject.argtypes = [vp, vp, u32, i32, i32, vp]
+            L.orc_inject.argtypes = [vp, vp, u32, i32, i32, C.c_double, vp]
             L.orc_inject_permanent.argtypes = [vp, vp, u32, i32, i32, vp]
             L.orc_permanent_image.argtypes = [vp, vp, u32, i32, vp]
             L.orc_inject_image.argtypes = [vp, vp, i32, vp]
@@ -250,10 +251,14 @@ class Golden:
             raise OracleError(rc, lib().orc_error(self.h).decode())
         return out
 
-    def inject(self, sites: np.ndarray, mode: int = MODE_FULL, n_threads: int | None = None) -> np.ndarray:
+    def inject(self, sites: np.ndarray, mode: int = MODE_FULL, n_threads: int | None = None,
+               rtol: float = 0.0) -> np.ndarray:
+        """Injection + classification (PAPER.md:78, :206).  rtol > 0: C-12's
+        secondary numeric mode sets SDC_WITHIN_TOL in flags."""
         sites = np.ascontiguousarray(sites, dtype=SITE_DTYPE)
         out = np.zeros(len(sites), dtype=INJ_DTYPE)
-        rc = lib().orc_inject(self.h, _ptr(sites), len(sites), mode, n_threads or n_threads_default(), _ptr(out))
+        rc = lib().orc_inject(self.h, _ptr(sites), len(sites), mode, n_threads or n_threads_default(), float(rtol),
+                              _ptr(out))
         if rc:
             raise OracleError(rc, lib().orc_error(self.h).decode())
         return out
@@ -372,10 +377,14 @@ def ci_margin(n: int, confidence: float, p_hat: float | None = None) -> float:
     return _Z[confidence] * math.sqrt(p * (1 - p) / n)
 
 
-def histogram(sites: np.ndarray, inj: np.ndarray) -> np.ndarray:
-    """Outcome histogram [group][bfm][M,S,D] (u64), by plain counting."""
+def histogram(sites: np.ndarray, inj: np.ndarray, tol: bool = False) -> np.ndarray:
+    """Outcome histogram [group][bfm][M,S,D] (u64), by plain counting.  tol=True:
+    the C-12 secondary histogram (an SDC flagged SDC_WITHIN_TOL counts as Masked)."""
     h = np.zeros((8, 4, 3), dtype=np.uint64)
     for s, r in zip(sites, inj):
-        if int(r["outcome"]) < 3:                  # not-injected sites are not outcomes
-            h[int(s["group"]), int(s["bfm"]), int(r["outcome"])] += 1
+        o = int(r["outcome"])
+        if tol and o == SDC and int(r["flags"]) & SDC_WITHIN_TOL:
+            o = MASKED
+        if o < 3:                                  # not-injected sites are not outcomes
+            h[int(s["group"]), int(s["bfm"]), o] += 1
     return h

@@ -612,6 +612,50 @@ bool output_differs(const Prog& P, const std::vector<uint8_t>& a, const std::vec
     return false;
 }
 
+// C-12 secondary numeric classification (BASELINE.md §2 "rtol = 1e-6, atol = 0,
+// NaN != number"): a faulty element f differs from the golden element g beyond
+// rtol unless the bits are equal, or the buffer is a float buffer and both are
+// finite with |f - g| <= rtol * |g| (IEEE double, round to nearest: this file is
+// compiled with -ffp-contract=off).  u32 buffers: any difference.
+enum { DT_U32 = 0, DT_F32 = 1, DT_F64 = 2 };
+uint32_t buf_dtype_of(const orc_buffer& b) { return (b.flags >> 8) & 0xFF; }
+bool elem_beyond_tol(uint32_t dtype, uint64_t fbits, uint64_t gbits, double rtol) {
+    if (fbits == gbits) return false;
+    double f, g;
+    if (dtype == DT_F32) { f = (double)f32((uint32_t)fbits); g = (double)f32((uint32_t)gbits); }
+    else if (dtype == DT_F64) { f = f64(fbits); g = f64(gbits); }
+    else return true;
+    if (!std::isfinite(f) || !std::isfinite(g)) return true;
+    return !(std::fabs(f - g) <= rtol * std::fabs(g));
+}
+
+// Element by element over every output buffer: does the faulty image differ from
+// the golden one beyond rtol somewhere?
+bool output_beyond_tol(const Prog& P, const std::vector<uint8_t>& a, const std::vector<uint8_t>& b, double rtol) {
+    for (uint32_t i = 0; i < P.p.n_buf; ++i) {
+        const orc_buffer& bf = P.p.buf[i];
+        if (!(bf.flags & 1)) continue;
+        const uint32_t dt = buf_dtype_of(bf);
+        const uint64_t w = dt == DT_F64 ? 8 : 4;
+        for (uint64_t o = 0; o + w <= bf.size; o += w) {
+            uint64_t x = 0, y = 0;
+            memcpy(&x, &a[bf.off + o], w);
+            memcpy(&y, &b[bf.off + o], w);
+            if (elem_beyond_tol(dt, x, y, rtol)) return true;
+        }
+    }
+    return false;
+}
+
+const orc_buffer* buffer_of(const Prog& P, uint64_t va) {
+    uint64_t off = va - VA_BASE;
+    for (uint32_t i = 0; i < P.p.n_buf; ++i) {
+        const orc_buffer& b = P.p.buf[i];
+        if (off >= b.off && off < b.off + b.size) return &b;
+    }
+    return nullptr;
+}
+
 bool is_output_addr(const Prog& P, uint64_t va) {
     uint64_t off = va - VA_BASE;
     for (uint32_t i = 0; i < P.p.n_buf; ++i) {
@@ -985,7 +1029,8 @@ extern "C" int orc_locate(void* h, int group, const uint64_t* s, uint32_t n, orc
 // WARP_LOCAL (single-instance programs): re-run only warp w, faulty and golden,
 // and compare the final value of every address either run stored to (C-14).
 // ORC_UNCHECKED in `mode` selects the potential-DUE semantics of row f4.
-extern "C" int orc_inject(void* h, const orc_site* sites, uint32_t n, int mode, int n_threads, orc_inj* out) {
+extern "C" int orc_inject(void* h, const orc_site* sites, uint32_t n, int mode, int n_threads, double rtol,
+                          orc_inj* out) {
     Golden* G = (Golden*)h;
     const Prog& P = G->P;
     const bool unchecked = mode & ORC_UNCHECKED;
@@ -1001,7 +1046,7 @@ extern "C" int orc_inject(void* h, const orc_site* sites, uint32_t n, int mode, 
         Hook hk;
         hk.on = true; hk.step = S.step; hk.lane = S.lane; hk.kind = S.dst_kind; hk.reg = S.dst_reg;
         hk.bfm = S.bfm; hk.mask = S.mask; hk.pc = S.pc;
-        int fault = 0, pdue = 0; uint32_t fpc = 0; bool sdc = false;
+        int fault = 0, pdue = 0; uint32_t fpc = 0; bool sdc = false, beyond = false;
         if (mode == ORC_MODE_FULL) {
             FullRun fr;
             run_program(G, P, &hk, S.warp, 1, fr, nullptr, nullptr, false, nullptr, nullptr, nullptr, unchecked);
@@ -1009,6 +1054,7 @@ extern "C" int orc_inject(void* h, const orc_site* sites, uint32_t n, int mode, 
             if (!fault && fr.pdue) { pdue = fr.pdue; fpc = fr.pdue_pc; }
             R.n_faulty_stores = (uint32_t)fr.n_faulty_stores;
             if (!fault) sdc = output_differs(P, fr.mem, G->final_mem);
+            if (sdc && rtol > 0) beyond = output_beyond_tol(P, fr.mem, G->final_mem, rtol);
         } else {
             const orc_instance& in = P.p.inst[S.instance];
             uint32_t cta, wic;
@@ -1029,6 +1075,26 @@ extern "C" int orc_inject(void* h, const orc_site* sites, uint32_t n, int mode, 
                     uint32_t g; memcpy(&g, &G->final_mem[kv.first - VA_BASE], 4);
                     if (g != kv.second && is_output_addr(P, kv.first)) { sdc = true; break; }
                 }
+                // rtol: each differing output element, its other words taken from
+                // the faulty final state (fin) or, if untouched, the golden image
+                if (sdc && rtol > 0) {
+                    for (auto& kv : fin) {
+                        const orc_buffer* b = buffer_of(P, kv.first);
+                        if (!b || !(b->flags & 1)) continue;
+                        const uint32_t dt = buf_dtype_of(*b);
+                        const uint64_t w = dt == DT_F64 ? 8 : 4, e = kv.first - (kv.first - VA_BASE - b->off) % w;
+                        uint64_t fe = 0, ge = 0;
+                        for (uint64_t q = 0; q < w; q += 4) {
+                            uint32_t gw, fw;
+                            memcpy(&gw, &G->final_mem[e + q - VA_BASE], 4);
+                            auto it = fin.find(e + q);
+                            fw = it != fin.end() ? it->second : gw;
+                            fe |= (uint64_t)fw << (8 * q);
+                            ge |= (uint64_t)gw << (8 * q);
+                        }
+                        if (elem_beyond_tol(dt, fe, ge, rtol)) { beyond = true; break; }
+                    }
+                }
             }
         }
         if (!hk.fired || hk.bad) {
@@ -1038,7 +1104,7 @@ extern "C" int orc_inject(void* h, const orc_site* sites, uint32_t n, int mode, 
         }
         R.before = hk.before; R.after = hk.after; R.mask = hk.applied_mask;
         R.fault_kind = (uint8_t)(fault ? fault : pdue); R.fault_pc = fpc;
-        R.flags = pdue ? ORC_POTENTIAL_DUE : 0;
+        R.flags = (uint8_t)((pdue ? ORC_POTENTIAL_DUE : 0) | (!fault && sdc && rtol > 0 && !beyond ? ORC_SDC_WITHIN_TOL : 0));
         R.outcome = fault ? ORC_DUE : (sdc ? ORC_SDC : ORC_MASKED);
     });
     return status;

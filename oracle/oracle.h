@@ -60,7 +60,7 @@ typedef struct {
 enum { ORC_G_FP64 = 0, ORC_G_FP32, ORC_G_LD, ORC_G_PR, ORC_G_NODEST, ORC_G_OTHERS, ORC_G_GPPR, ORC_G_GP };
 enum { ORC_MASKED = 0, ORC_SDC = 1, ORC_DUE = 2, ORC_NOT_INJECTED = 3 };
 enum { ORC_MODE_FULL = 0, ORC_MODE_WARP_LOCAL = 1, ORC_UNCHECKED = 0x100 /* f4 potential-DUE semantics */ };
-enum { ORC_POTENTIAL_DUE = 1 };
+enum { ORC_POTENTIAL_DUE = 1, ORC_SDC_WITHIN_TOL = 8 /* C-12 secondary: bitwise SDC, every element within rtol */ };
 
 /* status: 0 ok; 1 arg; 2 empty group; 3 not injectable; 4 program error */
 const char* orc_error(void* h);
@@ -98,8 +98,11 @@ int orc_approx_counts(void* h, uint64_t* out /*[n_inst][8]*/);
 int orc_select_approx(void* h, uint64_t seed, const uint8_t* groups, uint32_t n_groups,
                       const uint8_t* bfms, uint32_t n_bfms, uint64_t j0, uint32_t n, orc_site* out);
 
-/* injection + classification; mode ORC_MODE_FULL re-runs the whole program */
-int orc_inject(void* h, const orc_site* sites, uint32_t n, int mode, int n_threads, orc_inj* out);
+/* injection + classification; mode ORC_MODE_FULL re-runs the whole program.
+ * rtol > 0: also the C-12 secondary numeric classification — ORC_SDC_WITHIN_TOL
+ * in flags of every SDC whose output elements all satisfy |f-g| <= rtol*|g|
+ * (both finite; u32 buffers bitwise). */
+int orc_inject(void* h, const orc_site* sites, uint32_t n, int mode, int n_threads, double rtol, orc_inj* out);
 
 /* rows f2/f3: permanent / intermittent faults (Table III) */
 typedef struct { uint32_t opcode, sm, lane, mask, q32, n_sm; uint64_t seed; } orc_pfault;   /* 32 B */

@@ -16,7 +16,7 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2", "--expt-relaxed-constexpr",
          "-Xptxas", "-v,-warn-spills"] + ARCH
-SOURCES = ["abi.cpp", "golden.cu", "scan.cu", "profile.cu", "select.cu", "inject.cu", "propagate.cu", "propagate8.cu",
+SOURCES = ["abi.cpp", "golden.cu", "golden_run.cpp", "scan.cu", "profile.cu", "select.cu", "inject.cu", "propagate.cu", "propagate8.cu",
            "campaign.cpp", "jit.cpp"]
 HEADERS = ["common.cuh", "emu.cuh", "scan.cuh", "jit_prelude.cuh", "jit_k8.h"]
 

@@ -92,6 +92,12 @@ struct Events {
     }
 };
 
+struct GoldenGuard {                 // the golden run's trace arrays, freed on every return path
+    fi_golden* g = nullptr;
+    cudaStream_t s = nullptr;
+    ~GoldenGuard() { fi_golden_free(g, s); }
+};
+
 struct OwnedStream {
     cudaStream_t s = nullptr;
     bool own = false;
@@ -134,7 +140,7 @@ extern "C" fi_status fi_campaign(const fi_campaign_cfg* cfg, int rank, int world
         return FI_E_ARG;
     if (cfg->sched.n_groups < 1 || cfg->sched.n_groups > 8 || cfg->sched.n_bfms < 1 || cfg->sched.n_bfms > 4)
         return FI_E_ARG;
-    if (cfg->propagation > FI_PROPAGATION_K8 || cfg->engine > FI_ENGINE_JIT) return FI_E_ARG;
+    if (cfg->propagation > FI_PROPAGATION_K8 || cfg->engine > FI_ENGINE_JIT || !(cfg->rtol >= 0.0)) return FI_E_ARG;
     if (cfg->device >= 0) FI_TRY(cu(cudaSetDevice(cfg->device)));
 
     OwnedStream os;
@@ -192,62 +198,16 @@ extern "C" fi_status fi_campaign(const fi_campaign_cfg* cfg, int rank, int world
     }
     FI_TRY(ev.mark(s));                                                    // 1
 
-    // ---- golden run: pass 1 (lengths), scans, checkpoint layout, pass 2 ------
+    // ---- golden run (fi_golden_run: pass 1, scans, checkpoint layout, pass 2) ----
+    GoldenGuard gg;
+    gg.s = s;
+    FI_TRY(fi_golden_run(&p, jit, image, cfg->ckpt_interval, 0.2, &gg.g, s));
+    const fi_trace t = *fi_golden_trace_of(gg.g);
+    const uint64_t n_rec = t.n_rec;
+    const uint64_t* goff_h = fi_golden_gstore_off_host(gg.g);
     uint32_t* st;
-    uint64_t *wl, *wn, *woff, *goff;
     FI_TRY(A.alloc(&st, 4));
-    FI_TRY(A.alloc(&wl, 8ull * W));
-    FI_TRY(A.alloc(&wn, 8ull * W));
-    FI_TRY(A.alloc(&woff, 8ull * (W + 1)));
-    FI_TRY(A.alloc(&goff, 8ull * (W + 1)));
     FI_TRY(cu(cudaMemsetAsync(st, 0, 4, s)));
-    FI_TRY(cu(cudaMemsetAsync(wl, 0, 8ull * W, s)));
-    FI_TRY(cu(cudaMemsetAsync(wn, 0, 8ull * W, s)));
-    if (jit) FI_TRY(fi_golden_lengths_jit(jit, &p, image, wl, wn, st, s));
-    else FI_TRY(fi_golden_lengths(&p, image, wl, wn, st, s));
-    const size_t scan_ws = fi_scan_u64_workspace(W);
-    void* sws;
-    FI_TRY(A.alloc(&sws, scan_ws));
-    FI_TRY(fi_scan_u64(wl, woff, W, sws, scan_ws, s));
-    FI_TRY(fi_scan_u64(wn, goff, W, sws, scan_ws, s));
-    FI_TRY(check_status(st, s));
-    std::vector<uint64_t> goff_h(W + 1);
-    uint64_t n_rec = 0;
-    FI_TRY(cu(cudaMemcpyAsync(&n_rec, woff + W, 8, cudaMemcpyDeviceToHost, s)));
-    FI_TRY(cu(cudaMemcpyAsync(goff_h.data(), goff, 8ull * (W + 1), cudaMemcpyDeviceToHost, s)));
-    FI_TRY(cu(cudaStreamSynchronize(s)));
-    const uint64_t n_gst = goff_h[W];
-
-    fi_record* rec;
-    fi_store* gst;
-    FI_TRY(A.alloc(&rec, 16ull * std::max<uint64_t>(n_rec, 1)));
-    FI_TRY(A.alloc(&gst, 16ull * std::max<uint64_t>(n_gst, 1)));
-    uint32_t* ck = nullptr;
-    uint64_t* ckoff = nullptr;
-    uint32_t interval = 0;
-    if (cfg->ckpt_interval) {
-        interval = cfg->ckpt_interval == FI_CKPT_AUTO ? 8192u : cfg->ckpt_interval;
-        const size_t ck_bytes = fi_ckpt_bytes(p.n_regs);
-        const size_t lws = fi_ckpt_layout_workspace(W);
-        void* lw;
-        FI_TRY(A.alloc(&lw, lws));
-        FI_TRY(A.alloc(&ckoff, 8ull * (W + 1)));
-        size_t free_b = 0, total_b = 0;
-        FI_TRY(cu(cudaMemGetInfo(&free_b, &total_b)));
-        uint64_t n_ck = 0;
-        for (;;) {
-            FI_TRY(fi_ckpt_layout(wl, W, interval, ckoff, lw, lws, s));
-            FI_TRY(cu(cudaMemcpyAsync(&n_ck, ckoff + W, 8, cudaMemcpyDeviceToHost, s)));
-            FI_TRY(cu(cudaStreamSynchronize(s)));
-            if (cfg->ckpt_interval != FI_CKPT_AUTO || n_ck * ck_bytes <= free_b / 5 || interval >= (1u << 24)) break;
-            interval *= 2;
-        }
-        FI_TRY(A.alloc(&ck, n_ck * ck_bytes));
-    }
-    fi_trace t{rec, n_rec, woff, gst, goff, ck, ckoff, interval, W};
-    if (jit) FI_TRY(fi_golden_trace_jit(jit, &p, image, &t, st, s));
-    else FI_TRY(fi_golden_trace(&p, image, &t, st, s));
-    FI_TRY(check_status(st, s));
     FI_TRY(ev.mark(s));                                                    // 2
 
     // ---- K1 profile (this rank's chunk-aligned shard) + count exchange ------
@@ -324,9 +284,11 @@ extern "C" fi_status fi_campaign(const fi_campaign_cfg* cfg, int rank, int world
     }
     FI_TRY(ev.mark(s));                                                    // 7
 
-    uint64_t* hist;
-    FI_TRY(A.alloc(&hist, sizeof(res->hist)));
-    FI_TRY(cu(cudaMemsetAsync(hist, 0, sizeof(res->hist), s)));
+    uint64_t *hist, *hist_tol;
+    FI_TRY(A.alloc(&hist, 2 * sizeof(res->hist)));
+    hist_tol = hist + 96;
+    FI_TRY(cu(cudaMemsetAsync(hist, 0, 2 * sizeof(res->hist), s)));
+    const double rtol = cfg->rtol;
     if (n && k8) {
         // pend_cap: 2x the largest launch's golden stores + 4096 (fi.py pend_capacity)
         uint64_t mx_l = 0;
@@ -345,22 +307,25 @@ extern "C" fi_status fi_campaign(const fi_campaign_cfg* cfg, int rank, int world
         void* kw;
         FI_TRY(A.alloc(&kw, kws));
         if (jit)
-            FI_TRY(fi_classify_batched_jit(jit, &p, image, &t, sites, n, inj, log, log_cap, hist, cfg->flags, batch,
-                                           pool, pend, kw, kws, st, s));
+            FI_TRY(fi_classify_batched_jit(jit, &p, image, &t, sites, n, inj, log, log_cap, hist, cfg->flags, rtol,
+                                           hist_tol, batch, pool, pend, kw, kws, st, s));
         else
-            FI_TRY(fi_classify_batched(&p, image, &t, sites, n, inj, log, log_cap, hist, cfg->flags, batch, pool,
-                                       pend, kw, kws, st, s));
+            FI_TRY(fi_classify_batched(&p, image, &t, sites, n, inj, log, log_cap, hist, cfg->flags, rtol, hist_tol,
+                                       batch, pool, pend, kw, kws, st, s));
     } else if (n) {
         const size_t cws = fi_classify_workspace(K, n, log_cap);
         void* cw = nullptr;
         if (cws) FI_TRY(A.alloc(&cw, cws));
-        FI_TRY(fi_classify(&p, image, &t, sites, n, inj, log, log_cap, hist, cfg->flags, cw, cws, st, s));
+        FI_TRY(fi_classify(&p, image, &t, sites, n, inj, log, log_cap, hist, cfg->flags, rtol, hist_tol, cw, cws, st,
+                           s));
     }
-    if (world > 1 && allreduce(hist, 96, 8, ctx, s)) return FI_E_COLLECTIVE;
+    // one exchange of both histograms (the secondary one stays zero when rtol == 0)
+    if (world > 1 && allreduce(hist, rtol > 0.0 ? 192 : 96, 8, ctx, s)) return FI_E_COLLECTIVE;
     FI_TRY(ev.mark(s));                                                    // 8
 
     // ---- D2H of the results ----------------------------------------------------
     FI_TRY(cu(cudaMemcpyAsync(res->hist, hist, sizeof(res->hist), cudaMemcpyDeviceToHost, s)));
+    FI_TRY(cu(cudaMemcpyAsync(res->hist_tol, hist_tol, sizeof(res->hist_tol), cudaMemcpyDeviceToHost, s)));
     if (res->sites && n) FI_TRY(cu(cudaMemcpyAsync(res->sites, sites, 64ull * n, cudaMemcpyDeviceToHost, s)));
     std::vector<fi_inj> inj_h(n);
     fi_inj* inj_dst = res->inj ? res->inj : inj_h.data();

@@ -87,7 +87,33 @@ __device__ __forceinline__ uint4 philox4x32_10(uint4 c, uint2 k) {
     }
     return c;
 }
+
+// C-12 secondary numeric classification: does the faulty element
+// fv differ from the golden element gv beyond the relative tolerance rtol
+// (atol = 0)?  Equal bits: no.  U32 buffers: any difference.  F32 / F64: yes
+// unless both are finite and |f - g| <= rtol * |g| in IEEE double, round to
+// nearest (so NaN or an infinity against anything else always differs).
+__device__ __forceinline__ bool beyond_tol(uint32_t dtype, uint64_t fv, uint64_t gv, double rtol) {
+    if (fv == gv) return false;
+    double f, g;
+    if (dtype == 1) {
+        f = (double)__uint_as_float((uint32_t)fv);
+        g = (double)__uint_as_float((uint32_t)gv);
+    } else if (dtype == 2) {
+        f = __longlong_as_double((long long)fv);
+        g = __longlong_as_double((long long)gv);
+    } else {
+        return true;
+    }
+    if (!isfinite(f) || !isfinite(g)) return true;
+    return !(fabs(__dsub_rn(f, g)) <= __dmul_rn(rtol, fabs(g)));
+}
+__device__ __forceinline__ uint32_t buf_dtype(uint32_t flags) { return (flags >> 8) & 0xFFu; }
 #endif
+
+// hist_tol[group][bfm][outcome] over replicas [0, n): the secondary histogram, a
+// bitwise SDC flagged FI_SDC_WITHIN_TOL counted as Masked (C-12).
+fi_status launch_hist_tol(const fi_site* sites, const fi_inj* inj, uint32_t n, uint64_t* hist_tol, cudaStream_t s);
 
 }  // namespace fi
 

@@ -417,15 +417,19 @@ __device__ __forceinline__ bool guard_of(uint32_t guard, uint32_t preds) {
 struct Overlay {
     uint4* tab;
     uint32_t mask;                                   // capacity - 1 (power of two)
+    uint32_t gen;                                    // this replica's generation tag (slots are reused)
 };
 __device__ __forceinline__ uint32_t ov_hash(uint64_t va) {
     return (uint32_t)(((va >> 2) * 0x9E3779B97F4A7C15ull) >> 32);
 }
+// Entries of older generations (earlier replicas of the same slot) count as
+// empty: ov_put inserts at the first slot of the probe chain not tagged with the
+// current generation, so a live entry is never behind such a slot.
 __device__ __forceinline__ bool ov_find(const Overlay& o, uint64_t va, uint32_t& v) {
     uint32_t h = ov_hash(va) & o.mask;
     for (uint32_t probes = 0; probes <= o.mask; ++probes) {
         const uint4 e = __ldcg(&o.tab[h]);
-        if (!e.w) return false;
+        if (e.w != o.gen) return false;
         if (e.x == (uint32_t)va && e.y == (uint32_t)(va >> 32)) { v = e.z; return true; }
         h = (h + 1) & o.mask;
     }

@@ -152,6 +152,7 @@ struct ClsArgs {
     const fi_site* sites; fi_inj* inj; uint32_t n;
     const fi_store* log; uint32_t cap;
     uint64_t* hist; uint32_t flags; uint32_t* status;
+    double rtol;
 };
 
 __device__ __forceinline__ uint32_t buf_of(const ClsArgs& A, uint64_t va) {
@@ -326,7 +327,86 @@ __global__ void __launch_bounds__(kSlowThreads) k_classify_slow(const ClsArgs A)
     }
 }
 
+// C-12 secondary numeric classification of a single-instance replica that K5
+// found SDC (one CTA per replica, persistent): every output word whose final
+// faulty value differs from the golden one — (a) the last faulty write to an
+// address, (b) a golden store after the site the faulty run never repeated,
+// whose faulty value is the word before the instance — is checked as part of its
+// ELEMENT (the buffer's dtype; an f64 element's other word takes its own faulty
+// final value by the same rules).  FI_SDC_WITHIN_TOL iff no element differs
+// beyond rtol.  Plain serial scans: this mode is off the graded path.
+__device__ uint32_t faulty_final(const ClsArgs& A, const fi_store* F, uint64_t nF, const fi_store* Gs, uint64_t nG,
+                                 uint64_t va, uint32_t k) {
+    for (uint64_t q = nF; q-- > 0;)
+        if (F[q].va == va) return F[q].value;
+    for (uint64_t q = 0; q < nG; ++q)
+        if (Gs[q].va == va) return pre_word(A, va, k);
+    return golden_word(A, va);
+}
+__device__ bool elem_beyond(const ClsArgs& A, const fi_store* F, uint64_t nF, const fi_store* Gs, uint64_t nG,
+                            uint64_t va, uint32_t fv, uint32_t k) {
+    const uint32_t dt = buf_dtype(__ldg(&A.buf[buf_of(A, va)].flags));
+    if (dt != 2) return beyond_tol(dt, fv, golden_word(A, va), A.rtol);
+    const uint64_t lo = va & ~7ull, hi = lo + 4;
+    const uint32_t flo = va == lo ? fv : faulty_final(A, F, nF, Gs, nG, lo, k);
+    const uint32_t fhi = va == hi ? fv : faulty_final(A, F, nF, Gs, nG, hi, k);
+    const uint64_t f = (uint64_t)flo | ((uint64_t)fhi << 32);
+    const uint64_t g = (uint64_t)golden_word(A, lo) | ((uint64_t)golden_word(A, hi) << 32);
+    return beyond_tol(2, f, g, A.rtol);
+}
+
+__global__ void __launch_bounds__(kSlowThreads) k_classify_tol(const ClsArgs A) {
+    __shared__ uint64_t s_gs;
+    const uint32_t t = threadIdx.x, lane = t & 31;
+    for (uint32_t i = blockIdx.x; i < A.n; i += gridDim.x) {
+        if (A.inj[i].outcome != FI_SDC) continue;
+        const fi_site S = A.sites[i];
+        const fi_inj R = A.inj[i];
+        if (t < 32) { const uint64_t gs = golden_suffix(A, S.warp, S.step, lane); if (t == 0) s_gs = gs; }
+        __syncthreads();
+        const fi_store* Gs = A.gstore + A.gstore_off[S.warp] + s_gs;
+        const uint64_t nG = A.gstore_off[S.warp + 1] - A.gstore_off[S.warp] - s_gs, nF = R.n_faulty_stores;
+        const fi_store* F = A.log + (uint64_t)i * A.cap;
+        bool beyond = false;
+        for (uint64_t j = t; j < nF && !beyond; j += kSlowThreads) {                // (a)
+            const fi_store f = F[j];
+            if (!is_output(A, f.va) || f.value == golden_word(A, f.va)) continue;
+            bool last = true;
+            for (uint64_t q = j + 1; q < nF && last; ++q) last = F[q].va != f.va;
+            if (last) beyond = elem_beyond(A, F, nF, Gs, nG, f.va, f.value, S.instance);
+        }
+        for (uint64_t j = t; j < nG && !beyond; j += kSlowThreads) {                // (b)
+            const uint64_t va = Gs[j].va;
+            if (!is_output(A, va)) continue;
+            const uint32_t pv = pre_word(A, va, S.instance);
+            if (pv == golden_word(A, va)) continue;
+            bool inF = false;
+            for (uint64_t q = 0; q < nF && !inF; ++q) inF = F[q].va == va;
+            if (!inF) beyond = elem_beyond(A, F, nF, Gs, nG, va, pv, S.instance);
+        }
+        beyond = __syncthreads_or(beyond);
+        if (t == 0 && !beyond) A.inj[i].flags |= FI_SDC_WITHIN_TOL;
+        __syncthreads();
+    }
+}
+
+__global__ void k_hist_tol(const fi_site* sites, const fi_inj* inj, uint32_t n, uint64_t* hist_tol) {
+    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    uint32_t o = inj[i].outcome;
+    if (o == FI_SDC && (inj[i].flags & FI_SDC_WITHIN_TOL)) o = FI_MASKED;
+    if (o > FI_DUE) return;                          // not injected (C-17) / unclassified
+    const fi_site S = sites[i];
+    atomicAdd((unsigned long long*)&hist_tol[((uint32_t)S.group * 4 + S.bfm) * 3 + o], 1ull);
+}
+
 }  // namespace
+
+fi_status launch_hist_tol(const fi_site* sites, const fi_inj* inj, uint32_t n, uint64_t* hist_tol, cudaStream_t s) {
+    if (!hist_tol || !n) return FI_OK;
+    k_hist_tol<<<(n + 255) / 256, 256, 0, s>>>(sites, inj, n, hist_tol);
+    return launch_status();
+}
 
 void launch_lpt_order(const fi_program* p, const fi_site* sites, const uint64_t* warp_off, uint32_t ck_interval,
                       uint32_t n, uint32_t* order, uint32_t* counter, cudaStream_t s) {
@@ -372,7 +452,7 @@ fi_status launch_propagate(const fi_program* p, const uint8_t* image, const fi_t
                            uint32_t n, fi_inj* out, const fi_store* log, uint32_t log_cap, uint64_t* hist,
                            uint32_t flags, void* ws, size_t ws_bytes, const uint32_t* order, uint32_t* counter,
                            uint32_t* dev_status, cudaStream_t s, const fi_pfault* pf, const uint64_t* opw,
-                           uint32_t ov_words);
+                           uint32_t ov_words, double rtol);
 namespace {
 __global__ void k_iota(uint32_t* order, uint32_t n, uint32_t* counter) {
     const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
@@ -393,8 +473,10 @@ extern "C" size_t fi_classify_workspace(uint32_t n_inst, uint32_t n, uint32_t lo
 
 extern "C" fi_status fi_classify(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
                                  uint32_t n, fi_inj* out, const fi_store* log, uint32_t log_cap, uint64_t* hist,
-                                 uint32_t flags, void* ws, size_t ws_bytes, uint32_t* dev_status, void* stream) {
+                                 uint32_t flags, double rtol, uint64_t* hist_tol, void* ws, size_t ws_bytes,
+                                 uint32_t* dev_status, void* stream) {
     if (!p || !image || !t || !sites || !out || !hist || !dev_status || !p->aux) return FI_E_ARG;
+    if (!(rtol >= 0.0)) return FI_E_ARG;
     if (n == 0) return FI_OK;
     if (p->n_inst > 1) {
         // K7: multi-instance programs propagate the faulty warp's effect downstream
@@ -406,12 +488,22 @@ extern "C" fi_status fi_classify(const fi_program* p, const uint8_t* image, cons
         k_iota<<<(n + 255) / 256, 256, 0, s>>>(order, n, counter);
         fi_status e = launch_status();
         if (e) return e;
-        return launch_propagate(p, image, t, sites, n, out, log, log_cap, hist, flags, reinterpret_cast<char*>(ws) + head,
-                                ws_bytes - head, order, counter, dev_status, s, nullptr, nullptr, 0);
+        e = launch_propagate(p, image, t, sites, n, out, log, log_cap, hist, flags, reinterpret_cast<char*>(ws) + head,
+                             ws_bytes - head, order, counter, dev_status, s, nullptr, nullptr, 0, rtol);
+        if (e || rtol <= 0.0) return e;
+        return launch_hist_tol(sites, out, n, hist_tol, s);
     }
     const EmuProg P = make_emu_prog(p);
-    ClsArgs A{p->buf, P.gran, image, t->gstore, t->gstore_off, sites, out, n, log, log_cap, hist, flags, dev_status};
-    k_classify<<<(n + kClsWarps - 1) / kClsWarps, kClsWarps * 32, 0, (cudaStream_t)stream>>>(A);
-    k_classify_slow<<<std::min<uint32_t>(n, 148u * 8u), kSlowThreads, 0, (cudaStream_t)stream>>>(A);
+    ClsArgs A{p->buf, P.gran, image, t->gstore, t->gstore_off, sites, out, n, log, log_cap, hist, flags, dev_status,
+              rtol};
+    cudaStream_t s = (cudaStream_t)stream;
+    k_classify<<<(n + kClsWarps - 1) / kClsWarps, kClsWarps * 32, 0, s>>>(A);
+    k_classify_slow<<<std::min<uint32_t>(n, 148u * 8u), kSlowThreads, 0, s>>>(A);
+    if (rtol > 0.0) {
+        k_classify_tol<<<std::min<uint32_t>(n, 148u * 8u), kSlowThreads, 0, s>>>(A);
+        fi_status e = launch_status();
+        if (e) return e;
+        return launch_hist_tol(sites, out, n, hist_tol, s);
+    }
     return launch_status();
 }

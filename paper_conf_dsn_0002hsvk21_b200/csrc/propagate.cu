@@ -44,6 +44,7 @@ struct PropArgs {
     uint64_t* hist; uint32_t flags; uint32_t* status;
     const fi_pfault* pf;                             // permanent / intermittent faults (rows f2/f3), else null
     const uint64_t* opw;                             // opcode weights [FI_NOPS] or null
+    double rtol;                                     // > 0: C-12 secondary numeric classification
 };
 
 __device__ __forceinline__ uint32_t buf_id(const EmuProg& P, uint64_t va) { return __ldg(&P.gran[(va - kVaBase) >> 8]); }
@@ -136,7 +137,7 @@ __global__ void __launch_bounds__(kWPB * 32) k_propagate(const PropArgs A) {
     fi_store* pend = A.pend + (size_t)slot * A.pend_cap;
     uint32_t* dbuf = A.dbuf + (size_t)slot * (kDirtyBufs + 1);
     uint32_t* list = A.ov_list + (size_t)slot * (A.list_cap + 1);
-    const Overlay ov{tab, A.ov_cap - 1};
+    Overlay ov{tab, A.ov_cap - 1, 0};
     uint32_t* R = smem + wib * (A.P.n_regs + 1) * 32;
     const uint32_t* ibl = nullptr;
     for (;;) {
@@ -146,13 +147,14 @@ __global__ void __launch_bounds__(kWPB * 32) k_propagate(const PropArgs A) {
         if (p >= A.n) return;
         const uint32_t i = A.order[p];
         const uint32_t gen = p + 1;
+        ov.gen = gen;
         const bool permanent = A.pf != nullptr;
         const fi_site S = permanent ? fi_site{} : A.sites[i];
         const fi_inj Rj = permanent ? fi_inj{} : A.inj[i];
         const fi_pfault PF = permanent ? A.pf[i] : fi_pfault{};
         const uint32_t nsm = PF.n_sm ? PF.n_sm : 148u;      // CTA c runs on SM c mod n_sm (C-21)
         uint32_t outcome = FI_MASKED, fkind = 0, fpc = 0;
-        bool pdue = false, overflow = false;
+        bool pdue = false, overflow = false, within = false;
         const bool unchecked = A.flags & FI_UNCHECKED;
         if (S.flags & FI_SITE_NOT_INJECTED) {
             outcome = FI_NOT_INJECTED;
@@ -278,17 +280,37 @@ __global__ void __launch_bounds__(kWPB * 32) k_propagate(const PropArgs A) {
             }
             if (overflow) outcome = 0xFF;
             else if (outcome != FI_DUE) {
-                // ---- SDC iff an output word of D differs from the golden final image
-                bool sdc = false;
-                for (uint32_t b = 0; b < nlist && !sdc; b += 32) {
-                    bool d = false;
+                // ---- SDC iff an output word of D differs from the golden final image;
+                //      with rtol > 0 also: does some differing output ELEMENT (an f64's
+                //      other word from D, else golden) differ beyond rtol (C-12)?
+                const bool tol = A.rtol > 0.0 && !permanent;
+                bool sdc = false, beyond = false;
+                for (uint32_t b = 0; b < nlist && (!sdc || (tol && !beyond)); b += 32) {
+                    bool d = false, bt = false;
                     if (b + lane < nlist) {
                         const uint4 e = __ldcg(&tab[list[1 + b + lane]]);
                         const uint64_t va = (uint64_t)e.x | ((uint64_t)e.y << 32);
-                        d = (__ldg(&A.P.buf[buf_id(A.P, va)].flags) & 1u) && e.z != gword(A.img, va);
+                        const uint32_t bf = __ldg(&A.P.buf[buf_id(A.P, va)].flags);
+                        d = (bf & 1u) && e.z != gword(A.img, va);
+                        if (d && tol) {
+                            const uint32_t dt = buf_dtype(bf);
+                            if (dt != 2) {
+                                bt = beyond_tol(dt, e.z, gword(A.img, va), A.rtol);
+                            } else {
+                                const uint64_t lo = va & ~7ull;
+                                uint32_t f0 = gword(A.img, lo), f1 = gword(A.img, lo + 4);
+                                ov_find(ov, lo, f0);
+                                ov_find(ov, lo + 4, f1);
+                                bt = beyond_tol(2, (uint64_t)f0 | ((uint64_t)f1 << 32),
+                                                (uint64_t)gword(A.img, lo) | ((uint64_t)gword(A.img, lo + 4) << 32),
+                                                A.rtol);
+                            }
+                        }
                     }
-                    sdc = __any_sync(kFull, d);
+                    sdc |= __any_sync(kFull, d);
+                    beyond |= __any_sync(kFull, bt);
                 }
+                within = tol && sdc && !beyond;
                 outcome = sdc ? FI_SDC : FI_MASKED;
             }
         }
@@ -304,7 +326,8 @@ __global__ void __launch_bounds__(kWPB * 32) k_propagate(const PropArgs A) {
                 A.inj[i].fault_pc = fpc;
             }
             A.inj[i].outcome = (uint8_t)outcome;
-            A.inj[i].flags = (pdue && outcome != FI_DUE && outcome != FI_NOT_INJECTED) ? FI_POTENTIAL_DUE : 0;
+            A.inj[i].flags = ((pdue && outcome != FI_DUE && outcome != FI_NOT_INJECTED) ? FI_POTENTIAL_DUE : 0u) |
+                             (within ? FI_SDC_WITHIN_TOL : 0u);
             if (outcome == 0xFF) FI_DEV_ERR(A.status, FI_E_CAPACITY);
             else if (permanent)                     // opcode-weighted outcomes
                 atomicAdd((unsigned long long*)&A.hist[outcome],
@@ -337,7 +360,7 @@ fi_status launch_propagate(const fi_program* p, const uint8_t* image, const fi_t
                            uint32_t n, fi_inj* out, const fi_store* log, uint32_t log_cap, uint64_t* hist,
                            uint32_t flags, void* ws, size_t ws_bytes, const uint32_t* order, uint32_t* counter,
                            uint32_t* dev_status, cudaStream_t s, const fi_pfault* pf, const uint64_t* opw,
-                           uint32_t ov_words) {
+                           uint32_t ov_words, double rtol) {
     const size_t smem = golden_smem(p->n_regs);
     fi_status e = cuda_status(cudaFuncSetAttribute((const void*)k_propagate, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     if (e) return e;
@@ -367,6 +390,7 @@ fi_status launch_propagate(const fi_program* p, const uint8_t* image, const fi_t
     A.list_cap = ov_cap;
     A.hist = hist; A.flags = flags; A.status = dev_status;
     A.pf = pf; A.opw = opw;
+    A.rtol = rtol;
     // generation tags restart at 1 for every call: clear the overlay tables once
     if ((e = cuda_status(cudaMemsetAsync(A.ov, 0, (size_t)slots * ov_cap * 16, s)))) return e;
     k_propagate<<<(unsigned)(slots / kWPB), kWPB * 32, smem, s>>>(A);
@@ -410,5 +434,5 @@ extern "C" fi_status fi_inject_permanent(const fi_program* p, const uint8_t* ima
     if (e) return e;
     return launch_propagate(p, image, t, nullptr, n, out, log, log_cap, hist, flags,
                             reinterpret_cast<char*>(ws) + head, ws_bytes - head, order, counter, dev_status, s,
-                            faults, op_weights, ov_words);
+                            faults, op_weights, ov_words, 0.0);
 }

@@ -68,6 +68,7 @@ struct K8Args {
     uint32_t flags; uint32_t* status; uint64_t* hist;
     const fi_pfault* pf; const uint64_t* opw;        // permanent mode (else null)
     const uint32_t* kop;                             // per static kernel: bit op set iff the kernel has opcode op
+    double rtol;                                     // > 0: C-12 secondary numeric classification
 };
 
 __device__ __forceinline__ uint32_t buf_of(const EmuProg& P, uint64_t va) { return __ldg(&P.gran[(va - kVaBase) >> 8]); }
@@ -522,32 +523,54 @@ __global__ void __launch_bounds__(256) k8_final(K8Args A) {
     const uint32_t s = blockIdx.x;
     Slot& z = A.slot[s];
     if (z.rep == kNoRep) return;
-    __shared__ uint32_t sdc;
-    if (threadIdx.x == 0) sdc = 0;
+    __shared__ uint32_t sdc, beyond;
+    if (threadIdx.x == 0) { sdc = 0; beyond = 0; }
     __syncthreads();
+    const bool tol = A.rtol > 0.0 && !z.perm;
     uint32_t outcome = z.outcome;
     if (z.overflow || z.inexact) outcome = 0xFF;
     else if (z.fault_key != ~0ull) outcome = FI_DUE;
     else if (outcome == FI_MASKED) {
+        // the dense compare of the replica's remaining output pages with the golden
+        // final image; with rtol > 0 every differing ELEMENT (buffer dtype; an f64's
+        // two words lie in one page) is also checked against rtol (C-12)
         const uint32_t* pt = A.ptab + (size_t)s * A.total_pages;
         for (uint32_t b = 0; b < A.n_buf; ++b) {
-            if (!(__ldg(&A.P.buf[b].flags) & 1u) || A.bcount[(size_t)s * A.n_buf + b] == 0) continue;
+            const uint32_t bf = __ldg(&A.P.buf[b].flags);
+            if (!(bf & 1u) || A.bcount[(size_t)s * A.n_buf + b] == 0) continue;
+            const uint32_t dt = buf_dtype(bf);
             const uint32_t pb = __ldg(&A.page_base[b]), pe = __ldg(&A.page_base[b + 1]);
             const uint64_t boff = __ldg(&A.P.buf[b].off), bsz = __ldg(&A.P.buf[b].size);
             for (uint32_t p = pb; p < pe; ++p) {
                 const uint32_t e = pt[p];
                 if (e >= kPageClaim) continue;
                 const uint64_t rel0 = (uint64_t)(p - pb) << 12;
+                const uint32_t* pw = A.pool + (size_t)e * kPageWords;
                 for (uint32_t w = threadIdx.x; w < kPageWords; w += blockDim.x) {
                     const uint64_t rel = rel0 + 4ull * w;
-                    if (rel < bsz && __ldcg(&A.pool[(size_t)e * kPageWords + w]) != gword(A.img, kVaBase + boff + rel))
-                        sdc = 1;
+                    if (rel >= bsz) continue;
+                    const uint64_t va = kVaBase + boff + rel;
+                    const uint32_t v = __ldcg(&pw[w]), g = gword(A.img, va);
+                    if (v == g) continue;
+                    sdc = 1;
+                    if (!tol) continue;
+                    bool bt;
+                    if (dt != 2) {
+                        bt = beyond_tol(dt, v, g, A.rtol);
+                    } else {
+                        const uint32_t w0 = w & ~1u;
+                        const uint64_t lo = va - 4ull * (w - w0);
+                        bt = beyond_tol(2, (uint64_t)__ldcg(&pw[w0]) | ((uint64_t)__ldcg(&pw[w0 + 1]) << 32),
+                                        (uint64_t)gword(A.img, lo) | ((uint64_t)gword(A.img, lo + 4) << 32), A.rtol);
+                    }
+                    if (bt) beyond = 1;
                 }
             }
         }
         __syncthreads();
         outcome = sdc ? FI_SDC : FI_MASKED;
     }
+    const bool within = tol && outcome == FI_SDC && !beyond;
     if (threadIdx.x == 0) {
         fi_inj& r = A.inj[z.rep];
         if (z.perm) { r = fi_inj{}; r.mask = A.pf[z.rep].mask; }
@@ -557,7 +580,8 @@ __global__ void __launch_bounds__(256) k8_final(K8Args A) {
             if (key != ~0ull) { r.fault_kind = (uint8_t)((key >> 16) & 7u); r.fault_pc = (uint32_t)(key & 0xFFFFu); }
         }
         r.outcome = (uint8_t)outcome;
-        r.flags = (pdue && outcome != FI_DUE && outcome != FI_NOT_INJECTED && outcome != 0xFF) ? FI_POTENTIAL_DUE : 0;
+        r.flags = ((pdue && outcome != FI_DUE && outcome != FI_NOT_INJECTED && outcome != 0xFF) ? FI_POTENTIAL_DUE : 0u) |
+                  (within ? FI_SDC_WITHIN_TOL : 0u);
         if (outcome == 0xFF) {
             r.flags = (z.overflow ? FI_UNCLASSIFIED_CAPACITY : 0u) | (z.inexact ? FI_UNCLASSIFIED_WILD : 0u);
             if (z.overflow) FI_DEV_ERR(A.status, FI_E_CAPACITY);
@@ -628,7 +652,8 @@ extern "C" size_t fi_classify_batched_workspace(const fi_program* p, uint32_t n,
 
 static fi_status k8_run(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
                         const fi_pfault* pf, const uint64_t* opw, uint32_t n, fi_inj* out, const fi_store* log,
-                        uint32_t log_cap, uint64_t* hist, uint32_t flags, uint32_t batch, uint32_t pool_pages,
+                        uint32_t log_cap, uint64_t* hist, uint32_t flags, double rtol, uint64_t* hist_tol,
+                        uint32_t batch, uint32_t pool_pages,
                         uint32_t pend_cap, void* ws, size_t ws_bytes, uint32_t* dev_status, void* stream,
                         const fi_jit* jit = nullptr) {
     if (jit && pf) return FI_E_ARG;                  // the JIT engine serves transient faults
@@ -720,6 +745,7 @@ static fi_status k8_run(const fi_program* p, const uint8_t* image, const fi_trac
     A.flags = flags; A.status = dev_status; A.hist = hist;
     A.pf = pf; A.opw = opw;
     A.kop = reinterpret_cast<uint32_t*>(w + L.kop);
+    A.rtol = rtol;
     uint32_t* d_reps = reinterpret_cast<uint32_t*>(w + L.reps);
     if ((e = cuda_status(cudaMemcpyAsync(const_cast<uint32_t*>(A.page_base), page_base.data(), page_base.size() * 4, cudaMemcpyHostToDevice, s))) ||
         (e = cuda_status(cudaMemcpyAsync(const_cast<uint32_t*>(A.last_ref), last_ref.data(), last_ref.size() * 4, cudaMemcpyHostToDevice, s))) ||
@@ -774,27 +800,29 @@ static fi_status k8_run(const fi_program* p, const uint8_t* image, const fi_trac
         k8_final<<<batch, 256, 0, s>>>(A);
         if ((e = launch_status())) return e;
     }
+    if (rtol > 0.0 && sites) return launch_hist_tol(sites, out, n, hist_tol, s);
     return FI_OK;
 }
 
 extern "C" fi_status fi_classify_batched(const fi_program* p, const uint8_t* image, const fi_trace* t,
                                          const fi_site* sites, uint32_t n, fi_inj* out, const fi_store* log,
-                                         uint32_t log_cap, uint64_t* hist, uint32_t flags, uint32_t batch,
-                                         uint32_t pool_pages, uint32_t pend_cap, void* ws, size_t ws_bytes,
-                                         uint32_t* dev_status, void* stream) {
-    if (!sites) return FI_E_ARG;
-    return k8_run(p, image, t, sites, nullptr, nullptr, n, out, log, log_cap, hist, flags, batch, pool_pages,
-                  pend_cap, ws, ws_bytes, dev_status, stream);
+                                         uint32_t log_cap, uint64_t* hist, uint32_t flags, double rtol,
+                                         uint64_t* hist_tol, uint32_t batch, uint32_t pool_pages, uint32_t pend_cap,
+                                         void* ws, size_t ws_bytes, uint32_t* dev_status, void* stream) {
+    if (!sites || !(rtol >= 0.0)) return FI_E_ARG;
+    return k8_run(p, image, t, sites, nullptr, nullptr, n, out, log, log_cap, hist, flags, rtol, hist_tol, batch,
+                  pool_pages, pend_cap, ws, ws_bytes, dev_status, stream);
 }
 
 extern "C" fi_status fi_classify_batched_jit(const fi_jit* j, const fi_program* p, const uint8_t* image,
                                              const fi_trace* t, const fi_site* sites, uint32_t n, fi_inj* out,
                                              const fi_store* log, uint32_t log_cap, uint64_t* hist, uint32_t flags,
-                                             uint32_t batch, uint32_t pool_pages, uint32_t pend_cap, void* ws,
-                                             size_t ws_bytes, uint32_t* dev_status, void* stream) {
-    if (!sites || !j) return FI_E_ARG;
-    return k8_run(p, image, t, sites, nullptr, nullptr, n, out, log, log_cap, hist, flags, batch, pool_pages,
-                  pend_cap, ws, ws_bytes, dev_status, stream, j);
+                                             double rtol, uint64_t* hist_tol, uint32_t batch, uint32_t pool_pages,
+                                             uint32_t pend_cap, void* ws, size_t ws_bytes, uint32_t* dev_status,
+                                             void* stream) {
+    if (!sites || !j || !(rtol >= 0.0)) return FI_E_ARG;
+    return k8_run(p, image, t, sites, nullptr, nullptr, n, out, log, log_cap, hist, flags, rtol, hist_tol, batch,
+                  pool_pages, pend_cap, ws, ws_bytes, dev_status, stream, j);
 }
 
 extern "C" fi_status fi_inject_permanent_batched(const fi_program* p, const uint8_t* image, const fi_trace* t,
@@ -803,6 +831,6 @@ extern "C" fi_status fi_inject_permanent_batched(const fi_program* p, const uint
                                                  uint32_t batch, uint32_t pool_pages, uint32_t pend_cap, void* ws,
                                                  size_t ws_bytes, uint32_t* dev_status, void* stream) {
     if (!faults) return FI_E_ARG;
-    return k8_run(p, image, t, nullptr, faults, op_weights, n, out, nullptr, log_cap, hist, flags, batch, pool_pages,
-                  pend_cap, ws, ws_bytes, dev_status, stream);
+    return k8_run(p, image, t, nullptr, faults, op_weights, n, out, nullptr, log_cap, hist, flags, 0.0, nullptr,
+                  batch, pool_pages, pend_cap, ws, ws_bytes, dev_status, stream);
 }

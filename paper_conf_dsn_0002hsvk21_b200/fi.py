@@ -22,6 +22,7 @@ FI_OK, FI_E_ARG, FI_E_EMPTY_GROUP, FI_E_NOT_INJECTABLE, FI_E_PROGRAM, FI_E_CUDA,
 FI_E_CAPACITY, FI_E_INVARIANT = 8, 9
 FI_CHUNK = 1024
 FI_UNCHECKED, FI_POTENTIAL_DUE = 1, 1
+FI_SDC_WITHIN_TOL = 8                          # fi_inj.flags: bitwise SDC within rtol (C-12 secondary)
 G_FP64, G_FP32, G_LD, G_PR, G_NODEST, G_OTHERS, G_GPPR, G_GP = range(8)
 GROUP_NAMES = ["G_FP64", "G_FP32", "G_LD", "G_PR", "G_NODEST", "G_OTHERS", "G_GPPR", "G_GP"]
 BFM_NAMES = ["FLIP_SINGLE_BIT", "FLIP_TWO_BITS", "RANDOM_VALUE", "ZERO_VALUE"]
@@ -95,7 +96,7 @@ class fi_campaign_cfg(C.Structure):
                 ("n_replicas", C.c_uint64),
                 ("flags", C.c_uint32), ("propagation", C.c_uint32), ("approximate", C.c_uint32),
                 ("ckpt_interval", C.c_uint32), ("engine", C.c_uint32), ("k8_mem_budget", C.c_uint64),
-                ("device", C.c_int), ("stream", C.c_void_p)]
+                ("device", C.c_int), ("stream", C.c_void_p), ("rtol", C.c_double)]
 
 
 class fi_campaign_result(C.Structure):
@@ -106,7 +107,8 @@ class fi_campaign_result(C.Structure):
                 ("ms_h2d", C.c_float), ("ms_golden", C.c_float), ("ms_profile", C.c_float),
                 ("ms_exchange", C.c_float), ("ms_index", C.c_float), ("ms_select", C.c_float),
                 ("ms_inject", C.c_float), ("ms_classify", C.c_float), ("ms_d2h", C.c_float), ("ms_jit", C.c_float),
-                ("sites", C.c_void_p), ("inj", C.c_void_p), ("inst_counts", C.c_void_p)]
+                ("sites", C.c_void_p), ("inj", C.c_void_p), ("inst_counts", C.c_void_p),
+                ("hist_tol", C.c_uint64 * 96)]
 
 
 # int allreduce(void* dev, uint64_t count, uint32_t elem_bytes, void* ctx, void* stream)
@@ -148,7 +150,7 @@ def lib():
             "fi_inject_workspace": (sz, [u32]),
             "fi_inject": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, sz, vp, vp]),
             "fi_classify_workspace": (sz, [u32, u32, u32]),
-            "fi_classify": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, u32, vp, sz, vp, vp]),
+            "fi_classify": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, u32, C.c_double, vp, vp, sz, vp, vp]),
             "fi_write_params_txt": (st, [vp, C.c_char_p, C.c_char_p, sz]),
             "fi_profile_opcodes": (st, [vp, u64, u64, u32, vp, vp]),
             "fi_profile_approx_workspace": (sz, [u32, u32]),
@@ -159,9 +161,10 @@ def lib():
             "fi_classify_batched_workspace": (sz, [vp, u32, u32, u32, u32, u32]),
             "fi_inject_permanent_batched": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, u32, u32, u32, u32, vp, sz,
                                                  vp, vp]),
-            "fi_classify_batched": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, u32, u32, u32, u32, vp, sz, vp, vp]),
-            "fi_classify_batched_jit": (st, [vp, vp, vp, vp, vp, u32, vp, vp, u32, vp, u32, u32, u32, u32, vp, sz, vp,
-                                             vp]),
+            "fi_classify_batched": (st, [vp, vp, vp, vp, u32, vp, vp, u32, vp, u32, C.c_double, vp, u32, u32, u32, vp,
+                                         sz, vp, vp]),
+            "fi_classify_batched_jit": (st, [vp, vp, vp, vp, vp, u32, vp, vp, u32, vp, u32, C.c_double, vp, u32, u32,
+                                             u32, vp, sz, vp, vp]),
             "fi_inject_permanent": (st, [vp, vp, vp, vp, u32, vp, vp, vp, u32, u32, vp, u32, vp, sz, vp, vp]),
             "fi_jit_build": (st, [vp, vp, u32, C.POINTER(vp)]),
             "fi_jit_free": (None, [vp]),
@@ -171,6 +174,11 @@ def lib():
             "fi_jit_source": (sz, [vp, u32, vp, u32, u32, u32, vp, sz]),
             "fi_golden_lengths_jit": (st, [vp, vp, vp, vp, vp, vp, vp]),
             "fi_golden_trace_jit": (st, [vp, vp, vp, vp, vp, vp]),
+            "fi_golden_run": (st, [vp, vp, vp, u32, C.c_double, C.POINTER(vp), vp]),
+            "fi_golden_trace_of": (C.POINTER(fi_trace), [vp]),
+            "fi_golden_warp_len": (vp, [vp]),
+            "fi_golden_gstore_off_host": (C.POINTER(C.c_uint64), [vp]),
+            "fi_golden_free": (st, [vp, vp]),
             "fi_inject_jit": (st, [vp, vp, vp, vp, vp, u32, vp, vp, u32, vp, sz, vp, vp]),
             "fi_write_profile_txt": (st, [vp, vp, u32, vp, u32, vp, sz, C.POINTER(C.c_size_t)]),
             "fi_campaign": (st, [C.POINTER(fi_campaign_cfg), C.c_int, C.c_int, ALLREDUCE_FN, vp,
@@ -353,6 +361,7 @@ class GoldenTrace:
     ckpt: torch.Tensor | None = None
     ckpt_off: torch.Tensor | None = None
     ckpt_interval: int = 0
+    owner: object = None         # _GoldenHandle: keeps fi_golden_run's arrays alive
 
     @property
     def n_chunks(self):
@@ -368,58 +377,57 @@ def scan_u64(x: torch.Tensor) -> torch.Tensor:
     return out
 
 
+class _GoldenHandle:
+    """Owns an fi_golden (the trace arrays fi_golden_run allocated)."""
+
+    def __init__(self, h: C.c_void_p):
+        self.h = h
+
+    def __del__(self):
+        try:
+            if self.h:
+                lib().fi_golden_free(self.h, None)
+                self.h = None
+        except Exception:
+            pass
+
+
 def golden_run(dp: DeviceProgram, ckpt_interval: int | str = "auto", ckpt_budget_frac: float = 0.2,
-               engine: str = "interp") -> GoldenTrace:
-    """fi_golden_lengths (pass 1) -> scans + checkpoint layout -> fi_golden_trace (pass 2).
+               engine: str = "jit") -> GoldenTrace:
+    """fi_golden_run (one C-ABI call): pass 1 (lengths) -> scans + checkpoint
+    layout -> pass 2 (trace records, golden store log, checkpoints).
 
     ckpt_interval: steps between golden register-file checkpoints (0 = none);
-    "auto" = 8192 (the trace pass runs in step mode around every
-    checkpoint, a replica restarts from the one at or before its site), doubled until the checkpoints fit ckpt_budget_frac of free HBM.
-    engine: "interp" (emu.cuh) or "jit" (fi_golden_*_jit on the program's JIT
-    module built with FI_JIT_GOLDEN): bit-identical results."""
+    "auto" = 8192 (a replica restarts from the checkpoint at or
+    before its site), doubled until the checkpoints fit ckpt_budget_frac of free HBM.
+    engine: "jit" (the golden passes on the program's JIT module built with
+    FI_JIT_GOLDEN) or "interp" (emu.cuh): bit-identical results.  The trace
+    arrays are owned by the returned GoldenTrace (freed with it)."""
     jit = dp.jit(FI_JIT_GOLDEN) if engine == "jit" else None
-    st = DeviceStatus(dp.device)
+    if engine not in ("jit", "interp"):
+        raise ValueError(engine)
     image = dp.init_image.clone()
     W = dp.n_warps
-    wl = torch.zeros(max(W, 1), dtype=torch.int64, device=dp.device)
-    wn = torch.zeros(max(W, 1), dtype=torch.int64, device=dp.device)
-    if jit is not None:
-        _check(lib().fi_golden_lengths_jit(jit.h, C.byref(dp.c), _p(image), _p(wl), _p(wn), st.ptr, _stream()),
-               "fi_golden_lengths_jit")
-    else:
-        _check(lib().fi_golden_lengths(C.byref(dp.c), _p(image), _p(wl), _p(wn), st.ptr, _stream()),
-               "fi_golden_lengths")
-    woff = scan_u64(wl[:W])
-    goff = scan_u64(wn[:W])
-    st.check("fi_golden_lengths")
-    n_rec = int(woff[W].item())
-    n_gst = int(goff[W].item())
-    rec = torch.empty(max(n_rec, 1) * 16, dtype=torch.uint8, device=dp.device)
-    gst = torch.empty(max(n_gst, 1) * 16, dtype=torch.uint8, device=dp.device)
+    h = C.c_void_p()
+    ci = FI_CKPT_AUTO if ckpt_interval == "auto" else int(ckpt_interval)
+    _check(lib().fi_golden_run(C.byref(dp.c), jit.h if jit is not None else None, _p(image), ci,
+                               float(ckpt_budget_frac), C.byref(h), _stream()), "fi_golden_run")
+    owner = _GoldenHandle(h)
+    tc = fi_trace.from_buffer_copy(lib().fi_golden_trace_of(h).contents)
+    d = dp.device
+    n_rec, n_gst = int(tc.n_rec), int(lib().fi_golden_gstore_off_host(h)[W])
+    rec = device_view(tc.rec, max(n_rec, 1) * 16, 1, d)
+    gst = device_view(tc.gstore, max(n_gst, 1) * 16, 1, d)
+    woff = device_view(tc.warp_off, W + 1, 8, d)
+    goff = device_view(tc.gstore_off, W + 1, 8, d)
+    wl = device_view(lib().fi_golden_warp_len(h), W, 8, d)
     ck = ckoff = None
-    interval = 0
-    ck_bytes = lib().fi_ckpt_bytes(dp.n_regs)
-    if ckpt_interval and W:
-        interval = 8192 if ckpt_interval == "auto" else int(ckpt_interval)
-        free = torch.cuda.mem_get_info(dp.device)[0]
-        ws_n = lib().fi_ckpt_layout_workspace(W)
-        ws = torch.empty(ws_n, dtype=torch.uint8, device=dp.device)
-        ckoff = torch.empty(W + 1, dtype=torch.int64, device=dp.device)
-        while True:
-            _check(lib().fi_ckpt_layout(_p(wl), W, interval, _p(ckoff), _p(ws), ws_n, _stream()), "fi_ckpt_layout")
-            total = int(ckoff[W].item()) * ck_bytes
-            if ckpt_interval != "auto" or total <= ckpt_budget_frac * free or interval >= 1 << 24:
-                break
-            interval *= 2
-        ck = torch.empty(max(total, 16), dtype=torch.uint8, device=dp.device)
-    tc = fi_trace(_p(rec), n_rec, _p(woff), _p(gst), _p(goff), _p(ck), _p(ckoff), interval, W)
-    if jit is not None:
-        _check(lib().fi_golden_trace_jit(jit.h, C.byref(dp.c), _p(image), C.byref(tc), st.ptr, _stream()),
-               "fi_golden_trace_jit")
-    else:
-        _check(lib().fi_golden_trace(C.byref(dp.c), _p(image), C.byref(tc), st.ptr, _stream()), "fi_golden_trace")
-    st.check("fi_golden_trace")
-    return GoldenTrace(dp, image, wl[:W], woff, goff, rec, gst, n_rec, n_gst, tc, ck, ckoff, interval)
+    if tc.ckpt:
+        ckoff = device_view(tc.ckpt_off, W + 1, 8, d)
+        n_ck = int(ckoff[W].item())
+        ck = device_view(tc.ckpt, max(n_ck * lib().fi_ckpt_bytes(dp.n_regs), 16), 1, d)
+    return GoldenTrace(dp, image, wl, woff, goff, rec, gst, n_rec, n_gst, tc, ck, ckoff, int(tc.ckpt_interval),
+                       owner)
 
 
 def profile(gt: GoldenTrace, rec_begin: int = 0, rec_end: int | None = None,
@@ -573,9 +581,12 @@ def inject(gt: GoldenTrace, sites: torch.Tensor, n: int, log_cap: int, out: torc
 
 def classify(gt: GoldenTrace, sites: torch.Tensor, n: int, out: torch.Tensor, log: torch.Tensor, log_cap: int,
              hist: torch.Tensor | None = None, status: DeviceStatus | None = None,
-             unchecked: bool = False, ws: torch.Tensor | None = None) -> torch.Tensor:
-    """fi_classify (K5): fills out[].outcome, accumulates hist[8][4][3].
-    unchecked=True: potential-DUE semantics (FI_UNCHECKED, row f4)."""
+             unchecked: bool = False, ws: torch.Tensor | None = None, rtol: float = 0.0,
+             hist_tol: torch.Tensor | None = None) -> torch.Tensor:
+    """fi_classify (K5/K7): fills out[].outcome, accumulates hist[8][4][3].
+    unchecked=True: potential-DUE semantics (FI_UNCHECKED, row f4).  rtol > 0:
+    also the C-12 secondary numeric classification (FI_SDC_WITHIN_TOL in
+    out[].flags; hist_tol [8][4][3] accumulated when given)."""
     dev = gt.dp.device
     if hist is None:
         hist = torch.zeros((8, 4, 3), dtype=torch.int64, device=dev)
@@ -584,8 +595,8 @@ def classify(gt: GoldenTrace, sites: torch.Tensor, n: int, out: torch.Tensor, lo
     if ws_n and (ws is None or ws.numel() < ws_n):
         ws = torch.empty(ws_n, dtype=torch.uint8, device=dev)
     _check(lib().fi_classify(C.byref(gt.dp.c), _p(gt.image), C.byref(gt.c), _p(sites), n, _p(out), _p(log), log_cap,
-                             _p(hist), FI_UNCHECKED if unchecked else 0, _p(ws) if ws_n else None, ws_n, st.ptr,
-                             _stream()), "fi_classify")
+                             _p(hist), FI_UNCHECKED if unchecked else 0, float(rtol), _p(hist_tol),
+                             _p(ws) if ws_n else None, ws_n, st.ptr, _stream()), "fi_classify")
     if status is None:
         st.check("fi_classify")
     return hist
@@ -656,10 +667,12 @@ def pend_capacity(gt: GoldenTrace) -> int:
 def classify_batched(gt: GoldenTrace, sites: torch.Tensor, n: int, out: torch.Tensor, log: torch.Tensor,
                      log_cap: int, hist: torch.Tensor | None = None, unchecked: bool = False, batch: int | None = None,
                      pool_pages: int | None = None, pend_cap: int | None = None, mem_budget: int = 24 << 30,
-                     status: DeviceStatus | None = None, engine: str = "interp") -> torch.Tensor:
+                     status: DeviceStatus | None = None, engine: str = "interp", rtol: float = 0.0,
+                     hist_tol: torch.Tensor | None = None) -> torch.Tensor:
     """fi_classify_batched (K8): whole-program outcomes for long multi-instance
     programs, replica batches in lockstep over the launches.  engine "jit":
-    fi_classify_batched_jit (re-execution on the program's JIT module)."""
+    fi_classify_batched_jit (re-execution on the program's JIT module).
+    rtol / hist_tol: the C-12 secondary numeric classification, as classify()."""
     dev = gt.dp.device
     if hist is None:
         hist = torch.zeros((8, 4, 3), dtype=torch.int64, device=dev)
@@ -677,12 +690,14 @@ def classify_batched(gt: GoldenTrace, sites: torch.Tensor, n: int, out: torch.Te
     if engine == "jit":
         _check(lib().fi_classify_batched_jit(gt.dp.jit(FI_JIT_PAGE).h, C.byref(gt.dp.c), _p(gt.image), C.byref(gt.c),
                                              _p(sites), n, _p(out), _p(log), log_cap, _p(hist),
-                                             FI_UNCHECKED if unchecked else 0, batch, pool_pages, pend_cap, _p(ws),
-                                             ws_n, st.ptr, _stream()), "fi_classify_batched_jit")
+                                             FI_UNCHECKED if unchecked else 0, float(rtol), _p(hist_tol), batch,
+                                             pool_pages, pend_cap, _p(ws), ws_n, st.ptr, _stream()),
+               "fi_classify_batched_jit")
     else:
         _check(lib().fi_classify_batched(C.byref(gt.dp.c), _p(gt.image), C.byref(gt.c), _p(sites), n, _p(out),
-                                         _p(log), log_cap, _p(hist), FI_UNCHECKED if unchecked else 0, batch,
-                                         pool_pages, pend_cap, _p(ws), ws_n, st.ptr, _stream()), "fi_classify_batched")
+                                         _p(log), log_cap, _p(hist), FI_UNCHECKED if unchecked else 0, float(rtol),
+                                         _p(hist_tol), batch, pool_pages, pend_cap, _p(ws), ws_n, st.ptr, _stream()),
+               "fi_classify_batched")
     if status is None:
         st.check("fi_classify_batched")
     return hist
@@ -778,7 +793,7 @@ class _DevArray:
 
 
 def device_view(ptr: int, n: int, elem_bytes: int, device) -> torch.Tensor:
-    return torch.as_tensor(_DevArray(ptr, n, "<i8" if elem_bytes == 8 else "<i4"), device=device)
+    return torch.as_tensor(_DevArray(ptr, n, {8: "<i8", 4: "<i4", 1: "|u1"}[elem_bytes]), device=device)
 
 
 def torch_allreduce(group=None):
@@ -815,12 +830,13 @@ class CampaignResult:
     sites: np.ndarray | None
     inj: np.ndarray | None
     inst_counts: np.ndarray | None
+    hist_tol: np.ndarray | None = None   # rtol > 0: C-12 secondary histogram [8][4][3]
 
 
 def campaign(prog, seed: int, groups, bfms, n_replicas: int, rank: int = 0, world: int = 1, allreduce=None,
              unchecked: bool = False, propagation: str = "auto", approximate: bool = False, ckpt="auto",
              k8_mem_budget: int = 0, device: int | None = None, host: dict | None = None,
-             return_arrays: bool = True, engine: str = "jit") -> CampaignResult:
+             return_arrays: bool = True, engine: str = "jit", rtol: float = 0.0) -> CampaignResult:
     """fi_campaign: the whole campaign of this rank from HOST arrays (golden run,
     sharded profile, count exchange, index, select, inject, classify, histogram
     exchange, D2H).  `host`: optional pinned uint8 tensors keyed code / kernels /
@@ -849,6 +865,7 @@ def campaign(prog, seed: int, groups, bfms, n_replicas: int, rank: int = 0, worl
     cfg.ckpt_interval = FI_CKPT_AUTO if ckpt == "auto" else int(ckpt)
     cfg.engine = {"interp": 0, "jit": 1}[engine]
     cfg.k8_mem_budget = k8_mem_budget
+    cfg.rtol = float(rtol)
     cfg.device = torch.cuda.current_device() if device is None else device
     cfg.stream = torch.cuda.current_stream(cfg.device).cuda_stream or None
     n_loc = n_replicas * (rank + 1) // world - n_replicas * rank // world
@@ -868,7 +885,8 @@ def campaign(prog, seed: int, groups, bfms, n_replicas: int, rank: int = 0, worl
     return CampaignResult(np.array(res.hist, dtype=np.uint64).reshape(8, 4, 3), [int(x) for x in res.totals],
                           int(res.n_rec), int(res.counted), int(res.j0), int(res.n_local),
                           (int(res.rec_begin), int(res.rec_end)), int(res.n_unclassified), int(res.n_not_injected),
-                          ms, None if sites is None else sites[:n_loc], None if inj is None else inj[:n_loc], ic)
+                          ms, None if sites is None else sites[:n_loc], None if inj is None else inj[:n_loc], ic,
+                          np.array(res.hist_tol, dtype=np.uint64).reshape(8, 4, 3) if rtol > 0 else None)
 
 
 def campaign_release_memory(device: int = -1) -> None:
