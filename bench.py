@@ -133,40 +133,60 @@ class ClockSampler:
                 "reasons": reasons, "samples": len(self.samples)}
 
 
-def cpu_baseline(prog, sites_np, budget_s=12.0):
-    """The oracle as it stands, on this host's cores, over a bounded sample of the
-    same workload: interpretive count of the first warps (profile metric) and
-    warp-local injection of the first sampled replicas (injection metric)."""
+ORACLE_WARPS = 1024          # cpu_baseline and --impl reference interpret the same warps [0, 1024)
+ORACLE_SCAN_RECORDS = 1 << 27   # the trace-scan leg: the first 2^27 records (2 GiB) of the resident trace
+
+
+def oracle_count_sample(prog):
+    """The oracle's interpretive profile of a fixed bounded sample: warps
+    [0, ORACLE_WARPS) of the workload (golden interpretation + Table II count)."""
     import oracle as O
     nt = O.n_threads_default()
-    nw = max(1, min(prog.n_warps, nt))
+    nw = min(prog.n_warps, ORACLE_WARPS)
     t = time.perf_counter()
     n_rec, c = O.count_warps(prog, 0, nw, nt)
     dt = time.perf_counter() - t
-    while dt < budget_s / 3 and nw < prog.n_warps:
-        nw = min(prog.n_warps, nw * 2)
+    return int(c[4] + c[6]), int(n_rec), dt, nw, nt
+
+
+def cpu_baseline(prog, sites_np, camp=None, n_inj=1024):
+    """The oracle as it stands, on this host's cores, over bounded samples of the
+    same workload:
+      value       interpretive count of warps [0, ORACLE_WARPS) (the same sample the
+                  reference arm times each step);
+      trace_scan  the profiler's count over the first ORACLE_SCAN_RECORDS records of
+                  the resident trace, copied to host RAM first (copy not timed) —
+                  the CPU counterpart of K1;
+      injections  warp-local injection of replicas [0, n_inj)."""
+    import oracle as O
+    counted, n_rec, dt, nw, nt = oracle_count_sample(prog)
+    out = {
+        "value": counted / dt, "unit": "thread-dyn-instrs/s", "cores": nt, "kind": "oracle",
+        "value_per_core": counted / dt / nt,
+        "sample": f"oracle golden interpretation + Table II group count of warps [0,{nw}) of the workload "
+                  f"({n_rec} warp-records, {counted} thread-instrs) in {dt:.2f}s",
+    }
+    if camp is not None:
+        nr = min(camp.gt.n_rec, ORACLE_SCAN_RECORDS)
+        host = camp.gt.rec[:16 * nr].cpu().numpy()
         t = time.perf_counter()
-        n_rec, c = O.count_warps(prog, 0, nw, nt)
-        dt = time.perf_counter() - t
-    counted = int(c[4] + c[6])                     # NODEST + GPPR = all counted thread-instrs
-    prof_rate = counted / dt
-    ni = max(1, min(len(sites_np), nt))
+        c = O.scan_trace(host, camp.dp.n_inst, nt)
+        ds = time.perf_counter() - t
+        cs = int(c[:, 4].sum() + c[:, 6].sum())
+        out["trace_scan"] = {"value": cs / ds, "unit": "thread-dyn-instrs/s", "cores": nt,
+                             "value_per_core": cs / ds / nt, "records_per_s": nr / ds, "gb_per_s": 16 * nr / ds / 1e9,
+                             "sample": f"oracle scan (orc_scan_trace) of records [0,{nr}) of the resident trace "
+                                       f"({16 * nr / 2**30:.1f} GiB in host RAM, D2H not timed) in {ds:.2f}s"}
+        del host
+    ni = min(len(sites_np), n_inj)
     t = time.perf_counter()
     O.inject_local(prog, sites_np[:ni], nt)
     di = time.perf_counter() - t
-    while di < budget_s / 3 and ni < len(sites_np):      # grow the injection sample to ~budget/3 s as well
-        ni = min(len(sites_np), ni * 4)
-        t = time.perf_counter()
-        O.inject_local(prog, sites_np[:ni], nt)
-        di = time.perf_counter() - t
-    return {
-        "value": prof_rate, "unit": "thread-dyn-instrs/s", "cores": nt, "kind": "oracle",
-        "sample": f"oracle golden interpretation + Table II group count of warps [0,{nw}) of the workload "
-                  f"({n_rec} warp-records, {counted} thread-instrs) in {dt:.2f}s",
-        "injections_per_s": ni / di,
-        "injection_sample": f"oracle warp-local injection (golden + faulty re-execution of the site's warp, "
-                            f"classification) of replicas [0,{ni}) in {di:.2f}s",
-    }
+    out["injections_per_s"] = ni / di
+    out["injections_per_s_per_core"] = ni / di / nt
+    out["injection_sample"] = (f"oracle warp-local injection (golden + faulty re-execution of the site's warp, "
+                               f"classification) of replicas [0,{ni}) in {di:.2f}s")
+    return out
 
 
 def run_reference(args, rank, world):
@@ -175,17 +195,12 @@ def run_reference(args, rank, world):
         return
     prog, seed, groups, bfms, n = make_program(args.config)
     n = args.replicas or n
-    import oracle as O
-    nt = O.n_threads_default()
-    nw = max(1, min(prog.n_warps, nt))
     times, counted_tot = [], 0
     for i in range(args.warmup + args.steps):
-        t = time.perf_counter()
-        nr, c = O.count_warps(prog, 0, nw, nt)
-        dt = time.perf_counter() - t
+        counted, n_rec, dt, nw, nt = oracle_count_sample(prog)
         if i >= args.warmup:
             times.append(dt)
-            counted_tot += int(c[4] + c[6])
+            counted_tot += counted
     T = sum(times)
     val = counted_tot / T
     line = {"metric": "thread-dyn-instrs profiled/sec and injections/sec at 1/2/4/8 B200 (% HBM roofline)",
@@ -194,7 +209,9 @@ def run_reference(args, rank, world):
             "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
             "config": {"workload": workload_name(args.config, n)},
             "cpu_baseline": {"value": val, "unit": "thread-dyn-instrs/s", "cores": nt, "kind": "oracle",
-                             "sample": f"each step: oracle interpretation + group count of warps [0,{nw})"},
+                             "value_per_core": val / nt,
+                             "sample": f"each step: oracle golden interpretation + Table II group count of warps "
+                                       f"[0,{nw}) of the workload (the cpu_baseline sample of the fi arm)"},
             "e2e": {"value": val, "unit": "thread-dyn-instrs/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -244,7 +261,7 @@ def main():
     camp.check()
 
     stage_ms = {s: 0.0 for s in STAGES}
-    step_ms = []
+    step_ms, prof_ms, inj_ms = [], [], []
     emulated_steps = 0
     if world > 1:
         dist.barrier()
@@ -262,6 +279,8 @@ def main():
             stage_ms[s] += ev[prev].elapsed_time(ev[s])
             prev = s
         step_ms.append(ev["start"].elapsed_time(ev["end"]))
+        prof_ms.append(ev["start"].elapsed_time(ev["exchange"]))
+        inj_ms.append(ev["index"].elapsed_time(ev["classify"]))
         emulated_steps += int(camp.inj_ws[8:16].cpu().view(torch.int64).item())   # K4's own count (fi.h)
     t_timed1 = time.perf_counter()
     time.sleep(0.06)                                              # (the sample in flight at the end)
@@ -281,8 +300,11 @@ def main():
     T_k1 = allreduce_max(stage_ms["profile"] / 1e3, dev)
     T_inj = allreduce_max((stage_ms["select"] + stage_ms["inject"] + stage_ms["classify"]) / 1e3, dev)
     K = args.steps
-    value = counted * K / T_prof
-    inj_rate = n * K / T_inj
+    # value: the MEDIAN step, each rank's median, max over ranks
+    T_prof_med = allreduce_max(statistics.median(prof_ms) / 1e3, dev)
+    T_inj_med = allreduce_max(statistics.median(inj_ms) / 1e3, dev)
+    value = counted / T_prof_med
+    inj_rate = n / T_inj_med
 
     # K1 roofline: algorithmic bytes per launch = 16 B per record read + 32 B per chunk
     # written + 64 B per instance; duration = CUDA-event profile stage.
@@ -334,6 +356,8 @@ def main():
                    "l2": "flushed before every timed step (256 MiB write); trace 39 GB >> 126 MB L2",
                    "parallelism": f"replica+record sharding over {world} GPU(s)"},
         "injections_per_s": inj_rate,
+        "value_is": "median over the K timed steps of counted thread-instrs / (profile + count exchange time)",
+        "value_mean": counted * K / T_prof, "injections_per_s_mean": n * K / T_inj,
         "stages_ms_per_step": {s: stage_ms[s] / K for s in STAGES},
         "outcomes": {"masked": int(hist[..., 0].sum()), "sdc": int(hist[..., 1].sum()), "due": int(hist[..., 2].sum())},
         "roofline": k4,
@@ -353,7 +377,7 @@ def main():
     if rank == 0 and world == 1 and not args.no_secondary:
         line["secondary"] = secondary_c4(dev)
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        line["cpu_baseline"] = cpu_baseline(prog, camp.sites_np())
+        line["cpu_baseline"] = cpu_baseline(prog, camp.sites_np(), camp)
     if rank == 0:
         print(json.dumps(line), flush=True)
     if world > 1:

@@ -295,7 +295,9 @@ fi_status fi_inject(const fi_program* p, const uint8_t* image, const fi_trace* t
  * overlay, its stores diffed against its golden store log — and the replica is
  * classified on the whole program's outputs (PAPER.md:72 step (4), :206).
  * Scratch: fi_classify_workspace(n_inst, n, log_cap) bytes (0 for one instance).
- * Replicas whose overlay or update lists overflow get outcome 0xFF + FI_E_CAPACITY. */
+ * Replicas whose overlay or update lists overflow get outcome 0xFF + FI_E_CAPACITY.
+ * K7 CONSUMES `log`: a replica's log slot is reused as scratch for the stores of
+ * the later launches it re-executes (classify a log once; K5 and K8 only read it). */
 #define FI_UNCHECKED 1u
 #define FI_POTENTIAL_DUE 1u
 /* K8 outcome 0xFF (not classified) reasons in fi_inj.flags: a capacity was

@@ -97,6 +97,7 @@ def lib():
             L.orc_trace.argtypes = [vp, vp]
             L.orc_count_warps.restype = u64
             L.orc_count_warps.argtypes = [C.POINTER(_Program), u32, u32, i32, vp]
+            L.orc_scan_trace.argtypes = [vp, u64, u32, i32, vp]
             L.orc_select.argtypes = [vp, u64, vp, u32, vp, u32, u64, u32, vp]
             L.orc_locate.argtypes = [vp, i32, vp, u32, vp]
             L.orc_opcode_counts.argtypes = [vp, vp]
@@ -276,6 +277,16 @@ def count_warps(prog, w0: int, w1: int, n_threads: int | None = None) -> tuple[i
     out = np.zeros(8, dtype=np.uint64)
     n = lib().orc_count_warps(C.byref(p), w0, w1, n_threads or n_threads_default(), _ptr(out))
     return int(n), out
+
+
+def scan_trace(records: np.ndarray, n_inst: int, n_threads: int | None = None) -> np.ndarray:
+    """The profiler's count over an App. A.3 trace in host RAM (u64 [n_inst][8])."""
+    rec = np.ascontiguousarray(records).view(np.uint8).reshape(-1)
+    assert rec.size % 16 == 0
+    out = np.zeros((n_inst, 8), dtype=np.uint64)
+    if lib().orc_scan_trace(_ptr(rec), rec.size // 16, n_inst, n_threads or n_threads_default(), _ptr(out)):
+        raise OracleError(4, "record names an instance beyond n_inst")
+    return out
 
 
 def warp_site_rank(prog, warp: int, group: int, step: int, lane: int) -> tuple[int, int] | None:

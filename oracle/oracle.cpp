@@ -1277,3 +1277,34 @@ extern "C" int orc_inject_image(void* h, const orc_site* site, int mode, uint8_t
     if (!hk.fired || hk.bad) return -1;
     return fr.fault ? fr.fault : fr.pdue;
 }
+
+// The profiler's count over a trace already in host RAM ("dynamic
+// instruction counts ... Instructions that are not executed based on a predicate
+// register are not included"): for every App. A.3 record, popc(active & pred)
+// added to counts[instance][g] for each group g of its groupmask (Table II).  A
+// plain loop per record; threads take contiguous record ranges and their
+// partial sums are added at the end.  The CPU baseline of K1.
+extern "C" int orc_scan_trace(const orc_record* rec, uint64_t n, uint32_t n_inst, int n_threads, uint64_t* counts) {
+    n_threads = std::max(1, n_threads);
+    std::vector<std::vector<uint64_t>> part(n_threads, std::vector<uint64_t>((size_t)n_inst * 8, 0));
+    std::atomic<int> bad{0};
+    std::vector<std::thread> th;
+    for (int t = 0; t < n_threads; ++t)
+        th.emplace_back([&, t] {
+            const uint64_t r0 = n * (uint64_t)t / n_threads, r1 = n * (uint64_t)(t + 1) / n_threads;
+            uint64_t* c = part[t].data();
+            for (uint64_t r = r0; r < r1; ++r) {
+                const orc_record& R = rec[r];
+                if (R.instance >= n_inst) { bad = 1; return; }
+                const uint64_t k = (uint64_t)__builtin_popcount(R.active & R.pred);
+                const uint32_t gm = R.insn >> 24;
+                for (int g = 0; g < 8; ++g)
+                    if ((gm >> g) & 1) c[8 * (size_t)R.instance + g] += k;
+            }
+        });
+    for (auto& x : th) x.join();
+    std::fill(counts, counts + (size_t)n_inst * 8, 0);
+    for (int t = 0; t < n_threads; ++t)
+        for (size_t i = 0; i < (size_t)n_inst * 8; ++i) counts[i] += part[t][i];
+    return bad ? 1 : 0;
+}

@@ -84,6 +84,11 @@ uint64_t orc_n_golden_stores(void* h);
  * baselines.  Returns records interpreted. */
 uint64_t orc_count_warps(const orc_program* p, uint32_t w0, uint32_t w1, int n_threads, uint64_t* counts8);
 
+/* the profiler's count over a trace already in host RAM (K1's CPU baseline):
+ * counts[k][g] = sum over records of instance k with g in groupmask of
+ * popc(active & pred).  Returns 1 if a record names an instance >= n_inst. */
+int orc_scan_trace(const orc_record* rec, uint64_t n, uint32_t n_inst, int n_threads, uint64_t* counts);
+
 /* selection by enumeration (C-3..C-6).  With keep_trace=0 (single-
  * instance programs only) the site's warp comes from the per-warp counts and the
  * rank inside it from a re-interpretation of that warp — the same canonical order. */

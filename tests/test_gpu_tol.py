@@ -30,16 +30,16 @@ def _campaign(F, prog, seed, groups, bfms, n, how):
     os_ = g.select(seed, groups, bfms, 0, n)
     cap = F.log_capacity(gt)
     out, log = F.inject(gt, sites, n, cap)
-    out0 = out.clone()
+    out0, log0 = out.clone(), log.clone()          # (K7 reuses a replica's K4 log as scratch)
     import torch
     hist_tol = torch.zeros((8, 4, 3), dtype=torch.int64, device=dp.device)
     if how == "k5k7":
         hist = F.classify(gt, sites, n, out, log, cap, rtol=RTOL, hist_tol=hist_tol)
-        hist0 = F.classify(gt, sites, n, out0, log, cap)
+        hist0 = F.classify(gt, sites, n, out0, log0, cap)
     else:
         engine = "jit" if how == "k8jit" else "interp"
         hist = F.classify_batched(gt, sites, n, out, log, cap, rtol=RTOL, hist_tol=hist_tol, engine=engine)
-        hist0 = F.classify_batched(gt, sites, n, out0, log, cap, engine=engine)
+        hist0 = F.classify_batched(gt, sites, n, out0, log0, cap, engine=engine)
     gi = F.as_numpy(out, F.INJ_DTYPE, n)
     g0 = F.as_numpy(out0, F.INJ_DTYPE, n)
     oi = g.inject(os_, O.MODE_FULL, rtol=RTOL)

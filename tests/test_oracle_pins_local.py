@@ -207,3 +207,18 @@ def test_transient_address_fault_in_middle_launch_is_due():
         assert not prog.view(img, f"y{i}", "<u4").any()
     r = g.inject(site, O.MODE_FULL)[0]
     assert r["outcome"] == O.DUE and r["fault_kind"] == 2 and r["fault_pc"] == 17
+
+
+# ---------------------------------------------------------------------------
+# scan_trace (the K1 CPU baseline over a trace in host RAM)
+# ---------------------------------------------------------------------------
+def test_scan_trace_equals_counts_and_closed_form(mini_c2, c1):
+    """The per-record sum over the kept trace equals the interpreter's counts, the
+    C1 worked example and the mini-C2 closed form (Table II)."""
+    prog, g, _ = mini_c2
+    want, _ = sgemm_closed_form(256, 256, 256)
+    assert O.scan_trace(g.trace(), 1)[0].tolist() == want
+    assert O.scan_trace(c1.trace(), 1, n_threads=3)[0].tolist() == [0, 1024, 6144, 1024, 2048, 7168, 15360, 14336]
+    chain = O.Golden(P.multi_instance_chain(n_inst=3, shrink=20))
+    assert (O.scan_trace(chain.trace(), 3, n_threads=5) == chain.counts()).all()
+    assert (O.scan_trace(chain.trace()[:0], 3) == 0).all()
