@@ -169,14 +169,19 @@ def cpu_baseline(prog, sites_np, camp=None, n_inj=1024):
     if camp is not None:
         nr = min(camp.gt.n_rec, ORACLE_SCAN_RECORDS)
         host = camp.gt.rec[:16 * nr].cpu().numpy()
-        t = time.perf_counter()
-        c = O.scan_trace(host, camp.dp.n_inst, nt)
-        ds = time.perf_counter() - t
+        reps, t = 0, time.perf_counter()
+        while True:                                # repeat the scan for >= 2 s of CPU work
+            c = O.scan_trace(host, camp.dp.n_inst, nt)
+            reps += 1
+            ds = time.perf_counter() - t
+            if ds >= 2.0:
+                break
+        ds /= reps
         cs = int(c[:, 4].sum() + c[:, 6].sum())
         out["trace_scan"] = {"value": cs / ds, "unit": "thread-dyn-instrs/s", "cores": nt,
                              "value_per_core": cs / ds / nt, "records_per_s": nr / ds, "gb_per_s": 16 * nr / ds / 1e9,
                              "sample": f"oracle scan (orc_scan_trace) of records [0,{nr}) of the resident trace "
-                                       f"({16 * nr / 2**30:.1f} GiB in host RAM, D2H not timed) in {ds:.2f}s"}
+                                       f"({16 * nr / 2**30:.1f} GiB in host RAM, D2H not timed): {ds:.3f}s per scan, mean of {reps}"}
         del host
     ni = min(len(sites_np), n_inj)
     t = time.perf_counter()

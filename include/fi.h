@@ -410,6 +410,8 @@ double fi_jit_compile_seconds(const fi_jit* j);
 const char* fi_jit_log(void);
 fi_status fi_jit_compile_check(const fi_insn* code_host, uint32_t n_code, const fi_kernel* kern_host, uint32_t n_kern,
                                uint32_t n_regs, uint32_t modes, size_t* cubin_bytes);
+/* (fi_jit_source / fi_jit_compile_check also accept modes | 0x100: pass 1 as the
+ * control slice, as fi_jit_build picks it.) */
 size_t fi_jit_source(const fi_insn* code_host, uint32_t n_code, const fi_kernel* kern_host, uint32_t n_kern,
                      uint32_t n_regs, uint32_t modes, char* buf, size_t buf_bytes);
 /* K4 on the JIT module `j` built for p: same arguments, scratch, scheduling and
@@ -417,12 +419,19 @@ size_t fi_jit_source(const fi_insn* code_host, uint32_t n_code, const fi_kernel*
 fi_status fi_inject_jit(const fi_jit* j, const fi_program* p, const uint8_t* image, const fi_trace* t,
                         const fi_site* sites, uint32_t n, fi_inj* out, fi_store* log, uint32_t log_cap, void* ws,
                         size_t ws_bytes, uint32_t* dev_status, void* stream);
-/* The golden passes on a module built with FI_JIT_GOLDEN: same arguments and
- * results (trace records, store log, checkpoints, final image, lengths) as
- * fi_golden_lengths / fi_golden_trace, bit for bit. */
+/* The golden passes on a module built with FI_JIT_GOLDEN: same results (trace
+ * records, store log, checkpoints, final image, lengths) as fi_golden_lengths /
+ * fi_golden_trace, bit for bit, with one difference in who writes the image.
+ * fi_jit_build generates pass 1 as the CONTROL SLICE of each kernel (only the
+ * instructions that can reach a BRA / EXIT / STG guard, jit.cpp control_slice)
+ * when the program has one launch or no slice loads memory: that length pass
+ * leaves `image` untouched.  Pass 2 (fi_golden_trace_jit, one launch per instance
+ * in launch order) always stores into `image` (in: pass 1's image, out: the
+ * golden final image), so after both calls `image` is the golden final image
+ * either way. */
 fi_status fi_golden_lengths_jit(const fi_jit* j, const fi_program* p, uint8_t* image, uint64_t* warp_len,
                                 uint64_t* warp_nstore, uint32_t* dev_status, void* stream);
-fi_status fi_golden_trace_jit(const fi_jit* j, const fi_program* p, const uint8_t* image, const fi_trace* t,
+fi_status fi_golden_trace_jit(const fi_jit* j, const fi_program* p, uint8_t* image, const fi_trace* t,
                               uint32_t* dev_status, void* stream);
 /* fi_classify_batched with K8's per-launch re-execution on a module built with
  * FI_JIT_PAGE: same arguments, scratch and results (transient faults). */

@@ -69,6 +69,7 @@ struct Src {
 };
 
 constexpr int kJbcSlots = 4;                        // JBC_SLOTS of jit_prelude.cuh
+constexpr uint32_t kJitSliceLen = 0x100;            // internal modes bit: golden pass 1 = control slice
 
 struct Gen {
     uint32_t NR;                                      // register rows (fi_program.n_regs)
@@ -303,6 +304,8 @@ struct Gen {
 
     // LDG / STG.  `stepx` = this instruction's step.
     uint32_t mode = 0;                               // JM_INJ / JM_LEN / JM_TRACE of jit_prelude.cuh
+    std::vector<uint8_t> sl;                         // JM_LEN as the control slice: in-slice flag per pc (else empty)
+    bool skip(const fi_insn& I, uint32_t pc) const { return !sl.empty() && !sl[pc] && I.op != fi::BRA && I.op != fi::EXIT; }
     // buffer-cache entry (JBufCache slot) of each address register of the kernel being generated
     std::vector<int> slot_of = std::vector<int>(256, 0);
     int slot(const fi_insn& I) const { return slot_of[I.a & 0xFF]; }
@@ -328,6 +331,12 @@ struct Gen {
     void mem(Src& o, const fi_insn& I, uint32_t pc, const char* stepx) const {
         using namespace fi;
         const uint32_t lw = (I.mod & 3) > 2 ? 2 : (I.mod & 3), nw = 1u << lw;
+        if (skip(I, pc)) {                             // sliced length pass: count the stored words only
+            if (I.op == STG)
+                o("{ const bool pv = %s; const u32 exm_ = amask & __ballot_sync(JFULL, pv); nst += __popc(exm_) * %uu; }\n",
+                  guard(I.guard).c_str(), nw);
+            return;
+        }
         o("{ const bool pv = %s; const bool ex = inA && pv; ", guard(I.guard).c_str());
         rec(o, I, pc, stepx, "pv");
         o("const u64 va = %s + (u64)(i64)(i32)%s; ", R64(I.a).c_str(), hex(I.imm).c_str());
@@ -355,6 +364,15 @@ struct Gen {
                       R(I.b + 2).c_str(), R(I.b + 3).c_str());
                 o("} nst += __popc(exm_) * %uu; }\n", nw);
                 return;
+            }
+            if (mode == 2) {                           // golden pass 2: the stores into the image as well
+                o("if (ex && img_w) { u8* d_ = img_w + (va - JVA_BASE); ");
+                if (lw == 0) o("*reinterpret_cast<u32*>(d_) = %s; ", R(I.b).c_str());
+                else if (lw == 1) o("*reinterpret_cast<uint2*>(d_) = make_uint2(%s, %s); ", R(I.b).c_str(), R(I.b + 1).c_str());
+                else
+                    o("*reinterpret_cast<uint4*>(d_) = make_uint4(%s, %s, %s, %s); ", R(I.b).c_str(), R(I.b + 1).c_str(),
+                      R(I.b + 2).c_str(), R(I.b + 3).c_str());
+                o("} ");
             }
             o("const u32 sst_ = %s; if (%s) { if (ex) { const u32 idx_ = __popc(exm_ & lt_mask) * %uu; ",
               stepx, (mode == 2 || mode == 3) ? "true" : "sst_ > hstep", nw);
@@ -502,6 +520,49 @@ static std::vector<std::string> batch_strides(const Gen& G, const fi_insn* code,
     return st;
 }
 
+// The control slice of one static kernel (golden pass 1 as a length pass): the
+// instructions whose results can reach a BRA / EXIT / STG guard predicate — the
+// only things that decide the per-warp step count (min-pc scheduling, A.2) and
+// the stored-word count.  Flow-insensitive over registers: an instruction is in
+// the slice if it writes a GP register or predicate some slice instruction (or a
+// root guard) reads; reads are over-approximated like the liveness below (operand
+// fields a, a+1, c, c+1, b..b+3 unless b is an immediate; the guard; SEL's
+// predicate).  Everything else (FFMAs feeding only stores, loads feeding only
+// them) is skipped by the sliced pass: it cannot change the pc sequence or an
+// active / guard mask.
+std::vector<uint8_t> control_slice(const fi_insn* code, uint32_t n) {
+    using namespace fi;
+    std::vector<uint8_t> in(n, 0);
+    std::bitset<256> nr;
+    uint32_t np = 0;                                  // needed predicates (bits 0..6)
+    auto need_srcs = [&](const fi_insn& I) {
+        if ((I.guard & 7) != 7) np |= 1u << (I.guard & 7);
+        if (I.op == SEL && (I.c & 7) != 7) np |= 1u << (I.c & 7);
+        if (I.op == NOP || I.op == EXIT || I.op == BRA || I.op == S2R || I.op == LDC) return;
+        for (uint32_t r : {(uint32_t)I.a, I.a + 1u, (uint32_t)I.c, I.c + 1u}) if (r < kRZ) nr.set(r);
+        if (!(I.mod & 0x80)) for (uint32_t q = 0; q < 4; ++q) if (I.b + q < kRZ) nr.set(I.b + q);
+    };
+    for (uint32_t i = 0; i < n; ++i)
+        if ((code[i].op == BRA || code[i].op == EXIT || code[i].op == STG) && (code[i].guard & 7) != 7)
+            np |= 1u << (code[i].guard & 7);
+    for (bool ch = true; ch;) {
+        ch = false;
+        for (uint32_t i = 0; i < n; ++i) {
+            if (in[i]) continue;
+            const fi_insn& I = code[i];
+            if (I.op == BRA || I.op == EXIT || I.op == STG || I.op == NOP) continue;
+            const Dests d = dests_of(I.op, I.d0, I.d1, I.mod);
+            bool hit = d.has_pr && ((np >> d.pr) & 1u);
+            for (uint32_t q = 0; q < d.n_gp && !hit; ++q) hit = d.gp_base + q < 256 && nr[d.gp_base + q];
+            if (!hit) continue;
+            in[i] = 1;
+            need_srcs(I);
+            ch = true;
+        }
+    }
+    return in;
+}
+
 // Generate the device function of one static kernel (EMU_INJ mode).
 // Generate the device function of one static kernel in mode `mode` (JM_INJ,
 // JM_LEN, JM_TRACE); `blen`/leader tables are emitted once (with_tables).
@@ -513,10 +574,17 @@ const char* const kCtxNames[] = {"hstep", "hpc", "hlane", "hkind", "hreg", "hbfm
 // per lane in the context (JCtx arrays), not in registers
 const char* const kCtxLaneNames[] = {"nst", "fault", "fault_pc", "before", "after", "msk", "fired", "bad"};
 
-void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32_t n, uint32_t mode, bool with_tables) {
+void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32_t n, uint32_t mode, bool with_tables,
+                bool slice_len = false) {
     using namespace fi;
     Gen G = G0;
     G.mode = mode;
+    if (mode == 1 && slice_len) {
+        G.sl = control_slice(code, n);
+        o("__device__ const u8 kslice_%u[%u] = {", kid, n);
+        for (uint32_t i = 0; i < n; ++i) o("%u%s", G.sl[i], i + 1 < n ? "," : "");
+        o("};\n");
+    }
     // one cache entry per address register, in order of first use (wrapping beyond JBC_SLOTS)
     {
         std::vector<int> seen(256, -1);
@@ -574,7 +642,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
             if (I.op == BRA || I.op == EXIT) continue;
             Src t;
             if (I.op == LDG || I.op == STG) G.mem(t, I, i, "step");
-            else { t("{ const bool ex = true; "); G.plain(t, I); t("}"); }
+            else if (!G.skip(I, i)) { t("{ const bool ex = true; "); G.plain(t, I); t("}"); }
             const std::string& s = t.s;
             const bool uncond = G.guard(I.guard) == "true";
             for (size_t p = 0; p < s.size(); ++p) {
@@ -713,7 +781,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
             }
             continue;
         }
-        if (I.op == LDG) {
+        if (I.op == LDG && G.sl.empty()) {
             const uint32_t m = ldg_batch_len(code, n, i, leader);
             if (m >= 2) {
                 // the block holding the batch: from its leader L to its BRA / EXIT E
@@ -764,7 +832,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
         } else {
             if (I.op == LDG || I.op == STG) {
                 G.mem(o, I, i, stepx);
-            } else {
+            } else if (!G.skip(I, i)) {
                 o(" { const bool pv = %s; const bool ex = inA && pv; (void)pv; ", G.guard(I.guard).c_str());
                 G.rec(o, I, i, stepx, "pv");
                 G.plain(o, I);
@@ -791,9 +859,9 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "  __syncwarp();\n"
       "  JBufCache bcs_;                     // (step mode's own cache: bc's address never escapes, so it stays in registers)\n"
       "  const u32 done_ = jinterp<%u>(A, st_, bcs_, Rs, dec, kblen_%u, %uu, k, cta, wic, watchdog, hstep, hpc, hlane, "
-      "hkind, hreg, hbfm, hmask, st_out, st_cap, %uu, img_w, rec_out, ck, ck_interval, ins, pgp);\n"
+      "hkind, hreg, hbfm, hmask, st_out, st_cap, %uu, img_w, rec_out, ck, ck_interval, ins, pgp, %s);\n"
       "  __syncwarp();\n",
-      mode, kid, n, NR);
+      mode, kid, n, NR, G.sl.empty() ? "(const u8*)0" : ("kslice_" + std::to_string(kid)).c_str());
     for (uint32_t j = 0; j < NR; ++j) o("  R%u = Rs[%uu + lane];%s", j, j * 32, (j % 8 == 7) ? "\n" : "");
     o("\n  pc = st_.pc; live = st_.live; step = st_.step; livem = st_.livem; conv = st_.conv; upc = st_.upc; "
       "amask = st_.amask; npc = st_.npc; jx->nst_[lane] = st_.nst; jx->fault_[lane] = st_.fault; "
@@ -817,6 +885,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
 // that serve only it), or of every kernel (only < 0: fi_jit_source's combined view).
 std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern, uint32_t n_regs, uint32_t modes,
                      int only = -1) {
+    const bool slice_len = modes & kJitSliceLen;    // golden pass 1 as the control slice (fi_jit_build decides)
     // resident 128-thread CTAs per SM the register budget targets (3: <= 168 registers)
     uint32_t min_blocks = 3;
     if (const char* e = std::getenv("FI_JIT_MIN_BLOCKS")) min_blocks = (uint32_t)std::max(1, std::atoi(e));
@@ -830,7 +899,7 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
         bool tables = true;
         if (modes & FI_JIT_INJECT) { gen_kernel(o, G, k, code + kern[k].code_off, kern[k].code_len, 0, tables); tables = false; }
         if (modes & FI_JIT_GOLDEN) {
-            gen_kernel(o, G, k, code + kern[k].code_off, kern[k].code_len, 1, tables);
+            gen_kernel(o, G, k, code + kern[k].code_off, kern[k].code_len, 1, tables, slice_len);
             gen_kernel(o, G, k, code + kern[k].code_off, kern[k].code_len, 2, false);
             tables = false;
         }
@@ -927,7 +996,7 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
         // (one launch per instance k, like pass 1: each module serves its own kernel's instances)
         o("extern \"C\" __global__ void __launch_bounds__(128, %u) k_golden_trace_jit(const JArgs A, const u32 k, "
           "const u64* __restrict__ warp_off, const u64* __restrict__ gst_off, uint4* rec, jfi_store* gst, u32* ckpt, "
-          "const u64* __restrict__ ck_off, const u32 ck_interval, u32* status) {\n"
+          "const u64* __restrict__ ck_off, const u32 ck_interval, u32* status, u8* img_w) {\n"
           " extern __shared__ u32 jsmem[];\n const u32 lane = threadIdx.x & 31u;\n"
           " u32* Rs = jsmem + (threadIdx.x >> 5) * %uu;\n Rs[%uu + lane] = 0u;\n"
           " const jfi_instance in = A.inst[k];\n const u32 lw = blockIdx.x * 4u + (threadIdx.x >> 5);\n"
@@ -938,7 +1007,7 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
           min_blocks, rs, zrow, ckw);
         for (uint32_t k = 0; k < n_kern; ++k)
             if (mine(k)) o("  case %u: kern_%u_trace(A, 0xFFFFFFFFu, 0u, 0u, 0u, 0u, 0u, 0u, k, lw / wpc, lw %% wpc, 0xFFFFFFFFu, ck, "
-              "ck ? ck_interval : 0u, gst + g0, 0xFFFFFFFFu, o, Rs, A.dec + %uu, A.ins + %uu, (u8*)0, rec + r0, "
+              "ck ? ck_interval : 0u, gst + g0, 0xFFFFFFFFu, o, Rs, A.dec + %uu, A.ins + %uu, img_w, rec + r0, "
               "(const JPage*)0); break;\n",
               k, k, kern[k].code_off, kern[k].code_off);
         o("  default: o.steps = 0; o.fault = 9; o.nstore = 0; break;\n }\n"
@@ -1054,7 +1123,9 @@ extern "C" const char* fi_jit_log(void) { return g_jit_log.c_str(); }
 
 extern "C" size_t fi_jit_source(const fi_insn* code_host, uint32_t n_code, const fi_kernel* kern_host, uint32_t n_kern,
                                 uint32_t n_regs, uint32_t modes, char* buf, size_t buf_bytes) {
-    if (!code_host || !kern_host || !n_kern || n_regs == 0 || n_regs > fi::kRZ || !modes || modes > 7) return 0;
+    if (!code_host || !kern_host || !n_kern || n_regs == 0 || n_regs > fi::kRZ || !(modes & 7) ||
+        (modes & ~(7u | kJitSliceLen)))
+        return 0;
     for (uint32_t k = 0; k < n_kern; ++k)
         if ((uint64_t)kern_host[k].code_off + kern_host[k].code_len > n_code) return 0;
     const std::string s = generate(code_host, kern_host, n_kern, n_regs, modes);
@@ -1137,7 +1208,9 @@ fi_status compile_all(const fi_insn* code, const fi_kernel* kern, uint32_t n_ker
 
 extern "C" fi_status fi_jit_compile_check(const fi_insn* code_host, uint32_t n_code, const fi_kernel* kern_host,
                                           uint32_t n_kern, uint32_t n_regs, uint32_t modes, size_t* cubin_bytes) {
-    if (!code_host || !kern_host || !n_kern || n_regs == 0 || n_regs > fi::kRZ || !modes || modes > 7) return FI_E_ARG;
+    if (!code_host || !kern_host || !n_kern || n_regs == 0 || n_regs > fi::kRZ || !(modes & 7) ||
+        (modes & ~(7u | kJitSliceLen)))
+        return FI_E_ARG;
     if (!valid_kernels(kern_host, n_kern, n_code)) return FI_E_ARG;
     std::vector<std::vector<char>> cubins;
     size_t sb = 0;
@@ -1160,9 +1233,22 @@ extern "C" fi_status fi_jit_build(const fi_program* p, const fi_kernel* kern_hos
     const auto t0 = std::chrono::steady_clock::now();
     fi_status e0 = fi::cuda_status(cudaFree(0));       // bind the device's primary context to this thread
     if (e0) return e0;
+    // golden pass 1 as the control slice when its loads cannot see another launch's
+    // stores: a single-launch program, or no load in any kernel's slice (the sliced
+    // pass writes no image; pass 2 does, launch by launch)
+    bool slice = p->n_inst == 1;
+    if (!slice && p->inst_host) {
+        slice = true;
+        for (uint32_t k = 0; k < p->n_kern && slice; ++k) {
+            const fi_insn* c = p->code_host + kern_host[k].code_off;
+            const std::vector<uint8_t> sl = control_slice(c, kern_host[k].code_len);
+            for (uint32_t i = 0; i < kern_host[k].code_len && slice; ++i) slice = !(sl[i] && c[i].op == fi::LDG);
+        }
+    }
+    const uint32_t gen_modes = modes | ((slice && (modes & FI_JIT_GOLDEN)) ? kJitSliceLen : 0u);
     std::vector<std::vector<char>> cubins;
     size_t src_bytes = 0;
-    fi_status e = compile_all(p->code_host, kern_host, p->n_kern, p->n_regs, modes, cubins, src_bytes);
+    fi_status e = compile_all(p->code_host, kern_host, p->n_kern, p->n_regs, gen_modes, cubins, src_bytes);
     if (e) return e;
     fi_jit* j = new fi_jit();
     j->smem = jit_smem(p->n_regs);
@@ -1315,7 +1401,7 @@ extern "C" fi_status fi_golden_lengths_jit(const fi_jit* j, const fi_program* p,
     return FI_OK;
 }
 
-extern "C" fi_status fi_golden_trace_jit(const fi_jit* j, const fi_program* p, const uint8_t* image, const fi_trace* t,
+extern "C" fi_status fi_golden_trace_jit(const fi_jit* j, const fi_program* p, uint8_t* image, const fi_trace* t,
                                          uint32_t* dev_status, void* stream) {
     if (!j || !p || !image || !t || !t->warp_off || !t->gstore_off || !t->rec || !dev_status || !p->aux) return FI_E_ARG;
     if (!(j->modes & FI_JIT_GOLDEN) || j->n_regs != p->n_regs || j->n_code != p->n_code) return FI_E_ARG;
@@ -1335,7 +1421,7 @@ extern "C" fi_status fi_golden_trace_jit(const fi_jit* j, const fi_program* p, c
         if (!nw) continue;
         if (p->inst_host[k].kernel >= j->m.size()) return FI_E_ARG;
         uint32_t kk = k;
-        void* args[] = {&A, &kk, (void*)&woff, (void*)&goff, &rec, &gst, &ck, (void*)&ckoff, &iv, &dev_status};
+        void* args[] = {&A, &kk, (void*)&woff, (void*)&goff, &rec, &gst, &ck, (void*)&ckoff, &iv, &dev_status, &image};
         fi_status e = launch(j->m[p->inst_host[k].kernel].gtrace, (nw + 3) / 4, j->smem, (cudaStream_t)stream, args);
         if (e) return e;
     }

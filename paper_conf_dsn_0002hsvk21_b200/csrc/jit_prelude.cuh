@@ -253,8 +253,8 @@ struct JState {
     uint4 recbuf;                                    // golden trace pass: this lane's record of the 32-step window
 };
 #define JM_INJ 0                                     // injection replica (K4): hook, stores after the site logged
-#define JM_LEN 1                                     // golden pass 1: stores into the image, steps / stores counted
-#define JM_TRACE 2                                   // golden pass 2: trace records, store log, checkpoints
+#define JM_LEN 1                                     // golden pass 1: steps / stores counted (+ image stores unless sliced)
+#define JM_TRACE 2                                   // golden pass 2: trace records, store log, checkpoints, image stores
 
 __device__ __forceinline__ bool jguard(u32 guard, u32 preds) {
     const u32 gs = guard & 7;
@@ -478,7 +478,10 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
                                     const u32 hmask, jfi_store* __restrict__ st_out, const u32 st_cap,
                                     const u32 zr, u8* __restrict__ img_w, uint4* __restrict__ rec_out,
                                     u32* __restrict__ ck, const u32 ck_interval, const u32* __restrict__ ins,
-                                    const JPage* __restrict__ pg) {
+                                    const JPage* __restrict__ pg, const u8* __restrict__ slice) {
+    // slice (JM_LEN as the control slice, jit.cpp): 0 = the instruction cannot
+    // affect control flow or the store counts — only BRA / EXIT and STG counting
+    // run for it (no loads, no image stores)
     const u32 lane = threadIdx.x & 31, lt_mask = (1u << lane) - 1u;
     const JRegs F{reinterpret_cast<char*>(R + lane), R, zr * 128};
     const jfi_instance in = A.inst[k];
@@ -524,7 +527,9 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
         if (MODE == JM_TRACE && lane == 0)            // one trace record per step (App. A.3)
             rec_out[step] = make_uint4(k, __ldg(&ins[pcm]), active, pred);
         u32 taken = 0;
-        if (op == 1) {                                // EXIT
+        if (MODE == JM_LEN && slice && !slice[pcm] && op != 1 && op != 2) {
+            if (op == 23) nst += __popc(exm) * (1u << ((mod & 3) > 2 ? 2 : (mod & 3)));
+        } else if (op == 1) {                         // EXIT
             if (ex) live = false;
             livem &= ~exm;
             amask &= ~exm;
@@ -563,6 +568,12 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
                 u32 v[4];
 #pragma unroll
                 for (int i = 0; i < 4; ++i) v[i] = (u32)i < nw ? F.rd(min(ib + 128u * i, F.zb)) : 0u;
+                if (MODE == JM_TRACE && img_w && ex) {   // golden pass 2: stores go to the image too
+                    u8* dst = img_w + (va - JVA_BASE);
+                    if (lw == 0) *reinterpret_cast<u32*>(dst) = v[0];
+                    else if (lw == 1) *reinterpret_cast<uint2*>(dst) = make_uint2(v[0], v[1]);
+                    else *reinterpret_cast<uint4*>(dst) = make_uint4(v[0], v[1], v[2], v[3]);
+                }
                 if (MODE == JM_LEN) {                 // golden pass 1: stores go to the image
                     if (ex) {
                         u8* dst = img_w + (va - JVA_BASE);

@@ -38,13 +38,17 @@ def single(fi, prog, n, groups, engine, multi=False):
     hist_tol = torch.zeros((8, 4, 3), dtype=torch.int64, device=dp.device)
     fi.classify(gt, sites, n, out, log, cap, rtol=1e-6, hist_tol=hist_tol)
     if multi:
-        fi.classify_batched(gt, sites, n, out2, log, cap, engine=engine, rtol=1e-6, hist_tol=hist_tol)
+        fi.classify_batched(gt, sites, n, out2, log, cap, engine=engine, rtol=1e-6, hist_tol=hist_tol,
+                            mem_budget=1 << 30)
         pf = np.zeros(4, dtype=fi.PFAULT_DTYPE)
         pf["opcode"], pf["sm"], pf["lane"], pf["mask"], pf["n_sm"] = 16, [0, 1, 2, 3], [1, 5, 9, 30], 1 << 22, 4
         fi.inject_permanent(gt, pf)
-        fi.inject_permanent_batched(gt, pf)
+        fi.inject_permanent_batched(gt, pf, mem_budget=1 << 30)
     torch.cuda.synchronize()
-    return fi.as_numpy(out, fi.INJ_DTYPE, n)["outcome"]
+    r = fi.as_numpy(out, fi.INJ_DTYPE, n)["outcome"]
+    del gt, dp, out, out2, log, sites, idx, iidx
+    torch.cuda.empty_cache()
+    return r
 
 
 def _peer(rank, world, port):
