@@ -19,9 +19,12 @@
 //  * FFMA (the dominant opcode of GEMM-like kernels) has its own fast path;
 //  * each lane caches its last two buffers' bounds, so most LDG/STG skip the
 //    granule-table lookup;
-//  * the golden trace pass stores a register-file checkpoint every
-//    `interval` steps, and an injection replica restarts from the checkpoint at
-//    or before its site instead of re-executing the whole prefix (the prefix is
+//  * the golden trace pass stores register-file checkpoints: checkpoint c is the
+//    warp state before the first step s >= c*interval that follows a BRA or EXIT
+//    (or s = 0), its step s stored with it (absent: 0xFFFFFFFF), so no engine
+//    has to stop a straight-line block at a multiple of the interval; an
+//    injection replica restarts from the last checkpoint whose step is at or
+//    before its site instead of re-executing the whole prefix (the prefix is
 //    identical to the golden run by construction).
 //
 // Memory follows DESIGN.md §3.5: loads of instance k read the golden final
@@ -119,7 +122,8 @@ inline EmuProg make_emu_prog(const fi_program* p) {
 }
 
 // checkpoint = (n_regs + 3) rows of 32 words: registers, then pc, predicates, live
-__host__ __device__ inline size_t ckpt_bytes(uint32_t n_regs) { return (size_t)(n_regs + 3) * 128; }
+// rows: n_regs registers, pc, predicates, live, step (all lanes hold the step)
+__host__ __device__ inline size_t ckpt_bytes(uint32_t n_regs) { return (size_t)(n_regs + 4) * 128; }
 
 struct HookIn {
     uint32_t step, lane, kind, reg, bfm, mask, pc;   // transient site (EMU_INJ)
@@ -133,6 +137,7 @@ struct HookIn {
 
 struct EmuOut {
     uint32_t steps = 0, fault = 0, fault_pc = 0, nstore = 0;
+    uint32_t start = 0;                              // EMU_INJ: the step it restarted at (checkpoint)
     uint32_t before = 0, after = 0, mask = 0;
     bool fired = false, bad = false;
 };
@@ -476,7 +481,7 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
     const uint32_t* __restrict__ ins = P.ins + kn.code_off;
     const uint32_t* __restrict__ runl = P.run + kn.code_off;
     const uint32_t zr = P.n_regs;
-    const uint32_t ckw = (zr + 3) * 32;              // words per checkpoint
+    const uint32_t ckw = (zr + 4) * 32;              // words per checkpoint
     const RegFile F{reinterpret_cast<char*>(R + lane), R, zr * 128};
     const LaneCtx LC{lane, cta, wic, in.block, in.grid, in.cbank_len, P.cbank + in.cbank_off};
     const bool use_ck = ck != nullptr && ck_interval != 0;
@@ -487,16 +492,19 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
     uint32_t nl = in.block - wic * 32;
     bool live = lane < (nl > 32 ? 32u : nl);
     uint32_t pc = 0, preds = 0, step = 0;
+    EmuOut o;
     if (MODE == EMU_INJ && use_ck) {
-        // restart from the golden checkpoint at or before the site
-        const uint32_t c = hook.step / ck_interval;
+        // restart from the last golden checkpoint at or before the site
+        uint32_t c = hook.step / ck_interval;
+        while (c > 0 && __ldg(&ck[(size_t)c * ckw + (zr + 3) * 32]) > hook.step) --c;
         const uint32_t* src = ck + (size_t)c * ckw;
         for (uint32_t r = 0; r < zr; ++r) R[r * 32 + lane] = __ldg(&src[r * 32 + lane]);
         R[zr * 32 + lane] = 0u;
         pc = __ldg(&src[zr * 32 + lane]);
         preds = __ldg(&src[zr * 32 + 32 + lane]);
         live = __ldg(&src[zr * 32 + 64 + lane]) != 0u;
-        step = c * ck_interval;
+        step = __ldg(&src[(zr + 3) * 32 + lane]);
+        o.start = step;
     } else {
         for (uint32_t r = 0; r <= zr; ++r) R[r * 32 + lane] = 0u;
     }
@@ -507,8 +515,9 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
     // divergently, exits, or reaches npc (where parked lanes rejoin).
     bool conv = false;
     uint32_t upc = 0, amask = 0, npc = 0xFFFFFFFFu;
-    EmuOut o;
     uint32_t nst = 0;
+    bool brk = true;                                 // the last step was a BRA / EXIT (or none yet)
+    uint32_t ckn = 0;                                // EMU_TRACE: next checkpoint to write
     uint4 recbuf = make_uint4(0, 0, 0, 0);
     BufCache bc;
     __syncwarp();
@@ -526,13 +535,18 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
             conv = true; upc = pcm; amask = active;
         }
         const bool inA = (amask >> lane) & 1u;
-        if (MODE == EMU_TRACE && use_ck && (step % ck_interval) == 0) {
-            uint32_t* dst = ck + (size_t)(step / ck_interval) * ckw;
-            for (uint32_t r = 0; r < zr; ++r) dst[r * 32 + lane] = R[r * 32 + lane];
-            dst[zr * 32 + lane] = live ? (inA ? upc : pc) : 0u;
-            dst[zr * 32 + 32 + lane] = preds;
-            dst[zr * 32 + 64 + lane] = live ? 1u : 0u;
+        if (MODE == EMU_TRACE && use_ck && brk && step >= ckn * ck_interval) {
+            // checkpoints ckn .. step/interval: this state (one per multiple passed)
+            for (; ckn <= step / ck_interval; ++ckn) {
+                uint32_t* dst = ck + (size_t)ckn * ckw;
+                for (uint32_t r = 0; r < zr; ++r) dst[r * 32 + lane] = R[r * 32 + lane];
+                dst[zr * 32 + lane] = live ? (inA ? upc : pc) : 0u;
+                dst[zr * 32 + 32 + lane] = preds;
+                dst[zr * 32 + 64 + lane] = live ? 1u : 0u;
+                dst[(zr + 3) * 32 + lane] = step;
+            }
         }
+        brk = false;
         if (step >= watchdog) { o.fault = 3; o.fault_pc = pcm; break; }
         if (pcm >= kn.code_len) { o.fault = 4; o.fault_pc = pcm; break; }
 
@@ -541,7 +555,6 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
             const uint32_t rw = __ldg(&runl[pcm]);
             uint32_t run = rw & 0xFFFF, lr = (rw >> 16) & 0xFF, fr = rw >> 24;
             uint32_t lim = min(watchdog - step, npc - pcm);   // stop where parked lanes rejoin
-            if (MODE == EMU_TRACE && use_ck) lim = min(lim, ck_interval - step % ck_interval);
             if (MODE == EMU_INJ && hook.step >= step) lim = min(lim, hook.step - step);
             run = min(run, lim);
             lr = min(min(lr, lim), (uint32_t)kLdgBatch);
@@ -719,6 +732,7 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
         }
 
         uint32_t taken = 0;                           // lanes that branch
+        brk = op == EXIT || op == BRA;
         if (op == EXIT) {
             if (ex) live = false;
             livem &= ~exm;
@@ -845,6 +859,8 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
     if (MODE == EMU_TRACE) {
         const uint32_t rem = step & 31;
         if (rem && lane < rem) reinterpret_cast<uint4*>(rec_out)[step - rem + lane] = recbuf;
+        if (use_ck)                                   // checkpoints the warp never reached: absent
+            for (; ckn < (step + ck_interval - 1) / ck_interval; ++ckn) ck[(size_t)ckn * ckw + (zr + 3) * 32 + lane] = ~0u;
     }
     o.steps = step;
     o.nstore = nst;

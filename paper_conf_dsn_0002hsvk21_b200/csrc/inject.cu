@@ -139,8 +139,7 @@ k_inject(EmuProg P, const uint8_t* img, const uint64_t* __restrict__ warp_off, c
         r.n_faulty_stores = o.nstore;
         out[i] = r;
         if (!o.fired || o.bad) FI_DEV_ERR(status, FI_E_SITE);
-        const uint32_t start = (ckpt && ck_interval) ? S.step / ck_interval * ck_interval : 0u;
-        atomicAdd(reinterpret_cast<unsigned long long*>(counter + 2), (unsigned long long)(o.steps - start));
+        atomicAdd(reinterpret_cast<unsigned long long*>(counter + 2), (unsigned long long)(o.steps - o.start));
     }
     __syncwarp();
     }

@@ -715,37 +715,45 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
     o("\nconst u32 nl_ = in.block - wic * 32u; bool live = lane < (nl_ > 32u ? 32u : nl_);\n");
     o("u32 pc = 0u, step = 0u; bool Q0 = false, Q1 = false, Q2 = false, Q3 = false, Q4 = false, Q5 = false, "
       "Q6 = false;\n");
-    o("if (%s) {\n  const u32 c_ = hstep / ck_interval; const u32* __restrict__ src = ck + (u64)c_ * %uu;\n",
-      mode == 0 ? "ck" : "false", (NR + 3) * 32);
+    o("if (%s) {\n  u32 c_ = hstep / ck_interval;\n"
+      "  while (c_ > 0u && __ldg(&ck[(u64)c_ * %uu + %uu]) > hstep) --c_;   // the last checkpoint at or before the site\n"
+      "  const u32* __restrict__ src = ck + (u64)c_ * %uu;\n",
+      mode == 0 ? "ck" : "false", (NR + 4) * 32, (NR + 3) * 32, (NR + 4) * 32);
     for (uint32_t j = 0; j < NR; ++j) o("  R%u = __ldg(&src[%uu + lane]);\n", j, j * 32);
     o("  pc = __ldg(&src[%uu + lane]); const u32 pw_ = __ldg(&src[%uu + lane]); live = __ldg(&src[%uu + lane]) != 0u; "
-      "step = c_ * ck_interval;\n  Q0 = pw_ & 1u; Q1 = (pw_ >> 1) & 1u; Q2 = (pw_ >> 2) & 1u; Q3 = (pw_ >> 3) & 1u; "
+      "step = __ldg(&src[%uu + lane]); out_p.start = step;\n  Q0 = pw_ & 1u; Q1 = (pw_ >> 1) & 1u; Q2 = (pw_ >> 2) & 1u; Q3 = (pw_ >> 3) & 1u; "
       "Q4 = (pw_ >> 4) & 1u; Q5 = (pw_ >> 5) & 1u; Q6 = (pw_ >> 6) & 1u;\n} else {\n",
-      NR * 32, NR * 32 + 32, NR * 32 + 64);
+      NR * 32, NR * 32 + 32, NR * 32 + 64, NR * 32 + 96);
     for (uint32_t j = 0; j < NR; ++j) o("R%u = 0u;%s", j, (j % 16 == 15) ? "\n" : " ");
     o("\n}\n");
     o("u32 livem = __ballot_sync(JFULL, live);\nbool conv = false; u32 upc = 0u, amask = 0u, npc = 0xFFFFFFFFu;\n"
       "jx->nst_[lane] = 0u; jx->fault_[lane] = 0u; jx->fault_pc_[lane] = 0u; jx->before_[lane] = 0u; "
       "jx->after_[lane] = 0u; jx->msk_[lane] = 0u; jx->fired_[lane] = 0u; jx->bad_[lane] = 0u;\n"
       "JBufCache bc; uint4 recbuf = make_uint4(0u, 0u, 0u, 0u); (void)recbuf;\n"
+      "// golden trace pass: the last step was a BRA / EXIT; next checkpoint and its threshold step\n"
+      "u32 brk = 1u, ckn = 0u, ckx = %s; (void)brk; (void)ckn; (void)ckx;\n"
       "// blocks run only within [step, lim): lim = the watchdog, or the injection step while it is pending,\n"
       "// or the next checkpoint step (golden trace pass)\n"
-      "u32 lim = %s;\n", mode == 0 ? "(hstep >= step && hstep < watchdog) ? hstep : watchdog" : "watchdog");
+      "u32 lim = %s;\n", mode == 2 ? "ck ? 0u : 0xFFFFFFFFu" : "0xFFFFFFFFu",
+      mode == 0 ? "(hstep >= step && hstep < watchdog) ? hstep : watchdog" : "watchdog");
     o("for (;;) {\n if (!livem) break;\n u32 pcm, active;\n"
       " if (conv) { pcm = upc; active = amask; }\n"
       " else { pcm = __reduce_min_sync(JFULL, live ? pc : 0xFFFFFFFFu); active = __ballot_sync(JFULL, live && pc == pcm);\n"
       "   npc = active == livem ? 0xFFFFFFFFu : __reduce_min_sync(JFULL, (live && pc != pcm) ? pc : 0xFFFFFFFFu);\n"
       "   conv = true; upc = pcm; amask = active; }\n"
       " const bool inA = (amask >> lane) & 1u;\n");
-    if (mode == 2) {                                  // golden checkpoint every ck_interval steps (from registers)
-        o(" if (ck) {\n  if (step %% ck_interval == 0u) {\n   u32* dst_ = ck + (u64)(step / ck_interval) * %uu;\n",
-          (NR + 3) * 32);
+    if (mode == 2) {
+        // golden checkpoints (emu.cuh): the state before the first step at or past
+        // each multiple of ck_interval that follows a BRA / EXIT — every arrival here
+        // from block code is such a step, so blocks never stop at a multiple
+        o(" if (brk && step >= ckx) {\n  for (; ckn <= step / ck_interval; ++ckn) {\n"
+          "   u32* dst_ = ck + (u64)ckn * %uu;\n", (NR + 4) * 32);
         for (uint32_t j = 0; j < NR; ++j) o("   dst_[%uu + lane] = R%u;%s", j * 32, j, (j % 8 == 7) ? "\n" : "");
         o("\n   dst_[%uu + lane] = live ? (inA ? upc : pc) : 0u;\n"
           "   dst_[%uu + lane] = (u32)Q0 | ((u32)Q1 << 1) | ((u32)Q2 << 2) | ((u32)Q3 << 3) | ((u32)Q4 << 4) | "
-          "((u32)Q5 << 5) | ((u32)Q6 << 6);\n   dst_[%uu + lane] = live ? 1u : 0u;\n  }\n"
-          "  lim = min(watchdog, (step / ck_interval + 1u) * ck_interval);\n }\n",
-          NR * 32, NR * 32 + 32, NR * 32 + 64);
+          "((u32)Q5 << 5) | ((u32)Q6 << 6);\n   dst_[%uu + lane] = live ? 1u : 0u;\n   dst_[%uu + lane] = step;\n  }\n"
+          "  ckx = ckn * ck_interval;\n }\n",
+          NR * 32, NR * 32 + 32, NR * 32 + 64, NR * 32 + 96);
     }
     o(" if (step >= watchdog) { fault = 3u; fault_pc = pcm; break; }\n"
       " if (pcm >= %uu) { fault = 4u; fault_pc = pcm; break; }\n",
@@ -805,10 +813,11 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
             auto chain = [&](uint32_t L) -> std::string {
                 if (L >= n || !leader[L]) return "";
                 char b[256];
-                std::snprintf(b, sizeof b, "if (%uu <= npc && step + %uu <= lim) { pcm = %uu; ", L + blen[L], blen[L], L);
+                std::snprintf(b, sizeof b, "if (%uu <= npc && step + %uu <= lim%s) { pcm = %uu; ", L + blen[L], blen[L],
+                              mode == 2 ? " && step < ckx" : "", L);
                 return b + entry_kills(L) + "goto B" + std::to_string(L) + "; } ";
             };
-            o(" { const bool pv = %s; ", G.guard(I.guard).c_str());
+            o(" { const bool pv = %s; %s", G.guard(I.guard).c_str(), mode == 2 ? "brk = 1u; " : "");
             G.rec(o, I, i, stepx, "pv");
             G.flush_recs(o, code, run_start(i), i);
             const RSet keep_ft = use_kill ? lfrom[i + 1] : RSet();
@@ -821,7 +830,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
               i + 1, chain(i + 1).c_str(), kills(keep_ft).c_str(), i + 1, chain(I.imm).c_str(),
               kills(keep_tk).c_str(), I.imm, kills(keep_tk).c_str(), I.imm, i + 1);
         } else if (I.op == EXIT) {
-            o(" { const bool pv = %s; ", G.guard(I.guard).c_str());
+            o(" { const bool pv = %s; %s", G.guard(I.guard).c_str(), mode == 2 ? "brk = 1u; " : "");
             G.rec(o, I, i, stepx, "pv");
             G.flush_recs(o, code, run_start(i), i);
             o("const u32 exm_ = amask & __ballot_sync(JFULL, pv); step += %uu - pcm;\n"
@@ -855,7 +864,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "st_.fault_pc = jx->fault_pc_[lane]; st_.before = jx->before_[lane]; st_.after = jx->after_[lane]; "
       "st_.msk = jx->msk_[lane]; st_.fired = jx->fired_[lane]; st_.bad = jx->bad_[lane]; st_.lim = lim;\n"
       "  st_.preds = (u32)Q0 | ((u32)Q1 << 1) | ((u32)Q2 << 2) | ((u32)Q3 << 3) | ((u32)Q4 << 4) | ((u32)Q5 << 5) | "
-      "((u32)Q6 << 6); st_.recbuf = recbuf;\n"
+      "((u32)Q6 << 6); st_.recbuf = recbuf; st_.brk = brk; st_.ckn = ckn;\n"
       "  __syncwarp();\n"
       "  JBufCache bcs_;                     // (step mode's own cache: bc's address never escapes, so it stays in registers)\n"
       "  const u32 done_ = jinterp<%u>(A, st_, bcs_, Rs, dec, kblen_%u, %uu, k, cta, wic, watchdog, hstep, hpc, hlane, "
@@ -867,11 +876,14 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "amask = st_.amask; npc = st_.npc; jx->nst_[lane] = st_.nst; jx->fault_[lane] = st_.fault; "
       "jx->fault_pc_[lane] = st_.fault_pc; jx->before_[lane] = st_.before; jx->after_[lane] = st_.after; "
       "jx->msk_[lane] = st_.msk; jx->fired_[lane] = st_.fired; jx->bad_[lane] = st_.bad; lim = st_.lim; "
-      "recbuf = st_.recbuf;\n"
+      "recbuf = st_.recbuf; brk = st_.brk; ckn = st_.ckn; if (ck) ckx = ckn * ck_interval;\n"
       "  Q0 = st_.preds & 1u; Q1 = (st_.preds >> 1) & 1u; Q2 = (st_.preds >> 2) & 1u; Q3 = (st_.preds >> 3) & 1u; "
       "Q4 = (st_.preds >> 4) & 1u; Q5 = (st_.preds >> 5) & 1u; Q6 = (st_.preds >> 6) & 1u;\n"
       "  if (done_) goto finish;\n  continue;\n }\n}\n");
     o("finish:\n");
+    if (mode == 2)                                    // checkpoints the warp never reached: absent
+        o(" if (ck) for (; ckn < (step + ck_interval - 1u) / ck_interval; ++ckn) ck[(u64)ckn * %uu + %uu + lane] = 0xFFFFFFFFu;\n",
+          (NR + 4) * 32, (NR + 3) * 32);
     o("#undef out\n");
     o(" { JOut& out_ = *jx->out; out_.steps = step; out_.fault = jx->fault_[lane]; out_.fault_pc = jx->fault_pc_[lane]; "
       "out_.nstore = jx->nst_[lane];\n"
@@ -905,7 +917,7 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
         }
         if (modes & FI_JIT_PAGE) gen_kernel(o, G, k, code + kern[k].code_off, kern[k].code_len, 3, tables);
     }
-    const uint32_t rs = (n_regs + 1) * 32, zrow = n_regs * 32, ckw = (n_regs + 3) * 32;
+    const uint32_t rs = (n_regs + 1) * 32, zrow = n_regs * 32, ckw = (n_regs + 4) * 32;
     if (modes & FI_JIT_INJECT) {
     // K4 on the generated kernels: persistent warps over the LPT-ordered replicas
     // (same scheduling and outputs as inject.cu's k_inject)
@@ -927,7 +939,7 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
       "  const u64 L = warp_off[S.warp + 1] - warp_off[S.warp]; const u64 wd = 10ull * L + 1024ull;\n"
       "  const u32 watchdog = wd > 0xFFFFFFFFull ? 0xFFFFFFFFu : (u32)wd;\n"
       "  u32* ck = ckpt ? (u32*)ckpt + ck_off[S.warp] * %uull : (u32*)0;\n"
-      "  JOut o;\n  switch (in.kernel) {\n",
+      "  JOut o; o.start = 0u;\n  switch (in.kernel) {\n",
       rs, zrow, only <= 0 ? "true" : "false", only < 0 ? "false" : ("in.kernel != " + std::to_string(only) + "u").c_str(),
       ckw);
     for (uint32_t k = 0; k < n_kern; ++k)
@@ -940,8 +952,7 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
       "  if (lane == 0u) {\n   jfi_inj r; r.before = o.before; r.after = o.after; r.mask = o.mask; r.fault_pc = o.fault_pc;\n"
       "   r.fault_kind = (u8)o.fault; r.outcome = 0; r.overflow = o.nstore > cap; r.flags = 0; r.n_faulty_stores = o.nstore;\n"
       "   out[i] = r;\n   if (!o.fired || o.bad) atomicOr(status, 1u << 6);\n"
-      "   const u32 start = ck ? S.step / ck_interval * ck_interval : 0u;\n"
-      "   atomicAdd((unsigned long long*)(counter + 2), (unsigned long long)(o.steps - start));\n  }\n  __syncwarp();\n }\n}\n");
+      "   atomicAdd((unsigned long long*)(counter + 2), (unsigned long long)(o.steps - o.start));\n  }\n  __syncwarp();\n }\n}\n");
     }
     if (modes & FI_JIT_PAGE) {
         // K8's re-execution of instance t (propagate8.cu k8_exec) on the generated kernels
@@ -1143,8 +1154,17 @@ fi_status compile_cubin(const fi_insn* code, const fi_kernel* kern, uint32_t n_k
     Nvrtc& N = nvrtc();
     if (!N.ok) { g_jit_log = "libnvrtc.so.12 not found"; return FI_E_CUDA; }
     src = generate(code, kern, n_kern, n_regs, modes, only);
+    // FI_JIT_DUMP=<p> (profiling aid): the module's source and cubin are written to
+    // <p>[_k<kernel>].cu / .cubin, and the program is NAMED by that path, so the line
+    // table of the -lineinfo cubin points at a file that exists (ncu --import-source)
+    std::string dump;
+    if (const char* d = std::getenv("FI_JIT_DUMP"))
+        dump = std::string(d) + (only > 0 ? "_k" + std::to_string(only) : std::string());
+    if (!dump.empty())
+        if (FILE* f = std::fopen((dump + ".cu").c_str(), "wb")) { std::fwrite(src.data(), 1, src.size(), f); std::fclose(f); }
+    const std::string pname = dump.empty() ? std::string("fi_jit.cu") : dump + ".cu";
     void* prog = nullptr;
-    if (N.create(&prog, src.c_str(), "fi_jit.cu", 0, nullptr, nullptr)) { g_jit_log = "nvrtcCreateProgram failed"; return FI_E_CUDA; }
+    if (N.create(&prog, src.c_str(), pname.c_str(), 0, nullptr, nullptr)) { g_jit_log = "nvrtcCreateProgram failed"; return FI_E_CUDA; }
     std::vector<const char*> opts = {"--gpu-architecture=sm_100a", "--std=c++17", "--fmad=false", "-lineinfo"};
     std::string extra;                                // experiments: one more NVRTC option
     if (const char* e = std::getenv("FI_JIT_NVRTC_OPT")) if (*e) { extra = e; opts.push_back(extra.c_str()); }
@@ -1160,11 +1180,8 @@ fi_status compile_cubin(const fi_insn* code, const fi_kernel* kern, uint32_t n_k
     cubin.resize(cs);
     N.cubin(prog, cubin.data());
     N.destroy(&prog);
-    if (const char* d = std::getenv("FI_JIT_DUMP")) {     // profiling aid: the module's source and cubin
-        const std::string b = std::string(d) + (only > 0 ? "_k" + std::to_string(only) : std::string());
-        if (FILE* f = std::fopen((b + ".cu").c_str(), "wb")) { std::fwrite(src.data(), 1, src.size(), f); std::fclose(f); }
-        if (FILE* f = std::fopen((b + ".cubin").c_str(), "wb")) { std::fwrite(cubin.data(), 1, cubin.size(), f); std::fclose(f); }
-    }
+    if (!dump.empty())
+        if (FILE* f = std::fopen((dump + ".cubin").c_str(), "wb")) { std::fwrite(cubin.data(), 1, cubin.size(), f); std::fclose(f); }
     return FI_OK;
 }
 

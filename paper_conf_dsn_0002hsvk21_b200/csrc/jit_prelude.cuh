@@ -47,6 +47,7 @@ struct JArgs {
 
 struct JOut {
     u32 steps, fault, fault_pc, nstore, before, after, mask;
+    u32 start;                                       // K4: the step it restarted at (its checkpoint's)
     bool fired, bad;
 };
 // a generated kern_*'s arguments, per warp in shared memory after the 4 warps'
@@ -250,6 +251,7 @@ __device__ __forceinline__ u32 jldg(const JArgs& A, const u8* __restrict__ img, 
 // or faults.  Same semantics as emu.cuh's general step.
 struct JState {
     u32 pc, live, step, livem, conv, upc, amask, npc, nst, fault, fault_pc, before, after, msk, fired, bad, lim, preds;
+    u32 brk, ckn;                                    // last step was BRA / EXIT; next golden checkpoint (JM_TRACE)
     uint4 recbuf;                                    // golden trace pass: this lane's record of the 32-step window
 };
 #define JM_INJ 0                                     // injection replica (K4): hook, stores after the site logged
@@ -488,7 +490,7 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
     const u32* cb = A.cbank + in.cbank_off;
     bool live = S.live != 0, conv = S.conv != 0;
     u32 pc = S.pc, step = S.step, livem = S.livem, upc = S.upc, amask = S.amask, npc = S.npc, nst = S.nst;
-    u32 preds = S.preds, lim = S.lim;
+    u32 preds = S.preds, lim = S.lim, brk = S.brk, ckn = S.ckn;
     uint4 recbuf = S.recbuf;
     u32 done = 0;
     for (;;) {
@@ -501,16 +503,18 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
             npc = active == livem ? 0xFFFFFFFFu : __reduce_min_sync(JFULL, (live && pc != pcm) ? pc : 0xFFFFFFFFu);
             conv = true; upc = pcm; amask = active;
         }
-        if (MODE == JM_TRACE && ck) {                 // golden register-file checkpoint every ck_interval steps
-            if (step % ck_interval == 0) {
-                const bool inA = (amask >> lane) & 1u;
-                u32* dst = ck + (u64)(step / ck_interval) * (zr + 3) * 32;
+        if (MODE == JM_TRACE && ck && brk && step >= ckn * ck_interval) {
+            // golden checkpoints ckn .. step/interval (emu.cuh): the state before the
+            // first step at or past the multiple that follows a BRA / EXIT
+            const bool inA = (amask >> lane) & 1u;
+            for (; ckn <= step / ck_interval; ++ckn) {
+                u32* dst = ck + (u64)ckn * (zr + 4) * 32;
                 for (u32 r = 0; r < zr; ++r) dst[r * 32 + lane] = R[r * 32 + lane];
                 dst[zr * 32 + lane] = live ? (inA ? upc : pc) : 0u;
                 dst[zr * 32 + 32 + lane] = preds;
                 dst[zr * 32 + 64 + lane] = live ? 1u : 0u;
+                dst[zr * 32 + 96 + lane] = step;
             }
-            lim = min(watchdog, (step / ck_interval + 1) * ck_interval);
         }
         if (step >= watchdog) { S.fault = 3; S.fault_pc = pcm; done = 1; break; }
         if (pcm >= code_len) { S.fault = 4; S.fault_pc = pcm; done = 1; break; }
@@ -527,6 +531,7 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
         if (MODE == JM_TRACE && lane == 0)            // one trace record per step (App. A.3)
             rec_out[step] = make_uint4(k, __ldg(&ins[pcm]), active, pred);
         u32 taken = 0;
+        brk = op == 1 || op == 2;
         if (MODE == JM_LEN && slice && !slice[pcm] && op != 1 && op != 2) {
             if (op == 23) nst += __popc(exm) * (1u << ((mod & 3) > 2 ? 2 : (mod & 3)));
         } else if (op == 1) {                         // EXIT
@@ -628,7 +633,7 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
         if (MODE == JM_INJ && step > hstep) lim = watchdog;
     }
     S.pc = pc; S.live = live; S.step = step; S.livem = livem; S.conv = conv; S.upc = upc; S.amask = amask;
-    S.npc = npc; S.nst = nst; S.preds = preds; S.lim = lim; S.recbuf = recbuf;
+    S.npc = npc; S.nst = nst; S.preds = preds; S.lim = lim; S.recbuf = recbuf; S.brk = brk; S.ckn = ckn;
     return done;
 }
 
