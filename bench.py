@@ -375,6 +375,8 @@ def main():
         "gpu_launches": 10 * K,
     }
 
+    if world == 1:
+        line["shard_ratio"] = shard_ratio(camp, n)
     if camp.peers is not None:
         camp.peers.close()
     if not args.no_e2e:
@@ -387,6 +389,38 @@ def main():
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
+
+
+def shard_ratio(camp, n, G=8, reps=3):
+    """North star "near-linear 8-GPU speedup in injections/sec", checked on one GPU:
+    the injection stage (select + K4 + K5) of each rank's replica block
+    [r*n/G, (r+1)*n/G) timed alone (CUDA events, best of `reps`), against the whole
+    set.  The G-GPU stage time is the slowest block; ideal ratio = G."""
+    import torch
+    from paper_conf_dsn_0002hsvk21_b200 import fi
+    from paper_conf_dsn_0002hsvk21_b200.campaign import replica_block
+    idx = fi.SiteIndex(camp.gt, camp.inst_counts, camp.chunk_counts, camp.status)
+
+    def stage(j0, m):
+        best = None
+        for _ in range(reps):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            fi.select_sites(idx, camp.sched, j0, m, camp.sites, camp.status)
+            fi.inject(camp.gt, camp.sites, m, camp.cap, camp.out, camp.log, camp.status, camp.inj_ws, engine="jit")
+            h = torch.zeros((8, 4, 3), dtype=torch.int64, device=camp.device)
+            fi.classify(camp.gt, camp.sites, m, camp.out, camp.log, camp.cap, h, camp.status)
+            b.record()
+            torch.cuda.synchronize()
+            best = a.elapsed_time(b) if best is None else min(best, a.elapsed_time(b))
+        return best
+    blocks = [stage(*(lambda j: (j[0], j[1] - j[0]))(replica_block(n, r, G))) for r in range(G)]
+    full = stage(0, n)                                # last: camp.sites / out hold the whole set again
+    camp.check()
+    return {"G": G, "full_ms": full, "block_ms": blocks, "slowest_block_ms": max(blocks),
+            "ratio": full / max(blocks), "ideal": G,
+            "what": "injection stage (select + K4 + K5) of one rank's replica block [r*n/G,(r+1)*n/G) alone vs all n "
+                    "replicas, one GPU, best of 3: the G-GPU injections/s speedup bound"}
 
 
 def secondary_c4(dev, n=256):
@@ -449,7 +483,19 @@ def e2e(args, prog, seed, groups, bfms, n, rank, world, dev, camp):
     from paper_conf_dsn_0002hsvk21_b200.campaign import allreduce_max
     host = {k: torch.from_numpy(np.ascontiguousarray(getattr(prog, k)).view(np.uint8).reshape(-1).copy()).pin_memory()
             for k in ("code", "kernels", "instances", "cbank", "buffers", "init_image")}
-    h2d = sum(t.numel() for t in host.values())
+    # bytes fi_campaign moves host -> device: the tables, and the image minus the
+    # buffers with a writer (zeroed on the device), gaps < 1 MiB merged
+    h2d = sum(host[k].numel() for k in ("code", "kernels", "instances", "cbank", "buffers"))
+    rng = []
+    for b in prog.buffers:
+        if int(b["writer"]) >= 0 or not int(b["size"]):
+            continue
+        o, e = int(b["off"]), int(b["off"]) + int(b["size"])
+        if rng and o >= rng[-1][1] and o - rng[-1][1] < (1 << 20):
+            rng[-1][1] = max(rng[-1][1], e)
+        else:
+            rng.append([o, e])
+    h2d += sum(e - o for o, e in rng)
     del camp
     torch.cuda.empty_cache()
     times, r, jit_ms = [], None, []

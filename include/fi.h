@@ -187,7 +187,8 @@ fi_status fi_profile(const fi_trace* t, uint64_t rec_begin, uint64_t rec_end, ui
  * at [rank]; part_local: [K][8] u64 scratch of this rank; epoch: 1, 2, ... — the
  * number of fi_profile_peers calls this rank has made, the same on every rank.
  * Every rank must call it for every epoch (the wait spins on the device until the
- * others do; after 60 s without them it traps: a CUDA error, not a hung GPU).  A rank must not start epoch e+1 before every rank has consumed the
+ * others do; after 60 s without them it gives up and ORs FI_E_COLLECTIVE into
+ * dev_status — that epoch's counts are then invalid; no trap, the context lives on).  A rank must not start epoch e+1 before every rank has consumed the
  * chunk_counts / partials of epoch e (the bench's per-step barrier).
  * Errors: FI_E_ARG, FI_E_CUDA. */
 #define FI_MAX_PEERS 8
@@ -199,7 +200,7 @@ typedef struct {
 } fi_peers;
 fi_status fi_profile_peers(const fi_trace* t, uint64_t rec_begin, uint64_t rec_end, uint32_t n_inst,
                            const fi_peers* peers, uint64_t* part_local, uint32_t epoch, uint64_t* inst_counts,
-                           uint32_t* chunk_counts, void* stream);
+                           uint32_t* chunk_counts, uint32_t* dev_status, void* stream);
 /* Device memory shareable with the other ranks' processes (cudaMalloc +
  * cudaIpcGetMemHandle): *dev_ptr (zero-filled) and its 64-B handle; fi_ipc_open
  * maps a peer's handle into this process (peer access enabled lazily);
@@ -488,7 +489,8 @@ fi_status fi_write_profile_txt(const uint64_t* inst_counts_host, const fi_instan
 
 /* ---- fi_campaign: the whole campaign of one rank, host buffers in and out ----
  * PAPER.md:72 Fig. 1 steps (1)-(4) end to end, as the driver of SURVEY §8(e):
- * H2D of the program (from HOST arrays), golden run (passes 1 + 2, golden
+ * H2D of the program (from HOST arrays; buffers with a writer are zeroed on the
+ * device instead of copied — they start zeroed), golden run (passes 1 + 2, golden
  * checkpoints), K1 profile of this rank's chunk-aligned record shard
  * [chunk r*C/G, (r+1)*C/G), all-reduce(SUM) of inst_counts (u64) and
  * chunk_counts (u32) through `allreduce`, K2 index (+ a3 identities), K3 select

@@ -153,7 +153,7 @@ class Campaign:
         if self.peers is not None:
             # K1 with its rows stored into every peer, partial counts pushed, device-side
             # flag wait, partial sum: one stream-ordered call, the exchange inside it
-            self.peers.profile(self.gt, self.r0, self.r1, self.inst_counts)
+            self.peers.profile(self.gt, self.r0, self.r1, self.inst_counts, self.status)
             mark("profile")
         else:
             if self.world > 1:

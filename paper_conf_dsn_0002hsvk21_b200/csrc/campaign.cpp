@@ -179,8 +179,26 @@ extern "C" fi_status fi_campaign(const fi_campaign_cfg* cfg, int rank, int world
     if (cfg->n_cbank)
         FI_TRY(cu(cudaMemcpyAsync(cbank, cfg->cbank, 4ull * cfg->n_cbank, cudaMemcpyHostToDevice, s)));
     FI_TRY(cu(cudaMemcpyAsync(buf, cfg->buf, sizeof(fi_buffer) * cfg->n_buf, cudaMemcpyHostToDevice, s)));
-    if (cfg->image_bytes)
-        FI_TRY(cu(cudaMemcpyAsync(image, cfg->init_image, cfg->image_bytes, cudaMemcpyHostToDevice, s)));
+    if (cfg->image_bytes) {
+        // Buffers with a writer start zeroed (SSA: the emulator never
+        // reads their initial content), so only the other buffers cross PCIe: the
+        // image is zeroed on the device and the writer-less buffers copied, nearby
+        // ones (gap < 1 MiB) merged into one copy.
+        FI_TRY(cu(cudaMemsetAsync(image, 0, cfg->image_bytes, s)));
+        std::vector<std::pair<uint64_t, uint64_t>> rng;
+        for (uint32_t b = 0; b < cfg->n_buf; ++b) {
+            const fi_buffer& B = cfg->buf[b];
+            if (B.writer >= 0 || !B.size || B.off >= cfg->image_bytes) continue;
+            const uint64_t e = std::min<uint64_t>(B.off + B.size, cfg->image_bytes);
+            if (!rng.empty() && B.off >= rng.back().second && B.off - rng.back().second < (1u << 20))
+                rng.back().second = std::max(rng.back().second, e);
+            else
+                rng.push_back({B.off, e});
+        }
+        for (auto& r : rng)
+            FI_TRY(cu(cudaMemcpyAsync(image + r.first, cfg->init_image + r.first, r.second - r.first,
+                                      cudaMemcpyHostToDevice, s)));
+    }
 
     void* aux;
     FI_TRY(A.alloc(&aux, fi_program_aux_bytes(cfg->image_bytes, cfg->n_code, K)));

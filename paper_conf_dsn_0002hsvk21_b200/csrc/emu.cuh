@@ -605,7 +605,7 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
                         for (uint32_t b = 0; b < nb; ++b) {
                             const uint32_t s = sb + b;
                             if ((s & 31) == lane) recbuf = make_uint4(k, __ldg(&ins[pcm + (s - step)]), amask, kFull);
-                            if ((s & 31) == 31) reinterpret_cast<uint4*>(rec_out)[s - 31 + lane] = recbuf;
+                            if ((s & 31) == 31) __stcs(&reinterpret_cast<uint4*>(rec_out)[s - 31 + lane], recbuf);
                         }
                     }
                     fq += nb;
@@ -680,7 +680,7 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
                         if (MODE == EMU_TRACE) {
                             const uint32_t s = step + b;
                             if ((s & 31) == lane) recbuf = make_uint4(k, __ldg(&ins[pcm + b]), amask, preds_b[b]);
-                            if ((s & 31) == 31) reinterpret_cast<uint4*>(rec_out)[s - 31 + lane] = recbuf;
+                            if ((s & 31) == 31) __stcs(&reinterpret_cast<uint4*>(rec_out)[s - 31 + lane], recbuf);
                         }
                     }
                 }
@@ -704,7 +704,7 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
                     if (MODE == EMU_TRACE) {
                         const uint32_t s = step + j;
                         if ((s & 31) == lane) recbuf = make_uint4(k, __ldg(&ins[pcm + j]), amask, pred);
-                        if ((s & 31) == 31) reinterpret_cast<uint4*>(rec_out)[s - 31 + lane] = recbuf;
+                        if ((s & 31) == 31) __stcs(&reinterpret_cast<uint4*>(rec_out)[s - 31 + lane], recbuf);
                     }
                     exec_plain(F, LC, D, inA && pv, preds);
                 }
@@ -728,7 +728,7 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
 
         if (MODE == EMU_TRACE) {
             if ((step & 31) == lane) recbuf = make_uint4(k, __ldg(&ins[pcm]), active, pred);
-            if ((step & 31) == 31) reinterpret_cast<uint4*>(rec_out)[step - 31 + lane] = recbuf;
+            if ((step & 31) == 31) __stcs(&reinterpret_cast<uint4*>(rec_out)[step - 31 + lane], recbuf);
         }
 
         uint32_t taken = 0;                           // lanes that branch
@@ -858,9 +858,12 @@ __device__ __forceinline__ EmuOut emulate(const EmuProg P, uint8_t* img_w, const
     }
     if (MODE == EMU_TRACE) {
         const uint32_t rem = step & 31;
-        if (rem && lane < rem) reinterpret_cast<uint4*>(rec_out)[step - rem + lane] = recbuf;
-        if (use_ck)                                   // checkpoints the warp never reached: absent
-            for (; ckn < (step + ck_interval - 1) / ck_interval; ++ckn) ck[(size_t)ckn * ckw + (zr + 3) * 32 + lane] = ~0u;
+        if (rem && lane < rem) __stcs(&reinterpret_cast<uint4*>(rec_out)[step - rem + lane], recbuf);
+        if (use_ck)                                   // checkpoints the warp never reached: absent (zero rows, step ~0)
+            for (; ckn < (step + ck_interval - 1) / ck_interval; ++ckn) {
+                for (uint32_t r = 0; r < zr + 3; ++r) ck[(size_t)ckn * ckw + r * 32 + lane] = 0u;
+                ck[(size_t)ckn * ckw + (zr + 3) * 32 + lane] = ~0u;
+            }
     }
     o.steps = step;
     o.nstore = nst;

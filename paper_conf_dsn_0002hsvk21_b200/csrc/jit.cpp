@@ -326,7 +326,9 @@ struct Gen {
           E + 1);
         for (uint32_t q = L; q <= E; ++q)
             if (code[q].guard != 7) o("if (p_ == %uu) pr_ = gb_%u; ", q, q);
-        o("rec_out[step + j_] = make_uint4(k, __ldg(&ins[p_]), amask, pr_); } }\n");
+        // streaming stores (evict-first): the 16-B records are written once and read by
+        // other kernels, so they must not push the image lines the loads reuse out of L2
+        o("__stcs(&rec_out[step + j_], make_uint4(k, __ldg(&ins[p_]), amask, pr_)); } }\n");
     }
     void mem(Src& o, const fi_insn& I, uint32_t pc, const char* stepx) const {
         using namespace fi;
@@ -629,7 +631,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
     typedef std::bitset<256> RSet;
     std::vector<RSet> lin(n + 1), lfrom(n + 2);     // live-in per pc; lfrom[e] = union of lin[q], q >= e
     RSet shfl;
-    const bool use_kill = mode != 2 && !std::getenv("FI_JIT_NO_KILL");
+    const bool use_kill = mode != 2;
     if (use_kill) {
         std::vector<RSet> rd(n), kl(n);
         for (uint32_t i = 0; i < n; ++i) {
@@ -731,7 +733,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "jx->after_[lane] = 0u; jx->msk_[lane] = 0u; jx->fired_[lane] = 0u; jx->bad_[lane] = 0u;\n"
       "JBufCache bc; uint4 recbuf = make_uint4(0u, 0u, 0u, 0u); (void)recbuf;\n"
       "// golden trace pass: the last step was a BRA / EXIT; next checkpoint and its threshold step\n"
-      "u32 brk = 1u, ckn = 0u, ckx = %s; (void)brk; (void)ckn; (void)ckx;\n"
+      "u32 brk = 1u, ckn = 0u, ckx = %s; (void)brk; (void)ckn; (void)ckx;\nu32 lexm_ = 0u; (void)lexm_;\n"
       "// blocks run only within [step, lim): lim = the watchdog, or the injection step while it is pending,\n"
       "// or the next checkpoint step (golden trace pass)\n"
       "u32 lim = %s;\n", mode == 2 ? "ck ? 0u : 0xFFFFFFFFu" : "0xFFFFFFFFu",
@@ -748,7 +750,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
         // from block code is such a step, so blocks never stop at a multiple
         o(" if (brk && step >= ckx) {\n  for (; ckn <= step / ck_interval; ++ckn) {\n"
           "   u32* dst_ = ck + (u64)ckn * %uu;\n", (NR + 4) * 32);
-        for (uint32_t j = 0; j < NR; ++j) o("   dst_[%uu + lane] = R%u;%s", j * 32, j, (j % 8 == 7) ? "\n" : "");
+        for (uint32_t j = 0; j < NR; ++j) o("   __stcs(&dst_[%uu + lane], R%u);%s", j * 32, j, (j % 8 == 7) ? "\n" : "");
         o("\n   dst_[%uu + lane] = live ? (inA ? upc : pc) : 0u;\n"
           "   dst_[%uu + lane] = (u32)Q0 | ((u32)Q1 << 1) | ((u32)Q2 << 2) | ((u32)Q3 << 3) | ((u32)Q4 << 4) | "
           "((u32)Q5 << 5) | ((u32)Q6 << 6);\n   dst_[%uu + lane] = live ? 1u : 0u;\n   dst_[%uu + lane] = step;\n  }\n"
@@ -777,10 +779,36 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
     };
     auto flush_end = [&]() { G.flush_recs(o, code, run_start(n - 1), n - 1); };
     uint32_t batch_end = 0;                           // LDGs [.., batch_end) already emitted as a batch
+    uint32_t loop_L = ~0u;                            // leader of the self-loop being emitted
+    bool loop_dup = false;                            // ... emitted twice (full-warp copy + general)
+    std::string loop_saved;                           // the output before that loop's body
     for (uint32_t i = 0; i < n; ++i) {
         const fi_insn& I = code[i];
         std::snprintf(stepx, sizeof stepx, "step + (%uu - pcm)", i);
         if (leader[i]) o(" B%u:\n", i);
+        // a block whose BRA jumps back to its own leader is emitted as a structured
+        // inner loop: the uniform-taken back edge that fits is its `continue`, so the
+        // loop has one header and the compiler keeps loop-carried registers in place
+        // (chaining through the label made a multi-entry loop: the allocator gave the
+        // accumulators different homes at the top and the bottom and copied them on
+        // every iteration)
+        //   The loop body is emitted twice when no other pc inside it is a leader: a copy
+        // for a full warp (all 32 lanes in amask, constant over the loop since its only
+        // exit is the BRA), where `inA` is the constant true and every lane-predicated
+        // write becomes an unconditional one — predicated accumulators and loads made the
+        // allocator keep two homes per loop-carried register and copy between them on
+        // every iteration — and the general copy.
+        if (leader[i] && code[i + blen[i] - 1].op == BRA && code[i + blen[i] - 1].imm == i && blen[i] > 1) {
+            loop_L = i;
+            loop_dup = true;
+            for (uint32_t q = i + 1; q < i + blen[i]; ++q) loop_dup = loop_dup && !leader[q];
+            if (loop_dup) {
+                loop_saved = std::move(o.s);
+                o.s.clear();
+            } else {
+                o(" for (;;) {  // self-loop %u..%u\n", i, i + blen[i] - 1);
+            }
+        }
         if (i < batch_end) {
             if (i + 1 == n) {
                 flush_end();
@@ -801,8 +829,8 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
                 batch_end = i + m;
                 if (i + m == n) {
                     flush_end();
-                    o(" { step += %uu - pcm; upc = %uu; if (upc >= npc) { conv = false; if (inA) pc = upc; } continue; }\n",
-                      n, n);
+                    o(" { %sstep += %uu - pcm; upc = %uu; if (upc >= npc) { conv = false; if (inA) pc = upc; } continue; }\n",
+                      kills(RSet()).c_str(), n, n);
                 }
                 continue;
             }
@@ -822,12 +850,35 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
             G.flush_recs(o, code, run_start(i), i);
             const RSet keep_ft = use_kill ? lfrom[i + 1] : RSet();
             const RSet keep_tk = use_kill ? (I.imm < n ? lin[I.imm] : RSet()) | lfrom[i + 1] : RSet();
-            o("const u32 exm_ = amask & __ballot_sync(JFULL, pv); step += %uu - pcm;\n"
-              "   if (exm_ == 0u) { %s%supc = %uu; } else if (exm_ == amask) { %s%supc = %uu; }\n"
+            if (loop_L == I.imm && i + 1 == loop_L + blen[loop_L]) {
+                // the self-loop's back edge (uniform taken, next iteration fits), else its exit
+                const uint32_t L = loop_L;
+                o("lexm_ = amask & __ballot_sync(JFULL, pv); step += %uu - pcm;\n"
+                  "   if (lexm_ == amask && %uu <= npc && step + %uu <= lim%s) { pcm = %uu; %scontinue; } }\n"
+                  "   break;\n",
+                  i + 1, L + blen[L], blen[L], mode == 2 ? " && step < ckx" : "", L, entry_kills(L).c_str());
+                if (loop_dup) {
+                    std::string body = std::move(o.s);
+                    o.s = std::move(loop_saved);
+                    o(" if (amask == JFULL) { const bool inA = true; (void)inA;\n for (;;) {  // self-loop %u..%u, full warp\n",
+                      L, i);
+                    o.s += body;
+                    o(" } } else {\n for (;;) {  // self-loop %u..%u\n", L, i);
+                    o.s += body;
+                    o(" } }\n");
+                } else {
+                    o(" }\n");
+                }
+                o(" { const u32 exm_ = lexm_;\n");
+                loop_L = ~0u;
+            } else {
+                o("const u32 exm_ = amask & __ballot_sync(JFULL, pv); step += %uu - pcm;\n", i + 1);
+            }
+            o("   if (exm_ == 0u) { %s%supc = %uu; } else if (exm_ == amask) { %s%supc = %uu; }\n"
               "   else { %sconv = false; if (inA) pc = ((exm_ >> lane) & 1u) ? %uu : %uu; }\n"
               "   if (conv && (amask == 0u || upc >= npc)) { conv = false; if ((amask >> lane) & 1u) pc = upc; }\n"
               "   continue; }\n",
-              i + 1, chain(i + 1).c_str(), kills(keep_ft).c_str(), i + 1, chain(I.imm).c_str(),
+              chain(i + 1).c_str(), kills(keep_ft).c_str(), i + 1, chain(I.imm).c_str(),
               kills(keep_tk).c_str(), I.imm, kills(keep_tk).c_str(), I.imm, i + 1);
         } else if (I.op == EXIT) {
             o(" { const bool pv = %s; %s", G.guard(I.guard).c_str(), mode == 2 ? "brk = 1u; " : "");
@@ -882,8 +933,10 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "  if (done_) goto finish;\n  continue;\n }\n}\n");
     o("finish:\n");
     if (mode == 2)                                    // checkpoints the warp never reached: absent
-        o(" if (ck) for (; ckn < (step + ck_interval - 1u) / ck_interval; ++ckn) ck[(u64)ckn * %uu + %uu + lane] = 0xFFFFFFFFu;\n",
-          (NR + 4) * 32, (NR + 3) * 32);
+        o(" if (ck) for (; ckn < (step + ck_interval - 1u) / ck_interval; ++ckn) {\n"
+          "   for (u32 r_ = 0u; r_ < %uu; ++r_) ck[(u64)ckn * %uu + r_ * 32u + lane] = 0u;\n"
+          "   ck[(u64)ckn * %uu + %uu + lane] = 0xFFFFFFFFu; }\n",
+          NR + 3, (NR + 4) * 32, (NR + 4) * 32, (NR + 3) * 32);
     o("#undef out\n");
     o(" { JOut& out_ = *jx->out; out_.steps = step; out_.fault = jx->fault_[lane]; out_.fault_pc = jx->fault_pc_[lane]; "
       "out_.nstore = jx->nst_[lane];\n"
@@ -899,10 +952,8 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
                      int only = -1) {
     const bool slice_len = modes & kJitSliceLen;    // golden pass 1 as the control slice (fi_jit_build decides)
     // resident 128-thread CTAs per SM the register budget targets (3: <= 168 registers)
-    uint32_t min_blocks = 3;
-    if (const char* e = std::getenv("FI_JIT_MIN_BLOCKS")) min_blocks = (uint32_t)std::max(1, std::atoi(e));
+    const uint32_t min_blocks = 3;
     Src o;
-    if (std::getenv("FI_JIT_LDALLOC")) o.s = "#define JLD_L1 \"\"\n";
     o.s += kPrelude;
     Gen G{n_regs};
     auto mine = [&](uint32_t k) { return only < 0 || (uint32_t)only == k; };
@@ -1165,9 +1216,8 @@ fi_status compile_cubin(const fi_insn* code, const fi_kernel* kern, uint32_t n_k
     const std::string pname = dump.empty() ? std::string("fi_jit.cu") : dump + ".cu";
     void* prog = nullptr;
     if (N.create(&prog, src.c_str(), pname.c_str(), 0, nullptr, nullptr)) { g_jit_log = "nvrtcCreateProgram failed"; return FI_E_CUDA; }
-    std::vector<const char*> opts = {"--gpu-architecture=sm_100a", "--std=c++17", "--fmad=false", "-lineinfo"};
-    std::string extra;                                // experiments: one more NVRTC option
-    if (const char* e = std::getenv("FI_JIT_NVRTC_OPT")) if (*e) { extra = e; opts.push_back(extra.c_str()); }
+    // --fmad=false: FMUL + FADD are never contracted (C-13); fixed, not configurable
+    const std::vector<const char*> opts = {"--gpu-architecture=sm_100a", "--std=c++17", "--fmad=false", "-lineinfo"};
     const int rc = N.compile(prog, (int)opts.size(), opts.data());
     size_t ls = 0;
     N.log_size(prog, &ls);

@@ -143,7 +143,7 @@ __device__ __forceinline__ u32 jshfl_src(u32 lane, u32 bv, u32 m) {
 }
 
 #ifndef JLD_L1
-#define JLD_L1 ".L1::no_allocate"                    // image loads do not allocate in L1 (override: FI_JIT_LDALLOC)
+#define JLD_L1 ".L1::no_allocate"                    // image loads do not allocate in L1
 #endif
 __device__ __forceinline__ u32 jld32(const u8* p) {
     u32 r;
@@ -529,7 +529,7 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
         const bool ex = act && pv;
         const u32 exm = active & pred;
         if (MODE == JM_TRACE && lane == 0)            // one trace record per step (App. A.3)
-            rec_out[step] = make_uint4(k, __ldg(&ins[pcm]), active, pred);
+            __stcs(&rec_out[step], make_uint4(k, __ldg(&ins[pcm]), active, pred));
         u32 taken = 0;
         brk = op == 1 || op == 2;
         if (MODE == JM_LEN && slice && !slice[pcm] && op != 1 && op != 2) {

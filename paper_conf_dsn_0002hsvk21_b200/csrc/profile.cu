@@ -235,18 +235,19 @@ __global__ void k_signal(fi_peers P) {
     for (uint32_t r = 0; r < P.world; ++r) atomicAdd_system(P.flags[r], 1u);
 }
 // acquire: wait until every rank's increment of this epoch arrived.  Bounded: a
-// rank that never signals (it died) turns into a device trap after 60 s — a loud
-// CUDA error in this process instead of a GPU spinning forever.
+// rank that has not signalled after 60 s (it died, or is skewed by more than
+// that) makes the wait give up and set FI_E_COLLECTIVE in the caller's status
+// word — the call's counts are then not valid, but the context stays usable.
 __device__ __forceinline__ uint64_t globaltimer_ns() {
     uint64_t t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     return t;
 }
-__global__ void k_wait(const uint32_t* flag, uint32_t target) {
+__global__ void k_wait(const uint32_t* flag, uint32_t target, uint32_t* status) {
     const uint64_t t0 = globaltimer_ns();
     while (*reinterpret_cast<const volatile uint32_t*>(flag) < target) {
         __nanosleep(200);
-        if (globaltimer_ns() - t0 > 60ull * 1000000000ull) __trap();
+        if (globaltimer_ns() - t0 > 60ull * 1000000000ull) { FI_DEV_ERR(status, FI_E_COLLECTIVE); return; }
     }
     __threadfence_system();
 }
@@ -283,8 +284,10 @@ extern "C" fi_status fi_ipc_free(void* dev_ptr) { return cuda_status(cudaFree(de
 
 extern "C" fi_status fi_profile_peers(const fi_trace* t, uint64_t rec_begin, uint64_t rec_end, uint32_t n_inst,
                                       const fi_peers* peers, uint64_t* part_local, uint32_t epoch,
-                                      uint64_t* inst_counts, uint32_t* chunk_counts, void* stream) {
-    if (!t || !peers || !part_local || !inst_counts || !chunk_counts || rec_end > t->n_rec || rec_begin > rec_end)
+                                      uint64_t* inst_counts, uint32_t* chunk_counts, uint32_t* dev_status,
+                                      void* stream) {
+    if (!t || !peers || !part_local || !inst_counts || !chunk_counts || !dev_status || rec_end > t->n_rec ||
+        rec_begin > rec_end)
         return FI_E_ARG;
     if (rec_begin % FI_CHUNK || peers->world < 1 || peers->world > FI_MAX_PEERS || peers->rank >= peers->world ||
         epoch == 0)
@@ -317,7 +320,7 @@ extern "C" fi_status fi_profile_peers(const fi_trace* t, uint64_t rec_begin, uin
     const uint32_t pg = (uint32_t)std::min<uint64_t>(std::max<uint64_t>(1, (n + 255) / 256), 1184);
     k_push_partials<<<pg, 256, 0, s>>>(part_local, n, P);
     k_signal<<<1, 1, 0, s>>>(P);
-    k_wait<<<1, 1, 0, s>>>(P.flags[P.rank], epoch * P.world);
+    k_wait<<<1, 1, 0, s>>>(P.flags[P.rank], epoch * P.world, dev_status);
     k_sum_partials<<<pg, 256, 0, s>>>(P.partials[P.rank], n, P.world, inst_counts);
     if ((e = launch_status())) return e;
     const uint64_t C = (t->n_rec + FI_CHUNK - 1) / FI_CHUNK;  // every rank's rows, now complete, to the caller's array

@@ -184,7 +184,7 @@ def lib():
             "fi_campaign": (st, [C.POINTER(fi_campaign_cfg), C.c_int, C.c_int, ALLREDUCE_FN, vp,
                                  C.POINTER(fi_campaign_result)]),
             "fi_campaign_release_memory": (st, [C.c_int]),
-            "fi_profile_peers": (st, [vp, u64, u64, u32, vp, vp, u32, vp, vp, vp]),
+            "fi_profile_peers": (st, [vp, u64, u64, u32, vp, vp, u32, vp, vp, vp, vp]),
             "fi_ipc_alloc": (st, [sz, C.POINTER(C.c_void_p), vp]),
             "fi_ipc_open": (st, [vp, C.POINTER(C.c_void_p)]),
             "fi_ipc_close": (st, [vp]),
@@ -479,11 +479,17 @@ class PeerExchange:
         self.part_local = torch.empty((max(n_inst, 1), 8), dtype=torch.int64, device=self.device)
         self.chunk_counts = torch.zeros((max(n_chunks, 1), 8), dtype=torch.int32, device=self.device)
 
-    def profile(self, gt: "GoldenTrace", rec_begin: int, rec_end: int, inst_counts: torch.Tensor) -> None:
+    def profile(self, gt: "GoldenTrace", rec_begin: int, rec_end: int, inst_counts: torch.Tensor,
+                status: "DeviceStatus | None" = None) -> None:
+        """One epoch; a peer that never signals sets FI_E_COLLECTIVE in `status`
+        (checked here when no status is given)."""
         self.epoch += 1
+        st = status or DeviceStatus(self.device)
         _check(lib().fi_profile_peers(C.byref(gt.c), rec_begin, rec_end, gt.dp.n_inst, C.byref(self.peers),
                                       _p(self.part_local), self.epoch, _p(inst_counts), _p(self.chunk_counts),
-                                      _stream()), "fi_profile_peers")
+                                      st.ptr, _stream()), "fi_profile_peers")
+        if status is None:
+            st.check("fi_profile_peers")
 
     def close(self, group=None):
         """Unmap the peers' buffers, wait for every rank to have done the same, then

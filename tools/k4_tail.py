@@ -27,13 +27,25 @@ for _ in range(2):
 inj = fi.as_numpy(out, fi.INJ_DTYPE, n)
 st = fi.as_numpy(sites, fi.SITE_DTYPE, n)
 L = gt.warp_len.cpu().numpy()[st["warp"]]
-rem = L - (st["step"] // 4096) * 4096
+# restart step of each replica: the last golden checkpoint at or before its site
+# (checkpoint c's step is stored in its last row, ~0 when absent; no checkpoints: 0)
+start = np.zeros(n, dtype=np.int64)
+if gt.ckpt is not None and gt.ckpt_interval:
+    iv, rows = gt.ckpt_interval, gt.dp.n_regs + 4
+    ck = gt.ckpt.cpu().numpy().view(np.uint32)
+    off = gt.ckpt_off.cpu().numpy()
+    for i in range(n):
+        c = int(st["step"][i]) // iv
+        while c > 0 and ck[(off[st["warp"][i]] + c) * rows * 32 + (rows - 1) * 32] > st["step"][i]:
+            c -= 1
+        start[i] = ck[(off[st["warp"][i]] + c) * rows * 32 + (rows - 1) * 32]
+rem = L - start
 for k in range(5):
     m = inj["fault_kind"] == k
     if m.any():
         print("fault_kind", k, "n", int(m.sum()), "golden remaining steps mean", float(rem[m].mean()),
-              "max", int(rem[m].max()), "emulated est", float(np.where(k == 3, 10 * L[m] + 1024 - (st["step"][m] // 4096) * 4096, rem[m]).mean()))
-tot = np.where(inj["fault_kind"] == 3, 10 * L + 1024 - (st["step"] // 4096) * 4096, rem)
+              "max", int(rem[m].max()), "emulated est", float(np.where(k == 3, 10 * L[m] + 1024 - start[m], rem[m]).mean()))
+tot = np.where(inj["fault_kind"] == 3, 10 * L + 1024 - start, rem)
 print("total est emulated steps", int(tot.sum()), "of which watchdog", int(tot[inj["fault_kind"] == 3].sum()))
 wd = inj["fault_kind"] == 3
 print("watchdog sites: dst_reg", np.unique(st["dst_reg"][wd], return_counts=True), "pc", np.unique(st["pc"][wd], return_counts=True))
