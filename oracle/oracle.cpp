@@ -205,8 +205,32 @@ struct Prog {
     orc_program p;
     std::vector<uint32_t> gm;            // group mask per static instruction
     uint32_t n_warps = 0;
+    bool sorted = false;                 // allocations in ascending, non-overlapping order
     bool single_instance() const { return p.n_inst == 1; }
 };
+
+// The allocation that contains byte offset `off`, or nullptr.  A binary search
+// when the buffer table is sorted and non-overlapping (every generated program:
+// the lookup is the same "which allocation holds this address" as a linear scan,
+// which is kept for any other table); programs with thousands of SSA buffer
+// versions (C3) made the linear scan the oracle's dominant cost.
+const orc_buffer* find_buffer(const Prog& P, uint64_t off) {
+    if (P.sorted) {
+        uint32_t lo = 0, hi = P.p.n_buf;                 // first buffer with b.off > off
+        while (lo < hi) {
+            const uint32_t mid = (lo + hi) / 2;
+            if (P.p.buf[mid].off <= off) lo = mid + 1; else hi = mid;
+        }
+        if (lo == 0) return nullptr;
+        const orc_buffer& b = P.p.buf[lo - 1];
+        return off < b.off + b.size ? &b : nullptr;
+    }
+    for (uint32_t i = 0; i < P.p.n_buf; ++i) {
+        const orc_buffer& b = P.p.buf[i];
+        if (off >= b.off && off < b.off + b.size) return &b;
+    }
+    return nullptr;
+}
 
 struct StoreW { uint64_t va; uint32_t value; uint64_t step; };   // one 32-bit word
 
@@ -234,11 +258,8 @@ int check_access(const Prog& P, uint64_t va, uint32_t w) {
     if (va % w) return 1;
     if (va < VA_BASE) return 2;
     uint64_t off = va - VA_BASE;
-    for (uint32_t i = 0; i < P.p.n_buf; ++i) {
-        const orc_buffer& b = P.p.buf[i];
-        if (off >= b.off && off + w <= b.off + b.size) return 0;
-    }
-    return 2;
+    const orc_buffer* b = find_buffer(P, off);
+    return (b && off + w <= b->off + b->size) ? 0 : 2;
 }
 
 struct Warp {
@@ -525,6 +546,9 @@ bool prepare(Prog& P, const orc_program* p, std::string& err) {
         if (in.kernel >= p->n_kern) { err = "bad kernel id"; return false; }
     }
     P.n_warps = w;
+    P.sorted = true;
+    for (uint32_t i = 1; i < p->n_buf && P.sorted; ++i)
+        P.sorted = p->buf[i - 1].off + p->buf[i - 1].size <= p->buf[i].off;
     return true;
 }
 
@@ -647,22 +671,11 @@ bool output_beyond_tol(const Prog& P, const std::vector<uint8_t>& a, const std::
     return false;
 }
 
-const orc_buffer* buffer_of(const Prog& P, uint64_t va) {
-    uint64_t off = va - VA_BASE;
-    for (uint32_t i = 0; i < P.p.n_buf; ++i) {
-        const orc_buffer& b = P.p.buf[i];
-        if (off >= b.off && off < b.off + b.size) return &b;
-    }
-    return nullptr;
-}
+const orc_buffer* buffer_of(const Prog& P, uint64_t va) { return find_buffer(P, va - VA_BASE); }
 
 bool is_output_addr(const Prog& P, uint64_t va) {
-    uint64_t off = va - VA_BASE;
-    for (uint32_t i = 0; i < P.p.n_buf; ++i) {
-        const orc_buffer& b = P.p.buf[i];
-        if (off >= b.off && off < b.off + b.size) return b.flags & 1;
-    }
-    return false;
+    const orc_buffer* b = find_buffer(P, va - VA_BASE);
+    return b && (b->flags & 1);
 }
 
 }  // namespace

@@ -96,6 +96,7 @@ def main():
     ap.add_argument("--n", type=int, default=None)
     ap.add_argument("--subset", type=int, default=None)
     ap.add_argument("--programs", default=None, help="C5: comma-separated program indices")
+    ap.add_argument("--n-list", default=None, help="C5: comma-separated replica counts, one per selected program")
     ap.add_argument("--out", default=None)
     a = ap.parse_args()
     torch.cuda.set_device(0)
@@ -107,10 +108,11 @@ def main():
             a.n or 100000, a.subset or 32, a.out)
     else:
         progs = H.c5(full=True)
-        sel = range(len(progs)) if a.programs is None else [int(x) for x in a.programs.split(",")]
-        for i in sel:
+        sel = list(range(len(progs))) if a.programs is None else [int(x) for x in a.programs.split(",")]
+        ns = [int(x) for x in a.n_list.split(",")] if a.n_list else [a.n or 2000] * len(sel)
+        for i, n in zip(sel, ns):
             run("C5 " + progs[i].meta["config"], progs[i], H.C5_CAMPAIGN_SEED + i, [fi.G_GP], [0],
-                a.n or 2000, a.subset or 16, a.out)
+                n, a.subset or 16, a.out)
 
 
 if __name__ == "__main__":
