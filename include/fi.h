@@ -95,6 +95,7 @@ typedef struct {
             flags /* bit0 FI_SITE_NOT_INJECTED */;
 } fi_site;                                           /* 64 B */
 #define FI_SITE_NOT_INJECTED 1u
+#define FI_SITE_REMOTE 0x80u      /* fi_select_sites_shard: drawn here, located by the rank holding its records */
 
 typedef struct {
     uint64_t seed;                                   /* campaign seed (Philox key) */
@@ -251,6 +252,20 @@ fi_status fi_select_sites(const fi_program* p, const fi_trace* t, const uint32_t
                           uint32_t n_inst, uint64_t n_chunks, const uint64_t totals_host[8],
                           const fi_schedule* sched, uint64_t j0, uint32_t n, fi_site* sites, uint32_t* dev_status,
                           void* stream);
+
+/* Owner-computes K3: the same draw for replicas [j0, j0+n), but
+ * only sites whose chunk lies in this rank's record shard [rec_begin, rec_end)
+ * (chunk-aligned; the rank whose golden pass wrote those records) are located;
+ * the others are written with FI_SITE_REMOTE set and only s / u_dst / u_bit /
+ * group / bfm / mask filled.  fi_compact_sites then keeps the located ones. */
+fi_status fi_select_sites_shard(const fi_program* p, const fi_trace* t, const uint32_t* chunk_counts,
+                                const void* index, uint32_t n_inst, uint64_t n_chunks, const uint64_t totals_host[8],
+                                const fi_schedule* sched, uint64_t j0, uint32_t n, uint64_t rec_begin,
+                                uint64_t rec_end, fi_site* sites, uint32_t* dev_status, void* stream);
+/* Stable compaction of sites[0, n) without FI_SITE_REMOTE into out[0, *n_out)
+ * (device count), their replica indices j0 + i into out_j.  One CTA. */
+fi_status fi_compact_sites(const fi_site* sites, uint32_t n, uint64_t j0, fi_site* out, uint64_t* out_j,
+                           uint32_t* n_out, void* stream);
 
 /* K3 with an approximate profile (row f1): s is drawn over the approximate
  * totals and mapped to (instance k, instruction_count) by the approximate P_k;
@@ -434,6 +449,14 @@ fi_status fi_golden_lengths_jit(const fi_jit* j, const fi_program* p, uint8_t* i
                                 uint64_t* warp_nstore, uint32_t* dev_status, void* stream);
 fi_status fi_golden_trace_jit(const fi_jit* j, const fi_program* p, uint8_t* image, const fi_trace* t,
                               uint32_t* dev_status, void* stream);
+/* Pass 2 for the warps [w_lo, w_hi) only, image stores only from the warps
+ * [own_lo, own_hi) (the owner-computes golden run of fi_golden_run_shard). */
+fi_status fi_golden_trace_jit_range(const fi_jit* j, const fi_program* p, uint8_t* image, const fi_trace* t,
+                                    uint32_t w_lo, uint32_t w_hi, uint32_t own_lo, uint32_t own_hi,
+                                    uint32_t* dev_status, void* stream);
+/* 1 when fi_jit_build generated golden pass 1 as the control slice (it then leaves
+ * the image untouched; pass 2 writes it), else 0. */
+int fi_jit_len_sliced(const fi_jit* j);
 /* fi_classify_batched with K8's per-launch re-execution on a module built with
  * FI_JIT_PAGE: same arguments, scratch and results (transient faults). */
 fi_status fi_classify_batched_jit(const fi_jit* j, const fi_program* p, const uint8_t* image, const fi_trace* t,
@@ -463,6 +486,19 @@ fi_status fi_classify_batched_jit(const fi_jit* j, const fi_program* p, const ui
 typedef struct fi_golden fi_golden;
 fi_status fi_golden_run(const fi_program* p, const fi_jit* jit, uint8_t* image, uint32_t ckpt_interval,
                         double ckpt_budget_frac, fi_golden** out, void* stream);
+/* Owner-computes golden run of rank `rank` of `world` (a
+ * single-launch program and the JIT engine): pass 1 for every warp (the layout
+ * is global), pass 2 only for the warps holding the records of this rank's
+ * chunk-aligned shard [r0, r1) = fi_campaign's profile shard, and into `image`
+ * only the stores of the warps whose first record lies in it.  The trace of
+ * that shard, its checkpoints and store log are valid; the rest of the arrays is
+ * not written.  With a sliced pass 1 (fi_jit_len_sliced) the image then holds
+ * the golden words of this rank's warps only: the SUM over the ranks of the
+ * writer buffers (zero-initialised, SSA) is the golden final image.
+ * world = 1 is fi_golden_run. */
+fi_status fi_golden_run_shard(const fi_program* p, const fi_jit* jit, uint8_t* image, uint32_t ckpt_interval,
+                              double ckpt_budget_frac, int rank, int world, fi_golden** out, void* stream);
+void fi_golden_shard_range(const fi_golden* g, uint64_t* rec_begin, uint64_t* rec_end, uint32_t* w_lo, uint32_t* w_hi);
 const fi_trace* fi_golden_trace_of(const fi_golden* g);          /* host struct of device pointers */
 const uint64_t* fi_golden_warp_len(const fi_golden* g);          /* device [n_warps] golden steps per warp */
 const uint64_t* fi_golden_gstore_off_host(const fi_golden* g);   /* HOST [n_warps+1] copy of gstore_off */
@@ -543,6 +579,9 @@ typedef struct {
     int device;                  /* CUDA device ordinal (< 0 = current) */
     void* stream;                /* cudaStream_t (NULL = a stream fi_campaign creates) */
     double rtol;                 /* > 0: also the C-12 secondary numeric classification (hist_tol) */
+    uint32_t owner_computes;     /* world > 1, one launch, JIT: the golden run is sharded with the profile
+                                    (fi_golden_run_shard) and each rank injects the replicas whose site lies in
+                                    its record shard (fi_select_sites_shard) instead of the block [r*n/G, (r+1)*n/G) */
 } fi_campaign_cfg;
 
 typedef struct {
@@ -563,6 +602,7 @@ typedef struct {
     fi_inj* inj;                 /* [n_local] */
     uint64_t* inst_counts;       /* [n_inst][8] (after the exchange) */
     uint64_t hist_tol[8][4][3];  /* cfg->rtol > 0: secondary histogram (FI_SDC_WITHIN_TOL counted Masked), all ranks */
+    uint64_t* j;                 /* optional [n_local]: the replica index of each returned site / result row */
 } fi_campaign_result;
 
 fi_status fi_campaign(const fi_campaign_cfg* cfg, int rank, int world, fi_allreduce_fn allreduce, void* ctx,

@@ -219,7 +219,26 @@ extern "C" fi_status fi_campaign(const fi_campaign_cfg* cfg, int rank, int world
     // ---- golden run (fi_golden_run: pass 1, scans, checkpoint layout, pass 2) ----
     GoldenGuard gg;
     gg.s = s;
-    FI_TRY(fi_golden_run(&p, jit, image, cfg->ckpt_interval, 0.2, &gg.g, s));
+    // owner-computes: a single-launch program's golden run is sharded
+    // like the profile — this rank emulates (pass 2) only the warps of its record
+    // shard, and the golden image is completed by one SUM over the writer buffers
+    const bool owner = cfg->owner_computes && world > 1 && K == 1 && jit && !cfg->approximate;
+    if (owner) FI_TRY(fi_golden_run_shard(&p, jit, image, cfg->ckpt_interval, 0.2, rank, world, &gg.g, s));
+    else FI_TRY(fi_golden_run(&p, jit, image, cfg->ckpt_interval, 0.2, &gg.g, s));
+    if (owner && fi_jit_len_sliced(jit)) {
+        // writer buffers start zeroed (SSA, §3.5) and each word is stored by one warp,
+        // owned by one rank: the sum over the ranks is the golden final image
+        std::vector<std::pair<uint64_t, uint64_t>> wr;
+        for (uint32_t b = 0; b < cfg->n_buf; ++b) {
+            const fi_buffer& B = cfg->buf[b];
+            if (B.writer < 0 || !B.size) continue;
+            const uint64_t o = B.off & ~3ull, e = std::min<uint64_t>((B.off + B.size + 3) & ~3ull, cfg->image_bytes);
+            if (!wr.empty() && o <= wr.back().second) wr.back().second = std::max(wr.back().second, e);
+            else wr.push_back({o, e});
+        }
+        for (auto& r : wr)
+            if (allreduce(image + r.first, (r.second - r.first) / 4, 4, ctx, s)) return FI_E_COLLECTIVE;
+    }
     const fi_trace t = *fi_golden_trace_of(gg.g);
     const uint64_t n_rec = t.n_rec;
     const uint64_t* goff_h = fi_golden_gstore_off_host(gg.g);
@@ -269,16 +288,29 @@ extern "C" fi_status fi_campaign(const fi_campaign_cfg* cfg, int rank, int world
     FI_TRY(check_status(st, s));
     FI_TRY(ev.mark(s));                                                    // 5
 
-    // ---- K3 select / K4 inject / classify of this rank's replica block -------
-    const uint64_t j0 = cfg->n_replicas * (uint64_t)rank / world;
-    const uint64_t j1 = cfg->n_replicas * (uint64_t)(rank + 1) / world;
+    // ---- K3 select / K4 inject / classify of this rank's replicas -------------
+    // replica block [r*n/G, (r+1)*n/G); owner-computes: every replica is drawn, the
+    // rank keeps those whose site lies in its record shard (fi_select_sites_shard)
+    const uint64_t j0 = owner ? 0 : cfg->n_replicas * (uint64_t)rank / world;
+    const uint64_t j1 = owner ? cfg->n_replicas : cfg->n_replicas * (uint64_t)(rank + 1) / world;
     if (j1 - j0 > 0xFFFFFFFFull) return FI_E_ARG;
-    const uint32_t n = (uint32_t)(j1 - j0);
+    uint32_t n = (uint32_t)(j1 - j0);
     fi_site* sites;
     fi_inj* inj;
+    uint64_t* jidx = nullptr;
     FI_TRY(A.alloc(&sites, 64ull * std::max(n, 1u)));
     FI_TRY(A.alloc(&inj, 24ull * std::max(n, 1u)));
-    if (n) {
+    if (owner && n) {
+        fi_site* drawn;
+        uint32_t* n_dev;
+        FI_TRY(A.alloc(&drawn, 64ull * n));
+        FI_TRY(A.alloc(&jidx, 8ull * n));
+        FI_TRY(A.alloc(&n_dev, 4));
+        FI_TRY(fi_select_sites_shard(&p, &t, cc, index, K, n_chunks, totals, &cfg->sched, 0, n, r0, r1, drawn, st, s));
+        FI_TRY(fi_compact_sites(drawn, n, 0, sites, jidx, n_dev, s));
+        FI_TRY(cu(cudaMemcpyAsync(&n, n_dev, 4, cudaMemcpyDeviceToHost, s)));
+        FI_TRY(cu(cudaStreamSynchronize(s)));
+    } else if (n) {
         if (cfg->approximate)
             FI_TRY(fi_select_sites_approx(&p, &t, index, K, totals, &cfg->sched, j0, n, sites, st, s));
         else
@@ -345,6 +377,10 @@ extern "C" fi_status fi_campaign(const fi_campaign_cfg* cfg, int rank, int world
     FI_TRY(cu(cudaMemcpyAsync(res->hist, hist, sizeof(res->hist), cudaMemcpyDeviceToHost, s)));
     FI_TRY(cu(cudaMemcpyAsync(res->hist_tol, hist_tol, sizeof(res->hist_tol), cudaMemcpyDeviceToHost, s)));
     if (res->sites && n) FI_TRY(cu(cudaMemcpyAsync(res->sites, sites, 64ull * n, cudaMemcpyDeviceToHost, s)));
+    if (res->j && n) {                                   // the replica index of every returned row
+        if (jidx) FI_TRY(cu(cudaMemcpyAsync(res->j, jidx, 8ull * n, cudaMemcpyDeviceToHost, s)));
+        else for (uint32_t i = 0; i < n; ++i) res->j[i] = j0 + i;
+    }
     std::vector<fi_inj> inj_h(n);
     fi_inj* inj_dst = res->inj ? res->inj : inj_h.data();
     if (n) FI_TRY(cu(cudaMemcpyAsync(inj_dst, inj, 24ull * n, cudaMemcpyDeviceToHost, s)));

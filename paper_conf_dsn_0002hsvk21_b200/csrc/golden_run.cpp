@@ -20,6 +20,8 @@ struct fi_golden {
     uint64_t* warp_len = nullptr;
     uint64_t n_gstore = 0;
     std::vector<uint64_t> gstore_off_h;      // host copy [n_warps + 1]
+    uint64_t rec_begin = 0, rec_end = 0;     // this rank's record shard (owner-computes run), else all
+    uint32_t w_lo = 0, w_hi = 0;             // warps pass 2 ran
     template <class T>
     fi_status alloc(T** out, size_t bytes) {
         void* p = nullptr;
@@ -55,7 +57,7 @@ fi_status read_status(const uint32_t* dev_status, cudaStream_t s) {
 }
 
 fi_status run(const fi_program* p, const fi_jit* jit, uint8_t* image, uint32_t ckpt_interval, double budget_frac,
-              fi_golden* g) {
+              fi_golden* g, int rank = 0, int world = 1) {
     cudaStream_t s = g->s;
     const uint32_t W = p->n_warps;
     uint32_t* st;
@@ -114,6 +116,29 @@ fi_status run(const fi_program* p, const fi_jit* jit, uint8_t* image, uint32_t c
         GR_TRY(g->alloc(&ck, n_ck * ck_bytes));
     }
     g->t = fi_trace{rec, n_rec, woff, gst, goff, ck, ckoff, interval, W};
+    g->rec_begin = 0; g->rec_end = n_rec; g->w_lo = 0; g->w_hi = W;
+    if (world > 1) {
+        // owner-computes: this rank's chunk-aligned record shard (fi_campaign's profile
+        // shard); pass 2 runs the warps holding those records (a warp straddling two
+        // shards runs on both, bit-identically), the image takes the stores of the
+        // warps whose FIRST record is in the shard (each warp has exactly one owner)
+        std::vector<uint64_t> wo(W + 1);
+        GR_TRY(cu(cudaMemcpyAsync(wo.data(), woff, 8ull * (W + 1), cudaMemcpyDeviceToHost, s)));
+        GR_TRY(cu(cudaStreamSynchronize(s)));
+        const uint64_t C = (n_rec + FI_CHUNK - 1) / FI_CHUNK;
+        const uint64_t r0 = std::min<uint64_t>(C * (uint64_t)rank / world * FI_CHUNK, n_rec);
+        const uint64_t r1 = std::min<uint64_t>(C * (uint64_t)(rank + 1) / world * FI_CHUNK, n_rec);
+        uint32_t wa = 0, wb = 0, oa = 0, ob = 0;
+        if (r0 < r1) {
+            wa = (uint32_t)(std::upper_bound(wo.begin(), wo.end() - 1, r0) - wo.begin()) - 1;   // woff[wa] <= r0
+            wb = (uint32_t)(std::lower_bound(wo.begin(), wo.end() - 1, r1) - wo.begin());       // woff[wb] >= r1
+        }
+        oa = (uint32_t)(std::lower_bound(wo.begin(), wo.end() - 1, r0) - wo.begin());
+        ob = (uint32_t)(std::lower_bound(wo.begin(), wo.end() - 1, r1) - wo.begin());
+        g->rec_begin = r0; g->rec_end = r1; g->w_lo = wa; g->w_hi = wb;
+        GR_TRY(fi_golden_trace_jit_range(jit, p, image, &g->t, wa, wb, oa, ob, st, s));
+        return read_status(st, s);
+    }
     // pass 2: trace records, golden store log, checkpoints
     if (jit) GR_TRY(fi_golden_trace_jit(jit, p, image, &g->t, st, s));
     else GR_TRY(fi_golden_trace(p, image, &g->t, st, s));
@@ -137,6 +162,35 @@ extern "C" fi_status fi_golden_run(const fi_program* p, const fi_jit* jit, uint8
     }
     *out = g;
     return FI_OK;
+}
+
+extern "C" fi_status fi_golden_run_shard(const fi_program* p, const fi_jit* jit, uint8_t* image, uint32_t ckpt_interval,
+                                         double ckpt_budget_frac, int rank, int world, fi_golden** out, void* stream) {
+    if (!p || !jit || !image || !out || !p->n_warps || !p->aux || world < 1 || rank < 0 || rank >= world ||
+        p->n_inst != 1)
+        return FI_E_ARG;
+    *out = nullptr;
+    fi_golden* g = new (std::nothrow) fi_golden;
+    if (!g) return FI_E_ARG;
+    g->s = (cudaStream_t)stream;
+    const fi_status e = run(p, jit, image, ckpt_interval, ckpt_budget_frac, g, rank, world);
+    if (e != FI_OK) {
+        g->release(g->s);
+        cudaStreamSynchronize(g->s);
+        delete g;
+        return e;
+    }
+    *out = g;
+    return FI_OK;
+}
+
+extern "C" void fi_golden_shard_range(const fi_golden* g, uint64_t* rec_begin, uint64_t* rec_end, uint32_t* w_lo,
+                                      uint32_t* w_hi) {
+    if (!g) return;
+    if (rec_begin) *rec_begin = g->rec_begin;
+    if (rec_end) *rec_end = g->rec_end;
+    if (w_lo) *w_lo = g->w_lo;
+    if (w_hi) *w_hi = g->w_hi;
 }
 
 extern "C" const fi_trace* fi_golden_trace_of(const fi_golden* g) { return g ? &g->t : nullptr; }

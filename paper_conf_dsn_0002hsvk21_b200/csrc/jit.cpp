@@ -1058,11 +1058,14 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
         // (one launch per instance k, like pass 1: each module serves its own kernel's instances)
         o("extern \"C\" __global__ void __launch_bounds__(128, %u) k_golden_trace_jit(const JArgs A, const u32 k, "
           "const u64* __restrict__ warp_off, const u64* __restrict__ gst_off, uint4* rec, jfi_store* gst, u32* ckpt, "
-          "const u64* __restrict__ ck_off, const u32 ck_interval, u32* status, u8* img_w) {\n"
+          "const u64* __restrict__ ck_off, const u32 ck_interval, u32* status, u8* img_w_all, const u32 w_lo, const u32 w_hi, "
+          "const u32 own_lo, const u32 own_hi) {\n"
           " extern __shared__ u32 jsmem[];\n const u32 lane = threadIdx.x & 31u;\n"
           " u32* Rs = jsmem + (threadIdx.x >> 5) * %uu;\n Rs[%uu + lane] = 0u;\n"
           " const jfi_instance in = A.inst[k];\n const u32 lw = blockIdx.x * 4u + (threadIdx.x >> 5);\n"
           " if (lw >= in.warp_end - in.warp_begin) return;\n const u32 w = in.warp_begin + lw, wpc = (in.block + 31u) / 32u;\n"
+          " if (w < w_lo || w >= w_hi) return;            // another rank's warp (owner-computes golden run)\n"
+          " u8* img_w = (w >= own_lo && w < own_hi) ? img_w_all : (u8*)0;   // image stores: the owner only\n"
           " const u64 r0 = warp_off[w], g0 = gst_off[w];\n"
           " u32* ck = ckpt ? ckpt + ck_off[w] * %uull : (u32*)0;\n"
           " JOut o;\n switch (in.kernel) {\n",
@@ -1170,6 +1173,7 @@ struct fi_jit {
     uint32_t modes = 0;
     std::vector<fi_jit_mod> m;                        // [static kernel]
     uint32_t n_regs = 0, n_code = 0;
+    bool len_sliced = false;                          // golden pass 1 generated as the control slice
     double compile_s = 0;
     size_t src_bytes = 0, cubin_bytes = 0;
 };
@@ -1341,6 +1345,7 @@ extern "C" fi_status fi_jit_build(const fi_program* p, const fi_kernel* kern_hos
         return FI_E_CUDA;
     }
     j->modes = modes;
+    j->len_sliced = (gen_modes & kJitSliceLen) != 0;
     j->n_regs = p->n_regs;
     j->n_code = p->n_code;
     j->src_bytes = src_bytes;
@@ -1351,6 +1356,7 @@ extern "C" fi_status fi_jit_build(const fi_program* p, const fi_kernel* kern_hos
 }
 
 extern "C" double fi_jit_compile_seconds(const fi_jit* j) { return j ? j->compile_s : 0.0; }
+extern "C" int fi_jit_len_sliced(const fi_jit* j) { return j && j->len_sliced ? 1 : 0; }
 
 extern "C" void fi_jit_free(fi_jit* j) {
     if (!j) return;
@@ -1470,6 +1476,12 @@ extern "C" fi_status fi_golden_lengths_jit(const fi_jit* j, const fi_program* p,
 
 extern "C" fi_status fi_golden_trace_jit(const fi_jit* j, const fi_program* p, uint8_t* image, const fi_trace* t,
                                          uint32_t* dev_status, void* stream) {
+    return fi_golden_trace_jit_range(j, p, image, t, 0, p ? p->n_warps : 0, 0, p ? p->n_warps : 0, dev_status, stream);
+}
+
+extern "C" fi_status fi_golden_trace_jit_range(const fi_jit* j, const fi_program* p, uint8_t* image, const fi_trace* t,
+                                               uint32_t w_lo, uint32_t w_hi, uint32_t own_lo, uint32_t own_hi,
+                                               uint32_t* dev_status, void* stream) {
     if (!j || !p || !image || !t || !t->warp_off || !t->gstore_off || !t->rec || !dev_status || !p->aux) return FI_E_ARG;
     if (!(j->modes & FI_JIT_GOLDEN) || j->n_regs != p->n_regs || j->n_code != p->n_code) return FI_E_ARG;
     if (t->ckpt && (!t->ckpt_off || !t->ckpt_interval)) return FI_E_ARG;
@@ -1488,7 +1500,9 @@ extern "C" fi_status fi_golden_trace_jit(const fi_jit* j, const fi_program* p, u
         if (!nw) continue;
         if (p->inst_host[k].kernel >= j->m.size()) return FI_E_ARG;
         uint32_t kk = k;
-        void* args[] = {&A, &kk, (void*)&woff, (void*)&goff, &rec, &gst, &ck, (void*)&ckoff, &iv, &dev_status, &image};
+        if (p->inst_host[k].warp_end <= w_lo || p->inst_host[k].warp_begin >= w_hi) continue;   // no warp of this rank
+        void* args[] = {&A, &kk, (void*)&woff, (void*)&goff, &rec, &gst, &ck, (void*)&ckoff, &iv, &dev_status, &image,
+                        &w_lo, &w_hi, &own_lo, &own_hi};
         fi_status e = launch(j->m[p->inst_host[k].kernel].gtrace, (nw + 3) / 4, j->smem, (cudaStream_t)stream, args);
         if (e) return e;
     }

@@ -66,6 +66,7 @@ struct SelArgs {
     fi_schedule sched;
     uint64_t j0; uint32_t n;
     fi_site* sites; uint32_t* status;
+    uint64_t own_c0, own_c1;                      // owner-computes shard: chunks this rank holds the records of
 };
 
 constexpr int kWarps = 4;
@@ -116,6 +117,15 @@ __global__ void __launch_bounds__(kWarps * 32) k_select(const SelArgs A) {
         r -= total;
     }
 
+    if (c < A.own_c0 || c >= A.own_c1) {          // another rank's records: drawn here, located there
+        if (lane == 0) {
+            fi_site S{};
+            S.s = s; S.group = (uint8_t)g; S.bfm = (uint8_t)bfm; S.u_dst = u_dst; S.u_bit = u_bit;
+            S.mask = bfm_mask(bfm, u_bit); S.flags = FI_SITE_REMOTE;
+            A.sites[i] = S;
+        }
+        return;
+    }
     // scan the chunk's records for the r-th counted lane-instruction of group g
     const uint64_t base = c * FI_CHUNK;
     const uint32_t nrec = (uint32_t)min((uint64_t)FI_CHUNK, A.n_rec - base);
@@ -425,6 +435,80 @@ extern "C" fi_status fi_select_sites(const fi_program* p, const fi_trace* t, con
     for (int g = 0; g < 8; ++g) A.totals[g] = totals_host[g];
     A.sched = *sched;
     A.j0 = j0; A.n = n; A.sites = sites; A.status = dev_status;
+    A.own_c0 = 0; A.own_c1 = ~0ull;
     k_select<<<(n + kWarps - 1) / kWarps, kWarps * 32, 0, (cudaStream_t)stream>>>(A);
+    return launch_status();
+}
+
+extern "C" fi_status fi_select_sites_shard(const fi_program* p, const fi_trace* t, const uint32_t* chunk_counts,
+                                           const void* index, uint32_t n_inst, uint64_t n_chunks,
+                                           const uint64_t totals_host[8], const fi_schedule* sched, uint64_t j0,
+                                           uint32_t n, uint64_t rec_begin, uint64_t rec_end, fi_site* sites,
+                                           uint32_t* dev_status, void* stream) {
+    if (!p || !t || !index || !chunk_counts || !totals_host || !sched || !sites || !dev_status) return FI_E_ARG;
+    if (rec_begin % FI_CHUNK || rec_begin > rec_end || (rec_end % FI_CHUNK && rec_end != t->n_rec)) return FI_E_ARG;
+    fi_status e = check_schedule(sched, totals_host);
+    if (e || n == 0) return e;
+    const IndexLayout L = layout(n_inst, n_chunks);
+    const char* b = reinterpret_cast<const char*>(index);
+    SelArgs A;
+    A.code = p->code; A.kern = p->kern; A.inst = p->inst;
+    A.rec = reinterpret_cast<const uint4*>(t->rec); A.n_rec = t->n_rec; A.warp_off = t->warp_off; A.n_warps = t->n_warps;
+    A.Pk = reinterpret_cast<const uint64_t*>(b + L.pk); A.n_inst = n_inst;
+    A.Pt = reinterpret_cast<const uint64_t*>(b + L.pt); A.n_tiles = n_tiles_of(n_chunks);
+    A.cc = chunk_counts; A.n_chunks = n_chunks;
+    for (int g = 0; g < 8; ++g) A.totals[g] = totals_host[g];
+    A.sched = *sched;
+    A.j0 = j0; A.n = n; A.sites = sites; A.status = dev_status;
+    A.own_c0 = rec_begin / FI_CHUNK;
+    A.own_c1 = (rec_end + FI_CHUNK - 1) / FI_CHUNK;
+    k_select<<<(n + kWarps - 1) / kWarps, kWarps * 32, 0, (cudaStream_t)stream>>>(A);
+    return launch_status();
+}
+
+// Stable compaction of the sites this rank located (flags without FI_SITE_REMOTE):
+// one CTA, 1,024 sites per pass, a block-wide scan of the keep flags; the
+// replica index j0 + i of each kept site goes to out_j.
+namespace fi {
+namespace {
+__global__ void __launch_bounds__(1024) k_compact_sites(const fi_site* __restrict__ in, uint32_t n, uint64_t j0,
+                                                        fi_site* __restrict__ out, uint64_t* __restrict__ out_j,
+                                                        uint32_t* n_out) {
+    __shared__ uint32_t wsum[32];
+    __shared__ uint32_t carry;
+    const uint32_t t = threadIdx.x, lane = t & 31, wid = t >> 5;
+    if (t == 0) carry = 0;
+    __syncthreads();
+    for (uint32_t base = 0; base < n; base += 1024) {
+        const uint32_t i = base + t;
+        const bool keep = i < n && !(in[i].flags & FI_SITE_REMOTE);
+        const uint32_t m = __ballot_sync(0xFFFFFFFFu, keep);
+        if (lane == 0) wsum[wid] = __popc(m);
+        __syncthreads();
+        if (wid == 0) {
+            uint32_t v = wsum[lane], x = v;
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, d);
+                if (lane >= (uint32_t)d) x += y;
+            }
+            wsum[lane] = x - v;                       // exclusive prefix of the warps' counts
+        }
+        __syncthreads();
+        const uint32_t pos = carry + wsum[wid] + __popc(m & ((1u << lane) - 1));
+        if (keep) { out[pos] = in[i]; out_j[pos] = j0 + i; }
+        __syncthreads();
+        if (t == 1023) carry = pos + (keep ? 1u : 0u);
+        __syncthreads();
+    }
+    if (t == 0) *n_out = carry;
+}
+}  // namespace
+}  // namespace fi
+
+extern "C" fi_status fi_compact_sites(const fi_site* sites, uint32_t n, uint64_t j0, fi_site* out, uint64_t* out_j,
+                                      uint32_t* n_out, void* stream) {
+    if (!n_out || (n && (!sites || !out || !out_j))) return FI_E_ARG;
+    fi::k_compact_sites<<<1, 1024, 0, (cudaStream_t)stream>>>(sites, n, j0, out, out_j, n_out);
     return launch_status();
 }

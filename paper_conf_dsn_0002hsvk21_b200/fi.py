@@ -96,7 +96,7 @@ class fi_campaign_cfg(C.Structure):
                 ("n_replicas", C.c_uint64),
                 ("flags", C.c_uint32), ("propagation", C.c_uint32), ("approximate", C.c_uint32),
                 ("ckpt_interval", C.c_uint32), ("engine", C.c_uint32), ("k8_mem_budget", C.c_uint64),
-                ("device", C.c_int), ("stream", C.c_void_p), ("rtol", C.c_double)]
+                ("device", C.c_int), ("stream", C.c_void_p), ("rtol", C.c_double), ("owner_computes", C.c_uint32)]
 
 
 class fi_campaign_result(C.Structure):
@@ -108,7 +108,7 @@ class fi_campaign_result(C.Structure):
                 ("ms_exchange", C.c_float), ("ms_index", C.c_float), ("ms_select", C.c_float),
                 ("ms_inject", C.c_float), ("ms_classify", C.c_float), ("ms_d2h", C.c_float), ("ms_jit", C.c_float),
                 ("sites", C.c_void_p), ("inj", C.c_void_p), ("inst_counts", C.c_void_p),
-                ("hist_tol", C.c_uint64 * 96)]
+                ("hist_tol", C.c_uint64 * 96), ("j", C.c_void_p)]
 
 
 # int allreduce(void* dev, uint64_t count, uint32_t elem_bytes, void* ctx, void* stream)
@@ -837,12 +837,14 @@ class CampaignResult:
     inj: np.ndarray | None
     inst_counts: np.ndarray | None
     hist_tol: np.ndarray | None = None   # rtol > 0: C-12 secondary histogram [8][4][3]
+    j: np.ndarray | None = None          # the replica index of each returned row
 
 
 def campaign(prog, seed: int, groups, bfms, n_replicas: int, rank: int = 0, world: int = 1, allreduce=None,
              unchecked: bool = False, propagation: str = "auto", approximate: bool = False, ckpt="auto",
              k8_mem_budget: int = 0, device: int | None = None, host: dict | None = None,
-             return_arrays: bool = True, engine: str = "jit", rtol: float = 0.0) -> CampaignResult:
+             return_arrays: bool = True, engine: str = "jit", rtol: float = 0.0,
+             owner_computes: bool = False) -> CampaignResult:
     """fi_campaign: the whole campaign of this rank from HOST arrays (golden run,
     sharded profile, count exchange, index, select, inject, classify, histogram
     exchange, D2H).  `host`: optional pinned uint8 tensors keyed code / kernels /
@@ -872,16 +874,20 @@ def campaign(prog, seed: int, groups, bfms, n_replicas: int, rank: int = 0, worl
     cfg.engine = {"interp": 0, "jit": 1}[engine]
     cfg.k8_mem_budget = k8_mem_budget
     cfg.rtol = float(rtol)
+    cfg.owner_computes = 1 if owner_computes else 0
     cfg.device = torch.cuda.current_device() if device is None else device
     cfg.stream = torch.cuda.current_stream(cfg.device).cuda_stream or None
-    n_loc = n_replicas * (rank + 1) // world - n_replicas * rank // world
+    # rows this rank may return: its replica block, or (owner-computes) any replica
+    n_loc = n_replicas if (owner_computes and world > 1) else \
+        n_replicas * (rank + 1) // world - n_replicas * rank // world
     res = fi_campaign_result()
-    sites = inj = ic = None
+    sites = inj = ic = jj = None
     if return_arrays:
         sites = np.zeros(max(n_loc, 1), dtype=SITE_DTYPE)
         inj = np.zeros(max(n_loc, 1), dtype=INJ_DTYPE)
         ic = np.zeros((max(len(prog.instances), 1), 8), dtype=np.uint64)
-        res.sites, res.inj, res.inst_counts = sites.ctypes.data, inj.ctypes.data, ic.ctypes.data
+        jj = np.zeros(max(n_loc, 1), dtype=np.uint64)
+        res.sites, res.inj, res.inst_counts, res.j = sites.ctypes.data, inj.ctypes.data, ic.ctypes.data, jj.ctypes.data
     if world > 1 and allreduce is None:
         allreduce = torch_allreduce()
     cb = allreduce if allreduce is not None else ALLREDUCE_FN()
@@ -891,8 +897,9 @@ def campaign(prog, seed: int, groups, bfms, n_replicas: int, rank: int = 0, worl
     return CampaignResult(np.array(res.hist, dtype=np.uint64).reshape(8, 4, 3), [int(x) for x in res.totals],
                           int(res.n_rec), int(res.counted), int(res.j0), int(res.n_local),
                           (int(res.rec_begin), int(res.rec_end)), int(res.n_unclassified), int(res.n_not_injected),
-                          ms, None if sites is None else sites[:n_loc], None if inj is None else inj[:n_loc], ic,
-                          np.array(res.hist_tol, dtype=np.uint64).reshape(8, 4, 3) if rtol > 0 else None)
+                          ms, None if sites is None else sites[:res.n_local], None if inj is None else inj[:res.n_local],
+                          ic, np.array(res.hist_tol, dtype=np.uint64).reshape(8, 4, 3) if rtol > 0 else None,
+                          None if jj is None else jj[:res.n_local])
 
 
 def campaign_release_memory(device: int = -1) -> None:

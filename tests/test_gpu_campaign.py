@@ -178,3 +178,33 @@ def test_campaign_repeat_reuses_pool_then_release(F):
     F.campaign_release_memory()
     r3 = F.campaign(prog, 11, [F.G_GP], [0, 1, 2, 3], 64)
     assert np.array_equal(r1.hist, r3.hist)
+
+
+@pytest.mark.parametrize("world", [2, 3])
+@pytest.mark.parametrize("maker", [P.c1, lambda: P.c2(full=False), lambda: P.fuzz_program(4),
+                                   lambda: P.vector_add(n=1000)])
+def test_campaign_owner_computes_equals_single(F, world, maker):
+    """Owner-computes: each rank runs the golden pass 2 of its own
+    record shard's warps only, the golden image is completed by one SUM over the
+    writer buffers, and a rank injects exactly the replicas whose site lies in
+    its shard.  Every replica appears on exactly one rank, bit-identical to the
+    world-1 campaign; histograms and counts identical."""
+    prog = maker()
+    seed, groups, bfms, n = 0x0C0C, [F.G_GP, F.G_LD], [0, 1, 2, 3], 300
+    one = F.campaign(prog, seed, groups, bfms, n)
+    parts, calls = _run_world(F, prog, seed, groups, bfms, n, world, owner_computes=True)
+    assert calls == 4                                      # golden image, inst_counts, chunk_counts, histogram
+    j = np.concatenate([p.j for p in parts])
+    assert np.array_equal(np.sort(j), np.arange(n))       # each replica on exactly one rank
+    order = np.argsort(j)
+    sites = np.concatenate([p.sites for p in parts])[order]
+    inj = np.concatenate([p.inj for p in parts])[order]
+    assert np.array_equal(_site_rows(sites), _site_rows(one.sites))
+    assert np.array_equal(inj.view(np.uint8), one.inj.view(np.uint8))
+    for p in parts:
+        assert np.array_equal(p.hist, one.hist)
+        assert np.array_equal(p.inst_counts, one.inst_counts)
+        assert p.totals == one.totals
+        lo, hi = p.rec_range                               # its sites lie in its record shard
+        w0 = np.asarray(p.sites["warp"])
+        assert len(w0) == 0 or (p.n_local == len(p.j))
