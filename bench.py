@@ -377,6 +377,7 @@ def main():
 
     if world == 1:
         line["shard_ratio"] = shard_ratio(camp, n)
+        line["golden_shards"] = golden_shards(camp.dp)
     if camp.peers is not None:
         camp.peers.close()
     if not args.no_e2e:
@@ -421,6 +422,38 @@ def shard_ratio(camp, n, G=8, reps=3):
             "ratio": full / max(blocks), "ideal": G,
             "what": "injection stage (select + K4 + K5) of one rank's replica block [r*n/G,(r+1)*n/G) alone vs all n "
                     "replicas, one GPU, best of 3: the G-GPU injections/s speedup bound"}
+
+
+def golden_shards(dp, G=8, reps=2):
+    """The owner-computes golden run (fi_golden_run_shard) of each rank r of G on
+    this GPU, alone: CUDA events around the one C-ABI call (it synchronizes), best
+    of `reps`.  The G-GPU golden run takes the slowest rank's time."""
+    import torch
+    from paper_conf_dsn_0002hsvk21_b200 import fi
+    if dp.n_inst != 1:
+        return None
+    out = []
+    for r in range(G):
+        best = None
+        for _ in range(reps):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            gt = fi.golden_run(dp, rank=r, world=G)
+            b.record()
+            torch.cuda.synchronize()
+            best = a.elapsed_time(b) if best is None else min(best, a.elapsed_time(b))
+            del gt
+        out.append(best)
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record()
+    gt = fi.golden_run(dp)
+    b.record()
+    torch.cuda.synchronize()
+    del gt
+    full = a.elapsed_time(b)
+    return {"G": G, "full_ms": full, "rank_ms": out, "slowest_rank_ms": max(out), "ratio": full / max(out),
+            "what": "owner-computes golden run (fi_golden_run_shard: sliced pass 1 of all warps, pass 2 of the rank's "
+                    "record shard) of each rank alone on one GPU vs the whole golden run (fi_golden_run)"}
 
 
 def secondary_c4(dev, n=256):
@@ -505,7 +538,8 @@ def e2e(args, prog, seed, groups, bfms, n, rank, world, dev, camp):
             dist.barrier()
         torch.cuda.synchronize()
         t0 = time.perf_counter()
-        r = fi.campaign(prog, seed, groups, bfms, n, rank, world, host=host, engine="jit")
+        r = fi.campaign(prog, seed, groups, bfms, n, rank, world, host=host, engine="jit",
+                        owner_computes=(world > 1 and len(prog.instances) == 1))
         times.append(time.perf_counter() - t0)
         jit_ms.append(r.ms["jit"])
     fi.campaign_release_memory(dev.index if dev.index is not None else -1)

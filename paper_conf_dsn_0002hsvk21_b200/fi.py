@@ -179,6 +179,9 @@ def lib():
             "fi_golden_warp_len": (vp, [vp]),
             "fi_golden_gstore_off_host": (C.POINTER(C.c_uint64), [vp]),
             "fi_golden_free": (st, [vp, vp]),
+            "fi_golden_run_shard": (st, [vp, vp, vp, u32, C.c_double, C.c_int, C.c_int, C.POINTER(vp), vp]),
+            "fi_golden_shard_range": (None, [vp, vp, vp, vp, vp]),
+            "fi_jit_len_sliced": (C.c_int, [vp]),
             "fi_inject_jit": (st, [vp, vp, vp, vp, vp, u32, vp, vp, u32, vp, sz, vp, vp]),
             "fi_write_profile_txt": (st, [vp, vp, u32, vp, u32, vp, sz, C.POINTER(C.c_size_t)]),
             "fi_campaign": (st, [C.POINTER(fi_campaign_cfg), C.c_int, C.c_int, ALLREDUCE_FN, vp,
@@ -362,6 +365,7 @@ class GoldenTrace:
     ckpt_off: torch.Tensor | None = None
     ckpt_interval: int = 0
     owner: object = None         # _GoldenHandle: keeps fi_golden_run's arrays alive
+    shard: tuple = ()            # (rec_begin, rec_end, w_lo, w_hi) of the records / warps pass 2 wrote
 
     @property
     def n_chunks(self):
@@ -393,7 +397,7 @@ class _GoldenHandle:
 
 
 def golden_run(dp: DeviceProgram, ckpt_interval: int | str = "auto", ckpt_budget_frac: float = 0.2,
-               engine: str = "jit") -> GoldenTrace:
+               engine: str = "jit", rank: int = 0, world: int = 1) -> GoldenTrace:
     """fi_golden_run (one C-ABI call): pass 1 (lengths) -> scans + checkpoint
     layout -> pass 2 (trace records, golden store log, checkpoints).
 
@@ -402,7 +406,10 @@ def golden_run(dp: DeviceProgram, ckpt_interval: int | str = "auto", ckpt_budget
     before its site), doubled until the checkpoints fit ckpt_budget_frac of free HBM.
     engine: "jit" (the golden passes on the program's JIT module built with
     FI_JIT_GOLDEN) or "interp" (emu.cuh): bit-identical results.  The trace
-    arrays are owned by the returned GoldenTrace (freed with it)."""
+    arrays are owned by the returned GoldenTrace (freed with it).
+    world > 1 (single-launch program, JIT): fi_golden_run_shard — pass 2 of rank
+    `rank`'s record shard only (GoldenTrace.shard = (rec_begin, rec_end, w_lo, w_hi));
+    the image then holds that rank's warps' golden stores only."""
     jit = dp.jit(FI_JIT_GOLDEN) if engine == "jit" else None
     if engine not in ("jit", "interp"):
         raise ValueError(engine)
@@ -410,9 +417,17 @@ def golden_run(dp: DeviceProgram, ckpt_interval: int | str = "auto", ckpt_budget
     W = dp.n_warps
     h = C.c_void_p()
     ci = FI_CKPT_AUTO if ckpt_interval == "auto" else int(ckpt_interval)
-    _check(lib().fi_golden_run(C.byref(dp.c), jit.h if jit is not None else None, _p(image), ci,
-                               float(ckpt_budget_frac), C.byref(h), _stream()), "fi_golden_run")
+    if world > 1:
+        if jit is None:
+            raise ValueError("the owner-computes golden run needs the JIT engine")
+        _check(lib().fi_golden_run_shard(C.byref(dp.c), jit.h, _p(image), ci, float(ckpt_budget_frac), rank, world,
+                                         C.byref(h), _stream()), "fi_golden_run_shard")
+    else:
+        _check(lib().fi_golden_run(C.byref(dp.c), jit.h if jit is not None else None, _p(image), ci,
+                                   float(ckpt_budget_frac), C.byref(h), _stream()), "fi_golden_run")
     owner = _GoldenHandle(h)
+    sh = (C.c_uint64(), C.c_uint64(), C.c_uint32(), C.c_uint32())
+    lib().fi_golden_shard_range(h, *(C.byref(x) for x in sh))
     tc = fi_trace.from_buffer_copy(lib().fi_golden_trace_of(h).contents)
     d = dp.device
     n_rec, n_gst = int(tc.n_rec), int(lib().fi_golden_gstore_off_host(h)[W])
@@ -427,7 +442,7 @@ def golden_run(dp: DeviceProgram, ckpt_interval: int | str = "auto", ckpt_budget
         n_ck = int(ckoff[W].item())
         ck = device_view(tc.ckpt, max(n_ck * lib().fi_ckpt_bytes(dp.n_regs), 16), 1, d)
     return GoldenTrace(dp, image, wl, woff, goff, rec, gst, n_rec, n_gst, tc, ck, ckoff, int(tc.ckpt_interval),
-                       owner)
+                       owner, tuple(int(x.value) for x in sh))
 
 
 def profile(gt: GoldenTrace, rec_begin: int = 0, rec_end: int | None = None,
