@@ -499,6 +499,13 @@ fi_status fi_golden_run(const fi_program* p, const fi_jit* jit, uint8_t* image, 
 fi_status fi_golden_run_shard(const fi_program* p, const fi_jit* jit, uint8_t* image, uint32_t ckpt_interval,
                               double ckpt_budget_frac, int rank, int world, fi_golden** out, void* stream);
 void fi_golden_shard_range(const fi_golden* g, uint64_t* rec_begin, uint64_t* rec_end, uint32_t* w_lo, uint32_t* w_hi);
+/* The owner-computes partition (host only): from warp_off_host[n_warps+1], rank
+ * r of G's chunk-aligned record shard [rec_begin, rec_end) (fi_campaign's profile
+ * shard), the warps [w_lo, w_hi) holding its records (pass 2 runs them) and the
+ * warps [own_lo, own_hi) whose first record lies in it (they store into the
+ * image).  Over the ranks the own ranges partition every warp with a record. */
+fi_status fi_shard_warps(const uint64_t* warp_off_host, uint32_t n_warps, int rank, int world, uint64_t* rec_begin,
+                         uint64_t* rec_end, uint32_t* w_lo, uint32_t* w_hi, uint32_t* own_lo, uint32_t* own_hi);
 const fi_trace* fi_golden_trace_of(const fi_golden* g);          /* host struct of device pointers */
 const uint64_t* fi_golden_warp_len(const fi_golden* g);          /* device [n_warps] golden steps per warp */
 const uint64_t* fi_golden_gstore_off_host(const fi_golden* g);   /* HOST [n_warps+1] copy of gstore_off */

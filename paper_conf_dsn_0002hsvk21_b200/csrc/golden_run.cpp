@@ -125,16 +125,9 @@ fi_status run(const fi_program* p, const fi_jit* jit, uint8_t* image, uint32_t c
         std::vector<uint64_t> wo(W + 1);
         GR_TRY(cu(cudaMemcpyAsync(wo.data(), woff, 8ull * (W + 1), cudaMemcpyDeviceToHost, s)));
         GR_TRY(cu(cudaStreamSynchronize(s)));
-        const uint64_t C = (n_rec + FI_CHUNK - 1) / FI_CHUNK;
-        const uint64_t r0 = std::min<uint64_t>(C * (uint64_t)rank / world * FI_CHUNK, n_rec);
-        const uint64_t r1 = std::min<uint64_t>(C * (uint64_t)(rank + 1) / world * FI_CHUNK, n_rec);
+        uint64_t r0 = 0, r1 = 0;
         uint32_t wa = 0, wb = 0, oa = 0, ob = 0;
-        if (r0 < r1) {
-            wa = (uint32_t)(std::upper_bound(wo.begin(), wo.end() - 1, r0) - wo.begin()) - 1;   // woff[wa] <= r0
-            wb = (uint32_t)(std::lower_bound(wo.begin(), wo.end() - 1, r1) - wo.begin());       // woff[wb] >= r1
-        }
-        oa = (uint32_t)(std::lower_bound(wo.begin(), wo.end() - 1, r0) - wo.begin());
-        ob = (uint32_t)(std::lower_bound(wo.begin(), wo.end() - 1, r1) - wo.begin());
+        GR_TRY(fi_shard_warps(wo.data(), W, rank, world, &r0, &r1, &wa, &wb, &oa, &ob));
         g->rec_begin = r0; g->rec_end = r1; g->w_lo = wa; g->w_hi = wb;
         GR_TRY(fi_golden_trace_jit_range(jit, p, image, &g->t, wa, wb, oa, ob, st, s));
         return read_status(st, s);
@@ -161,6 +154,29 @@ extern "C" fi_status fi_golden_run(const fi_program* p, const fi_jit* jit, uint8
         return e;
     }
     *out = g;
+    return FI_OK;
+}
+
+extern "C" fi_status fi_shard_warps(const uint64_t* warp_off, uint32_t n_warps, int rank, int world,
+                                    uint64_t* rec_begin, uint64_t* rec_end, uint32_t* w_lo, uint32_t* w_hi,
+                                    uint32_t* own_lo, uint32_t* own_hi) {
+    if (!warp_off || world < 1 || rank < 0 || rank >= world || !rec_begin || !rec_end || !w_lo || !w_hi || !own_lo ||
+        !own_hi)
+        return FI_E_ARG;
+    const uint64_t* b = warp_off;
+    const uint64_t* e = warp_off + n_warps;                  // warp_off[0 .. n_warps) (the last entry is n_rec)
+    const uint64_t n_rec = warp_off[n_warps];
+    const uint64_t C = (n_rec + FI_CHUNK - 1) / FI_CHUNK;
+    const uint64_t r0 = std::min<uint64_t>(C * (uint64_t)rank / world * FI_CHUNK, n_rec);
+    const uint64_t r1 = std::min<uint64_t>(C * (uint64_t)(rank + 1) / world * FI_CHUNK, n_rec);
+    uint32_t wa = 0, wb = 0;
+    if (r0 < r1) {
+        wa = (uint32_t)(std::upper_bound(b, e, r0) - b) - 1;     // last warp starting at or before r0
+        wb = (uint32_t)(std::lower_bound(b, e, r1) - b);         // first warp starting at or after r1
+    }
+    *rec_begin = r0; *rec_end = r1; *w_lo = wa; *w_hi = wb;
+    *own_lo = (uint32_t)(std::lower_bound(b, e, r0) - b);        // warps whose first record is in [r0, r1)
+    *own_hi = (uint32_t)(std::lower_bound(b, e, r1) - b);
     return FI_OK;
 }
 

@@ -182,6 +182,7 @@ def lib():
             "fi_golden_run_shard": (st, [vp, vp, vp, u32, C.c_double, C.c_int, C.c_int, C.POINTER(vp), vp]),
             "fi_golden_shard_range": (None, [vp, vp, vp, vp, vp]),
             "fi_jit_len_sliced": (C.c_int, [vp]),
+            "fi_shard_warps": (st, [vp, u32, C.c_int, C.c_int, vp, vp, vp, vp, vp, vp]),
             "fi_inject_jit": (st, [vp, vp, vp, vp, vp, u32, vp, vp, u32, vp, sz, vp, vp]),
             "fi_write_profile_txt": (st, [vp, vp, u32, vp, u32, vp, sz, C.POINTER(C.c_size_t)]),
             "fi_campaign": (st, [C.POINTER(fi_campaign_cfg), C.c_int, C.c_int, ALLREDUCE_FN, vp,
@@ -915,6 +916,16 @@ def campaign(prog, seed: int, groups, bfms, n_replicas: int, rank: int = 0, worl
                           ms, None if sites is None else sites[:res.n_local], None if inj is None else inj[:res.n_local],
                           ic, np.array(res.hist_tol, dtype=np.uint64).reshape(8, 4, 3) if rtol > 0 else None,
                           None if jj is None else jj[:res.n_local])
+
+
+def shard_warps(warp_off: np.ndarray, rank: int, world: int) -> dict:
+    """fi_shard_warps (host): the owner-computes partition of rank `rank` of `world`."""
+    wo = np.ascontiguousarray(warp_off, dtype=np.uint64)
+    r0, r1 = C.c_uint64(), C.c_uint64()
+    wa, wb, oa, ob = C.c_uint32(), C.c_uint32(), C.c_uint32(), C.c_uint32()
+    _check(lib().fi_shard_warps(wo.ctypes.data, len(wo) - 1, rank, world, C.byref(r0), C.byref(r1), C.byref(wa),
+                                C.byref(wb), C.byref(oa), C.byref(ob)), "fi_shard_warps")
+    return dict(rec=(r0.value, r1.value), run=(wa.value, wb.value), own=(oa.value, ob.value))
 
 
 def campaign_release_memory(device: int = -1) -> None:
