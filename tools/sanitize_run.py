@@ -73,8 +73,13 @@ def main():
     from fi_inputs import programs as P
     from paper_conf_dsn_0002hsvk21_b200 import fi
     torch.cuda.set_device(0)
+    small = "--small" in sys.argv                  # racecheck: C1 and the chain only (it is slow)
     for engine in ("interp", "jit"):
         print("C1", engine, np.bincount(single(fi, P.c1(), 64, [fi.G_GP, fi.G_FP32], engine), minlength=3))
+        if small:
+            print("chain", engine, np.bincount(single(fi, P.multi_instance_chain(3), 32, [fi.G_GP], engine, True),
+                                               minlength=3))
+            continue
         print("mini-C2", engine, np.bincount(single(fi, P.c2(full=False), 24, [fi.G_GP], engine), minlength=3))
         print("chain", engine, np.bincount(single(fi, P.multi_instance_chain(4), 48, [fi.G_GP], engine, True),
                                            minlength=3))
