@@ -18,7 +18,7 @@ FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2", "--expt-re
          "-Xptxas", "-v,-warn-spills"] + ARCH
 SOURCES = ["abi.cpp", "golden.cu", "golden_run.cpp", "scan.cu", "profile.cu", "select.cu", "inject.cu", "propagate.cu", "propagate8.cu",
            "campaign.cpp", "jit.cpp"]
-HEADERS = ["common.cuh", "emu.cuh", "scan.cuh", "jit_prelude.cuh", "jit_k8.h"]
+HEADERS = ["common.cuh", "sem.cuh", "emu.cuh", "scan.cuh", "jit_prelude.cuh", "jit_k8.h"]
 
 
 def _stale(obj: str, deps: list[str]) -> bool:
@@ -30,11 +30,12 @@ def build(force: bool = False, verbose: bool = False) -> str:
     os.makedirs(objdir, exist_ok=True)
     hdrs = [os.path.join(CSRC, h) for h in HEADERS] + [os.path.join(ROOT, "include", "fi.h")]
     # the JIT prelude is embedded into libfi.so as a string (NVRTC compiles it per program)
+    # the JIT prelude is sem.cuh (the §3.2 semantics, shared with emu.cuh) + jit_prelude.cuh
     inc = os.path.join(objdir, "jit_prelude.inc")
-    pre = os.path.join(CSRC, "jit_prelude.cuh")
-    if force or _stale(inc, [pre]):
-        with open(pre) as f, open(inc, "w") as g:
-            g.write('R"FIJITPRELUDE(' + f.read() + ')FIJITPRELUDE"\n')
+    pre = [os.path.join(CSRC, "sem.cuh"), os.path.join(CSRC, "jit_prelude.cuh")]
+    if force or _stale(inc, pre):
+        with open(inc, "w") as g:
+            g.write('R"FIJITPRELUDE(' + "".join(open(x).read() for x in pre) + ')FIJITPRELUDE"\n')
     objs = []
     for src in SOURCES:
         s = os.path.join(CSRC, src)

@@ -39,6 +39,7 @@
 //              the site's instruction; log stores after the site; faults end the run
 #pragma once
 #include "common.cuh"
+#include "sem.cuh"
 
 namespace fi {
 
@@ -152,59 +153,15 @@ __device__ __forceinline__ uint32_t instance_of_warp(const fi_instance* inst, ui
     return lo;
 }
 
-__device__ __forceinline__ float u2f(uint32_t x) { return __uint_as_float(x); }
-__device__ __forceinline__ uint32_t fbits(float f) { return f != f ? kQNaN32 : __float_as_uint(f); }
-__device__ __forceinline__ double u2d(uint64_t x) { return __longlong_as_double((long long)x); }
-__device__ __forceinline__ uint64_t dbits(double d) { return d != d ? kQNaN64 : (uint64_t)__double_as_longlong(d); }
-
-__device__ __forceinline__ uint32_t dev_fmnmx(uint32_t a, uint32_t b, bool mx) {
-    float x = u2f(a), y = u2f(b);
-    bool xn = x != x, yn = y != y;
-    if (xn && yn) return kQNaN32;
-    if (xn) return b;
-    if (yn) return a;
-    if (x == y) {                                   // +0 / -0: -0 < +0 (C-13)
-        bool xneg = a >> 31;
-        return mx ? (xneg ? b : a) : (xneg ? a : b);
-    }
-    return mx ? (x > y ? a : b) : (x < y ? a : b);
-}
-
-__device__ __forceinline__ bool dev_cmp_f(double x, double y, uint32_t c) {
-    if (x != x || y != y) return false;             // ordered compares
-    switch (c) {
-        case 0: return x < y; case 1: return x <= y; case 2: return x > y;
-        case 3: return x >= y; case 4: return x == y; case 5: return x != y;
-    }
-    return false;
-}
-template <class T>
-__device__ __forceinline__ bool dev_cmp_i(T x, T y, uint32_t c) {
-    switch (c) {
-        case 0: return x < y; case 1: return x <= y; case 2: return x > y;
-        case 3: return x >= y; case 4: return x == y; case 5: return x != y;
-    }
-    return false;
-}
-
-__device__ __forceinline__ uint32_t dev_f2i(uint32_t a) {
-    float f = u2f(a);
-    if (f != f) return 0;
-    if (f >= 2147483648.0f) return 0x7FFFFFFFu;
-    if (f < -2147483648.0f) return 0x80000000u;
-    return (uint32_t)__float2int_rz(f);
-}
-
-__device__ __forceinline__ uint32_t dev_lop3(uint32_t a, uint32_t b, uint32_t c, uint32_t lut) {
-    // bit i of lut selects the minterm (i&4 ? a : ~a) & (i&2 ? b : ~b) & (i&1 ? c : ~c)
-    uint32_t r = 0;
-#pragma unroll
-    for (int i = 0; i < 8; ++i) {
-        uint32_t t = ((i & 4) ? a : ~a) & ((i & 2) ? b : ~b) & ((i & 1) ? c : ~c);
-        r |= ((lut >> i) & 1u) ? t : 0u;
-    }
-    return r;
-}
+// the §3.2 opcode semantics: ONE copy, shared with the JIT (sem.cuh)
+using fisem::u2f;
+using fisem::fbits;
+using fisem::u2d;
+using fisem::dbits;
+using fisem::RegFile;
+using fisem::LaneCtx;
+using fisem::exec_plain;
+using fisem::guard_of;
 
 // Image data loads bypass L1 allocation: the small L1 left next to the register
 // files must keep the decoded code, granule map and buffer table resident.
@@ -252,168 +209,6 @@ __device__ __forceinline__ uint32_t check_access(const EmuProg& P, BufCache& C, 
 }
 
 // Register-file access: Rb = this lane's column as a byte pointer, offsets are row*128.
-struct RegFile {
-    char* Rb;              // (char*)(R + lane)
-    uint32_t* R;           // row 0, lane 0
-    uint32_t zb;           // byte offset of the zero row
-    __device__ __forceinline__ uint32_t rd(uint32_t o) const { return *reinterpret_cast<const uint32_t*>(Rb + o); }
-    __device__ __forceinline__ uint64_t rd64(uint32_t o) const {
-        return (uint64_t)rd(o) | ((uint64_t)rd(min(o + 128u, zb)) << 32);
-    }
-    __device__ __forceinline__ void wr(uint32_t o, uint32_t v) const {
-        if (o < zb) *reinterpret_cast<uint32_t*>(Rb + o) = v;
-    }
-};
-
-struct LaneCtx {
-    uint32_t lane, cta, wic, block, grid, cbank_len;
-    const uint32_t* cb;
-};
-
-// One "plain" instruction (everything but BRA / EXIT / LDG / STG) in this lane.
-// All lanes call it together (SHFL needs the whole warp); `ex` = executes here.
-__device__ __forceinline__ void exec_plain(const RegFile& F, const LaneCtx& L, const uint4 D, const bool ex,
-                                           uint32_t& preds) {
-    const uint32_t op = D.x & 0xFF, mod = (D.x >> 16) & 0xFF, pb = D.x >> 24;
-    const uint32_t ia = D.y & 0xFFFF, ib = D.y >> 16, ic = D.z & 0xFFFF, id = D.z >> 16;
-    const uint32_t imm = D.w;
-    if (op == FFMA) {
-        const float x = u2f(F.rd(ia) ^ (mod << 31));
-        const float y = u2f(((mod & 0x80) ? imm : F.rd(ib)) ^ ((mod & 2) << 30));
-        const float z = u2f(F.rd(ic) ^ ((mod & 4) << 29));
-        const uint32_t r = fbits(__fmaf_rn(x, y, z));
-        if (ex) F.wr(id, r);
-        return;
-    }
-    const uint32_t bv = (mod & 0x80) ? imm : F.rd(ib);
-    switch (op) {
-        case MOV: if (ex) F.wr(id, bv); break;
-        case S2R: {
-            uint32_t v = 0;
-            switch (imm) {
-                case 0: v = L.wic * 32 + L.lane; break;
-                case 1: v = L.cta; break;
-                case 2: v = L.block; break;
-                case 3: v = L.grid; break;
-                case 4: v = L.lane; break;
-                case 5: v = L.wic; break;
-            }
-            if (ex) F.wr(id, v);
-            break;
-        }
-        case IADD3: {
-            const uint32_t a = F.rd(ia), c = F.rd(ic);
-            const uint32_t x = (mod & 1) ? 0u - a : a, y = (mod & 2) ? 0u - bv : bv;
-            const uint64_t s = (uint64_t)x + y + c;
-            if (ex) {
-                F.wr(id, (uint32_t)s);
-                if (pb != 7) preds = (preds & ~(1u << pb)) | ((uint32_t)((s >> 32) != 0) << pb);
-            }
-            break;
-        }
-        case IMAD: if (ex) F.wr(id, F.rd(ia) * bv + F.rd(ic)); break;
-        case IMAD_WIDE: {
-            const uint32_t a = F.rd(ia);
-            const uint64_t prod = (mod & 1) ? (uint64_t)a * (uint64_t)bv
-                                            : (uint64_t)((int64_t)(int32_t)a * (int64_t)(int32_t)bv);
-            const uint64_t r = prod + F.rd64(ic);
-            if (ex) { F.wr(id, (uint32_t)r); F.wr(id + 128, (uint32_t)(r >> 32)); }
-            break;
-        }
-        case SHF: {
-            const uint32_t a = F.rd(ia), s = bv > 32 ? 32 : bv, m = mod & 3;
-            uint32_t v;
-            if (m == 0) v = s >= 32 ? 0u : a << s;
-            else if (m == 1) v = s >= 32 ? 0u : a >> s;
-            else v = (uint32_t)((int32_t)a >> (s >= 32 ? 31 : s));
-            if (ex) F.wr(id, v);
-            break;
-        }
-        case LOP3: if (ex) F.wr(id, dev_lop3(F.rd(ia), bv, F.rd(ic), pb)); break;
-        case SEL: {
-            const uint32_t p = pb & 7;
-            const bool s = (((p == 7) ? 1u : ((preds >> p) & 1u)) ^ ((pb >> 3) & 1u)) != 0;
-            if (ex) F.wr(id, s ? F.rd(ia) : bv);
-            break;
-        }
-        case ISETP: case FSETP: case DSETP: {
-            bool v;
-            const uint32_t c = mod & 7;
-            if (op == ISETP) v = (mod & 8) ? dev_cmp_i<uint32_t>(F.rd(ia), bv, c)
-                                           : dev_cmp_i<int32_t>((int32_t)F.rd(ia), (int32_t)bv, c);
-            else if (op == FSETP) v = dev_cmp_f((double)u2f(F.rd(ia)), (double)u2f(F.rd(ib)), c);
-            else v = dev_cmp_f(u2d(F.rd64(ia)), u2d(F.rd64(ib)), c);
-            if (ex && pb != 7) preds = (preds & ~(1u << pb)) | ((uint32_t)v << pb);
-            break;
-        }
-        case FADD: case FMUL: {
-            const float x = u2f(F.rd(ia) ^ (mod << 31));
-            const float y = u2f(bv ^ ((mod & 2) << 30));
-            const float r = op == FADD ? __fadd_rn(x, y) : __fmul_rn(x, y);
-            if (ex) F.wr(id, fbits(r));
-            break;
-        }
-        case FMNMX: if (ex) F.wr(id, dev_fmnmx(F.rd(ia), bv, mod & 1)); break;
-        case DADD: case DMUL: case DFMA: {
-            const double x = u2d(F.rd64(ia) ^ ((uint64_t)(mod & 1) << 63));
-            const double y = u2d(F.rd64(ib) ^ ((uint64_t)(mod & 2) << 62));
-            const double z = u2d(F.rd64(ic) ^ ((uint64_t)(mod & 4) << 61));
-            const double r = op == DADD ? __dadd_rn(x, y) : op == DMUL ? __dmul_rn(x, y) : __fma_rn(x, y, z);
-            const uint64_t b = dbits(r);
-            if (ex) { F.wr(id, (uint32_t)b); F.wr(id + 128, (uint32_t)(b >> 32)); }
-            break;
-        }
-        case LDC: {
-            const uint32_t w0 = imm >> 2;
-            if (ex) {
-                F.wr(id, w0 < L.cbank_len ? __ldg(&L.cb[w0]) : 0u);
-                if (mod & 1) F.wr(id + 128, w0 + 1 < L.cbank_len ? __ldg(&L.cb[w0 + 1]) : 0u);
-            }
-            break;
-        }
-        case I2F: if (ex) F.wr(id, fbits((mod & 1) ? __uint2float_rn(F.rd(ia)) : __int2float_rn((int)F.rd(ia)))); break;
-        case F2I: if (ex) F.wr(id, dev_f2i(F.rd(ia))); break;
-        case F2F_F64_F32: {
-            const uint64_t b = dbits((double)u2f(F.rd(ia)));
-            if (ex) { F.wr(id, (uint32_t)b); F.wr(id + 128, (uint32_t)(b >> 32)); }
-            break;
-        }
-        case F2F_F32_F64: if (ex) F.wr(id, fbits(__double2float_rn(u2d(F.rd64(ia))))); break;
-        case SHFL: {
-            int64_t src;
-            switch (mod & 3) {
-                case 0: src = bv & 31; break;
-                case 1: src = L.lane ^ (bv & 31); break;
-                case 2: src = (int64_t)L.lane + (int64_t)bv; if (src > 31) src = L.lane; break;
-                default: src = (int64_t)L.lane - (int64_t)bv; if (src < 0) src = L.lane; break;
-            }
-            __syncwarp();
-            const uint32_t v = *reinterpret_cast<const uint32_t*>(reinterpret_cast<const char*>(F.R + src) + ia);
-            __syncwarp();
-            if (ex) F.wr(id, v);
-            break;
-        }
-        case MUFU_RCP64: {                            // 1/x in f64, round to nearest (§3.2)
-            const uint64_t b = dbits(__drcp_rn(u2d(F.rd64(ia))));
-            if (ex) { F.wr(id, (uint32_t)b); F.wr(id + 128, (uint32_t)(b >> 32)); }
-            break;
-        }
-        case IMNMX: {
-            const uint32_t a = F.rd(ia);
-            uint32_t v;
-            if (mod & 8) v = (mod & 1) ? max(a, bv) : min(a, bv);
-            else v = (uint32_t)((mod & 1) ? max((int32_t)a, (int32_t)bv) : min((int32_t)a, (int32_t)bv));
-            if (ex) F.wr(id, v);
-            break;
-        }
-        default: break;                               // NOP
-    }
-}
-
-__device__ __forceinline__ bool guard_of(uint32_t guard, uint32_t preds) {
-    const uint32_t gs = guard & 7;
-    return (((gs == 7) ? 1u : ((preds >> gs) & 1u)) ^ ((guard >> 3) & 1u)) != 0;
-}
 
 // Faulty-memory overlay of one replica during downstream propagation (K7): an
 // open-addressing table of 32-bit words {va_lo, va_hi, value, used}; a word

@@ -63,84 +63,22 @@ struct JCtx {
 #define JCTX_BYTES 1280u
 static_assert(sizeof(JCtx) <= JCTX_BYTES, "JCtx fits its smem slot");
 
-__device__ __forceinline__ float ju2f(u32 x) { return __uint_as_float(x); }
-__device__ __forceinline__ u32 jfbits(float f) { return f != f ? JQNAN32 : __float_as_uint(f); }
-__device__ __forceinline__ double ju2d(u64 x) { return __longlong_as_double((long long)x); }
-__device__ __forceinline__ u64 jdbits(double d) { return d != d ? JQNAN64 : (u64)__double_as_longlong(d); }
-__device__ __forceinline__ u64 jpair(u32 lo, u32 hi) { return (u64)lo | ((u64)hi << 32); }
-
-__device__ __forceinline__ u32 jfmnmx(u32 a, u32 b, bool mx) {
-    const float x = ju2f(a), y = ju2f(b);
-    const bool xn = x != x, yn = y != y;
-    if (xn && yn) return JQNAN32;
-    if (xn) return b;
-    if (yn) return a;
-    if (x == y) {                                   // -0 < +0 (C-13)
-        const bool xneg = a >> 31;
-        return mx ? (xneg ? b : a) : (xneg ? a : b);
-    }
-    return mx ? (x > y ? a : b) : (x < y ? a : b);
-}
-
-__device__ __forceinline__ bool jcmp_f(double x, double y, u32 c) {
-    if (x != x || y != y) return false;             // ordered compares
-    switch (c) {
-        case 0: return x < y; case 1: return x <= y; case 2: return x > y;
-        case 3: return x >= y; case 4: return x == y; case 5: return x != y;
-    }
-    return false;
-}
-__device__ __forceinline__ bool jcmp_s(i32 x, i32 y, u32 c) {
-    switch (c) {
-        case 0: return x < y; case 1: return x <= y; case 2: return x > y;
-        case 3: return x >= y; case 4: return x == y; case 5: return x != y;
-    }
-    return false;
-}
-__device__ __forceinline__ bool jcmp_u(u32 x, u32 y, u32 c) {
-    switch (c) {
-        case 0: return x < y; case 1: return x <= y; case 2: return x > y;
-        case 3: return x >= y; case 4: return x == y; case 5: return x != y;
-    }
-    return false;
-}
-
-__device__ __forceinline__ u32 jf2i(u32 a) {
-    const float f = ju2f(a);
-    if (f != f) return 0;
-    if (f >= 2147483648.0f) return 0x7FFFFFFFu;
-    if (f < -2147483648.0f) return 0x80000000u;
-    return (u32)__float2int_rz(f);
-}
-
+// The §3.2 opcode semantics come from sem.cuh (embedded ahead of this file): ONE
+// copy shared with the interpreter (emu.cuh).  The generated code spells them:
+__device__ __forceinline__ float ju2f(u32 x) { return fisem::u2f(x); }
+__device__ __forceinline__ u32 jfbits(float f) { return fisem::fbits(f); }
+__device__ __forceinline__ double ju2d(u64 x) { return fisem::u2d(x); }
+__device__ __forceinline__ u64 jdbits(double d) { return fisem::dbits(d); }
+__device__ __forceinline__ u64 jpair(u32 lo, u32 hi) { return fisem::pair(lo, hi); }
+__device__ __forceinline__ u32 jfmnmx(u32 a, u32 b, bool mx) { return fisem::fmnmx(a, b, mx); }
+__device__ __forceinline__ bool jcmp_f(double x, double y, u32 c) { return fisem::cmp_f(x, y, c); }
+__device__ __forceinline__ bool jcmp_s(i32 x, i32 y, u32 c) { return fisem::cmp_s(x, y, c); }
+__device__ __forceinline__ bool jcmp_u(u32 x, u32 y, u32 c) { return fisem::cmp_u(x, y, c); }
+__device__ __forceinline__ u32 jf2i(u32 a) { return fisem::f2i(a); }
 template <u32 LUT>
-__device__ __forceinline__ u32 jlop3(u32 a, u32 b, u32 c) {
-    u32 r = 0;
-#pragma unroll
-    for (int i = 0; i < 8; ++i) {
-        const u32 t = ((i & 4) ? a : ~a) & ((i & 2) ? b : ~b) & ((i & 1) ? c : ~c);
-        r |= ((LUT >> i) & 1u) ? t : 0u;
-    }
-    return r;
-}
-
-__device__ __forceinline__ u32 jshf(u32 a, u32 bv, u32 m) {
-    const u32 s = bv > 32 ? 32 : bv;
-    if (m == 0) return s >= 32 ? 0u : a << s;
-    if (m == 1) return s >= 32 ? 0u : a >> s;
-    return (u32)((i32)a >> (s >= 32 ? 31 : s));
-}
-
-__device__ __forceinline__ u32 jshfl_src(u32 lane, u32 bv, u32 m) {
-    i64 src;
-    switch (m) {
-        case 0: src = bv & 31; break;
-        case 1: src = lane ^ (bv & 31); break;
-        case 2: src = (i64)lane + (i64)bv; if (src > 31) src = lane; break;
-        default: src = (i64)lane - (i64)bv; if (src < 0) src = lane; break;
-    }
-    return (u32)src;
-}
+__device__ __forceinline__ u32 jlop3(u32 a, u32 b, u32 c) { return fisem::lop3(a, b, c, LUT); }
+__device__ __forceinline__ u32 jshf(u32 a, u32 bv, u32 m) { return fisem::shf(a, bv, m); }
+__device__ __forceinline__ u32 jshfl_src(u32 lane, u32 bv, u32 m) { return fisem::shfl_src(lane, bv, m); }
 
 #ifndef JLD_L1
 #define JLD_L1 ".L1::no_allocate"                    // image loads do not allocate in L1
@@ -258,143 +196,8 @@ struct JState {
 #define JM_LEN 1                                     // golden pass 1: steps / stores counted (+ image stores unless sliced)
 #define JM_TRACE 2                                   // golden pass 2: trace records, store log, checkpoints, image stores
 
-__device__ __forceinline__ bool jguard(u32 guard, u32 preds) {
-    const u32 gs = guard & 7;
-    return (((gs == 7) ? 1u : ((preds >> gs) & 1u)) ^ ((guard >> 3) & 1u)) != 0;
-}
-
-struct JRegs {                                      // this lane's column of the smem register file
-    char* Rb; u32* R; u32 zb;
-    __device__ __forceinline__ u32 rd(u32 o) const { return *reinterpret_cast<const u32*>(Rb + o); }
-    __device__ __forceinline__ u64 rd64(u32 o) const { return (u64)rd(o) | ((u64)rd(min(o + 128u, zb)) << 32); }
-    __device__ __forceinline__ void wr(u32 o, u32 v) const { if (o < zb) *reinterpret_cast<u32*>(Rb + o) = v; }
-};
-
-// one plain instruction (not BRA / EXIT / LDG / STG), all lanes together
-__device__ __forceinline__ void jexec_plain(const JRegs& F, const uint4 D, const bool ex, u32& preds, u32 lane, u32 cta,
-                                            u32 wic, const jfi_instance& in, const u32* cb) {
-    const u32 op = D.x & 0xFF, mod = (D.x >> 16) & 0xFF, pb = D.x >> 24;
-    const u32 ia = D.y & 0xFFFF, ib = D.y >> 16, ic = D.z & 0xFFFF, id = D.z >> 16;
-    const u32 imm = D.w;
-    const u32 bv = (mod & 0x80) ? imm : F.rd(ib);
-    switch (op) {
-        case 16: {                                    // FFMA
-            const float x = ju2f(F.rd(ia) ^ (mod << 31)), y = ju2f(bv ^ ((mod & 2) << 30)), z = ju2f(F.rd(ic) ^ ((mod & 4) << 29));
-            const u32 r = jfbits(__fmaf_rn(x, y, z));
-            if (ex) F.wr(id, r);
-            break;
-        }
-        case 3: if (ex) F.wr(id, bv); break;          // MOV
-        case 4: {                                     // S2R
-            u32 v = 0;
-            switch (imm) {
-                case 0: v = wic * 32 + lane; break; case 1: v = cta; break; case 2: v = in.block; break;
-                case 3: v = in.grid; break; case 4: v = lane; break; case 5: v = wic; break;
-            }
-            if (ex) F.wr(id, v);
-            break;
-        }
-        case 5: {                                     // IADD3
-            const u32 a = F.rd(ia), c = F.rd(ic);
-            const u32 x = (mod & 1) ? 0u - a : a, y = (mod & 2) ? 0u - bv : bv;
-            const u64 s = (u64)x + y + c;
-            if (ex) {
-                F.wr(id, (u32)s);
-                if (pb != 7) preds = (preds & ~(1u << pb)) | ((u32)((s >> 32) != 0) << pb);
-            }
-            break;
-        }
-        case 6: if (ex) F.wr(id, F.rd(ia) * bv + F.rd(ic)); break;      // IMAD
-        case 7: {                                     // IMAD.WIDE
-            const u32 a = F.rd(ia);
-            const u64 prod = (mod & 1) ? (u64)a * (u64)bv : (u64)((i64)(i32)a * (i64)(i32)bv);
-            const u64 r = prod + F.rd64(ic);
-            if (ex) { F.wr(id, (u32)r); F.wr(id + 128, (u32)(r >> 32)); }
-            break;
-        }
-        case 8: { const u32 v = jshf(F.rd(ia), bv, mod & 3); if (ex) F.wr(id, v); break; }     // SHF
-        case 9: {                                     // LOP3 (lut = pb)
-            const u32 a = F.rd(ia), c = F.rd(ic);
-            u32 r = 0;
-#pragma unroll
-            for (int i = 0; i < 8; ++i) {
-                const u32 t = ((i & 4) ? a : ~a) & ((i & 2) ? bv : ~bv) & ((i & 1) ? c : ~c);
-                r |= ((pb >> i) & 1u) ? t : 0u;
-            }
-            if (ex) F.wr(id, r);
-            break;
-        }
-        case 10: {                                    // SEL
-            const u32 p = pb & 7;
-            const bool s = (((p == 7) ? 1u : ((preds >> p) & 1u)) ^ ((pb >> 3) & 1u)) != 0;
-            if (ex) F.wr(id, s ? F.rd(ia) : bv);
-            break;
-        }
-        case 11: case 12: case 13: {                  // ISETP / FSETP / DSETP
-            bool v;
-            const u32 c = mod & 7;
-            if (op == 11) v = (mod & 8) ? jcmp_u(F.rd(ia), bv, c) : jcmp_s((i32)F.rd(ia), (i32)bv, c);
-            else if (op == 12) v = jcmp_f((double)ju2f(F.rd(ia)), (double)ju2f(F.rd(ib)), c);
-            else v = jcmp_f(ju2d(F.rd64(ia)), ju2d(F.rd64(ib)), c);
-            if (ex && pb != 7) preds = (preds & ~(1u << pb)) | ((u32)v << pb);
-            break;
-        }
-        case 14: case 15: {                           // FADD / FMUL
-            const float x = ju2f(F.rd(ia) ^ (mod << 31)), y = ju2f(bv ^ ((mod & 2) << 30));
-            const float r = op == 14 ? __fadd_rn(x, y) : __fmul_rn(x, y);
-            if (ex) F.wr(id, jfbits(r));
-            break;
-        }
-        case 17: if (ex) F.wr(id, jfmnmx(F.rd(ia), bv, mod & 1)); break;  // FMNMX
-        case 18: case 19: case 20: {                  // DADD / DMUL / DFMA
-            const double x = ju2d(F.rd64(ia) ^ ((u64)(mod & 1) << 63));
-            const double y = ju2d(F.rd64(ib) ^ ((u64)(mod & 2) << 62));
-            const double z = ju2d(F.rd64(ic) ^ ((u64)(mod & 4) << 61));
-            const double r = op == 18 ? __dadd_rn(x, y) : op == 19 ? __dmul_rn(x, y) : __fma_rn(x, y, z);
-            const u64 b = jdbits(r);
-            if (ex) { F.wr(id, (u32)b); F.wr(id + 128, (u32)(b >> 32)); }
-            break;
-        }
-        case 22: {                                    // LDC
-            const u32 w0 = imm >> 2;
-            if (ex) {
-                F.wr(id, w0 < in.cbank_len ? __ldg(&cb[w0]) : 0u);
-                if (mod & 1) F.wr(id + 128, w0 + 1 < in.cbank_len ? __ldg(&cb[w0 + 1]) : 0u);
-            }
-            break;
-        }
-        case 24: if (ex) F.wr(id, jfbits((mod & 1) ? __uint2float_rn(F.rd(ia)) : __int2float_rn((int)F.rd(ia)))); break;
-        case 25: if (ex) F.wr(id, jf2i(F.rd(ia))); break;
-        case 26: {                                    // F2F.F64.F32
-            const u64 b = jdbits((double)ju2f(F.rd(ia)));
-            if (ex) { F.wr(id, (u32)b); F.wr(id + 128, (u32)(b >> 32)); }
-            break;
-        }
-        case 27: if (ex) F.wr(id, jfbits(__double2float_rn(ju2d(F.rd64(ia))))); break;     // F2F.F32.F64
-        case 28: {                                    // SHFL: reads the source lane's register even if inactive
-            const u32 src = jshfl_src(lane, bv, mod & 3);
-            __syncwarp();
-            const u32 v = *reinterpret_cast<const u32*>(reinterpret_cast<const char*>(F.R + src) + ia);
-            __syncwarp();
-            if (ex) F.wr(id, v);
-            break;
-        }
-        case 30: {                                    // MUFU.RCP64
-            const u64 b = jdbits(__drcp_rn(ju2d(F.rd64(ia))));
-            if (ex) { F.wr(id, (u32)b); F.wr(id + 128, (u32)(b >> 32)); }
-            break;
-        }
-        case 29: {                                    // IMNMX
-            const u32 a = F.rd(ia);
-            u32 v;
-            if (mod & 8) v = (mod & 1) ? max(a, bv) : min(a, bv);
-            else v = (u32)((mod & 1) ? max((i32)a, (i32)bv) : min((i32)a, (i32)bv));
-            if (ex) F.wr(id, v);
-            break;
-        }
-        default: break;                               // NOP
-    }
-}
+__device__ __forceinline__ bool jguard(u32 guard, u32 preds) { return fisem::guard_of(guard, preds); }
+typedef fisem::RegFile JRegs;                        // this lane's column of the smem register file
 
 // ---------------------------------------------------------------------------
 // K8 (propagate8.cu) on the JIT module: re-execution of instance t for every
@@ -601,7 +404,7 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
                 }
             }
         } else {
-            jexec_plain(F, D, ex, preds, lane, cta, wic, in, cb);
+            fisem::exec_plain(F, fisem::LaneCtx{lane, cta, wic, in.block, in.grid, in.cbank_len, cb}, D, ex, preds);
         }
         if (taken == 0) upc = pcm + 1;
         else if (taken == active) upc = imm;
