@@ -732,6 +732,10 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "jx->nst_[lane] = 0u; jx->fault_[lane] = 0u; jx->fault_pc_[lane] = 0u; jx->before_[lane] = 0u; "
       "jx->after_[lane] = 0u; jx->msk_[lane] = 0u; jx->fired_[lane] = 0u; jx->bad_[lane] = 0u;\n"
       "JBufCache bc; uint4 recbuf = make_uint4(0u, 0u, 0u, 0u); (void)recbuf;\n"
+      "if (jx->bck == k) {                 // this warp's cache from its previous job of the same instance\n"
+      "#pragma unroll\n for (int s_ = 0; s_ < JBC_SLOTS; ++s_) { bc.lo[s_] = jx->bc_[s_ * 4][lane]; "
+      "bc.sz[s_] = jx->bc_[s_ * 4 + 1][lane]; bc.b[s_] = jx->bc_[s_ * 4 + 2][lane]; bc.pb[s_] = jx->bc_[s_ * 4 + 3][lane]; "
+      "bc.z[s_] = (jx->bcz_[lane] >> s_) & 1u; } }\n"
       "// golden trace pass: the last step was a BRA / EXIT; next checkpoint and its threshold step\n"
       "u32 brk = 1u, ckn = 0u, ckx = %s; (void)brk; (void)ckn; (void)ckx;\nu32 lexm_ = 0u; (void)lexm_;\n"
       "// blocks run only within [step, lim): lim = the watchdog, or the injection step while it is pending,\n"
@@ -932,6 +936,11 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "Q4 = (st_.preds >> 4) & 1u; Q5 = (st_.preds >> 5) & 1u; Q6 = (st_.preds >> 6) & 1u;\n"
       "  if (done_) goto finish;\n  continue;\n }\n}\n");
     o("finish:\n");
+    o(" {                                 // the buffer cache for this warp's next job\n"
+      "#pragma unroll\n  for (int s_ = 0; s_ < JBC_SLOTS; ++s_) { jx->bc_[s_ * 4][lane] = bc.lo[s_]; "
+      "jx->bc_[s_ * 4 + 1][lane] = bc.sz[s_]; jx->bc_[s_ * 4 + 2][lane] = bc.b[s_]; jx->bc_[s_ * 4 + 3][lane] = bc.pb[s_]; }\n"
+      "  u32 z_ = 0u;\n#pragma unroll\n  for (int s_ = 0; s_ < JBC_SLOTS; ++s_) z_ |= (u32)bc.z[s_] << s_;\n"
+      "  jx->bcz_[lane] = z_; __syncwarp(); if (lane == 0u) jx->bck = k; __syncwarp(); }\n");
     if (mode == 2)                                    // checkpoints the warp never reached: absent
         o(" if (ck) for (; ckn < (step + ck_interval - 1u) / ck_interval; ++ckn) {\n"
           "   for (u32 r_ = 0u; r_ < %uu; ++r_) ck[(u64)ckn * %uu + r_ * 32u + lane] = 0u;\n"
@@ -981,6 +990,8 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
       " const u32 lane = threadIdx.x & 31u;\n"
       " u32* Rs = jsmem + (threadIdx.x >> 5) * %uu;\n"
       " Rs[%uu + lane] = 0u;                     // the zero row (RZ, indices >= n_regs)\n"
+      " { JCtx* jx0_ = reinterpret_cast<JCtx*>(jsmem + %uu + (threadIdx.x >> 5) * (JCTX_BYTES / 4u)); "
+          "if ((threadIdx.x & 31u) == 0u) jx0_->bck = 0xFFFFFFFFu; __syncwarp(); }\n"
       " for (;;) {\n  u32 p = 0u; if (lane == 0u) p = atomicAdd(counter, 1u); p = __shfl_sync(JFULL, p, 0);\n"
       "  if (p >= n) return;\n  const u32 i = order[p]; const jfi_site S = sites[i];\n"
       "  if (S.flags & 1u) { if (%s && lane == 0u) { jfi_inj r; r.before = r.after = r.mask = r.fault_pc = 0u; "
@@ -991,8 +1002,8 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
       "  const u32 watchdog = wd > 0xFFFFFFFFull ? 0xFFFFFFFFu : (u32)wd;\n"
       "  u32* ck = ckpt ? (u32*)ckpt + ck_off[S.warp] * %uull : (u32*)0;\n"
       "  JOut o; o.start = 0u;\n  switch (in.kernel) {\n",
-      rs, zrow, only <= 0 ? "true" : "false", only < 0 ? "false" : ("in.kernel != " + std::to_string(only) + "u").c_str(),
-      ckw);
+      rs, zrow, 4 * rs, only <= 0 ? "true" : "false",
+      only < 0 ? "false" : ("in.kernel != " + std::to_string(only) + "u").c_str(), ckw);
     for (uint32_t k = 0; k < n_kern; ++k)
         if (mine(k)) o("   case %u: kern_%u_inj(A, S.step, S.pc, S.lane, S.dst_kind, S.dst_reg, S.bfm, S.mask, S.instance, lw / wpc, "
           "lw %% wpc, watchdog, ck, ck ? ck_interval : 0u, log + (u64)i * cap, cap, o, Rs, A.dec + %uu, A.ins + %uu, "
@@ -1010,6 +1021,7 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
         o("extern \"C\" __global__ void __launch_bounds__(128, %u) k8_exec_jit(const JArgs A, const JK8 K, const u32 t) {\n"
           " extern __shared__ u32 jsmem[];\n const u32 lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;\n"
           " u32* Rs = jsmem + wib * %uu;\n Rs[%uu + lane] = 0u;\n"
+          " { JCtx* jx0_ = reinterpret_cast<JCtx*>(jsmem + %uu + (threadIdx.x >> 5) * (JCTX_BYTES / 4u)); if ((threadIdx.x & 31u) == 0u) jx0_->bck = 0xFFFFFFFFu; __syncwarp(); }\n"
           " jfi_store* scr = K.scratch + (u64)(blockIdx.x * 4u + wib) * K.log_cap;\n"
           " const jfi_instance in = A.inst[t];\n const u32 nw = in.warp_end - in.warp_begin, wpc = (in.block + 31u) / 32u;\n"
           " const u64 items = (u64)(*K.n_active) * nw;\n const bool unchecked = K.flags & 1u;\n"
@@ -1021,7 +1033,7 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
           "  JPage pg; pg.ptab = K.ptab + (u64)s * K.total_pages; pg.pool = K.pool; pg.page_base = K.page_base; "
           "pg.last_ref = K.last_ref; pg.dropped = K.dropped + (u64)s * K.dwords; pg.inexact = &K.slot[s].inexact; pg.t = t;\n"
           "  JOut o;\n  switch (in.kernel) {\n",
-          min_blocks, rs, zrow);
+          min_blocks, rs, zrow, 4 * rs);
         for (uint32_t k = 0; k < n_kern; ++k)
             if (mine(k)) o("   case %u: kern_%u_page(A, 0xFFFFFFFFu, 0u, 0u, 0u, 0u, 0u, 0u, t, lw / wpc, lw %% wpc, watchdog, (u32*)0, "
               "0u, scr, K.log_cap, o, Rs, A.dec + %uu, A.ins + %uu, (u8*)0, (uint4*)0, &pg); break;\n",
@@ -1044,10 +1056,11 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
           "u8* img_w, u64* warp_len, u64* warp_nst, u32* status) {\n"
           " extern __shared__ u32 jsmem[];\n const u32 lane = threadIdx.x & 31u;\n"
           " u32* Rs = jsmem + (threadIdx.x >> 5) * %uu;\n Rs[%uu + lane] = 0u;\n"
+          " { JCtx* jx0_ = reinterpret_cast<JCtx*>(jsmem + %uu + (threadIdx.x >> 5) * (JCTX_BYTES / 4u)); if ((threadIdx.x & 31u) == 0u) jx0_->bck = 0xFFFFFFFFu; __syncwarp(); }\n"
           " const jfi_instance in = A.inst[k];\n const u32 lw = blockIdx.x * 4u + (threadIdx.x >> 5);\n"
           " if (lw >= in.warp_end - in.warp_begin) return;\n const u32 wpc = (in.block + 31u) / 32u;\n"
           " JOut o;\n switch (in.kernel) {\n",
-          min_blocks, rs, zrow);
+          min_blocks, rs, zrow, 4 * rs);
         for (uint32_t k = 0; k < n_kern; ++k)
             if (mine(k)) o("  case %u: kern_%u_len(A, 0xFFFFFFFFu, 0u, 0u, 0u, 0u, 0u, 0u, k, lw / wpc, lw %% wpc, 0xFFFFFFFFu, (u32*)0, "
               "0u, (jfi_store*)0, 0u, o, Rs, A.dec + %uu, A.ins + %uu, img_w, (uint4*)0, (const JPage*)0); break;\n",
@@ -1062,6 +1075,7 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
           "const u32 own_lo, const u32 own_hi) {\n"
           " extern __shared__ u32 jsmem[];\n const u32 lane = threadIdx.x & 31u;\n"
           " u32* Rs = jsmem + (threadIdx.x >> 5) * %uu;\n Rs[%uu + lane] = 0u;\n"
+          " { JCtx* jx0_ = reinterpret_cast<JCtx*>(jsmem + %uu + (threadIdx.x >> 5) * (JCTX_BYTES / 4u)); if ((threadIdx.x & 31u) == 0u) jx0_->bck = 0xFFFFFFFFu; __syncwarp(); }\n"
           " const jfi_instance in = A.inst[k];\n const u32 lw = blockIdx.x * 4u + (threadIdx.x >> 5);\n"
           " if (lw >= in.warp_end - in.warp_begin) return;\n const u32 w = in.warp_begin + lw, wpc = (in.block + 31u) / 32u;\n"
           " if (w < w_lo || w >= w_hi) return;            // another rank's warp (owner-computes golden run)\n"
@@ -1069,7 +1083,7 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
           " const u64 r0 = warp_off[w], g0 = gst_off[w];\n"
           " u32* ck = ckpt ? ckpt + ck_off[w] * %uull : (u32*)0;\n"
           " JOut o;\n switch (in.kernel) {\n",
-          min_blocks, rs, zrow, ckw);
+          min_blocks, rs, zrow, 4 * rs, ckw);
         for (uint32_t k = 0; k < n_kern; ++k)
             if (mine(k)) o("  case %u: kern_%u_trace(A, 0xFFFFFFFFu, 0u, 0u, 0u, 0u, 0u, 0u, k, lw / wpc, lw %% wpc, 0xFFFFFFFFu, ck, "
               "ck ? ck_interval : 0u, gst + g0, 0xFFFFFFFFu, o, Rs, A.dec + %uu, A.ins + %uu, img_w, rec + r0, "
@@ -1159,7 +1173,7 @@ thread_local std::string g_jit_log;
 
 // step mode's shared-memory register files: 4 warps x (n_regs + 1) rows x 32 lanes
 // + 4 warps' JCtx (JCTX_BYTES of jit_prelude.cuh)
-static size_t jit_smem(uint32_t n_regs) { return (size_t)4 * (n_regs + 1) * 128 + 4 * 1280; }
+static size_t jit_smem(uint32_t n_regs) { return (size_t)4 * (n_regs + 1) * 128 + 4 * 3584; }
 
 // one CUmodule per static kernel (compiled in parallel: ptxas time grows faster
 // than linearly with the size of one program), each with the entry kernels of

@@ -59,8 +59,14 @@ struct JCtx {
     const JPage* pgp;
     // per lane: warp state block code rarely touches (jit.cpp kCtxLaneNames)
     u32 nst_[32], fault_[32], fault_pc_[32], before_[32], after_[32], msk_[32], fired_[32], bad_[32];
+    // the lane's buffer cache (JBufCache) carried from one job of this CUDA warp to
+    // the next inside a launch: valid while the instance is bck (the writer rule of
+    // an entry depends on the instance); set invalid by every entry kernel
+    u32 bck;
+    u32 bc_[16][32];                                 // [slot * 4 + {lo, sz, b, pb}][lane]
+    u32 bcz_[32];                                    // bit slot: the entry's writer-rule flag
 };
-#define JCTX_BYTES 1280u
+#define JCTX_BYTES 3584u
 static_assert(sizeof(JCtx) <= JCTX_BYTES, "JCtx fits its smem slot");
 
 // The §3.2 opcode semantics come from sem.cuh (embedded ahead of this file): ONE
