@@ -424,33 +424,27 @@ def shard_ratio(camp, n, G=8, reps=3):
                     "replicas, one GPU, best of 3: the G-GPU injections/s speedup bound"}
 
 
-def golden_shards(dp, G=8, reps=2):
+def golden_shards(dp, G=8, reps=3):
     """The owner-computes golden run (fi_golden_run_shard) of each rank r of G on
     this GPU, alone: CUDA events around the one C-ABI call (it synchronizes), best
-    of `reps`.  The G-GPU golden run takes the slowest rank's time."""
+    of `reps` (libfi keeps the device pool's memory mapped between calls).  The G-GPU golden run takes the slowest rank's time."""
     import torch
     from paper_conf_dsn_0002hsvk21_b200 import fi
     if dp.n_inst != 1:
         return None
-    out = []
-    for r in range(G):
+    def best_of(**kw):
         best = None
         for _ in range(reps):
             a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             a.record()
-            gt = fi.golden_run(dp, rank=r, world=G)
+            gt = fi.golden_run(dp, **kw)
             b.record()
             torch.cuda.synchronize()
             best = a.elapsed_time(b) if best is None else min(best, a.elapsed_time(b))
             del gt
-        out.append(best)
-    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    a.record()
-    gt = fi.golden_run(dp)
-    b.record()
-    torch.cuda.synchronize()
-    del gt
-    full = a.elapsed_time(b)
+        return best
+    full = best_of()                      # (the first call also maps the pool the later calls reuse)
+    out = [best_of(rank=r, world=G) for r in range(G)]
     return {"G": G, "full_ms": full, "rank_ms": out, "slowest_rank_ms": max(out), "ratio": full / max(out),
             "what": "owner-computes golden run (fi_golden_run_shard: sliced pass 1 of all warps, pass 2 of the rank's "
                     "record shard) of each rank alone on one GPU vs the whole golden run (fi_golden_run)"}

@@ -18,16 +18,15 @@
 #include "../../include/fi.h"
 #include "common.cuh"
 
-namespace {
-
 // Device allocations of one fi_campaign call, stream-ordered from the device's
 // default memory pool and freed on every return path.  The pool keeps what it
 // holds between calls (release threshold raised once per device), so a repeated
 // campaign reuses its ~48 GB instead of paying cudaMalloc/cudaFree each time;
 // fi_campaign_release_memory() hands it back to the driver.
-void keep_pool(int dev) {
+void fi::keep_pool() {
     static std::once_flag once[64];
-    if (dev < 0 || dev >= 64) return;
+    int dev = -1;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return;
     std::call_once(once[dev], [dev] {
         cudaMemPool_t pool;
         if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
@@ -36,6 +35,8 @@ void keep_pool(int dev) {
         }
     });
 }
+
+namespace {
 struct Arena {
     cudaStream_t s = nullptr;
     std::vector<void*> ptrs;
@@ -151,9 +152,7 @@ extern "C" fi_status fi_campaign(const fi_campaign_cfg* cfg, int rank, int world
         os.own = true;
     }
     cudaStream_t s = os.s;
-    int cur_dev = 0;
-    FI_TRY(cu(cudaGetDevice(&cur_dev)));
-    keep_pool(cur_dev);
+    fi::keep_pool();
     Arena A;
     A.s = s;
     Events ev;

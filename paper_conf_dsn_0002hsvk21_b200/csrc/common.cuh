@@ -126,6 +126,10 @@ inline fi_status cuda_status(cudaError_t e) {
     return FI_E_CUDA;
 }
 inline fi_status launch_status() { return cuda_status(cudaGetLastError()); }
+// raise the release threshold of the current device's default memory pool once, so
+// the stream-ordered allocations of fi_campaign / fi_golden_run stay mapped between
+// calls (fi_campaign_release_memory hands them back)
+void keep_pool();
 }  // namespace fi
 
 #define FI_DEV_ERR(ptr, code) atomicOr((ptr), 1u << (code))

@@ -59,6 +59,7 @@ fi_status read_status(const uint32_t* dev_status, cudaStream_t s) {
 fi_status run(const fi_program* p, const fi_jit* jit, uint8_t* image, uint32_t ckpt_interval, double budget_frac,
               fi_golden* g, int rank = 0, int world = 1) {
     cudaStream_t s = g->s;
+    fi::keep_pool();
     const uint32_t W = p->n_warps;
     uint32_t* st;
     uint64_t *wn, *woff, *goff;

@@ -70,6 +70,7 @@ struct Src {
 
 constexpr int kJbcSlots = 4;                        // JBC_SLOTS of jit_prelude.cuh
 constexpr uint32_t kJitSliceLen = 0x100;            // internal modes bit: golden pass 1 = control slice
+constexpr uint32_t kTmplRecs = 128;                   // golden trace pass: record template per warp (records)
 
 struct Gen {
     uint32_t NR;                                      // register rows (fi_program.n_regs)
@@ -320,8 +321,20 @@ struct Gen {
     // the trace records of block steps [pcm, E] (App. A.3), lanes striding over them:
     // {instance, trace-insn word, active mask, guard-predicate mask}; call before the
     // step counter moves past the block
-    void flush_recs(Src& o, const fi_insn* code, uint32_t L, uint32_t E) const {
+    void flush_recs(Src& o, const fi_insn* code, uint32_t L, uint32_t E, uint32_t tmpl_L = ~0u) const {
         if (mode != 2) return;
+        if (tmpl_L != ~0u) {
+            // the full-warp copy of the templated self-loop (JFW_ = 1 there), entered at
+            // its leader, every guard true for all lanes: the records are the warp's
+            // template with only the position changing — one bulk (TMA) store of the
+            // template from shared memory, issued by lane 0
+            o("   if (JFW_ && pcm == %uu", tmpl_L);
+            std::string all;
+            for (uint32_t q = tmpl_L; q <= E; ++q)
+                if (code[q].guard != 7) all += (all.empty() ? "" : " & ") + std::string("gb_") + std::to_string(q);
+            if (!all.empty()) o(" && (%s) == JFULL", all.c_str());
+            o(") { if (lane == 0u) jbulk_st(&rec_out[step], jtm_, %uu); } else\n", (E + 1 - tmpl_L) * 16);
+        }
         o("   { const u32 n_ = %uu - pcm; for (u32 j_ = lane; j_ < n_; j_ += 32u) { const u32 p_ = pcm + j_; u32 pr_ = JFULL; ",
           E + 1);
         for (uint32_t q = L; q <= E; ++q)
@@ -742,6 +755,10 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "// or the next checkpoint step (golden trace pass)\n"
       "u32 lim = %s;\n", mode == 2 ? "ck ? 0u : 0xFFFFFFFFu" : "0xFFFFFFFFu",
       mode == 0 ? "(hstep >= step && hstep < watchdog) ? hstep : watchdog" : "watchdog");
+    if (mode == 2)
+        o("bool tmpl_ = false; (void)tmpl_;\nuint4* const jtm_ = reinterpret_cast<uint4*>(jsmem + %uu + (threadIdx.x >> 5) * "
+          "%uu); (void)jtm_;   // the warp's record template (after the 4 JCtx)\n",
+          4u * (NR + 1) * 32u + 4u * (3584u / 4u), kTmplRecs * 4u);
     o("for (;;) {\n if (!livem) break;\n u32 pcm, active;\n"
       " if (conv) { pcm = upc; active = amask; }\n"
       " else { pcm = __reduce_min_sync(JFULL, live ? pc : 0xFFFFFFFFu); active = __ballot_sync(JFULL, live && pc == pcm);\n"
@@ -783,6 +800,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
     };
     auto flush_end = [&]() { G.flush_recs(o, code, run_start(n - 1), n - 1); };
     uint32_t batch_end = 0;                           // LDGs [.., batch_end) already emitted as a batch
+    uint32_t tmpl_L = ~0u;                            // the self-loop whose records come from a template
     uint32_t loop_L = ~0u;                            // leader of the self-loop being emitted
     bool loop_dup = false;                            // ... emitted twice (full-warp copy + general)
     std::string loop_saved;                           // the output before that loop's body
@@ -806,6 +824,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
             loop_L = i;
             loop_dup = true;
             for (uint32_t q = i + 1; q < i + blen[i]; ++q) loop_dup = loop_dup && !leader[q];
+            if (loop_dup && mode == 2 && tmpl_L == ~0u && blen[i] <= kTmplRecs) tmpl_L = i;
             if (loop_dup) {
                 loop_saved = std::move(o.s);
                 o.s.clear();
@@ -851,7 +870,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
             };
             o(" { const bool pv = %s; %s", G.guard(I.guard).c_str(), mode == 2 ? "brk = 1u; " : "");
             G.rec(o, I, i, stepx, "pv");
-            G.flush_recs(o, code, run_start(i), i);
+            G.flush_recs(o, code, run_start(i), i, loop_L == I.imm && loop_L == tmpl_L ? tmpl_L : ~0u);
             const RSet keep_ft = use_kill ? lfrom[i + 1] : RSet();
             const RSet keep_tk = use_kill ? (I.imm < n ? lin[I.imm] : RSet()) | lfrom[i + 1] : RSet();
             if (loop_L == I.imm && i + 1 == loop_L + blen[loop_L]) {
@@ -864,10 +883,15 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
                 if (loop_dup) {
                     std::string body = std::move(o.s);
                     o.s = std::move(loop_saved);
-                    o(" if (amask == JFULL) { const bool inA = true; (void)inA;\n for (;;) {  // self-loop %u..%u, full warp\n",
-                      L, i);
+                    o(" if (amask == JFULL) { const bool inA = true; (void)inA;\n");
+                    if (L == tmpl_L)                  // the warp's record template of this block (once per job)
+                        o(" if (!tmpl_) { if (lane == 0u) jbulk_wait_read(); __syncwarp();\n"
+                          "   for (u32 j_ = lane; j_ < %uu; j_ += 32u) jtm_[j_] = make_uint4(k, __ldg(&ins[%uu + j_]), JFULL, JFULL);\n"
+                          "   jfence_async(); __syncwarp(); tmpl_ = true; }\n",
+                          i + 1 - L, L);
+                    o("#undef JFW_\n#define JFW_ 1\n for (;;) {  // self-loop %u..%u, full warp\n", L, i);
                     o.s += body;
-                    o(" } } else {\n for (;;) {  // self-loop %u..%u\n", L, i);
+                    o(" }\n#undef JFW_\n#define JFW_ 0\n } else {\n for (;;) {  // self-loop %u..%u\n", L, i);
                     o.s += body;
                     o(" } }\n");
                 } else {
@@ -941,6 +965,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "jx->bc_[s_ * 4 + 1][lane] = bc.sz[s_]; jx->bc_[s_ * 4 + 2][lane] = bc.b[s_]; jx->bc_[s_ * 4 + 3][lane] = bc.pb[s_]; }\n"
       "  u32 z_ = 0u;\n#pragma unroll\n  for (int s_ = 0; s_ < JBC_SLOTS; ++s_) z_ |= (u32)bc.z[s_] << s_;\n"
       "  jx->bcz_[lane] = z_; __syncwarp(); if (lane == 0u) jx->bck = k; __syncwarp(); }\n");
+    if (mode == 2) o(" if (lane == 0u) jbulk_wait();     // the template stores are complete\n");
     if (mode == 2)                                    // checkpoints the warp never reached: absent
         o(" if (ck) for (; ckn < (step + ck_interval - 1u) / ck_interval; ++ckn) {\n"
           "   for (u32 r_ = 0u; r_ < %uu; ++r_) ck[(u64)ckn * %uu + r_ * 32u + lane] = 0u;\n"
@@ -1174,6 +1199,8 @@ thread_local std::string g_jit_log;
 // step mode's shared-memory register files: 4 warps x (n_regs + 1) rows x 32 lanes
 // + 4 warps' JCtx (JCTX_BYTES of jit_prelude.cuh)
 static size_t jit_smem(uint32_t n_regs) { return (size_t)4 * (n_regs + 1) * 128 + 4 * 3584; }
+// ... + the golden trace pass's 4 record templates (16 B per record)
+static size_t jit_smem_trace(uint32_t n_regs) { return jit_smem(n_regs) + (size_t)4 * kTmplRecs * 16; }
 
 // one CUmodule per static kernel (compiled in parallel: ptxas time grows faster
 // than linearly with the size of one program), each with the entry kernels of
@@ -1183,7 +1210,7 @@ struct fi_jit_mod {
     CUfunction inject = nullptr, glen = nullptr, gtrace = nullptr, k8exec = nullptr;
 };
 struct fi_jit {
-    size_t smem = 0;
+    size_t smem = 0, smem_trace = 0;
     uint32_t modes = 0;
     std::vector<fi_jit_mod> m;                        // [static kernel]
     uint32_t n_regs = 0, n_code = 0;
@@ -1337,6 +1364,7 @@ extern "C" fi_status fi_jit_build(const fi_program* p, const fi_kernel* kern_hos
     if (e) return e;
     fi_jit* j = new fi_jit();
     j->smem = jit_smem(p->n_regs);
+    j->smem_trace = jit_smem_trace(p->n_regs);
     j->m.resize(p->n_kern);
     bool ok = true;
     size_t cubin_bytes = 0;
@@ -1344,13 +1372,16 @@ extern "C" fi_status fi_jit_build(const fi_program* p, const fi_kernel* kern_hos
         fi_jit_mod& M = j->m[k];
         cubin_bytes += cubins[k].size();
         ok = D.load(&M.mod, cubins[k].data()) == CUDA_SUCCESS;
-        auto get = [&](CUfunction* f, const char* name) {
+        auto get = [&](CUfunction* f, const char* name, size_t smem) {
             ok = ok && D.get(f, M.mod, name) == CUDA_SUCCESS &&
-                 D.set_attr(*f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)j->smem) == CUDA_SUCCESS;
+                 D.set_attr(*f, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)smem) == CUDA_SUCCESS;
         };
-        if (modes & FI_JIT_INJECT) get(&M.inject, "k_inject_jit");
-        if (modes & FI_JIT_GOLDEN) { get(&M.glen, "k_golden_len_jit"); get(&M.gtrace, "k_golden_trace_jit"); }
-        if (modes & FI_JIT_PAGE) get(&M.k8exec, "k8_exec_jit");
+        if (modes & FI_JIT_INJECT) get(&M.inject, "k_inject_jit", j->smem);
+        if (modes & FI_JIT_GOLDEN) {
+            get(&M.glen, "k_golden_len_jit", j->smem);
+            get(&M.gtrace, "k_golden_trace_jit", j->smem_trace);
+        }
+        if (modes & FI_JIT_PAGE) get(&M.k8exec, "k8_exec_jit", j->smem);
     }
     if (!ok) {
         g_jit_log += "\ncuModuleLoadData / cuModuleGetFunction / cuFuncSetAttribute failed";
@@ -1517,7 +1548,7 @@ extern "C" fi_status fi_golden_trace_jit_range(const fi_jit* j, const fi_program
         if (p->inst_host[k].warp_end <= w_lo || p->inst_host[k].warp_begin >= w_hi) continue;   // no warp of this rank
         void* args[] = {&A, &kk, (void*)&woff, (void*)&goff, &rec, &gst, &ck, (void*)&ckoff, &iv, &dev_status, &image,
                         &w_lo, &w_hi, &own_lo, &own_hi};
-        fi_status e = launch(j->m[p->inst_host[k].kernel].gtrace, (nw + 3) / 4, j->smem, (cudaStream_t)stream, args);
+        fi_status e = launch(j->m[p->inst_host[k].kernel].gtrace, (nw + 3) / 4, j->smem_trace, (cudaStream_t)stream, args);
         if (e) return e;
     }
     return FI_OK;

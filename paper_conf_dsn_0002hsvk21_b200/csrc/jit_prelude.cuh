@@ -67,6 +67,20 @@ struct JCtx {
     u32 bcz_[32];                                    // bit slot: the entry's writer-rule flag
 };
 #define JCTX_BYTES 3584u
+// golden trace pass: bulk (TMA) stores of a warp's record template from shared
+// memory (jit.cpp flush_recs), evict-first in L2 like the per-lane __stcs records;
+// lane 0 issues them and waits for them before the warp's job ends
+#define JFW_ 0
+__device__ __forceinline__ void jbulk_st(uint4* g, const uint4* s, u32 bytes) {
+    u64 pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group.L2::cache_hint [%0], [%1], %2, %3;\n\t"
+                 "cp.async.bulk.commit_group;" :: "l"(g), "r"((u32)__cvta_generic_to_shared(s)), "r"(bytes), "l"(pol)
+                 : "memory");
+}
+__device__ __forceinline__ void jbulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void jbulk_wait() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void jfence_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 static_assert(sizeof(JCtx) <= JCTX_BYTES, "JCtx fits its smem slot");
 
 // The §3.2 opcode semantics come from sem.cuh (embedded ahead of this file): ONE
