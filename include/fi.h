@@ -450,9 +450,15 @@ fi_status fi_golden_lengths_jit(const fi_jit* j, const fi_program* p, uint8_t* i
 fi_status fi_golden_trace_jit(const fi_jit* j, const fi_program* p, uint8_t* image, const fi_trace* t,
                               uint32_t* dev_status, void* stream);
 /* Pass 2 for the warps [w_lo, w_hi) only, image stores only from the warps
- * [own_lo, own_hi) (the owner-computes golden run of fi_golden_run_shard). */
+ * [own_lo, own_hi) (the owner-computes golden run of fi_golden_run_shard), and
+ * optionally the profile of those warps' records fused into the pass: with
+ * inst_counts ([n_inst][8] u64) and chunk_counts ([ceil(n_rec/FI_CHUNK)][8] u32),
+ * both device and ZEROED by the caller, the call ADDS what fi_profile over the
+ * records of warps [w_lo, w_hi) would write (PAPER.md:78 — the profiler counts
+ * during the golden run); both NULL = no profile; one NULL = FI_E_ARG. */
 fi_status fi_golden_trace_jit_range(const fi_jit* j, const fi_program* p, uint8_t* image, const fi_trace* t,
                                     uint32_t w_lo, uint32_t w_hi, uint32_t own_lo, uint32_t own_hi,
+                                    uint64_t* inst_counts, uint32_t* chunk_counts,
                                     uint32_t* dev_status, void* stream);
 /* 1 when fi_jit_build generated golden pass 1 as the control slice (it then leaves
  * the image untouched; pass 2 writes it), else 0. */
@@ -476,7 +482,9 @@ fi_status fi_classify_batched_jit(const fi_jit* j, const fi_program* p, const ui
  *   ckpt_interval 0 = no checkpoints, FI_CKPT_AUTO = 8192 steps doubled while the
  *                 checkpoints exceed ckpt_budget_frac (<= 0: 0.2) of free HBM
  *   *out          the trace: fi_golden_trace_of(*out) is the fi_trace every later
- *                 call reads (fi_profile, fi_select_sites, fi_inject*, fi_classify*)
+ *                 call reads (fi_profile, fi_select_sites, fi_inject*, fi_classify*),
+ *                 and the run's profile (fi_golden_profile, Fig. 1 step
+ *                 (2)): counted inside pass 2 on the JIT engine, K1 on the interpreter
  * Memory: UNLIKE the calls above, the trace arrays (records, store log,
  * checkpoints, offsets) are sized by pass 1 and allocated by this call,
  * stream-ordered from the current device's default memory pool; *out owns them
@@ -507,6 +515,12 @@ void fi_golden_shard_range(const fi_golden* g, uint64_t* rec_begin, uint64_t* re
 fi_status fi_shard_warps(const uint64_t* warp_off_host, uint32_t n_warps, int rank, int world, uint64_t* rec_begin,
                          uint64_t* rec_end, uint32_t* w_lo, uint32_t* w_hi, uint32_t* own_lo, uint32_t* own_hi);
 const fi_trace* fi_golden_trace_of(const fi_golden* g);          /* host struct of device pointers */
+/* The golden run's profile, Fig. 1 step (2): device pointers (owned by
+ * g) to inst_counts [n_inst][8] u64 and chunk_counts [ceil(n_rec/FI_CHUNK)][8] u32,
+ * equal to what fi_profile(trace, 0, n_rec, ...) writes — counted inside pass 2 on
+ * the JIT engine, by K1 over the finished trace on the interpreter.  FI_E_ARG for
+ * a handle of fi_golden_run_shard with world > 1 (no whole-trace profile). */
+fi_status fi_golden_profile(const fi_golden* g, const uint64_t** inst_counts, const uint32_t** chunk_counts);
 const uint64_t* fi_golden_warp_len(const fi_golden* g);          /* device [n_warps] golden steps per warp */
 const uint64_t* fi_golden_gstore_off_host(const fi_golden* g);   /* HOST [n_warps+1] copy of gstore_off */
 fi_status fi_golden_free(fi_golden* g, void* stream);            /* stream-ordered release; NULL g is a no-op */

@@ -246,32 +246,44 @@ extern "C" fi_status fi_campaign(const fi_campaign_cfg* cfg, int rank, int world
     FI_TRY(cu(cudaMemsetAsync(st, 0, 4, s)));
     FI_TRY(ev.mark(s));                                                    // 2
 
-    // ---- K1 profile (this rank's chunk-aligned shard) + count exchange ------
+    // ---- profile: the golden run's (fused), else K1 over this rank's chunk-aligned
+    // shard + count exchange (owner-computes, approximate profiling) ------------
     const uint64_t n_chunks = (n_rec + FI_CHUNK - 1) / FI_CHUNK;
     const uint64_t c0 = n_chunks * (uint64_t)rank / world, c1 = n_chunks * (uint64_t)(rank + 1) / world;
     const uint64_t r0 = std::min(c0 * FI_CHUNK, n_rec), r1 = std::min(c1 * FI_CHUNK, n_rec);
     uint64_t* ic;
     uint32_t* cc;
-    FI_TRY(A.alloc(&ic, 64ull * K));
-    FI_TRY(A.alloc(&cc, 32ull * std::max<uint64_t>(n_chunks, 1)));
-    FI_TRY(cu(cudaMemsetAsync(cc, 0, 32ull * std::max<uint64_t>(n_chunks, 1), s)));
-    if (cfg->approximate) {
-        // first instance of every static kernel only; every rank
-        // computes the same (small) counts, so there is nothing to exchange.
-        const size_t aws = fi_profile_approx_workspace(cfg->n_kern, K);
-        void* aw;
-        FI_TRY(A.alloc(&aw, aws));
-        FI_TRY(fi_profile_approx(&p, &t, ic, aw, aws, s));
+    const uint64_t* gic = nullptr;
+    const uint32_t* gcc = nullptr;
+    if (!cfg->approximate && fi_golden_profile(gg.g, &gic, &gcc) == FI_OK) {
+        // the golden run counted (fused into pass 2 on the JIT engine): every rank
+        // holds the whole profile, nothing to scan or exchange
+        ic = const_cast<uint64_t*>(gic);
+        cc = const_cast<uint32_t*>(gcc);
         FI_TRY(ev.mark(s));                                                // 3
         FI_TRY(ev.mark(s));                                                // 4
     } else {
-        FI_TRY(fi_profile(&t, r0, r1, K, ic, cc, s));
-        FI_TRY(ev.mark(s));                                                // 3
-        if (world > 1) {
-            if (allreduce(ic, 8ull * K, 8, ctx, s)) return FI_E_COLLECTIVE;
-            if (allreduce(cc, 8ull * n_chunks, 4, ctx, s)) return FI_E_COLLECTIVE;
+        FI_TRY(A.alloc(&ic, 64ull * K));
+        FI_TRY(A.alloc(&cc, 32ull * std::max<uint64_t>(n_chunks, 1)));
+        FI_TRY(cu(cudaMemsetAsync(cc, 0, 32ull * std::max<uint64_t>(n_chunks, 1), s)));
+        if (cfg->approximate) {
+            // first instance of every static kernel only; every rank
+            // computes the same (small) counts, so there is nothing to exchange.
+            const size_t aws = fi_profile_approx_workspace(cfg->n_kern, K);
+            void* aw;
+            FI_TRY(A.alloc(&aw, aws));
+            FI_TRY(fi_profile_approx(&p, &t, ic, aw, aws, s));
+            FI_TRY(ev.mark(s));                                                // 3
+            FI_TRY(ev.mark(s));                                                // 4
+        } else {
+            FI_TRY(fi_profile(&t, r0, r1, K, ic, cc, s));
+            FI_TRY(ev.mark(s));                                                // 3
+            if (world > 1) {
+                if (allreduce(ic, 8ull * K, 8, ctx, s)) return FI_E_COLLECTIVE;
+                if (allreduce(cc, 8ull * n_chunks, 4, ctx, s)) return FI_E_COLLECTIVE;
+            }
+            FI_TRY(ev.mark(s));                                                // 4
         }
-        FI_TRY(ev.mark(s));                                                // 4
     }
 
     // ---- K2 index + totals ---------------------------------------------------

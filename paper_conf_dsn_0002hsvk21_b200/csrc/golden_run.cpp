@@ -22,6 +22,8 @@ struct fi_golden {
     std::vector<uint64_t> gstore_off_h;      // host copy [n_warps + 1]
     uint64_t rec_begin = 0, rec_end = 0;     // this rank's record shard (owner-computes run), else all
     uint32_t w_lo = 0, w_hi = 0;             // warps pass 2 ran
+    uint64_t* inst_counts = nullptr;         // the run's profile (world 1): [n_inst][8]
+    uint32_t* chunk_counts = nullptr;        // ... [ceil(n_rec / FI_CHUNK)][8]
     template <class T>
     fi_status alloc(T** out, size_t bytes) {
         void* p = nullptr;
@@ -130,12 +132,22 @@ fi_status run(const fi_program* p, const fi_jit* jit, uint8_t* image, uint32_t c
         uint32_t wa = 0, wb = 0, oa = 0, ob = 0;
         GR_TRY(fi_shard_warps(wo.data(), W, rank, world, &r0, &r1, &wa, &wb, &oa, &ob));
         g->rec_begin = r0; g->rec_end = r1; g->w_lo = wa; g->w_hi = wb;
-        GR_TRY(fi_golden_trace_jit_range(jit, p, image, &g->t, wa, wb, oa, ob, st, s));
+        GR_TRY(fi_golden_trace_jit_range(jit, p, image, &g->t, wa, wb, oa, ob, nullptr, nullptr, st, s));
         return read_status(st, s);
     }
-    // pass 2: trace records, golden store log, checkpoints
-    if (jit) GR_TRY(fi_golden_trace_jit(jit, p, image, &g->t, st, s));
-    else GR_TRY(fi_golden_trace(p, image, &g->t, st, s));
+    // pass 2: trace records, golden store log, checkpoints — and the profile (K1's
+    // counts): fused into the JIT pass (JProf), else K1 over the written trace
+    const uint64_t n_chunks = (n_rec + FI_CHUNK - 1) / FI_CHUNK;
+    GR_TRY(g->alloc(&g->inst_counts, 64ull * std::max<uint32_t>(p->n_inst, 1)));
+    GR_TRY(g->alloc(&g->chunk_counts, 32ull * std::max<uint64_t>(n_chunks, 1)));
+    GR_TRY(cu(cudaMemsetAsync(g->inst_counts, 0, 64ull * std::max<uint32_t>(p->n_inst, 1), s)));
+    GR_TRY(cu(cudaMemsetAsync(g->chunk_counts, 0, 32ull * std::max<uint64_t>(n_chunks, 1), s)));
+    if (jit) {
+        GR_TRY(fi_golden_trace_jit_range(jit, p, image, &g->t, 0, W, 0, W, g->inst_counts, g->chunk_counts, st, s));
+    } else {
+        GR_TRY(fi_golden_trace(p, image, &g->t, st, s));
+        GR_TRY(fi_profile(&g->t, 0, n_rec, p->n_inst, g->inst_counts, g->chunk_counts, s));
+    }
     return read_status(st, s);                                        // synchronizes
 }
 }  // namespace
@@ -211,6 +223,12 @@ extern "C" void fi_golden_shard_range(const fi_golden* g, uint64_t* rec_begin, u
 }
 
 extern "C" const fi_trace* fi_golden_trace_of(const fi_golden* g) { return g ? &g->t : nullptr; }
+extern "C" fi_status fi_golden_profile(const fi_golden* g, const uint64_t** inst_counts, const uint32_t** chunk_counts) {
+    if (!g || !inst_counts || !chunk_counts || !g->inst_counts) return FI_E_ARG;
+    *inst_counts = g->inst_counts;
+    *chunk_counts = g->chunk_counts;
+    return FI_OK;
+}
 extern "C" const uint64_t* fi_golden_warp_len(const fi_golden* g) { return g ? g->warp_len : nullptr; }
 extern "C" const uint64_t* fi_golden_gstore_off_host(const fi_golden* g) {
     return g ? g->gstore_off_h.data() : nullptr;

@@ -70,7 +70,11 @@ struct Src {
 
 constexpr int kJbcSlots = 4;                        // JBC_SLOTS of jit_prelude.cuh
 constexpr uint32_t kJitSliceLen = 0x100;            // internal modes bit: golden pass 1 = control slice
-constexpr uint32_t kTmplRecs = 128;                   // golden trace pass: record template per warp (records)
+// loop prefetch distance in iterations: a lone warp's K-loop iteration (C2: 73
+// steps, ~210 SASS) issues in ~250 cycles, a quarter of an HBM miss
+constexpr uint32_t kPrefetchIters = 1;
+constexpr uint32_t kTmplRecs = 128;
+constexpr uint32_t kJctxBytes = 3712;                 // JCTX_BYTES of jit_prelude.cuh                   // golden trace pass: record template per warp (records)
 
 struct Gen {
     uint32_t NR;                                      // register rows (fi_program.n_regs)
@@ -333,15 +337,20 @@ struct Gen {
             for (uint32_t q = tmpl_L; q <= E; ++q)
                 if (code[q].guard != 7) all += (all.empty() ? "" : " & ") + std::string("gb_") + std::to_string(q);
             if (!all.empty()) o(" && (%s) == JFULL", all.c_str());
-            o(") { if (lane == 0u) jbulk_st(&rec_out[step], jtm_, %uu); } else\n", (E + 1 - tmpl_L) * 16);
+            o(") { if (lane == 0u) jbulk_st(&rec_out[step], jtm_, %uu);\n"
+              "     if (jx->prof.cc) { const u32 o_ = ((u32)jx->prof.rb + step) & 1023u; if (o_ + %uu < 1024u) { "
+              "if (lane < 8u) jx->prof.pcnt_[lane] += jx->prof.tcnt_[lane]; } else jprof_tmpl_cross(&jx->prof, lane, "
+              "1024u - o_); } } else\n", (E + 1 - tmpl_L) * 16, E + 1 - tmpl_L);
         }
-        o("   { const u32 n_ = %uu - pcm; for (u32 j_ = lane; j_ < n_; j_ += 32u) { const u32 p_ = pcm + j_; u32 pr_ = JFULL; ",
+        o("   { const u32 n_ = %uu - pcm; for (u32 jb_ = 0u; jb_ < n_; jb_ += 32u) { const u32 j_ = jb_ + lane; "
+          "const bool v_ = j_ < n_; const u32 p_ = pcm + j_; u32 pr_ = JFULL; ",
           E + 1);
         for (uint32_t q = L; q <= E; ++q)
             if (code[q].guard != 7) o("if (p_ == %uu) pr_ = gb_%u; ", q, q);
         // streaming stores (evict-first): the 16-B records are written once and read by
         // other kernels, so they must not push the image lines the loads reuse out of L2
-        o("__stcs(&rec_out[step + j_], make_uint4(k, __ldg(&ins[p_]), amask, pr_)); } }\n");
+        o("const u32 w_ = v_ ? __ldg(&ins[p_]) : 0u; if (v_) __stcs(&rec_out[step + j_], make_uint4(k, w_, amask, pr_));\n"
+          "     if (jx->prof.cc) jprof_round(&jx->prof, lane, jx->prof.rb + step + jb_, v_, __popc(amask & pr_), w_ >> 24); } }\n");
     }
     void mem(Src& o, const fi_insn& I, uint32_t pc, const char* stepx) const {
         using namespace fi;
@@ -419,11 +428,29 @@ struct Gen {
         // fast path: every executing lane hits its buffer cache (no table lookups, no
         // cache updates); otherwise the full checks in program order
         // (bitwise, not short-circuit: every test is evaluated, no branches)
+        // A load off the same address register, guard and width as an earlier one of
+        // the batch, at a positive offset delta that is a multiple of the width, only
+        // adds `lo32(va_first) - lo + delta < size16` to the first's check (same buffer,
+        // same high word, same alignment, same writer-rule flag)
         o("  if (__ballot_sync(JFULL, !(true");
         for (uint32_t j = 0; j < m; ++j) {
             const fi_insn& I = code[i0 + j];
             const uint32_t lw = (I.mod & 3) > 2 ? 2 : (I.mod & 3);
-            o(" & (!ex%u | jhit<%d>(bc, va%u, %uu, &z%u))", j, slot(I), j, 4u << lw, j);
+            uint32_t lead = j;
+            for (uint32_t q = 0; q < j && lead == j; ++q) {
+                const fi_insn& Q = code[i0 + q];
+                const uint32_t qw = (Q.mod & 3) > 2 ? 2 : (Q.mod & 3);
+                const int64_t d = (int64_t)(int32_t)I.imm - (int64_t)(int32_t)Q.imm;
+                if (Q.a == I.a && Q.guard == I.guard && qw == lw && slot(Q) == slot(I) && d > 0 && d < 4096 &&
+                    d % (4 << lw) == 0)
+                    lead = q;
+            }
+            if (lead != j) {
+                o(" & (!ex%u | jhit_more<%d>(bc, va%u, %uu, &z%u))", j, slot(I), lead,
+                  (uint32_t)((int64_t)(int32_t)I.imm - (int64_t)(int32_t)code[i0 + lead].imm), j);
+            } else {
+                o(" & (!ex%u | jhit<%d>(bc, va%u, %uu, &z%u))", j, slot(I), j, 4u << lw, j);
+            }
         }
         o("))) {\n");
         for (uint32_t j = 0; j < m; ++j) {
@@ -464,15 +491,17 @@ struct Gen {
                     if (W(I.d0 + q)) o("R%u = v_.%c; ", I.d0 + q, "xyzw"[q]);
             o("}\n");
         }
-        // the next iteration's lines of a loop-carried pointer (address + loop-invariant
-        // stride) into L1 while this iteration computes; a hint only (no architectural
-        // effect), issued only for addresses inside a cached buffer
+        // the lines of a loop-carried pointer (address + loop-invariant stride)
+        // kPrefetchIters iterations ahead into L1 while this one computes; a hint only
+        // (no architectural effect), issued only for addresses inside a cached buffer
         // (one per address pair: the batch's other loads off the same pointer are
         // usually in the same lines)
         for (uint32_t j = 0; j < m && j < stride.size(); ++j) {
             bool first = !stride[j].empty();
             for (uint32_t q = 0; q < j && first; ++q) first = code[i0 + q].a != code[i0 + j].a;
-            if (first) o("  if (ex%u) jprefetch<%d>(jimg, bc, va%u + (%s));\n", j, slot(code[i0 + j]), j, stride[j].c_str());
+            if (first)
+                o("  if (ex%u) jprefetch<%d>(jimg, bc, va%u + %uull * (%s));\n", j, slot(code[i0 + j]), j, kPrefetchIters,
+                  stride[j].c_str());
         }
         o(" }\n");
     }
@@ -758,7 +787,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
     if (mode == 2)
         o("bool tmpl_ = false; (void)tmpl_;\nuint4* const jtm_ = reinterpret_cast<uint4*>(jsmem + %uu + (threadIdx.x >> 5) * "
           "%uu); (void)jtm_;   // the warp's record template (after the 4 JCtx)\n",
-          4u * (NR + 1) * 32u + 4u * (3584u / 4u), kTmplRecs * 4u);
+          4u * (NR + 1) * 32u + 4u * (kJctxBytes / 4u), kTmplRecs * 4u);
     o("for (;;) {\n if (!livem) break;\n u32 pcm, active;\n"
       " if (conv) { pcm = upc; active = amask; }\n"
       " else { pcm = __reduce_min_sync(JFULL, live ? pc : 0xFFFFFFFFu); active = __ballot_sync(JFULL, live && pc == pcm);\n"
@@ -877,9 +906,13 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
                 // the self-loop's back edge (uniform taken, next iteration fits), else its exit
                 const uint32_t L = loop_L;
                 o("lexm_ = amask & __ballot_sync(JFULL, pv); step += %uu - pcm;\n"
-                  "   if (lexm_ == amask && %uu <= npc && step + %uu <= lim%s) { pcm = %uu; %scontinue; } }\n"
+                  "   if (lexm_ == amask && %uu <= npc && step + %uu <= lim%s) { pcm = %uu; %s@@BACK@@ } }\n"
                   "   break;\n",
                   i + 1, L + blen[L], blen[L], mode == 2 ? " && step < ckx" : "", L, entry_kills(L).c_str());
+                auto back = [](std::string b, const std::string& with) {
+                    const size_t at = b.rfind("@@BACK@@");
+                    return b.replace(at, 8, with);
+                };
                 if (loop_dup) {
                     std::string body = std::move(o.s);
                     o.s = std::move(loop_saved);
@@ -887,14 +920,21 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
                     if (L == tmpl_L)                  // the warp's record template of this block (once per job)
                         o(" if (!tmpl_) { if (lane == 0u) jbulk_wait_read(); __syncwarp();\n"
                           "   for (u32 j_ = lane; j_ < %uu; j_ += 32u) jtm_[j_] = make_uint4(k, __ldg(&ins[%uu + j_]), JFULL, JFULL);\n"
-                          "   jfence_async(); __syncwarp(); tmpl_ = true; }\n",
-                          i + 1 - L, L);
-                    o("#undef JFW_\n#define JFW_ 1\n for (;;) {  // self-loop %u..%u, full warp\n", L, i);
-                    o.s += body;
-                    o(" }\n#undef JFW_\n#define JFW_ 0\n } else {\n for (;;) {  // self-loop %u..%u\n", L, i);
-                    o.s += body;
+                          "   jfence_async(); __syncwarp(); tmpl_ = true; if (jx->prof.cc) jprof_tcnt(&jx->prof, lane, %uu, jtm_); }\n",
+                          i + 1 - L, L, i + 1 - L);
+                    // the full-warp copy unrolled twice: ptxas gives half of the loop-carried
+                    // registers alternating homes, copied back on every back edge of a
+                    // one-iteration loop; with two iterations per trip the homes swap roles
+                    o("#undef JFW_\n#define JFW_ 1\n for (;;) {  // self-loop %u..%u, full warp, two iterations per trip\n {\n",
+                      L, i);
+                    o.s += back(body, "goto U" + std::to_string(L) + "_;");
+                    o(" }\n U%u_: ;\n {\n", L);
+                    o.s += back(body, "continue;");
+                    o(" }\n }\n#undef JFW_\n#define JFW_ 0\n } else {\n for (;;) {  // self-loop %u..%u\n", L, i);
+                    o.s += back(body, "continue;");
                     o(" } }\n");
                 } else {
+                    o.s = back(std::move(o.s), "continue;");
                     o(" }\n");
                 }
                 o(" { const u32 exm_ = lexm_;\n");
@@ -947,9 +987,10 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "  __syncwarp();\n"
       "  JBufCache bcs_;                     // (step mode's own cache: bc's address never escapes, so it stays in registers)\n"
       "  const u32 done_ = jinterp<%u>(A, st_, bcs_, Rs, dec, kblen_%u, %uu, k, cta, wic, watchdog, hstep, hpc, hlane, "
-      "hkind, hreg, hbfm, hmask, st_out, st_cap, %uu, img_w, rec_out, ck, ck_interval, ins, pgp, %s);\n"
+      "hkind, hreg, hbfm, hmask, st_out, st_cap, %uu, img_w, rec_out, ck, ck_interval, ins, pgp, %s, %s);\n"
       "  __syncwarp();\n",
-      mode, kid, n, NR, G.sl.empty() ? "(const u8*)0" : ("kslice_" + std::to_string(kid)).c_str());
+      mode, kid, n, NR, G.sl.empty() ? "(const u8*)0" : ("kslice_" + std::to_string(kid)).c_str(),
+      mode == 2 ? "&jx->prof" : "(JProf*)0");
     for (uint32_t j = 0; j < NR; ++j) o("  R%u = Rs[%uu + lane];%s", j, j * 32, (j % 8 == 7) ? "\n" : "");
     o("\n  pc = st_.pc; live = st_.live; step = st_.step; livem = st_.livem; conv = st_.conv; upc = st_.upc; "
       "amask = st_.amask; npc = st_.npc; jx->nst_[lane] = st_.nst; jx->fault_[lane] = st_.fault; "
@@ -1097,15 +1138,19 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
         o("extern \"C\" __global__ void __launch_bounds__(128, %u) k_golden_trace_jit(const JArgs A, const u32 k, "
           "const u64* __restrict__ warp_off, const u64* __restrict__ gst_off, uint4* rec, jfi_store* gst, u32* ckpt, "
           "const u64* __restrict__ ck_off, const u32 ck_interval, u32* status, u8* img_w_all, const u32 w_lo, const u32 w_hi, "
-          "const u32 own_lo, const u32 own_hi) {\n"
+          "const u32 own_lo, const u32 own_hi, u32* pcc, unsigned long long* pic) {\n"
           " extern __shared__ u32 jsmem[];\n const u32 lane = threadIdx.x & 31u;\n"
           " u32* Rs = jsmem + (threadIdx.x >> 5) * %uu;\n Rs[%uu + lane] = 0u;\n"
-          " { JCtx* jx0_ = reinterpret_cast<JCtx*>(jsmem + %uu + (threadIdx.x >> 5) * (JCTX_BYTES / 4u)); if ((threadIdx.x & 31u) == 0u) jx0_->bck = 0xFFFFFFFFu; __syncwarp(); }\n"
+          " JCtx* const jx0_ = reinterpret_cast<JCtx*>(jsmem + %uu + (threadIdx.x >> 5) * (JCTX_BYTES / 4u));\n"
+          " if (lane == 0u) jx0_->bck = 0xFFFFFFFFu;\n __syncwarp();\n"
           " const jfi_instance in = A.inst[k];\n const u32 lw = blockIdx.x * 4u + (threadIdx.x >> 5);\n"
           " if (lw >= in.warp_end - in.warp_begin) return;\n const u32 w = in.warp_begin + lw, wpc = (in.block + 31u) / 32u;\n"
           " if (w < w_lo || w >= w_hi) return;            // another rank's warp (owner-computes golden run)\n"
           " u8* img_w = (w >= own_lo && w < own_hi) ? img_w_all : (u8*)0;   // image stores: the owner only\n"
           " const u64 r0 = warp_off[w], g0 = gst_off[w];\n"
+          " if (lane == 0u) { jx0_->prof.cc = pcc; jx0_->prof.rb = r0; }\n"
+          " if (lane < 8u) { jx0_->prof.pch_[lane] = (u32)(r0 >> 10); jx0_->prof.pcnt_[lane] = 0u; jx0_->prof.ptot_[lane] = 0ull; }\n"
+          " __syncwarp();\n"
           " u32* ck = ckpt ? ckpt + ck_off[w] * %uull : (u32*)0;\n"
           " JOut o;\n switch (in.kernel) {\n",
           min_blocks, rs, zrow, 4 * rs, ckw);
@@ -1116,7 +1161,10 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
               k, k, kern[k].code_off, kern[k].code_off);
         o("  default: o.steps = 0; o.fault = 9; o.nstore = 0; break;\n }\n"
           " if (lane == 0u && (o.fault || o.steps != warp_off[w + 1] - r0 || o.nstore != gst_off[w + 1] - g0)) "
-          "atomicOr(status, 1u << 4);\n}\n");
+          "atomicOr(status, 1u << 4);\n"
+          " if (pcc && lane < 8u) {            // the fused profile: the last chunk's counts, the warp's totals\n"
+          "  jprof_next(&jx0_->prof, lane);\n"
+          "  if (jx0_->prof.ptot_[lane]) atomicAdd(&pic[(u64)k * 8u + lane], (unsigned long long)jx0_->prof.ptot_[lane]); }\n}\n");
     }
     return o.s;
 }
@@ -1198,7 +1246,7 @@ thread_local std::string g_jit_log;
 
 // step mode's shared-memory register files: 4 warps x (n_regs + 1) rows x 32 lanes
 // + 4 warps' JCtx (JCTX_BYTES of jit_prelude.cuh)
-static size_t jit_smem(uint32_t n_regs) { return (size_t)4 * (n_regs + 1) * 128 + 4 * 3584; }
+static size_t jit_smem(uint32_t n_regs) { return (size_t)4 * (n_regs + 1) * 128 + 4 * kJctxBytes; }
 // ... + the golden trace pass's 4 record templates (16 B per record)
 static size_t jit_smem_trace(uint32_t n_regs) { return jit_smem(n_regs) + (size_t)4 * kTmplRecs * 16; }
 
@@ -1474,7 +1522,14 @@ extern "C" fi_status fi_inject_jit(const fi_jit* j, const fi_program* p, const u
             if (e) return e;
         }
         drv().occ(&per, j->m[k].inject, 128, j->smem);
-        const uint32_t grid = (uint32_t)std::min<uint64_t>((n + 3) / 4, (uint64_t)std::max(1, sms * std::max(1, per)));
+        // persistent warps: up to `per` CTAs per SM, fewer when the replicas are few —
+        // a lone warp per SM sub-partition runs its replica ~1.6x faster than three
+        // sharing one (C2: 181 vs 116 emulated steps/us), and with few replicas the
+        // longest one bounds the launch, so one CTA per SM below ~2.5 replicas per
+        // warp slot of that grid, two below ~2.5 per slot of two, else `per`
+        const uint64_t slots = 4ull * (uint64_t)std::max(1, sms);
+        const uint64_t cps = std::min<uint64_t>((uint64_t)std::max(1, per), std::max<uint64_t>(1, (2 * n + 5 * slots - 1) / (5 * slots)));
+        const uint32_t grid = (uint32_t)std::min<uint64_t>((n + 3) / 4, (uint64_t)std::max(1, sms) * cps);
         e = launch(j->m[k].inject, grid, j->smem, s, args);
         if (e) return e;
     }
@@ -1521,12 +1576,15 @@ extern "C" fi_status fi_golden_lengths_jit(const fi_jit* j, const fi_program* p,
 
 extern "C" fi_status fi_golden_trace_jit(const fi_jit* j, const fi_program* p, uint8_t* image, const fi_trace* t,
                                          uint32_t* dev_status, void* stream) {
-    return fi_golden_trace_jit_range(j, p, image, t, 0, p ? p->n_warps : 0, 0, p ? p->n_warps : 0, dev_status, stream);
+    return fi_golden_trace_jit_range(j, p, image, t, 0, p ? p->n_warps : 0, 0, p ? p->n_warps : 0, nullptr, nullptr,
+                                     dev_status, stream);
 }
 
 extern "C" fi_status fi_golden_trace_jit_range(const fi_jit* j, const fi_program* p, uint8_t* image, const fi_trace* t,
                                                uint32_t w_lo, uint32_t w_hi, uint32_t own_lo, uint32_t own_hi,
+                                               uint64_t* inst_counts, uint32_t* chunk_counts,
                                                uint32_t* dev_status, void* stream) {
+    if (!inst_counts != !chunk_counts) return FI_E_ARG;
     if (!j || !p || !image || !t || !t->warp_off || !t->gstore_off || !t->rec || !dev_status || !p->aux) return FI_E_ARG;
     if (!(j->modes & FI_JIT_GOLDEN) || j->n_regs != p->n_regs || j->n_code != p->n_code) return FI_E_ARG;
     if (t->ckpt && (!t->ckpt_off || !t->ckpt_interval)) return FI_E_ARG;
@@ -1547,7 +1605,7 @@ extern "C" fi_status fi_golden_trace_jit_range(const fi_jit* j, const fi_program
         uint32_t kk = k;
         if (p->inst_host[k].warp_end <= w_lo || p->inst_host[k].warp_begin >= w_hi) continue;   // no warp of this rank
         void* args[] = {&A, &kk, (void*)&woff, (void*)&goff, &rec, &gst, &ck, (void*)&ckoff, &iv, &dev_status, &image,
-                        &w_lo, &w_hi, &own_lo, &own_hi};
+                        &w_lo, &w_hi, &own_lo, &own_hi, &chunk_counts, &inst_counts};
         fi_status e = launch(j->m[p->inst_host[k].kernel].gtrace, (nw + 3) / 4, j->smem_trace, (cudaStream_t)stream, args);
         if (e) return e;
     }

@@ -53,6 +53,18 @@ struct JOut {
 // a generated kern_*'s arguments, per warp in shared memory after the 4 warps'
 // step-mode register files (jit.cpp kCtxNames, jit_smem)
 struct JPage;
+// golden pass 2's fused profile: K1's counts (profile.cu) taken
+// while the records are written.  Lane g < 8 keeps group g: pch_ = the chunk of the
+// warp's NEXT record, pcnt_ = its count so far; a finished chunk's count is added
+// to chunk_counts (atomics: a chunk can span two warps) and to the warp's total,
+// which goes to inst_counts at the end
+struct JProf {
+    u32* cc;                                         // chunk_counts [C][8], zeroed by the caller; 0 = off
+    u64 rb;                                          // the warp's first global record
+    u32 pch_[8], pcnt_[8], tcnt_[8];                 // per group: chunk, its count, one template pass's count
+    u64 ptot_[8];                                    // per group: the warp's finished chunks' total
+    u32 tmask_[4][8];                                // [word][group]: template record 32*word + bit has the group
+};
 struct JCtx {
     u32 hstep, hpc, hlane, hkind, hreg, hbfm, hmask, k, cta, wic, watchdog, ck_interval, st_cap;
     u32* ck; jfi_store* st_out; JOut* out; u32* Rs; const uint4* dec; const u32* ins; u8* img_w; uint4* rec_out;
@@ -65,8 +77,9 @@ struct JCtx {
     u32 bck;
     u32 bc_[16][32];                                 // [slot * 4 + {lo, sz, b, pb}][lane]
     u32 bcz_[32];                                    // bit slot: the entry's writer-rule flag
+    JProf prof;                                      // golden pass 2 only
 };
-#define JCTX_BYTES 3584u
+#define JCTX_BYTES 3712u
 // golden trace pass: bulk (TMA) stores of a warp's record template from shared
 // memory (jit.cpp flush_recs), evict-first in L2 like the per-lane __stcs records;
 // lane 0 issues them and waits for them before the warp's job ends
@@ -81,6 +94,72 @@ __device__ __forceinline__ void jbulk_st(uint4* g, const uint4* s, u32 bytes) {
 __device__ __forceinline__ void jbulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
 __device__ __forceinline__ void jbulk_wait() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 __device__ __forceinline__ void jfence_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+
+// ---- the fused profile (JProf): per record, popc(active & pred) thread-level
+// instructions to every group of its trace-insn word's group byte (K1's rule)
+__device__ __forceinline__ void jprof_next(JProf* P, u32 g) {         // lane g < 8: its chunk is complete
+    const u32 v = P->pcnt_[g];
+    if (v) atomicAdd(&P->cc[(u64)P->pch_[g] * 8u + g], v);
+    P->ptot_[g] += v;
+    P->pcnt_[g] = 0u;
+    P->pch_[g] += 1u;
+}
+// up to 32 consecutive records from global record rb0 (the warp's next): lane j's
+// is rb0 + j, valid for a prefix of the lanes, cnt threads, group byte gm
+__device__ __noinline__ void jprof_round(JProf* P, u32 lane, u64 rb0, bool v, u32 cnt, u32 gm) {
+    const u32 b = 1024u - (u32)(rb0 & 1023u);                         // lanes >= b: the next chunk
+    const u32 nv = __popc(__ballot_sync(JFULL, v));
+    u32 lo = 0u, hi = 0u;
+#pragma unroll
+    for (u32 g = 0; g < 8u; ++g) {
+        const u32 x = (v && ((gm >> g) & 1u)) ? cnt : 0u;
+        const u32 s0 = __reduce_add_sync(JFULL, lane < b ? x : 0u);
+        const u32 s1 = b < 32u ? __reduce_add_sync(JFULL, lane < b ? 0u : x) : 0u;
+        if (lane == g) { lo = s0; hi = s1; }
+    }
+    if (lane < 8u) {
+        P->pcnt_[lane] += lo;
+        if (nv >= b) { jprof_next(P, lane); P->pcnt_[lane] = hi; }
+    }
+}
+// the record template's per-group count and membership masks (full warp, every
+// guard true: 32 threads per record)
+__device__ __forceinline__ void jprof_tcnt(JProf* P, u32 lane, u32 n, const uint4* tm) {
+    u32 t = 0u;
+    for (u32 j = 0; j < 128u; j += 32u) {
+        const u32 i = j + lane;
+        const u32 gm = i < n ? tm[i].y >> 24 : 0u;
+#pragma unroll
+        for (u32 g = 0; g < 8u; ++g) {
+            const u32 m = __ballot_sync(JFULL, (gm >> g) & 1u);
+            if (lane == g) { t += 32u * __popc(m); P->tmask_[j >> 5][g] = m; }
+        }
+    }
+    if (lane < 8u) P->tcnt_[lane] = t;
+}
+// a template pass whose first o records end the current chunk
+__device__ __noinline__ void jprof_tmpl_cross(JProf* P, u32 lane, u32 o) {
+    if (lane < 8u) {
+        u32 pre = 0u;
+#pragma unroll
+        for (u32 w = 0; w < 4u; ++w) {
+            const u32 lo = w * 32u;
+            const u32 m = o >= lo + 32u ? 0xFFFFFFFFu : (o > lo ? (1u << (o - lo)) - 1u : 0u);
+            pre += __popc(P->tmask_[w][lane] & m);
+        }
+        pre *= 32u;
+        P->pcnt_[lane] += pre;
+        jprof_next(P, lane);
+        P->pcnt_[lane] = P->tcnt_[lane] - pre;
+    }
+}
+// a step-mode record (the same for every lane): record index r
+__device__ __forceinline__ void jprof_one(JProf* P, u32 lane, u64 r, u32 cnt, u32 gm) {
+    if (lane < 8u) {
+        if ((gm >> lane) & 1u) P->pcnt_[lane] += cnt;
+        if ((r & 1023u) == 1023u) jprof_next(P, lane);
+    }
+}
 static_assert(sizeof(JCtx) <= JCTX_BYTES, "JCtx fits its smem slot");
 
 // The §3.2 opcode semantics come from sem.cuh (embedded ahead of this file): ONE
@@ -150,6 +229,12 @@ __device__ __forceinline__ bool jhit(const JBufCache& C, u64 va, u32 w, bool* ze
     const u32 vlo = (u32)va;
     *zero = C.z[S];
     return ((u32)(va >> 32) == JVA_HI) & ((vlo & (w - 1)) == 0) & (vlo - C.lo[S] < C.sz[S]);
+}
+// the same check for va_first + delta, given jhit(va_first) (jit.cpp ldg_batch)
+template <int S>
+__device__ __forceinline__ bool jhit_more(const JBufCache& C, u64 va_first, u32 delta, bool* zero) {
+    *zero = C.z[S];
+    return (u32)va_first - C.lo[S] + delta < C.sz[S];
 }
 __device__ const uint4 jzero16[1] = {{0u, 0u, 0u, 0u}};   // the zero line of writer-rule loads
 // L1 prefetch of an address inside the buffer cached in entry S (else nothing)
@@ -303,7 +388,7 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
                                     const u32 hmask, jfi_store* __restrict__ st_out, const u32 st_cap,
                                     const u32 zr, u8* __restrict__ img_w, uint4* __restrict__ rec_out,
                                     u32* __restrict__ ck, const u32 ck_interval, const u32* __restrict__ ins,
-                                    const JPage* __restrict__ pg, const u8* __restrict__ slice) {
+                                    const JPage* __restrict__ pg, const u8* __restrict__ slice, JProf* prof) {
     // slice (JM_LEN as the control slice, jit.cpp): 0 = the instruction cannot
     // affect control flow or the store counts — only BRA / EXIT and STG counting
     // run for it (no loads, no image stores)
@@ -351,8 +436,11 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
         const u32 pred = guard == 7 ? JFULL : __ballot_sync(JFULL, pv);
         const bool ex = act && pv;
         const u32 exm = active & pred;
-        if (MODE == JM_TRACE && lane == 0)            // one trace record per step (App. A.3)
-            __stcs(&rec_out[step], make_uint4(k, __ldg(&ins[pcm]), active, pred));
+        if (MODE == JM_TRACE) {                       // one trace record per step (App. A.3)
+            const u32 w = __ldg(&ins[pcm]);
+            if (lane == 0) __stcs(&rec_out[step], make_uint4(k, w, active, pred));
+            if (prof->cc) jprof_one(prof, lane, prof->rb + step, __popc(active & pred), w >> 24);
+        }
         u32 taken = 0;
         brk = op == 1 || op == 2;
         if (MODE == JM_LEN && slice && !slice[pcm] && op != 1 && op != 2) {

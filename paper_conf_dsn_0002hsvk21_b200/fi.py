@@ -174,11 +174,13 @@ def lib():
             "fi_jit_source": (sz, [vp, u32, vp, u32, u32, u32, vp, sz]),
             "fi_golden_lengths_jit": (st, [vp, vp, vp, vp, vp, vp, vp]),
             "fi_golden_trace_jit": (st, [vp, vp, vp, vp, vp, vp]),
+            "fi_golden_trace_jit_range": (st, [vp, vp, vp, vp, u32, u32, u32, u32, vp, vp, vp, vp]),
             "fi_golden_run": (st, [vp, vp, vp, u32, C.c_double, C.POINTER(vp), vp]),
             "fi_golden_trace_of": (C.POINTER(fi_trace), [vp]),
             "fi_golden_warp_len": (vp, [vp]),
             "fi_golden_gstore_off_host": (C.POINTER(C.c_uint64), [vp]),
             "fi_golden_free": (st, [vp, vp]),
+            "fi_golden_profile": (st, [vp, C.POINTER(vp), C.POINTER(vp)]),
             "fi_golden_run_shard": (st, [vp, vp, vp, u32, C.c_double, C.c_int, C.c_int, C.POINTER(vp), vp]),
             "fi_golden_shard_range": (None, [vp, vp, vp, vp, vp]),
             "fi_jit_len_sliced": (C.c_int, [vp]),
@@ -367,6 +369,8 @@ class GoldenTrace:
     ckpt_interval: int = 0
     owner: object = None         # _GoldenHandle: keeps fi_golden_run's arrays alive
     shard: tuple = ()            # (rec_begin, rec_end, w_lo, w_hi) of the records / warps pass 2 wrote
+    inst_counts: torch.Tensor | None = None    # fi_golden_profile (world 1): [K][8] i64
+    chunk_counts: torch.Tensor | None = None   # ... [C][8] i32
 
     @property
     def n_chunks(self):
@@ -442,8 +446,23 @@ def golden_run(dp: DeviceProgram, ckpt_interval: int | str = "auto", ckpt_budget
         ckoff = device_view(tc.ckpt_off, W + 1, 8, d)
         n_ck = int(ckoff[W].item())
         ck = device_view(tc.ckpt, max(n_ck * lib().fi_ckpt_bytes(dp.n_regs), 16), 1, d)
+    ic = cc = None
+    pi, pc = C.c_void_p(), C.c_void_p()
+    if lib().fi_golden_profile(h, C.byref(pi), C.byref(pc)) == FI_OK:
+        ic = device_view(pi.value, max(dp.n_inst, 1) * 8, 8, d).view(max(dp.n_inst, 1), 8)
+        cc = device_view(pc.value, max((n_rec + FI_CHUNK - 1) // FI_CHUNK, 1) * 8, 4, d).view(-1, 8)
     return GoldenTrace(dp, image, wl, woff, goff, rec, gst, n_rec, n_gst, tc, ck, ckoff, int(tc.ckpt_interval),
-                       owner, tuple(int(x.value) for x in sh))
+                       owner, tuple(int(x.value) for x in sh), ic, cc)
+
+
+def golden_profile(gt: GoldenTrace):
+    """fi_golden_profile: the golden run's own profile (inst_counts [K][8] i64,
+    chunk_counts [C][8] i32) — fused into pass 2 on the JIT engine, K1 on the
+    interpreter; what profile(gt) computes over the whole trace.  Views of
+    arrays the GoldenTrace owns."""
+    if gt.inst_counts is None:
+        raise FIError(FI_E_ARG, "fi_golden_profile", "no whole-trace profile (owner-computes shard)")
+    return gt.inst_counts, gt.chunk_counts
 
 
 def profile(gt: GoldenTrace, rec_begin: int = 0, rec_end: int | None = None,

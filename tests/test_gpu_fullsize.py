@@ -13,6 +13,7 @@ Checks:
     (C-14) — every site field, before/after/mask, fault kind/pc
     and outcome identical, no replica left undecided;
   * the GPU golden final image equals the oracle's byte for byte;
+  * the golden run's own (fused) profile equals K1's scan of its trace;
   * a stratified sample again through build_site / inject_local (the checker
     without a golden handle, pinned in tests/test_oracle_pins_local.py).
 """
@@ -65,6 +66,15 @@ def test_c2_all_10000_replicas_vs_oracle(camp, oracle_c2):
     h = camp.hist.cpu().numpy()
     assert (h == O.histogram(osites, oi).astype(np.int64)).all()
     assert set(np.unique(oi["outcome"]).tolist()) == {0, 1, 2}
+
+
+def test_c2_golden_run_profile(camp):
+    """The profile counted inside the JIT golden pass 2 (record templates, chunk
+    crossings inside a block, step mode) equals K1's scan of the written trace."""
+    from paper_conf_dsn_0002hsvk21_b200 import fi
+    gi, gc = fi.golden_profile(camp.gt)
+    assert np.array_equal(gi.cpu().numpy(), camp.inst_counts.cpu().numpy())
+    assert np.array_equal(gc.cpu().numpy(), camp.chunk_counts.cpu().numpy())
 
 
 def test_c2_counts_closed_form(camp):

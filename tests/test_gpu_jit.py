@@ -97,6 +97,13 @@ def _golden_both(F, prog, ckpt):
     assert torch.equal(a.image, b.image), "golden final image"
     assert torch.equal(a.rec[: a.n_rec * 16], b.rec[: b.n_rec * 16]), "trace records"
     assert torch.equal(a.gstore[: a.n_gstore * 16], b.gstore[: b.n_gstore * 16]), "golden store log"
+    # the golden run's profile (fused into the JIT pass 2; K1 inside the interpreter
+    # run) is K1's over the finished trace
+    ic, cc = F.profile(b)
+    for g in (a, b):
+        gi, gc = F.golden_profile(g)
+        assert torch.equal(gi, ic), "golden-run inst_counts"
+        assert torch.equal(gc, cc), "golden-run chunk_counts"
     assert a.ckpt_interval == b.ckpt_interval
     if a.ckpt is not None:
         assert torch.equal(a.ckpt, b.ckpt), "register-file checkpoints"
@@ -109,7 +116,7 @@ def _golden_both(F, prog, ckpt):
                                    P.scatter_chain, lambda: P.c3(full=False), lambda: P.ffma_runs(5)])
 def test_jit_golden_passes(F, maker, ckpt):
     """Golden passes 1 and 2 on the JIT module: lengths, final image, trace records,
-    store log and checkpoints byte-identical to the interpreter's."""
+    store log, checkpoints and the run's profile byte-identical to the interpreter's."""
     _golden_both(F, maker(), ckpt)
 
 
