@@ -1522,14 +1522,7 @@ extern "C" fi_status fi_inject_jit(const fi_jit* j, const fi_program* p, const u
             if (e) return e;
         }
         drv().occ(&per, j->m[k].inject, 128, j->smem);
-        // persistent warps: up to `per` CTAs per SM, fewer when the replicas are few —
-        // a lone warp per SM sub-partition runs its replica ~1.6x faster than three
-        // sharing one (C2: 181 vs 116 emulated steps/us), and with few replicas the
-        // longest one bounds the launch, so one CTA per SM below ~2.5 replicas per
-        // warp slot of that grid, two below ~2.5 per slot of two, else `per`
-        const uint64_t slots = 4ull * (uint64_t)std::max(1, sms);
-        const uint64_t cps = std::min<uint64_t>((uint64_t)std::max(1, per), std::max<uint64_t>(1, (2 * n + 5 * slots - 1) / (5 * slots)));
-        const uint32_t grid = (uint32_t)std::min<uint64_t>((n + 3) / 4, (uint64_t)std::max(1, sms) * cps);
+        const uint32_t grid = (uint32_t)std::min<uint64_t>((n + 3) / 4, (uint64_t)std::max(1, sms * std::max(1, per)));
         e = launch(j->m[k].inject, grid, j->smem, s, args);
         if (e) return e;
     }
