@@ -179,23 +179,22 @@ __device__ __forceinline__ u32 jlop3(u32 a, u32 b, u32 c) { return fisem::lop3(a
 __device__ __forceinline__ u32 jshf(u32 a, u32 bv, u32 m) { return fisem::shf(a, bv, m); }
 __device__ __forceinline__ u32 jshfl_src(u32 lane, u32 bv, u32 m) { return fisem::shfl_src(lane, bv, m); }
 
-#ifndef JLD_L1
-#define JLD_L1 ".L1::no_allocate"                    // image loads do not allocate in L1
-#endif
+// image loads: read-only path, allocating in L1 (a CTA's warps share lines in the
+// golden passes; the loop prefetch puts the next iteration's lines there) — 3-5 %
+// faster than .L1::no_allocate for K4 and golden pass 2 on C2
 __device__ __forceinline__ u32 jld32(const u8* p) {
     u32 r;
-    asm volatile("ld.global.nc" JLD_L1 ".u32 %0, [%1];" : "=r"(r) : "l"(p));
+    asm volatile("ld.global.nc.u32 %0, [%1];" : "=r"(r) : "l"(p));
     return r;
 }
 __device__ __forceinline__ uint2 jld64(const u8* p) {
     uint2 r;
-    asm volatile("ld.global.nc" JLD_L1 ".v2.u32 {%0, %1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p));
+    asm volatile("ld.global.nc.v2.u32 {%0, %1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p));
     return r;
 }
 __device__ __forceinline__ uint4 jld128(const u8* p) {
     uint4 r;
-    asm volatile("ld.global.nc" JLD_L1 ".v4.u32 {%0, %1, %2, %3}, [%4];"
-                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+    asm volatile("ld.global.nc.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
     return r;
 }
 
