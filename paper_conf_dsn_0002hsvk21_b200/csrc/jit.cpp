@@ -459,15 +459,15 @@ struct Gen {
             o("   c%u = ex%u ? jcheck<%d>(A, bc, va%u, %uu, k, &z%u%s) : 0u;\n", j, j, slot(I), j, 4u << lw, j,
               mode == 3 ? ", PG.page_base" : "");
         }
-        o("  }\n");
-        o("  if (__ballot_sync(JFULL, 0u");
+        // (a fault needs a lane that missed its cache: the fault ballots are on the slow path only)
+        o("   if (__ballot_sync(JFULL, 0u");
         for (uint32_t j = 0; j < m; ++j) o(" | c%u", j);
         o(")) {\n");
         for (uint32_t j = 0; j < m; ++j)
-            o("   if (__ballot_sync(JFULL, c%u != 0u)) { fault = __ballot_sync(JFULL, c%u == 1u) ? 1u : 2u; "
+            o("    if (__ballot_sync(JFULL, c%u != 0u)) { fault = __ballot_sync(JFULL, c%u == 1u) ? 1u : 2u; "
               "fault_pc = %uu; step = step + (%uu - pcm); goto finish; }\n",
               j, j, i0 + j, i0 + j);
-        o("  }\n");
+        o("   }\n  }\n");
         for (uint32_t j = 0; j < m; ++j) {
             char sx[64], pvn[16];
             std::snprintf(sx, sizeof sx, "step + (%uu - pcm)", i0 + j);
