@@ -500,7 +500,8 @@ struct Gen {
             bool first = !stride[j].empty();
             for (uint32_t q = 0; q < j && first; ++q) first = code[i0 + q].a != code[i0 + j].a;
             if (first)
-                o("  if (ex%u) jprefetch<%d>(jimg, bc, va%u + %uull * (%s));\n", j, slot(code[i0 + j]), j, kPrefetchIters,
+                o("  if (ex%u) jprefetch<%d>(jimg, bc, va%u + %uull * (%s));\n", j, slot(code[i0 + j]), j,
+                  getenv("FI_EXP_PFD") ? (uint32_t)atoi(getenv("FI_EXP_PFD")) : kPrefetchIters,   // EXPERIMENT
                   stride[j].c_str());
         }
         o(" }\n");
