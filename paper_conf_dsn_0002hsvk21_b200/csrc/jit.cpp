@@ -70,8 +70,8 @@ struct Src {
 
 constexpr int kJbcSlots = 4;                        // JBC_SLOTS of jit_prelude.cuh
 constexpr uint32_t kJitSliceLen = 0x100;            // internal modes bit: golden pass 1 = control slice
-// loop prefetch distance in iterations: a lone warp's K-loop iteration (C2: 73
-// steps, ~210 SASS) issues in ~250 cycles, a quarter of an HBM miss
+// loop prefetch distance in iterations (C2, K4 / golden pass 2: 1 -> 6.37 / 14.8 ms,
+// 2 -> 6.62 / 15.1, 3 -> 6.62 / 15.1, none -> 6.86 / 20.1; profiles/r02/k4_prefetch_distance.log)
 constexpr uint32_t kPrefetchIters = 1;
 constexpr uint32_t kTmplRecs = 128;
 constexpr uint32_t kJctxBytes = 3712;                 // JCTX_BYTES of jit_prelude.cuh                   // golden trace pass: record template per warp (records)
@@ -500,8 +500,7 @@ struct Gen {
             bool first = !stride[j].empty();
             for (uint32_t q = 0; q < j && first; ++q) first = code[i0 + q].a != code[i0 + j].a;
             if (first)
-                o("  if (ex%u) jprefetch<%d>(jimg, bc, va%u + %uull * (%s));\n", j, slot(code[i0 + j]), j,
-                  getenv("FI_EXP_PFD") ? (uint32_t)atoi(getenv("FI_EXP_PFD")) : kPrefetchIters,   // EXPERIMENT
+                o("  if (ex%u) jprefetch<%d>(jimg, bc, va%u + %uull * (%s));\n", j, slot(code[i0 + j]), j, kPrefetchIters,
                   stride[j].c_str());
         }
         o(" }\n");
