@@ -415,7 +415,9 @@ void launch_lpt_order(const fi_program* p, const fi_site* sites, const uint64_t*
 
 using namespace fi;
 
-extern "C" size_t fi_inject_workspace(uint32_t n) { return 256 + (size_t)n * 4; }
+// [0, 256): queue counter and the emulated-step count; then the LPT order (u32 per
+// replica); then the JIT engine's per-SM deal counters (u32 per SM, up to 256 SMs)
+extern "C" size_t fi_inject_workspace(uint32_t n) { return 256 + (((size_t)n * 4 + 255) & ~(size_t)255) + 1024; }
 
 extern "C" fi_status fi_inject(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,
                                uint32_t n, fi_inj* out, fi_store* log, uint32_t log_cap, void* ws, size_t ws_bytes,

@@ -499,9 +499,10 @@ struct Gen {
         for (uint32_t j = 0; j < m && j < stride.size(); ++j) {
             bool first = !stride[j].empty();
             for (uint32_t q = 0; q < j && first; ++q) first = code[i0 + q].a != code[i0 + j].a;
-            if (first)
+            if (first) {
                 o("  if (ex%u) jprefetch<%d>(jimg, bc, va%u + %uull * (%s));\n", j, slot(code[i0 + j]), j, kPrefetchIters,
                   stride[j].c_str());
+            }
         }
         o(" }\n");
     }
@@ -630,6 +631,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
         o("};\n");
     }
     // one cache entry per address register, in order of first use (wrapping beyond JBC_SLOTS)
+    int nslots = 0;                                   // entries this kernel uses (the others stay empty)
     {
         std::vector<int> seen(256, -1);
         int next = 0;
@@ -639,6 +641,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
             if (seen[a] < 0) seen[a] = next++ % kJbcSlots;
             G.slot_of[a] = seen[a];
         }
+        nslots = std::min(next, kJbcSlots);
     }
     const uint32_t NR = G.NR;
     static const char* const mname[] = {"inj", "len", "trace", "page"};
@@ -775,14 +778,16 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "jx->after_[lane] = 0u; jx->msk_[lane] = 0u; jx->fired_[lane] = 0u; jx->bad_[lane] = 0u;\n"
       "JBufCache bc; uint4 recbuf = make_uint4(0u, 0u, 0u, 0u); (void)recbuf;\n"
       "if (jx->bck == k) {                 // this warp's cache from its previous job of the same instance\n"
-      "#pragma unroll\n for (int s_ = 0; s_ < JBC_SLOTS; ++s_) { bc.lo[s_] = jx->bc_[s_ * 4][lane]; "
-      "bc.sz[s_] = jx->bc_[s_ * 4 + 1][lane]; bc.b[s_] = jx->bc_[s_ * 4 + 2][lane]; bc.pb[s_] = jx->bc_[s_ * 4 + 3][lane]; "
+      "#pragma unroll\n for (int s_ = 0; s_ < %d; ++s_) { bc.lo[s_] = jx->bc_[s_ * 4][lane]; "
+      "bc.sz[s_] = jx->bc_[s_ * 4 + 1][lane]; %s"
       "bc.z[s_] = (jx->bcz_[lane] >> s_) & 1u; } }\n"
       "// golden trace pass: the last step was a BRA / EXIT; next checkpoint and its threshold step\n"
       "u32 brk = 1u, ckn = 0u, ckx = %s; (void)brk; (void)ckn; (void)ckx;\nu32 lexm_ = 0u; (void)lexm_;\n"
       "// blocks run only within [step, lim): lim = the watchdog, or the injection step while it is pending,\n"
       "// or the next checkpoint step (golden trace pass)\n"
-      "u32 lim = %s;\n", mode == 2 ? "ck ? 0u : 0xFFFFFFFFu" : "0xFFFFFFFFu",
+      "u32 lim = %s;\n", nslots,
+      mode == 3 ? "bc.b[s_] = jx->bc_[s_ * 4 + 2][lane]; bc.pb[s_] = jx->bc_[s_ * 4 + 3][lane]; " : "",
+      mode == 2 ? "ck ? 0u : 0xFFFFFFFFu" : "0xFFFFFFFFu",
       mode == 0 ? "(hstep >= step && hstep < watchdog) ? hstep : watchdog" : "watchdog");
     if (mode == 2)
         o("bool tmpl_ = false; (void)tmpl_;\nuint4* const jtm_ = reinterpret_cast<uint4*>(jsmem + %uu + (threadIdx.x >> 5) * "
@@ -1001,11 +1006,15 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "Q4 = (st_.preds >> 4) & 1u; Q5 = (st_.preds >> 5) & 1u; Q6 = (st_.preds >> 6) & 1u;\n"
       "  if (done_) goto finish;\n  continue;\n }\n}\n");
     o("finish:\n");
+    // (only the entries this kernel uses, and the K8 page fields only in PAGE mode:
+    // whatever the block code never reads would otherwise hold registers across it)
     o(" {                                 // the buffer cache for this warp's next job\n"
-      "#pragma unroll\n  for (int s_ = 0; s_ < JBC_SLOTS; ++s_) { jx->bc_[s_ * 4][lane] = bc.lo[s_]; "
-      "jx->bc_[s_ * 4 + 1][lane] = bc.sz[s_]; jx->bc_[s_ * 4 + 2][lane] = bc.b[s_]; jx->bc_[s_ * 4 + 3][lane] = bc.pb[s_]; }\n"
-      "  u32 z_ = 0u;\n#pragma unroll\n  for (int s_ = 0; s_ < JBC_SLOTS; ++s_) z_ |= (u32)bc.z[s_] << s_;\n"
-      "  jx->bcz_[lane] = z_; __syncwarp(); if (lane == 0u) jx->bck = k; __syncwarp(); }\n");
+      "#pragma unroll\n  for (int s_ = 0; s_ < %d; ++s_) { jx->bc_[s_ * 4][lane] = bc.lo[s_]; "
+      "jx->bc_[s_ * 4 + 1][lane] = bc.sz[s_]; %s}\n"
+      "#pragma unroll\n  for (int s_ = %d; s_ < JBC_SLOTS; ++s_) jx->bc_[s_ * 4 + 1][lane] = 0u;\n"
+      "  u32 z_ = 0u;\n#pragma unroll\n  for (int s_ = 0; s_ < %d; ++s_) z_ |= (u32)bc.z[s_] << s_;\n"
+      "  jx->bcz_[lane] = z_; __syncwarp(); if (lane == 0u) jx->bck = k; __syncwarp(); }\n", nslots,
+      mode == 3 ? "jx->bc_[s_ * 4 + 2][lane] = bc.b[s_]; jx->bc_[s_ * 4 + 3][lane] = bc.pb[s_]; " : "", nslots, nslots);
     if (mode == 2) o(" if (lane == 0u) jbulk_wait();     // the template stores are complete\n");
     if (mode == 2)                                    // checkpoints the warp never reached: absent
         o(" if (ck) for (; ckn < (step + ck_interval - 1u) / ck_interval; ++ckn) {\n"
@@ -1051,14 +1060,15 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
     o("const JArgs A, const u64* __restrict__ warp_off, "
       "const jfi_site* __restrict__ sites, const u32 n, jfi_inj* __restrict__ out, jfi_store* __restrict__ log, "
       "const u32 cap, const u32* ckpt, const u64* __restrict__ ck_off, const u32 ck_interval, "
-      "const u32* __restrict__ order, u32* counter, u32* status) {\n"
+      "const u32* __restrict__ order, u32* counter, u32* status, u32* smq, const u32 nsm, const u32 dealt) {\n"
       " extern __shared__ u32 jsmem[];\n"
       " const u32 lane = threadIdx.x & 31u;\n"
       " u32* Rs = jsmem + (threadIdx.x >> 5) * %uu;\n"
       " Rs[%uu + lane] = 0u;                     // the zero row (RZ, indices >= n_regs)\n"
       " { JCtx* jx0_ = reinterpret_cast<JCtx*>(jsmem + %uu + (threadIdx.x >> 5) * (JCTX_BYTES / 4u)); "
           "if ((threadIdx.x & 31u) == 0u) jx0_->bck = 0xFFFFFFFFu; __syncwarp(); }\n"
-      " for (;;) {\n  u32 p = 0u; if (lane == 0u) p = atomicAdd(counter, 1u); p = __shfl_sync(JFULL, p, 0);\n"
+      " const u32 sm_ = jsmid();\n"
+      " for (;;) {\n  u32 p = 0u; if (lane == 0u) p = jnext_job(counter, smq, sm_, nsm, dealt, n); p = __shfl_sync(JFULL, p, 0);\n"
       "  if (p >= n) return;\n  const u32 i = order[p]; const jfi_site S = sites[i];\n"
       "  if (S.flags & 1u) { if (%s && lane == 0u) { jfi_inj r; r.before = r.after = r.mask = r.fault_pc = 0u; "
       "r.fault_kind = 0; r.outcome = 3; r.overflow = 0; r.flags = 0; r.n_faulty_stores = 0u; out[i] = r; } continue; }\n"
@@ -1512,17 +1522,27 @@ extern "C" fi_status fi_inject_jit(const fi_jit* j, const fi_program* p, const u
     const uint64_t* warp_off = t->warp_off;
     const uint32_t* ckpt = t->ckpt;
     const uint64_t* ck_off = t->ckpt_off;
+    // the per-SM deal counters (jnext_job): after the order, 256-B aligned
+    uint32_t* smq = reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(ws) + 256 + (((size_t)n * 4 + 255) & ~(size_t)255));
+    uint32_t nsm = (uint32_t)std::min(std::max(sms, 1), 256), dealt = 0;
     void* args[] = {&A, (void*)&warp_off, (void*)&sites, &n, &out, &log, &log_cap, (void*)&ckpt, (void*)&ck_off,
-                    (void*)&ck_iv, &order, &counter, &dev_status};
+                    (void*)&ck_iv, &order, &counter, &dev_status, &smq, &nsm, &dealt};
     // each static kernel's module takes its own replicas off the LPT queue (k_lpt_order
-    // reset the queue counter; it is reset again before every later module)
+    // reset the queue counter; it is reset again before every later module).  The
+    // first `dealt` positions — the longest replicas, one per resident warp — are dealt
+    // to the SMs in snake order (every SM gets an equal share of the long ones whatever
+    // the hardware's CTA placement), the rest come off the shared queue; the grid is
+    // the whole persistent grid, so every SM has warps to take its share.
     for (size_t k = 0; k < j->m.size(); ++k) {
         if (k) {
             e = fi::cuda_status(cudaMemsetAsync(counter, 0, 4, s));
             if (e) return e;
         }
+        e = fi::cuda_status(cudaMemsetAsync(smq, 0, (size_t)nsm * 4, s));
+        if (e) return e;
         drv().occ(&per, j->m[k].inject, 128, j->smem);
-        const uint32_t grid = (uint32_t)std::min<uint64_t>((n + 3) / 4, (uint64_t)std::max(1, sms * std::max(1, per)));
+        const uint32_t grid = (uint32_t)std::max(1, sms * std::max(1, per));
+        dealt = (uint32_t)std::min<uint64_t>(n, (uint64_t)grid * 4);
         e = launch(j->m[k].inject, grid, j->smem, s, args);
         if (e) return e;
     }

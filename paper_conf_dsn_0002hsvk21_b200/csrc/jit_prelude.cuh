@@ -198,6 +198,30 @@ __device__ __forceinline__ uint4 jld128(const u8* p) {
     return r;
 }
 
+// K4's job queue (lane 0): LPT positions [0, dealt) are dealt to the SMs in snake
+// order — round r of SM s is position r*nsm + (r odd ? nsm-1-s : s) — and taken by
+// that SM's warps through its own counter; then [dealt, n) off the shared counter;
+// then the warp steals the rounds left in the other SMs' deals (an SM the hardware
+// gave no warps).  Every position is handed out exactly once: each (SM, round) by one
+// atomicAdd result.  Returns a position >= n when nothing is left.
+__device__ __forceinline__ u32 jsmid() { u32 r; asm volatile("mov.u32 %0, %%smid;" : "=r"(r)); return r; }
+__device__ __forceinline__ u32 jdeal_pos(u32 r, u32 s, u32 nsm) { return r * nsm + ((r & 1u) ? nsm - 1u - s : s); }
+__device__ __noinline__ u32 jnext_job(u32* counter, u32* smq, u32 sm, u32 nsm, u32 dealt, u32 n) {
+    if (sm < nsm) {
+        const u32 q = jdeal_pos(atomicAdd(&smq[sm], 1u), sm, nsm);
+        if (q < dealt) return q;
+    }
+    const u32 g = dealt + atomicAdd(counter, 1u);
+    if (g < n) return g;
+    for (u32 d = 1; d <= nsm; ++d) {
+        const u32 s = (sm + d) % nsm;
+        if (jdeal_pos(*(volatile u32*)&smq[s], s, nsm) >= dealt) continue;   // (that deal is used up)
+        const u32 q = jdeal_pos(atomicAdd(&smq[s], 1u), s, nsm);
+        if (q < dealt) return q;
+    }
+    return n;
+}
+
 // per-lane cache of buffer bounds, JBC_SLOTS entries, 32-bit: image offset `lo`
 // and the size floored to 16 B (`sz`; 0 = empty entry).  The generator gives each
 // memory instruction a fixed entry (slot) by its address register, so a loop that
