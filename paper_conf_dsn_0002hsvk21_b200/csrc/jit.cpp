@@ -731,7 +731,10 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
             o("%u%s", leader[i] ? std::min<uint32_t>(blen[i], 0xFFFF) : 0u, i + 1 < n ? "," : "");
         o("};\n");
     }
-    o("__device__ __noinline__ void kern_%u_%s(const JArgs& A_, const u32 hstep_p, const u32 hpc_p, const u32 hlane_p, "
+    // (inlined into its one entry kernel: as a separate function ptxas re-loaded the global
+    // memory descriptor into uniform registers before every image load, and spilled more;
+    // K4 6.29 -> 6.18 ms, golden pass 2 14.6 -> 14.2 ms on C2, profiles/r02/s6/k4_inline_ab.log)
+    o("__device__ __forceinline__ void kern_%u_%s(const JArgs& A_, const u32 hstep_p, const u32 hpc_p, const u32 hlane_p, "
       "const u32 hkind_p, const u32 hreg_p, const u32 hbfm_p, const u32 hmask_p, const u32 k_p, const u32 cta_p, "
       "const u32 wic_p, const u32 watchdog_p, u32* __restrict__ ck_p, const u32 ck_interval_p, "
       "jfi_store* __restrict__ st_out_p, const u32 st_cap_p, JOut& out_p, u32* __restrict__ Rs_p, "
