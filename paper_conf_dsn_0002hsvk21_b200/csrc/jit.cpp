@@ -133,8 +133,8 @@ struct Gen {
                 switch (I.imm) {
                     case 0: e = "wic * 32u + lane"; break;
                     case 1: e = "cta"; break;
-                    case 2: e = "in.block"; break;
-                    case 3: e = "in.grid"; break;
+                    case 2: e = "JIN_(block)"; break;
+                    case 3: e = "JIN_(grid)"; break;
                     case 4: e = "lane"; break;
                     case 5: e = "wic"; break;
                 }
@@ -759,10 +759,12 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
     // are used (cold paths), so they do not hold registers across the block code
     o("const JArgs& A = A_; const u8* __restrict__ const jimg = A_.img;\n");
     o("const u32 lane = threadIdx.x & 31u, lt_mask = (1u << lane) - 1u;\n");
-    o("const jfi_instance in = A.inst[k];\nconst u32 cbank_len = in.cbank_len; const u32* __restrict__ cb = A.cbank + "
-      "in.cbank_off;\n(void)cbank_len; (void)cb; (void)lt_mask;\n");
+    // the instance's fields are read where they are used (S2R, LDC: cold block code):
+    // cached in registers they would be live across every block of the dispatch loop
+    o("#define JIN_(f) (__ldg(&A.inst[k].f))\n#define cbank_len JIN_(cbank_len)\n#define cb (A.cbank + JIN_(cbank_off))\n"
+      "(void)lt_mask;\n");
     for (uint32_t j = 0; j < NR; ++j) o("u32 R%u;%s", j, (j % 16 == 15) ? "\n" : " ");
-    o("\nconst u32 nl_ = in.block - wic * 32u; bool live = lane < (nl_ > 32u ? 32u : nl_);\n");
+    o("\nconst u32 nl_ = JIN_(block) - wic * 32u; bool live = lane < (nl_ > 32u ? 32u : nl_);\n");
     o("u32 pc = 0u, step = 0u; bool Q0 = false, Q1 = false, Q2 = false, Q3 = false, Q4 = false, Q5 = false, "
       "Q6 = false;\n");
     o("if (%s) {\n  u32 c_ = hstep / ck_interval;\n"
@@ -1030,7 +1032,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       " out_.before = __shfl_sync(JFULL, jx->before_[lane], hlane); out_.after = __shfl_sync(JFULL, jx->after_[lane], hlane);\n"
       " out_.mask = __shfl_sync(JFULL, jx->msk_[lane], hlane); out_.fired = jx->fired_[lane]; out_.bad = jx->bad_[lane]; }\n}\n");
     for (const char* nm : kCtxNames) o("#undef %s\n", nm);
-    o("\n");
+    o("#undef JIN_\n#undef cbank_len\n#undef cb\n\n");
 }
 
 // The module source of static kernel `only` (its device functions, and entry kernels
@@ -1071,7 +1073,7 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
       " { JCtx* jx0_ = reinterpret_cast<JCtx*>(jsmem + %uu + (threadIdx.x >> 5) * (JCTX_BYTES / 4u)); "
           "if ((threadIdx.x & 31u) == 0u) jx0_->bck = 0xFFFFFFFFu; __syncwarp(); }\n"
       " const u32 sm_ = jsmid();\n"
-      " for (;;) {\n  u32 p = 0u; if (lane == 0u) p = jnext_job(counter, smq, sm_, nsm, dealt, n); p = __shfl_sync(JFULL, p, 0);\n"
+      " for (;;) {\n  const u32 p = jnext_job(counter, smq, sm_, nsm, dealt, n, lane);\n"
       "  if (p >= n) return;\n  const u32 i = order[p]; const jfi_site S = sites[i];\n"
       "  if (S.flags & 1u) { if (%s && lane == 0u) { jfi_inj r; r.before = r.after = r.mask = r.fault_pc = 0u; "
       "r.fault_kind = 0; r.outcome = 3; r.overflow = 0; r.flags = 0; r.n_faulty_stores = 0u; out[i] = r; } continue; }\n"

@@ -198,26 +198,41 @@ __device__ __forceinline__ uint4 jld128(const u8* p) {
     return r;
 }
 
-// K4's job queue (lane 0): LPT positions [0, dealt) are dealt to the SMs in snake
-// order — round r of SM s is position r*nsm + (r odd ? nsm-1-s : s) — and taken by
-// that SM's warps through its own counter; then [dealt, n) off the shared counter;
-// then the warp steals the rounds left in the other SMs' deals (an SM the hardware
-// gave no warps).  Every position is handed out exactly once: each (SM, round) by one
-// atomicAdd result.  Returns a position >= n when nothing is left.
+// K4's job queue (the whole warp calls it, the same result in every lane): LPT
+// positions [0, dealt) are dealt to the SMs in snake order — round r of SM s is
+// position r*nsm + (r odd ? nsm-1-s : s) — and taken by that SM's warps through its
+// own counter; then [dealt, n) off the shared counter; then the warp steals the
+// rounds left in the other SMs' deals (an SM the hardware gave no warps), the lanes
+// looking at 32 SMs' counters at a time.  Every position is handed out exactly once:
+// each (SM, round) by one atomicAdd result.  Returns a position >= n when nothing is
+// left.
 __device__ __forceinline__ u32 jsmid() { u32 r; asm volatile("mov.u32 %0, %%smid;" : "=r"(r)); return r; }
 __device__ __forceinline__ u32 jdeal_pos(u32 r, u32 s, u32 nsm) { return r * nsm + ((r & 1u) ? nsm - 1u - s : s); }
-__device__ __noinline__ u32 jnext_job(u32* counter, u32* smq, u32 sm, u32 nsm, u32 dealt, u32 n) {
-    if (sm < nsm) {
-        const u32 q = jdeal_pos(atomicAdd(&smq[sm], 1u), sm, nsm);
-        if (q < dealt) return q;
+__device__ __noinline__ u32 jnext_job(u32* counter, u32* smq, u32 sm, u32 nsm, u32 dealt, u32 n, u32 lane) {
+    u32 p = n;
+    if (lane == 0u) {
+        if (sm < nsm) {
+            const u32 q = jdeal_pos(atomicAdd(&smq[sm], 1u), sm, nsm);
+            if (q < dealt) p = q;
+        }
+        if (p >= n) {
+            const u32 g = dealt + atomicAdd(counter, 1u);
+            if (g < n) p = g;
+        }
     }
-    const u32 g = dealt + atomicAdd(counter, 1u);
-    if (g < n) return g;
-    for (u32 d = 1; d <= nsm; ++d) {
-        const u32 s = (sm + d) % nsm;
-        if (jdeal_pos(*(volatile u32*)&smq[s], s, nsm) >= dealt) continue;   // (that deal is used up)
-        const u32 q = jdeal_pos(atomicAdd(&smq[s], 1u), s, nsm);
-        if (q < dealt) return q;
+    p = __shfl_sync(0xFFFFFFFFu, p, 0);
+    if (p < n) return p;
+    for (u32 s0 = 0; s0 < nsm; s0 += 32u) {
+        const u32 s = s0 + lane;
+        u32 m = __ballot_sync(0xFFFFFFFFu, s < nsm && jdeal_pos(*(volatile u32*)&smq[s], s, nsm) < dealt);
+        while (m) {
+            const u32 t = s0 + (u32)__ffs(m) - 1u;
+            m &= m - 1u;
+            u32 q = dealt;
+            if (lane == 0u) q = jdeal_pos(atomicAdd(&smq[t], 1u), t, nsm);
+            q = __shfl_sync(0xFFFFFFFFu, q, 0);
+            if (q < dealt) return q;
+        }
     }
     return n;
 }

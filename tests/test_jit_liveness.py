@@ -18,8 +18,8 @@ def _functions(src: str, mode: str) -> dict[str, str]:
     """kern_<k>_<mode> bodies, from the block dispatch on (the register
     initialisation before the dispatch loop is not a kill)."""
     out = {}
-    for m in re.finditer(r"__noinline__ void (kern_\d+_%s)\(" % mode, src):
-        end = src.find("__noinline__ void kern_", m.end())
+    for m in re.finditer(r"__forceinline__ void (kern_\d+_%s)\(" % mode, src):
+        end = src.find("__forceinline__ void kern_", m.end())
         body = src[m.end(): end if end >= 0 else len(src)]
         out[m.group(1)] = body[body.index(" switch (pcm) {"):]
     return out
