@@ -338,7 +338,7 @@ struct Gen {
                 if (code[q].guard != 7) all += (all.empty() ? "" : " & ") + std::string("gb_") + std::to_string(q);
             if (!all.empty()) o(" && (%s) == JFULL", all.c_str());
             o(") { if (lane == 0u) jbulk_st(&rec_out[step], jtm_, %uu);\n"
-              "     if (jx->prof.cc) { const u32 o_ = ((u32)jx->prof.rb + step) & 1023u; if (o_ + %uu < 1024u) { "
+              "     if (JPCC_) { const u32 o_ = (JPRB_ + step) & 1023u; if (o_ + %uu < 1024u) { "
               "if (lane < 8u) jx->prof.pcnt_[lane] += jx->prof.tcnt_[lane]; } else jprof_tmpl_cross(&jx->prof, lane, "
               "1024u - o_); } } else\n", (E + 1 - tmpl_L) * 16, E + 1 - tmpl_L);
         }
@@ -935,12 +935,19 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
                     // the full-warp copy unrolled twice: ptxas gives half of the loop-carried
                     // registers alternating homes, copied back on every back edge of a
                     // one-iteration loop; with two iterations per trip the homes swap roles
+                    // (the template loop's profile state, constant over the loop, read once)
+                    if (L == tmpl_L)
+                        o(" const bool jpc_ = jx->prof.cc != nullptr; const u32 jrb_ = (u32)jx->prof.rb; (void)jpc_; (void)jrb_;\n"
+                          "#undef JPCC_\n#define JPCC_ jpc_\n#undef JPRB_\n#define JPRB_ jrb_\n");
                     o("#undef JFW_\n#define JFW_ 1\n for (;;) {  // self-loop %u..%u, full warp, two iterations per trip\n {\n",
                       L, i);
                     o.s += back(body, "goto U" + std::to_string(L) + "_;");
                     o(" }\n U%u_: ;\n {\n", L);
                     o.s += back(body, "continue;");
-                    o(" }\n }\n#undef JFW_\n#define JFW_ 0\n } else {\n for (;;) {  // self-loop %u..%u\n", L, i);
+                    o(" }\n }\n#undef JFW_\n#define JFW_ 0\n");
+                    if (L == tmpl_L)
+                        o("#undef JPCC_\n#define JPCC_ (jx->prof.cc != nullptr)\n#undef JPRB_\n#define JPRB_ ((u32)jx->prof.rb)\n");
+                    o(" } else {\n for (;;) {  // self-loop %u..%u\n", L, i);
                     o.s += back(body, "continue;");
                     o(" } }\n");
                 } else {

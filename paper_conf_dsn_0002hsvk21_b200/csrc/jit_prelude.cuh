@@ -84,6 +84,10 @@ struct JCtx {
 // memory (jit.cpp flush_recs), evict-first in L2 like the per-lane __stcs records;
 // lane 0 issues them and waits for them before the warp's job ends
 #define JFW_ 0
+// golden pass 2's fused profile: is it on, and the warp's first global record
+// (jit.cpp flush_recs; the template loop reads both once)
+#define JPCC_ (jx->prof.cc != nullptr)
+#define JPRB_ ((u32)jx->prof.rb)
 __device__ __forceinline__ void jbulk_st(uint4* g, const uint4* s, u32 bytes) {
     u64 pol;
     asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
