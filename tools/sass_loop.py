@@ -10,7 +10,7 @@ import sys
 
 src = open("/tmp/jit_sass/k.cu").read().splitlines()
 lo = next(i for i, l in enumerate(src, 1) if "full warp, two iterations per trip" in l)
-hi = next(i for i, l in enumerate(src, 1) if i > lo and re.match(r"\s*U\d+_: ;", l))
+hi = next(i for i, l in enumerate(src, 1) if i > lo and re.match(r"\s*U\d+_(\d+)?: ;", l))
 hi2 = next(i for i, l in enumerate(src, 1) if i > hi and "self-loop" in l)
 rows, cur, label = [], None, None
 for line in open("/tmp/jit_sass/k.sass"):
