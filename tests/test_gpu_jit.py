@@ -64,6 +64,33 @@ def test_jit_mini_c2(F):
     assert (a["fault_kind"] == 3).sum() + (a["fault_kind"] == 2).sum() > 0
 
 
+def test_jit_job_dealing_covers_every_replica(F):
+    """K4's job order (jit_prelude.cuh jnext_job): the head of the LPT list is dealt
+    to the SMs in snake order, the rest comes off the shared counter, idle warps steal
+    undealt rounds.  Every replica must be run exactly once whatever n is relative to
+    the resident warps (dealt = min(n, grid*4)): each subset's results equal the same
+    replicas' rows of one large launch, field by field, for n below, at and above
+    the dealt boundary."""
+    dp = F.DeviceProgram(P.c2(full=False))
+    gt = F.golden_run(dp)
+    ic, cc = F.profile(gt)
+    N = 4000
+    sites = F.select_sites(F.SiteIndex(gt, ic, cc), F.schedule(0x5151, [F.G_GP, F.G_LD], [0, 1, 2, 3]), 0, N)
+    cap = F.log_capacity(gt)
+    out, _ = F.inject(gt, sites, N, cap)
+    ref = F.as_numpy(out, F.INJ_DTYPE, N).copy()
+    sms = torch.cuda.get_device_properties(0).multi_processor_count
+    rows = sites.view(N, -1)
+    for n in (1, 2, sms - 1, sms + 1, 3 * sms * 4 - 1, 3 * sms * 4, 3 * sms * 4 + 1):
+        n = min(n, N)
+        o2, _ = F.inject(gt, rows[:n].contiguous().view(-1), n, cap)
+        torch.cuda.synchronize()
+        got = F.as_numpy(o2, F.INJ_DTYPE, n)
+        for f in ref.dtype.names:
+            bad = np.flatnonzero(got[f] != ref[f][:n])
+            assert bad.size == 0, f"n={n} {f}: replica {bad[0]}"
+
+
 @pytest.mark.parametrize("seed", [5, 6, 7])
 def test_jit_ffma_special_values(F, seed):
     _both(F, P.ffma_runs(seed), seed, [F.G_FP32, F.G_GP, F.G_LD], [0, 1, 2, 3], 300)
