@@ -1,7 +1,7 @@
 """K8 (fi_classify_batched, JIT re-execution) on a full-size multi-launch
 program, for ncu: golden run, profile, select n replicas, K4, then one timed
 K8 call (CUDA events) and the outcome digest.
-usage: k8_prof.py C3|C4|stencil|lbm|md|ep|cg [n] [batch]"""
+usage: k8_prof.py C3|C4|stencil|lbm|md|ep|cg [n] [batch] [mem_budget_GB]"""
 import hashlib
 import os
 import sys
@@ -15,7 +15,8 @@ from paper_conf_dsn_0002hsvk21_b200 import fi  # noqa: E402
 
 cfg = sys.argv[1] if len(sys.argv) > 1 else "C3"
 n = int(sys.argv[2]) if len(sys.argv) > 2 else 128
-batch = int(sys.argv[3]) if len(sys.argv) > 3 else None
+batch = int(sys.argv[3]) if len(sys.argv) > 3 and int(sys.argv[3]) > 0 else None
+budget = int(sys.argv[4]) << 30 if len(sys.argv) > 4 else 24 << 30
 if cfg == "C3":
     prog, seed = P.c3(full=True), P.CAMPAIGN_SEED[3]
 elif cfg == "C4":
@@ -36,7 +37,7 @@ torch.cuda.synchronize()
 print(f"setup {time.time() - t0:.1f} s, {dp.n_inst} launches, {gt.n_rec} records", flush=True)
 a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
 a.record()
-hist = fi.classify_batched(gt, sites, n, out, log, cap, batch=batch, engine="jit")
+hist = fi.classify_batched(gt, sites, n, out, log, cap, batch=batch, engine="jit", mem_budget=budget)
 b.record()
 torch.cuda.synchronize()
 ms = a.elapsed_time(b)
