@@ -350,7 +350,9 @@ fi_status fi_classify(const fi_program* p, const uint8_t* image, const fi_trace*
  * Replicas that exceed a capacity, or that later load a dropped corrupted word,
  * get outcome 0xFF and FI_E_CAPACITY — never a wrong class.  Fills out[].outcome
  * / flags (and fault_kind/fault_pc of the first downstream fault when K4 had
- * none), accumulates hist[8][4][3].  Scratch: fi_classify_batched_workspace(). */
+ * none), accumulates hist[8][4][3].  Scratch: fi_classify_batched_workspace();
+ * after fi_classify_batched_jit its first 8 bytes hold the u64 count of emulated
+ * warp-steps of every warp K8 re-executed (the work behind its issue roofline). */
 size_t fi_classify_batched_workspace(const fi_program* p, uint32_t n, uint32_t log_cap, uint32_t batch,
                                      uint32_t pool_pages, uint32_t pend_cap);
 fi_status fi_classify_batched(const fi_program* p, const uint8_t* image, const fi_trace* t, const fi_site* sites,

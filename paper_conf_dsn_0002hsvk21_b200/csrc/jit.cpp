@@ -1113,20 +1113,23 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
           " jfi_store* scr = K.scratch + (u64)(blockIdx.x * 4u + wib) * K.log_cap;\n"
           " const jfi_instance in = A.inst[t];\n const u32 nw = in.warp_end - in.warp_begin, wpc = (in.block + 31u) / 32u;\n"
           " const u64 items = (u64)(*K.n_active) * nw;\n const bool unchecked = K.flags & 1u;\n"
+          " u64 nsteps_ = 0ull;                       // this warp's emulated steps, one atomic at its end\n"
           " for (;;) {\n  u32 it = 0u; if (lane == 0u) it = atomicAdd(K.work, 1u); it = __shfl_sync(JFULL, it, 0);\n"
-          "  if (it >= items) return;\n  const u32 s = K.active[it / nw], lw = it %% nw, w = in.warp_begin + lw;\n"
+          "  if (it >= items) { if (lane == 0u && nsteps_) atomicAdd(K.steps, (unsigned long long)nsteps_); return; }\n"
+          "  const u32 s = K.active[it / nw], lw = it %% nw, w = in.warp_begin + lw;\n"
           "  if (K.slot[s].overflow) continue;\n"
           "  const u64 L = K.warp_off[w + 1] - K.warp_off[w]; const u64 wd = 10ull * L + 1024ull;\n"
           "  const u32 watchdog = wd > 0xFFFFFFFFull ? 0xFFFFFFFFu : (u32)wd;\n"
           "  JPage pg; pg.ptab = K.ptab + (u64)s * K.total_pages; pg.pool = K.pool; pg.page_base = K.page_base; "
           "pg.last_ref = K.last_ref; pg.dropped = K.dropped + (u64)s * K.dwords; pg.inexact = &K.slot[s].inexact; pg.t = t;\n"
-          "  JOut o;\n  switch (in.kernel) {\n",
+          "  JOut o; o.start = 0u;\n  switch (in.kernel) {\n",
           min_blocks, rs, zrow, 4 * rs);
         for (uint32_t k = 0; k < n_kern; ++k)
             if (mine(k)) o("   case %u: kern_%u_page(A, 0xFFFFFFFFu, 0u, 0u, 0u, 0u, 0u, 0u, t, lw / wpc, lw %% wpc, watchdog, (u32*)0, "
               "0u, scr, K.log_cap, o, Rs, A.dec + %uu, A.ins + %uu, (u8*)0, (uint4*)0, &pg); break;\n",
               k, k, kern[k].code_off, kern[k].code_off);
         o("   default: o.steps = 0; o.fault = 4; o.fault_pc = 0; o.nstore = 0; break;\n  }\n"
+          "  nsteps_ += o.steps - o.start;\n"
           "  if (o.fault) {\n   if (lane == 0u) {\n"
           "    const unsigned long long key = ((unsigned long long)t << 43) | ((unsigned long long)lw << 19) | "
           "((unsigned long long)o.fault << 16) | (o.fault_pc & 0xFFFFu);\n"

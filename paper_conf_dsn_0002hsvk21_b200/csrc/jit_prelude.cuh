@@ -369,6 +369,7 @@ struct JK8 {
     const u32* active; const u32* n_active; u32* work;
     jfi_store* scratch; u32 log_cap;
     u32 flags; u32* status;
+    unsigned long long* steps;                      // emulated warp-steps of the re-executed warps (summed)
 };
 // the replica slot's view of memory during instance t
 struct JPage {

@@ -602,7 +602,7 @@ __global__ void __launch_bounds__(256) k8_final(K8Args A) {
 using namespace fi;
 
 namespace {
-struct K8Layout { size_t slot, ptab, bcount, dropped, pool, fstack, ftop, pend, forn, active, nact, work, need, nneed,
+struct K8Layout { size_t steps, slot, ptab, bcount, dropped, pool, fstack, ftop, pend, forn, active, nact, work, need, nneed,
                   scratch, page_base, last_ref, dying_off, dying, reps, kop, total; };
 K8Layout k8_layout(uint64_t image_bytes, uint32_t n_buf, uint32_t n_inst, uint32_t n, uint32_t B, uint32_t pool_pages,
                    uint32_t pend_cap, uint32_t log_cap, uint32_t scratch_warps) {
@@ -611,6 +611,7 @@ K8Layout k8_layout(uint64_t image_bytes, uint32_t n_buf, uint32_t n_inst, uint32
     K8Layout L;
     size_t o = 0;
     auto take = [&](size_t bytes) { const size_t r = o; o += align256(bytes); return r; };
+    L.steps = take(8);                               // offset 0: emulated warp-steps of the JIT re-execution (fi.h)
     L.slot = take((size_t)B * sizeof(Slot));
     L.ptab = take((size_t)B * tp * 4);
     L.bcount = take((size_t)B * n_buf * 4);
@@ -768,7 +769,8 @@ static fi_status k8_run(const fi_program* p, const uint8_t* image, const fi_trac
     const uint32_t fix_grid = (uint32_t)std::max(1, sms * 4);
     JK8Host JK{A.warp_off, A.gst_off, A.gst, A.slot, A.ptab, A.total_pages, A.pool, A.page_base, A.last_ref,
                A.dropped, A.dwords, A.pend, A.pend_cap, A.forn, kForeignCap, A.active, A.n_active, A.work,
-               A.scratch, A.log_cap, A.flags, A.status};
+               A.scratch, A.log_cap, A.flags, A.status, reinterpret_cast<unsigned long long*>(w + L.steps)};
+    if ((e = cuda_status(cudaMemsetAsync(w + L.steps, 0, 8, s)))) return e;
 
     for (uint32_t b0 = 0; b0 < n; b0 += batch) {
         const uint32_t nb = std::min(batch, n - b0);

@@ -709,11 +709,13 @@ def classify_batched(gt: GoldenTrace, sites: torch.Tensor, n: int, out: torch.Te
                      log_cap: int, hist: torch.Tensor | None = None, unchecked: bool = False, batch: int | None = None,
                      pool_pages: int | None = None, pend_cap: int | None = None, mem_budget: int = 24 << 30,
                      status: DeviceStatus | None = None, engine: str = "interp", rtol: float = 0.0,
-                     hist_tol: torch.Tensor | None = None) -> torch.Tensor:
+                     hist_tol: torch.Tensor | None = None, steps_out: list | None = None) -> torch.Tensor:
     """fi_classify_batched (K8): whole-program outcomes for long multi-instance
     programs, replica batches in lockstep over the launches.  engine "jit":
     fi_classify_batched_jit (re-execution on the program's JIT module).
-    rtol / hist_tol: the C-12 secondary numeric classification, as classify()."""
+    rtol / hist_tol: the C-12 secondary numeric classification, as classify().
+    steps_out (engine "jit"): appended with the emulated warp-steps of the
+    re-executed warps (the workspace's first 8 bytes, fi.h; synchronises)."""
     dev = gt.dp.device
     if hist is None:
         hist = torch.zeros((8, 4, 3), dtype=torch.int64, device=dev)
@@ -734,6 +736,8 @@ def classify_batched(gt: GoldenTrace, sites: torch.Tensor, n: int, out: torch.Te
                                              FI_UNCHECKED if unchecked else 0, float(rtol), _p(hist_tol), batch,
                                              pool_pages, pend_cap, _p(ws), ws_n, st.ptr, _stream()),
                "fi_classify_batched_jit")
+        if steps_out is not None:
+            steps_out.append(int(ws[:8].view(torch.int64).item()))
     else:
         _check(lib().fi_classify_batched(C.byref(gt.dp.c), _p(gt.image), C.byref(gt.c), _p(sites), n, _p(out),
                                          _p(log), log_cap, _p(hist), FI_UNCHECKED if unchecked else 0, float(rtol),

@@ -185,6 +185,27 @@ def test_jit_k8(F, maker, unchecked):
     assert (a["outcome"] == F.SDC).sum() > 0
 
 
+def test_jit_k8_counts_its_steps(F):
+    """fi_classify_batched_jit leaves the emulated warp-steps of every warp it
+    re-executed in the workspace's first 8 bytes (fi.h; the bench's K8 roofline):
+    positive when replicas propagate, and at most every replica re-running every
+    warp of every launch after its faulty one (golden lengths, the watchdog aside),
+    and the same count on a second identical call."""
+    prog = P.multi_instance_chain(6, shrink=29)
+    dp = F.DeviceProgram(prog)
+    gt = F.golden_run(dp)
+    ic, cc = F.profile(gt)
+    n = 200
+    sites = F.select_sites(F.SiteIndex(gt, ic, cc), F.schedule(0x5A5, [F.G_GP], [0]), 0, n)
+    cap = F.log_capacity(gt)
+    out, log = F.inject(gt, sites, n, cap)
+    counts = []
+    for _ in range(2):
+        F.classify_batched(gt, sites, n, out.clone(), log, cap, engine="jit", steps_out=counts)
+    bound = n * int(gt.warp_len.cpu().numpy().astype(np.int64).sum())
+    assert 0 < counts[0] <= bound and counts[0] == counts[1], (counts, bound)
+
+
 @pytest.mark.parametrize("which", range(5))
 def test_jit_k8_c5_minis(F, which):
     _k8_both(F, H.c5(full=False)[which], 0xC5C5, [F.G_GP, F.G_GPPR], [0], 200, batch=64)
