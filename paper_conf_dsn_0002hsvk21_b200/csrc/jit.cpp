@@ -366,7 +366,7 @@ struct Gen {
         o("const u64 va = %s + (u64)(i64)(i32)%s; ", R64(I.a).c_str(), hex(I.imm).c_str());
         if (I.op == LDG) {
             o("uint4 v_; const u32 c_ = jldg<%uu, %d>(A, jimg, bc, va, k, ex, v_%s); ", lw, slot(I),
-              mode == 3 ? ", PG.page_base" : "");
+              mode == 3 ? ", &PG" : "");
             o("if (__ballot_sync(JFULL, c_ != 0u)) { fault = __ballot_sync(JFULL, c_ == 1u) ? 1u : 2u; fault_pc = %uu; "
               "step = %s; goto finish; } ", pc, stepx);
             if (mode == 3) o("if (ex) jpage_c<%uu, %d>(A, bc, PG, va, v_); ", nw, slot(I));
@@ -376,7 +376,7 @@ struct Gen {
         } else {
             o("const u32 exm_ = amask & __ballot_sync(JFULL, pv); bool z_ = false; "
               "const u32 c_ = ex ? jcheck<%d>(A, bc, va, %uu, k, &z_%s) : 0u; ", slot(I), 4u << lw,
-              mode == 3 ? ", PG.page_base" : "");
+              mode == 3 ? ", &PG" : "");
             o("if (__ballot_sync(JFULL, c_ != 0u)) { fault = __ballot_sync(JFULL, c_ == 1u) ? 1u : 2u; fault_pc = %uu; "
               "step = %s; goto finish; } ", pc, stepx);
             if (mode == 1) {                           // golden pass 1: into the image
@@ -457,7 +457,7 @@ struct Gen {
             const fi_insn& I = code[i0 + j];
             const uint32_t lw = (I.mod & 3) > 2 ? 2 : (I.mod & 3);
             o("   c%u = ex%u ? jcheck<%d>(A, bc, va%u, %uu, k, &z%u%s) : 0u;\n", j, j, slot(I), j, 4u << lw, j,
-              mode == 3 ? ", PG.page_base" : "");
+              mode == 3 ? ", &PG" : "");
         }
         // (a fault needs a lane that missed its cache: the fault ballots are on the slow path only)
         o("   if (__ballot_sync(JFULL, 0u");
@@ -782,7 +782,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "jx->nst_[lane] = 0u; jx->fault_[lane] = 0u; jx->fault_pc_[lane] = 0u; jx->before_[lane] = 0u; "
       "jx->after_[lane] = 0u; jx->msk_[lane] = 0u; jx->fired_[lane] = 0u; jx->bad_[lane] = 0u;\n"
       "JBufCache bc; uint4 recbuf = make_uint4(0u, 0u, 0u, 0u); (void)recbuf;\n"
-      "if (jx->bck == k) {                 // this warp's cache from its previous job of the same instance\n"
+      "if (jx->bck == k%s) {                 // this warp's cache from its previous job of the same instance\n"
       "#pragma unroll\n for (int s_ = 0; s_ < %d; ++s_) { bc.lo[s_] = jx->bc_[s_ * 4][lane]; "
       "bc.sz[s_] = jx->bc_[s_ * 4 + 1][lane]; %s"
       "bc.z[s_] = (jx->bcz_[lane] >> s_) & 1u; } }\n"
@@ -790,7 +790,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "u32 brk = 1u, ckn = 0u, ckx = %s; (void)brk; (void)ckn; (void)ckx;\nu32 lexm_ = 0u; (void)lexm_;\n"
       "// blocks run only within [step, lim): lim = the watchdog, or the injection step while it is pending,\n"
       "// or the next checkpoint step (golden trace pass)\n"
-      "u32 lim = %s;\n", nslots,
+      "u32 lim = %s;\n", mode == 3 ? " && jx->bckp == (u32)(size_t)PG.ptab" : "", nslots,
       mode == 3 ? "bc.b[s_] = jx->bc_[s_ * 4 + 2][lane]; bc.pb[s_] = jx->bc_[s_ * 4 + 3][lane]; " : "",
       mode == 2 ? "ck ? 0u : 0xFFFFFFFFu" : "0xFFFFFFFFu",
       mode == 0 ? "(hstep >= step && hstep < watchdog) ? hstep : watchdog" : "watchdog");
@@ -1025,8 +1025,10 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       "jx->bc_[s_ * 4 + 1][lane] = bc.sz[s_]; %s}\n"
       "#pragma unroll\n  for (int s_ = %d; s_ < JBC_SLOTS; ++s_) jx->bc_[s_ * 4 + 1][lane] = 0u;\n"
       "  u32 z_ = 0u;\n#pragma unroll\n  for (int s_ = 0; s_ < %d; ++s_) z_ |= (u32)bc.z[s_] << s_;\n"
-      "  jx->bcz_[lane] = z_; __syncwarp(); if (lane == 0u) jx->bck = k; __syncwarp(); }\n", nslots,
-      mode == 3 ? "jx->bc_[s_ * 4 + 2][lane] = bc.b[s_]; jx->bc_[s_ * 4 + 3][lane] = bc.pb[s_]; " : "", nslots, nslots);
+      "  jx->bcz_[lane] = z_; __syncwarp(); if (lane == 0u) { jx->bck = k; %s} __syncwarp(); }\n",
+      nslots,
+      mode == 3 ? "jx->bc_[s_ * 4 + 2][lane] = bc.b[s_]; jx->bc_[s_ * 4 + 3][lane] = bc.pb[s_]; " : "", nslots, nslots,
+      mode == 3 ? "jx->bckp = (u32)(size_t)PG.ptab; " : "");
     if (mode == 2) o(" if (lane == 0u) jbulk_wait();     // the template stores are complete\n");
     if (mode == 2)                                    // checkpoints the warp never reached: absent
         o(" if (ck) for (; ckn < (step + ck_interval - 1u) / ck_interval; ++ckn) {\n"
@@ -1121,7 +1123,8 @@ std::string generate(const fi_insn* code, const fi_kernel* kern, uint32_t n_kern
           "  const u64 L = K.warp_off[w + 1] - K.warp_off[w]; const u64 wd = 10ull * L + 1024ull;\n"
           "  const u32 watchdog = wd > 0xFFFFFFFFull ? 0xFFFFFFFFu : (u32)wd;\n"
           "  JPage pg; pg.ptab = K.ptab + (u64)s * K.total_pages; pg.pool = K.pool; pg.page_base = K.page_base; "
-          "pg.last_ref = K.last_ref; pg.dropped = K.dropped + (u64)s * K.dwords; pg.inexact = &K.slot[s].inexact; pg.t = t;\n"
+          "pg.last_ref = K.last_ref; pg.dropped = K.dropped + (u64)s * K.dwords; pg.bcount = K.bcount + (u64)s * K.n_buf; "
+          "pg.inexact = &K.slot[s].inexact; pg.t = t;\n"
           "  JOut o; o.start = 0u;\n  switch (in.kernel) {\n",
           min_blocks, rs, zrow, 4 * rs);
         for (uint32_t k = 0; k < n_kern; ++k)

@@ -19,6 +19,7 @@ struct JK8Host {
     fi_store* scratch; uint32_t log_cap;
     uint32_t flags; uint32_t* status;
     unsigned long long* steps;                      // emulated warp-steps of the re-executed warps (summed)
+    const uint32_t* bcount; uint32_t n_buf;         // [slot][buffer] page counts
 };
 fi_status jit_k8_exec(const fi_jit* j, const fi_program* p, const uint8_t* image, const JK8Host& K, uint32_t t,
                       uint32_t max_grid, cudaStream_t s);

@@ -75,6 +75,7 @@ struct JCtx {
     // the next inside a launch: valid while the instance is bck (the writer rule of
     // an entry depends on the instance); set invalid by every entry kernel
     u32 bck;
+    u32 bckp;                                        // PAGE mode: ... and the slot (its page table's low word)
     u32 bc_[16][32];                                 // [slot * 4 + {lo, sz, b, pb}][lane]
     u32 bcz_[32];                                    // bit slot: the entry's writer-rule flag
     JProf prof;                                      // golden pass 2 only
@@ -287,11 +288,19 @@ __device__ __forceinline__ void jprefetch(const u8* __restrict__ img, const JBuf
         asm volatile("prefetch.global.L1 [%0];" ::"l"(img + (va - JVA_BASE)));
 }
 
+// the replica slot's view of memory during instance t (K8, PAGE mode)
+struct JPage {
+    const u32* ptab;             // the slot's page table
+    const u32* pool; const u32* page_base; const u32* last_ref; const u32* dropped;
+    const u32* bcount;           // the slot's page count per buffer (constant during a launch)
+    u32* inexact; u32 t;
+};
+#define JPB_NONE 0xFFFFFFFFu     // cache entry's page base when the slot holds no page of the buffer
 // 0 ok, 1 misaligned, 2 unmapped (C-15); *zero = writer rule for instance k.
 // A miss refills entry S.
 template <int S>
 __device__ __forceinline__ u32 jcheck(const JArgs& A, JBufCache& C, u64 va, u32 w, u32 k, bool* zero,
-                                      const u32* page_base = nullptr) {
+                                      const JPage* pg = nullptr) {
     if (va & (w - 1)) return 1;
     if (jhit<S>(C, va, w, zero)) return 0;
     const u64 off = va - JVA_BASE;
@@ -305,7 +314,14 @@ __device__ __forceinline__ u32 jcheck(const JArgs& A, JBufCache& C, u64 va, u32 
     *zero = z;
     if ((lo & 15u) == 0 && lo + size <= 0x80000000ull && size >= 16) {
         C.lo[S] = (u32)lo; C.sz[S] = (u32)size & ~15u; C.z[S] = z; C.b[S] = b;
-        C.pb[S] = page_base ? __ldg(&page_base[b]) : 0u;
+        // PAGE mode: JPB_NONE when the slot has no page of the buffer and no page of it was
+        // dropped past its last reference — the golden words stand, jpage_c skips the
+        // page-table load
+        C.pb[S] = 0u;
+        if (pg) {
+            const bool dropped = __ldg(&pg->last_ref[b]) < pg->t && ((pg->dropped[b >> 5] >> (b & 31)) & 1u);
+            C.pb[S] = (pg->bcount[b] == 0u && !dropped) ? JPB_NONE : __ldg(&pg->page_base[b]);
+        }
     }
     return 0;
 }
@@ -313,9 +329,9 @@ __device__ __forceinline__ u32 jcheck(const JArgs& A, JBufCache& C, u64 va, u32 
 // one LDG of 1/2/4 words for this lane; returns the fault code (0 ok)
 template <u32 LW, int S>
 __device__ __forceinline__ u32 jldg(const JArgs& A, const u8* __restrict__ img, JBufCache& C, u64 va, u32 k, bool ex,
-                                    uint4& v, const u32* page_base = nullptr) {
+                                    uint4& v, const JPage* pg = nullptr) {
     bool zero = false;
-    const u32 c = ex ? jcheck<S>(A, C, va, 4u << LW, k, &zero, page_base) : 0u;
+    const u32 c = ex ? jcheck<S>(A, C, va, 4u << LW, k, &zero, pg) : 0u;
     v = make_uint4(0, 0, 0, 0);
     if (ex && !c && !zero) {
         const u8* src = img + (va - JVA_BASE);
@@ -370,12 +386,7 @@ struct JK8 {
     jfi_store* scratch; u32 log_cap;
     u32 flags; u32* status;
     unsigned long long* steps;                      // emulated warp-steps of the re-executed warps (summed)
-};
-// the replica slot's view of memory during instance t
-struct JPage {
-    const u32* ptab;             // the slot's page table
-    const u32* pool; const u32* page_base; const u32* last_ref; const u32* dropped;
-    u32* inexact; u32 t;
+    const u32* bcount; u32 n_buf;                   // [slot][buffer] page counts
 };
 
 // The replica's words of an aligned access of NW words (one 4 KB page): its page
@@ -402,6 +413,7 @@ template <u32 NW, int S>
 __device__ __forceinline__ void jpage_c(const JArgs& A, const JBufCache& C, const JPage& G, u64 va, uint4& v) {
     const u32 rel = (u32)va - C.lo[S];
     if (!(rel < C.sz[S])) { jpage<NW>(A, G, va, v); return; }
+    if (C.pb[S] == JPB_NONE) return;                 // no page of this buffer in the slot
     const u32 b = C.b[S];
     const u32 e = G.ptab[C.pb[S] + (rel >> 12)];
     if (e < JPAGE_CLAIM) {
@@ -498,7 +510,7 @@ __device__ __noinline__ u32 jinterp(const JArgs& A, JState& S, JBufCache& bc, u3
             const u32 lw = (mod & 3) > 2 ? 2 : (mod & 3), nw = 1u << lw, w = 4u << lw;
             const u64 va = F.rd64(ia) + (u64)(i64)(i32)imm;
             bool zero = false;
-            const u32 c = ex ? jcheck<0>(A, bc, va, w, k, &zero, MODE == JM_PAGE ? pg->page_base : nullptr) : 0u;
+            const u32 c = ex ? jcheck<0>(A, bc, va, w, k, &zero, MODE == JM_PAGE ? pg : nullptr) : 0u;
             if (__ballot_sync(JFULL, c != 0u)) {      // memory fault: DUE (C-9); the step has no effect
                 S.fault = __ballot_sync(JFULL, c == 1u) ? 1u : 2u;
                 S.fault_pc = pcm;

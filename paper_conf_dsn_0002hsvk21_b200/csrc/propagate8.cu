@@ -769,7 +769,8 @@ static fi_status k8_run(const fi_program* p, const uint8_t* image, const fi_trac
     const uint32_t fix_grid = (uint32_t)std::max(1, sms * 4);
     JK8Host JK{A.warp_off, A.gst_off, A.gst, A.slot, A.ptab, A.total_pages, A.pool, A.page_base, A.last_ref,
                A.dropped, A.dwords, A.pend, A.pend_cap, A.forn, kForeignCap, A.active, A.n_active, A.work,
-               A.scratch, A.log_cap, A.flags, A.status, reinterpret_cast<unsigned long long*>(w + L.steps)};
+               A.scratch, A.log_cap, A.flags, A.status, reinterpret_cast<unsigned long long*>(w + L.steps),
+               A.bcount, A.n_buf};
     if ((e = cuda_status(cudaMemsetAsync(w + L.steps, 0, 8, s)))) return e;
 
     for (uint32_t b0 = 0; b0 < n; b0 += batch) {
