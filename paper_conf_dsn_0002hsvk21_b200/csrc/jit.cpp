@@ -337,7 +337,7 @@ struct Gen {
             for (uint32_t q = tmpl_L; q <= E; ++q)
                 if (code[q].guard != 7) all += (all.empty() ? "" : " & ") + std::string("gb_") + std::to_string(q);
             if (!all.empty()) o(" && (%s) == JFULL", all.c_str());
-            o(") { if (lane == 0u) jbulk_st(&rec_out[step], jtm_, %uu);\n"
+            o(") { if (jelect()) jbulk_st(&rec_out[step], jtm_, %uu);\n"
               "     if (JPCC_) { const u32 o_ = (JPRB_ + step) & 1023u; if (o_ + %uu < 1024u) { "
               "if (lane < 8u) jx->prof.pcnt_[lane] += jx->prof.tcnt_[lane]; } else jprof_tmpl_cross(&jx->prof, lane, "
               "1024u - o_); } } else\n", (E + 1 - tmpl_L) * 16, E + 1 - tmpl_L);

@@ -89,6 +89,11 @@ struct JCtx {
 // (jit.cpp flush_recs; the template loop reads both once)
 #define JPCC_ (jx->prof.cc != nullptr)
 #define JPRB_ ((u32)jx->prof.rb)
+__device__ __forceinline__ bool jelect() {
+    u32 p;
+    asm volatile("{\n\t.reg .pred e;\n\telect.sync _|e, 0xFFFFFFFF;\n\tselp.u32 %0, 1, 0, e;\n\t}" : "=r"(p));
+    return p != 0u;
+}
 __device__ __forceinline__ void jbulk_st(uint4* g, const uint4* s, u32 bytes) {
     u64 pol;
     asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
