@@ -339,7 +339,7 @@ struct Gen {
             if (!all.empty()) o(" && (%s) == JFULL", all.c_str());
             o(") { if (jelect()) jbulk_st(&rec_out[step], jtm_, %uu);\n"
               "     if (JPCC_) { const u32 o_ = (JPRB_ + step) & 1023u; if (o_ + %uu < 1024u) { "
-              "if (lane < 8u) jx->prof.pcnt_[lane] += jx->prof.tcnt_[lane]; } else jprof_tmpl_cross(&jx->prof, lane, "
+              "if (lane < 8u) jx->prof.pcnt_[lane] += JTCNT_; } else jprof_tmpl_cross(&jx->prof, lane, "
               "1024u - o_); } } else\n", (E + 1 - tmpl_L) * 16, E + 1 - tmpl_L);
         }
         o("   { const u32 n_ = %uu - pcm; for (u32 jb_ = 0u; jb_ < n_; jb_ += 32u) { const u32 j_ = jb_ + lane; "
@@ -938,7 +938,8 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
                     // (the template loop's profile state, constant over the loop, read once)
                     if (L == tmpl_L)
                         o(" const bool jpc_ = jx->prof.cc != nullptr; const u32 jrb_ = (u32)jx->prof.rb; (void)jpc_; (void)jrb_;\n"
-                          "#undef JPCC_\n#define JPCC_ jpc_\n#undef JPRB_\n#define JPRB_ jrb_\n");
+                          " const u32 jtc_ = lane < 8u ? jx->prof.tcnt_[lane] : 0u; (void)jtc_;\n"
+                          "#undef JPCC_\n#define JPCC_ jpc_\n#undef JPRB_\n#define JPRB_ jrb_\n#undef JTCNT_\n#define JTCNT_ jtc_\n");
                     o("#undef JFW_\n#define JFW_ 1\n for (;;) {  // self-loop %u..%u, full warp, two iterations per trip\n {\n",
                       L, i);
                     o.s += back(body, "goto U" + std::to_string(L) + "_;");
@@ -946,7 +947,8 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
                     o.s += back(body, "continue;");
                     o(" }\n }\n#undef JFW_\n#define JFW_ 0\n");
                     if (L == tmpl_L)
-                        o("#undef JPCC_\n#define JPCC_ (jx->prof.cc != nullptr)\n#undef JPRB_\n#define JPRB_ ((u32)jx->prof.rb)\n");
+                        o("#undef JPCC_\n#define JPCC_ (jx->prof.cc != nullptr)\n#undef JPRB_\n#define JPRB_ ((u32)jx->prof.rb)\n"
+                          "#undef JTCNT_\n#define JTCNT_ (jx->prof.tcnt_[lane])\n");
                     o(" } else {\n for (;;) {  // self-loop %u..%u\n", L, i);
                     o.s += back(body, "continue;");
                     o(" } }\n");

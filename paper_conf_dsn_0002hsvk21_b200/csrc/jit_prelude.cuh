@@ -89,6 +89,7 @@ struct JCtx {
 // (jit.cpp flush_recs; the template loop reads both once)
 #define JPCC_ (jx->prof.cc != nullptr)
 #define JPRB_ ((u32)jx->prof.rb)
+#define JTCNT_ (jx->prof.tcnt_[lane])
 __device__ __forceinline__ bool jelect() {
     u32 p;
     asm volatile("{\n\t.reg .pred e;\n\telect.sync _|e, 0xFFFFFFFF;\n\tselp.u32 %0, 1, 0, e;\n\t}" : "=r"(p));
