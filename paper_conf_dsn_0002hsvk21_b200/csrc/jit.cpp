@@ -339,8 +339,8 @@ struct Gen {
             if (!all.empty()) o(" && (%s) == JFULL", all.c_str());
             o(") { if (jelect()) jbulk_st(&rec_out[step], jtm_, %uu);\n"
               "     if (JPCC_) { const u32 o_ = (JPRB_ + step) & 1023u; if (o_ + %uu < 1024u) { "
-              "if (lane < 8u) jx->prof.pcnt_[lane] += JTCNT_; } else jprof_tmpl_cross(&jx->prof, lane, "
-              "1024u - o_); } } else\n", (E + 1 - tmpl_L) * 16, E + 1 - tmpl_L);
+              "JPADD_; } else { JPFLUSH_; jprof_tmpl_cross(&jx->prof, lane, "
+              "1024u - o_); } } } else\n", (E + 1 - tmpl_L) * 16, E + 1 - tmpl_L);
         }
         o("   { const u32 n_ = %uu - pcm; for (u32 jb_ = 0u; jb_ < n_; jb_ += 32u) { const u32 j_ = jb_ + lane; "
           "const bool v_ = j_ < n_; const u32 p_ = pcm + j_; u32 pr_ = JFULL; ",
@@ -350,7 +350,7 @@ struct Gen {
         // streaming stores (evict-first): the 16-B records are written once and read by
         // other kernels, so they must not push the image lines the loads reuse out of L2
         o("const u32 w_ = v_ ? __ldg(&ins[p_]) : 0u; if (v_) __stcs(&rec_out[step + j_], make_uint4(k, w_, amask, pr_));\n"
-          "     if (jx->prof.cc) jprof_round(&jx->prof, lane, jx->prof.rb + step + jb_, v_, __popc(amask & pr_), w_ >> 24); } }\n");
+          "     if (jx->prof.cc) { JPFLUSH_; jprof_round(&jx->prof, lane, jx->prof.rb + step + jb_, v_, __popc(amask & pr_), w_ >> 24); } } }\n");
     }
     void mem(Src& o, const fi_insn& I, uint32_t pc, const char* stepx) const {
         using namespace fi;
@@ -938,17 +938,20 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
                     // (the template loop's profile state, constant over the loop, read once)
                     if (L == tmpl_L)
                         o(" const bool jpc_ = jx->prof.cc != nullptr; const u32 jrb_ = (u32)jx->prof.rb; (void)jpc_; (void)jrb_;\n"
-                          " const u32 jtc_ = lane < 8u ? jx->prof.tcnt_[lane] : 0u; (void)jtc_;\n"
-                          "#undef JPCC_\n#define JPCC_ jpc_\n#undef JPRB_\n#define JPRB_ jrb_\n#undef JTCNT_\n#define JTCNT_ jtc_\n");
+                          " const u32 jtc_ = lane < 8u ? jx->prof.tcnt_[lane] : 0u; u32 jpa_ = 0u; (void)jtc_; (void)jpa_;\n"
+                          "#undef JPCC_\n#define JPCC_ jpc_\n#undef JPRB_\n#define JPRB_ jrb_\n"
+                          "#undef JPADD_\n#define JPADD_ (jpa_ += jtc_)\n"
+                          "#undef JPFLUSH_\n#define JPFLUSH_ { if (lane < 8u) jx->prof.pcnt_[lane] += jpa_; jpa_ = 0u; }\n");
                     o("#undef JFW_\n#define JFW_ 1\n for (;;) {  // self-loop %u..%u, full warp, two iterations per trip\n {\n",
                       L, i);
                     o.s += back(body, "goto U" + std::to_string(L) + "_;");
                     o(" }\n U%u_: ;\n {\n", L);
                     o.s += back(body, "continue;");
                     o(" }\n }\n#undef JFW_\n#define JFW_ 0\n");
-                    if (L == tmpl_L)
-                        o("#undef JPCC_\n#define JPCC_ (jx->prof.cc != nullptr)\n#undef JPRB_\n#define JPRB_ ((u32)jx->prof.rb)\n"
-                          "#undef JTCNT_\n#define JTCNT_ (jx->prof.tcnt_[lane])\n");
+                    if (L == tmpl_L)   // (the loop is left only through its breaks: flush the register count there)
+                        o(" JPFLUSH_;\n#undef JPCC_\n#define JPCC_ (jx->prof.cc != nullptr)\n#undef JPRB_\n#define JPRB_ ((u32)jx->prof.rb)\n"
+                          "#undef JPADD_\n#define JPADD_ { if (lane < 8u) jx->prof.pcnt_[lane] += jx->prof.tcnt_[lane]; }\n"
+                          "#undef JPFLUSH_\n#define JPFLUSH_ {}\n");
                     o(" } else {\n for (;;) {  // self-loop %u..%u\n", L, i);
                     o.s += back(body, "continue;");
                     o(" } }\n");

@@ -89,7 +89,10 @@ struct JCtx {
 // (jit.cpp flush_recs; the template loop reads both once)
 #define JPCC_ (jx->prof.cc != nullptr)
 #define JPRB_ ((u32)jx->prof.rb)
-#define JTCNT_ (jx->prof.tcnt_[lane])
+// the template pass's count update, and the flush of a count kept in a register
+// (the full-warp template loop keeps it there; elsewhere it goes straight to smem)
+#define JPADD_ { if (lane < 8u) jx->prof.pcnt_[lane] += jx->prof.tcnt_[lane]; }
+#define JPFLUSH_ {}
 __device__ __forceinline__ bool jelect() {
     u32 p;
     asm volatile("{\n\t.reg .pred e;\n\telect.sync _|e, 0xFFFFFFFF;\n\tselp.u32 %0, 1, 0, e;\n\t}" : "=r"(p));
