@@ -337,7 +337,7 @@ struct Gen {
             for (uint32_t q = tmpl_L; q <= E; ++q)
                 if (code[q].guard != 7) all += (all.empty() ? "" : " & ") + std::string("gb_") + std::to_string(q);
             if (!all.empty()) o(" && (%s) == JFULL", all.c_str());
-            o(") { if (jelect()) jbulk_st(&rec_out[step], jtm_, %uu);\n"
+            o(") { if (jelect()) jbulk_st_p(&rec_out[step], jtm_, %uu, JPOL_);\n"
               "     if (JPCC_) { const u32 o_ = (JPRB_ + step) & 1023u; if (o_ + %uu < 1024u) { "
               "JPADD_; } else { JPFLUSH_; jprof_tmpl_cross(&jx->prof, lane, "
               "1024u - o_); } } } else\n", (E + 1 - tmpl_L) * 16, E + 1 - tmpl_L);
@@ -939,6 +939,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
                     if (L == tmpl_L)
                         o(" const bool jpc_ = jx->prof.cc != nullptr; const u32 jrb_ = (u32)jx->prof.rb; (void)jpc_; (void)jrb_;\n"
                           " const u32 jtc_ = lane < 8u ? jx->prof.tcnt_[lane] : 0u; u32 jpa_ = 0u; (void)jtc_; (void)jpa_;\n"
+                          " const u64 jpol_ = jpolicy_ef(); (void)jpol_;\n#undef JPOL_\n#define JPOL_ jpol_\n"
                           "#undef JPCC_\n#define JPCC_ jpc_\n#undef JPRB_\n#define JPRB_ jrb_\n"
                           "#undef JPADD_\n#define JPADD_ (jpa_ += jtc_)\n"
                           "#undef JPFLUSH_\n#define JPFLUSH_ { if (lane < 8u) jx->prof.pcnt_[lane] += jpa_; jpa_ = 0u; }\n");
@@ -951,7 +952,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
                     if (L == tmpl_L)   // (the loop is left only through its breaks: flush the register count there)
                         o(" JPFLUSH_;\n#undef JPCC_\n#define JPCC_ (jx->prof.cc != nullptr)\n#undef JPRB_\n#define JPRB_ ((u32)jx->prof.rb)\n"
                           "#undef JPADD_\n#define JPADD_ { if (lane < 8u) jx->prof.pcnt_[lane] += jx->prof.tcnt_[lane]; }\n"
-                          "#undef JPFLUSH_\n#define JPFLUSH_ {}\n");
+                          "#undef JPFLUSH_\n#define JPFLUSH_ {}\n#undef JPOL_\n#define JPOL_ jpolicy_ef()\n");
                     o(" } else {\n for (;;) {  // self-loop %u..%u\n", L, i);
                     o.s += back(body, "continue;");
                     o(" } }\n");

@@ -93,10 +93,21 @@ struct JCtx {
 // (the full-warp template loop keeps it there; elsewhere it goes straight to smem)
 #define JPADD_ { if (lane < 8u) jx->prof.pcnt_[lane] += jx->prof.tcnt_[lane]; }
 #define JPFLUSH_ {}
+#define JPOL_ jpolicy_ef()
 __device__ __forceinline__ bool jelect() {
     u32 p;
     asm volatile("{\n\t.reg .pred e;\n\telect.sync _|e, 0xFFFFFFFF;\n\tselp.u32 %0, 1, 0, e;\n\t}" : "=r"(p));
     return p != 0u;
+}
+__device__ __forceinline__ u64 jpolicy_ef() {
+    u64 pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ void jbulk_st_p(uint4* g, const uint4* s, u32 bytes, u64 pol) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group.L2::cache_hint [%0], [%1], %2, %3;\n\t"
+                 "cp.async.bulk.commit_group;" :: "l"(g), "r"((u32)__cvta_generic_to_shared(s)), "r"(bytes), "l"(pol)
+                 : "memory");
 }
 __device__ __forceinline__ void jbulk_st(uint4* g, const uint4* s, u32 bytes) {
     u64 pol;
