@@ -928,7 +928,9 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
                     o.s = std::move(loop_saved);
                     o(" if (amask == JFULL) { const bool inA = true; (void)inA;\n");
                     if (L == tmpl_L)                  // the warp's record template of this block (once per job)
-                        o(" if (!tmpl_) { if (lane == 0u) jbulk_wait_read(); __syncwarp();\n"
+                        // (every lane waits for its own bulk groups: the copies are issued by an
+                        // elected lane)
+                        o(" if (!tmpl_) { jbulk_wait_read(); __syncwarp();\n"
                           "   for (u32 j_ = lane; j_ < %uu; j_ += 32u) jtm_[j_] = make_uint4(k, __ldg(&ins[%uu + j_]), JFULL, JFULL);\n"
                           "   jfence_async(); __syncwarp(); tmpl_ = true; if (jx->prof.cc) jprof_tcnt(&jx->prof, lane, %uu, jtm_); }\n",
                           i + 1 - L, L, i + 1 - L);
@@ -1035,7 +1037,7 @@ void gen_kernel(Src& o, const Gen& G0, uint32_t kid, const fi_insn* code, uint32
       nslots,
       mode == 3 ? "jx->bc_[s_ * 4 + 2][lane] = bc.b[s_]; jx->bc_[s_ * 4 + 3][lane] = bc.pb[s_]; " : "", nslots, nslots,
       mode == 3 ? "jx->bckp = (u32)(size_t)PG.ptab; " : "");
-    if (mode == 2) o(" if (lane == 0u) jbulk_wait();     // the template stores are complete\n");
+    if (mode == 2) o(" jbulk_wait(); __syncwarp();     // the template stores are complete (each lane's own groups)\n");
     if (mode == 2)                                    // checkpoints the warp never reached: absent
         o(" if (ck) for (; ckn < (step + ck_interval - 1u) / ck_interval; ++ckn) {\n"
           "   for (u32 r_ = 0u; r_ < %uu; ++r_) ck[(u64)ckn * %uu + r_ * 32u + lane] = 0u;\n"

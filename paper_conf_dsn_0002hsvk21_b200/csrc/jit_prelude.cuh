@@ -83,7 +83,8 @@ struct JCtx {
 #define JCTX_BYTES 3712u
 // golden trace pass: bulk (TMA) stores of a warp's record template from shared
 // memory (jit.cpp flush_recs), evict-first in L2 like the per-lane __stcs records;
-// lane 0 issues them and waits for them before the warp's job ends
+// one elected lane issues them; every lane waits for its own groups before the
+// template is rewritten and before the warp's job ends
 #define JFW_ 0
 // golden pass 2's fused profile: is it on, and the warp's first global record
 // (jit.cpp flush_recs; the template loop reads both once)
@@ -105,13 +106,6 @@ __device__ __forceinline__ u64 jpolicy_ef() {
     return pol;
 }
 __device__ __forceinline__ void jbulk_st_p(uint4* g, const uint4* s, u32 bytes, u64 pol) {
-    asm volatile("cp.async.bulk.global.shared::cta.bulk_group.L2::cache_hint [%0], [%1], %2, %3;\n\t"
-                 "cp.async.bulk.commit_group;" :: "l"(g), "r"((u32)__cvta_generic_to_shared(s)), "r"(bytes), "l"(pol)
-                 : "memory");
-}
-__device__ __forceinline__ void jbulk_st(uint4* g, const uint4* s, u32 bytes) {
-    u64 pol;
-    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
     asm volatile("cp.async.bulk.global.shared::cta.bulk_group.L2::cache_hint [%0], [%1], %2, %3;\n\t"
                  "cp.async.bulk.commit_group;" :: "l"(g), "r"((u32)__cvta_generic_to_shared(s)), "r"(bytes), "l"(pol)
                  : "memory");
