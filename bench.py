@@ -383,7 +383,7 @@ def main():
     if not args.no_e2e:
         line["e2e"] = e2e(args, prog, seed, groups, bfms, n, rank, world, dev, camp)
     if rank == 0 and world == 1 and not args.no_secondary:
-        line["secondary"] = secondary_c4(dev)
+        line["secondary"] = secondary_c4(dev, sm_mhz=clk.get("sm_mhz") or clk.get("sm_max_mhz") or 1965.0)
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(prog, camp.sites_np(), camp)
     if rank == 0:
@@ -450,7 +450,7 @@ def golden_shards(dp, G=8, reps=3):
                     "record shard) of each rank alone on one GPU vs the whole golden run (fi_golden_run)"}
 
 
-def secondary_c4(dev, n=256):
+def secondary_c4(dev, n=256, sm_mhz=1965.0):
     """BASELINE configs[3]'s program (ResNet-50 v1.5 inference shape, 72 launches)
     on one GPU: golden run, exact profile, select, K4, K8 whole-program outcomes
     for a bounded replica sample (the 100 k campaign shards these over ranks).
@@ -499,7 +499,7 @@ def secondary_c4(dev, n=256):
             "ms": {"profile": ms[0], "index_select": ms[1], "inject_k4": ms[2], "propagate_classify_k8": ms[3]},
             "outcomes": {"masked": int(h[..., 0].sum()), "sdc": int(h[..., 1].sum()), "due": int(h[..., 2].sum())},
             "engine": "jit", "jit_compile_s": jit_s, "golden_run_s": golden_s,
-            "roofline_k8": k8_roofline(k8_steps[0] if k8_steps else 0, ms[3])}
+            "roofline_k8": k8_roofline(k8_steps[0] if k8_steps else 0, ms[3], sm_mhz)}
 
 
 def k8_roofline(steps, k8_ms, sm_mhz=1965.0):
@@ -511,7 +511,7 @@ def k8_roofline(steps, k8_ms, sm_mhz=1965.0):
     ach = steps / (k8_ms / 1e3) if k8_ms > 0 else 0.0
     return {"bound": "alu", "kernel": "k8_exec_jit + end-of-launch fix-ups (the whole K8 call)", "unit": "warp-inst/s",
             "achieved": ach, "peak": peak, "frac": ach / peak, "emulated_warp_steps": steps,
-            "peak_source": f"148 SMs x 4 SMSPs x 1 issue/clk x {sm_mhz:.0f} MHz"}
+            "peak_source": f"148 SMs x 4 SMSPs x 1 issue/clk x {sm_mhz:.0f} MHz (the SM clock sampled in the timed region)"}
 
 
 def e2e(args, prog, seed, groups, bfms, n, rank, world, dev, camp):
